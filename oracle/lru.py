@@ -1,0 +1,223 @@
+"""CPU ORACLE — address traces of the hot-path loops and an LRU L1D simulator.
+
+TEST INFRASTRUCTURE ONLY (see oracle/footprint.py header). Independent of the
+descriptors: the traces below are written from the loop bodies themselves
+(PolyBench/GPU and Rodinia kernels of Table 2; ATAX kernel 1 is
+Fig 1), one event per warp-level memory instruction, so they pin
+both the footprint model and the descriptors the library builds.
+
+LRU model: fully associative, LRU, `line_bytes` lines.
+Warps are interleaved round-robin, one memory instruction per turn. Only
+`a` warps per CTA and `m` CTAs per SM are runnable; a finished warp's slot
+goes to the next waiting warp of its CTA (semaphore semantics), a finished
+CTA's slot to the next CTA of the SM's list. A miss is an *intra-warp
+capacity miss* when the same warp touched that line before: the intra-thread
+/ intra-warp reuse CATT protects. Compulsory misses and lines
+another warp fetched do not count.
+"""
+from __future__ import annotations
+
+from collections import OrderedDict, deque
+from typing import Dict, List, Sequence, Tuple
+
+LINE = 128
+E = 4  # fp32
+
+
+def _line(arr: str, idx: int, line: int = LINE) -> Tuple[str, int]:
+    return (arr, (idx * E) // line)
+
+
+class Kernel:
+    """nblocks CTAs of W warps; events(b, w) -> list of frozensets of lines."""
+    nblocks: int
+    W: int
+    threads: int
+
+    def lanes(self, b: int, w: int):
+        for lane in range(32):
+            t = 32 * w + lane
+            if t < self.threads:
+                yield t
+
+
+class RowKernel(Kernel):
+    """Thread i = blockIdx.x*cta + threadIdx.x owns row i (i < M):
+         for j (step vec): for each matrix X: acc += X[i*N + j] * x[j]
+    vec = 4 models float4 loads (one 16-byte access per thread). With
+    with_tmp=True the accumulator is the global tmp[i] read every iteration
+    (Fig 1 literally)."""
+
+    def __init__(self, M, N, cta, vec=1, matrices=("A",), with_tmp=False):
+        self.M, self.N, self.vec, self.matrices, self.with_tmp = M, N, vec, matrices, with_tmp
+        self.threads = cta
+        self.W = (cta + 31) // 32
+        self.nblocks = (M + cta - 1) // cta
+
+    def events(self, b, w):
+        rows = [b * self.threads + t for t in self.lanes(b, w)]
+        rows = [i for i in rows if i < self.M]
+        ev = []
+        if not rows:
+            return ev
+        for j in range(0, self.N, self.vec):
+            if self.with_tmp:
+                ev.append(frozenset(_line("tmp", i) for i in rows))
+            for X in self.matrices:
+                ev.append(frozenset(_line(X, i * self.N + j) for i in rows))
+                ev.append(frozenset([_line("x", j)]))
+        return ev
+
+
+class ColKernel(Kernel):
+    """Thread j owns column j (j < N):  for i < M: acc += A[i*N + j] * v[i]."""
+
+    def __init__(self, M, N, cta):
+        self.M, self.N = M, N
+        self.threads = cta
+        self.W = (cta + 31) // 32
+        self.nblocks = (N + cta - 1) // cta
+
+    def events(self, b, w):
+        cols = [b * self.threads + t for t in self.lanes(b, w)]
+        cols = [j for j in cols if j < self.N]
+        ev = []
+        if not cols:
+            return ev
+        for i in range(self.M):
+            ev.append(frozenset(_line("A", i * self.N + j) for j in cols))
+            ev.append(frozenset([_line("v", i)]))
+        return ev
+
+
+class SyrkKernel(Kernel):
+    """PolyBench/GPU syrk, block (32, 8): j = bx*32 + tx, i = by*8 + ty,
+    for k < Mk: c += alpha * a[i*Mk + k] * a[j*Mk + k] (c in a register)."""
+
+    def __init__(self, N, Mk, bdim=(32, 8)):
+        self.N, self.Mk, self.bdim = N, Mk, bdim
+        self.threads = bdim[0] * bdim[1]
+        self.W = (self.threads + 31) // 32
+        self.gx = (N + bdim[0] - 1) // bdim[0]
+        self.gy = (N + bdim[1] - 1) // bdim[1]
+        self.nblocks = self.gx * self.gy
+
+    def events(self, b, w):
+        bx, by = b % self.gx, b // self.gx
+        th = []
+        for t in self.lanes(b, w):
+            tx, ty = t % self.bdim[0], t // self.bdim[0]
+            i, j = by * self.bdim[1] + ty, bx * self.bdim[0] + tx
+            if i < self.N and j < self.N:
+                th.append((i, j))
+        ev = []
+        if not th:
+            return ev
+        for k in range(self.Mk):
+            ev.append(frozenset(_line("a", i * self.Mk + k) for i, _ in th))
+            ev.append(frozenset(_line("a", j * self.Mk + k) for _, j in th))
+        return ev
+
+
+class KmeansKernel(Kernel):
+    """Rodinia kmeansPoint, feature-major: thread p (p < npoints):
+    for c < k: for f < nf: diff = feat[f*ld + p] - clusters[c*nf + f]
+    (clusters are staged in shared memory, so not traced)."""
+
+    def __init__(self, npoints, nf, k, ld, cta):
+        self.npoints, self.nf, self.k, self.ld = npoints, nf, k, ld
+        self.threads = cta
+        self.W = (cta + 31) // 32
+        self.nblocks = (npoints + cta - 1) // cta
+
+    def events(self, b, w):
+        pts = [b * self.threads + t for t in self.lanes(b, w)]
+        pts = [p for p in pts if p < self.npoints]
+        ev = []
+        if not pts:
+            return ev
+        for c in range(self.k):
+            for f in range(self.nf):
+                ev.append(frozenset(_line("F", f * self.ld + p) for p in pts))
+        return ev
+
+
+def simulate(kernel: Kernel, sm_blocks: Sequence[int], a: int, m: int, capacity: int) -> Dict:
+    """Run the warps of the CTAs in sm_blocks (in order) with at most a active
+    warps per CTA and m active CTAs; LRU of `capacity` lines."""
+    cache: "OrderedDict" = OrderedDict()
+    seen: Dict[Tuple[int, int], set] = {}
+    stats = dict(accesses=0, hits=0, misses=0, intra_warp_capacity_misses=0)
+    pending = deque(sm_blocks)
+    rotation: deque = deque()          # entries: [b, w, events, pos]
+    cta_wait: Dict[int, deque] = {}
+    cta_left: Dict[int, int] = {}
+
+    def start_cta():
+        b = pending.popleft()
+        ws = deque(range(kernel.W))
+        cta_wait[b] = ws
+        cta_left[b] = kernel.W
+        for _ in range(min(a, kernel.W)):
+            w = ws.popleft()
+            rotation.append([b, w, kernel.events(b, w), 0])
+
+    active_ctas = 0
+    while pending and active_ctas < m:
+        start_cta()
+        active_ctas += 1
+    while rotation:
+        ent = rotation.popleft()
+        b, w, ev, pos = ent
+        if pos < len(ev):
+            key = (b, w)
+            s = seen.setdefault(key, set())
+            for ln in ev[pos]:
+                stats["accesses"] += 1
+                if ln in cache:
+                    cache.move_to_end(ln)
+                    stats["hits"] += 1
+                else:
+                    stats["misses"] += 1
+                    if ln in s:
+                        stats["intra_warp_capacity_misses"] += 1
+                    cache[ln] = True
+                    if len(cache) > capacity:
+                        cache.popitem(last=False)
+                s.add(ln)
+            ent[3] = pos + 1
+        if ent[3] < len(ev):
+            rotation.append(ent)
+            continue
+        # warp done: refill its slot from its CTA
+        cta_left[b] -= 1
+        if cta_wait[b]:
+            w2 = cta_wait[b].popleft()
+            rotation.append([b, w2, kernel.events(b, w2), 0])
+        elif cta_left[b] == 0 and pending:
+            start_cta()
+    return stats
+
+
+def sm0_blocks(kernel: Kernel, num_sms: int, limit: int = 1 << 30) -> List[int]:
+    """Blocks the round-robin distribution gives SM 0: 0, #SM, 2*#SM, ..."""
+    return list(range(0, kernel.nblocks, num_sms))[:limit]
+
+
+def decide_by_lru(kernel: Kernel, W: int, T: int, capacity: int, num_sms: int, limit_blocks=None) -> Tuple[int, int, str]:
+    """Walk the Eq 9 candidate order and return the
+    first throttle with zero intra-warp capacity misses."""
+    blocks = sm0_blocks(kernel, num_sms, limit_blocks or max(T, 1))
+
+    def ok(a, m):
+        return simulate(kernel, blocks, a, m, capacity)["intra_warp_capacity_misses"] == 0
+
+    if ok(W, T):
+        return W, T, "none"
+    for N in range(2, W + 1):
+        if W % N == 0 and ok(W // N, T):
+            return W // N, T, "warp"
+    for m in range(T - 1, 0, -1):
+        if ok(1, m):
+            return 1, m, "cta"
+    return W, T, "unresolvable"
