@@ -167,23 +167,41 @@ def _lane_gids(loop: Loop, b: int, w: int, warp_size: int) -> List[Tuple[int, in
     return out
 
 
-def _window(ref: Ref, trips: Sequence[int], line: int) -> List[Tuple[int, ...]]:
-    """Iteration vectors whose lines the warp must retain until the reuse
-    (Eq 6; outer-loop reuse R10)."""
+def has_locality(ref: Ref, trips: Sequence[int], line: int) -> bool:
+    """Eq 6 with the trip counts: some line of the reference is
+    re-touched by the same thread (a level with |C_i|*e < line that actually
+    iterates, trip >= 2)."""
+    return any(abs(ref.c_iter[k]) * ref.elem_bytes < line and trips[k] >= 2 for k in range(len(trips)))
+
+
+def _window(ref: Ref, trips: Sequence[int], line: int):
+    """Iteration vectors whose lines the warp retains until the reuse, as a
+    function of the phase k of the innermost loop (Eq 6; R10, R11).
+
+    Returns (per_phase, iters): if per_phase, the ref is evaluated at the
+    single vector (0, .., 0, k) -- consecutive-iteration reuse (the line is
+    re-touched next iteration) or no reuse (the line lives one iteration);
+    otherwise `iters` is the fixed window of an outer-level reuse: all inner
+    iteration vectors with the outer indices at 0."""
     n = len(trips)
     if n == 0:
-        return [()]
+        return True, None
     L = n - 1
     if abs(ref.c_iter[L]) * ref.elem_bytes < line:        # consecutive-iteration reuse
-        return [(0,) * n]
+        return True, None
     for k in range(L - 1, -1, -1):
         if abs(ref.c_iter[k]) * ref.elem_bytes < line:    # reuse across level-k iterations
             inner = [range(trips[d]) for d in range(k + 1, n)]
             size = math.prod(len(r) for r in inner)
             if size > MAX_WINDOW:
                 raise Unlaunchable("reuse window too large to enumerate")
-            return [(0,) * (k + 1) + tuple(v) for v in itertools.product(*inner)]
-    return [(0,) * n]                                     # no reuse: one iteration's lines
+            return False, [(0,) * (k + 1) + tuple(v) for v in itertools.product(*inner)]
+    return True, None                                     # no reuse: one iteration's lines
+
+
+def _phase_iter(trips: Sequence[int], k: int):
+    n = len(trips)
+    return [()] if n == 0 else [(0,) * (n - 1) + (k,)]
 
 
 def _lines(ref: Ref, gids, iters, line: int, irregular_as_unit: bool = True):
@@ -220,29 +238,38 @@ class Model:
         self.W, self.T, self.carveout_kb, self.l1d_bytes = occupancy(loop, hw)
         self.line = hw["line_bytes"]
         self.paper = loop.mode == MODE_PAPER
+        # contention is measured only "for loops where cache locality presents"
+        self.locality = any(has_locality(r, loop.trips, self.line) for r in loop.refs
+                            if not (r.flags & REF_NOT_L1))
         if self.paper:
             self.req = sum(req_warp_paper(r, loop, hw) for r in loop.refs)
             self.lines_per_warp_iter = self.req
             self.reuse_span = self.req
         else:
             self.refs = [r for r in loop.refs if not (r.flags & (REF_NOT_L1 | REF_STORE))]
+            self.win = [_window(r, loop.trips, self.line) for r in self.refs]
             gx, gy, gz = loop.grid
             nblocks = gx * gy * gz
             # CTAs resident on SM 0 in the first wave: 0, #SM, 2*#SM, ...
             self.blocks = [k * hw["num_sms"] for k in range(self.T) if k * hw["num_sms"] < nblocks]
+            # phases of the innermost loop over which per-phase lines are
+            # evaluated: one line's worth of 4-byte steps covers every
+            # alignment of a row start (R11)
+            per_phase = any(pp for pp, _ in self.win)
+            self.phases = min(loop.trips[-1], hw["line_bytes"] // 4) if (per_phase and loop.trips) else 1
             self._R = {}
             gids00 = _lane_gids(loop, 0, 0, hw["warp_size"])
             it0 = [(0,) * len(loop.trips)]
             self.lines_per_warp_iter = sum(len(_lines(r, gids00, it0, self.line)) for r in self.refs)
-            self.reuse_span = len(self.retained(0, 0))
+            self.reuse_span = len(self.retained(0, 0, 0))
 
-    def retained(self, b: int, w: int):
-        key = (b, w)
+    def retained(self, b: int, w: int, k: int):
+        key = (b, w, k)
         if key not in self._R:
             gids = _lane_gids(self.loop, b, w, self.hw["warp_size"])
             s = set()
-            for r in self.refs:
-                s |= _lines(r, gids, _window(r, self.loop.trips, self.line), self.line)
+            for r, (pp, iters) in zip(self.refs, self.win):
+                s |= _lines(r, gids, _phase_iter(self.loop.trips, k) if pp else iters, self.line)
             self._R[key] = s
         return self._R[key]
 
@@ -250,13 +277,18 @@ class Model:
         """Footprint in lines with a active warps per CTA and m CTAs per SM."""
         if self.paper:
             return self.req * a * m                                      # Eq 8 / Eq 9
+        # any m consecutive CTAs of the SM's list may be co-resident (R9), any
+        # of the warp groups of Fig 4 (warps g*a .. g*a+a-1) may be active, and
+        # the innermost loop may be at any phase k (R11): take the maximum
         best = 0
-        for g in range(_ceil_div(self.W, a)):
-            s = set()
-            for b in self.blocks[:m]:
-                for w in range(g * a, min(self.W, g * a + a)):
-                    s |= self.retained(b, w)
-            best = max(best, len(s))
+        for s0 in range(max(1, len(self.blocks) - m + 1)):
+            for g in range(_ceil_div(self.W, a)):
+                for k in range(self.phases):
+                    s = set()
+                    for b in self.blocks[s0:s0 + m]:
+                        for w in range(g * a, min(self.W, g * a + a)):
+                            s |= self.retained(b, w, k)
+                    best = max(best, len(s))
         return best
 
     def fits(self, lines: int) -> bool:
@@ -277,7 +309,7 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
                    footprint_bytes=lines * M.line, flags=flag)
         return res
 
-    if M.fits(full):
+    if M.fits(full) or not M.locality:
         return done(W, T, full, FIT_NONE_NEEDED)
     for N in range(2, W + 1):                     # Eq 9, warp level first
         if W % N:

@@ -10,10 +10,15 @@ LRU model: fully associative, LRU, `line_bytes` lines.
 Warps are interleaved round-robin, one memory instruction per turn. Only
 `a` warps per CTA and `m` CTAs per SM are runnable; a finished warp's slot
 goes to the next waiting warp of its CTA (semaphore semantics), a finished
-CTA's slot to the next CTA of the SM's list. A miss is an *intra-warp
-capacity miss* when the same warp touched that line before: the intra-thread
-/ intra-warp reuse CATT protects. Compulsory misses and lines
-another warp fetched do not count.
+CTA's slot to the next CTA of the SM's list. A miss is an *intra-thread
+capacity miss* when the same thread touched that line before: the
+intra-thread locality CATT protects ("the fetched cache line
+is reused in the following iteration"). Compulsory misses and lines another
+thread fetched (inter-thread reuse, e.g. the line a row ends in and the next
+row starts in) do not count (reading R12).
+
+An event is one warp-level memory instruction: a tuple of (line, thread id)
+pairs, one per active lane.
 """
 from __future__ import annotations
 
@@ -29,7 +34,7 @@ def _line(arr: str, idx: int, line: int = LINE) -> Tuple[str, int]:
 
 
 class Kernel:
-    """nblocks CTAs of W warps; events(b, w) -> list of frozensets of lines."""
+    """nblocks CTAs of W warps; events(b, w) -> list of events."""
     nblocks: int
     W: int
     threads: int
@@ -62,10 +67,10 @@ class RowKernel(Kernel):
             return ev
         for j in range(0, self.N, self.vec):
             if self.with_tmp:
-                ev.append(frozenset(_line("tmp", i) for i in rows))
+                ev.append(tuple((_line("tmp", i), i) for i in rows))
             for X in self.matrices:
-                ev.append(frozenset(_line(X, i * self.N + j) for i in rows))
-                ev.append(frozenset([_line("x", j)]))
+                ev.append(tuple((_line(X, i * self.N + j), i) for i in rows))
+                ev.append(tuple((_line("x", j), i) for i in rows))
         return ev
 
 
@@ -85,8 +90,8 @@ class ColKernel(Kernel):
         if not cols:
             return ev
         for i in range(self.M):
-            ev.append(frozenset(_line("A", i * self.N + j) for j in cols))
-            ev.append(frozenset([_line("v", i)]))
+            ev.append(tuple((_line("A", i * self.N + j), j) for j in cols))
+            ev.append(tuple((_line("v", i), j) for j in cols))
         return ev
 
 
@@ -114,8 +119,8 @@ class SyrkKernel(Kernel):
         if not th:
             return ev
         for k in range(self.Mk):
-            ev.append(frozenset(_line("a", i * self.Mk + k) for i, _ in th))
-            ev.append(frozenset(_line("a", j * self.Mk + k) for _, j in th))
+            ev.append(tuple((_line("a", i * self.Mk + k), (i, j)) for i, j in th))
+            ev.append(tuple((_line("a", j * self.Mk + k), (i, j)) for i, j in th))
         return ev
 
 
@@ -138,7 +143,7 @@ class KmeansKernel(Kernel):
             return ev
         for c in range(self.k):
             for f in range(self.nf):
-                ev.append(frozenset(_line("F", f * self.ld + p) for p in pts))
+                ev.append(tuple((_line("F", f * self.ld + p), p) for p in pts))
         return ev
 
 
@@ -146,8 +151,8 @@ def simulate(kernel: Kernel, sm_blocks: Sequence[int], a: int, m: int, capacity:
     """Run the warps of the CTAs in sm_blocks (in order) with at most a active
     warps per CTA and m active CTAs; LRU of `capacity` lines."""
     cache: "OrderedDict" = OrderedDict()
-    seen: Dict[Tuple[int, int], set] = {}
-    stats = dict(accesses=0, hits=0, misses=0, intra_warp_capacity_misses=0)
+    seen: Dict[object, set] = {}
+    stats = dict(accesses=0, hits=0, misses=0, intra_thread_capacity_misses=0)
     pending = deque(sm_blocks)
     rotation: deque = deque()          # entries: [b, w, events, pos]
     cta_wait: Dict[int, deque] = {}
@@ -170,21 +175,30 @@ def simulate(kernel: Kernel, sm_blocks: Sequence[int], a: int, m: int, capacity:
         ent = rotation.popleft()
         b, w, ev, pos = ent
         if pos < len(ev):
-            key = (b, w)
-            s = seen.setdefault(key, set())
-            for ln in ev[pos]:
+            by_line: Dict[Tuple[str, int], list] = {}
+            for ln, tid in ev[pos]:
+                by_line.setdefault(ln, []).append(tid)
+            # one warp request: every tag is looked up first (hits refresh
+            # their lines), then the missing lines are filled, evicting LRU
+            # lines not touched by this request
+            missing = []
+            for ln, tids in by_line.items():
                 stats["accesses"] += 1
                 if ln in cache:
                     cache.move_to_end(ln)
                     stats["hits"] += 1
                 else:
-                    stats["misses"] += 1
-                    if ln in s:
-                        stats["intra_warp_capacity_misses"] += 1
-                    cache[ln] = True
-                    if len(cache) > capacity:
-                        cache.popitem(last=False)
-                s.add(ln)
+                    missing.append((ln, tids))
+            for ln, tids in missing:
+                stats["misses"] += 1
+                if any(ln in seen.get(t, ()) for t in tids):
+                    stats["intra_thread_capacity_misses"] += 1
+                cache[ln] = True
+                if len(cache) > capacity:
+                    cache.popitem(last=False)
+            for ln, tids in by_line.items():
+                for t in tids:
+                    seen.setdefault(t, set()).add(ln)
             ent[3] = pos + 1
         if ent[3] < len(ev):
             rotation.append(ent)
@@ -206,11 +220,11 @@ def sm0_blocks(kernel: Kernel, num_sms: int, limit: int = 1 << 30) -> List[int]:
 
 def decide_by_lru(kernel: Kernel, W: int, T: int, capacity: int, num_sms: int, limit_blocks=None) -> Tuple[int, int, str]:
     """Walk the Eq 9 candidate order and return the
-    first throttle with zero intra-warp capacity misses."""
+    first throttle with zero intra-thread capacity misses."""
     blocks = sm0_blocks(kernel, num_sms, limit_blocks or max(T, 1))
 
     def ok(a, m):
-        return simulate(kernel, blocks, a, m, capacity)["intra_warp_capacity_misses"] == 0
+        return simulate(kernel, blocks, a, m, capacity)["intra_thread_capacity_misses"] == 0
 
     if ok(W, T):
         return W, T, "none"
