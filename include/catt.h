@@ -1,0 +1,281 @@
+/*
+ * catt.h — C ABI of the B200-native CATT hot path.
+ *
+ * CATT = Compiler-Assisted Thread Throttling (Kim, Hong, Lee, Seo, Han,
+ * ICPP 2019). Citations "P:N" are lines of the paper text.
+ *
+ * Three parts sit behind this boundary:
+ *   1. the footprint analyser (host only): occupancy and carveout (Eq 1-4,
+ *      P:183-208), locality and lines per warp (Eq 5-7), footprint
+ *      and throttle factors (Eq 8-9);
+ *   2. hand-written sm_100a kernels for the loop families of Table 2/3
+ *      (ATAX, BICG, MVT, GESUMMV, SYRK, KMEANS-assign), each with an explicit
+ *      throttle: a per-CTA warp-gating semaphore in shared memory (the B200
+ *      form of Fig 4's warp-level throttling) and a per-SM CTA cap
+ *      (the B200 form of Fig 5's TB-level throttling);
+ *   3. helpers for measurement: the seeded input generator, the L1D capacity
+ *      probe (Fig 3 analog).
+ *
+ * Conventions (all entry points):
+ *   - extern "C", plain pointers and sizes; no exceptions cross the boundary.
+ *   - Device pointers are owned by the caller (the Python layer allocates them
+ *     with PyTorch). The library never frees caller memory. Its only state is
+ *     a per-device cache (hardware table, kernel attributes) and a per-device
+ *     array of num_sms int32 counters for the per-SM CTA cap, allocated on
+ *     first use and left zero by every kernel that uses it.
+ *   - Kernel entry points are asynchronous on `stream` (a cudaStream_t passed
+ *     as void*; NULL = legacy default stream). Nothing synchronises.
+ *   - Arguments are validated synchronously before any launch; invalid input
+ *     returns CATT_EINVAL and launches nothing. A launch failure returns
+ *     CATT_ECUDA (catt_last_cuda_error() gives the cudaError_t value).
+ *   - An unresolvable footprint is a result flag, not an error.
+ *   - fp32 row-major matrices; inputs and outputs must not alias.
+ *   - CTA caps that use the per-SM counters assume capped kernels on one
+ *     device do not run concurrently on different streams.
+ */
+#ifndef CATT_H
+#define CATT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  CATT_OK = 0,
+  CATT_EINVAL = -1,       /* bad argument or throttle (nothing launched)   */
+  CATT_ECUDA = -2,        /* CUDA runtime error (see catt_last_cuda_error)  */
+  CATT_EUNSUPPORTED = -3, /* valid but not supported (e.g. window too big)  */
+  CATT_ENOMEM = -4,       /* library workspace allocation failed            */
+  CATT_ENODEV = -5        /* no CUDA device                                 */
+} catt_status;
+
+enum { CATT_MAX_LOOPS = 4, CATT_MAX_CARVEOUTS = 16 };
+
+/* catt_ref.flags */
+enum {
+  CATT_REF_IRREGULAR = 1, /* indirect access: C_tid := 1                      */
+  CATT_REF_STORE = 2,     /* store: counted in paper mode, not in union mode          */
+  CATT_REF_NOT_L1 = 4     /* register / shared memory / L1-bypassing: not counted     */
+};
+
+/* catt_loop_desc.mode */
+enum {
+  CATT_MODE_UNION = 0, /* B200 default: exact distinct lines of co-resident warps */
+  CATT_MODE_PAPER = 1  /* Eq 7-9 as printed: per-warp sum of REQ_warp            */
+};
+
+/* catt_footprint_result.flags */
+enum {
+  CATT_FIT_NONE_NEEDED = 1, /* fits at full TLP, or the loop has no locality */
+  CATT_FIT_WARP = 2,        /* warp-level throttle (N of Eq 9)                         */
+  CATT_FIT_CTA = 4,         /* TB-level throttle (M of Eq 9), one warp per CTA          */
+  CATT_FIT_UNRESOLVABLE = 8 /* nothing fits even at (1,1): left unthrottled    */
+};
+
+/* One memory instruction in the loop (Eq 5):
+ *   element index = base + sum_d c_gid[d] * gid_d + sum_k c_iter[k] * i_k
+ * gid_d = blockIdx_d * blockDim_d + threadIdx_d (the paper's C_tid is c_gid[0]
+ * for 1-D blocks); i_k are the loop induction variables, outer to inner
+ * (C_i). Arrays are assumed to start on a line boundary; refs with the same
+ * array_id address the same array (their lines are shared). */
+typedef struct {
+  int64_t c_gid[3];
+  int64_t c_iter[CATT_MAX_LOOPS];
+  int64_t base;
+  int32_t elem_bytes;
+  int32_t flags;
+  int32_t array_id;
+  int32_t reserved_;
+} catt_ref;
+
+/* A loop and its launch. trip[k] = iterations of loop k (outer to inner).
+ * extent[d] > 0 bounds gid_d (threads with gid_d >= extent[d] do not access,
+ * the usual `if (i < N)` guard). regs_per_thread / smem_per_cta come from the
+ * compiled kernel (0 = no limit). force_carveout_kb >= 0 pins the shared
+ * memory option ("we configured the L1D to 32KB"); < 0 chooses it by
+ * Eq 4. */
+typedef struct {
+  int32_t n_refs;
+  int32_t n_loops;
+  const catt_ref* refs;
+  int64_t trip[CATT_MAX_LOOPS];
+  int32_t block[3];
+  int32_t mode;
+  int64_t grid[3];
+  int64_t extent[3];
+  int32_t regs_per_thread;
+  int32_t smem_per_cta;
+  int32_t force_carveout_kb;
+  int32_t reserved_;
+} catt_loop_desc;
+
+/* Hardware parameters. carveout_kb[i] are the configurable shared-memory
+ * sizes per SM (ascending); l1d_bytes[i] the L1D capacity that option leaves
+ * (measured on B200, see catt_hw_b200); carveout_pct[i] the
+ * cudaFuncAttributePreferredSharedMemoryCarveout value that selects it. */
+typedef struct {
+  int32_t num_sms, max_warps_sm, max_ctas_sm, regs_sm, reg_alloc_unit, warp_size;
+  int32_t smem_alloc_unit, reserved_smem_cta, line_bytes, n_carveouts;
+  int32_t carveout_kb[CATT_MAX_CARVEOUTS];
+  int32_t carveout_pct[CATT_MAX_CARVEOUTS];
+  int64_t l1d_bytes[CATT_MAX_CARVEOUTS];
+} catt_hw;
+
+typedef struct {
+  int64_t lines_per_warp_iter; /* sum over refs of lines warp 0 touches in iteration 0 (Eq 7) */
+  int64_t reuse_span;          /* lines warp 0 retains until reuse                             */
+  int64_t footprint_lines_full;/* F(#Warps_TB, #TB_SM), Eq 8                                    */
+  int64_t footprint_lines;     /* F at the chosen (active_warps, active_ctas), Eq 9            */
+  int64_t footprint_bytes;     /* footprint_lines * line_bytes                                  */
+  int64_t l1d_bytes;           /* L1D left by the chosen carveout                               */
+  int32_t base_warps, base_ctas;     /* (#Warps_TB, #TB_SM) at full TLP, Eq 1-3                */
+  int32_t active_warps, active_ctas; /* the throttle: warps per CTA, CTAs per SM                */
+  int32_t carveout_kb;               /* Eq 4 (or forced)                                        */
+  int32_t flags;                     /* CATT_FIT_*                                              */
+} catt_footprint_result;
+
+/* Kernel variants (all compute the same loop):
+ *   LITERAL  the paper's loop: one thread per output, scalar loads through L1,
+ *            sequential order (bit-exact to the sequential-fmaf oracle).
+ *   VEC4     one thread per output, 16-byte loads, same sequential order.
+ *   STAGED   one thread per output, tiles moved to shared memory by
+ *            cp.async.bulk (TMA bulk copies), same sequential order; does not
+ *            rely on L1 reuse.
+ *   COOP     warp-cooperative coalesced loads with shuffle/split reductions:
+ *            the HBM-roofline variant; summation order differs (fp64-oracle
+ *            tolerance, bit-exact on exact-dyadic inputs).
+ *   REGS     (KMEANS) the point's features are loaded once into registers.  */
+enum { CATT_VAR_LITERAL = 0, CATT_VAR_VEC4 = 1, CATT_VAR_STAGED = 2, CATT_VAR_COOP = 3, CATT_VAR_REGS = 4 };
+
+/* Warp-level mechanism: SEMAPHORE = per-CTA counting semaphore in shared
+ * memory (a finished warp's slot goes to the next waiting warp);
+ * BARRIER = Fig 4 literally (warp groups run in turn between __syncthreads). */
+enum { CATT_GATE_SEMAPHORE = 0, CATT_GATE_BARRIER = 1 };
+/* CTA-level mechanism: SM_COUNTER = per-SM counter in global memory (exact
+ * cap whatever the driver's carveout choice); SMEM_PAD = Fig 5 literally
+ * (dynamic shared memory pad sized so only active_ctas fit the carveout). */
+enum { CATT_CAP_SM_COUNTER = 0, CATT_CAP_SMEM_PAD = 1 };
+
+/* Launch + throttle of one loop. Zero-initialised = default launch (256
+ * threads, LITERAL, no throttle, carveout preference 0 %). */
+typedef struct {
+  int32_t cta_threads;  /* threads per CTA (multiple of 32, <= 1024); 0 = 256; SYRK: 2-D 32 x (cta_threads/32) */
+  int32_t active_warps; /* warps of a CTA allowed in the loop at once; 0 = all (#Warps_TB)                   */
+  int32_t active_ctas;  /* CTAs of an SM allowed in the loop at once; 0 = no cap                            */
+  int32_t carveout_kb;  /* shared-memory option to request; 0 = max L1D; < 0 = leave the driver default      */
+  int32_t variant;      /* CATT_VAR_*                                                                          */
+  int32_t gate;         /* CATT_GATE_*                                                                         */
+  int32_t cap;          /* CATT_CAP_*                                                                          */
+  int32_t reserved_;
+  uint64_t* probe;      /* optional device buffer: per warp {smid, t_start_ns, t_end_ns} around the loop,
+                           indexed by (linear CTA id * warps per CTA + warp) * 3; NULL = off             */
+} catt_throttle;
+
+/* Loop identifiers for catt_kernel_desc / catt_plan: one per loop of Table 3. */
+enum {
+  CATT_K_ATAX_1 = 0,  /* tmp = A x        (row per thread, memory-divergent)  */
+  CATT_K_ATAX_2 = 1,  /* y = A^T tmp      (column per thread, coalesced)      */
+  CATT_K_BICG_1 = 2,  /* s = A^T r        (column per thread)                 */
+  CATT_K_BICG_2 = 3,  /* q = A p          (row per thread)                    */
+  CATT_K_MVT_1 = 4,   /* x1 += A y1       (row per thread)                    */
+  CATT_K_MVT_2 = 5,   /* x2 += A^T y2     (column per thread)                 */
+  CATT_K_GESUMMV = 6, /* y = alpha A x + beta B x (row per thread, 2 matrices)*/
+  CATT_K_SYRK = 7,    /* C = beta C + alpha A A^T (2-D block 32 x 8)          */
+  CATT_K_KMEANS = 8,  /* membership = argmin_c |f_p - c|^2, feature-major     */
+  CATT_K_COUNT = 9
+};
+
+/* Problem sizes: ATAX/BICG m x n (rows, cols); MVT/GESUMMV n (m ignored);
+ * SYRK n x n output, k = inner size m; KMEANS m = npoints, n = nfeatures,
+ * k = clusters, ld = feature-major leading dimension. */
+typedef struct {
+  int32_t loop;
+  int32_t reserved_;
+  int64_t m, n, k, ld;
+} catt_problem;
+
+/* ------------------------------------------------------------------ hardware */
+/* Device properties + the L1D table of catt_hw_b200 (CATT_ENODEV without a GPU). */
+catt_status catt_hw_query(int device, catt_hw* out);
+/* B200 (sm_100a, 148 SMs) with the L1D capacities measured per carveout option
+ * by the Fig 3-style footprint sweep (profiles/round1_probe_hw.txt). No GPU needed. */
+catt_status catt_hw_b200(catt_hw* out);
+/* Titan V, the paper's GPU: Table 1, 64 warps/SM, shared
+ * memory options 0/8/16/32/64/96 KB with L1D = 128 KB - option. */
+catt_status catt_hw_titanv(catt_hw* out);
+
+/* ------------------------------------------------------------------ analyser */
+/* Steps a1-a5 (Eq 1-9). Host only, no device work; deterministic. */
+catt_status catt_footprint(const catt_loop_desc* desc, const catt_hw* hw, catt_footprint_result* out);
+
+/* The descriptor of this library's kernel for one loop of `prob` under the
+ * launch in `t` (cta_threads, variant; throttle fields ignored). refs_buf must
+ * hold `cap` refs (8 is enough for every loop). regs_per_thread comes from
+ * cudaFuncGetAttributes when a device is present, else 0 (unknown). */
+catt_status catt_kernel_desc(const catt_problem* prob, const catt_throttle* t, int32_t mode,
+                             catt_loop_desc* out, catt_ref* refs_buf, int32_t cap);
+
+/* catt_kernel_desc + catt_footprint, and the throttle to launch with: `out` =
+ * `launch` with active_warps / active_ctas / carveout_kb set to the CATT pick. */
+catt_status catt_plan(const catt_problem* prob, const catt_throttle* launch, const catt_hw* hw, int32_t mode,
+                      catt_throttle* out, catt_footprint_result* res);
+
+/* ------------------------------------------------------------------ kernels */
+/* ATAX (Table 3): tmp = A x (loop 1, throttle k1), then
+ * y = A^T tmp (loop 2, throttle k2). A is m x n; x[n], tmp[m], y[n] device
+ * pointers; tmp and y are overwritten. For a row shard, y is the shard's
+ * partial A_g^T tmp_g (the caller all-reduces). */
+catt_status catt_atax(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n,
+                      const catt_throttle* k1, const catt_throttle* k2, void* stream);
+
+/* BICG (Table 2, Table 3): s = A^T r (loop 1, k1) and q = A p
+ * (loop 2, k2). A is nx x ny; p[ny], r[nx], q[nx], s[ny]; q, s overwritten. */
+catt_status catt_bicg(const float* A, const float* p, const float* r, float* q, float* s, int64_t nx, int64_t ny,
+                      const catt_throttle* k1, const catt_throttle* k2, void* stream);
+
+/* MVT (Table 2, Table 3): x1 += A y1 (loop 1, k1) and
+ * x2 += A^T y2 (loop 2, k2). A is n x n; x1, x2 in/out. */
+catt_status catt_mvt(const float* A, const float* y1, const float* y2, float* x1, float* x2, int64_t n,
+                     const catt_throttle* k1, const catt_throttle* k2, void* stream);
+
+/* GESUMMV (Table 2, Table 3): tmp = A x, y = alpha*tmp + beta*(B x)
+ * in one loop over j. A, B n x n; x[n]; y[n], tmp[n] overwritten. */
+catt_status catt_gesummv(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t n,
+                         float alpha, float beta, const catt_throttle* t, void* stream);
+
+/* SYRK (Table 2): C = beta*C + alpha*A*A^T over the full n x n square.
+ * A is n x m; C in/out. LITERAL = 2-D block 32 x (cta_threads/32), one thread
+ * per C element; STAGED = shared-memory tiles, register blocking, same k order. */
+catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta,
+                      const catt_throttle* t, void* stream);
+
+/* KMEANS assignment (Table 2, Table 3): feat is feature-major,
+ * feat[f*ld + p] for f < nf, p < npoints (ld >= npoints); clusters is k x nf;
+ * membership[npoints] int32 overwritten with the lowest-index nearest centre.
+ * Requires nf * k <= 4096 (the centres are staged in shared memory). */
+catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters,
+                               int32_t k, int32_t* membership, const catt_throttle* t, void* stream);
+
+/* ------------------------------------------------------------------ helpers */
+/* dst[i] = value(seed, offset + i): the counter-based generator of
+ * seeded_inputs.py (mode 0 uniform [0,1), 1 dyadic k/16). Device pointer. */
+catt_status catt_fill_hash(float* dst, int64_t n, uint32_t seed, uint64_t offset, int32_t mode, void* stream);
+
+/* Fig 3 analog: one thread chases a cyclic chain of `kb` KiB (one
+ * load per 128-B line) under carveout preference `pct`, 4 passes; writes the
+ * mean cycles per load for each size. Synchronous. */
+catt_status catt_calibrate_l1(int device, int32_t pct, const int32_t* kb, int32_t n, float* cycles_out);
+
+/* Number of registers / static shared bytes of the kernel a loop+launch uses. */
+catt_status catt_kernel_attrs(const catt_problem* prob, const catt_throttle* t, int32_t* regs, int32_t* static_smem);
+
+const char* catt_status_str(catt_status s);
+int catt_last_cuda_error(void);
+int catt_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CATT_H */

@@ -53,6 +53,8 @@ def lib():
         L.orc_mvt.argtypes = [ctypes.c_int, f32p, f32p, f32p, f32p, f32p, i64]
         L.orc_gesummv.argtypes = [ctypes.c_int, f32p, f32p, f32p, f32p, f32p, i64, ctypes.c_float, ctypes.c_float]
         L.orc_syrk.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float]
+        L.orc_syrk_rows.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float,
+                                    ctypes.POINTER(ctypes.c_int64), i64, f32p]
         L.orc_kmeans_assign.argtypes = [ctypes.c_int, f32p, i64, i64, i32, f32p, i32,
                                         ctypes.POINTER(ctypes.c_int32), f32p]
         L.orc_atax_hashed.argtypes = [ctypes.c_int, u32, ctypes.c_int, f32p, i64, i64, f32p,
@@ -124,6 +126,16 @@ def syrk(A, C, alpha, beta, mode=SEQ_FMAF):
     n, m = A.shape
     lib().orc_syrk(mode, _p(A), _p(C), n, m, alpha, beta)
     return C
+
+
+def syrk_rows(A, C, alpha, beta, rows, mode=SEQ_FMAF):
+    """Rows `rows` of syrk(A, C, alpha, beta) without computing the rest."""
+    A, C = _f32(A), _f32(C)
+    n, m = A.shape
+    rows = np.ascontiguousarray(rows, dtype=np.int64)
+    out = np.empty((len(rows), n), np.float32)
+    lib().orc_syrk_rows(mode, _p(A), _p(C), n, m, alpha, beta, _p(rows), len(rows), _p(out))
+    return out
 
 
 def kmeans_assign(feat, ld, npoints, nf, clusters, mode=SEQ_FMAF):

@@ -214,6 +214,26 @@ int orc_syrk(int mode, const float* A, float* C, int64_t n, int64_t m, float alp
   return 0;
 }
 
+/* The same SYRK loop nest restricted to the output rows rows[0..nrows):
+ * out[r][j] for the r-th listed row (full-size sampled checks). */
+int orc_syrk_rows(int mode, const float* A, const float* C, int64_t n, int64_t m, float alpha, float beta,
+                  const int64_t* rows, int64_t nrows, float* out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t q = 0; q < nrows * n; ++q) {
+    const int64_t i = rows[q / n], j = q % n;
+    if (mode == ORC_SEQ_FMAF) {
+      float c = C[i * n + j] * beta;
+      for (int64_t k = 0; k < m; ++k) c = fmaf(alpha * A[i * m + k], A[j * m + k], c);
+      out[q] = c;
+    } else {
+      double c = (double)C[i * n + j] * (double)beta;
+      for (int64_t k = 0; k < m; ++k) c += (double)alpha * (double)A[i * m + k] * (double)A[j * m + k];
+      out[q] = (float)c;
+    }
+  }
+  return 0;
+}
+
 /* ---------------------------------------------------------------- KMEANS assign
  * Rodinia kmeans (Table 2; Table 3), assignment step
  * (kmeansPoint), features stored feature-major: feat[f*ld + p].

@@ -1,0 +1,362 @@
+"""Python binding of the CATT C ABI (include/catt.h) — argument marshalling only.
+
+Every step of the hot path runs in libcatt.so (hand-written sm_100a kernels and
+the C++ footprint analyser). There is no CPU fallback: if the library is
+missing or a call fails, an exception is raised. Device tensors are PyTorch
+tensors (float32, contiguous, on the current CUDA device); the stream is
+torch's current stream.
+
+Names follow the C ABI without the `catt_` prefix.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Tuple
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libcatt.so")
+
+# ------------------------------------------------------------------ constants (catt.h)
+OK, EINVAL, ECUDA, EUNSUPPORTED, ENOMEM, ENODEV = 0, -1, -2, -3, -4, -5
+MAX_LOOPS, MAX_CARVEOUTS = 4, 16
+REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
+MODE_UNION, MODE_PAPER = 0, 1
+FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE = 1, 2, 4, 8
+VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS = 0, 1, 2, 3, 4
+GATE_SEMAPHORE, GATE_BARRIER = 0, 1
+CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
+(K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS) = range(9)
+
+VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS}
+FLAG_NAMES = {FIT_NONE_NEEDED: "none", FIT_WARP: "warp", FIT_CTA: "cta", FIT_UNRESOLVABLE: "unresolvable"}
+
+
+class CattError(RuntimeError):
+    pass
+
+
+# ------------------------------------------------------------------ structs
+class Ref(ctypes.Structure):
+    _fields_ = [("c_gid", ctypes.c_int64 * 3), ("c_iter", ctypes.c_int64 * MAX_LOOPS), ("base", ctypes.c_int64),
+                ("elem_bytes", ctypes.c_int32), ("flags", ctypes.c_int32), ("array_id", ctypes.c_int32),
+                ("reserved_", ctypes.c_int32)]
+
+
+class LoopDesc(ctypes.Structure):
+    _fields_ = [("n_refs", ctypes.c_int32), ("n_loops", ctypes.c_int32), ("refs", ctypes.POINTER(Ref)),
+                ("trip", ctypes.c_int64 * MAX_LOOPS), ("block", ctypes.c_int32 * 3), ("mode", ctypes.c_int32),
+                ("grid", ctypes.c_int64 * 3), ("extent", ctypes.c_int64 * 3), ("regs_per_thread", ctypes.c_int32),
+                ("smem_per_cta", ctypes.c_int32), ("force_carveout_kb", ctypes.c_int32), ("reserved_", ctypes.c_int32)]
+
+
+class Hw(ctypes.Structure):
+    _fields_ = [("num_sms", ctypes.c_int32), ("max_warps_sm", ctypes.c_int32), ("max_ctas_sm", ctypes.c_int32),
+                ("regs_sm", ctypes.c_int32), ("reg_alloc_unit", ctypes.c_int32), ("warp_size", ctypes.c_int32),
+                ("smem_alloc_unit", ctypes.c_int32), ("reserved_smem_cta", ctypes.c_int32),
+                ("line_bytes", ctypes.c_int32), ("n_carveouts", ctypes.c_int32),
+                ("carveout_kb", ctypes.c_int32 * MAX_CARVEOUTS), ("carveout_pct", ctypes.c_int32 * MAX_CARVEOUTS),
+                ("l1d_bytes", ctypes.c_int64 * MAX_CARVEOUTS)]
+
+    def as_dict(self):
+        n = self.n_carveouts
+        d = {f: getattr(self, f) for f, _ in self._fields_[:10]}
+        d["carveout_kb"] = list(self.carveout_kb[:n])
+        d["carveout_pct"] = list(self.carveout_pct[:n])
+        d["l1d_bytes"] = list(self.l1d_bytes[:n])
+        return d
+
+    @classmethod
+    def from_dict(cls, d):
+        h = cls()
+        for f, _ in cls._fields_[:10]:
+            if f in d:
+                setattr(h, f, d[f])
+        n = len(d["carveout_kb"])
+        h.n_carveouts = n
+        for i in range(n):
+            h.carveout_kb[i] = d["carveout_kb"][i]
+            h.carveout_pct[i] = d.get("carveout_pct", [0] * n)[i]
+            h.l1d_bytes[i] = d["l1d_bytes"][i]
+        return h
+
+
+class FootprintResult(ctypes.Structure):
+    _fields_ = [("lines_per_warp_iter", ctypes.c_int64), ("reuse_span", ctypes.c_int64),
+                ("footprint_lines_full", ctypes.c_int64), ("footprint_lines", ctypes.c_int64),
+                ("footprint_bytes", ctypes.c_int64), ("l1d_bytes", ctypes.c_int64),
+                ("base_warps", ctypes.c_int32), ("base_ctas", ctypes.c_int32), ("active_warps", ctypes.c_int32),
+                ("active_ctas", ctypes.c_int32), ("carveout_kb", ctypes.c_int32), ("flags", ctypes.c_int32)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+class Throttle(ctypes.Structure):
+    """catt_throttle. Zero = default launch (256 threads, LITERAL, full TLP)."""
+    _fields_ = [("cta_threads", ctypes.c_int32), ("active_warps", ctypes.c_int32), ("active_ctas", ctypes.c_int32),
+                ("carveout_kb", ctypes.c_int32), ("variant", ctypes.c_int32), ("gate", ctypes.c_int32),
+                ("cap", ctypes.c_int32), ("reserved_", ctypes.c_int32), ("probe", ctypes.c_void_p)]
+
+    def __init__(self, cta_threads=0, active_warps=0, active_ctas=0, carveout_kb=0, variant=VAR_LITERAL,
+                 gate=GATE_SEMAPHORE, cap=CAP_SM_COUNTER, probe=None):
+        if isinstance(variant, str):
+            variant = VARIANTS[variant]
+        super().__init__(cta_threads, active_warps, active_ctas, carveout_kb, variant, gate, cap, 0,
+                         probe if probe is None else int(probe))
+
+    def copy(self, **kw):
+        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "reserved_"}
+        d.update(kw)
+        return Throttle(**d)
+
+    def __repr__(self):
+        return (f"Throttle(cta={self.cta_threads}, warps={self.active_warps}, ctas={self.active_ctas}, "
+                f"carveout={self.carveout_kb}KB, variant={self.variant}, gate={self.gate}, cap={self.cap})")
+
+
+class Problem(ctypes.Structure):
+    _fields_ = [("loop", ctypes.c_int32), ("reserved_", ctypes.c_int32), ("m", ctypes.c_int64),
+                ("n", ctypes.c_int64), ("k", ctypes.c_int64), ("ld", ctypes.c_int64)]
+
+
+# ------------------------------------------------------------------ library
+_lib = None
+
+
+def lib():
+    """Load libcatt.so (building it with nvcc if it is absent or stale)."""
+    global _lib
+    if _lib is None:
+        from . import build as _build
+        if not _build.up_to_date():
+            _build.build()
+        if not os.path.exists(LIB_PATH):
+            raise CattError(f"libcatt.so missing at {LIB_PATH}: the CUDA extension is required (no CPU fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        P, V, i32, i64, u32, u64, f32 = (ctypes.POINTER, ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64,
+                                         ctypes.c_uint32, ctypes.c_uint64, ctypes.c_float)
+        T = P(Throttle)
+        sig = {
+            "catt_hw_query": [ctypes.c_int, P(Hw)],
+            "catt_hw_b200": [P(Hw)],
+            "catt_hw_titanv": [P(Hw)],
+            "catt_footprint": [P(LoopDesc), P(Hw), P(FootprintResult)],
+            "catt_kernel_desc": [P(Problem), T, i32, P(LoopDesc), P(Ref), i32],
+            "catt_plan": [P(Problem), T, P(Hw), i32, T, P(FootprintResult)],
+            "catt_atax": [V, V, V, V, i64, i64, T, T, V],
+            "catt_bicg": [V, V, V, V, V, i64, i64, T, T, V],
+            "catt_mvt": [V, V, V, V, V, i64, T, T, V],
+            "catt_gesummv": [V, V, V, V, V, i64, f32, f32, T, V],
+            "catt_syrk": [V, V, i64, i64, f32, f32, T, V],
+            "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
+            "catt_fill_hash": [V, i64, u32, u64, i32, V],
+            "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
+            "catt_kernel_attrs": [P(Problem), T, P(i32), P(i32)],
+            "catt_status_str": [ctypes.c_int],
+            "catt_last_cuda_error": [],
+            "catt_abi_version": [],
+        }
+        for name, args in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = ctypes.c_int
+        L.catt_status_str.restype = ctypes.c_char_p
+        _lib = L
+    return _lib
+
+
+EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
+            "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_kmeans_assign",
+            "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
+            "catt_last_cuda_error", "catt_abi_version"]
+
+
+def _check(st: int, what: str):
+    if st != OK:
+        L = lib()
+        msg = L.catt_status_str(st).decode()
+        extra = f" (cudaError {L.catt_last_cuda_error()})" if st == ECUDA else ""
+        raise CattError(f"{what}: {msg}{extra}")
+
+
+# ------------------------------------------------------------------ hardware / analyser
+def hw_b200() -> Hw:
+    h = Hw()
+    _check(lib().catt_hw_b200(ctypes.byref(h)), "catt_hw_b200")
+    return h
+
+
+def hw_titanv() -> Hw:
+    h = Hw()
+    _check(lib().catt_hw_titanv(ctypes.byref(h)), "catt_hw_titanv")
+    return h
+
+
+def hw_query(device: int = 0) -> Hw:
+    h = Hw()
+    _check(lib().catt_hw_query(device, ctypes.byref(h)), "catt_hw_query")
+    return h
+
+
+def make_desc(refs, trips, block, grid, extent=(0, 0, 0), regs=0, smem=0, mode=MODE_UNION, force_carveout_kb=-1):
+    """Build a LoopDesc from plain tuples. refs: dicts with c_gid, c_iter and
+    optional base, elem_bytes, flags, array_id. Returns (desc, keepalive)."""
+    arr = (Ref * max(1, len(refs)))()
+    for i, r in enumerate(refs):
+        g = list(r["c_gid"]) + [0] * (3 - len(r["c_gid"]))
+        it = list(r["c_iter"]) + [0] * (MAX_LOOPS - len(r["c_iter"]))
+        arr[i].c_gid[:] = g
+        arr[i].c_iter[:] = it
+        arr[i].base = r.get("base", 0)
+        arr[i].elem_bytes = r.get("elem_bytes", 4)
+        arr[i].flags = r.get("flags", 0)
+        arr[i].array_id = r.get("array_id", 0)
+    d = LoopDesc()
+    d.n_refs = len(refs)
+    d.n_loops = len(trips)
+    d.refs = ctypes.cast(arr, ctypes.POINTER(Ref))
+    d.trip[:] = list(trips) + [0] * (MAX_LOOPS - len(trips))
+    d.block[:] = list(block)
+    d.grid[:] = list(grid)
+    d.extent[:] = list(extent)
+    d.mode = mode
+    d.regs_per_thread = regs
+    d.smem_per_cta = smem
+    d.force_carveout_kb = force_carveout_kb
+    return d, arr
+
+
+def footprint(desc: LoopDesc, hw: Hw) -> dict:
+    r = FootprintResult()
+    _check(lib().catt_footprint(ctypes.byref(desc), ctypes.byref(hw), ctypes.byref(r)), "catt_footprint")
+    return r.as_dict()
+
+
+def problem(loop: int, m=0, n=0, k=0, ld=0) -> Problem:
+    return Problem(loop, 0, m, n, k, ld)
+
+
+def kernel_desc(prob: Problem, launch: Optional[Throttle] = None, mode: int = MODE_UNION):
+    refs = (Ref * 8)()
+    d = LoopDesc()
+    _check(lib().catt_kernel_desc(ctypes.byref(prob), ctypes.byref(launch) if launch else None, mode,
+                                  ctypes.byref(d), refs, 8), "catt_kernel_desc")
+    return d, refs
+
+
+def plan(prob: Problem, launch: Optional[Throttle] = None, hw: Optional[Hw] = None,
+         mode: int = MODE_UNION) -> Tuple[Throttle, dict]:
+    """The CATT throttle for one loop (catt_plan)."""
+    if hw is None:
+        hw = hw_query()
+    out, r = Throttle(), FootprintResult()
+    _check(lib().catt_plan(ctypes.byref(prob), ctypes.byref(launch) if launch else None, ctypes.byref(hw), mode,
+                           ctypes.byref(out), ctypes.byref(r)), "catt_plan")
+    return out, r.as_dict()
+
+
+def kernel_attrs(prob: Problem, launch: Optional[Throttle] = None) -> Tuple[int, int]:
+    regs, smem = ctypes.c_int32(), ctypes.c_int32()
+    _check(lib().catt_kernel_attrs(ctypes.byref(prob), ctypes.byref(launch) if launch else None,
+                                   ctypes.byref(regs), ctypes.byref(smem)), "catt_kernel_attrs")
+    return regs.value, smem.value
+
+
+# ------------------------------------------------------------------ device calls
+def _torch():
+    import torch
+    return torch
+
+
+def _dev(t, name, dtype=None):
+    torch = _torch()
+    dtype = dtype or torch.float32
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise CattError(f"{name}: expected a CUDA tensor")
+    if t.dtype != dtype or not t.is_contiguous():
+        raise CattError(f"{name}: expected a contiguous {dtype} tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _stream():
+    return ctypes.c_void_p(_torch().cuda.current_stream().cuda_stream)
+
+
+def _tp(t: Optional[Throttle]):
+    return ctypes.byref(t) if t is not None else None
+
+
+def atax(A, x, tmp=None, y=None, k1: Optional[Throttle] = None, k2: Optional[Throttle] = None):
+    """tmp = A x; y = A^T tmp (catt_atax). Returns (tmp, y)."""
+    torch = _torch()
+    m, n = A.shape
+    tmp = torch.empty(m, device=A.device) if tmp is None else tmp
+    y = torch.empty(n, device=A.device) if y is None else y
+    _check(lib().catt_atax(_dev(A, "A"), _dev(x, "x"), _dev(tmp, "tmp"), _dev(y, "y"), m, n, _tp(k1), _tp(k2),
+                           _stream()), "catt_atax")
+    return tmp, y
+
+
+def bicg(A, p, r, q=None, s=None, k1: Optional[Throttle] = None, k2: Optional[Throttle] = None):
+    """s = A^T r (loop 1), q = A p (loop 2) (catt_bicg). Returns (q, s)."""
+    torch = _torch()
+    nx, ny = A.shape
+    q = torch.empty(nx, device=A.device) if q is None else q
+    s = torch.empty(ny, device=A.device) if s is None else s
+    _check(lib().catt_bicg(_dev(A, "A"), _dev(p, "p"), _dev(r, "r"), _dev(q, "q"), _dev(s, "s"), nx, ny,
+                           _tp(k1), _tp(k2), _stream()), "catt_bicg")
+    return q, s
+
+
+def mvt(A, y1, y2, x1, x2, k1: Optional[Throttle] = None, k2: Optional[Throttle] = None):
+    """x1 += A y1, x2 += A^T y2, in place (catt_mvt). Returns (x1, x2)."""
+    n = A.shape[0]
+    _check(lib().catt_mvt(_dev(A, "A"), _dev(y1, "y1"), _dev(y2, "y2"), _dev(x1, "x1"), _dev(x2, "x2"), n,
+                          _tp(k1), _tp(k2), _stream()), "catt_mvt")
+    return x1, x2
+
+
+def gesummv(A, B, x, alpha, beta, y=None, tmp=None, t: Optional[Throttle] = None):
+    """y = alpha A x + beta B x, tmp = A x (catt_gesummv). Returns (y, tmp)."""
+    torch = _torch()
+    n = A.shape[0]
+    y = torch.empty(n, device=A.device) if y is None else y
+    tmp = torch.empty(n, device=A.device) if tmp is None else tmp
+    _check(lib().catt_gesummv(_dev(A, "A"), _dev(B, "B"), _dev(x, "x"), _dev(y, "y"), _dev(tmp, "tmp"), n,
+                              float(alpha), float(beta), _tp(t), _stream()), "catt_gesummv")
+    return y, tmp
+
+
+def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):
+    """C = beta C + alpha A A^T in place (catt_syrk). Returns C."""
+    n, m = A.shape
+    _check(lib().catt_syrk(_dev(A, "A"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t), _stream()),
+           "catt_syrk")
+    return C
+
+
+def kmeans_assign(feat, ld, npoints, nf, clusters, membership=None, t: Optional[Throttle] = None):
+    """membership[p] = argmin_c |feat[:, p] - clusters[c]|^2 (catt_kmeans_assign)."""
+    torch = _torch()
+    k = clusters.shape[0]
+    membership = torch.empty(npoints, dtype=torch.int32, device=feat.device) if membership is None else membership
+    _check(lib().catt_kmeans_assign(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"), k,
+                                    _dev(membership, "membership", torch.int32), _tp(t), _stream()),
+           "catt_kmeans_assign")
+    return membership
+
+
+def fill_hash(t, seed: int, offset: int = 0, mode: int = 0):
+    """Fill a CUDA float32 tensor with the seeded_inputs generator (in device code)."""
+    _check(lib().catt_fill_hash(_dev(t, "t"), t.numel(), seed & 0xFFFFFFFF, offset, mode, _stream()),
+           "catt_fill_hash")
+    return t
+
+
+def calibrate_l1(device: int, pct: int, kb_list):
+    n = len(kb_list)
+    kb = (ctypes.c_int32 * n)(*kb_list)
+    out = (ctypes.c_float * n)()
+    _check(lib().catt_calibrate_l1(device, pct, kb, n, out), "catt_calibrate_l1")
+    return list(out)

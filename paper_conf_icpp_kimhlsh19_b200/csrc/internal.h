@@ -1,0 +1,39 @@
+// internal.h — host-side launch plumbing shared by the kernel files.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+#include "../../include/catt.h"
+#include "common.cuh"
+
+namespace catt {
+
+struct DevCtx {
+  int device = -1;
+  catt_hw hw{};
+  int* sm_counter = nullptr;  // hw.num_sms int32, zero between capped launches
+};
+
+// Per-device context of the current device (hardware table, CTA-cap counters).
+catt_status dev_ctx(DevCtx** out);
+
+// Validates the throttle for a kernel with `threads` threads per CTA, applies
+// the carveout preference to `func`, and fills the device-side Throttle.
+// dyn_smem is the kernel's own dynamic shared memory; *dyn_total receives it
+// plus the Fig 5 pad when cap == CATT_CAP_SMEM_PAD. allow_warp_gate=false
+// rejects active_warps < #warps (pipelined variants cannot gate warps).
+catt_status prepare_launch(const void* func, const catt_throttle* t, int threads, size_t dyn_smem,
+                           bool allow_warp_gate, Throttle* kt, size_t* dyn_total);
+
+// cudaGetLastError after a launch -> CATT_OK / CATT_ECUDA (and records it).
+catt_status after_launch();
+void record_cuda_error(cudaError_t e);
+
+inline int cta_threads_or(const catt_throttle* t, int def) {
+  return (t && t->cta_threads > 0) ? t->cta_threads : def;
+}
+inline int variant_of(const catt_throttle* t) { return t ? t->variant : CATT_VAR_LITERAL; }
+
+}  // namespace catt

@@ -1,0 +1,369 @@
+"""GPU parity tests: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bars:
+  - LITERAL / VEC4 / STAGED variants and SYRK STAGED keep the sequential
+    per-output order: bit-exact to the oracle's seq-fmaf mode;
+  - COOP variants reorder the sums: max relative error <= 1e-5 against the
+    fp64 oracle (BASELINE north_star), and bit-exact on exact-dyadic inputs;
+  - KMEANS membership: bit-exact (decided in fp32 in the same order);
+  - throttles never change results; the residency probe shows them enforced.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle
+import paper_conf_icpp_kimhlsh19_b200 as catt
+import seeded_inputs as si
+
+pytestmark = pytest.mark.gpu
+DYADIC = si.MODE_DYADIC
+TOL = 1e-5
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def relerr(got, ref):
+    got, ref = np.asarray(got, np.float64), np.asarray(ref, np.float64)
+    return float(np.max(np.abs(got - ref) / np.maximum(np.abs(ref), 1e-30))) if got.size else 0.0
+
+
+def bits_equal(a, b):
+    return np.array_equal(np.asarray(a, np.float32).view(np.uint32), np.asarray(b, np.float32).view(np.uint32))
+
+
+EXACT = ["literal", "vec4", "staged"]
+ROW_SHAPES = [(257, 36), (64, 1024), (1000, 132), (33, 4)]      # ragged rows/cols, several tiles and warps
+COL_SHAPES = [(36, 257), (1024, 64), (131, 1000), (4, 33)]
+
+
+# ------------------------------------------------------------------ generator
+@pytest.mark.parametrize("mode", [0, 1])
+def test_fill_hash_matches_generator(mode):
+    n = 1 << 20
+    t = torch.empty(n, device="cuda")
+    catt.fill_hash(t, 17, offset=(1 << 32) - 1000, mode=mode)
+    want = si.values(17, n, offset=(1 << 32) - 1000, mode=mode)
+    assert bits_equal(host(t), want)
+
+
+# ------------------------------------------------------------------ ATAX / BICG / MVT / GESUMMV
+def _vec_ok(variant, n):
+    return not (variant in ("vec4", "staged") and n % 4)
+
+
+@pytest.mark.parametrize("variant", EXACT)
+@pytest.mark.parametrize("m,n", ROW_SHAPES)
+def test_atax_exact(variant, m, n):
+    A, x = si.matrix(1, m, n), si.values(101, n)
+    tmp_o, y_o = oracle.atax(A, x)
+    t = catt.Throttle(variant=variant)
+    if not _vec_ok(variant, n):
+        with pytest.raises(catt.CattError):
+            catt.atax(dev(A), dev(x), k1=t)
+        return
+    tmp, y = catt.atax(dev(A), dev(x), k1=t, k2=catt.Throttle(variant="literal"))
+    assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y), y_o)
+
+
+@pytest.mark.parametrize("variant", EXACT + ["coop"])
+@pytest.mark.parametrize("m,n", COL_SHAPES)
+def test_bicg(variant, m, n):
+    A, p, r = si.matrix(2, m, n), si.values(102, n), si.values(202, m)
+    q_o, s_o = oracle.bicg(A, p, r)
+    q64, s64 = oracle.bicg(A, p, r, mode=oracle.SEQ_F64)
+    col_var = {"staged": "literal"}.get(variant, variant)     # no staged column loop
+    if not _vec_ok(variant, n):
+        with pytest.raises(catt.CattError):
+            catt.bicg(dev(A), dev(p), dev(r), k1=catt.Throttle(variant=col_var), k2=catt.Throttle(variant=variant))
+        return
+    q, s = catt.bicg(dev(A), dev(p), dev(r), k1=catt.Throttle(variant=col_var), k2=catt.Throttle(variant=variant))
+    q, s = host(q), host(s)
+    if variant == "coop":
+        assert relerr(q, q64) <= TOL and relerr(s, s64) <= TOL
+    else:
+        assert bits_equal(q, q_o) and bits_equal(s, s_o)
+
+
+@pytest.mark.parametrize("variant", EXACT + ["coop"])
+@pytest.mark.parametrize("n", [1, 36, 257, 1024])
+def test_mvt(variant, n):
+    a = si.matrix(3, n, n)
+    y1, y2, x1, x2 = (si.values(103 + 100 * k, n) for k in range(4))
+    o1, o2 = oracle.mvt(a, y1, y2, x1, x2)
+    e1, e2 = oracle.mvt(a, y1, y2, x1, x2, mode=oracle.SEQ_F64)
+    col_var = {"staged": "literal"}.get(variant, variant)
+    X1, X2 = dev(x1), dev(x2)
+    if not _vec_ok(variant, n):
+        with pytest.raises(catt.CattError):
+            catt.mvt(dev(a), dev(y1), dev(y2), X1, X2, k1=catt.Throttle(variant=variant))
+        return
+    catt.mvt(dev(a), dev(y1), dev(y2), X1, X2, k1=catt.Throttle(variant=variant), k2=catt.Throttle(variant=col_var))
+    if variant == "coop":
+        assert relerr(host(X1), e1) <= TOL and relerr(host(X2), e2) <= TOL
+    else:
+        assert bits_equal(host(X1), o1) and bits_equal(host(X2), o2)
+
+
+@pytest.mark.parametrize("variant", EXACT + ["coop"])
+@pytest.mark.parametrize("n", [36, 130, 1024])
+def test_gesummv(variant, n):
+    A, B, x = si.matrix(5, n, n), si.matrix(105, n, n), si.values(205, n)
+    y_o, t_o = oracle.gesummv(A, B, x, 1.5, 1.2)
+    y64, t64 = oracle.gesummv(A, B, x, 1.5, 1.2, mode=oracle.SEQ_F64)
+    if not _vec_ok(variant, n):
+        return
+    y, tmp = catt.gesummv(dev(A), dev(B), dev(x), 1.5, 1.2, t=catt.Throttle(variant=variant))
+    if variant == "coop":
+        assert relerr(host(y), y64) <= TOL and relerr(host(tmp), t64) <= TOL
+    else:
+        assert bits_equal(host(y), y_o) and bits_equal(host(tmp), t_o)
+
+
+@pytest.mark.parametrize("n", [64, 1024])
+def test_coop_bit_exact_on_dyadic_inputs(n):
+    A, p, r = (si.matrix(9, n, n, DYADIC), si.values(19, n, mode=DYADIC), si.values(29, n, mode=DYADIC))
+    q_o, s_o = oracle.bicg(A, p, r)
+    q, s = catt.bicg(dev(A), dev(p), dev(r), k1=catt.Throttle(variant="coop"), k2=catt.Throttle(variant="coop"))
+    assert bits_equal(host(q), q_o) and bits_equal(host(s), s_o)
+
+
+def test_empty_and_degenerate_shapes():
+    # n = 0 columns: tmp is the empty sum 0, y is empty; m = 0 rows: y = 0
+    A = torch.empty((5, 0), device="cuda")
+    tmp, y = catt.atax(A, torch.empty(0, device="cuda"))
+    assert np.all(host(tmp) == 0) and y.numel() == 0
+    A = torch.empty((0, 7), device="cuda")
+    tmp, y = catt.atax(A, torch.ones(7, device="cuda"))
+    assert tmp.numel() == 0 and np.all(host(y) == 0)
+    A = dev(si.matrix(4, 1, 1))
+    tmp, y = catt.atax(A, dev(np.array([2.0], np.float32)))
+    a = float(host(A)[0, 0])
+    assert float(host(tmp)[0]) == np.float32(a * 2) and float(host(y)[0]) == np.float32(np.float32(a * 2) * a)
+
+
+def test_invalid_arguments_raise():
+    A, x = dev(si.matrix(1, 64, 64)), dev(si.values(2, 64))
+    with pytest.raises(catt.CattError):
+        catt.atax(A, x, k1=catt.Throttle(active_warps=9))                   # > warps per CTA
+    with pytest.raises(catt.CattError):
+        catt.atax(A, x, k1=catt.Throttle(carveout_kb=50))                   # not an option
+    with pytest.raises(catt.CattError):
+        catt.atax(A, x, k1=catt.Throttle(cta_threads=100))                  # not a warp multiple
+    with pytest.raises(catt.CattError):
+        catt.atax(A, x, k1=catt.Throttle(variant="staged", active_warps=1, cta_threads=64))
+    with pytest.raises(catt.CattError):
+        catt.atax(A.cpu(), x)                                                 # host tensor
+
+
+# ------------------------------------------------------------------ throttles never change results
+THROTTLES = [
+    catt.Throttle(active_warps=1),
+    catt.Throttle(active_warps=3),
+    catt.Throttle(active_warps=4, gate=catt.GATE_BARRIER),
+    catt.Throttle(active_warps=2, active_ctas=2),
+    catt.Throttle(active_warps=1, active_ctas=1, carveout_kb=228),
+    catt.Throttle(active_ctas=3, cap=catt.CAP_SMEM_PAD, carveout_kb=64),
+    catt.Throttle(cta_threads=1024, active_warps=5, carveout_kb=196),
+    catt.Throttle(cta_threads=64, active_warps=1, variant="vec4"),
+]
+
+
+@pytest.mark.parametrize("t", THROTTLES, ids=repr)
+def test_throttled_results_identical(t):
+    m, n = 3000, 68
+    A, x = si.matrix(1, m, n), si.values(101, n)
+    tmp_o, y_o = oracle.atax(A, x)
+    tmp, y = catt.atax(dev(A), dev(x), k1=t, k2=t.copy(variant=catt.VAR_LITERAL))
+    assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y), y_o)
+
+
+# ------------------------------------------------------------------ SYRK
+@pytest.mark.parametrize("variant", ["literal", "staged"])
+@pytest.mark.parametrize("n,m", [(64, 40), (130, 37), (256, 256)])
+def test_syrk_exact(variant, n, m):
+    A, C = si.matrix(6, n, m), si.matrix(106, n, n)
+    C_o = oracle.syrk(A, C, 1.5, 1.2)
+    Cd = dev(C)
+    catt.syrk(dev(A), Cd, 1.5, 1.2, t=catt.Throttle(variant=variant))
+    assert bits_equal(host(Cd), C_o)
+
+
+def test_syrk_throttled():
+    A, C = si.matrix(6, 96, 64), si.matrix(106, 96, 96)
+    C_o = oracle.syrk(A, C, 1.5, 1.2)
+    for t in (catt.Throttle(active_warps=2), catt.Throttle(active_warps=1, active_ctas=2),
+              catt.Throttle(cta_threads=512, active_warps=4, gate=catt.GATE_BARRIER)):
+        Cd = dev(C)
+        catt.syrk(dev(A), Cd, 1.5, 1.2, t=t)
+        assert bits_equal(host(Cd), C_o)
+
+
+# ------------------------------------------------------------------ KMEANS
+@pytest.mark.parametrize("variant", ["literal", "regs"])
+@pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 3), (4099, 34, 5, 29), (257, 7, 3, 0), (300, 50, 4, 1)])
+def test_kmeans_exact(variant, npts, nf, k, pad):
+    ld = npts + pad
+    feat = si.values(4, nf * ld)
+    clusters = feat.reshape(nf, ld)[:, :k].T.copy()          # centres = first k points
+    memb_o, _ = oracle.kmeans_assign(feat, ld, npts, nf, clusters)
+    for t in (catt.Throttle(variant=variant), catt.Throttle(variant=variant, active_warps=2, active_ctas=3)):
+        memb = catt.kmeans_assign(dev(feat), ld, npts, nf, dev(clusters), t=t)
+        assert np.array_equal(host(memb), memb_o)
+
+
+# ------------------------------------------------------------------ full BASELINE sizes
+def test_bicg_mvt_4096_full():
+    n = 4096
+    A = torch.empty(n * n, device="cuda")
+    catt.fill_hash(A, si.SEED_BICG)
+    Ah = oracle.fill(si.SEED_BICG, n * n).reshape(n, n)
+    p, r = si.values(si.sub_seed(si.SEED_BICG, 1), n), si.values(si.sub_seed(si.SEED_BICG, 2), n)
+    q_o, s_o = oracle.bicg(Ah, p, r)
+    q64, s64 = oracle.bicg(Ah, p, r, mode=oracle.SEQ_F64)
+    A = A.view(n, n)
+    for v in ("literal", "vec4", "staged", "coop"):
+        q, s = catt.bicg(A, dev(p), dev(r), k1=catt.Throttle(variant="coop" if v == "coop" else "literal"),
+                         k2=catt.Throttle(variant=v))
+        q, s = host(q), host(s)
+        if v == "coop":
+            assert relerr(q, q64) <= TOL and relerr(s, s64) <= TOL
+        else:
+            assert bits_equal(q, q_o) and bits_equal(s, s_o)
+
+
+def test_kmeans_rodinia_shape_full():
+    npts, nf, k = 494020, 34, 5
+    for ld in (494020, 494048):
+        feat = torch.empty(nf * ld, device="cuda")
+        catt.fill_hash(feat, si.SEED_KMEANS)
+        fh = oracle.fill(si.SEED_KMEANS, nf * ld)
+        clusters = fh.reshape(nf, ld)[:, :k].T.copy()
+        memb_o, _ = oracle.kmeans_assign(fh, ld, npts, nf, clusters)
+        hw = catt.hw_query()
+        t, r = catt.plan(catt.problem(catt.K_KMEANS, m=npts, n=nf, k=k, ld=ld), catt.Throttle(), hw)
+        for tt in (catt.Throttle(), t, catt.Throttle(variant="regs")):
+            memb = catt.kmeans_assign(feat, ld, npts, nf, dev(clusters), t=tt)
+            assert np.array_equal(host(memb), memb_o)
+
+
+def test_gesummv_8192_full():
+    n = 8192
+    A, B = torch.empty(n * n, device="cuda"), torch.empty(n * n, device="cuda")
+    catt.fill_hash(A, si.SEED_GESUMMV)
+    catt.fill_hash(B, si.sub_seed(si.SEED_GESUMMV, 1))
+    x = si.values(si.sub_seed(si.SEED_GESUMMV, 2), n)
+    Ah = oracle.fill(si.SEED_GESUMMV, n * n).reshape(n, n)
+    Bh = oracle.fill(si.sub_seed(si.SEED_GESUMMV, 1), n * n).reshape(n, n)
+    y_o, t_o = oracle.gesummv(Ah, Bh, x, 1.5, 1.2)
+    y64, _ = oracle.gesummv(Ah, Bh, x, 1.5, 1.2, mode=oracle.SEQ_F64)
+    for v in ("literal", "staged", "coop"):
+        y, tmp = catt.gesummv(A.view(n, n), B.view(n, n), dev(x), 1.5, 1.2, t=catt.Throttle(variant=v))
+        if v == "coop":
+            assert relerr(host(y), y64) <= TOL
+        else:
+            assert bits_equal(host(y), y_o) and bits_equal(host(tmp), t_o)
+
+
+def test_syrk_2048_sampled_rows():
+    n = m = 2048
+    A = torch.empty(n * m, device="cuda")
+    C = torch.empty(n * n, device="cuda")
+    catt.fill_hash(A, si.SEED_SYRK)
+    catt.fill_hash(C, si.sub_seed(si.SEED_SYRK, 1))
+    Ah = oracle.fill(si.SEED_SYRK, n * m).reshape(n, m)
+    Ch = oracle.fill(si.sub_seed(si.SEED_SYRK, 1), n * n).reshape(n, n)
+    rows = np.array([0, 1, 127, 128, 1000, 2047])
+    want = oracle.syrk_rows(Ah, Ch, 1.5, 1.2, rows)
+    for v in ("literal", "staged"):
+        Cd = C.clone().view(n, n)
+        catt.syrk(A.view(n, m), Cd, 1.5, 1.2, t=catt.Throttle(variant=v))
+        assert bits_equal(host(Cd)[rows], want), v
+
+
+def test_atax_65536x16384_sampled():
+    m, n = 65536, 16384
+    A = torch.empty(m * n, device="cuda")
+    catt.fill_hash(A, si.SEED_ATAX_SHARDED)
+    x = si.values(si.sub_seed(si.SEED_ATAX_SHARDED, 1), n)
+    cols = np.array([0, 1, 31, 32, 4097, 16383])
+    tmp_o, y_o = oracle.atax_hashed(si.SEED_ATAX_SHARDED, 0, x, m, n, cols)
+    tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="staged"), k2=catt.Throttle())
+    assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y)[cols], y_o)
+    tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="coop"), k2=catt.Throttle(variant="coop"))
+    t64, y64 = oracle.atax_hashed(si.SEED_ATAX_SHARDED, 0, x, m, n, cols, mode=oracle.SEQ_F64)
+    assert relerr(host(tmp), t64) <= TOL and relerr(host(y)[cols], y64) <= TOL
+
+
+# ------------------------------------------------------------------ throttle enforcement (residency probe)
+def _concurrency(rec, W):
+    """rec: [ncta*W, 3] (smid, t0, t1). Max warps of one CTA inside the loop at
+    once, and max CTAs of one SM with a warp inside the loop at once."""
+    rec = rec.reshape(-1, W, 3)
+    valid = rec[:, :, 2] > 0
+    max_w = 0
+    for c in range(rec.shape[0]):
+        ev = sorted([(rec[c, w, 1], 1) for w in range(W) if valid[c, w]] +
+                    [(rec[c, w, 2], -1) for w in range(W) if valid[c, w]], key=lambda e: (e[0], e[1]))
+        cur = 0
+        for _, d in ev:
+            cur += d
+            max_w = max(max_w, cur)
+    cta_iv = {}
+    for c in range(rec.shape[0]):
+        if not valid[c].any():
+            continue
+        sm = int(rec[c, valid[c], 0][0])
+        cta_iv.setdefault(sm, []).append((rec[c, valid[c], 1].min(), rec[c, valid[c], 2].max()))
+    max_c = 0
+    for sm, ivs in cta_iv.items():
+        ev = sorted([(a, 1) for a, b in ivs] + [(b, -1) for a, b in ivs], key=lambda e: (e[0], e[1]))
+        cur = 0
+        for _, d in ev:
+            cur += d
+            max_c = max(max_c, cur)
+    return max_w, max_c
+
+
+@pytest.mark.parametrize("t,want", [
+    (catt.Throttle(), (8, 8)),
+    (catt.Throttle(active_warps=2), (2, 8)),
+    (catt.Throttle(active_warps=4, gate=catt.GATE_BARRIER), (4, 8)),
+    (catt.Throttle(active_warps=1, active_ctas=3), (1, 3)),
+    (catt.Throttle(active_ctas=2, cap=catt.CAP_SMEM_PAD, carveout_kb=64), (8, 2)),
+], ids=repr)
+def test_residency_probe_enforces_throttle(t, want):
+    # long rows so CTAs overlap in time; 148 SMs x 8 CTAs x 256 rows x 2 waves
+    m, n = 148 * 8 * 256 * 2, 512
+    A = torch.empty(m * n, device="cuda")
+    catt.fill_hash(A, 1)
+    x = torch.ones(n, device="cuda")
+    ncta = m // 256
+    probe = torch.zeros(ncta * 8 * 3, dtype=torch.int64, device="cuda")
+    tt = t.copy(probe=probe.data_ptr())
+    catt.atax(A.view(m, n), x, k1=tt)
+    mw, mc = _concurrency(host(probe).astype(np.int64), 8)
+    assert mw <= want[0] and mc <= want[1]
+    assert mw == want[0]                                   # the slots are actually used
+    assert mc >= min(want[1], 2)
+
+
+def test_plan_on_device_matches_occupancy_api():
+    hw = catt.hw_query()
+    assert hw.num_sms == 148
+    for prob, launch in [(catt.problem(catt.K_ATAX_1, m=1 << 20, n=256), catt.Throttle()),
+                         (catt.problem(catt.K_KMEANS, m=494020, n=34, k=5, ld=494020), catt.Throttle()),
+                         (catt.problem(catt.K_SYRK, n=2048, k=2048), catt.Throttle())]:
+        d, keep = catt.kernel_desc(prob, launch)
+        regs, smem = catt.kernel_attrs(prob, launch)
+        assert d.regs_per_thread == regs and regs <= 32      # full TLP is not register-limited
+        t, r = catt.plan(prob, launch, hw)
+        assert r["base_ctas"] == 8

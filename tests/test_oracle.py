@@ -160,6 +160,13 @@ def test_syrk_vs_numpy_and_symmetry():
     assert np.array_equal(b, (C * np.float32(1.2)).astype(np.float32))
 
 
+def test_syrk_rows_equals_full_rows():
+    A, C = si.matrix(6, 50, 33), si.matrix(106, 50, 50)
+    full = oracle.syrk(A, C, 1.5, 1.2)
+    rows = np.array([0, 7, 49])
+    assert np.array_equal(oracle.syrk_rows(A, C, 1.5, 1.2, rows), full[rows])
+
+
 def test_kmeans_vs_bruteforce_argmin():
     npts, nf, k = 1000, 34, 5
     ld = npts + 3                                         # misaligned leading dimension
