@@ -258,6 +258,25 @@ catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alph
 catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters,
                                int32_t k, int32_t* membership, const catt_throttle* t, void* stream);
 
+/* ------------------------------------------------------------------ single loops
+ * CATT throttles per loop: these run one loop each and
+ * are what the application entry points above are made of.
+ *
+ * Row loop (ATAX#1, BICG#2, MVT#1, GESUMMV; memory-divergent): for i < m,
+ *   mode CATT_ROWS_STORE:   y[i] = sum_j A[i*n + j] * x[j]
+ *   mode CATT_ROWS_ACCUM:   y[i] = y[i] + sum_j A[i*n + j] * x[j]   (y in/out)
+ *   mode CATT_ROWS_GESUMMV: tmp[i] = sum_j A[i*n+j] x[j];
+ *                           y[i] = alpha*tmp[i] + beta*sum_j B[i*n+j] x[j]
+ * B and tmp are used only by CATT_ROWS_GESUMMV (else may be NULL).
+ * Column loop (ATAX#2, BICG#1, MVT#2; coalesced): for j < n,
+ *   y[j] = (accumulate ? y[j] : 0) + sum_i A[i*n + j] * v[i].
+ * A is m x n row-major in both. */
+enum { CATT_ROWS_STORE = 0, CATT_ROWS_ACCUM = 1, CATT_ROWS_GESUMMV = 2 };
+catt_status catt_rows(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t m, int64_t n,
+                      float alpha, float beta, int32_t mode, const catt_throttle* t, void* stream);
+catt_status catt_cols(const float* A, const float* v, float* y, int64_t m, int64_t n, int32_t accumulate,
+                      const catt_throttle* t, void* stream);
+
 /* ------------------------------------------------------------------ helpers */
 /* dst[i] = value(seed, offset + i): the counter-based generator of
  * seeded_inputs.py (mode 0 uniform [0,1), 1 dyadic k/16). Device pointer. */

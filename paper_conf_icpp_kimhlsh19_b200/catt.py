@@ -24,6 +24,7 @@ REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
 MODE_UNION, MODE_PAPER = 0, 1
 FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE = 1, 2, 4, 8
 VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS = 0, 1, 2, 3, 4
+ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
 (K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS) = range(9)
@@ -150,6 +151,8 @@ def lib():
             "catt_gesummv": [V, V, V, V, V, i64, f32, f32, T, V],
             "catt_syrk": [V, V, i64, i64, f32, f32, T, V],
             "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
+            "catt_rows": [V, V, V, V, V, i64, i64, f32, f32, i32, T, V],
+            "catt_cols": [V, V, V, i64, i64, i32, T, V],
             "catt_fill_hash": [V, i64, u32, u64, i32, V],
             "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
             "catt_kernel_attrs": [P(Problem), T, P(i32), P(i32)],
@@ -168,7 +171,7 @@ def lib():
 
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_kmeans_assign",
-            "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
+            "catt_rows", "catt_cols", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version"]
 
 
@@ -326,6 +329,23 @@ def gesummv(A, B, x, alpha, beta, y=None, tmp=None, t: Optional[Throttle] = None
     _check(lib().catt_gesummv(_dev(A, "A"), _dev(B, "B"), _dev(x, "x"), _dev(y, "y"), _dev(tmp, "tmp"), n,
                               float(alpha), float(beta), _tp(t), _stream()), "catt_gesummv")
     return y, tmp
+
+
+def rows(A, x, y, mode=ROWS_STORE, B=None, tmp=None, alpha=0.0, beta=0.0, t: Optional[Throttle] = None):
+    """One row loop (catt_rows): y = A x (STORE), y += A x (ACCUM), or GESUMMV."""
+    m, n = A.shape
+    _check(lib().catt_rows(_dev(A, "A"), _dev(B, "B") if B is not None else None, _dev(x, "x"), _dev(y, "y"),
+                           _dev(tmp, "tmp") if tmp is not None else None, m, n, float(alpha), float(beta), mode,
+                           _tp(t), _stream()), "catt_rows")
+    return y
+
+
+def cols(A, v, y, accumulate=False, t: Optional[Throttle] = None):
+    """One column loop (catt_cols): y (+)= A^T v."""
+    m, n = A.shape
+    _check(lib().catt_cols(_dev(A, "A"), _dev(v, "v"), _dev(y, "y"), m, n, int(bool(accumulate)), _tp(t),
+                           _stream()), "catt_cols")
+    return y
 
 
 def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):

@@ -573,3 +573,18 @@ extern "C" catt_status catt_gesummv(const float* A, const float* B, const float*
   if (check_common(n, n) != CATT_OK || (n > 0 && (!A || !B || !x || !y || !tmp))) return CATT_EINVAL;
   return launch_row(A, B, x, y, tmp, n, n, alpha, beta, EPI_GESUMMV, t, static_cast<cudaStream_t>(stream));
 }
+
+extern "C" catt_status catt_rows(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t m,
+                                 int64_t n, float alpha, float beta, int32_t mode, const catt_throttle* t,
+                                 void* stream) {
+  if (check_common(m, n) != CATT_OK || mode < CATT_ROWS_STORE || mode > CATT_ROWS_GESUMMV) return CATT_EINVAL;
+  if ((m * n > 0 && !A) || (n > 0 && !x) || (m > 0 && !y)) return CATT_EINVAL;
+  if (mode == CATT_ROWS_GESUMMV && ((m * n > 0 && !B) || (m > 0 && !tmp))) return CATT_EINVAL;
+  return launch_row(A, B, x, y, tmp, m, n, alpha, beta, mode, t, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" catt_status catt_cols(const float* A, const float* v, float* y, int64_t m, int64_t n, int32_t accumulate,
+                                 const catt_throttle* t, void* stream) {
+  if (check_common(m, n) != CATT_OK || (m * n > 0 && !A) || (m > 0 && !v) || (n > 0 && !y)) return CATT_EINVAL;
+  return launch_col(A, v, y, m, n, accumulate ? EPI_ACCUM : EPI_STORE, t, static_cast<cudaStream_t>(stream));
+}
