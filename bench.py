@@ -199,8 +199,9 @@ class BicgMvt(Workload):
             Loop("mvt2 x2+=A^T y2", lambda: catt.cols(self.Am, self.y2, self.x2, acc2, tm2),
                  mat + 4 * (rows + (2 if acc2 else 1) * n), "cols"),
         ]
-        self.study = dict(prob=P(catt.K_BICG_2, m=rows, n=n), A=self.Ab, x=self.p, y=self.q,
-                          launches=[(1024, 196), (256, 228)])
+        self.study = dict(name="bicg2 q=A p (literal, row per thread)", prob=P(catt.K_BICG_2, m=rows, n=n),
+                          A=self.Ab, x=self.p, y=self.q,
+                          launches=[(1024, 132), (1024, 196), (1024, 228), (256, 196), (256, 228)])
 
     def collective(self):
         if self.world > 1:
@@ -242,7 +243,8 @@ class Kmeans(Workload):
         nbytes = self.np_ * self.nf * 4 + self.np_ * 4 + self.k * self.nf * 4
         self.loops = [Loop("kmeans assign", lambda: catt.kmeans_assign(self.feat, self.ld, self.np_, self.nf,
                                                                          self.clusters, self.memb, t=t), nbytes, "kmeans")]
-        self.study = dict(prob=prob, kmeans=True, launches=[(256, 0), (256, 100), (256, 228)])
+        self.study = dict(name="kmeans assign (literal, feature-major)", prob=prob, kmeans=True,
+                          launches=[(256, 0), (256, 100), (256, 228)])
 
     def inputs(self):
         return [self.feat]
@@ -276,7 +278,8 @@ class Gesummv(Workload):
                       catt.Throttle(cta_threads=256 if self.variant == "coop" else 64, variant=self.variant))
         self.loops = [Loop("gesummv", lambda: catt.rows(self.A, self.x, self.y, catt.ROWS_GESUMMV, self.B, self.tmp,
                                                          1.5, 1.2, t), 2 * n * n * 4 + 12 * n, "rows")]
-        self.study = dict(prob=catt.problem(catt.K_GESUMMV, n=n), gesummv=True, launches=[(1024, 196), (256, 196)])
+        self.study = dict(name="gesummv (literal, row per thread)", prob=catt.problem(catt.K_GESUMMV, n=n),
+                          gesummv=True, launches=[(1024, 0), (1024, 196), (256, 196), (256, 228)])
 
     def inputs(self):
         return [self.A, self.B, self.x]
@@ -350,8 +353,8 @@ class Atax(Workload):
                            mat + 4 * (rows + n), "rows"),
                       Loop("atax2 y=A^T tmp", lambda: catt.cols(self.A, self.tmp, self.y, False, t2),
                            mat + 4 * (rows + n), "cols")]
-        self.study = dict(prob=catt.problem(catt.K_ATAX_1, m=rows, n=n), A=self.A, x=self.x, y=self.tmp,
-                          launches=[(1024, 196), (256, 228)])
+        self.study = dict(name="atax1 tmp=A x (literal, row per thread)", prob=catt.problem(catt.K_ATAX_1, m=rows, n=n),
+                          A=self.A, x=self.x, y=self.tmp, launches=[(1024, 196), (256, 228)])
 
     def collective(self):
         if self.world > 1:
@@ -442,9 +445,11 @@ def throttle_study(catt, torch, w, flush):
 
     out = []
     S = w.study
+    paper_hw = catt.paper_rule(hw)
     for cta, carve in S["launches"]:
         launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
-        t, r = catt.plan(S["prob"], launch, hw)
+        t, r = catt.plan(S["prob"], launch, hw)               # B200 rule (guards on)
+        tp, rp = catt.plan(S["prob"], launch, paper_hw)       # the paper's Eq 9 rule
         W, T = r["base_warps"], r["base_ctas"]
         cands = []
         for a in [d for d in range(W, 0, -1) if W % d == 0]:
@@ -461,13 +466,18 @@ def throttle_study(catt, torch, w, flush):
                 fn = lambda th=th: catt.rows(S["A"], S["x"], S["y"], catt.ROWS_STORE, t=th)
             times[(a, m)] = med(fn)
         pick = (t.active_warps or W, t.active_ctas or T)
+        pick_p = (tp.active_warps or W, tp.active_ctas or T)
         best = min(times, key=times.get)
-        out.append(dict(loop=f"{S['prob'].loop} literal", cta_threads=cta, carveout_kb=r["carveout_kb"],
-                        base=[W, T], footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
-                        contended=r["flags"] != catt.FIT_NONE_NEEDED, catt=list(pick),
-                        catt_ms=round(times[pick], 4), full_ms=round(times[(W, T)], 4), best=list(best),
-                        best_ms=round(times[best], 4), catt_over_best=round(times[pick] / times[best], 3),
+        out.append(dict(loop=S["name"], cta_threads=cta, carveout_kb=r["carveout_kb"], base=[W, T],
+                        footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
+                        contended=rp["flags"] != catt.FIT_NONE_NEEDED,
+                        catt=list(pick), catt_rule=catt.FLAG_NAMES.get(r["flags"], r["flags"]),
+                        catt_ms=round(times[pick], 4),
+                        catt_paper=list(pick_p), catt_paper_ms=round(times[pick_p], 4),
+                        full_ms=round(times[(W, T)], 4), best=list(best), best_ms=round(times[best], 4),
+                        catt_over_best=round(times[pick] / times[best], 3),
                         catt_over_full=round(times[pick] / times[(W, T)], 3),
+                        paper_over_best=round(times[pick_p] / times[best], 3),
                         swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()}))
     return out
 

@@ -71,7 +71,8 @@ enum {
   CATT_FIT_NONE_NEEDED = 1, /* fits at full TLP, or the loop has no locality */
   CATT_FIT_WARP = 2,        /* warp-level throttle (N of Eq 9)                         */
   CATT_FIT_CTA = 4,         /* TB-level throttle (M of Eq 9), one warp per CTA          */
-  CATT_FIT_UNRESOLVABLE = 8 /* nothing fits even at (1,1): left unthrottled    */
+  CATT_FIT_UNRESOLVABLE = 8, /* nothing fits even at (1,1): left unthrottled    */
+  CATT_FIT_GUARDED = 16      /* a B200 guard (divergence / TLP floor) limited the throttle */
 };
 
 /* One memory instruction in the loop (Eq 5):
@@ -114,10 +115,15 @@ typedef struct {
 /* Hardware parameters. carveout_kb[i] are the configurable shared-memory
  * sizes per SM (ascending); l1d_bytes[i] the L1D capacity that option leaves
  * (measured on B200, see catt_hw_b200); carveout_pct[i] the
- * cudaFuncAttributePreferredSharedMemoryCarveout value that selects it. */
+ * cudaFuncAttributePreferredSharedMemoryCarveout value that selects it.
+ * min_warps_sm / divergent_lines are the B200 guards of union mode (0 = off;
+ * DESIGN.md reading R18): a loop is throttled only if one of its reused
+ * references touches >= divergent_lines lines per warp request, and never to
+ * fewer than min_warps_sm active warps per SM. Paper mode ignores them. */
 typedef struct {
   int32_t num_sms, max_warps_sm, max_ctas_sm, regs_sm, reg_alloc_unit, warp_size;
   int32_t smem_alloc_unit, reserved_smem_cta, line_bytes, n_carveouts;
+  int32_t min_warps_sm, divergent_lines;
   int32_t carveout_kb[CATT_MAX_CARVEOUTS];
   int32_t carveout_pct[CATT_MAX_CARVEOUTS];
   int64_t l1d_bytes[CATT_MAX_CARVEOUTS];

@@ -24,6 +24,11 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
   a5  Eq 9 (order P:357 + P:371): N over the divisors of
       #Warps_TB (ascending, R6) first; then TB-level, M = 1 .. #TB_SM-1 with
       one warp per TB (R7); give up (CORR) if nothing fits.
+      B200 guards (union mode only, R18; hw keys min_warps_sm and
+      divergent_lines, 0 = off): no throttle unless a reused reference touches
+      at least divergent_lines lines per warp request (the memory divergence
+      of P:32); no candidate below min_warps_sm active warps per SM, and if
+      none at or above it fits, the most throttled one that respects it.
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -46,6 +51,7 @@ FIT_NONE_NEEDED = 1
 FIT_WARP = 2
 FIT_CTA = 4
 FIT_UNRESOLVABLE = 8
+FIT_GUARDED = 16
 
 MAX_LOOPS = 4
 MAX_WINDOW = 1 << 20
@@ -238,6 +244,7 @@ class Model:
         self.W, self.T, self.carveout_kb, self.l1d_bytes = occupancy(loop, hw)
         self.line = hw["line_bytes"]
         self.paper = loop.mode == MODE_PAPER
+        self.divergent = True
         # contention is measured only "for loops where cache locality presents"
         self.locality = any(has_locality(r, loop.trips, self.line) for r in loop.refs
                             if not (r.flags & REF_NOT_L1))
@@ -260,7 +267,11 @@ class Model:
             self._R = {}
             gids00 = _lane_gids(loop, 0, 0, hw["warp_size"])
             it0 = [(0,) * len(loop.trips)]
-            self.lines_per_warp_iter = sum(len(_lines(r, gids00, it0, self.line)) for r in self.refs)
+            per_ref = [len(_lines(r, gids00, it0, self.line)) for r in self.refs]
+            self.lines_per_warp_iter = sum(per_ref)
+            div = hw.get("divergent_lines", 0)
+            self.divergent = div <= 0 or any(
+                n >= div for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line))
             self.reuse_span = len(self.retained(0, 0, 0))
 
     def retained(self, b: int, w: int, k: int):
@@ -311,15 +322,33 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
 
     if M.fits(full) or not M.locality:
         return done(W, T, full, FIT_NONE_NEEDED)
+    floor_w = 0 if M.paper else hw.get("min_warps_sm", 0)
+    if not M.paper and not M.divergent:
+        return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
+    last = None
+    stopped = False
     for N in range(2, W + 1):                     # Eq 9, warp level first
         if W % N:
             continue
         a = W // N
+        if a * T < floor_w:
+            stopped = True
+            break
         f = M.F(a, T)
         if M.fits(f):
             return done(a, T, f, FIT_WARP)
-    for m in range(T - 1, 0, -1):                 # then TB level with one warp per TB
-        f = M.F(1, m)
-        if M.fits(f):
-            return done(1, m, f, FIT_CTA)
+        last = (a, T, FIT_WARP)
+    if not stopped:
+        for m in range(T - 1, 0, -1):             # then TB level with one warp per TB
+            if m < floor_w:
+                break
+            f = M.F(1, m)
+            if M.fits(f):
+                return done(1, m, f, FIT_CTA)
+            last = (1, m, FIT_CTA)
+    if floor_w > 0:
+        if last is None:
+            return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
+        a, m, fl = last
+        return done(a, m, M.F(a, m), fl | FIT_GUARDED)
     return done(W, T, full, FIT_UNRESOLVABLE)     # P:244, P:395 (CORR): leave as is

@@ -22,7 +22,7 @@ OK, EINVAL, ECUDA, EUNSUPPORTED, ENOMEM, ENODEV = 0, -1, -2, -3, -4, -5
 MAX_LOOPS, MAX_CARVEOUTS = 4, 16
 REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
 MODE_UNION, MODE_PAPER = 0, 1
-FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE = 1, 2, 4, 8
+FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE, FIT_GUARDED = 1, 2, 4, 8, 16
 VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS = 0, 1, 2, 3, 4
 ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
@@ -30,7 +30,9 @@ CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
 (K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS) = range(9)
 
 VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS}
-FLAG_NAMES = {FIT_NONE_NEEDED: "none", FIT_WARP: "warp", FIT_CTA: "cta", FIT_UNRESOLVABLE: "unresolvable"}
+FLAG_NAMES = {FIT_NONE_NEEDED: "none", FIT_WARP: "warp", FIT_CTA: "cta", FIT_UNRESOLVABLE: "unresolvable",
+              FIT_NONE_NEEDED | FIT_GUARDED: "none(guard)", FIT_WARP | FIT_GUARDED: "warp(guard)",
+              FIT_CTA | FIT_GUARDED: "cta(guard)"}
 
 
 class CattError(RuntimeError):
@@ -56,12 +58,13 @@ class Hw(ctypes.Structure):
                 ("regs_sm", ctypes.c_int32), ("reg_alloc_unit", ctypes.c_int32), ("warp_size", ctypes.c_int32),
                 ("smem_alloc_unit", ctypes.c_int32), ("reserved_smem_cta", ctypes.c_int32),
                 ("line_bytes", ctypes.c_int32), ("n_carveouts", ctypes.c_int32),
+                ("min_warps_sm", ctypes.c_int32), ("divergent_lines", ctypes.c_int32),
                 ("carveout_kb", ctypes.c_int32 * MAX_CARVEOUTS), ("carveout_pct", ctypes.c_int32 * MAX_CARVEOUTS),
                 ("l1d_bytes", ctypes.c_int64 * MAX_CARVEOUTS)]
 
     def as_dict(self):
         n = self.n_carveouts
-        d = {f: getattr(self, f) for f, _ in self._fields_[:10]}
+        d = {f: getattr(self, f) for f, _ in self._fields_[:12]}
         d["carveout_kb"] = list(self.carveout_kb[:n])
         d["carveout_pct"] = list(self.carveout_pct[:n])
         d["l1d_bytes"] = list(self.l1d_bytes[:n])
@@ -70,7 +73,7 @@ class Hw(ctypes.Structure):
     @classmethod
     def from_dict(cls, d):
         h = cls()
-        for f, _ in cls._fields_[:10]:
+        for f, _ in cls._fields_[:12]:
             if f in d:
                 setattr(h, f, d[f])
         n = len(d["carveout_kb"])
@@ -187,6 +190,14 @@ def _check(st: int, what: str):
 def hw_b200() -> Hw:
     h = Hw()
     _check(lib().catt_hw_b200(ctypes.byref(h)), "catt_hw_b200")
+    return h
+
+
+def paper_rule(hw: Hw) -> Hw:
+    """A copy of hw with the B200 guards off: the paper's Eq 9 rule as printed."""
+    h = Hw.from_dict(hw.as_dict())
+    h.min_warps_sm = 0
+    h.divergent_lines = 0
     return h
 
 

@@ -220,10 +220,15 @@ class Model {
     const std::vector<G3> g00 = lane_gids(d_, 0, 0, hw_.warp_size);
     const std::vector<int64_t> it0(d_.n_loops, 0);
     lines_per_warp_iter_ = 0;
+    divergent_ = hw_.divergent_lines <= 0;
     for (const catt_ref& r : refs_) {
       std::unordered_set<uint64_t> s;
       add_lines(r, g00, it0, d_.n_loops, line_, &s);
       lines_per_warp_iter_ += int64_t(s.size());
+      bool reuse = false;
+      for (int k = 0; k < d_.n_loops; ++k)
+        if (iabs(r.c_iter[k]) * r.elem_bytes < line_ && d_.trip[k] >= 2) reuse = true;
+      if (reuse && int64_t(s.size()) >= hw_.divergent_lines) divergent_ = true;
     }
     reuse_span_ = int64_t(retained(0, 0, 0).size());
     return CATT_OK;
@@ -275,6 +280,7 @@ class Model {
   bool fits(int64_t lines) const { return lines * line_ <= o_.l1d; }
 
   bool locality_ = false;
+  bool divergent_ = true;  // some reused reference is memory-divergent (B200 guard)
   int64_t lines_per_warp_iter_ = 0, reuse_span_ = 0;
 
  private:
@@ -312,6 +318,7 @@ catt_status validate(const catt_loop_desc* d, const catt_hw* hw) {
   if (hw->warp_size != 32 || hw->num_sms < 1 || hw->max_warps_sm < 1 || hw->max_ctas_sm < 1) return CATT_EINVAL;
   if (hw->line_bytes < 4 || hw->n_carveouts < 1 || hw->n_carveouts > CATT_MAX_CARVEOUTS) return CATT_EINVAL;
   if (hw->smem_alloc_unit < 1 || hw->reg_alloc_unit < 1 || hw->regs_sm < 1) return CATT_EINVAL;
+  if (hw->min_warps_sm < 0 || hw->divergent_lines < 0) return CATT_EINVAL;
   for (int i = 1; i < hw->n_carveouts; ++i)
     if (hw->carveout_kb[i] <= hw->carveout_kb[i - 1]) return CATT_EINVAL;
   return CATT_OK;
@@ -350,14 +357,33 @@ extern "C" catt_status catt_footprint(const catt_loop_desc* desc, const catt_hw*
     return CATT_OK;
   };
   if (M.fits(full) || !M.locality_) return done(W, T, full, CATT_FIT_NONE_NEEDED);
-  for (int32_t N = 2; N <= W; ++N) {                     // Eq 9: warp level first
+  const bool paper = desc->mode == CATT_MODE_PAPER;
+  const int32_t floor_w = paper ? 0 : std::max(0, hw->min_warps_sm);
+  if (!paper && !M.divergent_) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
+  int32_t la = -1, lm = -1, lflag = 0;                  // most throttled candidate above the floor
+  bool stopped = false;
+  for (int32_t N = 2; N <= W && !stopped; ++N) {        // Eq 9: warp level first
     if (W % N) continue;
+    if ((W / N) * T < floor_w) {
+      stopped = true;
+      break;
+    }
     const int64_t f = M.F(W / N, T);
     if (M.fits(f)) return done(W / N, T, f, CATT_FIT_WARP);
+    la = W / N, lm = T, lflag = CATT_FIT_WARP;
   }
-  for (int32_t m = T - 1; m >= 1; --m) {                 // then TB level, one warp per TB
+  for (int32_t m = T - 1; m >= 1 && !stopped; --m) {    // then TB level, one warp per TB
+    if (m < floor_w) {
+      stopped = true;
+      break;
+    }
     const int64_t f = M.F(1, m);
     if (M.fits(f)) return done(1, m, f, CATT_FIT_CTA);
+    la = 1, lm = m, lflag = CATT_FIT_CTA;
+  }
+  if (floor_w > 0) {
+    if (la < 0) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
+    return done(la, lm, M.F(la, lm), lflag | CATT_FIT_GUARDED);
   }
   return done(W, T, full, CATT_FIT_UNRESOLVABLE);
 }
@@ -396,6 +422,11 @@ extern "C" catt_status catt_hw_b200(catt_hw* out) {
   out->smem_alloc_unit = 128;
   out->reserved_smem_cta = 1024;   // cudaDevAttrReservedSharedMemoryPerBlock
   out->line_bytes = 128;
+  // B200 guards (reading R18, profiles/round1_ncu_cases_a_raw.csv): 4 warps per
+  // SM sub-partition to hide L2 latency; a request must touch >= 8 lines for
+  // its misses to cost more than the TLP a throttle gives up.
+  out->min_warps_sm = 16;
+  out->divergent_lines = 8;
   // Shared-memory options (KB) and the carveout percentage that selects each
   // (percent of the 228 KB maximum; the driver rounds up to the next option).
   // L1D capacity per option, measured on B200 by the Fig 3-style sweep

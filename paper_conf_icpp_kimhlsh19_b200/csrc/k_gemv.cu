@@ -15,6 +15,8 @@
 #include <algorithm>
 #include <cstdint>
 
+#include <cooperative_groups.h>
+
 #include "internal.h"
 
 namespace catt {
@@ -115,48 +117,54 @@ __global__ void __launch_bounds__(1024, (NMAT == 2 && VEC) ? 1 : 2) row_thread_k
   cta_exit(a.t);
 }
 
-// ---------------------------------------------------------------- row, warp per row (COOP)
-template <int NMAT, int EPI, bool VEC>
-__global__ void __launch_bounds__(1024) row_warp_kernel(RowArgs a) {
+// ---------------------------------------------------------------- row, warps per row (COOP)
+// S warps share a row (S = 1, 2, 4, 8; 8 warps per CTA, 8/S rows per CTA):
+// warp part p reads 16-byte chunks p*32 + lane + 32*S*t of the row, U chunks
+// in flight per lane; lane partial sums are added by a fixed xor tree, the S
+// warp partials in warp order (deterministic).
+template <int NMAT, int EPI, bool VEC, int S>
+__global__ void __launch_bounds__(256, VEC ? 2 : 3) row_warp_kernel(RowArgs a) {
+  constexpr int U = NMAT == 2 ? 4 : 8;
   __shared__ int slots;
+  __shared__ float red[2][8];
   gate_init(&slots, a.t);
   __syncthreads();
   cta_enter(a.t);
-  const int lane = threadIdx.x & 31;
-  const int64_t i = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, part = warp % S;
+  const int64_t i = int64_t(blockIdx.x) * (8 / S) + warp / S;
+  float acc = 0.0f, acc2 = 0.0f;
   throttled(a.t, &slots, [&]() {
     if (i >= a.M) return;  // warp-uniform
     const int64_t N = a.N;
-    float acc = 0.0f, acc2 = 0.0f;
     if (VEC) {
       const float4* ar = reinterpret_cast<const float4*>(a.A + i * N);
       const float4* br = reinterpret_cast<const float4*>(NMAT == 2 ? a.B + i * N : a.A);
       const float4* x4 = reinterpret_cast<const float4*>(a.x);
-      const int64_t n4 = N >> 2;
-      int64_t j = lane;
-      for (; j + 96 < n4; j += 128) {
-        float4 v[4], w[4], xv[4];
+      const int64_t n4 = N >> 2, step = 32 * S;
+      int64_t j = part * 32 + lane;
+      for (; j + (U - 1) * step < n4; j += U * step) {
+        float4 v[U], w[NMAT == 2 ? U : 1];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          v[u] = ld_na4(ar + j + 32 * u);
-          if (NMAT == 2) w[u] = ld_na4(br + j + 32 * u);
-          xv[u] = x4[j + 32 * u];
+        for (int u = 0; u < U; ++u) {
+          v[u] = ld_na4(ar + j + u * step);
+          if (NMAT == 2) w[u] = ld_na4(br + j + u * step);
         }
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          acc = fmaf(v[u].x, xv[u].x, acc);
-          acc = fmaf(v[u].y, xv[u].y, acc);
-          acc = fmaf(v[u].z, xv[u].z, acc);
-          acc = fmaf(v[u].w, xv[u].w, acc);
+        for (int u = 0; u < U; ++u) {
+          const float4 xv = x4[j + u * step];
+          acc = fmaf(v[u].x, xv.x, acc);
+          acc = fmaf(v[u].y, xv.y, acc);
+          acc = fmaf(v[u].z, xv.z, acc);
+          acc = fmaf(v[u].w, xv.w, acc);
           if (NMAT == 2) {
-            acc2 = fmaf(w[u].x, xv[u].x, acc2);
-            acc2 = fmaf(w[u].y, xv[u].y, acc2);
-            acc2 = fmaf(w[u].z, xv[u].z, acc2);
-            acc2 = fmaf(w[u].w, xv[u].w, acc2);
+            acc2 = fmaf(w[u].x, xv.x, acc2);
+            acc2 = fmaf(w[u].y, xv.y, acc2);
+            acc2 = fmaf(w[u].z, xv.z, acc2);
+            acc2 = fmaf(w[u].w, xv.w, acc2);
           }
         }
       }
-      for (; j < n4; j += 32) {
+      for (; j < n4; j += step) {
         const float4 v = ld_na4(ar + j), xv = x4[j];
         acc = fmaf(v.x, xv.x, acc);
         acc = fmaf(v.y, xv.y, acc);
@@ -174,7 +182,7 @@ __global__ void __launch_bounds__(1024) row_warp_kernel(RowArgs a) {
       const float* ar = a.A + i * N;
       const float* br = NMAT == 2 ? a.B + i * N : a.A;
 #pragma unroll 4
-      for (int64_t j = lane; j < N; j += 32) {
+      for (int64_t j = part * 32 + lane; j < N; j += 32 * S) {
         const float xv = a.x[j];
         acc = fmaf(ld_na(ar + j), xv, acc);
         if (NMAT == 2) acc2 = fmaf(ld_na(br + j), xv, acc2);
@@ -185,118 +193,22 @@ __global__ void __launch_bounds__(1024) row_warp_kernel(RowArgs a) {
       acc += __shfl_xor_sync(0xffffffffu, acc, o);
       if (NMAT == 2) acc2 += __shfl_xor_sync(0xffffffffu, acc2, o);
     }
-    if (lane == 0) {
-      if (EPI == EPI_ACCUM) acc = a.y[i] + acc;
-      row_epilogue<NMAT, EPI>(a, i, acc, acc2);
-    }
   });
-  cta_exit(a.t);
-}
-
-// ---------------------------------------------------------------- row, staged (cp.async.bulk + mbarrier)
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "LAB_WAIT:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@P1 bra DONE;\n"
-      "bra LAB_WAIT;\n"
-      "DONE:\n"
-      "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(dst)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar))
-      : "memory");
-}
-
-constexpr int kStageKT = 128;               // columns per stage (512 B per row segment)
-constexpr int kStagePitch = kStageKT + 4;   // +16 B per row: conflict-free float4 column reads
-
-// One thread per row; each thread copies its own row segment of every stage
-// into shared memory (one bulk copy per stage) and consumes it in order, so
-// the per-row order of operations is the literal loop's.
-template <int NMAT, int EPI>
-__global__ void __launch_bounds__(256) row_staged_kernel(RowArgs a, int stages) {
-  extern __shared__ __align__(128) unsigned char dyn[];
-  uint64_t* bar = reinterpret_cast<uint64_t*>(dyn);
-  float* tiles = reinterpret_cast<float*>(dyn + 128);
-  const int R = blockDim.x;
-  const int t = threadIdx.x;
-  const int64_t row0 = int64_t(blockIdx.x) * R;
-  const int64_t i = row0 + t;
-  const int64_t N = a.N;
-  const int nvalid = int(imin64(R, a.M - row0));
-  const int64_t ntiles = (N + kStageKT - 1) / kStageKT;
-  const int64_t stage_floats = int64_t(NMAT) * R * kStagePitch;
-
-  if (t == 0) {
-    for (int s = 0; s < stages; ++s) mbar_init(&bar[s], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  cta_enter(a.t);
-  if (i < a.M) {
-    auto issue = [&](int64_t c) {
-      const int s = int(c % stages);
-      const int64_t j0 = c * kStageKT;
-      const int len = int(imin64(kStageKT, N - j0));
-      const uint32_t bytes = uint32_t(len) * 4u;
-      if (t == 0) mbar_arrive_expect_tx(&bar[s], bytes * uint32_t(nvalid) * NMAT);
-      float* dst = tiles + s * stage_floats + int64_t(t) * kStagePitch;
-      bulk_g2s(dst, a.A + i * N + j0, bytes, &bar[s]);
-      if (NMAT == 2) bulk_g2s(dst + int64_t(R) * kStagePitch, a.B + i * N + j0, bytes, &bar[s]);
-    };
-    const int64_t pro = imin64(stages, ntiles);
-    for (int64_t c = 0; c < pro; ++c) issue(c);
-    float acc = (EPI == EPI_ACCUM) ? a.y[i] : 0.0f;
-    float acc2 = 0.0f;
-    const float4* x4 = reinterpret_cast<const float4*>(a.x);
-    for (int64_t c = 0; c < ntiles; ++c) {
-      const int s = int(c % stages);
-      mbar_wait(&bar[s], uint32_t((c / stages) & 1));
-      const float4* ra = reinterpret_cast<const float4*>(tiles + s * stage_floats + int64_t(t) * kStagePitch);
-      const float4* rb = ra + R * kStagePitch / 4;
-      const int64_t j0 = c * kStageKT;
-      const int len4 = int(imin64(kStageKT, N - j0)) >> 2;
-#pragma unroll 8
-      for (int q = 0; q < len4; ++q) {
-        const float4 xv = x4[(j0 >> 2) + q];
-        const float4 v = ra[q];
-        acc = fmaf(v.x, xv.x, acc);
-        acc = fmaf(v.y, xv.y, acc);
-        acc = fmaf(v.z, xv.z, acc);
-        acc = fmaf(v.w, xv.w, acc);
-        if (NMAT == 2) {
-          const float4 w = rb[q];
-          acc2 = fmaf(w.x, xv.x, acc2);
-          acc2 = fmaf(w.y, xv.y, acc2);
-          acc2 = fmaf(w.z, xv.z, acc2);
-          acc2 = fmaf(w.w, xv.w, acc2);
-        }
-      }
-      if (c + stages < ntiles) {
-        // this thread's generic reads of its slot are done before the async
-        // proxy overwrites it
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        issue(c + stages);
+  if (S > 1) {
+    if (lane == 0) {
+      red[0][warp] = acc;
+      red[1][warp] = acc2;
+    }
+    __syncthreads();
+    if (part == 0 && lane == 0) {
+      for (int p = 1; p < S; ++p) {
+        acc += red[0][warp + p];
+        acc2 += red[1][warp + p];
       }
     }
+  }
+  if (part == 0 && lane == 0 && i < a.M) {
+    if (EPI == EPI_ACCUM) acc = a.y[i] + acc;
     row_epilogue<NMAT, EPI>(a, i, acc, acc2);
   }
   cta_exit(a.t);
@@ -382,10 +294,126 @@ __global__ void __launch_bounds__(1024, 1) col_warp_kernel(ColArgs a) {
   cta_exit(a.t);
 }
 
+// ---------------------------------------------------------------- column, cluster of CTAs per 128-column block (COOP)
+// Lane l owns 16-byte column chunk c0 + l (4 columns); the R CTAs of a
+// cluster split the rows; warp w of CTA r sums rows r*Mr + w + 8*t. Warp
+// partials are added in warp order in shared memory, then CTA 0 adds the R
+// CTA partials in rank order through distributed shared memory.
+template <int EPI>
+__global__ void __launch_bounds__(256) col_cluster_kernel(ColArgs a) {
+  namespace cg = cooperative_groups;
+  constexpr int U = 8, NW = 8;
+  __shared__ int slots;
+  __shared__ float4 red[NW][32];
+  __shared__ float4 partial[32];
+  cg::cluster_group cluster = cg::this_cluster();
+  const int R = int(cluster.num_blocks()), rank = int(cluster.block_rank());
+  gate_init(&slots, a.t);
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t n4 = a.N >> 2;
+  const int64_t jq = int64_t(blockIdx.x) * 32 + lane;
+  const int64_t Mr = (a.M + R - 1) / R;
+  const int64_t r0 = rank * Mr, r1 = imin64(a.M, r0 + Mr);
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  throttled(a.t, &slots, [&]() {
+    if (jq >= n4) return;
+    const float4* col = reinterpret_cast<const float4*>(a.A) + jq;
+    int64_t i = r0 + warp;
+    for (; i + (U - 1) * NW < r1; i += U * NW) {
+      float4 w[U];
+      float vv[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        w[u] = ld_na4(col + (i + int64_t(u) * NW) * n4);
+        vv[u] = a.v[i + int64_t(u) * NW];
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        acc.x = fmaf(w[u].x, vv[u], acc.x);
+        acc.y = fmaf(w[u].y, vv[u], acc.y);
+        acc.z = fmaf(w[u].z, vv[u], acc.z);
+        acc.w = fmaf(w[u].w, vv[u], acc.w);
+      }
+    }
+    for (; i < r1; i += NW) {
+      const float4 w = ld_na4(col + i * n4);
+      const float vi = a.v[i];
+      acc.x = fmaf(w.x, vi, acc.x);
+      acc.y = fmaf(w.y, vi, acc.y);
+      acc.z = fmaf(w.z, vi, acc.z);
+      acc.w = fmaf(w.w, vi, acc.w);
+    }
+  });
+  red[warp][lane] = acc;
+  __syncthreads();
+  if (warp == 0) {
+    float4 s = red[0][lane];
+    for (int w = 1; w < NW; ++w) {
+      s.x += red[w][lane].x;
+      s.y += red[w][lane].y;
+      s.z += red[w][lane].z;
+      s.w += red[w][lane].w;
+    }
+    partial[lane] = s;
+  }
+  cluster.sync();
+  if (rank == 0 && warp == 0 && jq < n4) {
+    float4 s = partial[lane];
+    for (int q = 1; q < R; ++q) {
+      const float4 o = cluster.map_shared_rank(partial, q)[lane];
+      s.x += o.x;
+      s.y += o.y;
+      s.z += o.z;
+      s.w += o.w;
+    }
+    float4* y4 = reinterpret_cast<float4*>(a.y);
+    if (EPI == EPI_ACCUM) {
+      const float4 y0 = y4[jq];
+      s = make_float4(y0.x + s.x, y0.y + s.y, y0.z + s.z, y0.w + s.w);
+    }
+    y4[jq] = s;
+  }
+  cluster.sync();
+}
+
 // ---------------------------------------------------------------- host launchers
+catt_status launch_row_tma(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t M, int64_t N,
+                           float alpha, float beta, int epi, const catt_throttle* t, cudaStream_t s);
+catt_status launch_col_tma(const float* A, const float* v, float* y, int64_t M, int64_t N, int accumulate,
+                           const catt_throttle* t, cudaStream_t s);
+
 namespace {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+// warps per row for the COOP row loop: enough warps to fill the GPU
+int coop_split(int64_t M) {
+  const int64_t target = 148 * 32;
+  int S = 1;
+  while (S < 8 && M * S < target) S *= 2;
+  return S;
+}
+
+template <int NMAT, int EPI, bool VEC>
+const void* row_warp_func(int S) {
+  switch (S) {
+    case 1: return (const void*)row_warp_kernel<NMAT, EPI, VEC, 1>;
+    case 2: return (const void*)row_warp_kernel<NMAT, EPI, VEC, 2>;
+    case 4: return (const void*)row_warp_kernel<NMAT, EPI, VEC, 4>;
+    default: return (const void*)row_warp_kernel<NMAT, EPI, VEC, 8>;
+  }
+}
+
+template <int NMAT, int EPI, bool VEC>
+void row_warp_launch(int S, unsigned grid, size_t dyn, cudaStream_t s, const RowArgs& a) {
+  switch (S) {
+    case 1: row_warp_kernel<NMAT, EPI, VEC, 1><<<grid, 256, dyn, s>>>(a); break;
+    case 2: row_warp_kernel<NMAT, EPI, VEC, 2><<<grid, 256, dyn, s>>>(a); break;
+    case 4: row_warp_kernel<NMAT, EPI, VEC, 4><<<grid, 256, dyn, s>>>(a); break;
+    default: row_warp_kernel<NMAT, EPI, VEC, 8><<<grid, 256, dyn, s>>>(a); break;
+  }
+}
 
 template <int NMAT, int EPI>
 catt_status launch_row_t(RowArgs a, const catt_throttle* t, cudaStream_t s) {
@@ -408,37 +436,21 @@ catt_status launch_row_t(RowArgs a, const catt_throttle* t, cudaStream_t s) {
     return after_launch();
   }
   if (var == CATT_VAR_COOP) {
-    const int threads = cta_threads_or(t, 256);
-    const void* f = vec_ok ? (const void*)row_warp_kernel<NMAT, EPI, true>
-                           : (const void*)row_warp_kernel<NMAT, EPI, false>;
+    if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
+    const int S = coop_split(a.M);
+    const void* f = vec_ok ? row_warp_func<NMAT, EPI, true>(S) : row_warp_func<NMAT, EPI, false>(S);
     size_t dyn = 0;
-    catt_status st = prepare_launch(f, t, threads, 0, true, &a.t, &dyn);
+    catt_status st = prepare_launch(f, t, 256, 0, true, &a.t, &dyn);
     if (st != CATT_OK) return st;
-    const int64_t grid = (a.M + threads / 32 - 1) / (threads / 32);
+    const unsigned grid = unsigned((a.M + (8 / S) - 1) / (8 / S));
     if (vec_ok)
-      row_warp_kernel<NMAT, EPI, true><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
+      row_warp_launch<NMAT, EPI, true>(S, grid, dyn, s, a);
     else
-      row_warp_kernel<NMAT, EPI, false><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
+      row_warp_launch<NMAT, EPI, false>(S, grid, dyn, s, a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) {
-    if (!vec_ok) return CATT_EINVAL;
-    const int R = cta_threads_or(t, 32);
-    if (R > 256) return CATT_EINVAL;
-    const int64_t stage_bytes = int64_t(NMAT) * R * kStagePitch * 4;
-    const int stages = int(std::min<int64_t>(16, (200 * 1024) / stage_bytes));
-    if (stages < 2) return CATT_EINVAL;
-    const size_t dyn = 128 + size_t(stages) * size_t(stage_bytes);
-    const void* f = (const void*)row_staged_kernel<NMAT, EPI>;
-    if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn)) != cudaSuccess)
-      return after_launch();
-    size_t dyn_total = 0;
-    catt_status st = prepare_launch(f, t, R, dyn, false, &a.t, &dyn_total);
-    if (st != CATT_OK) return st;
-    const int64_t grid = (a.M + R - 1) / R;
-    row_staged_kernel<NMAT, EPI><<<dim3(unsigned(grid)), R, dyn_total, s>>>(a, stages);
-    return after_launch();
-  }
+  if (var == CATT_VAR_STAGED)
+    return launch_row_tma(a.A, a.B, a.x, a.y, a.tmp, a.M, a.N, a.alpha, a.beta, EPI, t, s);
   return CATT_EINVAL;
 }
 
@@ -463,6 +475,36 @@ catt_status launch_col_t(ColArgs a, const catt_throttle* t, cudaStream_t s) {
     return after_launch();
   }
   if (var == CATT_VAR_COOP) {
+    const bool vec = (a.N % 4 == 0) && aligned16(a.A) && aligned16(a.y);
+    const bool capped = t && t->active_ctas > 0;
+    if (vec && !capped) {
+      if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
+      const void* f = (const void*)col_cluster_kernel<EPI>;
+      size_t dyn = 0;
+      catt_status st = prepare_launch(f, t, 256, 0, true, &a.t, &dyn);
+      if (st != CATT_OK) return st;
+      const int64_t nblk = (a.N / 4 + 31) / 32;
+      int R = 1;
+      while (R < 8 && nblk * R < 2 * 148) R *= 2;
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(unsigned(nblk), unsigned(R), 1);
+      cfg.blockDim = dim3(256, 1, 1);
+      cfg.dynamicSmemBytes = dyn;
+      cfg.stream = s;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeClusterDimension;
+      attr[0].val.clusterDim.x = 1;
+      attr[0].val.clusterDim.y = unsigned(R);
+      attr[0].val.clusterDim.z = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      cudaError_t e = cudaLaunchKernelEx(&cfg, col_cluster_kernel<EPI>, a);
+      if (e != cudaSuccess) {
+        record_cuda_error(e);
+        return CATT_ECUDA;
+      }
+      return after_launch();
+    }
     const int threads = cta_threads_or(t, 1024);
     const void* f = (const void*)col_warp_kernel<EPI>;
     size_t dyn = 0;
@@ -472,6 +514,7 @@ catt_status launch_col_t(ColArgs a, const catt_throttle* t, cudaStream_t s) {
     col_warp_kernel<EPI><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
     return after_launch();
   }
+  if (var == CATT_VAR_STAGED) return launch_col_tma(a.A, a.v, a.y, a.M, a.N, EPI == EPI_ACCUM, t, s);
   return CATT_EINVAL;
 }
 
@@ -483,39 +526,39 @@ catt_status check_common(int64_t m, int64_t n) {
 
 }  // namespace
 
+const void* row_tma_func(int nmat);
+const void* col_tma_func();
+
 // Kernel instance a loop + variant launches (for attributes / descriptors).
 const void* gemv_func(int loop, int variant, bool vec_ok) {
   const bool row = loop == CATT_K_ATAX_1 || loop == CATT_K_BICG_2 || loop == CATT_K_MVT_1 || loop == CATT_K_GESUMMV;
   if (row) {
+    const int nmat = loop == CATT_K_GESUMMV ? 2 : 1;
+    if (variant == CATT_VAR_STAGED) return row_tma_func(nmat);
     if (loop == CATT_K_GESUMMV) {
       if (variant == CATT_VAR_VEC4) return (const void*)row_thread_kernel<2, EPI_GESUMMV, true>;
       if (variant == CATT_VAR_COOP)
-        return vec_ok ? (const void*)row_warp_kernel<2, EPI_GESUMMV, true> : (const void*)row_warp_kernel<2, EPI_GESUMMV, false>;
-      if (variant == CATT_VAR_STAGED) return (const void*)row_staged_kernel<2, EPI_GESUMMV>;
+        return vec_ok ? row_warp_func<2, EPI_GESUMMV, true>(1) : row_warp_func<2, EPI_GESUMMV, false>(1);
       return (const void*)row_thread_kernel<2, EPI_GESUMMV, false>;
     }
     if (loop == CATT_K_MVT_1) {
       if (variant == CATT_VAR_VEC4) return (const void*)row_thread_kernel<1, EPI_ACCUM, true>;
       if (variant == CATT_VAR_COOP)
-        return vec_ok ? (const void*)row_warp_kernel<1, EPI_ACCUM, true> : (const void*)row_warp_kernel<1, EPI_ACCUM, false>;
-      if (variant == CATT_VAR_STAGED) return (const void*)row_staged_kernel<1, EPI_ACCUM>;
+        return vec_ok ? row_warp_func<1, EPI_ACCUM, true>(1) : row_warp_func<1, EPI_ACCUM, false>(1);
       return (const void*)row_thread_kernel<1, EPI_ACCUM, false>;
     }
     if (variant == CATT_VAR_VEC4) return (const void*)row_thread_kernel<1, EPI_STORE, true>;
     if (variant == CATT_VAR_COOP)
-      return vec_ok ? (const void*)row_warp_kernel<1, EPI_STORE, true> : (const void*)row_warp_kernel<1, EPI_STORE, false>;
-    if (variant == CATT_VAR_STAGED) return (const void*)row_staged_kernel<1, EPI_STORE>;
+      return vec_ok ? row_warp_func<1, EPI_STORE, true>(1) : row_warp_func<1, EPI_STORE, false>(1);
     return (const void*)row_thread_kernel<1, EPI_STORE, false>;
   }
   const bool acc = loop == CATT_K_MVT_2;
+  if (variant == CATT_VAR_STAGED) return col_tma_func();
   if (variant == CATT_VAR_VEC4) return acc ? (const void*)col_thread_kernel<EPI_ACCUM, true> : (const void*)col_thread_kernel<EPI_STORE, true>;
-  if (variant == CATT_VAR_COOP) return acc ? (const void*)col_warp_kernel<EPI_ACCUM> : (const void*)col_warp_kernel<EPI_STORE>;
+  if (variant == CATT_VAR_COOP)
+    return vec_ok ? (acc ? (const void*)col_cluster_kernel<EPI_ACCUM> : (const void*)col_cluster_kernel<EPI_STORE>)
+                  : (acc ? (const void*)col_warp_kernel<EPI_ACCUM> : (const void*)col_warp_kernel<EPI_STORE>);
   return acc ? (const void*)col_thread_kernel<EPI_ACCUM, false> : (const void*)col_thread_kernel<EPI_STORE, false>;
-}
-
-int staged_stages(int nmat, int rows) {
-  const int64_t stage_bytes = int64_t(nmat) * rows * kStagePitch * 4;
-  return int(std::min<int64_t>(16, (200 * 1024) / stage_bytes));
 }
 
 catt_status launch_row(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t M, int64_t N,

@@ -11,7 +11,10 @@
 namespace catt {
 
 const void* gemv_func(int loop, int variant, bool vec_ok);
-int staged_stages(int nmat, int rows);
+int row_tma_stages(int nmat, int rows, int boxes);
+int col_tma_stages(int cols, int rows_per_stage);
+int row_tma_stage_bytes(int nmat, int rows, int boxes);
+int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
 const void* kmeans_func(int variant, int nf);
 
@@ -187,7 +190,6 @@ catt_ref mkref(int64_t cx, int64_t cy, int64_t c0, int64_t c1, int32_t e, int32_
 
 int default_threads(int loop, int variant) {
   if (variant == CATT_VAR_STAGED) return loop == CATT_K_SYRK ? 256 : 32;
-  if (variant == CATT_VAR_COOP && (loop == CATT_K_ATAX_2 || loop == CATT_K_BICG_1 || loop == CATT_K_MVT_2)) return 1024;
   return 256;
 }
 
@@ -268,8 +270,9 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       if (two) refs[n++] = mkref(N / 4, 0, 1, 0, 16, 3, NL);
       out->trip[0] = N / 4;
       out->grid[0] = (M + threads - 1) / threads;
-      const int stages = staged_stages(two ? 2 : 1, threads);
-      dyn = 128 + int64_t(stages) * (two ? 2 : 1) * threads * (128 + 4) * 4;
+      const int nmat = two ? 2 : 1;
+      const int boxes = std::max(1, std::min(8, 16384 / (nmat * threads * 128)));
+      dyn = 1024 + int64_t(row_tma_stages(nmat, threads, boxes)) * row_tma_stage_bytes(nmat, threads, boxes);
     } else if (var == CATT_VAR_COOP) {
       // warp per row: lane = gid_x (block 32 x W), row = gid_y
       const int64_t C4 = (N % 4 == 0) ? N / 4 : N;
@@ -313,6 +316,15 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       refs[n++] = mkref(1, N, int64_t(NW) * N, 0, 4, 1, NL);
       refs[n++] = mkref(0, 1, NW, 0, 4, 2, 0);
       out->trip[0] = (M + NW - 1) / NW;
+    } else if (var == CATT_VAR_STAGED) {
+      if (N % 4) return CATT_EINVAL;
+      const int RB = std::max(8, std::min(256, 16384 / (threads * 4)));
+      refs[n++] = mkref(1, 0, N, 0, 4, 1, NL);                     // tiles arrive by TMA
+      refs[n++] = mkref(0, 0, 1, 0, 4, 2, 0);                      // v[i] broadcast
+      out->trip[0] = M;
+      out->grid[0] = (N + threads - 1) / threads;
+      out->extent[0] = N;
+      dyn = 1024 + int64_t(col_tma_stages(threads, RB)) * col_tma_stage_bytes(threads, RB);
     } else {
       return CATT_EINVAL;
     }

@@ -70,7 +70,7 @@ def test_atax_exact(variant, m, n):
         with pytest.raises(catt.CattError):
             catt.atax(dev(A), dev(x), k1=t)
         return
-    tmp, y = catt.atax(dev(A), dev(x), k1=t, k2=catt.Throttle(variant="literal"))
+    tmp, y = catt.atax(dev(A), dev(x), k1=t, k2=catt.Throttle(variant=variant))
     assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y), y_o)
 
 
@@ -80,7 +80,7 @@ def test_bicg(variant, m, n):
     A, p, r = si.matrix(2, m, n), si.values(102, n), si.values(202, m)
     q_o, s_o = oracle.bicg(A, p, r)
     q64, s64 = oracle.bicg(A, p, r, mode=oracle.SEQ_F64)
-    col_var = {"staged": "literal"}.get(variant, variant)     # no staged column loop
+    col_var = variant
     if not _vec_ok(variant, n):
         with pytest.raises(catt.CattError):
             catt.bicg(dev(A), dev(p), dev(r), k1=catt.Throttle(variant=col_var), k2=catt.Throttle(variant=variant))
@@ -100,7 +100,7 @@ def test_mvt(variant, n):
     y1, y2, x1, x2 = (si.values(103 + 100 * k, n) for k in range(4))
     o1, o2 = oracle.mvt(a, y1, y2, x1, x2)
     e1, e2 = oracle.mvt(a, y1, y2, x1, x2, mode=oracle.SEQ_F64)
-    col_var = {"staged": "literal"}.get(variant, variant)
+    col_var = variant
     X1, X2 = dev(x1), dev(x2)
     if not _vec_ok(variant, n):
         with pytest.raises(catt.CattError):
@@ -231,8 +231,7 @@ def test_bicg_mvt_4096_full():
     q64, s64 = oracle.bicg(Ah, p, r, mode=oracle.SEQ_F64)
     A = A.view(n, n)
     for v in ("literal", "vec4", "staged", "coop"):
-        q, s = catt.bicg(A, dev(p), dev(r), k1=catt.Throttle(variant="coop" if v == "coop" else "literal"),
-                         k2=catt.Throttle(variant=v))
+        q, s = catt.bicg(A, dev(p), dev(r), k1=catt.Throttle(variant=v), k2=catt.Throttle(variant=v))
         q, s = host(q), host(s)
         if v == "coop":
             assert relerr(q, q64) <= TOL and relerr(s, s64) <= TOL
@@ -296,7 +295,7 @@ def test_atax_65536x16384_sampled():
     x = si.values(si.sub_seed(si.SEED_ATAX_SHARDED, 1), n)
     cols = np.array([0, 1, 31, 32, 4097, 16383])
     tmp_o, y_o = oracle.atax_hashed(si.SEED_ATAX_SHARDED, 0, x, m, n, cols)
-    tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="staged"), k2=catt.Throttle())
+    tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="staged"), k2=catt.Throttle(variant="staged"))
     assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y)[cols], y_o)
     tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="coop"), k2=catt.Throttle(variant="coop"))
     t64, y64 = oracle.atax_hashed(si.SEED_ATAX_SHARDED, 0, x, m, n, cols, mode=oracle.SEQ_F64)

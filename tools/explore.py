@@ -46,12 +46,12 @@ def gemv_4096():
     y = torch.empty(n, device=dev)
     nbytes = n * n * 4
     for var, ctas in [("literal", [32, 64, 128, 256, 1024]), ("vec4", [32, 64, 128, 256]),
-                      ("staged", [32, 64, 128]), ("coop", [128, 256, 512])]:
+                      ("staged", [32, 64, 128]), ("coop", [256])]:
         for c in ctas:
             t = catt.Throttle(cta_threads=c, variant=var)
             ms = timeit(lambda: catt.rows(A, x, y, t=t))
             report(f"rows 4096 {var} cta={c}", ms, nbytes)
-    for var, ctas in [("literal", [32, 64, 128, 256]), ("vec4", [32, 64, 128]), ("coop", [256, 512, 1024])]:
+    for var, ctas in [("literal", [32, 64, 128, 256]), ("vec4", [32, 64, 128]), ("staged", [32, 64, 128]), ("coop", [256])]:
         for c in ctas:
             t = catt.Throttle(cta_threads=c, variant=var)
             ms = timeit(lambda: catt.cols(A, x, y, t=t))
@@ -139,7 +139,7 @@ def atax_big():
         t = catt.Throttle(cta_threads=c, variant=var)
         ms = timeit(lambda: catt.rows(A, x, tmp, t=t), reps=5)
         report(f"rows 65536x16384 {var} cta={c}", ms, nbytes)
-    for var, c in [("literal", 256), ("vec4", 256), ("coop", 1024)]:
+    for var, c in [("literal", 256), ("vec4", 256), ("staged", 32), ("staged", 64), ("coop", 256)]:
         t = catt.Throttle(cta_threads=c, variant=var)
         ms = timeit(lambda: catt.cols(A, tmp, y, t=t), reps=5)
         report(f"cols 65536x16384 {var} cta={c}", ms, nbytes)
