@@ -180,9 +180,9 @@ class BicgMvt(Workload):
         for k, v in enumerate((self.r, self.y2, self.x1)):
             catt.fill_hash(v, si.sub_seed(si.SEED_MVT, k + 1), offset=rank * rows)
         var = self.variant
-        col_var = "coop" if var in ("coop",) else "literal"
+        col_var = var if var in ("coop", "staged") else "literal"
         cta_row = {"coop": 256, "staged": 32, "vec4": 32, "literal": 32}[var]
-        cta_col = 1024 if col_var == "coop" else 256
+        cta_col = {"coop": 256, "staged": 32, "literal": 256}[col_var]
         P = catt.problem
         tb1 = self.plan("bicg1 s=A^T r", P(catt.K_BICG_1, m=rows, n=n), catt.Throttle(cta_threads=cta_col, variant=col_var))
         tb2 = self.plan("bicg2 q=A p", P(catt.K_BICG_2, m=rows, n=n), catt.Throttle(cta_threads=cta_row, variant=var))
@@ -345,9 +345,9 @@ class Atax(Workload):
         var = self.variant
         t1 = self.plan("atax1 tmp=A x", catt.problem(catt.K_ATAX_1, m=rows, n=n),
                        catt.Throttle(cta_threads=256 if var == "coop" else 32, variant=var))
-        cv = "coop" if var == "coop" else "literal"
+        cv = var if var in ("coop", "staged") else "literal"
         t2 = self.plan("atax2 y=A^T tmp", catt.problem(catt.K_ATAX_2, m=rows, n=n),
-                       catt.Throttle(cta_threads=1024 if cv == "coop" else 256, variant=cv))
+                       catt.Throttle(cta_threads={"coop": 256, "staged": 32, "literal": 256}[cv], variant=cv))
         mat = rows * n * 4
         self.loops = [Loop("atax1 tmp=A x", lambda: catt.rows(self.A, self.x, self.tmp, catt.ROWS_STORE, t=t1),
                            mat + 4 * (rows + n), "rows"),

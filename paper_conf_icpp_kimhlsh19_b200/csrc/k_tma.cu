@@ -136,15 +136,25 @@ __global__ void __launch_bounds__(256) row_tma_kernel(const __grid_constant__ CU
       const unsigned char* rowp = st + t * 128;
       const float4* xs = reinterpret_cast<const float4*>(st + x_off);
       if (len == KT) {
-        // full tile: branch-free, all 8 chunks of a box loaded before the FMAs
-        for (int b = 0; b < B; ++b) {
-          const unsigned char* bp = rowp + b * box_bytes;
-          float4 v[8], w[NMAT == 2 ? 8 : 1], xv[8];
+        // full tile: software-pipelined one box (8 chunks) ahead, so the
+        // shared-memory latency overlaps the previous box's FMA chain
+        float4 v[8], w[NMAT == 2 ? 8 : 1], xv[8];
 #pragma unroll
-          for (int k = 0; k < 8; ++k) {
-            v[k] = *reinterpret_cast<const float4*>(bp + ((k ^ sw) << 4));
-            if (NMAT == 2) w[k] = *reinterpret_cast<const float4*>(bp + B * box_bytes + ((k ^ sw) << 4));
-            xv[k] = xs[b * 8 + k];
+        for (int k = 0; k < 8; ++k) {
+          v[k] = *reinterpret_cast<const float4*>(rowp + ((k ^ sw) << 4));
+          if (NMAT == 2) w[k] = *reinterpret_cast<const float4*>(rowp + B * box_bytes + ((k ^ sw) << 4));
+          xv[k] = xs[k];
+        }
+        for (int b = 0; b < B; ++b) {
+          float4 vn[8], wn[NMAT == 2 ? 8 : 1], xn[8];
+          if (b + 1 < B) {
+            const unsigned char* bp = rowp + (b + 1) * box_bytes;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+              vn[k] = *reinterpret_cast<const float4*>(bp + ((k ^ sw) << 4));
+              if (NMAT == 2) wn[k] = *reinterpret_cast<const float4*>(bp + B * box_bytes + ((k ^ sw) << 4));
+              xn[k] = xs[(b + 1) * 8 + k];
+            }
           }
 #pragma unroll
           for (int k = 0; k < 8; ++k) {
@@ -157,6 +167,14 @@ __global__ void __launch_bounds__(256) row_tma_kernel(const __grid_constant__ CU
               acc2 = fmaf(w[k].y, xv[k].y, acc2);
               acc2 = fmaf(w[k].z, xv[k].z, acc2);
               acc2 = fmaf(w[k].w, xv[k].w, acc2);
+            }
+          }
+          if (b + 1 < B) {
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+              v[k] = vn[k];
+              if (NMAT == 2) w[k] = wn[k];
+              xv[k] = xn[k];
             }
           }
         }
@@ -247,15 +265,31 @@ __global__ void __launch_bounds__(256) col_tma_kernel(const __grid_constant__ CU
       const float* tp = reinterpret_cast<const float*>(st) + t;
       const float* vs = reinterpret_cast<const float*>(st + tile_bytes);
       if (rows == RB) {
-        for (int r0 = 0; r0 < RB; r0 += 8) {
-          float w[8], vv[8];
+        // pipelined 16 rows ahead of the FMA chain
+        float w[16], vv[16];
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {
-            w[u] = tp[(r0 + u) * CB];
-            vv[u] = vs[r0 + u];
+        for (int u = 0; u < 16; ++u) {
+          w[u] = tp[u * CB];
+          vv[u] = vs[u];
+        }
+        for (int r0 = 0; r0 < RB; r0 += 16) {
+          float wn[16], vn[16];
+          if (r0 + 16 < RB) {
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+              wn[u] = tp[(r0 + 16 + u) * CB];
+              vn[u] = vs[r0 + 16 + u];
+            }
           }
 #pragma unroll
-          for (int u = 0; u < 8; ++u) acc = fmaf(w[u], vv[u], acc);
+          for (int u = 0; u < 16; ++u) acc = fmaf(w[u], vv[u], acc);
+          if (r0 + 16 < RB) {
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+              w[u] = wn[u];
+              vv[u] = vn[u];
+            }
+          }
         }
       } else {
         for (int r = 0; r < rows; ++r) acc = fmaf(tp[r * CB], vs[r], acc);
@@ -362,7 +396,7 @@ catt_status launch_col_tma(const float* A, const float* v, float* y, int64_t M, 
   if (!tma_ok(A, N) || (reinterpret_cast<uintptr_t>(v) & 15u)) return CATT_EINVAL;
   const int CB = cta_threads_or(t, 32);
   if (CB > 256 || CB % 32) return CATT_EINVAL;
-  const int RB = std::max(8, std::min(256, 16384 / (CB * 4)));              // ~16 KB per stage
+  const int RB = std::max(16, std::min(256, 16384 / (CB * 4))) / 16 * 16;  // ~16 KB per stage, multiple of 16
   const int stages = col_tma_stages(CB, RB);
   const size_t dyn = 1024 + size_t(stages) * col_tma_stage_bytes(CB, RB);
   CUtensorMap ma;

@@ -318,7 +318,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->trip[0] = (M + NW - 1) / NW;
     } else if (var == CATT_VAR_STAGED) {
       if (N % 4) return CATT_EINVAL;
-      const int RB = std::max(8, std::min(256, 16384 / (threads * 4)));
+      const int RB = std::max(16, std::min(256, 16384 / (threads * 4))) / 16 * 16;
       refs[n++] = mkref(1, 0, N, 0, 4, 1, NL);                     // tiles arrive by TMA
       refs[n++] = mkref(0, 0, 1, 0, 4, 2, 0);                      // v[i] broadcast
       out->trip[0] = M;

@@ -1,0 +1,96 @@
+"""Row-sharded multi-GPU ATAX / BICG / MVT / GESUMMV.
+
+One process per GPU (torch.distributed, NCCL over NVLink/NVSwitch). Rows of A
+are split across ranks; every rank runs the CATT-throttled loops on its own
+rows through the C ABI, and the A^T partial sums are added with one
+all_reduce(SUM) -- the only exchange these loops have:
+
+    ATAX   tmp_g = A_g x (local),      y = sum_g A_g^T tmp_g        (all-reduce)
+    BICG   q_g   = A_g p (local),      s = sum_g A_g^T r_g          (all-reduce)
+    MVT    x1_g += A_g y1 (local),     x2 = x2 + sum_g A_g^T y2_g   (all-reduce;
+           only rank 0 adds the initial x2, so the sum carries it once)
+    GESUMMV y_g = alpha A_g x + beta B_g x (local, no collective)
+
+The per-rank loop calls are injected (`ops`), so the partitioning and the
+collective composition can be tested on CPU over gloo with any loop
+implementation; the default ops are the CUDA kernels (catt.rows / catt.cols).
+"""
+from __future__ import annotations
+
+from typing import Callable, Optional, Tuple
+
+from . import catt
+
+
+def row_range(m: int, world: int, rank: int) -> Tuple[int, int]:
+    """Contiguous, balanced row block [lo, hi) of rank `rank` (first m % world ranks get one more)."""
+    base, extra = divmod(m, world)
+    lo = rank * base + min(rank, extra)
+    return lo, lo + base + (1 if rank < extra else 0)
+
+
+class CudaOps:
+    """Per-rank loops on the local GPU (the product path)."""
+
+    @staticmethod
+    def rows(A, x, y, mode, t=None, B=None, tmp=None, alpha=0.0, beta=0.0):
+        return catt.rows(A, x, y, mode, B=B, tmp=tmp, alpha=alpha, beta=beta, t=t)
+
+    @staticmethod
+    def cols(A, v, y, accumulate, t=None):
+        return catt.cols(A, v, y, accumulate, t=t)
+
+
+def _reduce(t, group):
+    import torch.distributed as dist
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t
+
+
+def _rank(group):
+    import torch.distributed as dist
+    return dist.get_rank(group) if dist.is_initialized() else 0
+
+
+def atax_rowshard(A_g, x, tmp_g=None, y=None, k1=None, k2=None, group=None, ops=CudaOps):
+    """tmp_g = A_g x; y = sum over ranks of A_g^T tmp_g."""
+    import torch
+    m, n = A_g.shape
+    tmp_g = torch.empty(m, dtype=A_g.dtype, device=A_g.device) if tmp_g is None else tmp_g
+    y = torch.empty(n, dtype=A_g.dtype, device=A_g.device) if y is None else y
+    ops.rows(A_g, x, tmp_g, catt.ROWS_STORE, k1)
+    ops.cols(A_g, tmp_g, y, False, k2)
+    _reduce(y, group)
+    return tmp_g, y
+
+
+def bicg_rowshard(A_g, p, r_g, q_g=None, s=None, k1=None, k2=None, group=None, ops=CudaOps):
+    """s = sum over ranks of A_g^T r_g (k1); q_g = A_g p (k2)."""
+    import torch
+    m, n = A_g.shape
+    q_g = torch.empty(m, dtype=A_g.dtype, device=A_g.device) if q_g is None else q_g
+    s = torch.empty(n, dtype=A_g.dtype, device=A_g.device) if s is None else s
+    ops.cols(A_g, r_g, s, False, k1)
+    ops.rows(A_g, p, q_g, catt.ROWS_STORE, k2)
+    _reduce(s, group)
+    return q_g, s
+
+
+def mvt_rowshard(A_g, y1, y2_g, x1_g, x2, k1=None, k2=None, group=None, ops=CudaOps):
+    """x1_g += A_g y1 (local rows); x2 = x2 + sum over ranks of A_g^T y2_g.
+    A_g is the rank's rows of the square A; x2 is replicated, updated in place."""
+    ops.rows(A_g, y1, x1_g, catt.ROWS_ACCUM, k1)
+    ops.cols(A_g, y2_g, x2, _rank(group) == 0, k2)   # only rank 0 carries the initial x2
+    _reduce(x2, group)
+    return x1_g, x2
+
+
+def gesummv_rowshard(A_g, B_g, x, alpha, beta, y_g=None, tmp_g=None, t=None, ops=CudaOps):
+    """y_g = alpha A_g x + beta B_g x, tmp_g = A_g x: fully local, no collective."""
+    import torch
+    m = A_g.shape[0]
+    y_g = torch.empty(m, dtype=A_g.dtype, device=A_g.device) if y_g is None else y_g
+    tmp_g = torch.empty(m, dtype=A_g.dtype, device=A_g.device) if tmp_g is None else tmp_g
+    ops.rows(A_g, x, y_g, catt.ROWS_GESUMMV, t, B=B_g, tmp=tmp_g, alpha=alpha, beta=beta)
+    return y_g, tmp_g

@@ -1,0 +1,173 @@
+"""Multi-process tests of the row-sharded path.
+
+CPU, world_size 2 over gloo: the partitioning and the collective composition
+of paper_conf_icpp_kimhlsh19_b200.dist with oracle-backed per-rank loops.
+On exact-dyadic inputs the sharded result is bit-identical to the unsharded
+oracle (every partial sum is exact, so the all-reduce order cannot matter);
+on uniform inputs it is within the 1e-5 bar of the fp64 oracle.
+GPU (1 device): the same functions through the CUDA kernels with a
+single-rank NCCL group.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import seeded_inputs as si
+from paper_conf_icpp_kimhlsh19_b200 import catt as catt_mod
+from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+
+
+class OracleOps:
+    """Per-rank loops computed by the CPU oracle (test infrastructure). The
+    accumulate forms reuse the oracle's MVT loops (init first, then the
+    sequential fmaf sum), zero-padding the row shard to a square matrix."""
+
+    @staticmethod
+    def rows(A, x, y, mode, t=None, B=None, tmp=None, alpha=0.0, beta=0.0):
+        An, xn = A.numpy(), x.numpy()
+        m, n = An.shape
+        if mode == catt_mod.ROWS_GESUMMV:
+            yy, tt = oracle.gesummv(An, B.numpy(), xn, alpha, beta)
+            y.copy_(torch.from_numpy(yy))
+            tmp.copy_(torch.from_numpy(tt))
+        elif mode == catt_mod.ROWS_ACCUM:                       # y += A x  (MVT loop 1)
+            sq = np.zeros((n, n), np.float32)
+            sq[:m] = An
+            x1 = np.zeros(n, np.float32)
+            x1[:m] = y.numpy()
+            o1, _ = oracle.mvt(sq, xn, np.zeros(n, np.float32), x1, np.zeros(n, np.float32))
+            y.copy_(torch.from_numpy(o1[:m].copy()))
+        else:                                                   # y = A x   (BICG loop 2)
+            q, _ = oracle.bicg(An, xn, np.zeros(m, np.float32))
+            y.copy_(torch.from_numpy(q))
+        return y
+
+    @staticmethod
+    def cols(A, v, y, accumulate, t=None):
+        An, vn = A.numpy(), v.numpy()
+        m, n = An.shape
+        if accumulate:                                          # y += A^T v  (MVT loop 2)
+            sq = np.zeros((n, n), np.float32)
+            sq[:m] = An
+            y2 = np.zeros(n, np.float32)
+            y2[:m] = vn
+            _, o2 = oracle.mvt(sq, np.zeros(n, np.float32), y2, np.zeros(n, np.float32), y.numpy())
+            y.copy_(torch.from_numpy(o2))
+        else:                                                   # y = A^T v   (BICG loop 1)
+            _, s = oracle.bicg(An, np.zeros(n, np.float32), vn)
+            y.copy_(torch.from_numpy(s))
+        return y
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _worker(rank, world, port, mode, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        m, n = 301, 96                                  # ragged: 151 + 150 rows
+        A = si.matrix(7, m, n, mode=mode)
+        x, p = si.values(8, n, mode=mode), si.values(9, n, mode=mode)
+        r, y2 = si.values(10, m, mode=mode), si.values(11, m, mode=mode)
+        lo, hi = cdist.row_range(m, world, rank)
+        T = torch.from_numpy
+        tmp_g, y = cdist.atax_rowshard(T(A[lo:hi].copy()), T(x), ops=OracleOps)
+        q_g, s = cdist.bicg_rowshard(T(A[lo:hi].copy()), T(p), T(r[lo:hi].copy()), ops=OracleOps)
+        sq = si.matrix(12, n, n, mode=mode)             # MVT is square
+        lo2, hi2 = cdist.row_range(n, world, rank)
+        x1 = si.values(13, n, mode=mode)
+        x2 = T(si.values(14, n, mode=mode))
+        y1 = si.values(15, n, mode=mode)
+        y2s = si.values(16, n, mode=mode)
+        x1_g, x2 = cdist.mvt_rowshard(T(sq[lo2:hi2].copy()), T(y1), T(y2s[lo2:hi2].copy()),
+                                      T(x1[lo2:hi2].copy()), x2, ops=OracleOps)
+        q.put((rank, lo, hi, tmp_g.numpy(), y.numpy(), q_g.numpy(), s.numpy(), lo2, hi2, x1_g.numpy(), x2.numpy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("mode", [si.MODE_DYADIC, si.MODE_UNIFORM])
+def test_rowshard_world2_gloo(mode):
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, mode, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = sorted([q.get(timeout=180) for _ in range(world)], key=lambda t: t[0])
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    m, n = 301, 96
+    A = si.matrix(7, m, n, mode=mode)
+    x, p = si.values(8, n, mode=mode), si.values(9, n, mode=mode)
+    r = si.values(10, m, mode=mode)
+    tmp_o, y_o = oracle.atax(A, x)
+    q_o, s_o = oracle.bicg(A, p, r)
+    sq = si.matrix(12, n, n, mode=mode)
+    x1_o, x2_o = oracle.mvt(sq, si.values(15, n, mode=mode), si.values(16, n, mode=mode),
+                            si.values(13, n, mode=mode), si.values(14, n, mode=mode))
+    tmp = np.concatenate([t[3] for t in res])
+    q_all = np.concatenate([t[5] for t in res])
+    x1 = np.concatenate([t[9] for t in res])
+    assert [(t[1], t[2]) for t in res] == [(0, 151), (151, 301)]
+    assert np.array_equal(tmp, tmp_o) and np.array_equal(q_all, q_o) and np.array_equal(x1, x1_o)
+    for t in res:                                     # the all-reduced vectors are replicated
+        assert np.array_equal(t[4], res[0][4]) and np.array_equal(t[6], res[0][6]) and np.array_equal(t[10], res[0][10])
+    y, s, x2 = res[0][4], res[0][6], res[0][10]
+    if mode == si.MODE_DYADIC:
+        assert np.array_equal(y, y_o) and np.array_equal(s, s_o) and np.array_equal(x2, x2_o)
+    else:
+        _, y64 = oracle.atax(A, x, mode=oracle.SEQ_F64)
+        _, s64 = oracle.bicg(A, p, r, mode=oracle.SEQ_F64)
+        _, x2_64 = oracle.mvt(sq, si.values(15, n, mode=mode), si.values(16, n, mode=mode),
+                              si.values(13, n, mode=mode), si.values(14, n, mode=mode), mode=oracle.SEQ_F64)
+        for got, ref in ((y, y64), (s, s64), (x2, x2_64)):
+            assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-5
+
+
+def test_row_range_partitions():
+    for m in (0, 1, 7, 301, 65536):
+        for world in (1, 2, 3, 8):
+            rr = [cdist.row_range(m, world, g) for g in range(world)]
+            assert rr[0][0] == 0 and rr[-1][1] == m
+            assert all(rr[g][1] == rr[g + 1][0] for g in range(world - 1))
+            assert max(h - l for l, h in rr) - min(h - l for l, h in rr) <= 1
+
+
+@pytest.mark.gpu
+def test_rowshard_single_rank_nccl():
+    """The product path (CUDA kernels + NCCL) on a one-rank group."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(_free_port()))
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        m, n = 1000, 256
+        A = si.matrix(7, m, n, mode=si.MODE_DYADIC)
+        x, r = si.values(8, n, mode=si.MODE_DYADIC), si.values(10, m, mode=si.MODE_DYADIC)
+        tmp, y = cdist.atax_rowshard(torch.from_numpy(A).cuda(), torch.from_numpy(x).cuda(),
+                                     k1=catt_mod.Throttle(variant="coop"), k2=catt_mod.Throttle(variant="coop"))
+        q, s = cdist.bicg_rowshard(torch.from_numpy(A).cuda(), torch.from_numpy(x).cuda(), torch.from_numpy(r).cuda(),
+                                   k1=catt_mod.Throttle(variant="staged"), k2=catt_mod.Throttle(variant="staged"))
+        tmp_o, y_o = oracle.atax(A, x)
+        _, y64 = oracle.atax(A, x, mode=oracle.SEQ_F64)
+        q_o, s_o = oracle.bicg(A, x, r)
+        torch.cuda.synchronize()
+        # tmp is exact (dyadic); y multiplies by the derived tmp, so partial sums
+        # exceed 2^24 ulps and the coop order may differ: fp64 bar
+        assert np.array_equal(tmp.cpu().numpy(), tmp_o)
+        assert np.max(np.abs(y.cpu().numpy() - y64) / np.abs(y64)) <= 1e-5
+        assert np.array_equal(q.cpu().numpy(), q_o) and np.array_equal(s.cpu().numpy(), s_o)
+    finally:
+        dist.destroy_process_group()

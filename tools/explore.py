@@ -145,9 +145,27 @@ def atax_big():
         report(f"cols 65536x16384 {var} cta={c}", ms, nbytes)
 
 
+def staged_only():
+    n = 4096
+    A = torch.empty(n, n, device=dev)
+    catt.fill_hash(A, 2)
+    x = torch.rand(n, device=dev)
+    y = torch.empty(n, device=dev)
+    for c in (32, 64):
+        for kind in ("rows", "cols"):
+            t = catt.Throttle(cta_threads=c, variant="staged")
+            f = (lambda: catt.rows(A, x, y, t=t)) if kind == "rows" else (lambda: catt.cols(A, x, y, t=t))
+            report(f"{kind} 4096 staged cta={c}", timeit(f), n * n * 4)
+    for kind in ("rows", "cols"):
+        t = catt.Throttle(variant="coop")
+        f = (lambda: catt.rows(A, x, y, t=t)) if kind == "rows" else (lambda: catt.cols(A, x, y, t=t))
+        report(f"{kind} 4096 coop", timeit(f), n * n * 4)
+
+
 if __name__ == "__main__":
     which = sys.argv[1:] or ["gemv", "kmeans", "syrk", "gesummv", "atax"]
-    fns = dict(gemv=gemv_4096, kmeans=kmeans, syrk=syrk, gesummv=gesummv, atax=atax_big)
+    fns = dict(gemv=gemv_4096, kmeans=kmeans, syrk=syrk, gesummv=gesummv, atax=atax_big,
+               staged=lambda: staged_only())
     for w in which:
         fns[w]()
     json.dump(out, open("gpurun_out/explore.json", "w"), indent=1)
