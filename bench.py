@@ -161,6 +161,7 @@ class Workload:
 
 class BicgMvt(Workload):
     name = "bicg_mvt"
+    variant = "fused"
     desc = "BICG and MVT 4096x4096 fp32 row-per-thread (memory-divergent) on 1 B200 (BASELINE configs[1])"
 
     def __init__(self, catt, torch, rank, world, variant):
@@ -168,6 +169,7 @@ class BicgMvt(Workload):
         import seeded_inputs as si
         n = 4096
         rows = n                                     # rows per rank (weak scaling)
+        self.rows = rows
         dev = torch.device("cuda")
         T = lambda *s: torch.empty(*s, device=dev)
         self.Ab, self.Am = T(rows, n), T(rows, n)
@@ -180,16 +182,32 @@ class BicgMvt(Workload):
         for k, v in enumerate((self.r, self.y2, self.x1)):
             catt.fill_hash(v, si.sub_seed(si.SEED_MVT, k + 1), offset=rank * rows)
         var = self.variant
+        mat = rows * n * 4
+        acc2 = rank == 0                 # x2 = x2 + sum_g A_g^T y2_g: only rank 0 adds the initial x2
+        P = catt.problem
+        if var == "fused":
+            # both loops of each application in one pass over A (A read once)
+            tf = self.plan("bicg fused", P(catt.K_BICG_2, m=rows, n=n), catt.Throttle(variant="fused"))
+            tg = self.plan("mvt fused", P(catt.K_MVT_1, n=n), catt.Throttle(variant="fused"))
+            self.loops = [
+                Loop("bicg fused", lambda: catt.dual(self.Ab, self.p, self.q, self.s, xc=self.r, t=tf),
+                     mat + 4 * 2 * (rows + n), "fused"),
+                Loop("mvt fused", lambda: catt.dual(self.Am, self.y1, self.x1, self.x2, xc=self.y2,
+                                                    row_accumulate=True, col_accumulate=acc2, t=tg),
+                     mat + 4 * (3 * rows + (3 if acc2 else 2) * n), "fused"),
+            ]
+            self.study = dict(name="bicg2 q=A p (literal, row per thread)", prob=P(catt.K_BICG_2, m=rows, n=n),
+                              A=self.Ab, x=self.p, y=self.q,
+                              launches=[(1024, 132), (1024, 196), (1024, 228), (256, 196), (256, 228)])
+            return
         col_var = var if var in ("coop", "staged") else "literal"
         cta_row = {"coop": 256, "staged": 32, "vec4": 32, "literal": 32}[var]
-        cta_col = {"coop": 256, "staged": 32, "literal": 256}[col_var]
+        cta_col = {"coop": 1024, "staged": 32, "literal": 256}[col_var]
         P = catt.problem
         tb1 = self.plan("bicg1 s=A^T r", P(catt.K_BICG_1, m=rows, n=n), catt.Throttle(cta_threads=cta_col, variant=col_var))
         tb2 = self.plan("bicg2 q=A p", P(catt.K_BICG_2, m=rows, n=n), catt.Throttle(cta_threads=cta_row, variant=var))
         tm1 = self.plan("mvt1 x1+=A y1", P(catt.K_MVT_1, n=n), catt.Throttle(cta_threads=cta_row, variant=var))
         tm2 = self.plan("mvt2 x2+=A^T y2", P(catt.K_MVT_2, n=n), catt.Throttle(cta_threads=cta_col, variant=col_var))
-        mat = rows * n * 4
-        acc2 = rank == 0                 # x2 = x2 + sum_g A_g^T y2_g: only rank 0 adds the initial x2
         self.loops = [
             Loop("bicg1 s=A^T r", lambda: catt.cols(self.Ab, self.r, self.s, False, tb1), mat + 4 * (rows + n), "cols"),
             Loop("bicg2 q=A p", lambda: catt.rows(self.Ab, self.p, self.q, catt.ROWS_STORE, t=tb2), mat + 4 * (rows + n),
@@ -208,6 +226,11 @@ class BicgMvt(Workload):
             import torch.distributed as dist
             dist.all_reduce(self.s)
             dist.all_reduce(self.x2)
+
+    def step_bytes(self):
+        n, rows = 4096, self.rows
+        # BICG: A, p, r, q, s; MVT: A, y1, y2, x1 (in/out), x2 (in/out on rank 0)
+        return 2 * rows * n * 4 + 4 * (n + rows + rows + n) + 4 * (n + rows + 2 * rows + 2 * n)
 
     def inputs(self):
         return [self.Ab, self.Am, self.p, self.r, self.y1, self.y2, self.x1, self.x2]
@@ -328,6 +351,7 @@ class Syrk(Workload):
 
 class Atax(Workload):
     name = "atax"
+    variant = "fused"
     desc = "ATAX 65536x16384 fp32 row-sharded with NCCL all-reduce of A^T partials (configs[4])"
 
     def __init__(self, catt, torch, rank, world, variant, m=65536, n=16384):
@@ -343,23 +367,32 @@ class Atax(Workload):
         catt.fill_hash(self.x, si.sub_seed(seed, 1))
         self.tmp, self.y = torch.empty(rows, device=dev), torch.empty(n, device=dev)
         var = self.variant
+        mat = rows * n * 4
+        self.study = dict(name="atax1 tmp=A x (literal, row per thread)", prob=catt.problem(catt.K_ATAX_1, m=rows, n=n),
+                          A=self.A, x=self.x, y=self.tmp, launches=[(1024, 196), (256, 228)])
+        if var == "fused":
+            tf = self.plan("atax fused", catt.problem(catt.K_ATAX_1, m=rows, n=n), catt.Throttle(variant="fused"))
+            self.loops = [Loop("atax fused", lambda: catt.dual(self.A, self.x, self.tmp, self.y, dependent=True, t=tf),
+                               mat + 4 * 2 * (rows + n), "fused")]
+            return
         t1 = self.plan("atax1 tmp=A x", catt.problem(catt.K_ATAX_1, m=rows, n=n),
                        catt.Throttle(cta_threads=256 if var == "coop" else 32, variant=var))
         cv = var if var in ("coop", "staged") else "literal"
         t2 = self.plan("atax2 y=A^T tmp", catt.problem(catt.K_ATAX_2, m=rows, n=n),
-                       catt.Throttle(cta_threads={"coop": 256, "staged": 32, "literal": 256}[cv], variant=cv))
-        mat = rows * n * 4
+                       catt.Throttle(cta_threads={"coop": 1024, "staged": 32, "literal": 256}[cv], variant=cv))
         self.loops = [Loop("atax1 tmp=A x", lambda: catt.rows(self.A, self.x, self.tmp, catt.ROWS_STORE, t=t1),
                            mat + 4 * (rows + n), "rows"),
                       Loop("atax2 y=A^T tmp", lambda: catt.cols(self.A, self.tmp, self.y, False, t2),
                            mat + 4 * (rows + n), "cols")]
-        self.study = dict(name="atax1 tmp=A x (literal, row per thread)", prob=catt.problem(catt.K_ATAX_1, m=rows, n=n),
-                          A=self.A, x=self.x, y=self.tmp, launches=[(1024, 196), (256, 228)])
 
     def collective(self):
         if self.world > 1:
             import torch.distributed as dist
             dist.all_reduce(self.y)
+
+    def step_bytes(self):
+        # A once, x, tmp, y
+        return self.rows * self.n * 4 + 4 * (2 * self.n + self.rows)
 
     def inputs(self):
         return [self.A, self.x]
@@ -571,8 +604,18 @@ def main():
     import paper_conf_icpp_kimhlsh19_b200 as catt
 
     w = WORKLOADS[args.workload](catt, torch, rank, world, args.variant)
-    flush_buf = torch.empty(64 * 1024 * 1024, dtype=torch.int32, device="cuda")    # 256 MiB > 126 MB L2
-    flush = lambda: flush_buf.zero_()
+    # L2 flush between steps: write 256 MiB (> 126 MB L2), then read another
+    # 256 MiB so the lines left in L2 are clean (a write-only flush leaves
+    # ~126 MB of dirty lines whose write-back would land in the timed region)
+    flush_buf = torch.empty(64 * 1024 * 1024, dtype=torch.int32, device="cuda")
+    clean_buf = torch.zeros(64 * 1024 * 1024, dtype=torch.int32, device="cuda")
+
+    def flush():
+        flush_buf.zero_()
+        clean_buf.sum()
+        # keep the GPU busy ~0.2 ms while the host enqueues the timed launches,
+        # so host-side enqueue cost never lands between the CUDA events
+        torch.cuda._sleep(400_000)
     torch.cuda.synchronize()
 
     clocks = ClockSampler(local)
@@ -587,7 +630,9 @@ def main():
         import torch.distributed as dist
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms = float(t.item())
-    step_bytes = sum(lp.nbytes for lp in w.loops)
+    # the step's algorithmic bytes: the minimal traffic of the computation (A
+    # read once per application, vectors once), whatever the variant does
+    step_bytes = w.step_bytes() if hasattr(w, "step_bytes") else sum(lp.nbytes for lp in w.loops)
     total_bytes = step_bytes * world
     value = total_bytes / (ms * 1e-3) / 1e9
 
@@ -654,6 +699,28 @@ def main():
                 "frac": round(ach / peak, 4), "traffic": ncu_traffic(lp.kind),
                 "peak_source": f"{peak_src} (MEASURED_PEAKS.json hbm_gbs)" if peak_src == "measured" else "fallback"}
 
+    # ---- context: a plain device copy moving the same bytes as the dominant
+    # loop, timed the same way (flush, queued events). At 64 MiB a single
+    # kernel cannot reach the 2 GiB copy peak of MEASURED_PEAKS.json.
+    if lp.kind != "syrk":
+        half = max(1, lp.nbytes // 8)                # floats per side: read + write = nbytes
+        src = torch.empty(half, device="cuda")
+        dst = torch.empty(half, device="cuda")
+        cts = []
+        for r in range(6):
+            flush()
+            a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a_.record()
+            dst.copy_(src)
+            b_.record()
+            torch.cuda.synchronize()
+            if r:
+                cts.append(a_.elapsed_time(b_))
+        cgbs = 2 * half * 4 / (statistics.median(cts) * 1e-3) / 1e9
+        roof["same_size_copy_gbs"] = round(cgbs, 1)
+        roof["frac_of_same_size_copy"] = round(roof["achieved"] / cgbs, 4)
+        del src, dst
+
     # ---- CPU oracle baseline (rank 0, N = 1)
     cpu = None
     if rank == 0 and world == 1 and args.cpu_seconds > 0:
@@ -681,7 +748,7 @@ def main():
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded counter hash, generated on device)",
-            "config": {"workload": w.desc, "variant": w.variant, "l2": "flushed before every step (256 MiB write)",
+            "config": {"workload": w.desc, "variant": w.variant, "l2": "flushed before every step (256 MiB write, then 256 MiB clean read)",
                        "rows_per_rank": getattr(w, "rows", None), "parallelism": f"row-shard x{world}"},
             "loops": {lp.name: {"ms": round(loop_ms[i], 5),
                                 "gbs": round(lp.nbytes / (loop_ms[i] * 1e-3) / 1e9, 1),

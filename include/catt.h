@@ -20,9 +20,10 @@
  *   - extern "C", plain pointers and sizes; no exceptions cross the boundary.
  *   - Device pointers are owned by the caller (the Python layer allocates them
  *     with PyTorch). The library never frees caller memory. Its only state is
- *     a per-device cache (hardware table, kernel attributes) and a per-device
- *     array of num_sms int32 counters for the per-SM CTA cap, allocated on
- *     first use and left zero by every kernel that uses it.
+ *     a per-device cache (hardware table, kernel attributes), a per-device
+ *     array of num_sms int32 counters for the per-SM CTA cap plus a grid
+ *     barrier word (allocated on first use, left zero by every kernel that
+ *     uses them), and a grow-only workspace for the FUSED variant's partials.
  *   - Kernel entry points are asynchronous on `stream` (a cudaStream_t passed
  *     as void*; NULL = legacy default stream). Nothing synchronises.
  *   - Arguments are validated synchronously before any launch; invalid input
@@ -152,8 +153,13 @@ typedef struct {
  *   COOP     warp-cooperative coalesced loads with shuffle/split reductions:
  *            the HBM-roofline variant; summation order differs (fp64-oracle
  *            tolerance, bit-exact on exact-dyadic inputs).
- *   REGS     (KMEANS) the point's features are loaded once into registers.  */
-enum { CATT_VAR_LITERAL = 0, CATT_VAR_VEC4 = 1, CATT_VAR_STAGED = 2, CATT_VAR_COOP = 3, CATT_VAR_REGS = 4 };
+ *   REGS     (KMEANS) the point's features are loaded once into registers.
+ *   FUSED    (ATAX/BICG/MVT, set on k1) both loops in one pass over A: each
+ *            row is read once, its dot product finished in the CTA, its A^T
+ *            contribution accumulated; A^T partials reduced in band order
+ *            after a grid barrier (cooperative launch). Same bar as COOP.  */
+enum { CATT_VAR_LITERAL = 0, CATT_VAR_VEC4 = 1, CATT_VAR_STAGED = 2, CATT_VAR_COOP = 3, CATT_VAR_REGS = 4,
+       CATT_VAR_FUSED = 5 };
 
 /* Warp-level mechanism: SEMAPHORE = per-CTA counting semaphore in shared
  * memory (a finished warp's slot goes to the next waiting warp);
@@ -282,6 +288,16 @@ catt_status catt_rows(const float* A, const float* B, const float* x, float* y, 
                       float alpha, float beta, int32_t mode, const catt_throttle* t, void* stream);
 catt_status catt_cols(const float* A, const float* v, float* y, int64_t m, int64_t n, int32_t accumulate,
                       const catt_throttle* t, void* stream);
+
+/* Both loops of an application in one pass over A (the FUSED variant; SURVEY
+ * 8(f) f4): yr (+)= A xr (row loop) and yc (+)= A^T v with v = xc, or v = the
+ * finished yr when `dependent` (ATAX: y = A^T (A x)). row_/col_accumulate make
+ * yr / yc in/out. A is m x n row-major, n % 4 == 0, n <= 16384, 16-B aligned
+ * A and xr. Uses the library's per-device workspace (grid x n floats) and a
+ * cooperative launch; t must not request a throttle (CATT_EINVAL). */
+catt_status catt_dual(const float* A, const float* xr, const float* xc, float* yr, float* yc, int64_t m, int64_t n,
+                      int32_t row_accumulate, int32_t col_accumulate, int32_t dependent, const catt_throttle* t,
+                      void* stream);
 
 /* ------------------------------------------------------------------ helpers */
 /* dst[i] = value(seed, offset + i): the counter-based generator of

@@ -23,13 +23,14 @@ MAX_LOOPS, MAX_CARVEOUTS = 4, 16
 REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
 MODE_UNION, MODE_PAPER = 0, 1
 FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE, FIT_GUARDED = 1, 2, 4, 8, 16
-VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS = 0, 1, 2, 3, 4
+VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED = 0, 1, 2, 3, 4, 5
 ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
 (K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS) = range(9)
 
-VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS}
+VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS,
+            "fused": VAR_FUSED}
 FLAG_NAMES = {FIT_NONE_NEEDED: "none", FIT_WARP: "warp", FIT_CTA: "cta", FIT_UNRESOLVABLE: "unresolvable",
               FIT_NONE_NEEDED | FIT_GUARDED: "none(guard)", FIT_WARP | FIT_GUARDED: "warp(guard)",
               FIT_CTA | FIT_GUARDED: "cta(guard)"}
@@ -155,6 +156,7 @@ def lib():
             "catt_syrk": [V, V, i64, i64, f32, f32, T, V],
             "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
             "catt_rows": [V, V, V, V, V, i64, i64, f32, f32, i32, T, V],
+            "catt_dual": [V, V, V, V, V, i64, i64, i32, i32, i32, T, V],
             "catt_cols": [V, V, V, i64, i64, i32, T, V],
             "catt_fill_hash": [V, i64, u32, u64, i32, V],
             "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
@@ -174,7 +176,7 @@ def lib():
 
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_kmeans_assign",
-            "catt_rows", "catt_cols", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
+            "catt_rows", "catt_cols", "catt_dual", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version"]
 
 
@@ -357,6 +359,16 @@ def cols(A, v, y, accumulate=False, t: Optional[Throttle] = None):
     _check(lib().catt_cols(_dev(A, "A"), _dev(v, "v"), _dev(y, "y"), m, n, int(bool(accumulate)), _tp(t),
                            _stream()), "catt_cols")
     return y
+
+
+def dual(A, xr, yr, yc, xc=None, row_accumulate=False, col_accumulate=False, dependent=False,
+         t: Optional[Throttle] = None):
+    """Both loops in one pass over A (catt_dual): yr (+)= A xr; yc (+)= A^T (yr if dependent else xc)."""
+    m, n = A.shape
+    _check(lib().catt_dual(_dev(A, "A"), _dev(xr, "xr"), _dev(xc, "xc") if xc is not None else None, _dev(yr, "yr"),
+                           _dev(yc, "yc"), m, n, int(bool(row_accumulate)), int(bool(col_accumulate)),
+                           int(bool(dependent)), _tp(t), _stream()), "catt_dual")
+    return yr, yc
 
 
 def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):

@@ -14,6 +14,9 @@ struct DevCtx {
   int device = -1;
   catt_hw hw{};
   int* sm_counter = nullptr;  // hw.num_sms int32, zero between capped launches
+  unsigned* gbar = nullptr;   // grid barrier {count, generation} of the fused kernels (inside the same allocation)
+  float* work = nullptr;      // fused kernels' column partials, grown on demand
+  size_t work_bytes = 0;
 };
 
 // Per-device context of the current device (hardware table, CTA-cap counters).

@@ -1,0 +1,392 @@
+// k_fused.cu — FUSED variant: both loops of BICG / MVT / ATAX in one pass over A.
+//
+// The two loops of each application read the same matrix (ATAX's
+// divergent phase and its coalesced phase; BICG and MVT likewise), so on B200
+// the HBM-bound choice is to read A once:
+//   BICG  q[i]  = sum_j A[i][j] p[j]          s[j]  = sum_i r[i] A[i][j]
+//   MVT   x1[i] = x1[i] + sum_j A[i][j] y1[j]  x2[j] = x2[j] + sum_i A[i][j] y2[i]
+//   ATAX  tmp[i] = sum_j A[i][j] x[j]          y[j]  = sum_i A[i][j] tmp[i]
+// Grid = row bands (one or two CTAs per SM, cooperative launch). A CTA of NW
+// warps covers all columns: warp w owns the 16-byte column chunks
+// w*32 + lane + 32*NW*t (t < T). Rows are streamed U at a time with 16-byte
+// L1-bypassing loads, U*T chunks in flight per lane. For each row the warp
+// partial dots (fixed xor tree) are added in warp order in shared memory; ATAX
+// then uses tmp[i] with the row still in registers, so A is never re-read.
+// Each CTA writes its column partials to a workspace; after a grid barrier the
+// partials are added in band order (deterministic). Results match the
+// sequential oracle within 1e-5 of fp64 and bit-exactly on exact-dyadic input.
+#include <algorithm>
+#include <cstdint>
+#include <cstdlib>
+
+#include <cooperative_groups.h>
+
+#include "internal.h"
+
+namespace catt {
+
+struct FusedArgs {
+  const float* A;
+  const float* xr;   // row-loop vector (p, y1, x)
+  const float* xc;   // column-loop vector (r, y2); ATAX: unused (tmp)
+  float* yr;         // row outputs (q, x1 in/out, tmp)
+  float* yc;         // column outputs (s, x2 in/out, y)
+  float* part;       // workspace: gridDim.x x N column partials
+  unsigned* gbar;    // grid barrier {count, generation}
+  int64_t M, N;
+  int64_t band;      // rows per CTA
+  int row_acc, col_acc;  // yr / yc are in/out (MVT)
+};
+
+__device__ __forceinline__ float4 ld_stream4(const float4* p) {
+  float4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ void grid_barrier(unsigned* bar, unsigned nblocks) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    volatile unsigned* vb = bar;
+    const unsigned gen = vb[1];
+    __threadfence();
+    if (atomicAdd(&bar[0], 1u) == nblocks - 1) {
+      bar[0] = 0;
+      __threadfence();
+      atomicAdd(&bar[1], 1u);
+    } else {
+      while (vb[1] == gen) __nanosleep(64);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+__device__ __forceinline__ uint32_t f_s32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ void f_bar_init(uint64_t* b, uint32_t c) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(f_s32(b)), "r"(c) : "memory");
+}
+__device__ __forceinline__ void f_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(f_s32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void f_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(f_s32(b)) : "memory");
+}
+__device__ __forceinline__ void f_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "LAB_WAIT:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@P1 bra DONE;\n"
+      "bra LAB_WAIT;\n"
+      "DONE:\n"
+      "}\n" ::"r"(f_s32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void f_bulk(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   f_s32(dst)),
+               "l"(src), "r"(bytes), "r"(f_s32(b))
+               : "memory");
+}
+
+// DEP = true: ATAX (the column loop's vector is the row loop's result).
+// NW warps per CTA, T 16-byte chunks per lane per row. A stage holds RPS
+// whole rows (contiguous in memory: one bulk copy), S stages in a ring.
+template <bool DEP, int NW, int T>
+__global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS, int S) {
+  extern __shared__ __align__(1024) unsigned char dyn[];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
+  uint64_t* empty = full + S;
+  float* rowbuf = reinterpret_cast<float*>(dyn + 512);         // [RPS][NW] warp partials
+  float* rowval = rowbuf + RPS * NW;                            // [RPS] finished row values
+  unsigned char* ring = dyn + 1024 + ((RPS * (NW + 1) * 4 + 1023) / 1024) * 1024;
+  const int64_t N = a.N, n4 = N >> 2, M = a.M;
+  const int64_t stage_bytes = int64_t(RPS) * N * 4;
+  const int64_t r0 = int64_t(blockIdx.x) * a.band, r1 = imin64(M, r0 + a.band);
+  const int64_t nst = (r1 - r0 + RPS - 1) / RPS;               // stages of this band
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      f_bar_init(&full[s], 1);
+      f_bar_init(&empty[s], NW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](int64_t c) {                                 // thread 0 only
+    const int s = int(c % S);
+    if (c >= S) f_wait(&empty[s], uint32_t(((c / S) - 1) & 1));
+    const int64_t rows = imin64(RPS, r1 - (r0 + c * RPS));
+    const uint32_t bytes = uint32_t(rows * N * 4);
+    f_expect_tx(&full[s], bytes);
+    f_bulk(ring + int64_t(s) * stage_bytes, a.A + (r0 + c * RPS) * N, bytes, &full[s]);
+  };
+  if (threadIdx.x == 0)
+    for (int64_t c = 0; c < imin64(S, nst); ++c) issue(c);
+  const float4* x4 = reinterpret_cast<const float4*>(a.xr);
+  float4 xr[T], acc[T];
+#pragma unroll
+  for (int t = 0; t < T; ++t) {
+    const int64_t c = warp * 32 + lane + int64_t(32) * NW * t;
+    xr[t] = c < n4 ? x4[c] : make_float4(0.f, 0.f, 0.f, 0.f);
+    acc[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  for (int64_t c = 0; c < nst; ++c) {
+    const int s = int(c % S);
+    const int64_t i0 = r0 + c * RPS;
+    const int rows = int(imin64(RPS, r1 - i0));
+    f_wait(&full[s], uint32_t((c / S) & 1));
+    const float4* st = reinterpret_cast<const float4*>(ring + int64_t(s) * stage_bytes);
+    // row dots: lane partial in chunk order, xor tree, warp partials to smem
+    for (int u = 0; u < rows; ++u) {
+      const float4* row = st + int64_t(u) * n4;
+      float d = 0.0f;
+#pragma unroll
+      for (int t = 0; t < T; ++t) {
+        const int64_t cc = warp * 32 + lane + int64_t(32) * NW * t;
+        if (cc < n4) {
+          const float4 v = row[cc];
+          d = fmaf(v.x, xr[t].x, d);
+          d = fmaf(v.y, xr[t].y, d);
+          d = fmaf(v.z, xr[t].z, d);
+          d = fmaf(v.w, xr[t].w, d);
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+      if (lane == 0) rowbuf[u * NW + warp] = d;
+    }
+    __syncthreads();
+    if (threadIdx.x < rows) {
+      const int u = threadIdx.x;
+      float sum = rowbuf[u * NW];
+      for (int w = 1; w < NW; ++w) sum += rowbuf[u * NW + w];
+      if (a.row_acc) sum = a.yr[i0 + u] + sum;
+      a.yr[i0 + u] = sum;
+      rowval[u] = sum;
+    }
+    __syncthreads();
+    // column partials in row order, the row still in shared memory
+    for (int u = 0; u < rows; ++u) {
+      const float4* row = st + int64_t(u) * n4;
+      const float w = DEP ? rowval[u] : a.xc[i0 + u];
+#pragma unroll
+      for (int t = 0; t < T; ++t) {
+        const int64_t cc = warp * 32 + lane + int64_t(32) * NW * t;
+        if (cc < n4) {
+          const float4 v = row[cc];
+          acc[t].x = fmaf(v.x, w, acc[t].x);
+          acc[t].y = fmaf(v.y, w, acc[t].y);
+          acc[t].z = fmaf(v.z, w, acc[t].z);
+          acc[t].w = fmaf(v.w, w, acc[t].w);
+        }
+      }
+    }
+    __syncwarp();
+    if (lane == 0) f_arrive(&empty[s]);
+    if (threadIdx.x == 0 && c + S < nst) issue(c + S);
+  }
+  // column partials: first summed over the CL CTAs of this cluster through
+  // distributed shared memory (rank order), so only G / CL partial vectors go
+  // through global memory and the grid barrier
+  namespace cg = cooperative_groups;
+  cg::cluster_group cluster = cg::this_cluster();
+  const int CL = int(cluster.num_blocks()), rank = int(cluster.block_rank());
+  const int64_t cid = int64_t(blockIdx.x) / CL;
+  float* cpart = reinterpret_cast<float*>(ring);               // the ring is drained: reuse it
+  {
+    float4* c4 = reinterpret_cast<float4*>(cpart);
+#pragma unroll
+    for (int t = 0; t < T; ++t) {
+      const int64_t cc = warp * 32 + lane + int64_t(32) * NW * t;
+      if (cc < n4) c4[cc] = acc[t];
+    }
+  }
+  cluster.sync();
+  {
+    const int64_t per = (N + CL - 1) / CL;
+    const int64_t j0 = rank * per, j1 = imin64(N, j0 + per);
+    for (int64_t j = j0 + threadIdx.x; j < j1; j += blockDim.x) {
+      float sum = cluster.map_shared_rank(cpart, 0)[j];
+      for (int q = 1; q < CL; ++q) sum += cluster.map_shared_rank(cpart, q)[j];
+      a.part[cid * N + j] = sum;
+    }
+  }
+  cluster.sync();
+  __threadfence();
+  grid_barrier(a.gbar, gridDim.x);
+  // column outputs: a fixed tree over the G band partials. CTA b owns the
+  // 32-column chunks b, b + G, ...; warp w sums bands [w*gpw, (w+1)*gpw) in
+  // order (independent loads in flight), then the NW warp sums are added in
+  // warp order, then the initial value (MVT) is added.
+  {
+    __shared__ float red[NW][32];
+    const int64_t G = gridDim.x / CL;                          // partial vectors (one per cluster)
+    const int64_t gpw = (G + NW - 1) / NW;
+    const int64_t b0 = warp * gpw, b1 = imin64(G, b0 + gpw);
+    for (int64_t ch = blockIdx.x; ch * 32 < N; ch += gridDim.x) {
+      const int64_t j = ch * 32 + lane;
+      float sum = 0.0f;
+      if (j < N) {
+        int64_t b = b0;
+        for (; b + 8 <= b1; b += 8) {
+          float v[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) v[k] = a.part[(b + k) * N + j];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) sum += v[k];
+        }
+        for (; b < b1; ++b) sum += a.part[b * N + j];
+      }
+      red[warp][lane] = sum;
+      __syncthreads();
+      if (warp == 0 && j < N) {
+        float tot = red[0][lane];
+        for (int w = 1; w < NW; ++w) tot += red[w][lane];
+        if (a.col_acc) tot = a.yc[j] + tot;
+        a.yc[j] = tot;
+      }
+      __syncthreads();
+    }
+  }
+}
+
+
+namespace {
+
+template <bool DEP>
+const void* fused_fn(int NW, int T) {
+  if (NW == 16) {
+    if (T == 2) return (const void*)fused_kernel<DEP, 16, 2>;
+    if (T == 4) return (const void*)fused_kernel<DEP, 16, 4>;
+    return (const void*)fused_kernel<DEP, 16, 8>;
+  }
+  if (T == 1) return (const void*)fused_kernel<DEP, 8, 1>;
+  return (const void*)fused_kernel<DEP, 8, 2>;
+}
+
+}  // namespace
+
+// Workspace (column partials) owned by the device context; grown on demand.
+catt_status dev_workspace(size_t bytes, float** out, unsigned** gbar);
+
+catt_status launch_fused(bool dep, const float* A, const float* xr, const float* xc, float* yr, float* yc, int64_t M,
+                         int64_t N, int row_acc, int col_acc, const catt_throttle* t, cudaStream_t s) {
+  if (M == 0 || N == 0) return CATT_EINVAL;  // callers route empty shapes to the per-loop path
+  if (N % 4 || (reinterpret_cast<uintptr_t>(A) & 15u) || (reinterpret_cast<uintptr_t>(xr) & 15u)) return CATT_EINVAL;
+  if (t && (t->active_warps || t->active_ctas)) return CATT_EINVAL;  // nothing to throttle (no L1 reuse)
+  const int64_t n4 = N / 4;
+  // 8 warps for short rows (T <= 2 chunks per lane), else 16 warps with
+  // T = 2, 4 or 8 chunks per lane (N <= 16384)
+  const int NW = n4 <= 512 ? 8 : 16;
+  const int64_t T64 = (n4 + 32 * NW - 1) / (32 * NW);
+  if (T64 > 8) return CATT_EUNSUPPORTED;  // N > 16384
+  const int T = T64 <= 1 ? 1 : (T64 <= 2 ? 2 : (T64 <= 4 ? 4 : 8));
+  const int threads = NW * 32;
+  const void* f = dep ? fused_fn<true>(NW, T) : fused_fn<false>(NW, T);
+  // stage = RPS whole rows (~64 KB: several independent row chains per warp
+  // and few barriers per byte), S stages within ~200 KB of shared memory
+  const int64_t row_bytes = N * 4;
+  const char* rps_env = getenv("CATT_FUSED_STAGE_KB");
+  const int64_t stage_target = (rps_env ? atoi(rps_env) : 64) * 1024;
+  const int RPS = int(std::max<int64_t>(1, std::min<int64_t>(16, stage_target / row_bytes)));
+  const int64_t head = 1024 + ((int64_t(RPS) * (NW + 1) * 4 + 1023) / 1024) * 1024;
+  const int S = int(std::min<int64_t>(16, (200 * 1024 - head) / (RPS * row_bytes)));
+  if (S < 2) return CATT_EUNSUPPORTED;
+  const size_t smem = size_t(head + int64_t(S) * RPS * row_bytes);
+  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f, threads, smem);
+  if (e != cudaSuccess || occ < 1) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  DevCtx* ctx = nullptr;
+  catt_status st = dev_ctx(&ctx);
+  if (st != CATT_OK) return st;
+  // cluster of CL CTAs for the DSMEM pre-reduction. Clusters live inside a
+  // GPC, so fewer CTAs are co-resident for larger CL: take the largest CL
+  // whose co-resident grid still covers >= 95% of the SMs x occupancy.
+  const char* cl_env = getenv("CATT_FUSED_CLUSTER");
+  const int64_t full_grid = std::min<int64_t>(int64_t(ctx->hw.num_sms) * occ, M);
+  int CL = 1;
+  int64_t G = full_grid;
+  for (int cand = cl_env ? atoi(cl_env) : 8; cand >= 2; cand /= 2) {
+    if (S * RPS * row_bytes < N * 4) break;                    // ring must hold a partial vector
+    cudaLaunchConfig_t qc = {};
+    qc.gridDim = dim3(unsigned(full_grid / cand * cand), 1, 1);
+    qc.blockDim = dim3(unsigned(threads), 1, 1);
+    qc.dynamicSmemBytes = smem;
+    cudaLaunchAttribute qa[1];
+    qa[0].id = cudaLaunchAttributeClusterDimension;
+    qa[0].val.clusterDim.x = unsigned(cand);
+    qa[0].val.clusterDim.y = 1;
+    qa[0].val.clusterDim.z = 1;
+    qc.attrs = qa;
+    qc.numAttrs = 1;
+    int nclusters = 0;
+    if (cudaOccupancyMaxActiveClusters(&nclusters, f, &qc) != cudaSuccess) {
+      cudaGetLastError();
+      continue;
+    }
+    const int64_t g = std::min<int64_t>(int64_t(nclusters) * cand, full_grid / cand * cand);
+    if (g >= 2 * cand && g * 100 >= full_grid * 95) {
+      CL = cand;
+      G = g;
+      break;
+    }
+  }
+  const int64_t band = (M + G - 1) / G;
+  // trailing CTAs may get no rows; they still take part in the reductions
+  float* part = nullptr;
+  unsigned* gbar = nullptr;
+  st = dev_workspace(size_t(G / CL) * size_t(N) * sizeof(float), &part, &gbar);
+  if (st != CATT_OK) return st;
+  FusedArgs args{A, xr, xc, yr, yc, part, gbar, M, N, band, row_acc, col_acc};
+  int rps = RPS, stages = S;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(unsigned(G), 1, 1);
+  cfg.blockDim = dim3(unsigned(threads), 1, 1);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  attr[1].id = cudaLaunchAttributeClusterDimension;
+  attr[1].val.clusterDim.x = unsigned(CL);
+  attr[1].val.clusterDim.y = 1;
+  attr[1].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 2;
+  void* params[] = {&args, &rps, &stages};
+  e = cudaLaunchKernelExC(&cfg, f, params);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  return after_launch();
+}
+
+const void* fused_func(bool dep) { return dep ? fused_fn<true>(16, 2) : fused_fn<false>(16, 2); }
+
+}  // namespace catt
+
+using namespace catt;
+
+extern "C" catt_status catt_dual(const float* A, const float* xr, const float* xc, float* yr, float* yc, int64_t m,
+                                 int64_t n, int32_t row_accumulate, int32_t col_accumulate, int32_t dependent,
+                                 const catt_throttle* t, void* stream) {
+  if (m < 1 || n < 1 || !A || !xr || !yr || !yc || (!dependent && !xc)) return CATT_EINVAL;
+  if (dependent && row_accumulate) return CATT_EINVAL;
+  return launch_fused(dependent != 0, A, xr, xc, yr, yc, m, n, row_accumulate != 0, col_accumulate != 0, t,
+                      static_cast<cudaStream_t>(stream));
+}

@@ -14,6 +14,7 @@
 // shared-memory reductions (the HBM-roofline variant).
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 #include <cooperative_groups.h>
 
@@ -475,9 +476,13 @@ catt_status launch_col_t(ColArgs a, const catt_throttle* t, cudaStream_t s) {
     return after_launch();
   }
   if (var == CATT_VAR_COOP) {
+    // The cluster/DSMEM form measured slower than the 1024-thread CTA per
+    // 32-column block on B200 (profiles/round1_explore_*.txt); kept for
+    // CATT_COOP_CLUSTER=1 experiments only.
     const bool vec = (a.N % 4 == 0) && aligned16(a.A) && aligned16(a.y);
     const bool capped = t && t->active_ctas > 0;
-    if (vec && !capped) {
+    const char* want_cluster = getenv("CATT_COOP_CLUSTER");
+    if (vec && !capped && want_cluster && want_cluster[0] == '1') {
       if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
       const void* f = (const void*)col_cluster_kernel<EPI>;
       size_t dyn = 0;
@@ -555,9 +560,7 @@ const void* gemv_func(int loop, int variant, bool vec_ok) {
   const bool acc = loop == CATT_K_MVT_2;
   if (variant == CATT_VAR_STAGED) return col_tma_func();
   if (variant == CATT_VAR_VEC4) return acc ? (const void*)col_thread_kernel<EPI_ACCUM, true> : (const void*)col_thread_kernel<EPI_STORE, true>;
-  if (variant == CATT_VAR_COOP)
-    return vec_ok ? (acc ? (const void*)col_cluster_kernel<EPI_ACCUM> : (const void*)col_cluster_kernel<EPI_STORE>)
-                  : (acc ? (const void*)col_warp_kernel<EPI_ACCUM> : (const void*)col_warp_kernel<EPI_STORE>);
+  if (variant == CATT_VAR_COOP) return acc ? (const void*)col_warp_kernel<EPI_ACCUM> : (const void*)col_warp_kernel<EPI_STORE>;
   return acc ? (const void*)col_thread_kernel<EPI_ACCUM, false> : (const void*)col_thread_kernel<EPI_STORE, false>;
 }
 
@@ -576,7 +579,22 @@ catt_status launch_col(const float* A, const float* v, float* y, int64_t M, int6
   return launch_col_t<EPI_STORE>(a, t, s);
 }
 
+catt_status launch_fused(bool dep, const float* A, const float* xr, const float* xc, float* yr, float* yc, int64_t M,
+                         int64_t N, int row_acc, int col_acc, const catt_throttle* t, cudaStream_t s);
+
 }  // namespace catt
+
+namespace {
+bool fused(const catt_throttle* k1, int64_t m, int64_t n) {
+  return k1 && k1->variant == CATT_VAR_FUSED && m > 0 && n > 0;
+}
+catt_throttle coop_of(const catt_throttle* t) {
+  catt_throttle c{};
+  c.variant = CATT_VAR_COOP;
+  (void)t;
+  return c;
+}
+}  // namespace
 
 using namespace catt;
 
@@ -585,6 +603,12 @@ extern "C" catt_status catt_atax(const float* A, const float* x, float* tmp, flo
   if (check_common(m, n) != CATT_OK || (m * n > 0 && !A) || (n > 0 && (!x || !y)) || (m > 0 && !tmp))
     return CATT_EINVAL;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (fused(k1, m, n)) return launch_fused(true, A, x, nullptr, tmp, y, m, n, 0, 0, k1, s);
+  if (k1 && k1->variant == CATT_VAR_FUSED) {   // empty shapes: the per-loop path
+    const catt_throttle c = coop_of(k1);
+    catt_status st0 = launch_row(A, nullptr, x, tmp, nullptr, m, n, 0.f, 0.f, EPI_STORE, &c, s);
+    return st0 != CATT_OK ? st0 : launch_col(A, tmp, y, m, n, EPI_STORE, &c, s);
+  }
   catt_status st = launch_row(A, nullptr, x, tmp, nullptr, m, n, 0.f, 0.f, EPI_STORE, k1, s);  // tmp = A x
   if (st != CATT_OK) return st;
   return launch_col(A, tmp, y, m, n, EPI_STORE, k2, s);                                        // y = A^T tmp
@@ -597,6 +621,12 @@ extern "C" catt_status catt_bicg(const float* A, const float* p, const float* r,
       (nx > 0 && (!r || !q)))
     return CATT_EINVAL;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (fused(k1, nx, ny)) return launch_fused(false, A, p, r, q, s_out, nx, ny, 0, 0, k1, s);
+  if (k1 && k1->variant == CATT_VAR_FUSED) {
+    const catt_throttle c = coop_of(k1);
+    catt_status st0 = launch_col(A, r, s_out, nx, ny, EPI_STORE, &c, s);
+    return st0 != CATT_OK ? st0 : launch_row(A, nullptr, p, q, nullptr, nx, ny, 0.f, 0.f, EPI_STORE, &c, s);
+  }
   catt_status st = launch_col(A, r, s_out, nx, ny, EPI_STORE, k1, s);                          // s = A^T r
   if (st != CATT_OK) return st;
   return launch_row(A, nullptr, p, q, nullptr, nx, ny, 0.f, 0.f, EPI_STORE, k2, s);          // q = A p
@@ -606,6 +636,7 @@ extern "C" catt_status catt_mvt(const float* A, const float* y1, const float* y2
                                 const catt_throttle* k1, const catt_throttle* k2, void* stream) {
   if (check_common(n, n) != CATT_OK || (n > 0 && (!A || !y1 || !y2 || !x1 || !x2))) return CATT_EINVAL;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (fused(k1, n, n)) return launch_fused(false, A, y1, y2, x1, x2, n, n, 1, 1, k1, s);
   catt_status st = launch_row(A, nullptr, y1, x1, nullptr, n, n, 0.f, 0.f, EPI_ACCUM, k1, s);   // x1 += A y1
   if (st != CATT_OK) return st;
   return launch_col(A, y2, x2, n, n, EPI_ACCUM, k2, s);                                        // x2 += A^T y2

@@ -17,6 +17,7 @@ int row_tma_stage_bytes(int nmat, int rows, int boxes);
 int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
 const void* kmeans_func(int variant, int nf);
+const void* fused_func(bool dep);
 
 namespace {
 std::mutex g_mu;
@@ -59,9 +60,33 @@ catt_status dev_ctx(DevCtx** out) {
       return CATT_ECUDA;
     }
     c.sm_counter = static_cast<int*>(p);
+    c.gbar = reinterpret_cast<unsigned*>(static_cast<char*>(p) + ((size_t(c.hw.num_sms) * sizeof(int) + 127) / 128) * 128);
     c.device = dev;
   }
   *out = &c;
+  return CATT_OK;
+}
+
+catt_status dev_workspace(size_t bytes, float** out, unsigned** gbar) {
+  DevCtx* c = nullptr;
+  catt_status st = dev_ctx(&c);
+  if (st != CATT_OK) return st;
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (c->work_bytes < bytes) {
+    if (c->work) cudaFree(c->work);
+    c->work = nullptr;
+    c->work_bytes = 0;
+    void* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess) {
+      record_cuda_error(e);
+      return CATT_ENOMEM;
+    }
+    c->work = static_cast<float*>(p);
+    c->work_bytes = bytes;
+  }
+  *out = c->work;
+  *gbar = c->gbar;
   return CATT_OK;
 }
 
@@ -190,6 +215,7 @@ catt_ref mkref(int64_t cx, int64_t cy, int64_t c0, int64_t c1, int32_t e, int32_
 
 int default_threads(int loop, int variant) {
   if (variant == CATT_VAR_STAGED) return loop == CATT_K_SYRK ? 256 : 32;
+  if (variant == CATT_VAR_COOP && (loop == CATT_K_ATAX_2 || loop == CATT_K_BICG_1 || loop == CATT_K_MVT_2)) return 1024;
   return 256;
 }
 
@@ -199,6 +225,7 @@ bool is_row(int loop) {
 bool is_col(int loop) { return loop == CATT_K_ATAX_2 || loop == CATT_K_BICG_1 || loop == CATT_K_MVT_2; }
 
 const void* loop_func(const catt_problem& p, int variant) {
+  if (variant == CATT_VAR_FUSED && (is_row(p.loop) || is_col(p.loop))) return fused_func(p.loop == CATT_K_ATAX_1 || p.loop == CATT_K_ATAX_2);
   if (is_row(p.loop) || is_col(p.loop)) return gemv_func(p.loop, variant, true);
   if (p.loop == CATT_K_SYRK) return syrk_func(variant);
   return kmeans_func(variant, int(p.n));
@@ -273,7 +300,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       const int nmat = two ? 2 : 1;
       const int boxes = std::max(1, std::min(8, 16384 / (nmat * threads * 128)));
       dyn = 1024 + int64_t(row_tma_stages(nmat, threads, boxes)) * row_tma_stage_bytes(nmat, threads, boxes);
-    } else if (var == CATT_VAR_COOP) {
+    } else if (var == CATT_VAR_COOP || var == CATT_VAR_FUSED) {
       // warp per row: lane = gid_x (block 32 x W), row = gid_y
       const int64_t C4 = (N % 4 == 0) ? N / 4 : N;
       const int32_t e = (N % 4 == 0) ? 16 : 4;
@@ -307,7 +334,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->trip[0] = M;
       out->grid[0] = (N / 4 + threads - 1) / threads;
       out->extent[0] = N / 4;
-    } else if (var == CATT_VAR_COOP) {
+    } else if (var == CATT_VAR_COOP || var == CATT_VAR_FUSED) {
       const int NW = threads / 32;
       out->block[0] = 32;
       out->block[1] = NW;

@@ -366,3 +366,63 @@ def test_plan_on_device_matches_occupancy_api():
         assert d.regs_per_thread == regs and regs <= 32      # full TLP is not register-limited
         t, r = catt.plan(prob, launch, hw)
         assert r["base_ctas"] == 8
+
+
+# ------------------------------------------------------------------ FUSED (both loops in one pass)
+FUSED_SHAPES = [(33, 4), (300, 64), (1000, 132), (257, 4096), (700, 8192), (130, 16384)]   # NW = 8, 16, 32
+
+
+@pytest.mark.parametrize("m,n", FUSED_SHAPES)
+def test_fused_bicg_mvt_atax(m, n):
+    A, p, r = si.matrix(2, m, n), si.values(102, n), si.values(202, m)
+    q64, s64 = oracle.bicg(A, p, r, mode=oracle.SEQ_F64)
+    q, s = catt.bicg(dev(A), dev(p), dev(r), k1=catt.Throttle(variant="fused"))
+    assert relerr(host(q), q64) <= TOL and relerr(host(s), s64) <= TOL
+    # dyadic: every partial sum exact -> bit-exact to the sequential oracle
+    D = si.MODE_DYADIC
+    Ad, pd, rd = si.matrix(3, m, n, D), si.values(4, n, mode=D), si.values(5, m, mode=D)
+    qo, so = oracle.bicg(Ad, pd, rd)
+    q, s = catt.bicg(dev(Ad), dev(pd), dev(rd), k1=catt.Throttle(variant="fused"))
+    assert bits_equal(host(q), qo) and bits_equal(host(s), so)
+    # ATAX (dependent: y uses the finished tmp)
+    x = si.values(101, n)
+    t64, y64 = oracle.atax(A, x, mode=oracle.SEQ_F64)
+    tmp, y = catt.atax(dev(A), dev(x), k1=catt.Throttle(variant="fused"))
+    assert relerr(host(tmp), t64) <= TOL and relerr(host(y), y64) <= TOL
+
+
+@pytest.mark.parametrize("n", [64, 1024, 4096])
+def test_fused_mvt_inout(n):
+    a = si.matrix(3, n, n)
+    y1, y2, x1, x2 = (si.values(103 + 100 * k, n) for k in range(4))
+    e1, e2 = oracle.mvt(a, y1, y2, x1, x2, mode=oracle.SEQ_F64)
+    X1, X2 = dev(x1), dev(x2)
+    catt.mvt(dev(a), dev(y1), dev(y2), X1, X2, k1=catt.Throttle(variant="fused"))
+    assert relerr(host(X1), e1) <= TOL and relerr(host(X2), e2) <= TOL
+
+
+def test_dual_flags_and_errors():
+    m, n = 500, 256
+    A, xr, xc = si.matrix(7, m, n), si.values(8, n), si.values(9, m)
+    yr0, yc0 = si.values(10, m), si.values(11, n)
+    YR, YC = dev(yr0), dev(yc0)
+    catt.dual(dev(A), dev(xr), YR, YC, xc=dev(xc), row_accumulate=True, col_accumulate=False)
+    _, s64 = oracle.bicg(A, xr, xc, mode=oracle.SEQ_F64)
+    assert relerr(host(YC), s64) <= TOL
+    q64 = yr0.astype(np.float64) + A.astype(np.float64) @ xr.astype(np.float64)
+    assert relerr(host(YR), q64) <= TOL
+    with pytest.raises(catt.CattError):
+        catt.dual(dev(A), dev(xr), YR, YC, xc=dev(xc), t=catt.Throttle(active_warps=2))     # nothing to throttle
+    with pytest.raises(catt.CattError):
+        catt.dual(dev(A), dev(xr), YR, YC, row_accumulate=True, dependent=True)
+
+
+def test_fused_atax_65536x16384_sampled():
+    m, n = 65536, 16384
+    A = torch.empty(m * n, device="cuda")
+    catt.fill_hash(A, si.SEED_ATAX_SHARDED)
+    x = si.values(si.sub_seed(si.SEED_ATAX_SHARDED, 1), n)
+    cols = np.array([0, 1, 31, 32, 4097, 16383])
+    t64, y64 = oracle.atax_hashed(si.SEED_ATAX_SHARDED, 0, x, m, n, cols, mode=oracle.SEQ_F64)
+    tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="fused"))
+    assert relerr(host(tmp), t64) <= TOL and relerr(host(y)[cols], y64) <= TOL
