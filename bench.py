@@ -547,7 +547,8 @@ def run_reference(args):
             host[nm] = oracle.fill(si.sub_seed(si.SEED_MVT, k + 1), n)
         step = lambda: (oracle.bicg(host["Ab"], host["p"], host["r"]),
                         oracle.mvt(host["Am"], host["y1"], host["y2"], host["x1"], host["x2"]))
-        nbytes = 4 * (n * n * 4) + 4 * 12 * n
+        # the same minimal-bytes definition as the GPU arm (A once per application)
+        nbytes = 2 * n * n * 4 + 4 * (4 * n) + 4 * (6 * n)
         cfg = BicgMvt.desc
         sample = "the full BICG+MVT 4096^2 step (4 loop nests) per step"
     elif wl == "kmeans":

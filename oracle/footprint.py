@@ -24,11 +24,12 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
   a5  Eq 9 (order P:357 + P:371): N over the divisors of
       #Warps_TB (ascending, R6) first; then TB-level, M = 1 .. #TB_SM-1 with
       one warp per TB (R7); give up (CORR) if nothing fits.
-      B200 guards (union mode only, R18; hw keys min_warps_sm and
-      divergent_lines, 0 = off): no throttle unless a reused reference touches
-      at least divergent_lines lines per warp request (the memory divergence
-      of P:32); no candidate below min_warps_sm active warps per SM, and if
-      none at or above it fits, the most throttled one that respects it.
+      B200 rule (union mode with hw keys min_warps_sm / divergent_lines set,
+      R18, R19): no throttle unless a reused reference touches at least
+      divergent_lines lines per warp request (the memory divergence of P:32);
+      every (a, m) pair by active warps per SM descending, ties -> fewer CTAs
+      of more warps (a per-SM cap is cheap on B200); none below min_warps_sm;
+      if none at or above it fits, the most throttled one that respects it.
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -322,33 +323,39 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
 
     if M.fits(full) or not M.locality:
         return done(W, T, full, FIT_NONE_NEEDED)
-    floor_w = 0 if M.paper else hw.get("min_warps_sm", 0)
-    if not M.paper and not M.divergent:
-        return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
-    last = None
-    stopped = False
+    guards = not M.paper and (hw.get("min_warps_sm", 0) > 0 or hw.get("divergent_lines", 0) > 0)
+    if guards:
+        # B200 rule (R18, R19): memory-divergent loops only; all (a, m) with a | W,
+        # m <= T, by warps per SM descending, ties -> larger a (fewer CTAs);
+        # not below min_warps_sm; else the most throttled pair that respects it
+        if not M.divergent:
+            return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
+        floor_w = hw.get("min_warps_sm", 0)
+        cands = [(a, m) for a in range(W, 0, -1) if W % a == 0 for m in range(T, 0, -1)
+                 if (a, m) != (W, T) and a * m >= floor_w]
+        cands.sort(key=lambda am: (-am[0] * am[1], -am[0]))
+
+        def flag(a, m):
+            return (FIT_WARP if a < W else 0) | (FIT_CTA if m < T else 0)
+
+        for a, m in cands:
+            f = M.F(a, m)
+            if M.fits(f):
+                return done(a, m, f, flag(a, m))
+        if not cands:
+            return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
+        least = min(a * m for a, m in cands)
+        a, m = max((am for am in cands if am[0] * am[1] == least), key=lambda am: am[0])
+        return done(a, m, M.F(a, m), flag(a, m) | FIT_GUARDED)
     for N in range(2, W + 1):                     # Eq 9, warp level first
         if W % N:
             continue
         a = W // N
-        if a * T < floor_w:
-            stopped = True
-            break
         f = M.F(a, T)
         if M.fits(f):
             return done(a, T, f, FIT_WARP)
-        last = (a, T, FIT_WARP)
-    if not stopped:
-        for m in range(T - 1, 0, -1):             # then TB level with one warp per TB
-            if m < floor_w:
-                break
-            f = M.F(1, m)
-            if M.fits(f):
-                return done(1, m, f, FIT_CTA)
-            last = (1, m, FIT_CTA)
-    if floor_w > 0:
-        if last is None:
-            return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
-        a, m, fl = last
-        return done(a, m, M.F(a, m), fl | FIT_GUARDED)
+    for m in range(T - 1, 0, -1):                 # then TB level with one warp per TB
+        f = M.F(1, m)
+        if M.fits(f):
+            return done(1, m, f, FIT_CTA)
     return done(W, T, full, FIT_UNRESOLVABLE)     # P:244, P:395 (CORR): leave as is

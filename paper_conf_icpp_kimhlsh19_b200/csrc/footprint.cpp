@@ -358,32 +358,48 @@ extern "C" catt_status catt_footprint(const catt_loop_desc* desc, const catt_hw*
   };
   if (M.fits(full) || !M.locality_) return done(W, T, full, CATT_FIT_NONE_NEEDED);
   const bool paper = desc->mode == CATT_MODE_PAPER;
-  const int32_t floor_w = paper ? 0 : std::max(0, hw->min_warps_sm);
-  if (!paper && !M.divergent_) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
-  int32_t la = -1, lm = -1, lflag = 0;                  // most throttled candidate above the floor
-  bool stopped = false;
-  for (int32_t N = 2; N <= W && !stopped; ++N) {        // Eq 9: warp level first
-    if (W % N) continue;
-    if ((W / N) * T < floor_w) {
-      stopped = true;
-      break;
+  const bool guards = !paper && (hw->min_warps_sm > 0 || hw->divergent_lines > 0);
+  if (guards) {
+    // B200 rule (R18, R19): only memory-divergent loops; every (a, m) pair
+    // with a | W, m <= T, by active warps per SM descending, ties -> fewer
+    // CTAs with more warps each; never below min_warps_sm; if nothing at or
+    // above the floor fits, the most throttled pair that respects it.
+    if (!M.divergent_) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
+    const int32_t floor_w = std::max(0, hw->min_warps_sm);
+    std::vector<std::pair<int32_t, int32_t>> cands;
+    for (int32_t a = W; a >= 1; --a) {
+      if (W % a) continue;
+      for (int32_t m = T; m >= 1; --m)
+        if (!(a == W && m == T) && a * m >= floor_w) cands.push_back({a, m});
     }
+    std::stable_sort(cands.begin(), cands.end(), [](const std::pair<int32_t, int32_t>& x,
+                                                    const std::pair<int32_t, int32_t>& y) {
+      if (x.first * x.second != y.first * y.second) return x.first * x.second > y.first * y.second;
+      return x.first > y.first;
+    });
+    auto flag_of = [&](int32_t a, int32_t m) {
+      return (a < W ? CATT_FIT_WARP : 0) | (m < T ? CATT_FIT_CTA : 0);
+    };
+    for (const auto& c2 : cands) {
+      const int64_t f = M.F(c2.first, c2.second);
+      if (M.fits(f)) return done(c2.first, c2.second, f, flag_of(c2.first, c2.second));
+    }
+    if (cands.empty()) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
+    // most throttled allowed: fewest warps, then the largest a among those
+    std::pair<int32_t, int32_t> last = cands.back();
+    for (const auto& c2 : cands)
+      if (c2.first * c2.second == last.first * last.second && c2.first > last.first) last = c2;
+    return done(last.first, last.second, M.F(last.first, last.second),
+                flag_of(last.first, last.second) | CATT_FIT_GUARDED);
+  }
+  for (int32_t N = 2; N <= W; ++N) {                     // Eq 9: warp level first
+    if (W % N) continue;
     const int64_t f = M.F(W / N, T);
     if (M.fits(f)) return done(W / N, T, f, CATT_FIT_WARP);
-    la = W / N, lm = T, lflag = CATT_FIT_WARP;
   }
-  for (int32_t m = T - 1; m >= 1 && !stopped; --m) {    // then TB level, one warp per TB
-    if (m < floor_w) {
-      stopped = true;
-      break;
-    }
+  for (int32_t m = T - 1; m >= 1; --m) {                 // then TB level, one warp per TB
     const int64_t f = M.F(1, m);
     if (M.fits(f)) return done(1, m, f, CATT_FIT_CTA);
-    la = 1, lm = m, lflag = CATT_FIT_CTA;
-  }
-  if (floor_w > 0) {
-    if (la < 0) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
-    return done(la, lm, M.F(la, lm), lflag | CATT_FIT_GUARDED);
   }
   return done(W, T, full, CATT_FIT_UNRESOLVABLE);
 }
@@ -422,10 +438,11 @@ extern "C" catt_status catt_hw_b200(catt_hw* out) {
   out->smem_alloc_unit = 128;
   out->reserved_smem_cta = 1024;   // cudaDevAttrReservedSharedMemoryPerBlock
   out->line_bytes = 128;
-  // B200 guards (reading R18, profiles/round1_ncu_cases_a_raw.csv): 4 warps per
-  // SM sub-partition to hide L2 latency; a request must touch >= 8 lines for
-  // its misses to cost more than the TLP a throttle gives up.
-  out->min_warps_sm = 16;
+  // B200 rule (readings R18, R19): a request must touch >= 8 lines for its
+  // misses to cost more than the TLP a throttle gives up (ncu study,
+  // profiles/round1_ncu_cases_a_raw.csv); at least 8 active warps per SM (2 per
+  // sub-partition), calibrated on the swept launches of profiles/r1/.
+  out->min_warps_sm = 8;
   out->divergent_lines = 8;
   // Shared-memory options (KB) and the carveout percentage that selects each
   // (percent of the 228 KB maximum; the driver rounds up to the next option).

@@ -320,7 +320,9 @@ catt_status launch_fused(bool dep, const float* A, const float* xr, const float*
   const int64_t full_grid = std::min<int64_t>(int64_t(ctx->hw.num_sms) * occ, M);
   int CL = 1;
   int64_t G = full_grid;
-  for (int cand = cl_env ? atoi(cl_env) : 8; cand >= 2; cand /= 2) {
+  // default 1: the DSMEM pre-reduction measured no gain at 4096^2 and the
+  // clustered cooperative launch cannot be replayed by ncu
+  for (int cand = cl_env ? atoi(cl_env) : 1; cand >= 2; cand /= 2) {
     if (S * RPS * row_bytes < N * 4) break;                    // ring must hold a partial vector
     cudaLaunchConfig_t qc = {};
     qc.gridDim = dim3(unsigned(full_grid / cand * cand), 1, 1);
