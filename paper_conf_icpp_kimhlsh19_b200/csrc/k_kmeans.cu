@@ -10,8 +10,15 @@
 // until the next centre (outer-loop reuse, reading R10). At 494020 points and
 // 64 warps per SM this exceeds the L1D at every carveout on B200 (SURVEY 0
 // finding 3): the contended configuration where CATT throttles.
-// REGS: the point's features are read once into registers (same arithmetic
-// order, bit-identical membership); no L1 reuse is needed.
+// REGS: the features are streamed once (16 B-per-warp-lane loads that do not
+// allocate in L1) while the k partial distances of the point stay in
+// registers: for f: v = feat[f*ld + p]; for c: d[c] = fmaf(v - C[c][f], ...).
+// Every (point, centre) pair still accumulates f = 0, 1, ... in order, so the
+// membership is bit-identical to LITERAL; no L1 reuse is needed.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
 #include <cfloat>
 #include <cstdint>
 
@@ -28,11 +35,9 @@ struct KmArgs {
   Throttle t;
 };
 
-constexpr int kMaxRegsFeatures = 64;
-
-// MAXF = 0: LITERAL; MAXF > 0: REGS with up to MAXF features in registers
+// MAXF = 0: LITERAL (the only instance; REGS is kmeans_stream_kernel below)
 template <int MAXF>
-__global__ void __launch_bounds__(MAXF == 0 ? 1024 : 256, MAXF == 0 ? 2 : (MAXF <= 40 ? 2 : 1)) kmeans_kernel(KmArgs a) {
+__global__ void __launch_bounds__(1024, 2) kmeans_kernel(KmArgs a) {
   extern __shared__ float s_c[];
   __shared__ int slots;
   const int nck = a.nf * a.k;
@@ -87,14 +92,241 @@ __global__ void __launch_bounds__(MAXF == 0 ? 1024 : 256, MAXF == 0 ? 2 : (MAXF 
   cta_exit(a.t);
 }
 
+// REGS: centres transposed in shared memory (s_ct[f*k + c]) so the k values
+// of one feature are a broadcast; KMAX partial distances per thread.
+template <int KMAX>
+__global__ void __launch_bounds__(256) kmeans_stream_kernel(KmArgs a) {
+  extern __shared__ float s_ct[];
+  __shared__ int slots;
+  const int nf = a.nf, k = a.k;
+  for (int q = threadIdx.x; q < nf * k; q += blockDim.x) {
+    const int c = q / nf, f = q % nf;
+    s_ct[f * k + c] = a.clusters[q];
+  }
+  gate_init(&slots, a.t);
+  __syncthreads();
+  cta_enter(a.t);
+  const int64_t p = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  throttled(a.t, &slots, [&]() {
+    if (p >= a.npoints) return;
+    const float* f0 = a.feat + p;
+    const int64_t ld = a.ld;
+    float d[KMAX];
+#pragma unroll
+    for (int c = 0; c < KMAX; ++c) d[c] = 0.0f;
+    int f = 0;
+    for (; f + 8 <= nf; f += 8) {
+      float v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const float* q = f0 + int64_t(f + u) * ld;
+        asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[u]) : "l"(q));
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const float* cc = s_ct + (f + u) * k;
+#pragma unroll
+        for (int c = 0; c < KMAX; ++c) {
+          if (c < k) {
+            const float diff = v[u] - cc[c];
+            d[c] = fmaf(diff, diff, d[c]);
+          }
+        }
+      }
+    }
+    for (; f < nf; ++f) {
+      const float v = f0[int64_t(f) * ld];
+      const float* cc = s_ct + f * k;
+#pragma unroll
+      for (int c = 0; c < KMAX; ++c) {
+        if (c < k) {
+          const float diff = v - cc[c];
+          d[c] = fmaf(diff, diff, d[c]);
+        }
+      }
+    }
+    int index = -1;
+    float best = FLT_MAX;
+#pragma unroll
+    for (int c = 0; c < KMAX; ++c) {
+      if (c < k && d[c] < best) {
+        best = d[c];
+        index = c;
+      }
+    }
+    a.membership[p] = index;
+  });
+  cta_exit(a.t);
+}
+
+
+// STAGED: persistent CTAs; 2-D TMA copies of {256 points x nf features} tiles
+// (one request per tile) into an S-stage ring; thread t computes point
+// tile*256 + t from shared memory (column t of every feature row: conflict
+// free), k partial distances in registers, f ascending: bit-exact membership.
+namespace {
+__device__ __forceinline__ uint32_t k_s32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ void k_bar_init(uint64_t* b, uint32_t c) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(k_s32(b)), "r"(c) : "memory");
+}
+__device__ __forceinline__ void k_expect_tx(uint64_t* b, uint32_t n) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(k_s32(b)), "r"(n) : "memory");
+}
+__device__ __forceinline__ void k_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(k_s32(b)) : "memory");
+}
+__device__ __forceinline__ void k_wait(uint64_t* b, uint32_t ph) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "LAB_WAIT:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@P1 bra DONE;\n"
+      "bra LAB_WAIT;\n"
+      "DONE:\n"
+      "}\n" ::"r"(k_s32(b)),
+      "r"(ph)
+      : "memory");
+}
+__device__ __forceinline__ void k_tma2d(void* dst, const CUtensorMap* m, int32_t c0, int32_t c1, uint64_t* b) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          k_s32(dst)),
+      "l"(m), "r"(c0), "r"(c1), "r"(k_s32(b))
+      : "memory");
+}
+}  // namespace
+
+template <int KMAX>
+__global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constant__ CUtensorMap map, KmArgs a,
+                                                            int S) {
+  extern __shared__ __align__(1024) unsigned char dyn[];
+  const int t = threadIdx.x, lane = t & 31, nw = blockDim.x >> 5;
+  const int nf = a.nf, k = a.k;
+  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
+  uint64_t* empty = full + S;
+  float* s_ct = reinterpret_cast<float*>(dyn + 512);                    // [nf][k] transposed centres
+  const int head = 512 + ((nf * k * 4 + 511) / 512) * 512;
+  float* ring = reinterpret_cast<float*>(dyn + ((head + 1023) / 1024) * 1024);
+  const int tile_floats = nf * 256;
+  const int64_t ntiles_all = (a.npoints + 255) / 256;
+  const int64_t G = gridDim.x;
+  const int64_t mytiles = ntiles_all > blockIdx.x ? (ntiles_all - blockIdx.x + G - 1) / G : 0;
+  for (int q = t; q < nf * k; q += blockDim.x) s_ct[(q % nf) * k + q / nf] = a.clusters[q];
+  if (t == 0) {
+    for (int s = 0; s < S; ++s) {
+      k_bar_init(&full[s], 1);
+      k_bar_init(&empty[s], nw);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](int64_t c) {
+    const int s = int(c % S);
+    if (c >= S) k_wait(&empty[s], uint32_t(((c / S) - 1) & 1));
+    k_expect_tx(&full[s], uint32_t(tile_floats) * 4u);
+    k_tma2d(ring + int64_t(s) * tile_floats, &map, int32_t((blockIdx.x + c * G) * 256), 0, &full[s]);
+  };
+  if (t == 0)
+    for (int64_t c = 0; c < imin64(S, mytiles); ++c) issue(c);
+  for (int64_t c = 0; c < mytiles; ++c) {
+    const int s = int(c % S);
+    k_wait(&full[s], uint32_t((c / S) & 1));
+    const int64_t p = (blockIdx.x + c * G) * 256 + t;
+    if (p < a.npoints) {
+      const float* col = ring + int64_t(s) * tile_floats + t;
+      float d[KMAX];
+#pragma unroll
+      for (int cc = 0; cc < KMAX; ++cc) d[cc] = 0.0f;
+#pragma unroll 4
+      for (int f = 0; f < nf; ++f) {
+        const float v = col[f * 256];
+        const float* cf = s_ct + f * k;
+#pragma unroll
+        for (int cc = 0; cc < KMAX; ++cc) {
+          if (cc < k) {
+            const float diff = v - cf[cc];
+            d[cc] = fmaf(diff, diff, d[cc]);
+          }
+        }
+      }
+      int index = -1;
+      float best = FLT_MAX;
+#pragma unroll
+      for (int cc = 0; cc < KMAX; ++cc) {
+        if (cc < k && d[cc] < best) {
+          best = d[cc];
+          index = cc;
+        }
+      }
+      a.membership[p] = index;
+    }
+    __syncwarp();
+    if (lane == 0) k_arrive(&empty[s]);
+    if (t == 0 && c + S < mytiles) issue(c + S);
+  }
+}
+
 const void* kmeans_func(int variant, int nf) {
+  (void)nf;
+  if (variant == CATT_VAR_STAGED) return (const void*)kmeans_tma_kernel<8>;
   if (variant != CATT_VAR_REGS) return (const void*)kmeans_kernel<0>;
-  return nf <= 40 ? (const void*)kmeans_kernel<40> : (const void*)kmeans_kernel<kMaxRegsFeatures>;
+  return (const void*)kmeans_stream_kernel<8>;
 }
 
 }  // namespace catt
 
 using namespace catt;
+
+namespace {
+
+catt_status launch_kmeans_tma(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters,
+                              int32_t k, int32_t* membership, const catt_throttle* t, void* stream) {
+  if (k > 32 || nf > 256 || ld % 4 || (reinterpret_cast<uintptr_t>(feat) & 15u)) return CATT_EINVAL;
+  if (t && (t->active_warps || t->active_ctas || (t->cta_threads && t->cta_threads != 256))) return CATT_EINVAL;
+  void* fnp = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fnp, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess)
+    return CATT_ECUDA;
+  auto enc = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fnp);
+  CUtensorMap map;
+  const cuuint64_t dims[2] = {cuuint64_t(npoints), cuuint64_t(nf)};
+  const cuuint64_t strides[1] = {cuuint64_t(ld) * 4};
+  const cuuint32_t box[2] = {256, cuuint32_t(nf)};
+  const cuuint32_t es[2] = {1, 1};
+  if (enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(feat), dims, strides, box, es,
+          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return CATT_EINVAL;
+  const int tile_bytes = nf * 256 * 4;
+  const int head = ((512 + ((nf * k * 4 + 511) / 512) * 512 + 1023) / 1024) * 1024;
+  const int S = std::max(2, std::min(8, (200 * 1024 - head) / tile_bytes));
+  const size_t smem = size_t(head) + size_t(S) * tile_bytes;
+  const void* f = k <= 8 ? (const void*)kmeans_tma_kernel<8> : (const void*)kmeans_tma_kernel<32>;
+  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  KmArgs a{feat, clusters, membership, ld, npoints, nf, k, Throttle{}};
+  size_t dyn_total = 0;
+  catt_status st = prepare_launch(f, t, 256, smem, false, &a.t, &dyn_total);
+  if (st != CATT_OK) return st;
+  DevCtx* ctx = nullptr;
+  st = dev_ctx(&ctx);
+  if (st != CATT_OK) return st;
+  const int64_t tiles = (npoints + 255) / 256;
+  const unsigned grid = unsigned(std::min<int64_t>(tiles, ctx->hw.num_sms));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (k <= 8)
+    kmeans_tma_kernel<8><<<grid, 256, dyn_total, s>>>(map, a, S);
+  else
+    kmeans_tma_kernel<32><<<grid, 256, dyn_total, s>>>(map, a, S);
+  return after_launch();
+}
+
+}  // namespace
 
 extern "C" catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t npoints, int32_t nf,
                                           const float* clusters, int32_t k, int32_t* membership,
@@ -103,12 +335,14 @@ extern "C" catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t
   if (npoints > 0 && (!feat || !clusters || !membership)) return CATT_EINVAL;
   if (npoints == 0) return CATT_OK;
   const int var = variant_of(t);
+  if (var == CATT_VAR_STAGED) return launch_kmeans_tma(feat, ld, npoints, nf, clusters, k, membership, t, stream);
   if (var != CATT_VAR_LITERAL && var != CATT_VAR_REGS) return CATT_EINVAL;
   const int threads = cta_threads_or(t, 256);
-  if (var == CATT_VAR_REGS && (nf > kMaxRegsFeatures || threads > 256)) return CATT_EINVAL;
+  if (var == CATT_VAR_REGS && (k > 32 || threads > 256)) return CATT_EINVAL;
   KmArgs a{feat, clusters, membership, ld, npoints, nf, k, Throttle{}};
   const size_t dyn = size_t(nf) * size_t(k) * sizeof(float);
-  const void* f = kmeans_func(var, nf);
+  const void* f = var == CATT_VAR_REGS ? (k <= 8 ? (const void*)kmeans_stream_kernel<8> : (const void*)kmeans_stream_kernel<32>)
+                                       : (const void*)kmeans_kernel<0>;
   if (dyn > 48 * 1024 && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn)) != cudaSuccess)
     return after_launch();
   size_t dyn_total = 0;
@@ -116,10 +350,10 @@ extern "C" catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t
   if (st != CATT_OK) return st;
   const int64_t grid = (npoints + threads - 1) / threads;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  if (var == CATT_VAR_REGS && nf <= 40)
-    kmeans_kernel<40><<<dim3(unsigned(grid)), threads, dyn_total, s>>>(a);
+  if (var == CATT_VAR_REGS && k <= 8)
+    kmeans_stream_kernel<8><<<dim3(unsigned(grid)), threads, dyn_total, s>>>(a);
   else if (var == CATT_VAR_REGS)
-    kmeans_kernel<kMaxRegsFeatures><<<dim3(unsigned(grid)), threads, dyn_total, s>>>(a);
+    kmeans_stream_kernel<32><<<dim3(unsigned(grid)), threads, dyn_total, s>>>(a);
   else
     kmeans_kernel<0><<<dim3(unsigned(grid)), threads, dyn_total, s>>>(a);
   return after_launch();

@@ -392,7 +392,11 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
     } else if (var == CATT_VAR_REGS) {
       out->n_loops = 1;
       out->trip[0] = nf;
-      refs[n++] = mkref(1, 0, ld, 0, 4, 1, 0);                     // read once into registers
+      refs[n++] = mkref(1, 0, ld, 0, 4, 1, 0);                     // streamed once
+    } else if (var == CATT_VAR_STAGED) {
+      out->n_loops = 1;
+      out->trip[0] = nf;
+      refs[n++] = mkref(1, 0, ld, 0, 4, 1, CATT_REF_NOT_L1);       // TMA tiles in shared memory
     } else {
       return CATT_EINVAL;
     }

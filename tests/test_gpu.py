@@ -208,14 +208,20 @@ def test_syrk_throttled():
 
 
 # ------------------------------------------------------------------ KMEANS
-@pytest.mark.parametrize("variant", ["literal", "regs"])
-@pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 3), (4099, 34, 5, 29), (257, 7, 3, 0), (300, 50, 4, 1)])
+@pytest.mark.parametrize("variant", ["literal", "regs", "staged"])
+@pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 4), (4099, 34, 5, 29), (257, 7, 3, 3), (300, 50, 12, 4),
+                                           (70000, 34, 5, 4)])
 def test_kmeans_exact(variant, npts, nf, k, pad):
     ld = npts + pad
+    if variant == "staged" and ld % 4:
+        ld += 4 - ld % 4                                 # TMA rows need a 16-byte stride
     feat = si.values(4, nf * ld)
     clusters = feat.reshape(nf, ld)[:, :k].T.copy()          # centres = first k points
     memb_o, _ = oracle.kmeans_assign(feat, ld, npts, nf, clusters)
-    for t in (catt.Throttle(variant=variant), catt.Throttle(variant=variant, active_warps=2, active_ctas=3)):
+    ts = [catt.Throttle(variant=variant)]
+    if variant != "staged":                              # staged has no L1 reuse to throttle
+        ts.append(catt.Throttle(variant=variant, active_warps=2, active_ctas=3))
+    for t in ts:
         memb = catt.kmeans_assign(dev(feat), ld, npts, nf, dev(clusters), t=t)
         assert np.array_equal(host(memb), memb_o)
 
@@ -249,7 +255,7 @@ def test_kmeans_rodinia_shape_full():
         memb_o, _ = oracle.kmeans_assign(fh, ld, npts, nf, clusters)
         hw = catt.hw_query()
         t, r = catt.plan(catt.problem(catt.K_KMEANS, m=npts, n=nf, k=k, ld=ld), catt.Throttle(), hw)
-        for tt in (catt.Throttle(), t, catt.Throttle(variant="regs")):
+        for tt in (catt.Throttle(), t, catt.Throttle(variant="regs"), catt.Throttle(variant="staged")):
             memb = catt.kmeans_assign(feat, ld, npts, nf, dev(clusters), t=tt)
             assert np.array_equal(host(memb), memb_o)
 
