@@ -199,7 +199,9 @@ class BicgMvt(Workload):
             self.study = dict(name="bicg2 q=A p (literal, row per thread)", prob=P(catt.K_BICG_2, m=rows, n=n),
                               A=self.Ab, x=self.p, y=self.q,
                               launches=[(1024, 132), (1024, 196), (1024, 228), (256, 196), (256, 228)])
+            self._app_study_setup(catt, P, rows, n)
             return
+        self._app_study_setup(catt, P, rows, n)
         col_var = var if var in ("coop", "staged") else "literal"
         cta_row = {"coop": 256, "staged": 32, "vec4": 32, "literal": 32}[var]
         cta_col = {"coop": 1024, "staged": 32, "literal": 256}[col_var]
@@ -220,6 +222,15 @@ class BicgMvt(Workload):
         self.study = dict(name="bicg2 q=A p (literal, row per thread)", prob=P(catt.K_BICG_2, m=rows, n=n),
                           A=self.Ab, x=self.p, y=self.q,
                           launches=[(1024, 132), (1024, 196), (1024, 228), (256, 196), (256, 228)])
+
+    def _app_study_setup(self, catt, P, rows, n):
+        """BICG's two literal loops for the per-application BFTT vs per-loop
+        CATT comparison (P:7)."""
+        self.app_study = dict(
+            name="BICG (s = A^T r, q = A p), literal loops",
+            loops=[(P(catt.K_BICG_1, m=rows, n=n), lambda th: catt.cols(self.Ab, self.r, self.s, False, th)),
+                   (P(catt.K_BICG_2, m=rows, n=n), lambda th: catt.rows(self.Ab, self.p, self.q, catt.ROWS_STORE, t=th))],
+            launches=[(1024, 196), (1024, 228), (1024, 132)])
 
     def collective(self):
         if self.world > 1:
@@ -514,6 +525,62 @@ def throttle_study(catt, torch, w, flush):
     return out
 
 
+def app_study(catt, torch, w, flush):
+    """Per-loop CATT vs per-application BFTT (the paper's comparison, P:377,
+    P:395): BFTT applies one static (a, m) to every loop of the application
+    (the best such setting for the sum); CATT picks each loop's throttle."""
+    S = getattr(w, "app_study", None)
+    if not S:
+        return None
+
+    def med(fn, reps=3):
+        ts = []
+        for _ in range(reps + 1):
+            flush()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        ts = sorted(ts[1:])
+        return ts[len(ts) // 2]
+
+    out = []
+    paper_hw = catt.paper_rule(w.hw)
+    for cta, carve in S["launches"]:
+        launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
+        per_loop, picks, picks_p = [], [], []
+        for prob, mk in S["loops"]:
+            t, r = catt.plan(prob, launch, w.hw)
+            tp, rp = catt.plan(prob, launch, paper_hw)
+            W, T = r["base_warps"], r["base_ctas"]
+            times = {}
+            for a in [d for d in range(W, 0, -1) if W % d == 0]:
+                for m in range(T, 0, -1):
+                    times[(a, m)] = med(lambda a=a, m=m: mk(launch.copy(active_warps=a, active_ctas=m if m < T else 0)))
+            per_loop.append(times)
+            picks.append((t.active_warps or W, t.active_ctas or T))
+            picks_p.append((tp.active_warps or W, tp.active_ctas or T))
+        common = set(per_loop[0])
+        for tms in per_loop[1:]:
+            common &= set(tms)
+        bftt = min(common, key=lambda am: sum(tms[am] for tms in per_loop))
+        bftt_ms = sum(tms[bftt] for tms in per_loop)
+        catt_ms = sum(tms[pk] for tms, pk in zip(per_loop, picks))
+        paper_ms = sum(tms[pk] for tms, pk in zip(per_loop, picks_p))
+        full = [max(tms) for tms in per_loop]
+        full_ms = sum(tms[f] for tms, f in zip(per_loop, full))
+        out.append(dict(application=S["name"], cta_threads=cta, carveout_kb=carve,
+                        catt_picks=[list(p) for p in picks], catt_ms=round(catt_ms, 4),
+                        paper_picks=[list(p) for p in picks_p], paper_ms=round(paper_ms, 4),
+                        bftt=list(bftt), bftt_ms=round(bftt_ms, 4), full_ms=round(full_ms, 4),
+                        catt_speedup_over_bftt=round(bftt_ms / catt_ms, 4),
+                        paper_speedup_over_bftt=round(bftt_ms / paper_ms, 4),
+                        catt_speedup_over_full=round(full_ms / catt_ms, 4)))
+    return out
+
+
 def ncu_traffic(kernel_hint):
     """dram bytes per launch of the dominant kernel from the committed ncu summary."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -677,9 +744,10 @@ def main():
         e2e = {"value": round(total_bytes / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(e2e_ms, 4),
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
 
-    study = None
+    study = app = None
     if rank == 0 and not args.no_study:
         study = throttle_study(catt, torch, w, flush)
+        app = app_study(catt, torch, w, flush)
 
     # ---- roofline of the dominant loop
     dom = max(range(len(w.loops)), key=lambda i: loop_ms[i])
@@ -776,6 +844,7 @@ def main():
             "gpu_launches": len(w.loops) * args.steps,
             "clocks": clk,
             "throttle_study": study,
+            "bftt_vs_catt": app,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
