@@ -45,7 +45,8 @@ def parse():
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--workload", default="bicg_mvt",
                    choices=["bicg_mvt", "kmeans", "gesummv", "syrk", "atax256", "atax"])
-    p.add_argument("--variant", default=None, help="kernel variant for the streaming loops (default: per workload)")
+    p.add_argument("--variant", default=None,
+                   help="fused (default for bicg_mvt/atax), fused1, coop, staged, vec4, literal, regs (kmeans)")
     p.add_argument("--impl", default="catt", choices=["catt", "reference"])
     p.add_argument("--no-study", action="store_true", help="skip the throttle sweep")
     p.add_argument("--no-e2e", action="store_true")
@@ -185,17 +186,28 @@ class BicgMvt(Workload):
         mat = rows * n * 4
         acc2 = rank == 0                 # x2 = x2 + sum_g A_g^T y2_g: only rank 0 adds the initial x2
         P = catt.problem
-        if var == "fused":
-            # both loops of each application in one pass over A (A read once)
+        if var in ("fused", "fused1"):
+            # both loops of each application in one pass over A (A read once);
+            # "fused" also groups BICG and MVT into one launch (one 128 MiB
+            # stream instead of two 64 MiB ones), "fused1" is one launch each
             tf = self.plan("bicg fused", P(catt.K_BICG_2, m=rows, n=n), catt.Throttle(variant="fused"))
             tg = self.plan("mvt fused", P(catt.K_MVT_1, n=n), catt.Throttle(variant="fused"))
-            self.loops = [
-                Loop("bicg fused", lambda: catt.dual(self.Ab, self.p, self.q, self.s, xc=self.r, t=tf),
-                     mat + 4 * 2 * (rows + n), "fused"),
-                Loop("mvt fused", lambda: catt.dual(self.Am, self.y1, self.x1, self.x2, xc=self.y2,
-                                                    row_accumulate=True, col_accumulate=acc2, t=tg),
-                     mat + 4 * (3 * rows + (3 if acc2 else 2) * n), "fused"),
-            ]
+            bicg_b = mat + 4 * 2 * (rows + n)
+            mvt_b = mat + 4 * (3 * rows + (3 if acc2 else 2) * n)
+            if var == "fused":
+                group = [dict(A=self.Ab, xr=self.p, xc=self.r, yr=self.q, yc=self.s),
+                         dict(A=self.Am, xr=self.y1, xc=self.y2, yr=self.x1, yc=self.x2, row_accumulate=True,
+                              col_accumulate=acc2)]
+                self.loops = [Loop("bicg+mvt fused (one launch)", lambda: catt.dual_group(group, t=tf),
+                                   bicg_b + mvt_b, "fused")]
+            else:
+                self.loops = [
+                    Loop("bicg fused", lambda: catt.dual(self.Ab, self.p, self.q, self.s, xc=self.r, t=tf),
+                         bicg_b, "fused"),
+                    Loop("mvt fused", lambda: catt.dual(self.Am, self.y1, self.x1, self.x2, xc=self.y2,
+                                                        row_accumulate=True, col_accumulate=acc2, t=tg),
+                         mvt_b, "fused"),
+                ]
             self.study = dict(name="bicg2 q=A p (literal, row per thread)", prob=P(catt.K_BICG_2, m=rows, n=n),
                               A=self.Ab, x=self.p, y=self.q,
                               launches=[(1024, 132), (1024, 196), (1024, 228), (256, 196), (256, 228)])

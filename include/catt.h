@@ -299,6 +299,22 @@ catt_status catt_dual(const float* A, const float* xr, const float* xc, float* y
                       int32_t row_accumulate, int32_t col_accumulate, int32_t dependent, const catt_throttle* t,
                       void* stream);
 
+/* Several independent dual problems with the same n in one grouped launch
+ * (up to 4; e.g. BICG and MVT of one step): one longer stream instead of
+ * several short ones. Semantics per problem as catt_dual; `dependent` applies
+ * to all of them. */
+typedef struct {
+  const float* A;
+  const float* xr;
+  const float* xc;
+  float* yr;
+  float* yc;
+  int64_t m, n;
+  int32_t row_accumulate, col_accumulate;
+} catt_dual_problem;
+catt_status catt_dual_group(const catt_dual_problem* probs, int32_t count, int32_t dependent, const catt_throttle* t,
+                            void* stream);
+
 /* ------------------------------------------------------------------ helpers */
 /* dst[i] = value(seed, offset + i): the counter-based generator of
  * seeded_inputs.py (mode 0 uniform [0,1), 1 dyadic k/16). Device pointer. */

@@ -120,6 +120,12 @@ class Throttle(ctypes.Structure):
                 f"carveout={self.carveout_kb}KB, variant={self.variant}, gate={self.gate}, cap={self.cap})")
 
 
+class DualProblem(ctypes.Structure):
+    _fields_ = [("A", ctypes.c_void_p), ("xr", ctypes.c_void_p), ("xc", ctypes.c_void_p), ("yr", ctypes.c_void_p),
+                ("yc", ctypes.c_void_p), ("m", ctypes.c_int64), ("n", ctypes.c_int64),
+                ("row_accumulate", ctypes.c_int32), ("col_accumulate", ctypes.c_int32)]
+
+
 class Problem(ctypes.Structure):
     _fields_ = [("loop", ctypes.c_int32), ("reserved_", ctypes.c_int32), ("m", ctypes.c_int64),
                 ("n", ctypes.c_int64), ("k", ctypes.c_int64), ("ld", ctypes.c_int64)]
@@ -157,6 +163,7 @@ def lib():
             "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
             "catt_rows": [V, V, V, V, V, i64, i64, f32, f32, i32, T, V],
             "catt_dual": [V, V, V, V, V, i64, i64, i32, i32, i32, T, V],
+            "catt_dual_group": [P(DualProblem), i32, i32, T, V],
             "catt_cols": [V, V, V, i64, i64, i32, T, V],
             "catt_fill_hash": [V, i64, u32, u64, i32, V],
             "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
@@ -176,7 +183,7 @@ def lib():
 
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_kmeans_assign",
-            "catt_rows", "catt_cols", "catt_dual", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
+            "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version"]
 
 
@@ -369,6 +376,19 @@ def dual(A, xr, yr, yc, xc=None, row_accumulate=False, col_accumulate=False, dep
                            _dev(yc, "yc"), m, n, int(bool(row_accumulate)), int(bool(col_accumulate)),
                            int(bool(dependent)), _tp(t), _stream()), "catt_dual")
     return yr, yc
+
+
+def dual_group(problems, dependent=False, t: Optional[Throttle] = None):
+    """Grouped catt_dual: problems = [dict(A=, xr=, yr=, yc=, xc=None, row_accumulate=False,
+    col_accumulate=False)], same column count, one launch."""
+    arr = (DualProblem * len(problems))()
+    for i, p in enumerate(problems):
+        m, n = p["A"].shape
+        arr[i] = DualProblem(_dev(p["A"], "A").value, _dev(p["xr"], "xr").value,
+                             _dev(p["xc"], "xc").value if p.get("xc") is not None else None,
+                             _dev(p["yr"], "yr").value, _dev(p["yc"], "yc").value, m, n,
+                             int(bool(p.get("row_accumulate"))), int(bool(p.get("col_accumulate"))))
+    _check(lib().catt_dual_group(arr, len(problems), int(bool(dependent)), _tp(t), _stream()), "catt_dual_group")
 
 
 def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):

@@ -432,3 +432,24 @@ def test_fused_atax_65536x16384_sampled():
     t64, y64 = oracle.atax_hashed(si.SEED_ATAX_SHARDED, 0, x, m, n, cols, mode=oracle.SEQ_F64)
     tmp, y = catt.atax(A.view(m, n), dev(x), k1=catt.Throttle(variant="fused"))
     assert relerr(host(tmp), t64) <= TOL and relerr(host(y)[cols], y64) <= TOL
+
+
+@pytest.mark.parametrize("shapes", [[(1000, 132), (300, 132)], [(4096, 4096), (4096, 4096)], [(33, 64), (5000, 64), (7, 64)]])
+def test_dual_group_bicg_and_mvt_in_one_launch(shapes):
+    """BICG and MVT problems (same n) in one grouped fused launch."""
+    probs, want = [], []
+    for k, (m, n) in enumerate(shapes):
+        A = si.matrix(20 + k, m, n, si.MODE_DYADIC)
+        xr, xc = si.values(30 + k, n, mode=si.MODE_DYADIC), si.values(40 + k, m, mode=si.MODE_DYADIC)
+        yr0, yc0 = si.values(50 + k, m, mode=si.MODE_DYADIC), si.values(60 + k, n, mode=si.MODE_DYADIC)
+        acc = k % 2 == 1                                   # odd problems: MVT-style in/out
+        YR, YC = dev(yr0), dev(yc0)
+        probs.append(dict(A=dev(A), xr=dev(xr), xc=dev(xc), yr=YR, yc=YC, row_accumulate=acc, col_accumulate=acc))
+        q, s = oracle.bicg(A, xr, xc)                         # dyadic: exact, any order
+        if acc:
+            q = (yr0.astype(np.float64) + q).astype(np.float32)
+            s = (yc0.astype(np.float64) + s).astype(np.float32)
+        want.append((YR, YC, q, s))
+    catt.dual_group(probs)
+    for YR, YC, q, s in want:
+        assert bits_equal(host(YR), q) and bits_equal(host(YC), s)
