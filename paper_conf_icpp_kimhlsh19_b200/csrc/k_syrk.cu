@@ -5,7 +5,7 @@
 //     c = C[i][j] * beta;  for k < m: c = fmaf(alpha * a[i][k], a[j][k], c)
 // a[j][k] is memory-divergent across the warp (32 rows of A) and reused for
 // 32 consecutive k; a[i][k] is a broadcast. CATT throttles this loop.
-// STAGED: 128 x 128 output tiles, 8 k per stage in shared memory (alpha*a_i
+// STAGED: 128 x 128 output tiles, 16 k per stage in shared memory (alpha*a_i
 // pre-multiplied with the same rounding), 8 x 8 outputs per thread held in
 // registers; every output still accumulates k = 0, 1, ..., m-1 in order, so
 // the result is bit-identical to LITERAL. FP32 CUDA-core bound (no tensor
@@ -44,10 +44,24 @@ __global__ void __launch_bounds__(1024, 2) syrk_thread_kernel(SyrkArgs a) {
   cta_exit(a.t);
 }
 
-constexpr int BM = 128, BK = 8, TM = 8;
-constexpr int PITCH = BM + 4;  // conflict-free transposed stores, 16-B aligned rows
+constexpr int BM = 128, BK = 16, TM = 8;
+constexpr int PITCH = BM + 4;  // transposed tiles: 16-B aligned rows, spread store banks
 
-__global__ void __launch_bounds__(256) syrk_tiled_kernel(SyrkArgs a) {
+// One k-step of the 8 x 8 register tile: c[r][q] = fmaf(alpha*a_i[r], a_j[q], c[r][q]).
+__device__ __forceinline__ void syrk_kstep(float (&c)[TM][TM], const float* as, const float* bs, int ty, int tx) {
+  const float4 a0 = *reinterpret_cast<const float4*>(as + ty * TM);
+  const float4 a1 = *reinterpret_cast<const float4*>(as + ty * TM + 4);
+  const float4 b0 = *reinterpret_cast<const float4*>(bs + tx * TM);
+  const float4 b1 = *reinterpret_cast<const float4*>(bs + tx * TM + 4);
+  const float av[TM] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+  const float bv[TM] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+  for (int r = 0; r < TM; ++r)
+#pragma unroll
+    for (int q = 0; q < TM; ++q) c[r][q] = fmaf(av[r], bv[q], c[r][q]);
+}
+
+__global__ void __launch_bounds__(256, 2) syrk_tiled_kernel(SyrkArgs a) {
   __shared__ __align__(16) float As[2][BK][PITCH];  // alpha * a[i][k], transposed
   __shared__ __align__(16) float Bs[2][BK][PITCH];  // a[j][k], transposed
   cta_enter(a.t);
@@ -55,8 +69,9 @@ __global__ void __launch_bounds__(256) syrk_tiled_kernel(SyrkArgs a) {
   const int tx = tid & 15, ty = tid >> 4;
   const int64_t i0 = int64_t(blockIdx.y) * BM, j0 = int64_t(blockIdx.x) * BM;
   const int64_t n = a.n, m = a.m;
-  // loader mapping: thread -> (row r = tid / 2, k sub-block (tid & 1) * 4)
-  const int lr = tid >> 1, lk = (tid & 1) * 4;
+  // loader: thread -> row lr = tid / 2 of the tile, k sub-block (tid & 1) * 8 (two float4)
+  const int lr = tid >> 1, lk = (tid & 1) * 8;
+  const bool vec = (m % 4) == 0 && (reinterpret_cast<uintptr_t>(a.A) & 15u) == 0;
   float c[TM][TM];
 #pragma unroll
   for (int r = 0; r < TM; ++r)
@@ -65,19 +80,33 @@ __global__ void __launch_bounds__(256) syrk_tiled_kernel(SyrkArgs a) {
       const int64_t gi = i0 + ty * TM + r, gj = j0 + tx * TM + q;
       c[r][q] = (gi < n && gj < n) ? __fmul_rn(a.C[gi * n + gj], a.beta) : 0.0f;
     }
-  float ra[4], rb[4];
+  float ra[8], rb[8];
   auto gload = [&](int64_t k0) {
-    const int64_t gi = i0 + lr, gj = j0 + lr;
+    const int64_t gi = i0 + lr, gj = j0 + lr, kb = k0 + lk;
+    if (vec && kb + 8 <= m) {
+      const float4* pa = reinterpret_cast<const float4*>(a.A + gi * m + kb);
+      const float4* pb = reinterpret_cast<const float4*>(a.A + gj * m + kb);
+      const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+      const float4 a0 = gi < n ? pa[0] : z, a1 = gi < n ? pa[1] : z;
+      const float4 b0 = gj < n ? pb[0] : z, b1 = gj < n ? pb[1] : z;
+      ra[0] = __fmul_rn(a.alpha, a0.x); ra[1] = __fmul_rn(a.alpha, a0.y);
+      ra[2] = __fmul_rn(a.alpha, a0.z); ra[3] = __fmul_rn(a.alpha, a0.w);
+      ra[4] = __fmul_rn(a.alpha, a1.x); ra[5] = __fmul_rn(a.alpha, a1.y);
+      ra[6] = __fmul_rn(a.alpha, a1.z); ra[7] = __fmul_rn(a.alpha, a1.w);
+      rb[0] = b0.x; rb[1] = b0.y; rb[2] = b0.z; rb[3] = b0.w;
+      rb[4] = b1.x; rb[5] = b1.y; rb[6] = b1.z; rb[7] = b1.w;
+    } else {
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int64_t k = k0 + lk + u;
-      ra[u] = (gi < n && k < m) ? __fmul_rn(a.alpha, a.A[gi * m + k]) : 0.0f;
-      rb[u] = (gj < n && k < m) ? a.A[gj * m + k] : 0.0f;
+      for (int u = 0; u < 8; ++u) {
+        const int64_t k = kb + u;
+        ra[u] = (gi < n && k < m) ? __fmul_rn(a.alpha, a.A[gi * m + k]) : 0.0f;
+        rb[u] = (gj < n && k < m) ? a.A[gj * m + k] : 0.0f;
+      }
     }
   };
   auto sstore = [&](int buf) {
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < 8; ++u) {
       As[buf][lk + u][lr] = ra[u];
       Bs[buf][lk + u][lr] = rb[u];
     }
@@ -90,28 +119,29 @@ __global__ void __launch_bounds__(256) syrk_tiled_kernel(SyrkArgs a) {
     const int buf = int(kt & 1);
     if (kt + 1 < ktiles) gload((kt + 1) * BK);
     const int kvalid = int(imin64(BK, m - kt * BK));  // uniform: never run k >= m
-    for (int kk = 0; kk < kvalid; ++kk) {
-      const float4 a0 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * TM]);
-      const float4 a1 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * TM + 4]);
-      const float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * TM]);
-      const float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * TM + 4]);
-      const float av[TM] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-      const float bv[TM] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+    if (kvalid == BK) {
 #pragma unroll
-      for (int r = 0; r < TM; ++r)
-#pragma unroll
-        for (int q = 0; q < TM; ++q) c[r][q] = fmaf(av[r], bv[q], c[r][q]);
+      for (int kk = 0; kk < BK; ++kk) syrk_kstep(c, &As[buf][kk][0], &Bs[buf][kk][0], ty, tx);
+    } else {
+      for (int kk = 0; kk < kvalid; ++kk) syrk_kstep(c, &As[buf][kk][0], &Bs[buf][kk][0], ty, tx);
     }
     if (kt + 1 < ktiles) sstore(buf ^ 1);
     __syncthreads();
   }
 #pragma unroll
-  for (int r = 0; r < TM; ++r)
+  for (int r = 0; r < TM; ++r) {
+    const int64_t gi = i0 + ty * TM + r;
+    if (gi >= n) continue;
+    float* crow = a.C + gi * n + j0 + tx * TM;
+    if (j0 + tx * TM + TM <= n && (n % 4) == 0) {
+      reinterpret_cast<float4*>(crow)[0] = make_float4(c[r][0], c[r][1], c[r][2], c[r][3]);
+      reinterpret_cast<float4*>(crow)[1] = make_float4(c[r][4], c[r][5], c[r][6], c[r][7]);
+    } else {
 #pragma unroll
-    for (int q = 0; q < TM; ++q) {
-      const int64_t gi = i0 + ty * TM + r, gj = j0 + tx * TM + q;
-      if (gi < n && gj < n) a.C[gi * n + gj] = c[r][q];
+      for (int q = 0; q < TM; ++q)
+        if (j0 + tx * TM + q < n) crow[q] = c[r][q];
     }
+  }
   cta_exit(a.t);
 }
 
