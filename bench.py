@@ -44,7 +44,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--workload", default="bicg_mvt",
-                   choices=["bicg_mvt", "kmeans", "gesummv", "syrk", "atax256", "atax"])
+                   choices=["bicg_mvt", "kmeans", "gesummv", "syrk", "syr2k", "atax256", "atax"])
     p.add_argument("--variant", default=None,
                    help="fused (default for bicg_mvt/atax), fused1, coop, staged, vec4, literal, regs (kmeans)")
     p.add_argument("--impl", default="catt", choices=["catt", "reference"])
@@ -371,6 +371,42 @@ class Syrk(Workload):
         oracle.syrk_rows(host["A"], host["C"], 1.5, 1.2, np.arange(16))
 
 
+class Syr2k(Workload):
+    name = "syr2k"
+    desc = "SYR2K 2048 fp32 (Table 2 P:77 size; SURVEY 8(f) f3)"
+    variant = "staged"
+
+    def __init__(self, catt, torch, rank, world, variant):
+        super().__init__(catt, torch, rank, world, variant)
+        import seeded_inputs as si
+        n = 2048
+        dev = torch.device("cuda")
+        self.A, self.B, self.C = (torch.empty(n, n, device=dev) for _ in range(3))
+        catt.fill_hash(self.A, si.SEED_SYR2K + rank)
+        catt.fill_hash(self.B, si.sub_seed(si.SEED_SYR2K, 1) + rank)
+        catt.fill_hash(self.C, si.sub_seed(si.SEED_SYR2K, 2) + rank)
+        t = self.plan("syr2k", catt.problem(catt.K_SYR2K, n=n, k=n), catt.Throttle(variant=self.variant))
+        self.flops = 4 * n * n * n
+        self.loops = [Loop("syr2k", lambda: catt.syr2k(self.A, self.B, self.C, 1.5, 1.2, t=t), 4 * n * n * 4, "syr2k")]
+        Cs = self.C.clone()
+        self.study = dict(name="syr2k (literal, 2-D block 32 x 8)", prob=catt.problem(catt.K_SYR2K, n=n, k=n),
+                          launches=[(256, 228), (256, 100)], reps=2,
+                          fn=lambda th: (lambda: catt.syr2k(self.A, self.B, Cs, 1.5, 1.2, t=th)))
+
+    def inputs(self):
+        return [self.A, self.B, self.C]
+
+    def outputs(self):
+        return [self.C]
+
+    def host_copy(self):
+        return {k: getattr(self, k).cpu().numpy() for k in ("A", "B", "C")}
+
+    def cpu_oracle_step(self, oracle, host):
+        import numpy as np
+        oracle.syr2k_rows(host["A"], host["B"], host["C"], 1.5, 1.2, np.arange(16))
+
+
 class Atax(Workload):
     name = "atax"
     variant = "fused"
@@ -437,7 +473,7 @@ class Atax256(Atax):
         super().__init__(catt, torch, rank, world, variant, m=256, n=256)
 
 
-WORKLOADS = {"bicg_mvt": BicgMvt, "kmeans": Kmeans, "gesummv": Gesummv, "syrk": Syrk, "atax256": Atax256,
+WORKLOADS = {"bicg_mvt": BicgMvt, "kmeans": Kmeans, "gesummv": Gesummv, "syrk": Syrk, "syr2k": Syr2k, "atax256": Atax256,
              "atax": Atax}
 
 
@@ -513,13 +549,15 @@ def throttle_study(catt, torch, w, flush):
         times = {}
         for a, m in cands:
             th = launch.copy(active_warps=a, active_ctas=m if m < T else 0)
-            if S.get("kmeans"):
+            if S.get("fn"):
+                fn = S["fn"](th)
+            elif S.get("kmeans"):
                 fn = lambda th=th: catt.kmeans_assign(w.feat, w.ld, w.np_, w.nf, w.clusters, w.memb, t=th)
             elif S.get("gesummv"):
                 fn = lambda th=th: catt.rows(w.A, w.x, w.y, catt.ROWS_GESUMMV, w.B, w.tmp, 1.5, 1.2, th)
             else:
                 fn = lambda th=th: catt.rows(S["A"], S["x"], S["y"], catt.ROWS_STORE, t=th)
-            times[(a, m)] = med(fn)
+            times[(a, m)] = med(fn, S.get("reps", 5))
         pick = (t.active_warps or W, t.active_ctas or T)
         pick_p = (tp.active_warps or W, tp.active_ctas or T)
         best = min(times, key=times.get)
@@ -765,13 +803,13 @@ def main():
     dom = max(range(len(w.loops)), key=lambda i: loop_ms[i])
     lp = w.loops[dom]
     peak, peak_src = peak_hbm()
-    if lp.kind == "syrk":
+    if lp.kind in ("syrk", "syr2k"):
         # FP32 CUDA-core bound: 148 SMs x 128 FP32 lanes x 2 flop x clock
         clk_mhz = clk.get("sm_mhz") or 1965.0
         peak_t = 148 * 128 * 2 * clk_mhz * 1e6 / 1e12
         ach = w.flops / (loop_ms[dom] * 1e-3) / 1e12
         roof = {"bound": "alu", "kernel": lp.name, "achieved": round(ach, 3), "peak": round(peak_t, 3),
-                "unit": "TFLOP/s", "frac": round(ach / peak_t, 4), "traffic": ncu_traffic("syrk"),
+                "unit": "TFLOP/s", "frac": round(ach / peak_t, 4), "traffic": ncu_traffic(lp.kind),
                 "peak_source": f"derived: 148 SM x 128 FP32 lanes x 2 x {clk_mhz:.0f} MHz (median under load)"}
     else:
         ach = lp.nbytes / (loop_ms[dom] * 1e-3) / 1e9
@@ -782,7 +820,7 @@ def main():
     # ---- context: a plain device copy moving the same bytes as the dominant
     # loop, timed the same way (flush, queued events). At 64 MiB a single
     # kernel cannot reach the 2 GiB copy peak of MEASURED_PEAKS.json.
-    if lp.kind != "syrk":
+    if lp.kind not in ("syrk", "syr2k"):
         half = max(1, lp.nbytes // 8)                # floats per side: read + write = nbytes
         src = torch.empty(half, device="cuda")
         dst = torch.empty(half, device="cuda")
@@ -830,7 +868,7 @@ def main():
                 reps += 1
             sec = (time.perf_counter() - t0) / reps
             cpu_bytes = step_bytes
-            if w.name == "syrk":
+            if w.name in ("syrk", "syr2k"):
                 cpu_bytes = step_bytes * 16 / 2048
             if w.name == "atax":
                 cpu_bytes = step_bytes * min(w.rows, 8192) / w.rows

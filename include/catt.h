@@ -196,11 +196,12 @@ enum {
   CATT_K_GESUMMV = 6, /* y = alpha A x + beta B x (row per thread, 2 matrices)*/
   CATT_K_SYRK = 7,    /* C = beta C + alpha A A^T (2-D block 32 x 8)          */
   CATT_K_KMEANS = 8,  /* membership = argmin_c |f_p - c|^2, feature-major     */
-  CATT_K_COUNT = 9
+  CATT_K_SYR2K = 9,   /* C = beta C + alpha (A B^T + B A^T), 2-D block 32 x 8 */
+  CATT_K_COUNT = 10
 };
 
 /* Problem sizes: ATAX/BICG m x n (rows, cols); MVT/GESUMMV n (m ignored);
- * SYRK n x n output, k = inner size m; KMEANS m = npoints, n = nfeatures,
+ * SYRK/SYR2K n x n output, k = inner size m; KMEANS m = npoints, n = nfeatures,
  * k = clusters, ld = feature-major leading dimension. */
 typedef struct {
   int32_t loop;
@@ -262,6 +263,15 @@ catt_status catt_gesummv(const float* A, const float* B, const float* x, float* 
  * per C element; STAGED = shared-memory tiles, register blocking, same k order. */
 catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta,
                       const catt_throttle* t, void* stream);
+
+/* SYR2K (Table 2, Table 3; the paper's 2-D cache-sensitive kernel):
+ * C = beta*C + alpha*(A B^T + B A^T) over the full square, A and B n x m,
+ * C in/out. Per element, k ascending: p = alpha*a_ik, q = alpha*b_ik,
+ * s = fmaf(p, b_jk, q*a_jk), c = c + s (every intermediate rounded; DESIGN.md
+ * R20). LITERAL = 2-D block 32 x (cta_threads/32); STAGED = shared-memory
+ * tiles with the same order. */
+catt_status catt_syr2k(const float* A, const float* B, float* C, int64_t n, int64_t m, float alpha, float beta,
+                       const catt_throttle* t, void* stream);
 
 /* KMEANS assignment (Table 2, Table 3): feat is feature-major,
  * feat[f*ld + p] for f < nf, p < npoints (ld >= npoints); clusters is k x nf;

@@ -55,6 +55,9 @@ def lib():
         L.orc_syrk.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float]
         L.orc_syrk_rows.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float,
                                     ctypes.POINTER(ctypes.c_int64), i64, f32p]
+        L.orc_syr2k.argtypes = [ctypes.c_int, f32p, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float]
+        L.orc_syr2k_rows.argtypes = [ctypes.c_int, f32p, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float,
+                                     ctypes.POINTER(ctypes.c_int64), i64, f32p]
         L.orc_kmeans_assign.argtypes = [ctypes.c_int, f32p, i64, i64, i32, f32p, i32,
                                         ctypes.POINTER(ctypes.c_int32), f32p]
         L.orc_atax_hashed.argtypes = [ctypes.c_int, u32, ctypes.c_int, f32p, i64, i64, f32p,
@@ -135,6 +138,23 @@ def syrk_rows(A, C, alpha, beta, rows, mode=SEQ_FMAF):
     rows = np.ascontiguousarray(rows, dtype=np.int64)
     out = np.empty((len(rows), n), np.float32)
     lib().orc_syrk_rows(mode, _p(A), _p(C), n, m, alpha, beta, _p(rows), len(rows), _p(out))
+    return out
+
+
+def syr2k(A, B, C, alpha, beta, mode=SEQ_FMAF):
+    A, B = _f32(A), _f32(B)
+    C = _f32(C).copy()
+    n, m = A.shape
+    lib().orc_syr2k(mode, _p(A), _p(B), _p(C), n, m, alpha, beta)
+    return C
+
+
+def syr2k_rows(A, B, C, alpha, beta, rows, mode=SEQ_FMAF):
+    A, B, C = _f32(A), _f32(B), _f32(C)
+    n, m = A.shape
+    rows = np.ascontiguousarray(rows, dtype=np.int64)
+    out = np.empty((len(rows), n), np.float32)
+    lib().orc_syr2k_rows(mode, _p(A), _p(B), _p(C), n, m, alpha, beta, _p(rows), len(rows), _p(out))
     return out
 
 

@@ -234,6 +234,51 @@ int orc_syrk_rows(int mode, const float* A, const float* C, int64_t n, int64_t m
   return 0;
 }
 
+/* ---------------------------------------------------------------- SYR2K
+ * PolyBench/GPU syr2k (Table 2; Table 3, the paper's 2-D CS
+ * kernel), A and B are n x m, C is n x n in/out, full square:
+ *   c[i][j] *= beta;
+ *   for k: c[i][j] += alpha*a[i][k]*b[j][k] + alpha*b[i][k]*a[j][k]
+ * The evaluation order of the right-hand side is fixed (R20):
+ *   p = alpha*a_ik (rounded), q = alpha*b_ik (rounded),
+ *   s = fmaf(p, b_jk, q*a_jk (rounded)),  c = c + s (rounded).          */
+static float orc_syr2k_elem(int mode, const float* A, const float* B, const float* C, int64_t n, int64_t m,
+                            float alpha, float beta, int64_t i, int64_t j) {
+  if (mode == ORC_SEQ_FMAF) {
+    float c = C[i * n + j] * beta;
+    for (int64_t k = 0; k < m; ++k) {
+      const float p = alpha * A[i * m + k];
+      const float q = alpha * B[i * m + k];
+      const float t = q * A[j * m + k];
+      const float s = fmaf(p, B[j * m + k], t);
+      c = c + s;
+    }
+    return c;
+  }
+  double c = (double)C[i * n + j] * (double)beta;
+  for (int64_t k = 0; k < m; ++k)
+    c += (double)alpha * (double)A[i * m + k] * (double)B[j * m + k] +
+         (double)alpha * (double)B[i * m + k] * (double)A[j * m + k];
+  return (float)c;
+}
+
+int orc_syr2k(int mode, const float* A, const float* B, float* C, int64_t n, int64_t m, float alpha, float beta) {
+  float* out = (float*)malloc(sizeof(float) * (size_t)(n > 0 ? n * n : 1));
+  if (!out) return -1;
+#pragma omp parallel for schedule(static)
+  for (int64_t q = 0; q < n * n; ++q) out[q] = orc_syr2k_elem(mode, A, B, C, n, m, alpha, beta, q / n, q % n);
+  memcpy(C, out, sizeof(float) * (size_t)(n * n));
+  free(out);
+  return 0;
+}
+
+int orc_syr2k_rows(int mode, const float* A, const float* B, const float* C, int64_t n, int64_t m, float alpha,
+                   float beta, const int64_t* rows, int64_t nrows, float* out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t q = 0; q < nrows * n; ++q) out[q] = orc_syr2k_elem(mode, A, B, C, n, m, alpha, beta, rows[q / n], q % n);
+  return 0;
+}
+
 /* ---------------------------------------------------------------- KMEANS assign
  * Rodinia kmeans (Table 2; Table 3), assignment step
  * (kmeansPoint), features stored feature-major: feat[f*ld + p].

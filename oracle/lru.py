@@ -124,6 +124,27 @@ class SyrkKernel(Kernel):
         return ev
 
 
+class Syr2kKernel(SyrkKernel):
+    """PolyBench/GPU syr2k, block (32, 8), same thread map as syrk; for k < Mk:
+    c += alpha*a[i*Mk + k]*b[j*Mk + k] + alpha*b[i*Mk + k]*a[j*Mk + k]."""
+
+    def events(self, b, w):
+        bx, by = b % self.gx, b // self.gx
+        th = []
+        for t in self.lanes(b, w):
+            tx, ty = t % self.bdim[0], t // self.bdim[0]
+            i, j = by * self.bdim[1] + ty, bx * self.bdim[0] + tx
+            if i < self.N and j < self.N:
+                th.append((i, j))
+        ev = []
+        if not th:
+            return ev
+        for k in range(self.Mk):
+            for X, row in (("a", 0), ("b", 0), ("b", 1), ("a", 1)):
+                ev.append(tuple((_line(X, (i, j)[row] * self.Mk + k), (i, j)) for i, j in th))
+        return ev
+
+
 class KmeansKernel(Kernel):
     """Rodinia kmeansPoint, feature-major: thread p (p < npoints):
     for c < k: for f < nf: diff = feat[f*ld + p] - clusters[c*nf + f]

@@ -27,7 +27,7 @@ VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED = 0, 1, 2, 3, 4
 ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
-(K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS) = range(9)
+(K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K) = range(10)
 
 VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS,
             "fused": VAR_FUSED}
@@ -160,6 +160,7 @@ def lib():
             "catt_mvt": [V, V, V, V, V, i64, T, T, V],
             "catt_gesummv": [V, V, V, V, V, i64, f32, f32, T, V],
             "catt_syrk": [V, V, i64, i64, f32, f32, T, V],
+            "catt_syr2k": [V, V, V, i64, i64, f32, f32, T, V],
             "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
             "catt_rows": [V, V, V, V, V, i64, i64, f32, f32, i32, T, V],
             "catt_dual": [V, V, V, V, V, i64, i64, i32, i32, i32, T, V],
@@ -182,7 +183,7 @@ def lib():
 
 
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
-            "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_kmeans_assign",
+            "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_kmeans_assign",
             "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version"]
 
@@ -396,6 +397,14 @@ def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):
     n, m = A.shape
     _check(lib().catt_syrk(_dev(A, "A"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t), _stream()),
            "catt_syrk")
+    return C
+
+
+def syr2k(A, B, C, alpha, beta, t: Optional[Throttle] = None):
+    """C = beta C + alpha (A B^T + B A^T) in place (catt_syr2k). Returns C."""
+    n, m = A.shape
+    _check(lib().catt_syr2k(_dev(A, "A"), _dev(B, "B"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t),
+                            _stream()), "catt_syr2k")
     return C
 
 

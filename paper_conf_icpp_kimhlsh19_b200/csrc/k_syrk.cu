@@ -5,11 +5,13 @@
 //     c = C[i][j] * beta;  for k < m: c = fmaf(alpha * a[i][k], a[j][k], c)
 // a[j][k] is memory-divergent across the warp (32 rows of A) and reused for
 // 32 consecutive k; a[i][k] is a broadcast. CATT throttles this loop.
-// STAGED: 128 x 128 output tiles, 16 k per stage in shared memory (alpha*a_i
-// pre-multiplied with the same rounding), 8 x 8 outputs per thread held in
-// registers; every output still accumulates k = 0, 1, ..., m-1 in order, so
-// the result is bit-identical to LITERAL. FP32 CUDA-core bound (no tensor
-// cores: TF32 would break the 1e-5 bar, BASELINE north_star).
+// STAGED: 128 x 128 output tiles in shared memory (alpha*a_i pre-multiplied
+// with the same rounding), 8 x 8 outputs per thread held in registers; every
+// output still accumulates k = 0, 1, ..., m-1 in order, so the result is
+// bit-identical to LITERAL. FP32 CUDA-core bound (no tensor cores: TF32 would
+// break the 1e-5 bar, BASELINE north_star). SYR2K (below) shares the tiled
+// kernel; its literal kernel is the paper's 2-D CS loop.
+#include <cstdlib>
 #include <cstdint>
 
 #include "internal.h"
@@ -44,109 +46,280 @@ __global__ void __launch_bounds__(1024, 2) syrk_thread_kernel(SyrkArgs a) {
   cta_exit(a.t);
 }
 
-constexpr int BM = 128, BK = 16, TM = 8;
-constexpr int PITCH = BM + 4;  // transposed tiles: 16-B aligned rows, spread store banks
+// ---------------------------------------------------------------- SYR2K
+// PolyBench/GPU syr2k (Table 2; Table 3): the paper's 2-D CS
+// kernel. Per element, k ascending, with the evaluation order of R20:
+//   p = alpha*a[i][k], q = alpha*b[i][k], s = fmaf(p, b[j][k], q*a[j][k]), c = c + s.
+struct Syr2kArgs {
+  const float* A;
+  const float* B;
+  float* C;
+  int64_t n, m;
+  float alpha, beta;
+  Throttle t;
+};
 
-// One k-step of the 8 x 8 register tile: c[r][q] = fmaf(alpha*a_i[r], a_j[q], c[r][q]).
-__device__ __forceinline__ void syrk_kstep(float (&c)[TM][TM], const float* as, const float* bs, int ty, int tx) {
-  const float4 a0 = *reinterpret_cast<const float4*>(as + ty * TM);
-  const float4 a1 = *reinterpret_cast<const float4*>(as + ty * TM + 4);
-  const float4 b0 = *reinterpret_cast<const float4*>(bs + tx * TM);
-  const float4 b1 = *reinterpret_cast<const float4*>(bs + tx * TM + 4);
-  const float av[TM] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-  const float bv[TM] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
-#pragma unroll
-  for (int r = 0; r < TM; ++r)
-#pragma unroll
-    for (int q = 0; q < TM; ++q) c[r][q] = fmaf(av[r], bv[q], c[r][q]);
+__global__ void __launch_bounds__(1024, 2) syr2k_thread_kernel(Syr2kArgs a) {
+  __shared__ int slots;
+  gate_init(&slots, a.t);
+  __syncthreads();
+  cta_enter(a.t);
+  const int64_t j = int64_t(blockIdx.x) * 32 + threadIdx.x;
+  const int64_t i = int64_t(blockIdx.y) * blockDim.y + threadIdx.y;
+  throttled(a.t, &slots, [&]() {
+    if (i >= a.n || j >= a.n) return;
+    const int64_t m = a.m;
+    const float* __restrict__ ai = a.A + i * m;
+    const float* __restrict__ bi = a.B + i * m;
+    const float* __restrict__ aj = a.A + j * m;
+    const float* __restrict__ bj = a.B + j * m;
+    float c = __fmul_rn(a.C[i * a.n + j], a.beta);
+#pragma unroll 2
+    for (int64_t k = 0; k < m; ++k) {
+      const float p = __fmul_rn(a.alpha, ai[k]);
+      const float q = __fmul_rn(a.alpha, bi[k]);
+      const float s = fmaf(p, bj[k], __fmul_rn(q, aj[k]));
+      c = __fadd_rn(c, s);
+    }
+    a.C[i * a.n + j] = c;
+  });
+  cta_exit(a.t);
 }
 
-__global__ void __launch_bounds__(256, 2) syrk_tiled_kernel(SyrkArgs a) {
-  __shared__ __align__(16) float As[2][BK][PITCH];  // alpha * a[i][k], transposed
-  __shared__ __align__(16) float Bs[2][BK][PITCH];  // a[j][k], transposed
+// ---------------------------------------------------------------- tiled
+// STAGED SYRK / SYR2K: 128 x 128 output tile per 256-thread CTA, 8 x 8 outputs
+// per thread on rows {ty*4 + r, 64 + ty*4 + r} x cols {tx*4 + q, 64 + tx*4 + q}
+// (conflict-free float4 fragment reads), BK k per shared-memory stage, double-
+// buffered stages and double-buffered register fragments. Every output runs
+// k = 0, 1, ..., m-1 in order with the literal kernel's per-step rounding, so
+// the result is bit-identical to LITERAL (and to the oracle). Stage arrays:
+//   SYRK : 0 = alpha*a[i][k], 1 = a[j][k]
+//   SYR2K: 0 = alpha*a[i][k], 1 = b[j][k], 2 = alpha*b[i][k], 3 = a[j][k]
+constexpr int BM = 128, TM = 8;
+constexpr int PITCH = BM + 4;  // transposed stage rows: 16-B aligned, store banks spread
+
+struct TileArgs {
+  const float* A;
+  const float* B;  // SYR2K only
+  float* C;
+  int64_t n, m;
+  float alpha, beta;
+  int vec;  // m % 4 == 0 and A, B 16-B aligned: float4 global loads
+  int cvec; // n % 4 == 0 and C 16-B aligned
+  Throttle t;
+};
+
+template <bool TWO>
+struct TileCfg {
+  static constexpr int BK = TWO ? 8 : 16;
+  static constexpr int NA = TWO ? 4 : 2;
+  static constexpr int KQ = BK / 4;            // float4 per stage row
+  static constexpr int NV = BM * KQ / 256;     // float4 per thread per array per stage
+};
+
+__device__ __forceinline__ int tile_off(int t, int r) { return r < 4 ? t * 4 + r : 64 + t * 4 + (r - 4); }
+
+template <bool TWO, int MINB>
+__global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
+  using Cfg = TileCfg<TWO>;
+  constexpr int BK = Cfg::BK, NA = Cfg::NA, KQ = Cfg::KQ, NV = Cfg::NV;
+  __shared__ __align__(16) float S[2][NA][BK][PITCH];
   cta_enter(a.t);
   const int tid = threadIdx.x;
   const int tx = tid & 15, ty = tid >> 4;
   const int64_t i0 = int64_t(blockIdx.y) * BM, j0 = int64_t(blockIdx.x) * BM;
   const int64_t n = a.n, m = a.m;
-  // loader: thread -> row lr = tid / 2 of the tile, k sub-block (tid & 1) * 8 (two float4)
-  const int lr = tid >> 1, lk = (tid & 1) * 8;
-  const bool vec = (m % 4) == 0 && (reinterpret_cast<uintptr_t>(a.A) & 15u) == 0;
+
   float c[TM][TM];
 #pragma unroll
-  for (int r = 0; r < TM; ++r)
+  for (int r = 0; r < TM; ++r) {
+    const int64_t gi = i0 + tile_off(ty, r);
 #pragma unroll
-    for (int q = 0; q < TM; ++q) {
-      const int64_t gi = i0 + ty * TM + r, gj = j0 + tx * TM + q;
-      c[r][q] = (gi < n && gj < n) ? __fmul_rn(a.C[gi * n + gj], a.beta) : 0.0f;
+    for (int h = 0; h < 2; ++h) {
+      const int64_t gj = j0 + 64 * h + tx * 4;
+      if (a.cvec && gi < n && gj + 3 < n) {
+        const float4 v = *reinterpret_cast<const float4*>(a.C + gi * n + gj);
+        c[r][4 * h] = __fmul_rn(v.x, a.beta);
+        c[r][4 * h + 1] = __fmul_rn(v.y, a.beta);
+        c[r][4 * h + 2] = __fmul_rn(v.z, a.beta);
+        c[r][4 * h + 3] = __fmul_rn(v.w, a.beta);
+      } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          c[r][4 * h + q] = (gi < n && gj + q < n) ? __fmul_rn(a.C[gi * n + gj + q], a.beta) : 0.0f;
+      }
     }
-  float ra[8], rb[8];
+  }
+
+  // stage array s: source matrix, whether its row is the output row i (and
+  // pre-scaled by alpha) or the output column j
+  auto src = [&](int s) -> const float* { return (s == 0 || s == 3 || (!TWO && s == 1)) ? a.A : a.B; };
+  auto is_row = [](int s) { return s == 0 || s == 2; };
+  float4 ld[NA][NV];
   auto gload = [&](int64_t k0) {
-    const int64_t gi = i0 + lr, gj = j0 + lr, kb = k0 + lk;
-    if (vec && kb + 8 <= m) {
-      const float4* pa = reinterpret_cast<const float4*>(a.A + gi * m + kb);
-      const float4* pb = reinterpret_cast<const float4*>(a.A + gj * m + kb);
-      const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
-      const float4 a0 = gi < n ? pa[0] : z, a1 = gi < n ? pa[1] : z;
-      const float4 b0 = gj < n ? pb[0] : z, b1 = gj < n ? pb[1] : z;
-      ra[0] = __fmul_rn(a.alpha, a0.x); ra[1] = __fmul_rn(a.alpha, a0.y);
-      ra[2] = __fmul_rn(a.alpha, a0.z); ra[3] = __fmul_rn(a.alpha, a0.w);
-      ra[4] = __fmul_rn(a.alpha, a1.x); ra[5] = __fmul_rn(a.alpha, a1.y);
-      ra[6] = __fmul_rn(a.alpha, a1.z); ra[7] = __fmul_rn(a.alpha, a1.w);
-      rb[0] = b0.x; rb[1] = b0.y; rb[2] = b0.z; rb[3] = b0.w;
-      rb[4] = b1.x; rb[5] = b1.y; rb[6] = b1.z; rb[7] = b1.w;
-    } else {
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const int64_t k = kb + u;
-        ra[u] = (gi < n && k < m) ? __fmul_rn(a.alpha, a.A[gi * m + k]) : 0.0f;
-        rb[u] = (gj < n && k < m) ? a.A[gj * m + k] : 0.0f;
+    for (int v = 0; v < NV; ++v) {
+      const int idx = tid + v * 256;
+      const int row = idx / KQ;
+      const int64_t k = k0 + (idx % KQ) * 4;
+#pragma unroll
+      for (int s = 0; s < NA; ++s) {
+        const int64_t g = (is_row(s) ? i0 : j0) + row;
+        const float* M = src(s);
+        if (a.vec && g < n && k + 3 < m) {
+          ld[s][v] = __ldg(reinterpret_cast<const float4*>(M + g * m + k));
+        } else {
+          const bool ok = g < n;
+          ld[s][v].x = (ok && k < m) ? M[g * m + k] : 0.0f;
+          ld[s][v].y = (ok && k + 1 < m) ? M[g * m + k + 1] : 0.0f;
+          ld[s][v].z = (ok && k + 2 < m) ? M[g * m + k + 2] : 0.0f;
+          ld[s][v].w = (ok && k + 3 < m) ? M[g * m + k + 3] : 0.0f;
+        }
       }
     }
   };
   auto sstore = [&](int buf) {
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      As[buf][lk + u][lr] = ra[u];
-      Bs[buf][lk + u][lr] = rb[u];
+    for (int v = 0; v < NV; ++v) {
+      const int idx = tid + v * 256;
+      const int row = idx / KQ, kq = (idx % KQ) * 4;
+#pragma unroll
+      for (int s = 0; s < NA; ++s) {
+        float4 x = ld[s][v];
+        if (is_row(s)) {
+          x.x = __fmul_rn(a.alpha, x.x);
+          x.y = __fmul_rn(a.alpha, x.y);
+          x.z = __fmul_rn(a.alpha, x.z);
+          x.w = __fmul_rn(a.alpha, x.w);
+        }
+        S[buf][s][kq][row] = x.x;
+        S[buf][s][kq + 1][row] = x.y;
+        S[buf][s][kq + 2][row] = x.z;
+        S[buf][s][kq + 3][row] = x.w;
+      }
     }
   };
+  float f[2][NA][TM];
+  auto fload = [&](int fb, int buf, int kk) {
+#pragma unroll
+    for (int s = 0; s < NA; ++s) {
+      const int t = is_row(s) ? ty : tx;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const float4 v = *reinterpret_cast<const float4*>(&S[buf][s][kk][64 * h + t * 4]);
+        f[fb][s][4 * h] = v.x;
+        f[fb][s][4 * h + 1] = v.y;
+        f[fb][s][4 * h + 2] = v.z;
+        f[fb][s][4 * h + 3] = v.w;
+      }
+    }
+  };
+  auto fma_step = [&](int fb) {
+#pragma unroll
+    for (int r = 0; r < TM; ++r)
+#pragma unroll
+      for (int q = 0; q < TM; ++q) {
+        if constexpr (TWO)
+          c[r][q] = __fadd_rn(c[r][q], fmaf(f[fb][0][r], f[fb][1][q], __fmul_rn(f[fb][2][r], f[fb][3][q])));
+        else
+          c[r][q] = fmaf(f[fb][0][r], f[fb][1][q], c[r][q]);
+      }
+  };
+
   const int64_t ktiles = (m + BK - 1) / BK;
-  gload(0);
-  sstore(0);
-  __syncthreads();
+  if (ktiles > 0) {
+    gload(0);
+    sstore(0);
+    __syncthreads();
+    fload(0, 0, 0);
+  }
   for (int64_t kt = 0; kt < ktiles; ++kt) {
     const int buf = int(kt & 1);
-    if (kt + 1 < ktiles) gload((kt + 1) * BK);
-    const int kvalid = int(imin64(BK, m - kt * BK));  // uniform: never run k >= m
+    const bool more = kt + 1 < ktiles;
+    if (more) gload((kt + 1) * BK);
+    const int kvalid = int(imin64(BK, m - kt * BK));
     if (kvalid == BK) {
 #pragma unroll
-      for (int kk = 0; kk < BK; ++kk) syrk_kstep(c, &As[buf][kk][0], &Bs[buf][kk][0], ty, tx);
-    } else {
-      for (int kk = 0; kk < kvalid; ++kk) syrk_kstep(c, &As[buf][kk][0], &Bs[buf][kk][0], ty, tx);
+      for (int kk = 0; kk < BK; ++kk) {
+        if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
+        fma_step(kk & 1);
+      }
+    } else {  // ragged last stage: exactly kvalid steps
+      fma_step(0);
+      for (int kk = 1; kk < kvalid; ++kk) {
+        fload(0, buf, kk);
+        fma_step(0);
+      }
     }
-    if (kt + 1 < ktiles) sstore(buf ^ 1);
-    __syncthreads();
+    if (more) {
+      sstore(buf ^ 1);
+      __syncthreads();
+      fload(0, buf ^ 1, 0);
+    }
   }
+
 #pragma unroll
   for (int r = 0; r < TM; ++r) {
-    const int64_t gi = i0 + ty * TM + r;
+    const int64_t gi = i0 + tile_off(ty, r);
     if (gi >= n) continue;
-    float* crow = a.C + gi * n + j0 + tx * TM;
-    if (j0 + tx * TM + TM <= n && (n % 4) == 0) {
-      reinterpret_cast<float4*>(crow)[0] = make_float4(c[r][0], c[r][1], c[r][2], c[r][3]);
-      reinterpret_cast<float4*>(crow)[1] = make_float4(c[r][4], c[r][5], c[r][6], c[r][7]);
-    } else {
 #pragma unroll
-      for (int q = 0; q < TM; ++q)
-        if (j0 + tx * TM + q < n) crow[q] = c[r][q];
+    for (int h = 0; h < 2; ++h) {
+      const int64_t gj = j0 + 64 * h + tx * 4;
+      if (a.cvec && gj + 3 < n) {
+        *reinterpret_cast<float4*>(a.C + gi * n + gj) =
+            make_float4(c[r][4 * h], c[r][4 * h + 1], c[r][4 * h + 2], c[r][4 * h + 3]);
+      } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (gj + q < n) a.C[gi * n + gj + q] = c[r][4 * h + q];
+      }
     }
   }
   cta_exit(a.t);
 }
 
+// Register budget per kernel: MINB = 1 (up to 255 registers, one 256-thread
+// CTA per SM) or 2 (128 registers). CATT_TILED_MINB overrides (tools only).
+static int tiled_minb(bool two) {
+  static const int env = [] {
+    const char* e = getenv("CATT_TILED_MINB");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 1 || env == 2) return env;
+  return 1;
+  (void)two;
+}
+
+template <bool TWO>
+static const void* tiled_func() {
+  return tiled_minb(TWO) == 2 ? (const void*)tiled_kernel<TWO, 2> : (const void*)tiled_kernel<TWO, 1>;
+}
+
+template <bool TWO>
+static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t s) {
+  if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
+  size_t dyn = 0;
+  catt_status st = prepare_launch(tiled_func<TWO>(), t, 256, 0, false, &a.t, &dyn);
+  if (st != CATT_OK) return st;
+  const int64_t tiles = (a.n + BM - 1) / BM;
+  if (tiles > 65535) return CATT_EINVAL;
+  auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
+  a.vec = (a.m % 4 == 0) && al(a.A) && (!TWO || al(a.B));
+  a.cvec = (a.n % 4 == 0) && al(a.C);
+  const dim3 grid{unsigned(tiles), unsigned(tiles), 1u};
+  if (tiled_minb(TWO) == 2)
+    tiled_kernel<TWO, 2><<<grid, 256, dyn, s>>>(a);
+  else
+    tiled_kernel<TWO, 1><<<grid, 256, dyn, s>>>(a);
+  return after_launch();
+}
+
 const void* syrk_func(int variant) {
-  return variant == CATT_VAR_STAGED ? (const void*)syrk_tiled_kernel : (const void*)syrk_thread_kernel;
+  return variant == CATT_VAR_STAGED ? tiled_func<false>() : (const void*)syrk_thread_kernel;
+}
+
+const void* syr2k_func(int variant) {
+  return variant == CATT_VAR_STAGED ? tiled_func<true>() : (const void*)syr2k_thread_kernel;
 }
 
 }  // namespace catt
@@ -156,7 +329,7 @@ using namespace catt;
 extern "C" catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta,
                                  const catt_throttle* t, void* stream) {
   if (n < 0 || m < 0 || n > (int64_t(1) << 31) || m > (int64_t(1) << 31)) return CATT_EINVAL;
-  if (n > 0 && (!A || !C)) return CATT_EINVAL;
+  if (n > 0 && (!C || (m > 0 && !A))) return CATT_EINVAL;  // A is never read when m == 0
   if (n == 0) return CATT_OK;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   SyrkArgs a{A, C, n, m, alpha, beta, Throttle{}};
@@ -173,15 +346,30 @@ extern "C" catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m,
     syrk_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) {
-    if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
+  if (var == CATT_VAR_STAGED) return launch_tiled<false>(TileArgs{A, nullptr, C, n, m, alpha, beta, 0, 0, {}}, t, s);
+  return CATT_EINVAL;
+}
+
+extern "C" catt_status catt_syr2k(const float* A, const float* B, float* C, int64_t n, int64_t m, float alpha,
+                                  float beta, const catt_throttle* t, void* stream) {
+  if (n < 0 || m < 0 || n > (int64_t(1) << 31) || m > (int64_t(1) << 31)) return CATT_EINVAL;
+  if (n > 0 && (!C || (m > 0 && (!A || !B)))) return CATT_EINVAL;  // A, B unread when m == 0
+  if (n == 0) return CATT_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  Syr2kArgs a{A, B, C, n, m, alpha, beta, Throttle{}};
+  const int var = variant_of(t);
+  if (var == CATT_VAR_LITERAL) {
+    const int threads = cta_threads_or(t, 256);
+    if (threads % 32) return CATT_EINVAL;
+    const int by = threads / 32;
     size_t dyn = 0;
-    catt_status st = prepare_launch((const void*)syrk_tiled_kernel, t, 256, 0, false, &a.t, &dyn);
+    catt_status st = prepare_launch((const void*)syr2k_thread_kernel, t, threads, 0, true, &a.t, &dyn);
     if (st != CATT_OK) return st;
-    dim3 grid(unsigned((n + BM - 1) / BM), unsigned((n + BM - 1) / BM));
+    dim3 grid(unsigned((n + 31) / 32), unsigned((n + by - 1) / by));
     if (grid.y > 65535) return CATT_EINVAL;
-    syrk_tiled_kernel<<<grid, 256, dyn, s>>>(a);
+    syr2k_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
+  if (var == CATT_VAR_STAGED) return launch_tiled<true>(TileArgs{A, B, C, n, m, alpha, beta, 0, 0, {}}, t, s);
   return CATT_EINVAL;
 }

@@ -16,6 +16,7 @@ int col_tma_stages(int cols, int rows_per_stage);
 int row_tma_stage_bytes(int nmat, int rows, int boxes);
 int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
+const void* syr2k_func(int variant);
 const void* kmeans_func(int variant, int nf);
 const void* fused_func(bool dep);
 
@@ -214,7 +215,7 @@ catt_ref mkref(int64_t cx, int64_t cy, int64_t c0, int64_t c1, int32_t e, int32_
 }
 
 int default_threads(int loop, int variant) {
-  if (variant == CATT_VAR_STAGED) return loop == CATT_K_SYRK ? 256 : 32;
+  if (variant == CATT_VAR_STAGED) return (loop == CATT_K_SYRK || loop == CATT_K_SYR2K) ? 256 : 32;
   if (variant == CATT_VAR_COOP && (loop == CATT_K_ATAX_2 || loop == CATT_K_BICG_1 || loop == CATT_K_MVT_2)) return 1024;
   return 256;
 }
@@ -228,6 +229,7 @@ const void* loop_func(const catt_problem& p, int variant) {
   if (variant == CATT_VAR_FUSED && (is_row(p.loop) || is_col(p.loop))) return fused_func(p.loop == CATT_K_ATAX_1 || p.loop == CATT_K_ATAX_2);
   if (is_row(p.loop) || is_col(p.loop)) return gemv_func(p.loop, variant, true);
   if (p.loop == CATT_K_SYRK) return syrk_func(variant);
+  if (p.loop == CATT_K_SYR2K) return syr2k_func(variant);
   return kmeans_func(variant, int(p.n));
 }
 
@@ -375,6 +377,31 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->grid[0] = (N + 127) / 128;
       out->grid[1] = (N + 127) / 128;
       refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);                     // staged through shared memory
+    } else {
+      return CATT_EINVAL;
+    }
+  } else if (loop == CATT_K_SYR2K) {
+    const int64_t N = prob->n, Mk = prob->k;
+    if (N < 1 || Mk < 1) return CATT_EINVAL;
+    out->n_loops = 1;
+    out->trip[0] = Mk;
+    if (var == CATT_VAR_LITERAL) {
+      const int by = threads / 32;
+      out->block[0] = 32;
+      out->block[1] = by;
+      out->grid[0] = (N + 31) / 32;
+      out->grid[1] = (N + by - 1) / by;
+      out->extent[0] = N;
+      out->extent[1] = N;
+      refs[n++] = mkref(0, Mk, 1, 0, 4, 1, 0);                     // a[i*M + k]
+      refs[n++] = mkref(0, Mk, 1, 0, 4, 2, 0);                     // b[i*M + k]
+      refs[n++] = mkref(Mk, 0, 1, 0, 4, 1, 0);                     // a[j*M + k]
+      refs[n++] = mkref(Mk, 0, 1, 0, 4, 2, 0);                     // b[j*M + k]
+    } else if (var == CATT_VAR_STAGED) {
+      out->block[0] = 256;
+      out->grid[0] = (N + 127) / 128;
+      out->grid[1] = (N + 127) / 128;
+      refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);
     } else {
       return CATT_EINVAL;
     }

@@ -171,6 +171,7 @@ KERNEL_CASES = [
     ("kmeans", catt.problem(catt.K_KMEANS, m=2040, n=6, k=3, ld=2044), catt.Throttle(cta_threads=128),
      lru.KmeansKernel(2040, 6, 3, 2044, 128)),
     ("syrk", catt.problem(catt.K_SYRK, n=128, k=64), catt.Throttle(), lru.SyrkKernel(128, 64)),
+    ("syr2k", catt.problem(catt.K_SYR2K, n=128, k=64), catt.Throttle(), lru.Syr2kKernel(128, 64)),
 ]
 
 

@@ -207,6 +207,54 @@ def test_syrk_throttled():
         assert bits_equal(host(Cd), C_o)
 
 
+# ------------------------------------------------------------------ SYR2K
+@pytest.mark.parametrize("variant", ["literal", "staged"])
+@pytest.mark.parametrize("n,m", [(64, 40), (130, 37), (257, 8), (256, 256), (1, 3)])
+def test_syr2k_exact(variant, n, m):
+    A, B, C = si.matrix(8, n, m), si.matrix(108, n, m), si.matrix(208, n, n)
+    C_o = oracle.syr2k(A, B, C, 1.5, 1.2)
+    Cd = dev(C)
+    catt.syr2k(dev(A), dev(B), Cd, 1.5, 1.2, t=catt.Throttle(variant=variant))
+    assert bits_equal(host(Cd), C_o)
+
+
+def test_syr2k_empty_inner_and_throttled():
+    n = 96
+    C = si.matrix(208, n, n)
+    Cd = dev(C)
+    z = torch.empty(n, 0, device="cuda")
+    catt.syr2k(z, z, Cd, 1.5, 1.25)
+    assert bits_equal(host(Cd), (C * np.float32(1.25)).astype(np.float32))
+    A, B = si.matrix(8, n, 64), si.matrix(108, n, 64)
+    C_o = oracle.syr2k(A, B, C, 1.5, 1.2)
+    for t in (catt.Throttle(active_warps=2), catt.Throttle(active_warps=4, active_ctas=2),
+              catt.Throttle(cta_threads=512, active_warps=4, gate=catt.GATE_BARRIER),
+              catt.Throttle(variant="staged", active_ctas=1)):
+        Cd = dev(C)
+        catt.syr2k(dev(A), dev(B), Cd, 1.5, 1.2, t=t)
+        assert bits_equal(host(Cd), C_o)
+
+
+def test_syr2k_2048_sampled_rows():
+    """Table 2 P:77 size, both variants, rows spanning tile edges."""
+    n = m = 2048
+    A = torch.empty(n * m, device="cuda")
+    B = torch.empty(n * m, device="cuda")
+    C = torch.empty(n * n, device="cuda")
+    catt.fill_hash(A, si.SEED_SYR2K)
+    catt.fill_hash(B, si.sub_seed(si.SEED_SYR2K, 1))
+    catt.fill_hash(C, si.sub_seed(si.SEED_SYR2K, 2))
+    Ah = oracle.fill(si.SEED_SYR2K, n * m).reshape(n, m)
+    Bh = oracle.fill(si.sub_seed(si.SEED_SYR2K, 1), n * m).reshape(n, m)
+    Ch = oracle.fill(si.sub_seed(si.SEED_SYR2K, 2), n * n).reshape(n, n)
+    rows = np.array([0, 7, 127, 128, 1111, 2047])
+    want = oracle.syr2k_rows(Ah, Bh, Ch, 1.5, 1.2, rows)
+    for v in ("literal", "staged"):
+        Cd = C.clone().view(n, n)
+        catt.syr2k(A.view(n, m), B.view(n, m), Cd, 1.5, 1.2, t=catt.Throttle(variant=v))
+        assert bits_equal(host(Cd)[rows], want), v
+
+
 # ------------------------------------------------------------------ KMEANS
 @pytest.mark.parametrize("variant", ["literal", "regs", "staged"])
 @pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 4), (4099, 34, 5, 29), (257, 7, 3, 3), (300, 50, 12, 4),

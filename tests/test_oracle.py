@@ -167,6 +167,27 @@ def test_syrk_rows_equals_full_rows():
     assert np.array_equal(oracle.syrk_rows(A, C, 1.5, 1.2, rows), full[rows])
 
 
+def test_syr2k_vs_numpy_and_special_cases():
+    n, m = 60, 37
+    A, B, C = si.matrix(8, n, m), si.matrix(108, n, m), si.matrix(208, n, n)
+    out = oracle.syr2k(A, B, C, 1.5, 1.2)
+    A64, B64 = A.astype(np.float64), B.astype(np.float64)
+    ref = 1.2 * C.astype(np.float64) + 1.5 * (A64 @ B64.T + B64 @ A64.T)
+    assert _rel(out, ref) < 4 * m * 2.0 ** -24
+    # swapping A and B gives the same matrix mathematically (A B^T + B A^T)
+    assert _rel(oracle.syr2k(B, A, C, 1.5, 1.2), ref) < 4 * m * 2.0 ** -24      # symmetric in (A, B) mathematically
+    # B = 0 -> beta * C exactly (every s is 0); alpha = 0 likewise
+    assert np.array_equal(oracle.syr2k(A, np.zeros_like(B), C, 1.5, 1.2), (C * np.float32(1.2)).astype(np.float32))
+    # exact dyadic inputs: bit-equal to float64 (alpha = 1.5, beta = 1.25 dyadic)
+    D = si.MODE_DYADIC
+    Ad, Bd, Cd = si.matrix(9, n, m, D), si.matrix(109, n, m, D), si.matrix(209, n, n, D)
+    refd = 1.25 * Cd.astype(np.float64) + 1.5 * (Ad.astype(np.float64) @ Bd.T.astype(np.float64)
+                                                 + Bd.astype(np.float64) @ Ad.T.astype(np.float64))
+    assert np.array_equal(oracle.syr2k(Ad, Bd, Cd, 1.5, 1.25), refd.astype(np.float32))
+    rows = np.array([0, 17, 59])
+    assert np.array_equal(oracle.syr2k_rows(A, B, C, 1.5, 1.2, rows), out[rows])
+
+
 def test_kmeans_vs_bruteforce_argmin():
     npts, nf, k = 1000, 34, 5
     ld = npts + 3                                         # misaligned leading dimension
