@@ -49,7 +49,8 @@ typedef enum {
   CATT_ECUDA = -2,        /* CUDA runtime error (see catt_last_cuda_error)  */
   CATT_EUNSUPPORTED = -3, /* valid but not supported (e.g. window too big)  */
   CATT_ENOMEM = -4,       /* library workspace allocation failed            */
-  CATT_ENODEV = -5        /* no CUDA device                                 */
+  CATT_ENODEV = -5,       /* no CUDA device                                 */
+  CATT_EINEXACT = -6      /* KMEANS sums: a value outside the exact range   */
 } catt_status;
 
 enum { CATT_MAX_LOOPS = 4, CATT_MAX_CARVEOUTS = 16 };
@@ -197,7 +198,8 @@ enum {
   CATT_K_SYRK = 7,    /* C = beta C + alpha A A^T (2-D block 32 x 8)          */
   CATT_K_KMEANS = 8,  /* membership = argmin_c |f_p - c|^2, feature-major     */
   CATT_K_SYR2K = 9,   /* C = beta C + alpha (A B^T + B A^T), 2-D block 32 x 8 */
-  CATT_K_COUNT = 10
+  CATT_K_KMEANS_T = 10, /* KM transpose: out[f*ld + p] = in[p*nf + f]          */
+  CATT_K_COUNT = 11
 };
 
 /* Problem sizes: ATAX/BICG m x n (rows, cols); MVT/GESUMMV n (m ignored);
@@ -279,6 +281,64 @@ catt_status catt_syr2k(const float* A, const float* B, float* C, int64_t n, int6
  * Requires nf * k <= 4096 (the centres are staged in shared memory). */
 catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters,
                                int32_t k, int32_t* membership, const catt_throttle* t, void* stream);
+
+/* ------------------------------------------------------------------ KMEANS iteration
+ * the steps around the assignment (Rodinia kmeans; the KM
+ * rows of Table 3 P:338-339 are its two loops). DESIGN.md reading R21.
+ *
+ * Transpose (KM's other loop): out[f*ld + p] = in[p*nf + f] for p < npoints,
+ * f < nf; in is point-major (npoints x nf), out feature-major with ld >=
+ * npoints (columns >= npoints untouched). Variants: LITERAL (thread per
+ * point, the divergent CATT loop CATT_K_KMEANS_T, throttle honoured) and COOP
+ * (256-point shared-memory tiles, coalesced; no throttle). Bit-exact copy.
+ *
+ * Exact centroid sums. acc is a device int64 array of
+ * catt_kmeans_acc_words(k, nf) = 4*k*nf + k + 2 words:
+ *   acc[(c*nf + f)*4 + l], l < 4  limbs of the sum, over the points assigned to
+ *                                 c, of feature f as the two's-complement
+ *                                 128-bit integer v = x * 2^64. Each 128-bit
+ *                                 partial is split v = l0 + l1*2^32 + l2*2^64 +
+ *                                 l3*2^96 (l0..l2 unsigned 32-bit chunks, l3 a
+ *                                 signed 32-bit chunk) and chunk l is added to
+ *                                 limb l. The sum is S = sum_l acc[..+l]*2^(32l).
+ *   acc[4*k*nf + c]               points assigned to c
+ *   acc[4*k*nf + k]               delta: points whose membership changed
+ *   acc[4*k*nf + k + 1]           inexact: feature values not representable
+ *                                 (non-zero bits below 2^-64, |x| >= 2^31,
+ *                                 subnormal, inf, NaN); 0 means S is exact
+ * All limbs are integer sums, so adding acc arrays (e.g. an integer
+ * all-reduce across GPUs, each holding a shard of the points) gives exactly
+ * the acc of the whole point set. Limits: nf <= 64, k <= 16, npoints < 2^31. */
+int64_t catt_kmeans_acc_words(int32_t k, int32_t nf);
+catt_status catt_kmeans_transpose(const float* in, float* out, int64_t npoints, int32_t nf, int64_t ld,
+                                  const catt_throttle* t, void* stream);
+
+/* One pass over the points: assignment exactly as catt_kmeans_assign (reading
+ * membership's previous value first: -1 = none), then acc += the point's
+ * features into its centre's sums, counts and delta. acc is accumulated into
+ * (zero it before the first pass). */
+catt_status catt_kmeans_accumulate(const float* feat, int64_t ld, int64_t npoints, int32_t nf,
+                                   const float* clusters, int32_t k, int32_t* membership, int64_t* acc,
+                                   void* stream);
+
+/* clusters[c][f] = round-to-nearest-even fp32 of (S * 2^-64) / count[c] when
+ * count[c] > 0, else unchanged (a centre without points keeps its value).
+ * stats (device int64[3], may be NULL) receives {delta, inexact, sum of
+ * counts}. zero_acc != 0 zeroes acc afterwards (ready for the next pass). */
+catt_status catt_kmeans_finalize(int64_t* acc, int32_t k, int32_t nf, float* clusters, int64_t* stats,
+                                 int32_t zero_acc, void* stream);
+
+/* The k-means loop on one GPU: membership := -1, then up to max_iter
+ * iterations of accumulate + finalize; stops after the first iteration whose
+ * delta <= max_changes. clusters (k x nf, in: initial centres, out: final).
+ * ws: device int64 workspace of catt_kmeans_acc_words(k, nf) + 4 words.
+ * Iterations are queued without host round trips (a device-side done flag
+ * turns the remaining queued passes into no-ops); the call synchronizes the
+ * stream and writes the iteration count to *iterations (host, may be NULL).
+ * Returns CATT_EINEXACT when any sum was not exact. */
+catt_status catt_kmeans(const float* feat, int64_t ld, int64_t npoints, int32_t nf, float* clusters, int32_t k,
+                        int32_t* membership, int32_t max_iter, int64_t max_changes, int64_t* ws,
+                        int32_t* iterations, void* stream);
 
 /* ------------------------------------------------------------------ single loops
  * CATT throttles per loop: these run one loop each and

@@ -18,7 +18,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libcatt.so")
 
 # ------------------------------------------------------------------ constants (catt.h)
-OK, EINVAL, ECUDA, EUNSUPPORTED, ENOMEM, ENODEV = 0, -1, -2, -3, -4, -5
+OK, EINVAL, ECUDA, EUNSUPPORTED, ENOMEM, ENODEV, EINEXACT = 0, -1, -2, -3, -4, -5, -6
 MAX_LOOPS, MAX_CARVEOUTS = 4, 16
 REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
 MODE_UNION, MODE_PAPER = 0, 1
@@ -27,7 +27,8 @@ VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED = 0, 1, 2, 3, 4
 ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
-(K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K) = range(10)
+(K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K,
+ K_KMEANS_T) = range(11)
 
 VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS,
             "fused": VAR_FUSED}
@@ -162,6 +163,10 @@ def lib():
             "catt_syrk": [V, V, i64, i64, f32, f32, T, V],
             "catt_syr2k": [V, V, V, i64, i64, f32, f32, T, V],
             "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
+            "catt_kmeans_transpose": [V, V, i64, i32, i64, T, V],
+            "catt_kmeans_accumulate": [V, i64, i64, i32, V, i32, V, V, V],
+            "catt_kmeans_finalize": [V, i32, i32, V, V, i32, V],
+            "catt_kmeans": [V, i64, i64, i32, V, i32, V, i32, i64, V, P(i32), V],
             "catt_rows": [V, V, V, V, V, i64, i64, f32, f32, i32, T, V],
             "catt_dual": [V, V, V, V, V, i64, i64, i32, i32, i32, T, V],
             "catt_dual_group": [P(DualProblem), i32, i32, T, V],
@@ -178,13 +183,16 @@ def lib():
             fn.argtypes = args
             fn.restype = ctypes.c_int
         L.catt_status_str.restype = ctypes.c_char_p
+        L.catt_kmeans_acc_words.argtypes = [i32, i32]
+        L.catt_kmeans_acc_words.restype = ctypes.c_int64
         _lib = L
     return _lib
 
 
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_kmeans_assign",
-            "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
+            "catt_kmeans_acc_words", "catt_kmeans_transpose", "catt_kmeans_accumulate", "catt_kmeans_finalize",
+            "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version"]
 
 
@@ -417,6 +425,52 @@ def kmeans_assign(feat, ld, npoints, nf, clusters, membership=None, t: Optional[
                                     _dev(membership, "membership", torch.int32), _tp(t), _stream()),
            "catt_kmeans_assign")
     return membership
+
+
+def kmeans_acc_words(k: int, nf: int) -> int:
+    """Length of the exact-sum buffer (catt_kmeans_acc_words)."""
+    return int(lib().catt_kmeans_acc_words(k, nf))
+
+
+def kmeans_transpose(feat_pm, npoints, nf, out, ld, t: Optional[Throttle] = None):
+    """out[f*ld + p] = feat_pm[p*nf + f] (catt_kmeans_transpose). Returns out."""
+    _check(lib().catt_kmeans_transpose(_dev(feat_pm, "in"), _dev(out, "out"), npoints, nf, ld, _tp(t), _stream()),
+           "catt_kmeans_transpose")
+    return out
+
+
+def kmeans_accumulate(feat, ld, npoints, nf, clusters, membership, acc):
+    """Assignment + exact centroid sums into acc (catt_kmeans_accumulate)."""
+    torch = _torch()
+    _check(lib().catt_kmeans_accumulate(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"),
+                                        clusters.shape[0], _dev(membership, "membership", torch.int32),
+                                        _dev(acc, "acc", torch.int64), _stream()), "catt_kmeans_accumulate")
+
+
+def kmeans_finalize(acc, clusters, stats=None, zero_acc=True):
+    """clusters := exact means from acc (catt_kmeans_finalize)."""
+    torch = _torch()
+    k, nf = clusters.shape
+    sp = _dev(stats, "stats", torch.int64) if stats is not None else None
+    _check(lib().catt_kmeans_finalize(_dev(acc, "acc", torch.int64), k, nf, _dev(clusters, "clusters"), sp,
+                                      int(bool(zero_acc)), _stream()), "catt_kmeans_finalize")
+    return clusters
+
+
+def kmeans(feat, ld, npoints, nf, clusters, membership=None, max_iter=500, max_changes=0, ws=None):
+    """The k-means loop on one GPU (catt_kmeans); clusters updated in place.
+    Returns (membership, iterations)."""
+    torch = _torch()
+    k = clusters.shape[0]
+    if membership is None:
+        membership = torch.empty(npoints, dtype=torch.int32, device=feat.device)
+    if ws is None:
+        ws = torch.empty(kmeans_acc_words(k, nf) + 4, dtype=torch.int64, device=feat.device)
+    it = ctypes.c_int32(0)
+    _check(lib().catt_kmeans(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"), k,
+                             _dev(membership, "membership", torch.int32), max_iter, max_changes,
+                             _dev(ws, "ws", torch.int64), ctypes.byref(it), _stream()), "catt_kmeans")
+    return membership, it.value
 
 
 def fill_hash(t, seed: int, offset: int = 0, mode: int = 0):

@@ -18,6 +18,7 @@ int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
 const void* syr2k_func(int variant);
 const void* kmeans_func(int variant, int nf);
+const void* kmeans_t_func(int variant);
 const void* fused_func(bool dep);
 
 namespace {
@@ -230,6 +231,7 @@ const void* loop_func(const catt_problem& p, int variant) {
   if (is_row(p.loop) || is_col(p.loop)) return gemv_func(p.loop, variant, true);
   if (p.loop == CATT_K_SYRK) return syrk_func(variant);
   if (p.loop == CATT_K_SYR2K) return syr2k_func(variant);
+  if (p.loop == CATT_K_KMEANS_T) return kmeans_t_func(variant);
   return kmeans_func(variant, int(p.n));
 }
 
@@ -405,6 +407,22 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
     } else {
       return CATT_EINVAL;
     }
+  } else if (loop == CATT_K_KMEANS_T) {
+    const int64_t np = prob->m, nf = prob->n, ld = prob->ld;
+    if (np < 1 || nf < 1 || ld < np) return CATT_EINVAL;
+    out->grid[0] = (np + threads - 1) / threads;
+    out->extent[0] = np;
+    out->n_loops = 1;
+    out->trip[0] = nf;
+    if (var == CATT_VAR_LITERAL) {
+      refs[n++] = mkref(nf, 0, 1, 0, 4, 1, 0);                     // in[p*nf + f]: divergent, reused over f
+      refs[n++] = mkref(1, 0, ld, 0, 4, 2, CATT_REF_STORE);        // out[f*ld + p]
+    } else if (var == CATT_VAR_COOP) {
+      dyn = 256 * (nf | 1) * 4;
+      refs[n++] = mkref(0, 0, 1, 0, 4, 1, CATT_REF_NOT_L1);        // shared-memory tile
+    } else {
+      return CATT_EINVAL;
+    }
   } else {  // KMEANS
     const int64_t np = prob->m, nf = prob->n, k = prob->k, ld = prob->ld;
     if (np < 1 || nf < 1 || k < 1 || ld < np) return CATT_EINVAL;
@@ -546,6 +564,7 @@ extern "C" const char* catt_status_str(catt_status s) {
     case CATT_EUNSUPPORTED: return "unsupported";
     case CATT_ENOMEM: return "out of memory";
     case CATT_ENODEV: return "no CUDA device";
+    case CATT_EINEXACT: return "inexact: a KMEANS feature value outside the exact fixed-point range";
   }
   return "unknown status";
 }

@@ -10,6 +10,10 @@ all_reduce(SUM) -- the only exchange these loops have:
     MVT    x1_g += A_g y1 (local),     x2 = x2 + sum_g A_g^T y2_g   (all-reduce;
            only rank 0 adds the initial x2, so the sum carries it once)
     GESUMMV y_g = alpha A_g x + beta B_g x (local, no collective)
+    KMEANS points sharded; per iteration the exact centroid sums (int64 limbs,
+           counts, delta) are all-reduced, then every rank finalizes the
+           same centres. Integer sums: the result is
+           bit-identical at any world size.
 
 The per-rank loop calls are injected (`ops`), so the partitioning and the
 collective composition can be tested on CPU over gloo with any loop
@@ -39,6 +43,14 @@ class CudaOps:
     @staticmethod
     def cols(A, v, y, accumulate, t=None):
         return catt.cols(A, v, y, accumulate, t=t)
+
+    @staticmethod
+    def kmeans_accumulate(feat, ld, npoints, nf, clusters, memb, acc):
+        catt.kmeans_accumulate(feat, ld, npoints, nf, clusters, memb, acc)
+
+    @staticmethod
+    def kmeans_finalize(acc, clusters, stats):
+        catt.kmeans_finalize(acc, clusters, stats, zero_acc=True)
 
 
 def _reduce(t, group):
@@ -94,3 +106,29 @@ def gesummv_rowshard(A_g, B_g, x, alpha, beta, y_g=None, tmp_g=None, t=None, ops
     tmp_g = torch.empty(m, dtype=A_g.dtype, device=A_g.device) if tmp_g is None else tmp_g
     ops.rows(A_g, x, y_g, catt.ROWS_GESUMMV, t, B=B_g, tmp=tmp_g, alpha=alpha, beta=beta)
     return y_g, tmp_g
+
+
+def kmeans_pointshard(feat_g, ld_g, npoints_g, nf, clusters, memb_g=None, max_iter=500, max_changes=0, group=None,
+                      ops=CudaOps):
+    """k-means over points sharded across ranks. feat_g is this rank's points,
+    feature-major (feat_g[f*ld_g + p]); clusters (k x nf) is replicated and
+    updated in place. Per iteration: assignment + exact sums on the local
+    points, all_reduce(SUM) of the int64 sums/counts/delta (the iteration's
+    one exchange), then every rank rounds the same means. Returns
+    (memb_g, iterations)."""
+    import torch
+    k = clusters.shape[0]
+    acc = torch.zeros(catt.kmeans_acc_words(k, nf), dtype=torch.int64, device=clusters.device)
+    stats = torch.zeros(3, dtype=torch.int64, device=clusters.device)
+    if memb_g is None:
+        memb_g = torch.empty(npoints_g, dtype=torch.int32, device=clusters.device)
+    memb_g.fill_(-1)
+    it = 0
+    while it < max_iter:
+        ops.kmeans_accumulate(feat_g, ld_g, npoints_g, nf, clusters, memb_g, acc)
+        _reduce(acc, group)
+        ops.kmeans_finalize(acc, clusters, stats)
+        it += 1
+        if int(stats[0].item()) <= max_changes:            # global delta (all-reduced)
+            break
+    return memb_g, it

@@ -20,7 +20,7 @@ GOLDEN = os.path.join(ROOT, "tests", "golden")
 def test_library_loads_and_exports_every_declared_symbol():
     L = catt.lib()
     header = open(os.path.join(ROOT, "include", "catt.h")).read()
-    declared = set(re.findall(r"^\s*(?:catt_status|const char\*|int)\s+(catt_\w+)\s*\(", header, re.M))
+    declared = set(re.findall(r"^\s*(?:catt_status|const char\*|int64_t|int)\s+(catt_\w+)\s*\(", header, re.M))
     assert declared == set(catt.catt.EXPORTED)
     for name in declared:
         assert hasattr(L, name), name

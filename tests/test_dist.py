@@ -65,6 +65,56 @@ class OracleOps:
         return y
 
 
+class OracleKmeansOps:
+    """Per-rank k-means steps by the oracle, writing the exact sums in the
+    acc layout catt.h defines (the 128-bit two's complement of sum*2^64 as
+    four 32-bit chunks, the top one signed), so that the all-reduce and the
+    finalize composition of dist.kmeans_pointshard are what is tested."""
+
+    @staticmethod
+    def kmeans_accumulate(feat, ld, npoints, nf, clusters, memb, acc):
+        from oracle import kmeans as okm
+        cl = clusters.numpy()
+        k = cl.shape[0]
+        new, _ = oracle.kmeans_assign(feat.numpy(), ld, npoints, nf, cl)
+        old = memb.numpy().copy()
+        memb.copy_(torch.from_numpy(new))
+        fe = feat.numpy()
+        a = acc.numpy()
+        K4 = 4 * k * nf
+        for c in range(k):
+            sel = np.nonzero(new == c)[0]
+            a[K4 + c] += len(sel)
+            for f in range(nf):
+                v = okm.exact_sum(fe[f * ld + sel]) * 2 ** 64
+                assert v.denominator == 1
+                u = int(v) % (1 << 128)
+                for l in range(4):
+                    chunk = (u >> (32 * l)) & 0xFFFFFFFF
+                    if l == 3 and chunk >= 1 << 31:
+                        chunk -= 1 << 32
+                    a[(c * nf + f) * 4 + l] += chunk
+        a[K4 + k] += int(np.count_nonzero(new != old))
+
+    @staticmethod
+    def kmeans_finalize(acc, clusters, stats):
+        from fractions import Fraction
+        from oracle import kmeans as okm
+        a = acc.numpy()
+        cl = clusters.numpy()
+        k, nf = cl.shape
+        K4 = 4 * k * nf
+        for c in range(k):
+            cnt = int(a[K4 + c])
+            if cnt == 0:
+                continue
+            for f in range(nf):
+                S = sum(int(a[(c * nf + f) * 4 + l]) << (32 * l) for l in range(4))
+                cl[c, f] = okm.round_f32(Fraction(S, cnt << 64))
+        stats[0], stats[1], stats[2] = int(a[K4 + k]), int(a[K4 + k + 1]), int(a[K4:K4 + k].sum())
+        acc.zero_()
+
+
 def _free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
@@ -136,6 +186,45 @@ def test_rowshard_world2_gloo(mode):
                               si.values(13, n, mode=mode), si.values(14, n, mode=mode), mode=oracle.SEQ_F64)
         for got, ref in ((y, y64), (s, s64), (x2, x2_64)):
             assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-5
+
+
+def _km_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        npts, nf, k = 301, 6, 3
+        feat = si.values(21, nf * npts)                  # uniform, feature-major, ld = npts
+        lo, hi = cdist.row_range(npts, world, rank)
+        shard = np.concatenate([feat[f * npts + lo:f * npts + hi] for f in range(nf)])
+        init = np.stack([feat[f * npts:f * npts + k] for f in range(nf)], axis=1)   # first k points
+        cl = torch.from_numpy(init.copy())
+        memb, it = cdist.kmeans_pointshard(torch.from_numpy(shard), hi - lo, hi - lo, nf, cl, max_iter=8,
+                                           ops=OracleKmeansOps)
+        q.put((rank, memb.numpy(), cl.numpy(), it))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_kmeans_pointshard_world2_gloo_bit_identical():
+    """Integer sums: two ranks give the unsharded oracle loop's bits exactly."""
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_km_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = sorted([q.get(timeout=180) for _ in range(world)], key=lambda t: t[0])
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    from oracle import kmeans as okm
+    npts, nf, k = 301, 6, 3
+    feat = si.values(21, nf * npts)
+    init = np.stack([feat[f * npts:f * npts + k] for f in range(nf)], axis=1)
+    cl_o, memb_o, it_o, _ = okm.kmeans(feat, npts, npts, nf, init, max_iter=8)
+    assert np.array_equal(np.concatenate([r[1] for r in res]), memb_o)
+    for r in res:
+        assert np.array_equal(r[2], cl_o) and r[3] == it_o
 
 
 def test_row_range_partitions():
