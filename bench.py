@@ -44,7 +44,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--workload", default="bicg_mvt",
-                   choices=["bicg_mvt", "kmeans", "gesummv", "syrk", "syr2k", "atax256", "atax"])
+                   choices=["bicg_mvt", "kmeans", "kmeans_iter", "gesummv", "syrk", "syr2k", "atax256", "atax"])
     p.add_argument("--variant", default=None,
                    help="fused (default for bicg_mvt/atax), fused1, coop, staged, vec4, literal, regs (kmeans)")
     p.add_argument("--impl", default="catt", choices=["catt", "reference"])
@@ -304,6 +304,61 @@ class Kmeans(Workload):
         oracle.kmeans_assign(host["feat"], self.ld, self.np_, self.nf, host["clusters"])
 
 
+class KmeansIter(Workload):
+    name = "kmeans_iter"
+    desc = ("KMEANS full iteration (assign + exact centroid update), 494020 points x 34 features, k=5, "
+            "feature-major, points sharded per rank (SURVEY 8(f) f2)")
+    variant = "fused"
+
+    def __init__(self, catt, torch, rank, world, variant):
+        super().__init__(catt, torch, rank, world, variant)
+        import seeded_inputs as si
+        self.np_, self.nf, self.k, self.ld = 494020, 34, 5, 494020
+        dev = torch.device("cuda")
+        self.feat = torch.empty(self.nf * self.ld, device=dev)
+        catt.fill_hash(self.feat, si.SEED_KMEANS, offset=rank * self.nf * self.ld)
+        self.clusters = self.feat.view(self.nf, self.ld)[:, : self.k].t().contiguous()
+        self.memb = torch.full((self.np_,), -1, dtype=torch.int32, device=dev)
+        self.acc = torch.zeros(catt.kmeans_acc_words(self.k, self.nf), dtype=torch.int64, device=dev)
+        nbytes = self.np_ * self.nf * 4 + 8 * self.np_ + self.k * self.nf * 4
+        self.loops = [Loop("kmeans assign+sums", lambda: catt.kmeans_accumulate(
+                               self.feat, self.ld, self.np_, self.nf, self.clusters, self.memb, self.acc),
+                           nbytes, "kmeans_acc"),
+                      Loop("kmeans finalize", lambda: catt.kmeans_finalize(self.acc, self.clusters),
+                           self.acc.numel() * 8 * 2 + self.k * self.nf * 4, "kmeans_fin")]
+        if world > 1:                    # the iteration's one exchange: integer sums, between the two kernels
+            import torch.distributed as dist
+            self.loops.insert(1, Loop("kmeans all-reduce of the sums", lambda: dist.all_reduce(self.acc),
+                                      self.acc.numel() * 8, "collective"))
+        # the KM transpose loop (Rodinia invert_mapping), CATT-planned and studied
+        self.pm = torch.empty(self.np_ * self.nf, device=dev)
+        catt.fill_hash(self.pm, si.sub_seed(si.SEED_KMEANS, 3))
+        self.fm = torch.empty(self.nf * self.ld, device=dev)
+        probt = catt.problem(catt.K_KMEANS_T, m=self.np_, n=self.nf, ld=self.ld)
+        self.plan("kmeans transpose (literal)", probt, catt.Throttle(cta_threads=256))
+        self.study = dict(name="kmeans transpose (literal, point-major -> feature-major)", prob=probt,
+                          launches=[(256, 0), (256, 228), (1024, 196)], reps=3,
+                          fn=lambda th: (lambda: catt.kmeans_transpose(self.pm, self.np_, self.nf, self.fm, self.ld,
+                                                                       t=th)))
+
+    def step_bytes(self):
+        return self.np_ * self.nf * 4 + 8 * self.np_
+
+    def inputs(self):
+        return [self.feat]
+
+    def outputs(self):
+        return [self.memb, self.clusters]
+
+    def host_copy(self):
+        return {"feat": self.feat.cpu().numpy(), "clusters": self.clusters.cpu().numpy()}
+
+    def cpu_oracle_step(self, oracle, host):
+        from oracle import kmeans as okm
+        memb, _ = oracle.kmeans_assign(host["feat"], self.ld, self.np_, self.nf, host["clusters"])
+        okm.update(host["feat"], self.ld, self.np_, self.nf, memb, host["clusters"])
+
+
 class Gesummv(Workload):
     name = "gesummv"
     desc = "GESUMMV 8192 fp32 (configs[3])"
@@ -473,7 +528,7 @@ class Atax256(Atax):
         super().__init__(catt, torch, rank, world, variant, m=256, n=256)
 
 
-WORKLOADS = {"bicg_mvt": BicgMvt, "kmeans": Kmeans, "gesummv": Gesummv, "syrk": Syrk, "syr2k": Syr2k, "atax256": Atax256,
+WORKLOADS = {"bicg_mvt": BicgMvt, "kmeans": Kmeans, "kmeans_iter": KmeansIter, "gesummv": Gesummv, "syrk": Syrk, "syr2k": Syr2k, "atax256": Atax256,
              "atax": Atax}
 
 
@@ -800,7 +855,7 @@ def main():
         app = app_study(catt, torch, w, flush)
 
     # ---- roofline of the dominant loop
-    dom = max(range(len(w.loops)), key=lambda i: loop_ms[i])
+    dom = max((i for i in range(len(w.loops)) if w.loops[i].kind != "collective"), key=lambda i: loop_ms[i])
     lp = w.loops[dom]
     peak, peak_src = peak_hbm()
     if lp.kind in ("syrk", "syr2k"):

@@ -22,6 +22,7 @@
 #include <cooperative_groups.h>
 
 #include "internal.h"
+#include "tma.cuh"
 
 namespace catt {
 
@@ -71,36 +72,6 @@ __device__ __forceinline__ void grid_barrier(unsigned* bar, unsigned nblocks) {
   __syncthreads();
 }
 
-__device__ __forceinline__ uint32_t f_s32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
-__device__ __forceinline__ void f_bar_init(uint64_t* b, uint32_t c) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(f_s32(b)), "r"(c) : "memory");
-}
-__device__ __forceinline__ void f_expect_tx(uint64_t* b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(f_s32(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void f_arrive(uint64_t* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(f_s32(b)) : "memory");
-}
-__device__ __forceinline__ void f_wait(uint64_t* b, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "LAB_WAIT:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@P1 bra DONE;\n"
-      "bra LAB_WAIT;\n"
-      "DONE:\n"
-      "}\n" ::"r"(f_s32(b)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void f_bulk(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   f_s32(dst)),
-               "l"(src), "r"(bytes), "r"(f_s32(b))
-               : "memory");
-}
-
 // DEP = true: ATAX (the column loop's vector is the row loop's result).
 // NW warps per CTA, T 16-byte chunks per lane per row. A stage holds RPS
 // whole rows (contiguous in memory: one bulk copy), S stages in a ring.
@@ -123,19 +94,19 @@ __global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS,
   const int64_t nst = (r1 - r0 + RPS - 1) / RPS;               // stages of this band
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
-      f_bar_init(&full[s], 1);
-      f_bar_init(&empty[s], NW);
+      bar_init(&full[s], 1);
+      bar_init(&empty[s], NW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
   auto issue = [&](int64_t c) {                                 // thread 0 only
     const int s = int(c % S);
-    if (c >= S) f_wait(&empty[s], uint32_t(((c / S) - 1) & 1));
+    if (c >= S) bar_wait(&empty[s], uint32_t(((c / S) - 1) & 1));
     const int64_t rows = imin64(RPS, r1 - (r0 + c * RPS));
     const uint32_t bytes = uint32_t(rows * N * 4);
-    f_expect_tx(&full[s], bytes);
-    f_bulk(ring + int64_t(s) * stage_bytes, Ap + (r0 + c * RPS) * N, bytes, &full[s]);
+    bar_expect_tx(&full[s], bytes);
+    bulk_1d(ring + int64_t(s) * stage_bytes, Ap + (r0 + c * RPS) * N, bytes, &full[s]);
   };
   if (threadIdx.x == 0)
     for (int64_t c = 0; c < imin64(S, nst); ++c) issue(c);
@@ -151,7 +122,7 @@ __global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS,
     const int s = int(c % S);
     const int64_t i0 = r0 + c * RPS;
     const int rows = int(imin64(RPS, r1 - i0));
-    f_wait(&full[s], uint32_t((c / S) & 1));
+    bar_wait(&full[s], uint32_t((c / S) & 1));
     const float4* st = reinterpret_cast<const float4*>(ring + int64_t(s) * stage_bytes);
     // row dots: lane partial in chunk order, xor tree, warp partials to smem
     for (int u = 0; u < rows; ++u) {
@@ -199,7 +170,7 @@ __global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS,
       }
     }
     __syncwarp();
-    if (lane == 0) f_arrive(&empty[s]);
+    if (lane == 0) bar_arrive(&empty[s]);
     if (threadIdx.x == 0 && c + S < nst) issue(c + S);
   }
   // column partials: first summed over the CL CTAs of this cluster through

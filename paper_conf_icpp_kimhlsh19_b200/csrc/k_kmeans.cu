@@ -23,6 +23,7 @@
 #include <cstdint>
 
 #include "internal.h"
+#include "tma.cuh"
 
 namespace catt {
 
@@ -164,38 +165,6 @@ __global__ void __launch_bounds__(256) kmeans_stream_kernel(KmArgs a) {
 // (one request per tile) into an S-stage ring; thread t computes point
 // tile*256 + t from shared memory (column t of every feature row: conflict
 // free), k partial distances in registers, f ascending: bit-exact membership.
-namespace {
-__device__ __forceinline__ uint32_t k_s32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
-__device__ __forceinline__ void k_bar_init(uint64_t* b, uint32_t c) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(k_s32(b)), "r"(c) : "memory");
-}
-__device__ __forceinline__ void k_expect_tx(uint64_t* b, uint32_t n) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(k_s32(b)), "r"(n) : "memory");
-}
-__device__ __forceinline__ void k_arrive(uint64_t* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(k_s32(b)) : "memory");
-}
-__device__ __forceinline__ void k_wait(uint64_t* b, uint32_t ph) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "LAB_WAIT:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@P1 bra DONE;\n"
-      "bra LAB_WAIT;\n"
-      "DONE:\n"
-      "}\n" ::"r"(k_s32(b)),
-      "r"(ph)
-      : "memory");
-}
-__device__ __forceinline__ void k_tma2d(void* dst, const CUtensorMap* m, int32_t c0, int32_t c1, uint64_t* b) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-          k_s32(dst)),
-      "l"(m), "r"(c0), "r"(c1), "r"(k_s32(b))
-      : "memory");
-}
-}  // namespace
 
 template <int KMAX>
 __global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constant__ CUtensorMap map, KmArgs a,
@@ -215,23 +184,23 @@ __global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constan
   for (int q = t; q < nf * k; q += blockDim.x) s_ct[(q % nf) * k + q / nf] = a.clusters[q];
   if (t == 0) {
     for (int s = 0; s < S; ++s) {
-      k_bar_init(&full[s], 1);
-      k_bar_init(&empty[s], nw);
+      bar_init(&full[s], 1);
+      bar_init(&empty[s], nw);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
   auto issue = [&](int64_t c) {
     const int s = int(c % S);
-    if (c >= S) k_wait(&empty[s], uint32_t(((c / S) - 1) & 1));
-    k_expect_tx(&full[s], uint32_t(tile_floats) * 4u);
-    k_tma2d(ring + int64_t(s) * tile_floats, &map, int32_t((blockIdx.x + c * G) * 256), 0, &full[s]);
+    if (c >= S) bar_wait(&empty[s], uint32_t(((c / S) - 1) & 1));
+    bar_expect_tx(&full[s], uint32_t(tile_floats) * 4u);
+    tma_2d(ring + int64_t(s) * tile_floats, &map, int32_t((blockIdx.x + c * G) * 256), 0, &full[s]);
   };
   if (t == 0)
     for (int64_t c = 0; c < imin64(S, mytiles); ++c) issue(c);
   for (int64_t c = 0; c < mytiles; ++c) {
     const int s = int(c % S);
-    k_wait(&full[s], uint32_t((c / S) & 1));
+    bar_wait(&full[s], uint32_t((c / S) & 1));
     const int64_t p = (blockIdx.x + c * G) * 256 + t;
     if (p < a.npoints) {
       const float* col = ring + int64_t(s) * tile_floats + t;
@@ -262,7 +231,7 @@ __global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constan
       a.membership[p] = index;
     }
     __syncwarp();
-    if (lane == 0) k_arrive(&empty[s]);
+    if (lane == 0) bar_arrive(&empty[s]);
     if (t == 0 && c + S < mytiles) issue(c + S);
   }
 }

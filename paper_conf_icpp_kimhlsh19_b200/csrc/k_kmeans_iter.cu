@@ -22,8 +22,10 @@
 #include <algorithm>
 #include <cfloat>
 #include <cstdint>
+#include <cstring>
 
 #include "internal.h"
+#include "tma.cuh"
 
 namespace catt {
 
@@ -79,32 +81,75 @@ const void* kmeans_t_func(int variant) {
 // ------------------------------------------------------------------ exact sums
 typedef unsigned __int128 u128;
 
+// PTX shifts clamp amounts >= 64 (as unsigned) to 64: the result is 0. That
+// makes the conversion below branch-free.
+__device__ __forceinline__ uint64_t shl64(uint64_t x, uint32_t n) {
+  uint64_t r;
+  asm("shl.b64 %0, %1, %2;" : "=l"(r) : "l"(x), "r"(n));
+  return r;
+}
+__device__ __forceinline__ uint64_t shr64(uint64_t x, uint32_t n) {
+  uint64_t r;
+  asm("shr.b64 %0, %1, %2;" : "=l"(r) : "l"(x), "r"(n));
+  return r;
+}
+
 // x * 2^64 as a two's-complement 128-bit integer. Exact for x = 0 and for
 // 2^-64 <= ulp(x), |x| < 2^31; anything else (non-zero bits below 2^-64,
-// |x| >= 2^31, subnormal, inf, NaN) counts in `inexact`.
+// |x| >= 2^31, subnormal, inf, NaN) counts in `inexact` (and converts to
+// the truncated value, or 0 when |x| >= 2^31).
 __device__ __forceinline__ u128 to_fixed(float x, int& inexact) {
   const uint32_t b = __float_as_uint(x);
-  const int e = int((b >> 23) & 0xffu);
-  uint32_t m = b & 0x7fffffu;
-  if (e == 0) {
-    inexact += (m != 0u);
-    return 0;
+  const uint32_t e = (b >> 23) & 0xffu, mant = b & 0x7fffffu;
+  const bool big = e >= 158u;
+  const uint64_t m = (e == 0u || big) ? 0ull : uint64_t(mant | 0x800000u);
+  const uint32_t sh = e - 86u;  // x * 2^64 = m * 2^(e-86); "negative" values wrap to huge amounts
+  const uint64_t lo = shl64(m, sh) | shr64(m, 0u - sh);
+  const uint64_t hi = shr64(m, 64u - sh) | shl64(m, sh - 64u);
+  const uint64_t lost = shl64(m, 64u + sh);  // the bits shifted out when e < 86 (0 otherwise)
+  inexact += int(big | (e == 0u && mant != 0u) | (e != 0u && e < 63u) | (lost != 0ull));
+  const uint64_t neg = 0ull - uint64_t(b >> 31);  // all ones for negative x
+  const u128 u = (u128(hi ^ neg) << 64) | u128(lo ^ neg);
+  return u + u128(neg & 1ull);  // ones' complement + 1 = two's complement negation
+}
+
+// An fp64 value that is a multiple of 2^-64 with |s| < 2^63, as the
+// two's-complement 128-bit integer s * 2^64 (exact).
+__device__ __forceinline__ u128 d_to_fixed(double s) {
+  const uint64_t b = uint64_t(__double_as_longlong(s));
+  const uint32_t e = uint32_t(b >> 52) & 0x7ffu;
+  const uint64_t m = e ? ((b & 0xfffffffffffffull) | 0x10000000000000ull) : 0ull;
+  const uint32_t sh = e - 1011u;  // s * 2^64 = m * 2^(e - 1075 + 64)
+  const uint64_t lo = shl64(m, sh) | shr64(m, 0u - sh);
+  const uint64_t hi = shr64(m, 64u - sh) | shl64(m, sh - 64u);
+  const uint64_t neg = 0ull - (b >> 63);
+  const u128 u = (u128(hi ^ neg) << 64) | u128(lo ^ neg);
+  return u + u128(neg & 1ull);
+}
+
+// Exact sum of row[idx[i]], i in [lo, hi), as a 128-bit fixed-point value.
+// Fast path: the values are summed in fp64 and the sum is provably exact when
+// every value is a multiple of u = 2^(emin-150) (emin = smallest exponent
+// field of the non-zero values) and sum |x| <= 2^52 u: every partial sum is
+// then an integer multiple of u below 2^53 u. u >= 2^-64 and |x| < 2^31 keep
+// the result inside the fixed-point contract. Otherwise: value by value.
+__device__ __forceinline__ u128 segment_sum(const float* __restrict__ row, const unsigned short* __restrict__ idx,
+                                            int lo, int hi, int& inexact) {
+  double sum = 0.0, bnd = 0.0;
+  uint32_t amin = 0xffffffffu;  // min over non-zero x of |x|'s bits - 1 (zeros wrap to the max)
+  for (int i = lo; i < hi; ++i) {
+    const float x = row[idx[i]];
+    amin = min(amin, (__float_as_uint(x) & 0x7fffffffu) - 1u);
+    const double xd = double(x);
+    sum += xd;
+    bnd += fabs(xd);
   }
-  if (e >= 158) {
-    ++inexact;
-    return 0;
-  }
-  m |= 0x800000u;
-  const int sh = e - 86;  // x = m * 2^(e-150); x * 2^64 = m * 2^(e-86)
-  u128 u;
-  if (sh >= 0) {
-    u = u128(m) << sh;
-  } else {
-    const int r = -sh;
-    inexact += (r >= 24) || (m & ((1u << r) - 1u)) != 0u;
-    u = r >= 24 ? u128(0) : u128(m >> r);
-  }
-  return (b >> 31) ? u128(0) - u : u;
+  const int emin = amin == 0xffffffffu ? 255 : int((amin + 1u) >> 23);
+  // bnd < 2^31 bounds every |x| (and rejects inf/NaN); emin >= 86: u >= 2^-64
+  if (emin >= 86 && bnd < 2147483648.0 && bnd <= ldexp(1.0, emin - 98)) return d_to_fixed(sum);
+  u128 v = 0;
+  for (int i = lo; i < hi; ++i) v += to_fixed(row[idx[i]], inexact);
+  return v;
 }
 
 constexpr int KT = 256;      // points per tile = threads per CTA
@@ -120,83 +165,128 @@ struct AccArgs {
   int nf, k;
 };
 
-template <int KMAX, int FB>
-__global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(AccArgs a) {
+// Dynamic shared memory: {mbarrier | centres [nf][KP] | TMA stage [nf][256]
+// (TMA only) | tile [nf][KTP] | 128-bit accumulators}.
+struct AccSmem {
+  int ct, stage, tile, acc, total;
+  __host__ __device__ AccSmem(int nf, int k, int KP, int FB, bool tma) {
+    ct = 128;
+    stage = ((ct + nf * KP * 4 + 127) / 128) * 128;
+    tile = stage + (tma ? nf * KT * 4 : 0);
+    acc = ((tile + nf * KTP * 4 + 15) / 16) * 16;
+    total = acc + (KT / 32) * FB * k * 32 * 16;
+  }
+};
+
+// TMA = true: the tile {256 points x nf} arrives by one 2-D tensor copy into
+// the stage while the previous tile's sort and phase 2 run (map over feat:
+// dims {npoints, nf}, row stride ld*4 bytes; out-of-range points read 0).
+template <int KMAX, int FB, bool TMA>
+__global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_constant__ CUtensorMap map, AccArgs a) {
   if (a.done && *a.done) return;
-  extern __shared__ __align__(16) unsigned char dyn[];
+  extern __shared__ __align__(128) unsigned char dyn[];
   const int nf = a.nf, k = a.k;
-  float* s_ct = reinterpret_cast<float*>(dyn);                         // [nf][k]
-  float* tile = s_ct + ((nf * k + 3) & ~3);                             // [nf][KTP]
+  constexpr int KP = (KMAX + 3) & ~3;                                   // centre pitch (float4 reads)
+  const AccSmem L(nf, k, KP, FB, TMA);
+  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
+  float* s_ct = reinterpret_cast<float*>(dyn + L.ct);                  // [nf][KP], padding = +inf
+  float* stage = reinterpret_cast<float*>(dyn + L.stage);              // [nf][256] (TMA)
+  float* tile = reinterpret_cast<float*>(dyn + L.tile);                // [nf][KTP]
   __shared__ int s_cnt[KMAX], s_start[KMAX + 1], s_tot[KMAX];
   __shared__ unsigned short s_idx[KT];
   const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-  for (int q = t; q < nf * k; q += KT) s_ct[(q % nf) * k + q / nf] = a.clusters[q];
+  // a padded centre at +inf is never strictly nearer than FLT_MAX: same decisions
+  for (int q = t; q < nf * KP; q += KT) {
+    const int f = q / KP, cc = q - f * KP;
+    s_ct[q] = cc < k ? a.clusters[cc * nf + f] : __int_as_float(0x7f800000);
+  }
   if (t < KMAX) s_tot[t] = 0;
   long long delta = 0;
   int inexact = 0;
-  u128 acc[FB][KMAX];
-#pragma unroll
-  for (int fb = 0; fb < FB; ++fb)
-#pragma unroll
-    for (int c = 0; c < KMAX; ++c) acc[fb][c] = 0;
+  // per-lane private 128-bit accumulators: s_acc[((w*FB + g)*k + c)*32 + lane]
+  u128* s_acc = reinterpret_cast<u128*>(dyn + L.acc);
+  for (int q = t; q < (KT / 32) * FB * k * 32; q += KT) s_acc[q] = 0;
 
   const int64_t ntiles = (a.npoints + KT - 1) / KT;
+  const uint32_t tile_bytes = uint32_t(nf) * KT * 4u;
+  if (TMA && t == 0) {
+    bar_init(full, 1);
+    fence_barrier_init();
+    if (int64_t(blockIdx.x) < ntiles) {
+      bar_expect_tx(full, tile_bytes);
+      tma_2d(stage, &map, int32_t(blockIdx.x) * KT, 0, full);
+    }
+  }
+  uint32_t parity = 0;
   for (int64_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
     if (t < KMAX) s_cnt[t] = 0;
-    __syncthreads();  // s_ct ready; the previous tile's phase 2 is done with `tile`
     const int64_t p = tl * KT + t;
+    const int old = p < a.npoints ? a.memb[p] : -1;
+    __syncthreads();  // s_ct / barrier ready; the previous tile's phase 2 is done with `tile`
+    if (TMA) {
+      bar_wait(full, parity);
+      parity ^= 1u;
+    }
     int c = -1, rank = 0, changed = 0;
     if (p < a.npoints) {
       const float* f0 = a.feat + p;
       float d[KMAX];
 #pragma unroll
       for (int cc = 0; cc < KMAX; ++cc) d[cc] = 0.0f;
+      auto feature = [&](int f, float v) {
+        tile[f * KTP + t] = v;
+        const float4* cf = reinterpret_cast<const float4*>(s_ct + f * KP);
+#pragma unroll
+        for (int q = 0; q < KP / 4; ++q) {
+          const float4 c4 = cf[q];
+          const float cv[4] = {c4.x, c4.y, c4.z, c4.w};
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+            if (4 * q + j < KMAX) {
+              const float diff = v - cv[j];
+              d[4 * q + j] = fmaf(diff, diff, d[4 * q + j]);
+            }
+        }
+      };
       int f = 0;
-      for (; f + 8 <= nf; f += 8) {
+      if (TMA) {
+#pragma unroll 8
+        for (; f < nf; ++f) feature(f, stage[f * KT + t]);
+      }
+      for (; f + 32 <= nf; f += 32) {  // 32 loads in flight per thread
+        float v[32];
+#pragma unroll
+        for (int u = 0; u < 32; ++u)
+          asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[u]) : "l"(f0 + int64_t(f + u) * a.ld));
+#pragma unroll
+        for (int u = 0; u < 32; ++u) feature(f + u, v[u]);
+      }
+      for (; f < nf; f += 8) {
         float v[8];
 #pragma unroll
         for (int u = 0; u < 8; ++u)
-          asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[u]) : "l"(f0 + int64_t(f + u) * a.ld));
+          if (f + u < nf)
+            asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[u]) : "l"(f0 + int64_t(f + u) * a.ld));
 #pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          tile[(f + u) * KTP + t] = v[u];
-          const float* cf = s_ct + (f + u) * k;
-#pragma unroll
-          for (int cc = 0; cc < KMAX; ++cc)
-            if (cc < k) {
-              const float diff = v[u] - cf[cc];
-              d[cc] = fmaf(diff, diff, d[cc]);
-            }
-        }
-      }
-      for (; f < nf; ++f) {
-        const float v = f0[int64_t(f) * a.ld];
-        tile[f * KTP + t] = v;
-        const float* cf = s_ct + f * k;
-#pragma unroll
-        for (int cc = 0; cc < KMAX; ++cc)
-          if (cc < k) {
-            const float diff = v - cf[cc];
-            d[cc] = fmaf(diff, diff, d[cc]);
-          }
+        for (int u = 0; u < 8; ++u)
+          if (f + u < nf) feature(f + u, v[u]);
       }
       float best = FLT_MAX;
 #pragma unroll
       for (int cc = 0; cc < KMAX; ++cc)
-        if (cc < k && d[cc] < best) {
+        if (d[cc] < best) {
           best = d[cc];
           c = cc;
         }
-      if (c >= 0) {
-        changed = a.memb[p] != c;
-        a.memb[p] = c;
-        rank = atomicAdd(&s_cnt[c], 1);
-      } else {  // every distance is NaN or >= FLT_MAX: no centre (as catt_kmeans_assign)
-        changed = a.memb[p] != -1;
-        a.memb[p] = -1;
-      }
+      changed = old != c;  // c = -1: every distance NaN or >= FLT_MAX (as catt_kmeans_assign)
+      a.memb[p] = c;
+      if (c >= 0) rank = atomicAdd(&s_cnt[c], 1);
     }
-    const int nchg = __syncthreads_count(changed);
+    const int nchg = __syncthreads_count(changed);  // every thread is done with the stage
+    if (TMA && t == 0 && tl + gridDim.x < ntiles) {  // prefetch the next tile during sort + phase 2
+      bar_expect_tx(full, tile_bytes);
+      tma_2d(stage, &map, int32_t((tl + gridDim.x) * KT), 0, full);
+    }
     if (t == 0) {
       delta += nchg;
       s_start[0] = 0;
@@ -208,50 +298,45 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(AccArgs a) {
     __syncthreads();
     if (c >= 0) s_idx[s_start[c] + rank] = static_cast<unsigned short>(t);
     __syncthreads();
-    // phase 2: warp w owns sorted entries [32w, 32w + 32); lane = feature
-    const int lo_w = w * 32, hi_w = lo_w + 32;
+    // phase 2: warp w owns sorted entries [32w, 32w + 32). Group g holds
+    // features [32g, 32g + 32); a group with fg < 32 features (the last one)
+    // spreads its lanes as fg features x (32/fg) sub-chunks of fg entries.
+    // The centre of a sorted segment is warp-uniform, so acc[g][cc] has a
+    // static index.
 #pragma unroll
-    for (int fb = 0; fb < FB; ++fb) {
-      const int f = lane + 32 * fb;
-      if (f < nf) {
-        const float* row = tile + f * KTP;
-#pragma unroll
-        for (int cc = 0; cc < KMAX; ++cc) {
-          if (cc < k) {
-            const int lo = max(s_start[cc], lo_w), hi = min(s_start[cc + 1], hi_w);
-            u128 sum = 0;
-            for (int i = lo; i < hi; ++i) sum += to_fixed(row[s_idx[i]], inexact);
-            acc[fb][cc] += sum;
-          }
+    for (int g = 0; g < FB; ++g) {
+      const int rem = nf - 32 * g;
+      if (rem > 0) {
+        const int fg = rem >= 32 ? 32 : (rem > 16 ? 32 : rem > 8 ? 16 : rem > 4 ? 8 : rem > 2 ? 4 : rem);
+        const int fl = lane & (fg - 1), h = lane / fg;
+        const int s_lo = w * 32 + h * fg, s_hi = s_lo + fg;
+        const bool fok = fl < rem;
+        const float* row = tile + (32 * g + fl) * KTP;
+        u128* mine = s_acc + (w * FB + g) * k * 32 + lane;
+        for (int cc = 0; cc < k; ++cc) {
+          const int lo = max(s_start[cc], s_lo), hi = fok ? min(s_start[cc + 1], s_hi) : lo;
+          if (lo < hi) mine[cc * 32] += segment_sum(row, s_idx, lo, hi, inexact);
         }
       }
     }
   }
   __syncthreads();
-  // epilogue: per centre, the CTA's warps summed exactly, then four 32-bit
-  // chunks of the 128-bit sum added into the int64 limbs (exact, any order)
-  u128* red = reinterpret_cast<u128*>(tile);  // [8 warps][FB*32]
+  // epilogue: per (centre, feature) the CTA's lanes summed exactly, then the
+  // four 32-bit chunks of the 128-bit sum added into the int64 limbs
   const int K4 = k * nf * 4;
-#pragma unroll
-  for (int cc = 0; cc < KMAX; ++cc) {
-    if (cc < k) {
-#pragma unroll
-      for (int fb = 0; fb < FB; ++fb) red[w * (FB * 32) + fb * 32 + lane] = acc[fb][cc];
-      __syncthreads();
-      if (t < nf) {
-        u128 s = 0;
-        for (int ww = 0; ww < KT / 32; ++ww) s += red[ww * (FB * 32) + t];
-        unsigned long long* limb = a.acc + (int64_t(cc) * nf + t) * 4;
-        const uint32_t c0 = uint32_t(s), c1 = uint32_t(s >> 32), c2 = uint32_t(s >> 64);
-        const int32_t c3 = int32_t(uint32_t(s >> 96));
-        if (s != 0) {
-          atomicAdd(limb + 0, (unsigned long long)c0);
-          atomicAdd(limb + 1, (unsigned long long)c1);
-          atomicAdd(limb + 2, (unsigned long long)c2);
-          atomicAdd(limb + 3, (unsigned long long)(long long)c3);
-        }
-      }
-      __syncthreads();
+  for (int q = t; q < k * nf; q += KT) {
+    const int cc = q / nf, f = q - cc * nf;
+    const int g = f >> 5, fl = f & 31, rem = nf - 32 * g;
+    const int fg = rem >= 32 ? 32 : (rem > 16 ? 32 : rem > 8 ? 16 : rem > 4 ? 8 : rem > 2 ? 4 : rem);
+    u128 s = 0;
+    for (int ww = 0; ww < KT / 32; ++ww)
+      for (int l = fl; l < 32; l += fg) s += s_acc[((ww * FB + g) * k + cc) * 32 + l];
+    if (s != 0) {
+      unsigned long long* limb = a.acc + int64_t(q) * 4;
+      atomicAdd(limb + 0, (unsigned long long)uint32_t(s));
+      atomicAdd(limb + 1, (unsigned long long)uint32_t(s >> 32));
+      atomicAdd(limb + 2, (unsigned long long)uint32_t(s >> 64));
+      atomicAdd(limb + 3, (unsigned long long)(long long)int32_t(uint32_t(s >> 96)));
     }
   }
   if (t < k && s_tot[t]) atomicAdd(a.acc + K4 + t, (unsigned long long)s_tot[t]);
@@ -340,18 +425,44 @@ struct AccLaunch {
   int grid;
 };
 
-template <int KMAX, int FB>
+template <int KMAX, int FB, bool TMA>
 const void* acc_fn() {
-  return (const void*)km_accumulate_kernel<KMAX, FB>;
+  return (const void*)km_accumulate_kernel<KMAX, FB, TMA>;
 }
 
 catt_status acc_launch(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters, int32_t k,
                        int32_t* memb, int64_t* acc, const long long* done, cudaStream_t s) {
+  // TMA needs a 16-B aligned base and a row stride that is a multiple of 16 B;
+  // otherwise the general form (per-thread loads, centres padded to 16)
+  const bool tma = (reinterpret_cast<uintptr_t>(feat) & 15u) == 0 && ld % 4 == 0 && encode_fn() != nullptr;
   const int FB = nf <= 32 ? 1 : 2;
-  const int KMAX = k <= 8 ? 8 : 16;
-  const void* f = KMAX == 8 ? (FB == 1 ? acc_fn<8, 1>() : acc_fn<8, 2>()) : (FB == 1 ? acc_fn<16, 1>() : acc_fn<16, 2>());
-  const size_t tile_bytes = std::max<size_t>(size_t(nf) * KTP * 4, size_t(8) * FB * 32 * 16);
-  const size_t smem = size_t((nf * k + 3) & ~3) * 4 + tile_bytes;
+  const int KMAX = !tma ? 16 : k <= 4 ? 4 : k == 5 ? 5 : k <= 8 ? 8 : 16;
+  const int FBx = tma ? FB : 2;
+  const void* f = nullptr;
+  switch (KMAX * 4 + FBx) {
+    case 17: f = acc_fn<4, 1, true>(); break;
+    case 18: f = acc_fn<4, 2, true>(); break;
+    case 21: f = acc_fn<5, 1, true>(); break;
+    case 22: f = acc_fn<5, 2, true>(); break;
+    case 33: f = acc_fn<8, 1, true>(); break;
+    case 34: f = acc_fn<8, 2, true>(); break;
+    case 65: f = acc_fn<16, 1, true>(); break;
+    default: f = tma ? acc_fn<16, 2, true>() : acc_fn<16, 2, false>(); break;
+  }
+  const AccSmem L(nf, k, (KMAX + 3) & ~3, FBx, tma);
+  const size_t smem = size_t(L.total);
+  CUtensorMap map;
+  memset(&map, 0, sizeof(map));
+  if (tma) {
+    const cuuint64_t dims[2] = {cuuint64_t(npoints), cuuint64_t(nf)};
+    const cuuint64_t strides[1] = {cuuint64_t(ld) * 4};
+    const cuuint32_t box[2] = {cuuint32_t(KT), cuuint32_t(nf)};
+    const cuuint32_t es[2] = {1, 1};
+    if (encode_fn()(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(feat), dims, strides, box, es,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return CATT_EINVAL;
+  }
   cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) {
     record_cuda_error(e);
@@ -369,7 +480,7 @@ catt_status acc_launch(const float* feat, int64_t ld, int64_t npoints, int32_t n
   const int64_t tiles = (npoints + KT - 1) / KT;
   const int grid = int(std::min<int64_t>(tiles, int64_t(per_sm) * ctx->hw.num_sms));
   AccArgs a{feat, clusters, memb, reinterpret_cast<unsigned long long*>(acc), done, ld, npoints, nf, k};
-  void* args[] = {&a};
+  void* args[] = {&map, &a};
   e = cudaLaunchKernel(f, dim3(unsigned(grid)), dim3(KT), args, smem, s);
   if (e != cudaSuccess) {
     record_cuda_error(e);
