@@ -50,6 +50,8 @@ def parse():
     p.add_argument("--impl", default="catt", choices=["catt", "reference"])
     p.add_argument("--no-study", action="store_true", help="skip the throttle sweep")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--flush-order", default="flush_sleep", choices=["flush_sleep", "sleep_flush"],
+                   help="order of the L2 flush and the enqueue-cover GPU sleep before each timed step")
     p.add_argument("--cpu-seconds", type=float, default=8.0, help="CPU-oracle sample budget")
     return p.parse_args()
 
@@ -686,17 +688,13 @@ def app_study(catt, torch, w, flush):
     return out
 
 
-def ncu_traffic(kernel_hint):
-    """dram bytes per launch of the dominant kernel from the committed ncu summary."""
+def ncu_traffic(workload):
+    """DRAM bytes per launch of the workload's dominant kernel from the committed ncu summary."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
-        d = json.load(open(path))
+        return json.load(open(path)).get(workload)
     except Exception:
         return None
-    for k, v in d.items():
-        if kernel_hint in k:
-            return v
-    return None
 
 
 def run_reference(args):
@@ -783,11 +781,16 @@ def main():
     clean_buf = torch.zeros(64 * 1024 * 1024, dtype=torch.int32, device="cuda")
 
     def flush():
+        # keep the GPU busy ~0.2 ms while the host enqueues the timed launches,
+        # so host-side enqueue cost never lands between the CUDA events. Order
+        # "sleep_flush" sleeps first, so HBM is busy with the flush right up to
+        # the timed kernels; "flush_sleep" leaves it idle for the sleep.
+        if args.flush_order == "sleep_flush":
+            torch.cuda._sleep(400_000)
         flush_buf.zero_()
         clean_buf.sum()
-        # keep the GPU busy ~0.2 ms while the host enqueues the timed launches,
-        # so host-side enqueue cost never lands between the CUDA events
-        torch.cuda._sleep(400_000)
+        if args.flush_order == "flush_sleep":
+            torch.cuda._sleep(400_000)
     torch.cuda.synchronize()
 
     clocks = ClockSampler(local)
@@ -864,12 +867,12 @@ def main():
         peak_t = 148 * 128 * 2 * clk_mhz * 1e6 / 1e12
         ach = w.flops / (loop_ms[dom] * 1e-3) / 1e12
         roof = {"bound": "alu", "kernel": lp.name, "achieved": round(ach, 3), "peak": round(peak_t, 3),
-                "unit": "TFLOP/s", "frac": round(ach / peak_t, 4), "traffic": ncu_traffic(lp.kind),
+                "unit": "TFLOP/s", "frac": round(ach / peak_t, 4), "traffic": ncu_traffic(w.name) if w.variant == type(w).variant else None,
                 "peak_source": f"derived: 148 SM x 128 FP32 lanes x 2 x {clk_mhz:.0f} MHz (median under load)"}
     else:
         ach = lp.nbytes / (loop_ms[dom] * 1e-3) / 1e9
         roof = {"bound": "hbm", "kernel": lp.name, "achieved": round(ach, 2), "peak": peak, "unit": "GB/s",
-                "frac": round(ach / peak, 4), "traffic": ncu_traffic(lp.kind),
+                "frac": round(ach / peak, 4), "traffic": ncu_traffic(w.name) if w.variant == type(w).variant else None,
                 "peak_source": f"{peak_src} (MEASURED_PEAKS.json hbm_gbs)" if peak_src == "measured" else "fallback"}
 
     # ---- context: a plain device copy moving the same bytes as the dominant
@@ -937,7 +940,7 @@ def main():
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded counter hash, generated on device)",
-            "config": {"workload": w.desc, "variant": w.variant, "l2": "flushed before every step (256 MiB write, then 256 MiB clean read)",
+            "config": {"workload": w.desc, "variant": w.variant, "l2": "flushed before every step (256 MiB write, then 256 MiB clean read)", "flush_order": args.flush_order,
                        "rows_per_rank": getattr(w, "rows", None), "parallelism": f"row-shard x{world}"},
             "loops": {lp.name: {"ms": round(loop_ms[i], 5),
                                 "gbs": round(lp.nbytes / (loop_ms[i] * 1e-3) / 1e9, 1),
