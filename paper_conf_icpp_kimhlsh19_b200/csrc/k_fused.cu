@@ -27,6 +27,7 @@
 namespace catt {
 
 constexpr int kMaxDual = 4;
+constexpr int kBandMax = 2048;  // rows per CTA whose xc / yr are staged in shared memory
 
 // Up to kMaxDual independent problems with the same column count N share one
 // launch (a grouped pass): CTAs [cta0[p], cta0[p+1]) stream problem p.
@@ -42,6 +43,7 @@ struct FusedArgs {
   int cta0[kMaxDual + 1];
   int row_acc[kMaxDual], col_acc[kMaxDual];
   int nprob;
+  int bandcap;                // rows per CTA whose xc / yr fit the shared-memory band buffer (nd kernel)
   unsigned* gbar;             // grid barrier {count, generation}
   int64_t N;
 };
@@ -242,10 +244,244 @@ __global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS,
   }
 }
 
+// Independent pair (BICG, MVT: the column weights xc are inputs), one read
+// of each element: every float4 of a row feeds the row dot and the column
+// partial. Warp roles: NW consumer warps own 16-byte column chunks (as in
+// fused_kernel) and do only the streaming math; one producer warp issues the
+// stage copies and adds the row partials, so neither sits on the consumers'
+// path. Rows go 4 at a time (4 independent dot chains); the 4 lane partials
+// are reduced by a fixed butterfly (offset 16 halves the rows per lane, 8
+// again, then 4, 2, 1: 6 shuffles for 4 rows) and written to a row-partial
+// ring of 2S slots. Per stage c: consumers wait full[c%S], compute, publish
+// partials (part_full[c%2S]) and release the stage (empty[c%S]); the producer
+// waits part_full, adds the NW partials of each row with a fixed xor tree,
+// writes the row outputs, then refills slot c%S with stage c+S. Slot c%2S is
+// rewritten only at stage c+2S, whose copy is issued after totals(c+S).
+template <int NW, int T>
+__global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a, int RPS, int S) {
+  extern __shared__ __align__(1024) unsigned char dyn[];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const bool producer = warp == NW;
+  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
+  uint64_t* empty = full + S;
+  uint64_t* part_full = empty + S;                                // [2S]
+  float* rowbuf = reinterpret_cast<float*>(dyn + 1024);          // [2S][RPS][NW] warp partials
+  float* bandbuf = rowbuf + 2 * S * RPS * NW;                   // [2][bandcap] xc and yr of the band
+  const int BC = a.bandcap;
+  unsigned char* ring = dyn + 1024 + ((int64_t(2 * S) * RPS * NW * 4 + 2 * int64_t(BC) * 4 + 1023) / 1024) * 1024;
+  int pi = 0;
+  while (pi + 1 < a.nprob && int(blockIdx.x) >= a.cta0[pi + 1]) ++pi;
+  const float* __restrict__ Ap = a.A[pi];
+  const float* __restrict__ xc = a.xc[pi];
+  float* __restrict__ yr = a.yr[pi];
+  const int lb = int(blockIdx.x) - a.cta0[pi];
+  const int64_t N = a.N, n4 = N >> 2, M = a.M[pi];
+  const int64_t stage_bytes = int64_t(RPS) * N * 4;
+  const int64_t r0 = int64_t(lb) * a.band[pi], r1 = imin64(M, r0 + a.band[pi]);
+  const int64_t nst = r1 > r0 ? (r1 - r0 + RPS - 1) / RPS : 0;
+  const bool racc = a.row_acc[pi] != 0;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      bar_init(&full[s], 1);
+      bar_init(&empty[s], NW);
+    }
+    for (int s = 0; s < 2 * S; ++s) bar_init(&part_full[s], NW);
+    fence_barrier_init();
+  }
+  auto issue = [&](int64_t c) {                                 // producer lane 0
+    const int s = int(c % S);
+    const int64_t rows = imin64(RPS, r1 - (r0 + c * RPS));
+    const uint32_t bytes = uint32_t(rows * N * 4);
+    bar_expect_tx(&full[s], bytes);
+    bulk_1d(ring + int64_t(s) * stage_bytes, Ap + (r0 + c * RPS) * N, bytes, &full[s]);
+  };
+  __syncthreads();
+  if (producer && lane == 0)
+    for (int64_t c = 0; c < imin64(S, nst); ++c) issue(c);
+  // the band's column weights and initial row values, all loads in flight at once
+  const bool inband = r1 - r0 <= BC;
+  if (inband) {
+    for (int64_t i = threadIdx.x; i < r1 - r0; i += blockDim.x) {
+      bandbuf[i] = xc[r0 + i];
+      bandbuf[BC + i] = racc ? yr[r0 + i] : 0.0f;
+    }
+  }
+  __syncthreads();
+  float4 acc[T];
+#pragma unroll
+  for (int t = 0; t < T; ++t) acc[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+
+  if (producer) {
+    // row totals, then refill the consumed slot
+    constexpr int RPP = 32 / NW;
+    for (int64_t c = 0; c < nst; ++c) {
+      const int64_t i0 = r0 + c * RPS;
+      const int rows = int(imin64(RPS, r1 - i0));
+      const int q = int(c % (2 * S));
+      const float* rb = rowbuf + int64_t(q) * RPS * NW;
+      bar_wait(&part_full[q], uint32_t((c / (2 * S)) & 1));
+      for (int u0 = 0; u0 < rows; u0 += RPP) {
+        const int u = u0 + lane / NW;
+        float v = u < rows ? rb[u * NW + (lane % NW)] : 0.0f;
+#pragma unroll
+        for (int o = NW / 2; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (lane % NW == 0 && u < rows) {
+          const float y0 = racc ? (inband ? bandbuf[BC + (i0 + u - r0)] : yr[i0 + u]) : 0.0f;
+          yr[i0 + u] = racc ? y0 + v : v;
+        }
+      }
+      if (lane == 0 && c + S < nst) {
+        bar_wait(&empty[c % S], uint32_t((c / S) & 1));
+        issue(c + S);
+      }
+      __syncwarp();
+    }
+  } else {
+    const float4* x4 = reinterpret_cast<const float4*>(a.xr[pi]);
+    float4 xr[T];
+    bool ok[T];
+    int64_t col[T];
+#pragma unroll
+    for (int t = 0; t < T; ++t) {
+      col[t] = warp * 32 + lane + int64_t(32) * NW * t;
+      ok[t] = col[t] < n4;
+      xr[t] = ok[t] ? x4[col[t]] : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    const bool b4 = (lane & 16) != 0, b3 = (lane & 8) != 0;
+    for (int64_t c = 0; c < nst; ++c) {
+      const int s = int(c % S);
+      const int q = int(c % (2 * S));
+      const int64_t i0 = r0 + c * RPS;
+      const int rows = int(imin64(RPS, r1 - i0));
+      const float wl = lane < rows ? (inband ? bandbuf[i0 - r0 + lane] : xc[i0 + lane]) : 0.0f;
+      bar_wait(&full[s], uint32_t((c / S) & 1));
+      const float4* st = reinterpret_cast<const float4*>(ring + int64_t(s) * stage_bytes);
+      float* rb = rowbuf + int64_t(q) * RPS * NW;
+      for (int u0 = 0; u0 < rows; u0 += 4) {
+        float d[4] = {0.f, 0.f, 0.f, 0.f};
+        float w[4];
+#pragma unroll
+        for (int r = 0; r < 4; ++r) w[r] = __shfl_sync(0xffffffffu, wl, (u0 + r) & 31);
+        const float4* g = st + int64_t(u0) * n4;
+        auto row4 = [&](int r, int t) {
+          const float4 v = g[int64_t(r) * n4 + col[t]];
+          d[r] = fmaf(v.x, xr[t].x, d[r]);
+          d[r] = fmaf(v.y, xr[t].y, d[r]);
+          d[r] = fmaf(v.z, xr[t].z, d[r]);
+          d[r] = fmaf(v.w, xr[t].w, d[r]);
+          acc[t].x = fmaf(v.x, w[r], acc[t].x);
+          acc[t].y = fmaf(v.y, w[r], acc[t].y);
+          acc[t].z = fmaf(v.z, w[r], acc[t].z);
+          acc[t].w = fmaf(v.w, w[r], acc[t].w);
+        };
+        if (u0 + 4 <= rows) {   // full group: no per-row guards
+#pragma unroll
+          for (int t = 0; t < T; ++t)
+            if (ok[t]) {
+#pragma unroll
+              for (int r = 0; r < 4; ++r) row4(r, t);
+            }
+        } else {
+#pragma unroll
+          for (int t = 0; t < T; ++t)
+            if (ok[t]) {
+#pragma unroll
+              for (int r = 0; r < 4; ++r)
+                if (u0 + r < rows) row4(r, t);
+            }
+        }
+        // butterfly: after offset 16 a lane holds rows {2*b4, 2*b4+1}, after 8 row 2*b4+b3
+        const float s0 = b4 ? d[0] : d[2], s1 = b4 ? d[1] : d[3];
+        const float k0 = b4 ? d[2] : d[0], k1 = b4 ? d[3] : d[1];
+        const float e0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 16);
+        const float e1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 16);
+        float f = (b3 ? e1 : e0) + __shfl_xor_sync(0xffffffffu, b3 ? e0 : e1, 8);
+        f += __shfl_xor_sync(0xffffffffu, f, 4);
+        f += __shfl_xor_sync(0xffffffffu, f, 2);
+        f += __shfl_xor_sync(0xffffffffu, f, 1);
+        const int r = lane >> 3;
+        if ((lane & 7) == 0 && u0 + r < rows) rb[(u0 + r) * NW + warp] = f;
+      }
+      __syncwarp();
+      if (lane == 0) {
+        bar_arrive(&part_full[q]);
+        bar_arrive(&empty[s]);
+      }
+    }
+  }
+  // column partials -> workspace (the producer's acc is zero and unused);
+  // grid barrier; fixed-tree column outputs
+  float* part = a.part[pi] + int64_t(lb) * N;
+  if (!producer) {
+#pragma unroll
+    for (int t = 0; t < T; ++t) {
+      const int64_t cc = warp * 32 + lane + int64_t(32) * NW * t;
+      if (cc < n4) reinterpret_cast<float4*>(part)[cc] = acc[t];
+    }
+  }
+  __threadfence();
+  grid_barrier(a.gbar, gridDim.x);
+  // column outputs in one round: chunks of CW = 32*L columns (L per lane,
+  // chosen so every problem's chunks fit the grid); consumer warp w sums band
+  // partials [w*gpw, (w+1)*gpw) in order, then the NW warp sums in warp order
+  {
+    constexpr int LMAX = 4;
+    __shared__ float red[NW][32 * LMAX];
+    const int64_t per_cta = (N * a.nprob + gridDim.x - 1) / gridDim.x;
+    const int L = per_cta <= 32 ? 1 : per_cta <= 64 ? 2 : per_cta <= 96 ? 3 : 4;
+    const int64_t CW = 32 * L;
+    const int64_t chunks = (N + CW - 1) / CW;
+    for (int64_t gch = blockIdx.x; gch < chunks * a.nprob; gch += gridDim.x) {
+      const int q = int(gch / chunks);
+      const int64_t ch = gch % chunks;
+      const int64_t G = a.cta0[q + 1] - a.cta0[q];
+      const int64_t gpw = (G + NW - 1) / NW;
+      const int64_t b0 = warp * gpw, b1 = imin64(G, b0 + gpw);
+      const float* pq = a.part[q];
+      if (!producer) {
+        float sum[LMAX];
+#pragma unroll
+        for (int l = 0; l < LMAX; ++l) sum[l] = 0.0f;
+        for (int64_t b = b0; b < b1; ++b) {
+#pragma unroll
+          for (int l = 0; l < LMAX; ++l) {
+            const int64_t j = ch * CW + l * 32 + lane;
+            if (l < L && j < N) sum[l] += pq[b * N + j];
+          }
+        }
+#pragma unroll
+        for (int l = 0; l < LMAX; ++l) red[warp][l * 32 + lane] = sum[l];
+      }
+      __syncthreads();
+      if (warp == 0) {
+        for (int l = 0; l < L; ++l) {
+          const int64_t j = ch * CW + l * 32 + lane;
+          if (j < N) {
+            float tot = red[0][l * 32 + lane];
+            for (int w = 1; w < NW; ++w) tot += red[w][l * 32 + lane];
+            if (a.col_acc[q]) tot = a.yc[q][j] + tot;
+            a.yc[q][j] = tot;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
 namespace {
 
 template <bool DEP>
 const void* fused_fn(int NW, int T) {
+  if (!DEP && getenv("CATT_FUSED_ND") == nullptr) {  // the single-read kernel (CATT_FUSED_ND set: old form)
+    if (NW == 16) {
+      if (T == 2) return (const void*)fused_nd_kernel<16, 2>;
+      if (T == 4) return (const void*)fused_nd_kernel<16, 4>;
+      return (const void*)fused_nd_kernel<16, 8>;
+    }
+    if (T == 1) return (const void*)fused_nd_kernel<8, 1>;
+    return (const void*)fused_nd_kernel<8, 2>;
+  }
   if (NW == 16) {
     if (T == 2) return (const void*)fused_kernel<DEP, 16, 2>;
     if (T == 4) return (const void*)fused_kernel<DEP, 16, 4>;
@@ -288,7 +524,8 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   const int64_t T64 = (n4 + 32 * NW - 1) / (32 * NW);
   if (T64 > 8) return CATT_EUNSUPPORTED;  // N > 16384
   const int T = T64 <= 1 ? 1 : (T64 <= 2 ? 2 : (T64 <= 4 ? 4 : 8));
-  const int threads = NW * 32;
+  const bool nd = !dep && getenv("CATT_FUSED_ND") == nullptr;  // single-read kernel (+1 producer warp)
+  const int threads = (NW + (nd ? 1 : 0)) * 32;
   const void* f = dep ? fused_fn<true>(NW, T) : fused_fn<false>(NW, T);
   // stage = RPS whole rows (~64 KB: several independent row chains per warp
   // and few barriers per byte), S stages within ~200 KB of shared memory
@@ -296,9 +533,20 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   const char* rps_env = getenv("CATT_FUSED_STAGE_KB");
   const int64_t stage_target = (rps_env ? atoi(rps_env) : 64) * 1024;
   const int RPS = int(std::max<int64_t>(1, std::min<int64_t>(16, stage_target / row_bytes)));
-  const int64_t head = 1024 + ((int64_t(RPS) * (NW + 1) * 4 + 1023) / 1024) * 1024;
   const char* budget_env = getenv("CATT_FUSED_SMEM_KB");
   const int64_t budget = (budget_env ? atoi(budget_env) : 200) * 1024;
+  // head: barriers in the first 1 KB, then the row partials (DEP: [RPS][NW+1];
+  // single-read kernel: [S][RPS][NW], sized for up to 16 stages)
+  DevCtx* ctx = nullptr;
+  catt_status st = dev_ctx(&ctx);
+  if (st != CATT_OK) return st;
+  int64_t Mmax = 0;
+  for (int i = 0; i < np; ++i) Mmax = std::max<int64_t>(Mmax, pr[i].M);
+  // ~2x the expected band (one CTA per SM, CTAs split by rows): larger bands
+  // fall back to loading xc / yr per stage
+  const int bandcap = dep ? 0 : int(std::min<int64_t>(kBandMax, (2 * Mmax * np) / ctx->hw.num_sms + 64));
+  const int64_t head =
+      1024 + ((int64_t(RPS) * (NW + 1) * 4 * (dep ? 1 : 32) + 2 * int64_t(bandcap) * 4 + 1023) / 1024) * 1024;
   const int S = int(std::min<int64_t>(16, (budget - head) / (RPS * row_bytes)));
   if (S < 2) return CATT_EUNSUPPORTED;
   const size_t smem = size_t(head + int64_t(S) * RPS * row_bytes);
@@ -313,9 +561,6 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
     record_cuda_error(e);
     return CATT_ECUDA;
   }
-  DevCtx* ctx = nullptr;
-  catt_status st = dev_ctx(&ctx);
-  if (st != CATT_OK) return st;
   // cluster of CL CTAs for the DSMEM pre-reduction (single problem only;
   // default 1: no measured gain at 4096^2, and clustered cooperative launches
   // cannot be replayed by ncu)
@@ -323,7 +568,8 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   const int64_t slots = int64_t(ctx->hw.num_sms) * occ;
   int CL = 1;
   int64_t Gall = std::min<int64_t>(slots, Mtot);
-  for (int cand = (cl_env && np == 1) ? atoi(cl_env) : 1; cand >= 2; cand /= 2) {
+  // the single-read kernel has no cluster pre-reduction
+  for (int cand = (cl_env && np == 1 && !nd) ? atoi(cl_env) : 1; cand >= 2; cand /= 2) {
     if (S * RPS * row_bytes < N * 4) break;
     cudaLaunchConfig_t qc = {};
     qc.gridDim = dim3(unsigned(Gall / cand * cand), 1, 1);
@@ -352,6 +598,7 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   FusedArgs args{};
   args.nprob = np;
   args.N = N;
+  args.bandcap = bandcap;
   int64_t given = 0;
   int cta = 0;
   for (int i = 0; i < np; ++i) {
