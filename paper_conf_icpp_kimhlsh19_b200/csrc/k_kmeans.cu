@@ -19,6 +19,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cfloat>
 #include <cstdint>
 
@@ -166,28 +167,35 @@ __global__ void __launch_bounds__(256) kmeans_stream_kernel(KmArgs a) {
 // tile*256 + t from shared memory (column t of every feature row: conflict
 // free), k partial distances in registers, f ascending: bit-exact membership.
 
-template <int KMAX>
-__global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constant__ CUtensorMap map, KmArgs a,
-                                                            int S) {
+// KP = KMAX rounded up to 4: centres [nf][KP] in shared memory, read as
+// float4; the padding centres are +inf, never strictly nearer than FLT_MAX,
+// so every distance runs unpredicated (k = 5 uses KMAX = 5: no wasted work).
+template <int KMAX, int MINB>
+__global__ void __launch_bounds__(256, MINB) kmeans_tma_kernel(const __grid_constant__ CUtensorMap map, KmArgs a,
+                                                               int S) {
+  constexpr int KP = (KMAX + 3) & ~3;
   extern __shared__ __align__(1024) unsigned char dyn[];
   const int t = threadIdx.x, lane = t & 31, nw = blockDim.x >> 5;
   const int nf = a.nf, k = a.k;
   uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
   uint64_t* empty = full + S;
-  float* s_ct = reinterpret_cast<float*>(dyn + 512);                    // [nf][k] transposed centres
-  const int head = 512 + ((nf * k * 4 + 511) / 512) * 512;
+  float* s_ct = reinterpret_cast<float*>(dyn + 512);                    // [nf][KP] transposed centres
+  const int head = 512 + ((nf * KP * 4 + 511) / 512) * 512;
   float* ring = reinterpret_cast<float*>(dyn + ((head + 1023) / 1024) * 1024);
   const int tile_floats = nf * 256;
   const int64_t ntiles_all = (a.npoints + 255) / 256;
   const int64_t G = gridDim.x;
   const int64_t mytiles = ntiles_all > blockIdx.x ? (ntiles_all - blockIdx.x + G - 1) / G : 0;
-  for (int q = t; q < nf * k; q += blockDim.x) s_ct[(q % nf) * k + q / nf] = a.clusters[q];
+  for (int q = t; q < nf * KP; q += blockDim.x) {
+    const int f = q / KP, cc = q - f * KP;
+    s_ct[q] = cc < k ? a.clusters[cc * nf + f] : __int_as_float(0x7f800000);
+  }
   if (t == 0) {
     for (int s = 0; s < S; ++s) {
       bar_init(&full[s], 1);
       bar_init(&empty[s], nw);
     }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    fence_barrier_init();
   }
   __syncthreads();
   auto issue = [&](int64_t c) {
@@ -210,20 +218,24 @@ __global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constan
 #pragma unroll 4
       for (int f = 0; f < nf; ++f) {
         const float v = col[f * 256];
-        const float* cf = s_ct + f * k;
+        const float4* cf = reinterpret_cast<const float4*>(s_ct + f * KP);
 #pragma unroll
-        for (int cc = 0; cc < KMAX; ++cc) {
-          if (cc < k) {
-            const float diff = v - cf[cc];
-            d[cc] = fmaf(diff, diff, d[cc]);
-          }
+        for (int q = 0; q < KP / 4; ++q) {
+          const float4 c4 = cf[q];
+          const float cv[4] = {c4.x, c4.y, c4.z, c4.w};
+#pragma unroll
+          for (int jj = 0; jj < 4; ++jj)
+            if (4 * q + jj < KMAX) {
+              const float diff = v - cv[jj];
+              d[4 * q + jj] = fmaf(diff, diff, d[4 * q + jj]);
+            }
         }
       }
       int index = -1;
       float best = FLT_MAX;
 #pragma unroll
       for (int cc = 0; cc < KMAX; ++cc) {
-        if (cc < k && d[cc] < best) {
+        if (d[cc] < best) {
           best = d[cc];
           index = cc;
         }
@@ -236,9 +248,27 @@ __global__ void __launch_bounds__(256, 1) kmeans_tma_kernel(const __grid_constan
   }
 }
 
+template <int MINB>
+const void* kmeans_tma_fn(int k) {
+  if (k <= 4) return (const void*)kmeans_tma_kernel<4, MINB>;
+  if (k == 5) return (const void*)kmeans_tma_kernel<5, MINB>;
+  if (k <= 8) return (const void*)kmeans_tma_kernel<8, MINB>;
+  if (k <= 16) return (const void*)kmeans_tma_kernel<16, MINB>;
+  return (const void*)kmeans_tma_kernel<32, MINB>;
+}
+
+// CTAs per SM of the STAGED kernel (2 by default; CATT_KMEANS_CTAS_PER_SM=1: one CTA, more stages)
+int kmeans_tma_minb() {
+  static const int v = [] {
+    const char* e = getenv("CATT_KMEANS_CTAS_PER_SM");
+    return (e && atoi(e) == 1) ? 1 : 2;
+  }();
+  return v;
+}
+
 const void* kmeans_func(int variant, int nf) {
   (void)nf;
-  if (variant == CATT_VAR_STAGED) return (const void*)kmeans_tma_kernel<8>;
+  if (variant == CATT_VAR_STAGED) return kmeans_tma_minb() == 2 ? kmeans_tma_fn<2>(8) : kmeans_tma_fn<1>(8);
   if (variant != CATT_VAR_REGS) return (const void*)kmeans_kernel<0>;
   return (const void*)kmeans_stream_kernel<8>;
 }
@@ -269,10 +299,14 @@ catt_status launch_kmeans_tma(const float* feat, int64_t ld, int64_t npoints, in
           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
     return CATT_EINVAL;
   const int tile_bytes = nf * 256 * 4;
-  const int head = ((512 + ((nf * k * 4 + 511) / 512) * 512 + 1023) / 1024) * 1024;
-  const int S = std::max(2, std::min(8, (200 * 1024 - head) / tile_bytes));
+  const int KMAX = k <= 4 ? 4 : k == 5 ? 5 : k <= 8 ? 8 : k <= 16 ? 16 : 32;
+  const int KP = (KMAX + 3) & ~3;
+  const int head = ((512 + ((nf * KP * 4 + 511) / 512) * 512 + 1023) / 1024) * 1024;
+  const int minb = kmeans_tma_minb();
+  const int budget = (minb == 2 ? 108 : 200) * 1024;
+  const int S = std::max(2, std::min(8, (budget - head) / tile_bytes));
   const size_t smem = size_t(head) + size_t(S) * tile_bytes;
-  const void* f = k <= 8 ? (const void*)kmeans_tma_kernel<8> : (const void*)kmeans_tma_kernel<32>;
+  const void* f = minb == 2 ? kmeans_tma_fn<2>(k) : kmeans_tma_fn<1>(k);
   cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) {
     record_cuda_error(e);
@@ -285,13 +319,22 @@ catt_status launch_kmeans_tma(const float* feat, int64_t ld, int64_t npoints, in
   DevCtx* ctx = nullptr;
   st = dev_ctx(&ctx);
   if (st != CATT_OK) return st;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, 256, dyn_total);
+  if (e != cudaSuccess || per_sm < 1) {
+    record_cuda_error(e == cudaSuccess ? cudaErrorInvalidConfiguration : e);
+    return CATT_ECUDA;
+  }
   const int64_t tiles = (npoints + 255) / 256;
-  const unsigned grid = unsigned(std::min<int64_t>(tiles, ctx->hw.num_sms));
+  const unsigned grid = unsigned(std::min<int64_t>(tiles, int64_t(std::min(per_sm, minb)) * ctx->hw.num_sms));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  if (k <= 8)
-    kmeans_tma_kernel<8><<<grid, 256, dyn_total, s>>>(map, a, S);
-  else
-    kmeans_tma_kernel<32><<<grid, 256, dyn_total, s>>>(map, a, S);
+  int stages = S;
+  void* args[] = {&map, &a, &stages};
+  e = cudaLaunchKernel(f, dim3(grid), dim3(256), args, dyn_total, s);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
   return after_launch();
 }
 
