@@ -412,7 +412,12 @@ class Syrk(Workload):
         t = self.plan("syrk", catt.problem(catt.K_SYRK, n=n, k=n), catt.Throttle(variant=self.variant))
         self.flops = 2 * n * n * n
         self.loops = [Loop("syrk", lambda: catt.syrk(self.A, self.C, 1.5, 1.2, t=t), 3 * n * n * 4, "syrk")]
-        self.study = None
+        # SURVEY 8(d) [3]: the discriminating experiment. Paper mode predicts a
+        # throttle at the 8 KB carveout, union mode none; the measurement decides.
+        Cs = self.C.clone()
+        self.study = dict(name="syrk (literal, 2-D block 32 x 8)", prob=catt.problem(catt.K_SYRK, n=n, k=n),
+                          launches=[(256, 8), (256, 100), (256, 228)], reps=2,
+                          fn=lambda th: (lambda: catt.syrk(self.A, Cs, 1.5, 1.2, t=th)))
 
     def inputs(self):
         return [self.A, self.C]
@@ -570,6 +575,18 @@ def time_loops(torch, w, flush, steps, warmup, barrier):
     return steps_ms, per_loop, coll
 
 
+def study_fn(catt, w, th):
+    """The study loop of workload w launched with throttle th (a callable)."""
+    S = w.study
+    if S.get("fn"):
+        return S["fn"](th)
+    if S.get("kmeans"):
+        return lambda: catt.kmeans_assign(w.feat, w.ld, w.np_, w.nf, w.clusters, w.memb, t=th)
+    if S.get("gesummv"):
+        return lambda: catt.rows(w.A, w.x, w.y, catt.ROWS_GESUMMV, w.B, w.tmp, 1.5, 1.2, th)
+    return lambda: catt.rows(S["A"], S["x"], S["y"], catt.ROWS_STORE, t=th)
+
+
 def throttle_study(catt, torch, w, flush):
     """CATT's pick vs full TLP vs the exhaustively swept best static throttle
     for the paper's literal loop at launches where the union model says the
@@ -606,15 +623,7 @@ def throttle_study(catt, torch, w, flush):
         times = {}
         for a, m in cands:
             th = launch.copy(active_warps=a, active_ctas=m if m < T else 0)
-            if S.get("fn"):
-                fn = S["fn"](th)
-            elif S.get("kmeans"):
-                fn = lambda th=th: catt.kmeans_assign(w.feat, w.ld, w.np_, w.nf, w.clusters, w.memb, t=th)
-            elif S.get("gesummv"):
-                fn = lambda th=th: catt.rows(w.A, w.x, w.y, catt.ROWS_GESUMMV, w.B, w.tmp, 1.5, 1.2, th)
-            else:
-                fn = lambda th=th: catt.rows(S["A"], S["x"], S["y"], catt.ROWS_STORE, t=th)
-            times[(a, m)] = med(fn, S.get("reps", 5))
+            times[(a, m)] = med(study_fn(catt, w, th), S.get("reps", 5))
         pick = (t.active_warps or W, t.active_ctas or T)
         pick_p = (tp.active_warps or W, tp.active_ctas or T)
         best = min(times, key=times.get)
