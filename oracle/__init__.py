@@ -55,6 +55,8 @@ def lib():
         L.orc_syrk.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float]
         L.orc_syrk_rows.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float,
                                     ctypes.POINTER(ctypes.c_int64), i64, f32p]
+        L.orc_gemm.argtypes = [ctypes.c_int, f32p, f32p, f32p, i64, i64, i64, ctypes.c_float, ctypes.c_float]
+        L.orc_corr.argtypes = [ctypes.c_int, f32p, i64, i64, f32p, f32p, f32p]
         L.orc_syr2k.argtypes = [ctypes.c_int, f32p, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float]
         L.orc_syr2k_rows.argtypes = [ctypes.c_int, f32p, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float,
                                      ctypes.POINTER(ctypes.c_int64), i64, f32p]
@@ -156,6 +158,26 @@ def syr2k_rows(A, B, C, alpha, beta, rows, mode=SEQ_FMAF):
     out = np.empty((len(rows), n), np.float32)
     lib().orc_syr2k_rows(mode, _p(A), _p(B), _p(C), n, m, alpha, beta, _p(rows), len(rows), _p(out))
     return out
+
+
+def gemm(A, B, C, alpha, beta, mode=SEQ_FMAF):
+    """C := beta C + alpha A B (PolyBench gemm order); returns the new C."""
+    A, B, C = _f32(A), _f32(B), _f32(C).copy()
+    ni, nk = A.shape
+    nj = B.shape[1]
+    lib().orc_gemm(mode, _p(A), _p(B), _p(C), ni, nj, nk, alpha, beta)
+    return C
+
+
+def corr(data, mode=SEQ_FMAF):
+    """PolyBench correlation of the columns of data (n x m).
+    Returns (symmat m x m, mean, std, centred-and-scaled data)."""
+    d = _f32(data).copy()
+    n, m = d.shape
+    mean, std = np.empty(m, np.float32), np.empty(m, np.float32)
+    sym = np.empty((m, m), np.float32)
+    lib().orc_corr(mode, _p(d), n, m, _p(mean), _p(std), _p(sym))
+    return sym, mean, std, d
 
 
 def kmeans_assign(feat, ld, npoints, nf, clusters, mode=SEQ_FMAF):

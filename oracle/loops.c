@@ -279,6 +279,95 @@ int orc_syr2k_rows(int mode, const float* A, const float* B, const float* C, int
   return 0;
 }
 
+/* ---------------------------------------------------------------- GEMM
+ * PolyBench/GPU gemm (Table 2 CI group; the cache-insensitive
+ * negative control of SURVEY 8(f) f3 / P:397). A is ni x nk, B nk x nj,
+ * C ni x nj in/out:
+ *   c[i][j] *= beta;  for k: c[i][j] += alpha * a[i][k] * b[k][j]
+ * evaluated as c = fmaf(alpha * a_ik (rounded), b_kj, c), k ascending.   */
+int orc_gemm(int mode, const float* A, const float* B, float* C, int64_t ni, int64_t nj, int64_t nk, float alpha,
+             float beta) {
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < ni; ++i) {
+    for (int64_t j = 0; j < nj; ++j) {
+      if (mode == ORC_SEQ_FMAF) {
+        float c = C[i * nj + j] * beta;
+        for (int64_t k = 0; k < nk; ++k) c = fmaf(alpha * A[i * nk + k], B[k * nj + j], c);
+        C[i * nj + j] = c;
+      } else {
+        double c = (double)C[i * nj + j] * (double)beta;
+        for (int64_t k = 0; k < nk; ++k) c += (double)alpha * (double)A[i * nk + k] * (double)B[k * nj + j];
+        C[i * nj + j] = (float)c;
+      }
+    }
+  }
+  return 0;
+}
+
+/* ---------------------------------------------------------------- CORR
+ * PolyBench/GPU correlation (Table 2; Table 3; the give-up case
+ * of P:244 and P:395). data is n x m (rows = observations, columns =
+ * variables), centred and scaled in place; per column, i ascending:
+ *   mean[j] = (sum_i data[i][j]) / fn
+ *   std[j]  = sqrtf((sum_i fmaf(d, d, .), d = data[i][j] - mean[j]) / fn),
+ *             std[j] = 1 if std[j] <= eps
+ *   data[i][j] = (data[i][j] - mean[j]) / (sqrtf(fn) * std[j])
+ *   symmat[j1][j1] = 1;  for j2 > j1: s = 0; for i: s = fmaf(data[i][j1], data[i][j2], s);
+ *                        symmat[j1][j2] = symmat[j2][j1] = s
+ * with fn = (float)n and eps = 0.005f (R22). Mode ORC_SEQ_F64
+ * runs the same steps in double (rounded to float at the end of each). */
+int orc_corr(int mode, float* data, int64_t n, int64_t m, float* mean, float* stdv, float* symmat) {
+  const float fn = (float)n, eps = 0.005f;
+#pragma omp parallel for schedule(static)
+  for (int64_t j = 0; j < m; ++j) {
+    if (mode == ORC_SEQ_FMAF) {
+      float mu = 0.0f;
+      for (int64_t i = 0; i < n; ++i) mu = mu + data[i * m + j];
+      mu = mu / fn;
+      float sd = 0.0f;
+      for (int64_t i = 0; i < n; ++i) {
+        const float d = data[i * m + j] - mu;
+        sd = fmaf(d, d, sd);
+      }
+      sd = sqrtf(sd / fn);
+      if (sd <= eps) sd = 1.0f;
+      const float scale = sqrtf(fn) * sd;
+      for (int64_t i = 0; i < n; ++i) data[i * m + j] = (data[i * m + j] - mu) / scale;
+      mean[j] = mu;
+      stdv[j] = sd;
+    } else {
+      double mu = 0.0;
+      for (int64_t i = 0; i < n; ++i) mu += data[i * m + j];
+      mu /= (double)n;
+      double sd = 0.0;
+      for (int64_t i = 0; i < n; ++i) sd += ((double)data[i * m + j] - mu) * ((double)data[i * m + j] - mu);
+      sd = sqrt(sd / (double)n);
+      if (sd <= (double)eps) sd = 1.0;
+      for (int64_t i = 0; i < n; ++i) data[i * m + j] = (float)(((double)data[i * m + j] - mu) / (sqrt((double)n) * sd));
+      mean[j] = (float)mu;
+      stdv[j] = (float)sd;
+    }
+  }
+#pragma omp parallel for schedule(dynamic, 4)
+  for (int64_t j1 = 0; j1 < m; ++j1) {
+    symmat[j1 * m + j1] = 1.0f;
+    for (int64_t j2 = j1 + 1; j2 < m; ++j2) {
+      float s;
+      if (mode == ORC_SEQ_FMAF) {
+        s = 0.0f;
+        for (int64_t i = 0; i < n; ++i) s = fmaf(data[i * m + j1], data[i * m + j2], s);
+      } else {
+        double d = 0.0;
+        for (int64_t i = 0; i < n; ++i) d += (double)data[i * m + j1] * (double)data[i * m + j2];
+        s = (float)d;
+      }
+      symmat[j1 * m + j2] = s;
+      symmat[j2 * m + j1] = s;
+    }
+  }
+  return 0;
+}
+
 /* ---------------------------------------------------------------- KMEANS assign
  * Rodinia kmeans (Table 2; Table 3), assignment step
  * (kmeansPoint), features stored feature-major: feat[f*ld + p].

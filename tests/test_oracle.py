@@ -435,3 +435,51 @@ def test_no_locality_no_throttle():
     hw = _hw_small([4, 4, 4, 4])
     res = fp.analyse(_row_loop(256, 4, 256, 1, vec=4), hw)
     assert res["flags"] == fp.FIT_NONE_NEEDED and res["active_warps"] == 8
+
+
+def test_gemm_pins():
+    """PolyBench gemm (CI negative control)."""
+    rng = np.random.default_rng(11)
+    A = rng.random((37, 23), dtype=np.float32)
+    B = rng.random((23, 19), dtype=np.float32)          # non-square: a transposed operand fails
+    C = rng.random((37, 19), dtype=np.float32)
+    got = oracle.gemm(A, B, C, 1.5, 1.2)
+    ref = 1.2 * C.astype(np.float64) + 1.5 * (A.astype(np.float64) @ B.astype(np.float64))
+    assert np.max(np.abs(got - ref) / np.abs(ref)) < 4 * 23 * 2.0 ** -24
+    assert np.array_equal(oracle.gemm(A, B, C, 0.0, 1.25), (C * np.float32(1.25)).astype(np.float32))
+    # the same evaluation order as SYRK: gemm(A, A^T) is syrk(A) bit for bit
+    S = rng.random((29, 17), dtype=np.float32)
+    Cs = rng.random((29, 29), dtype=np.float32)
+    assert np.array_equal(oracle.gemm(S, np.ascontiguousarray(S.T), Cs, 1.5, 1.2), oracle.syrk(S, Cs, 1.5, 1.2))
+    # exact-dyadic inputs: every partial sum exact -> equal to numpy exactly
+    Ad = (rng.integers(0, 16, (40, 31)) / 16).astype(np.float32)
+    Bd = (rng.integers(0, 16, (31, 12)) / 16).astype(np.float32)
+    Cd = (rng.integers(0, 16, (40, 12)) / 16).astype(np.float32)
+    want = (np.float64(1.25) * Cd + 1.5 * (Ad.astype(np.float64) @ Bd)).astype(np.float32)
+    assert np.array_equal(oracle.gemm(Ad, Bd, Cd, 1.5, 1.25), want)
+
+
+def test_corr_pins():
+    """PolyBench correlation: Pearson correlation of the columns."""
+    rng = np.random.default_rng(12)
+    n, m = 300, 9
+    data = (rng.standard_normal((n, m)) * rng.uniform(0.5, 3, m) + rng.uniform(-2, 2, m)).astype(np.float32)
+    data[:, 3] += 0.7 * data[:, 1]                        # a correlated pair
+    sym, mean, std, centred = oracle.corr(data)
+    ref = np.corrcoef(data.astype(np.float64).T)
+    assert np.max(np.abs(sym - ref)) < 2e-5
+    assert np.array_equal(sym, sym.T) and np.all(np.diag(sym) == 1.0)
+    assert np.allclose(mean, data.astype(np.float64).mean(0), rtol=1e-5, atol=1e-6)
+    assert np.allclose(std, data.astype(np.float64).std(0), rtol=1e-5)
+    assert np.allclose(centred, (data - data.mean(0)) / (np.sqrt(n) * data.std(0)), rtol=1e-4, atol=1e-6)
+    # affine invariance of the definition
+    sym2, _, _, _ = oracle.corr(data * 2.0 + 3.0)
+    assert np.max(np.abs(sym2 - sym)) < 2e-5
+    # a constant column: std <= eps -> 1, so its correlations are ~0, not NaN
+    data[:, 5] = 0.25
+    sym3, _, std3, _ = oracle.corr(data)
+    assert std3[5] == 1.0 and np.all(np.isfinite(sym3))
+    assert np.max(np.abs(np.delete(sym3[5], 5))) < 1e-6
+    # the fp64 mode is the textbook value
+    sym64, _, _, _ = oracle.corr(data[:, :5], mode=oracle.SEQ_F64)
+    assert np.max(np.abs(sym64 - np.corrcoef(data[:, :5].astype(np.float64).T))) < 1e-6
