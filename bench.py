@@ -44,7 +44,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--workload", default="bicg_mvt",
-                   choices=["bicg_mvt", "kmeans", "kmeans_iter", "gesummv", "syrk", "syr2k", "atax256", "atax"])
+                   choices=["bicg_mvt", "kmeans", "kmeans_iter", "gesummv", "syrk", "syr2k", "corr", "gemm", "atax256", "atax"])
     p.add_argument("--variant", default=None,
                    help="fused (default for bicg_mvt/atax), fused1, coop, staged, vec4, literal, regs (kmeans)")
     p.add_argument("--impl", default="catt", choices=["catt", "reference"])
@@ -469,6 +469,80 @@ class Syr2k(Workload):
         oracle.syr2k_rows(host["A"], host["B"], host["C"], 1.5, 1.2, np.arange(16))
 
 
+class Corr(Workload):
+    name = "corr"
+    desc = "CORR 2048 x 2048 fp32 (Table 2 P:81; the give-up case of P:395; SURVEY 8(f) f3)"
+    variant = "staged"
+
+    def __init__(self, catt, torch, rank, world, variant):
+        super().__init__(catt, torch, rank, world, variant)
+        import seeded_inputs as si
+        n = m = 2048
+        self.n, self.m = n, m
+        dev = torch.device("cuda")
+        self.data = torch.empty(n, m, device=dev)
+        catt.fill_hash(self.data, si.SEED_CORR + rank)
+        self.mean, self.std = torch.empty(m, device=dev), torch.empty(m, device=dev)
+        self.sym = torch.empty(m, m, device=dev)
+        self.work = torch.empty(n * m, device=dev)
+        prob = catt.problem(catt.K_CORR, n=m, k=n)
+        t = self.plan("corr", prob, catt.Throttle(variant=self.variant))
+        self.flops = m * m * n                               # the symmetric half, 2 flop per fmaf
+        self.loops = [Loop("corr", lambda: catt.corr(self.data, self.mean, self.std, self.sym, self.work, t=t),
+                           n * m * 4 * 2 + m * m * 4, "corr")]
+        d2 = self.data.clone()
+        self.study = dict(name="corr loop (literal, thread per column j1)", prob=prob,
+                          launches=[(256, 8), (256, 228)], reps=2,
+                          fn=lambda th: (lambda: catt.corr(d2, self.mean, self.std, self.sym, t=th)))
+
+    def inputs(self):
+        return [self.data]
+
+    def outputs(self):
+        return [self.sym]
+
+    def host_copy(self):
+        return {"data": self.data.cpu().numpy()[:256, :256].copy()}
+
+    def cpu_oracle_step(self, oracle, host):
+        oracle.corr(host["data"])
+
+
+class Gemm(Workload):
+    name = "gemm"
+    desc = "GEMM 512 x 512 fp32 (Table 2 CI group: the cache-insensitive negative control, P:397)"
+    variant = "staged"
+
+    def __init__(self, catt, torch, rank, world, variant):
+        super().__init__(catt, torch, rank, world, variant)
+        import seeded_inputs as si
+        n = 512
+        dev = torch.device("cuda")
+        self.A, self.B, self.C = (torch.empty(n, n, device=dev) for _ in range(3))
+        for q, x in enumerate((self.A, self.B, self.C)):
+            catt.fill_hash(x, si.sub_seed(si.SEED_GEMM, q) + rank)
+        prob = catt.problem(catt.K_GEMM, m=n, n=n, k=n)
+        t = self.plan("gemm", prob, catt.Throttle(variant=self.variant))
+        self.flops = 2 * n * n * n
+        self.loops = [Loop("gemm", lambda: catt.gemm(self.A, self.B, self.C, 1.5, 1.2, t=t), 4 * n * n * 4, "gemm")]
+        Cs = self.C.clone()
+        self.study = dict(name="gemm (literal, 2-D block 32 x 8)", prob=prob,
+                          launches=[(256, 8), (256, 228), (1024, 196)], reps=3,
+                          fn=lambda th: (lambda: catt.gemm(self.A, self.B, Cs, 1.5, 1.2, t=th)))
+
+    def inputs(self):
+        return [self.A, self.B, self.C]
+
+    def outputs(self):
+        return [self.C]
+
+    def host_copy(self):
+        return {k: getattr(self, k).cpu().numpy() for k in ("A", "B", "C")}
+
+    def cpu_oracle_step(self, oracle, host):
+        oracle.gemm(host["A"], host["B"], host["C"], 1.5, 1.2)
+
+
 class Atax(Workload):
     name = "atax"
     variant = "fused"
@@ -535,7 +609,8 @@ class Atax256(Atax):
         super().__init__(catt, torch, rank, world, variant, m=256, n=256)
 
 
-WORKLOADS = {"bicg_mvt": BicgMvt, "kmeans": Kmeans, "kmeans_iter": KmeansIter, "gesummv": Gesummv, "syrk": Syrk, "syr2k": Syr2k, "atax256": Atax256,
+WORKLOADS = {"bicg_mvt": BicgMvt, "kmeans": Kmeans, "kmeans_iter": KmeansIter, "gesummv": Gesummv, "syrk": Syrk, "syr2k": Syr2k,
+             "corr": Corr, "gemm": Gemm, "atax256": Atax256,
              "atax": Atax}
 
 
@@ -870,7 +945,7 @@ def main():
     dom = max((i for i in range(len(w.loops)) if w.loops[i].kind != "collective"), key=lambda i: loop_ms[i])
     lp = w.loops[dom]
     peak, peak_src = peak_hbm()
-    if lp.kind in ("syrk", "syr2k"):
+    if lp.kind in ("syrk", "syr2k", "corr", "gemm"):
         # FP32 CUDA-core bound: 148 SMs x 128 FP32 lanes x 2 flop x clock
         clk_mhz = clk.get("sm_mhz") or 1965.0
         peak_t = 148 * 128 * 2 * clk_mhz * 1e6 / 1e12
@@ -887,7 +962,7 @@ def main():
     # ---- context: a plain device copy moving the same bytes as the dominant
     # loop, timed the same way (flush, queued events). At 64 MiB a single
     # kernel cannot reach the 2 GiB copy peak of MEASURED_PEAKS.json.
-    if lp.kind not in ("syrk", "syr2k"):
+    if lp.kind not in ("syrk", "syr2k", "corr", "gemm"):
         half = max(1, lp.nbytes // 8)                # floats per side: read + write = nbytes
         src = torch.empty(half, device="cuda")
         dst = torch.empty(half, device="cuda")
@@ -937,6 +1012,8 @@ def main():
             cpu_bytes = step_bytes
             if w.name in ("syrk", "syr2k"):
                 cpu_bytes = step_bytes * 16 / 2048
+            if w.name == "corr":                         # the oracle runs a 256 x 256 sample of the data
+                cpu_bytes = 256 * 256 * 4 * 3
             if w.name == "atax":
                 cpu_bytes = step_bytes * min(w.rows, 8192) / w.rows
             cpu = {"value": round(cpu_bytes / sec / 1e9, 3), "unit": "GB/s", "cores": oracle.num_threads(),

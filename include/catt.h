@@ -199,11 +199,14 @@ enum {
   CATT_K_KMEANS = 8,  /* membership = argmin_c |f_p - c|^2, feature-major     */
   CATT_K_SYR2K = 9,   /* C = beta C + alpha (A B^T + B A^T), 2-D block 32 x 8 */
   CATT_K_KMEANS_T = 10, /* KM transpose: out[f*ld + p] = in[p*nf + f]          */
-  CATT_K_COUNT = 11
+  CATT_K_CORR = 11,   /* CORR loop: symmat[j1][j2] = sum_i d[i][j1] d[i][j2]   */
+  CATT_K_GEMM = 12,   /* C = beta C + alpha A B, 2-D block 32 x 8 (CI control) */
+  CATT_K_COUNT = 13
 };
 
 /* Problem sizes: ATAX/BICG m x n (rows, cols); MVT/GESUMMV n (m ignored);
- * SYRK/SYR2K n x n output, k = inner size m; KMEANS m = npoints, n = nfeatures,
+ * SYRK/SYR2K n x n output, k = inner size m; GEMM m = ni, n = nj, k = nk;
+ * CORR n = columns m, k = rows n; KMEANS m = npoints, n = nfeatures,
  * k = clusters, ld = feature-major leading dimension. */
 typedef struct {
   int32_t loop;
@@ -274,6 +277,24 @@ catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alph
  * tiles with the same order. */
 catt_status catt_syr2k(const float* A, const float* B, float* C, int64_t n, int64_t m, float alpha, float beta,
                        const catt_throttle* t, void* stream);
+
+/* GEMM (Table 2 CI group; the cache-insensitive negative control):
+ * C (ni x nj, in/out) = beta*C + alpha*A*B, A ni x nk, B nk x nj, row-major.
+ * Per element, k ascending: c = fmaf(alpha*a_ik, b_kj, c) (alpha*a_ik rounded).
+ * LITERAL = 2-D block 32 x (cta_threads/32); STAGED = the tiled kernel. */
+catt_status catt_gemm(const float* A, const float* B, float* C, int64_t ni, int64_t nj, int64_t nk, float alpha,
+                      float beta, const catt_throttle* t, void* stream);
+
+/* CORR (Table 2; Table 3; the give-up case of P:244):
+ * Pearson correlation of the m columns of data (n x m, row-major). data is
+ * centred and scaled in place; mean[m], stdv[m] and symmat[m x m] are
+ * outputs (R22 gives the per-column order, fn = n, eps = 0.005).
+ * LITERAL: thread per column for the statistics, then the paper's loop
+ * (thread per j1; the throttle applies to it, CATT_K_CORR). STAGED: work is
+ * a device buffer of m*n floats (the transposed columns) and symmat is
+ * computed by the tiled SYRK kernel: bit-identical to LITERAL. */
+catt_status catt_corr(float* data, int64_t n, int64_t m, float* mean, float* stdv, float* symmat, float* work,
+                      const catt_throttle* t, void* stream);
 
 /* KMEANS assignment (Table 2, Table 3): feat is feature-major,
  * feat[f*ld + p] for f < nf, p < npoints (ld >= npoints); clusters is k x nf;

@@ -145,6 +145,35 @@ class Syr2kKernel(SyrkKernel):
         return ev
 
 
+class GemmKernel(Kernel):
+    """PolyBench/GPU gemm, block (32, 8): j = bx*32 + tx, i = by*8 + ty,
+    for k < nk: c += alpha * a[i*nk + k] * b[k*nj + j]."""
+
+    def __init__(self, ni, nj, nk, bdim=(32, 8)):
+        self.ni, self.nj, self.nk, self.bdim = ni, nj, nk, bdim
+        self.threads = bdim[0] * bdim[1]
+        self.W = (self.threads + 31) // 32
+        self.gx = (nj + bdim[0] - 1) // bdim[0]
+        self.gy = (ni + bdim[1] - 1) // bdim[1]
+        self.nblocks = self.gx * self.gy
+
+    def events(self, b, w):
+        bx, by = b % self.gx, b // self.gx
+        th = []
+        for t in self.lanes(b, w):
+            tx, ty = t % self.bdim[0], t // self.bdim[0]
+            i, j = by * self.bdim[1] + ty, bx * self.bdim[0] + tx
+            if i < self.ni and j < self.nj:
+                th.append((i, j))
+        ev = []
+        if not th:
+            return ev
+        for k in range(self.nk):
+            ev.append(tuple((_line("a", i * self.nk + k), (i, j)) for i, j in th))
+            ev.append(tuple((_line("b", k * self.nj + j), (i, j)) for i, j in th))
+        return ev
+
+
 class KmeansKernel(Kernel):
     """Rodinia kmeansPoint, feature-major: thread p (p < npoints):
     for c < k: for f < nf: diff = feat[f*ld + p] - clusters[c*nf + f]

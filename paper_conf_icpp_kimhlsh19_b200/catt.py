@@ -28,7 +28,7 @@ ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
 (K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K,
- K_KMEANS_T) = range(11)
+ K_KMEANS_T, K_CORR, K_GEMM) = range(13)
 
 VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS,
             "fused": VAR_FUSED}
@@ -162,6 +162,8 @@ def lib():
             "catt_gesummv": [V, V, V, V, V, i64, f32, f32, T, V],
             "catt_syrk": [V, V, i64, i64, f32, f32, T, V],
             "catt_syr2k": [V, V, V, i64, i64, f32, f32, T, V],
+            "catt_gemm": [V, V, V, i64, i64, i64, f32, f32, T, V],
+            "catt_corr": [V, i64, i64, V, V, V, V, T, V],
             "catt_kmeans_assign": [V, i64, i64, i32, V, i32, V, T, V],
             "catt_kmeans_transpose": [V, V, i64, i32, i64, T, V],
             "catt_kmeans_accumulate": [V, i64, i64, i32, V, i32, V, V, V],
@@ -190,7 +192,7 @@ def lib():
 
 
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
-            "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_kmeans_assign",
+            "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_gemm", "catt_corr", "catt_kmeans_assign",
             "catt_kmeans_acc_words", "catt_kmeans_transpose", "catt_kmeans_accumulate", "catt_kmeans_finalize",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version"]
@@ -425,6 +427,34 @@ def kmeans_assign(feat, ld, npoints, nf, clusters, membership=None, t: Optional[
                                     _dev(membership, "membership", torch.int32), _tp(t), _stream()),
            "catt_kmeans_assign")
     return membership
+
+
+def gemm(A, B, C, alpha, beta, t: Optional[Throttle] = None):
+    """C = beta C + alpha A B in place (catt_gemm). Returns C."""
+    ni, nk = A.shape
+    nj = B.shape[1]
+    _check(lib().catt_gemm(_dev(A, "A"), _dev(B, "B"), _dev(C, "C"), ni, nj, nk, float(alpha), float(beta), _tp(t),
+                           _stream()), "catt_gemm")
+    return C
+
+
+def corr(data, mean=None, stdv=None, symmat=None, work=None, t: Optional[Throttle] = None):
+    """Pearson correlation of the columns of data (n x m, centred and scaled in
+    place). Returns (symmat, mean, stdv). STAGED needs a work buffer of n*m floats
+    (allocated here when not given)."""
+    torch = _torch()
+    n, m = data.shape
+    mk = lambda shape: torch.empty(shape, dtype=torch.float32, device=data.device)
+    mean = mk(m) if mean is None else mean
+    stdv = mk(m) if stdv is None else stdv
+    symmat = mk((m, m)) if symmat is None else symmat
+    staged = t is not None and t.variant == VAR_STAGED
+    if staged and work is None:
+        work = mk(n * m)
+    wp = _dev(work, "work") if work is not None else None
+    _check(lib().catt_corr(_dev(data, "data"), n, m, _dev(mean, "mean"), _dev(stdv, "stdv"), _dev(symmat, "symmat"),
+                           wp, _tp(t), _stream()), "catt_corr")
+    return symmat, mean, stdv
 
 
 def kmeans_acc_words(k: int, nf: int) -> int:

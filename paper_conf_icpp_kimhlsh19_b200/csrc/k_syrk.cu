@@ -95,40 +95,45 @@ __global__ void __launch_bounds__(1024, 2) syr2k_thread_kernel(Syr2kArgs a) {
 // the result is bit-identical to LITERAL (and to the oracle). Stage arrays:
 //   SYRK : 0 = alpha*a[i][k], 1 = a[j][k]
 //   SYR2K: 0 = alpha*a[i][k], 1 = b[j][k], 2 = alpha*b[i][k], 3 = a[j][k]
+//   GEMM : 0 = alpha*a[i][k], 1 = b[k][j] (B is k-major: loaded without a transpose)
+// C is ni x nj (SYRK/SYR2K: ni = nj = n), the inner size is m.
+constexpr int MODE_SYRK = 0, MODE_SYR2K = 1, MODE_GEMM = 2;
 constexpr int BM = 128, TM = 8;
 constexpr int PITCH = BM + 4;  // transposed stage rows: 16-B aligned, store banks spread
 
 struct TileArgs {
   const float* A;
-  const float* B;  // SYR2K only
+  const float* B;  // SYR2K, GEMM
   float* C;
-  int64_t n, m;
+  int64_t ni, nj, m;
   float alpha, beta;
-  int vec;  // m % 4 == 0 and A, B 16-B aligned: float4 global loads
-  int cvec; // n % 4 == 0 and C 16-B aligned
+  int vec;  // m % 4 == 0 and A (SYR2K: and B) 16-B aligned: float4 loads along k
+  int bvec; // GEMM: nj % 4 == 0 and B 16-B aligned: float4 loads of B rows
+  int cvec; // nj % 4 == 0 and C 16-B aligned
   Throttle t;
 };
 
-template <bool TWO>
+template <int MODE>
 struct TileCfg {
-  static constexpr int BK = TWO ? 8 : 16;
-  static constexpr int NA = TWO ? 4 : 2;
+  static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
+  static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int KQ = BK / 4;            // float4 per stage row
   static constexpr int NV = BM * KQ / 256;     // float4 per thread per array per stage
 };
 
 __device__ __forceinline__ int tile_off(int t, int r) { return r < 4 ? t * 4 + r : 64 + t * 4 + (r - 4); }
 
-template <bool TWO, int MINB>
+template <int MODE, int MINB>
 __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
-  using Cfg = TileCfg<TWO>;
+  constexpr bool TWO = MODE == MODE_SYR2K, GEMM = MODE == MODE_GEMM;
+  using Cfg = TileCfg<MODE>;
   constexpr int BK = Cfg::BK, NA = Cfg::NA, KQ = Cfg::KQ, NV = Cfg::NV;
   __shared__ __align__(16) float S[2][NA][BK][PITCH];
   cta_enter(a.t);
   const int tid = threadIdx.x;
   const int tx = tid & 15, ty = tid >> 4;
   const int64_t i0 = int64_t(blockIdx.y) * BM, j0 = int64_t(blockIdx.x) * BM;
-  const int64_t n = a.n, m = a.m;
+  const int64_t ni = a.ni, nj = a.nj, m = a.m;
 
   float c[TM][TM];
 #pragma unroll
@@ -137,8 +142,8 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
       const int64_t gj = j0 + 64 * h + tx * 4;
-      if (a.cvec && gi < n && gj + 3 < n) {
-        const float4 v = *reinterpret_cast<const float4*>(a.C + gi * n + gj);
+      if (a.cvec && gi < ni && gj + 3 < nj) {
+        const float4 v = *reinterpret_cast<const float4*>(a.C + gi * nj + gj);
         c[r][4 * h] = __fmul_rn(v.x, a.beta);
         c[r][4 * h + 1] = __fmul_rn(v.y, a.beta);
         c[r][4 * h + 2] = __fmul_rn(v.z, a.beta);
@@ -146,7 +151,7 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
       } else {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          c[r][4 * h + q] = (gi < n && gj + q < n) ? __fmul_rn(a.C[gi * n + gj + q], a.beta) : 0.0f;
+          c[r][4 * h + q] = (gi < ni && gj + q < nj) ? __fmul_rn(a.C[gi * nj + gj + q], a.beta) : 0.0f;
       }
     }
   }
@@ -164,12 +169,28 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
       const int64_t k = k0 + (idx % KQ) * 4;
 #pragma unroll
       for (int s = 0; s < NA; ++s) {
+        if (GEMM && s == 1) {  // B rows k0 + kk, columns j0 + 4*c4 .. +3
+          const int kk = idx >> 5, c4 = idx & 31;
+          const int64_t kb = k0 + kk, jb = j0 + 4 * c4;
+          const float* Bp = a.B + kb * nj + jb;
+          if (a.bvec && kb < m && jb + 3 < nj) {
+            ld[1][v] = __ldg(reinterpret_cast<const float4*>(Bp));
+          } else {
+            const bool ok = kb < m;
+            ld[1][v].x = (ok && jb < nj) ? Bp[0] : 0.0f;
+            ld[1][v].y = (ok && jb + 1 < nj) ? Bp[1] : 0.0f;
+            ld[1][v].z = (ok && jb + 2 < nj) ? Bp[2] : 0.0f;
+            ld[1][v].w = (ok && jb + 3 < nj) ? Bp[3] : 0.0f;
+          }
+          continue;
+        }
         const int64_t g = (is_row(s) ? i0 : j0) + row;
+        const int64_t gl = is_row(s) ? ni : nj;
         const float* M = src(s);
-        if (a.vec && g < n && k + 3 < m) {
+        if (a.vec && g < gl && k + 3 < m) {
           ld[s][v] = __ldg(reinterpret_cast<const float4*>(M + g * m + k));
         } else {
-          const bool ok = g < n;
+          const bool ok = g < gl;
           ld[s][v].x = (ok && k < m) ? M[g * m + k] : 0.0f;
           ld[s][v].y = (ok && k + 1 < m) ? M[g * m + k + 1] : 0.0f;
           ld[s][v].z = (ok && k + 2 < m) ? M[g * m + k + 2] : 0.0f;
@@ -186,6 +207,10 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 #pragma unroll
       for (int s = 0; s < NA; ++s) {
         float4 x = ld[s][v];
+        if (GEMM && s == 1) {
+          *reinterpret_cast<float4*>(&S[buf][1][idx >> 5][4 * (idx & 31)]) = x;
+          continue;
+        }
         if (is_row(s)) {
           x.x = __fmul_rn(a.alpha, x.x);
           x.y = __fmul_rn(a.alpha, x.y);
@@ -261,17 +286,17 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 #pragma unroll
   for (int r = 0; r < TM; ++r) {
     const int64_t gi = i0 + tile_off(ty, r);
-    if (gi >= n) continue;
+    if (gi >= ni) continue;
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
       const int64_t gj = j0 + 64 * h + tx * 4;
-      if (a.cvec && gj + 3 < n) {
-        *reinterpret_cast<float4*>(a.C + gi * n + gj) =
+      if (a.cvec && gj + 3 < nj) {
+        *reinterpret_cast<float4*>(a.C + gi * nj + gj) =
             make_float4(c[r][4 * h], c[r][4 * h + 1], c[r][4 * h + 2], c[r][4 * h + 3]);
       } else {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          if (gj + q < n) a.C[gi * n + gj + q] = c[r][4 * h + q];
+          if (gj + q < nj) a.C[gi * nj + gj + q] = c[r][4 * h + q];
       }
     }
   }
@@ -290,36 +315,74 @@ static int tiled_minb(bool two) {
   (void)two;
 }
 
-template <bool TWO>
+template <int MODE>
 static const void* tiled_func() {
-  return tiled_minb(TWO) == 2 ? (const void*)tiled_kernel<TWO, 2> : (const void*)tiled_kernel<TWO, 1>;
+  return tiled_minb(MODE == MODE_SYR2K) == 2 ? (const void*)tiled_kernel<MODE, 2> : (const void*)tiled_kernel<MODE, 1>;
 }
 
-template <bool TWO>
+template <int MODE>
 static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t s) {
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
   size_t dyn = 0;
-  catt_status st = prepare_launch(tiled_func<TWO>(), t, 256, 0, false, &a.t, &dyn);
+  catt_status st = prepare_launch(tiled_func<MODE>(), t, 256, 0, false, &a.t, &dyn);
   if (st != CATT_OK) return st;
-  const int64_t tiles = (a.n + BM - 1) / BM;
-  if (tiles > 65535) return CATT_EINVAL;
+  const int64_t ty = (a.ni + BM - 1) / BM, tx = (a.nj + BM - 1) / BM;
+  if (ty > 65535 || tx > (int64_t(1) << 31) - 1) return CATT_EINVAL;
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
-  a.vec = (a.m % 4 == 0) && al(a.A) && (!TWO || al(a.B));
-  a.cvec = (a.n % 4 == 0) && al(a.C);
-  const dim3 grid{unsigned(tiles), unsigned(tiles), 1u};
-  if (tiled_minb(TWO) == 2)
-    tiled_kernel<TWO, 2><<<grid, 256, dyn, s>>>(a);
+  a.vec = (a.m % 4 == 0) && al(a.A) && (MODE != MODE_SYR2K || al(a.B));
+  a.bvec = MODE == MODE_GEMM && (a.nj % 4 == 0) && al(a.B);
+  a.cvec = (a.nj % 4 == 0) && al(a.C);
+  const dim3 grid{unsigned(tx), unsigned(ty), 1u};
+  if (tiled_minb(MODE == MODE_SYR2K) == 2)
+    tiled_kernel<MODE, 2><<<grid, 256, dyn, s>>>(a);
   else
-    tiled_kernel<TWO, 1><<<grid, 256, dyn, s>>>(a);
+    tiled_kernel<MODE, 1><<<grid, 256, dyn, s>>>(a);
   return after_launch();
 }
 
 const void* syrk_func(int variant) {
-  return variant == CATT_VAR_STAGED ? tiled_func<false>() : (const void*)syrk_thread_kernel;
+  return variant == CATT_VAR_STAGED ? tiled_func<MODE_SYRK>() : (const void*)syrk_thread_kernel;
 }
 
 const void* syr2k_func(int variant) {
-  return variant == CATT_VAR_STAGED ? tiled_func<true>() : (const void*)syr2k_thread_kernel;
+  return variant == CATT_VAR_STAGED ? tiled_func<MODE_SYR2K>() : (const void*)syr2k_thread_kernel;
+}
+
+// ---------------------------------------------------------------- GEMM
+// PolyBench/GPU gemm (Table 2 CI group; the cache-insensitive negative
+// control): thread (i = by*BY + ty, j = bx*32 + tx),
+//   c = C[i][j] * beta; for k: c = fmaf(alpha * a[i][k], b[k][j], c)
+// a[i][k] is a broadcast in the warp, b[k][j] coalesced: nothing to throttle.
+struct GemmArgs {
+  const float* A;
+  const float* B;
+  float* C;
+  int64_t ni, nj, nk;
+  float alpha, beta;
+  Throttle t;
+};
+
+__global__ void __launch_bounds__(1024, 2) gemm_thread_kernel(GemmArgs a) {
+  __shared__ int slots;
+  gate_init(&slots, a.t);
+  __syncthreads();
+  cta_enter(a.t);
+  const int64_t j = int64_t(blockIdx.x) * 32 + threadIdx.x;
+  const int64_t i = int64_t(blockIdx.y) * blockDim.y + threadIdx.y;
+  throttled(a.t, &slots, [&]() {
+    if (i >= a.ni || j >= a.nj) return;
+    const float* __restrict__ ai = a.A + i * a.nk;
+    const float* __restrict__ bj = a.B + j;
+    float c = __fmul_rn(a.C[i * a.nj + j], a.beta);
+#pragma unroll 2
+    for (int64_t k = 0; k < a.nk; ++k) c = fmaf(__fmul_rn(a.alpha, ai[k]), bj[k * a.nj], c);
+    a.C[i * a.nj + j] = c;
+  });
+  cta_exit(a.t);
+}
+
+const void* gemm_func(int variant) {
+  return variant == CATT_VAR_STAGED ? tiled_func<MODE_GEMM>() : (const void*)gemm_thread_kernel;
 }
 
 }  // namespace catt
@@ -346,7 +409,7 @@ extern "C" catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m,
     syrk_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) return launch_tiled<false>(TileArgs{A, nullptr, C, n, m, alpha, beta, 0, 0, {}}, t, s);
+  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_SYRK>(TileArgs{A, nullptr, C, n, n, m, alpha, beta, 0, 0, 0, {}}, t, s);
   return CATT_EINVAL;
 }
 
@@ -370,6 +433,31 @@ extern "C" catt_status catt_syr2k(const float* A, const float* B, float* C, int6
     syr2k_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) return launch_tiled<true>(TileArgs{A, B, C, n, m, alpha, beta, 0, 0, {}}, t, s);
+  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_SYR2K>(TileArgs{A, B, C, n, n, m, alpha, beta, 0, 0, 0, {}}, t, s);
+  return CATT_EINVAL;
+}
+
+extern "C" catt_status catt_gemm(const float* A, const float* B, float* C, int64_t ni, int64_t nj, int64_t nk,
+                                 float alpha, float beta, const catt_throttle* t, void* stream) {
+  if (ni < 0 || nj < 0 || nk < 0 || ni > (int64_t(1) << 31) || nj > (int64_t(1) << 31) || nk > (int64_t(1) << 31))
+    return CATT_EINVAL;
+  if (ni > 0 && nj > 0 && (!C || (nk > 0 && (!A || !B)))) return CATT_EINVAL;
+  if (ni == 0 || nj == 0) return CATT_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int var = variant_of(t);
+  if (var == CATT_VAR_LITERAL) {
+    GemmArgs a{A, B, C, ni, nj, nk, alpha, beta, Throttle{}};
+    const int threads = cta_threads_or(t, 256);
+    if (threads % 32) return CATT_EINVAL;
+    const int by = threads / 32;
+    size_t dyn = 0;
+    catt_status st = prepare_launch((const void*)gemm_thread_kernel, t, threads, 0, true, &a.t, &dyn);
+    if (st != CATT_OK) return st;
+    dim3 grid(unsigned((nj + 31) / 32), unsigned((ni + by - 1) / by));
+    if (grid.y > 65535) return CATT_EINVAL;
+    gemm_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
+    return after_launch();
+  }
+  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_GEMM>(TileArgs{A, B, C, ni, nj, nk, alpha, beta, 0, 0, 0, {}}, t, s);
   return CATT_EINVAL;
 }

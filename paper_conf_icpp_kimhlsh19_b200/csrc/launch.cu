@@ -19,6 +19,8 @@ const void* syrk_func(int variant);
 const void* syr2k_func(int variant);
 const void* kmeans_func(int variant, int nf);
 const void* kmeans_t_func(int variant);
+const void* corr_func(int variant);
+const void* gemm_func(int variant);
 const void* fused_func(bool dep);
 
 namespace {
@@ -216,7 +218,8 @@ catt_ref mkref(int64_t cx, int64_t cy, int64_t c0, int64_t c1, int32_t e, int32_
 }
 
 int default_threads(int loop, int variant) {
-  if (variant == CATT_VAR_STAGED) return (loop == CATT_K_SYRK || loop == CATT_K_SYR2K) ? 256 : 32;
+  if (variant == CATT_VAR_STAGED)
+    return (loop == CATT_K_SYRK || loop == CATT_K_SYR2K || loop == CATT_K_GEMM || loop == CATT_K_CORR) ? 256 : 32;
   if (variant == CATT_VAR_COOP && (loop == CATT_K_ATAX_2 || loop == CATT_K_BICG_1 || loop == CATT_K_MVT_2)) return 1024;
   return 256;
 }
@@ -232,6 +235,8 @@ const void* loop_func(const catt_problem& p, int variant) {
   if (p.loop == CATT_K_SYRK) return syrk_func(variant);
   if (p.loop == CATT_K_SYR2K) return syr2k_func(variant);
   if (p.loop == CATT_K_KMEANS_T) return kmeans_t_func(variant);
+  if (p.loop == CATT_K_CORR) return corr_func(variant);
+  if (p.loop == CATT_K_GEMM) return gemm_func(variant);
   return kmeans_func(variant, int(p.n));
 }
 
@@ -407,6 +412,50 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
     } else {
       return CATT_EINVAL;
     }
+  } else if (loop == CATT_K_CORR) {
+    const int64_t Mc = prob->n, Nr = prob->k;  // Mc columns (threads), Nr rows (inner trip)
+    if (Mc < 1 || Nr < 1) return CATT_EINVAL;
+    if (var == CATT_VAR_STAGED) {                                  // the tiled SYRK of the transposed columns
+      out->n_loops = 1;
+      out->trip[0] = Nr;
+      out->block[0] = 256;
+      out->grid[0] = (Mc + 127) / 128;
+      out->grid[1] = (Mc + 127) / 128;
+      refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);
+      goto done_refs;
+    }
+    if (var != CATT_VAR_LITERAL) return CATT_EINVAL;
+    out->grid[0] = (Mc + threads - 1) / threads;
+    out->extent[0] = Mc;
+    out->n_loops = 2;
+    out->trip[0] = Mc;                                             // j2 (up to m - j1 - 1 iterations)
+    out->trip[1] = Nr;                                             // i
+    refs[n++] = mkref(1, 0, 0, Mc, 4, 1, 0);                     // data[i*m + j1]: reused only across j2
+    refs[n++] = mkref(0, 0, 1, Mc, 4, 1, 0);                     // data[i*m + j2]: broadcast
+    refs[n++] = mkref(Mc, 0, 1, 0, 4, 2, CATT_REF_STORE);        // symmat[j1*m + j2]
+  } else if (loop == CATT_K_GEMM) {
+    const int64_t Ni = prob->m, Nj = prob->n, Nk = prob->k;
+    if (Ni < 1 || Nj < 1 || Nk < 1) return CATT_EINVAL;
+    out->n_loops = 1;
+    out->trip[0] = Nk;
+    if (var == CATT_VAR_LITERAL) {
+      const int by = threads / 32;
+      out->block[0] = 32;
+      out->block[1] = by;
+      out->grid[0] = (Nj + 31) / 32;
+      out->grid[1] = (Ni + by - 1) / by;
+      out->extent[0] = Nj;
+      out->extent[1] = Ni;
+      refs[n++] = mkref(0, Nk, 1, 0, 4, 1, 0);                   // a[i*nk + k]: broadcast in the warp
+      refs[n++] = mkref(1, 0, Nj, 0, 4, 2, 0);                   // b[k*nj + j]: coalesced
+    } else if (var == CATT_VAR_STAGED) {
+      out->block[0] = 256;
+      out->grid[0] = (Nj + 127) / 128;
+      out->grid[1] = (Ni + 127) / 128;
+      refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);
+    } else {
+      return CATT_EINVAL;
+    }
   } else if (loop == CATT_K_KMEANS_T) {
     const int64_t np = prob->m, nf = prob->n, ld = prob->ld;
     if (np < 1 || nf < 1 || ld < np) return CATT_EINVAL;
@@ -446,6 +495,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       return CATT_EINVAL;
     }
   }
+done_refs:
   out->n_refs = n;
   int32_t regs = 0, ssm = 16;  // without a device: the 4-byte gate slot, 16-byte aligned
   int32_t r2 = 0, s2 = 0;

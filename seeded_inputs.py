@@ -66,6 +66,7 @@ def matrix(seed: int, rows: int, cols: int, mode: int = MODE_UNIFORM, row0: int 
 
 # Seeds per workload; each array of a workload gets seed + 100*k.
 SEED_ATAX, SEED_BICG, SEED_MVT, SEED_KMEANS, SEED_GESUMMV, SEED_SYRK, SEED_ATAX_SHARDED, SEED_SYR2K = 1, 2, 3, 4, 5, 6, 7, 8
+SEED_CORR, SEED_GEMM = 9, 10
 
 
 def sub_seed(seed: int, k: int) -> int:

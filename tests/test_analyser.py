@@ -172,6 +172,7 @@ KERNEL_CASES = [
      lru.KmeansKernel(2040, 6, 3, 2044, 128)),
     ("syrk", catt.problem(catt.K_SYRK, n=128, k=64), catt.Throttle(), lru.SyrkKernel(128, 64)),
     ("syr2k", catt.problem(catt.K_SYR2K, n=128, k=64), catt.Throttle(), lru.Syr2kKernel(128, 64)),
+    ("gemm", catt.problem(catt.K_GEMM, m=96, n=64, k=48), catt.Throttle(), lru.GemmKernel(96, 64, 48)),
 ]
 
 
@@ -232,3 +233,25 @@ def test_guards_do_not_touch_paper_mode():
                                  force_carveout_kb=96)
         r = catt.footprint(d, hw)
         assert (r["active_warps"], r["active_ctas"]) == tuple(c["catt_32kb"])
+
+
+def test_corr_gives_up_and_gemm_keeps_full_tlp():
+    """CORR's footprint does not fit at any TLP (the reused line of
+    data[i*m + j1] returns only after n rows), so CATT keeps the baseline;
+    Table 3 P:353 lists CORR #2 at (8,1) everywhere. P:397: the CI control
+    (GEMM) keeps baseline TLP."""
+    corr = catt.problem(catt.K_CORR, n=2048, k=2048)
+    gemm = catt.problem(catt.K_GEMM, m=512, n=512, k=512)
+    b200 = catt.hw_b200()
+    for hw, carves in ((catt.paper_rule(b200), (8, 100, 228)), (catt.hw_titanv(), (32, 96))):
+        for carve in carves:
+            t, r = catt.plan(corr, catt.Throttle(carveout_kb=carve), hw)
+            assert r["flags"] == catt.FIT_UNRESOLVABLE
+            assert (r["base_warps"], r["base_ctas"]) == (8, 1) and t.active_warps == 0 and t.active_ctas == 0
+            t, r = catt.plan(gemm, catt.Throttle(carveout_kb=carve), hw)
+            assert r["flags"] == catt.FIT_NONE_NEEDED and t.active_warps == 0 and t.active_ctas == 0
+    for carve in (8, 100, 228):   # B200 rule: the reused reference is coalesced -> guard, no throttle
+        t, r = catt.plan(corr, catt.Throttle(carveout_kb=carve), b200)
+        assert r["flags"] == catt.FIT_NONE_NEEDED | catt.FIT_GUARDED and t.active_warps == 0
+        t, r = catt.plan(gemm, catt.Throttle(carveout_kb=carve, cta_threads=1024), b200)
+        assert r["flags"] == catt.FIT_NONE_NEEDED

@@ -255,6 +255,57 @@ def test_syr2k_2048_sampled_rows():
         assert bits_equal(host(Cd)[rows], want), v
 
 
+# ------------------------------------------------------------------ GEMM (CI control)
+@pytest.mark.parametrize("variant", ["literal", "staged"])
+@pytest.mark.parametrize("ni,nj,nk", [(64, 64, 64), (130, 70, 37), (257, 129, 8), (1, 3, 2), (512, 512, 512),
+                                      (100, 130, 1)])
+def test_gemm_exact(variant, ni, nj, nk):
+    A, B, C = si.matrix(21, ni, nk), si.matrix(22, nk, nj), si.matrix(23, ni, nj)
+    C_o = oracle.gemm(A, B, C, 1.5, 1.2)
+    Cd = dev(C)
+    catt.gemm(dev(A), dev(B), Cd, 1.5, 1.2, t=catt.Throttle(variant=variant))
+    assert bits_equal(host(Cd), C_o)
+
+
+def test_gemm_throttled_and_empty():
+    A, B, C = si.matrix(21, 96, 40), si.matrix(22, 40, 70), si.matrix(23, 96, 70)
+    C_o = oracle.gemm(A, B, C, 1.5, 1.2)
+    for t in (catt.Throttle(active_warps=2), catt.Throttle(active_warps=4, active_ctas=1),
+              catt.Throttle(cta_threads=512, active_warps=4, gate=catt.GATE_BARRIER)):
+        Cd = dev(C)
+        catt.gemm(dev(A), dev(B), Cd, 1.5, 1.2, t=t)
+        assert bits_equal(host(Cd), C_o)
+    Cd = dev(C)
+    z1, z2 = torch.empty(96, 0, device="cuda"), torch.empty(0, 70, device="cuda")
+    catt.gemm(z1, z2, Cd, 1.5, 1.25)
+    assert bits_equal(host(Cd), (C * np.float32(1.25)).astype(np.float32))
+
+
+# ------------------------------------------------------------------ CORR (give-up case)
+@pytest.mark.parametrize("variant", ["literal", "staged"])
+@pytest.mark.parametrize("n,m", [(300, 70), (128, 257), (33, 5), (1000, 129)])
+def test_corr_exact(variant, n, m):
+    data = si.matrix(24, n, m)
+    data[:, 2] = 0.5                                  # a constant column: the eps branch
+    sym_o, mean_o, std_o, d_o = oracle.corr(data)
+    D = dev(data)
+    sym, mean, std = catt.corr(D, t=catt.Throttle(variant=variant))
+    assert bits_equal(host(D), d_o) and bits_equal(host(mean), mean_o) and bits_equal(host(std), std_o)
+    assert bits_equal(host(sym), sym_o)
+
+
+def test_corr_2048_full_size():
+    """Table 2 P:81 size (2K x 2K), both variants, and a throttled literal run."""
+    n = m = 2048
+    data = oracle.fill(si.SEED_CORR, n * m).reshape(n, m)
+    sym_o, mean_o, std_o, _ = oracle.corr(data)
+    for t in (catt.Throttle(variant="staged"), catt.Throttle(), catt.Throttle(active_warps=4)):
+        D = torch.empty(n * m, device="cuda")
+        catt.fill_hash(D, si.SEED_CORR)
+        sym, mean, std = catt.corr(D.view(n, m), t=t)
+        assert bits_equal(host(sym), sym_o) and bits_equal(host(mean), mean_o), t
+
+
 # ------------------------------------------------------------------ KMEANS
 @pytest.mark.parametrize("variant", ["literal", "regs", "staged"])
 @pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 4), (4099, 34, 5, 29), (257, 7, 3, 3), (300, 50, 12, 4),
