@@ -789,6 +789,8 @@ def run_reference(args):
     import numpy as np
     import oracle
     import seeded_inputs as si
+    if world > 1:            # torchrun exports OMP_NUM_THREADS=1; rank 0 alone runs, on every host core
+        oracle.set_num_threads(os.cpu_count() or 1)
     wl = args.workload
     t0 = time.perf_counter()
     if wl == "bicg_mvt":
@@ -848,10 +850,18 @@ def main():
     import torch
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    # CATT_BENCH_SHARE_GPU=1 (tests only): every rank on cuda:0 over gloo, so
+    # the N > 1 path can be exercised on a one-GPU box; never a bench number
+    share = os.environ.get("CATT_BENCH_SHARE_GPU") == "1"
+    if share:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         barrier = lambda: dist.barrier()
     else:
         barrier = lambda: None

@@ -65,6 +65,8 @@ def lib():
         L.orc_atax_hashed.argtypes = [ctypes.c_int, u32, ctypes.c_int, f32p, i64, i64, f32p,
                                       ctypes.POINTER(ctypes.c_int64), i64, f32p]
         L.orc_num_threads.restype = ctypes.c_int
+        L.orc_set_num_threads.argtypes = [ctypes.c_int]
+        L.orc_set_num_threads.restype = None
         _lib = L
     return _lib
 
@@ -86,6 +88,11 @@ def _f32(a):
 
 def num_threads() -> int:
     return int(lib().orc_num_threads())
+
+
+def set_num_threads(n: int):
+    """OpenMP threads for the loop nests (torchrun exports OMP_NUM_THREADS=1)."""
+    lib().orc_set_num_threads(int(n))
 
 
 def fill(seed: int, n: int, offset: int = 0, mode: int = 0) -> np.ndarray:

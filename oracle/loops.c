@@ -449,6 +449,15 @@ int orc_atax_hashed(int mode, uint32_t seedA, int amode, const float* x, int64_t
   return 0;
 }
 
+void orc_set_num_threads(int n) {
+#ifdef _OPENMP
+  extern void omp_set_num_threads(int);
+  if (n > 0) omp_set_num_threads(n);
+#else
+  (void)n;
+#endif
+}
+
 int orc_num_threads(void) {
 #ifdef _OPENMP
   extern int omp_get_max_threads(void);
