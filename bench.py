@@ -702,6 +702,11 @@ def throttle_study(catt, torch, w, flush):
         pick = (t.active_warps or W, t.active_ctas or T)
         pick_p = (tp.active_warps or W, tp.active_ctas or T)
         best = min(times, key=times.get)
+        # the bypass alternative: the same literal row loop with L2-only
+        # matrix loads at full TLP (row-loop studies only)
+        byp = None
+        if not S.get("fn") and not S.get("kmeans"):
+            byp = med(study_fn(catt, w, launch.copy(variant=catt.VAR_BYPASS)), S.get("reps", 5))
         out.append(dict(loop=S["name"], cta_threads=cta, carveout_kb=r["carveout_kb"], base=[W, T],
                         footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
                         contended=rp["flags"] != catt.FIT_NONE_NEEDED,
@@ -712,6 +717,8 @@ def throttle_study(catt, torch, w, flush):
                         catt_over_best=round(times[pick] / times[best], 3),
                         catt_over_full=round(times[pick] / times[(W, T)], 3),
                         paper_over_best=round(times[pick_p] / times[best], 3),
+                        bypass_ms=round(byp, 4) if byp is not None else None,
+                        bypass_over_best=round(byp / times[best], 3) if byp is not None else None,
                         swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()}))
     return out
 

@@ -155,12 +155,15 @@ typedef struct {
  *            the HBM-roofline variant; summation order differs (fp64-oracle
  *            tolerance, bit-exact on exact-dyadic inputs).
  *   REGS     (KMEANS) the point's features are loaded once into registers.
+ *   BYPASS   (row loops) the literal loop with L2-only (ld.global.cg) matrix
+ *            loads: the divergent rows never occupy L1, nothing to throttle
+ *            (the bypass alternative of P:137).
  *   FUSED    (ATAX/BICG/MVT, set on k1) both loops in one pass over A: each
  *            row is read once, its dot product finished in the CTA, its A^T
  *            contribution accumulated; A^T partials reduced in band order
  *            after a grid barrier (cooperative launch). Same bar as COOP.  */
 enum { CATT_VAR_LITERAL = 0, CATT_VAR_VEC4 = 1, CATT_VAR_STAGED = 2, CATT_VAR_COOP = 3, CATT_VAR_REGS = 4,
-       CATT_VAR_FUSED = 5 };
+       CATT_VAR_FUSED = 5, CATT_VAR_BYPASS = 6 };
 
 /* Warp-level mechanism: SEMAPHORE = per-CTA counting semaphore in shared
  * memory (a finished warp's slot goes to the next waiting warp);

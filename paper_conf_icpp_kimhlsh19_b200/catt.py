@@ -23,7 +23,7 @@ MAX_LOOPS, MAX_CARVEOUTS = 4, 16
 REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
 MODE_UNION, MODE_PAPER = 0, 1
 FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE, FIT_GUARDED = 1, 2, 4, 8, 16
-VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED = 0, 1, 2, 3, 4, 5
+VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED, VAR_BYPASS = 0, 1, 2, 3, 4, 5, 6
 ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
@@ -31,7 +31,7 @@ CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
  K_KMEANS_T, K_CORR, K_GEMM) = range(13)
 
 VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS,
-            "fused": VAR_FUSED}
+            "fused": VAR_FUSED, "bypass": VAR_BYPASS}
 FLAG_NAMES = {FIT_NONE_NEEDED: "none", FIT_WARP: "warp", FIT_CTA: "cta", FIT_UNRESOLVABLE: "unresolvable",
               FIT_NONE_NEEDED | FIT_GUARDED: "none(guard)", FIT_WARP | FIT_GUARDED: "warp(guard)",
               FIT_CTA | FIT_GUARDED: "cta(guard)"}

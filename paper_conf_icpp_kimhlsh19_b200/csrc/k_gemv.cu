@@ -69,8 +69,13 @@ __device__ __forceinline__ void row_epilogue(const RowArgs& a, int64_t i, float 
 }
 
 // ---------------------------------------------------------------- row, thread per row
-template <int NMAT, int EPI, bool VEC>
-__global__ void __launch_bounds__(1024, (NMAT == 2 && VEC) ? 1 : 2) row_thread_kernel(RowArgs a) {
+// VM: 0 = the literal scalar loop (loads through L1), 1 = VEC4 (16-byte loads),
+// 2 = BYPASS (the literal loop with ld.global.cg matrix loads: cached in L2
+// only, so the divergent rows never occupy L1; the alternative to throttling
+// that the paper discusses as related work)
+template <int NMAT, int EPI, int VM>
+__global__ void __launch_bounds__(1024, (NMAT == 2 && VM == 1) ? 1 : 2) row_thread_kernel(RowArgs a) {
+  constexpr bool VEC = VM == 1, BYPASS = VM == 2;
   __shared__ int slots;
   gate_init(&slots, a.t);
   __syncthreads();
@@ -88,8 +93,8 @@ __global__ void __launch_bounds__(1024, (NMAT == 2 && VEC) ? 1 : 2) row_thread_k
 #pragma unroll 2
       for (int64_t j = 0; j < N; ++j) {
         const float xv = x[j];
-        acc = fmaf(ar[j], xv, acc);
-        if (NMAT == 2) acc2 = fmaf(br[j], xv, acc2);
+        acc = fmaf(BYPASS ? __ldcg(ar + j) : ar[j], xv, acc);
+        if (NMAT == 2) acc2 = fmaf(BYPASS ? __ldcg(br + j) : br[j], xv, acc2);
       }
     } else {
       const float4* __restrict__ a4 = reinterpret_cast<const float4*>(ar);
@@ -421,19 +426,22 @@ catt_status launch_row_t(RowArgs a, const catt_throttle* t, cudaStream_t s) {
   const int var = variant_of(t);
   if (a.M == 0) return CATT_OK;
   const bool vec_ok = (a.N % 4 == 0) && aligned16(a.A) && aligned16(a.x) && (NMAT == 1 || aligned16(a.B));
-  if (var == CATT_VAR_LITERAL || var == CATT_VAR_VEC4) {
+  if (var == CATT_VAR_LITERAL || var == CATT_VAR_VEC4 || var == CATT_VAR_BYPASS) {
     const int threads = cta_threads_or(t, 256);
     if (var == CATT_VAR_VEC4 && !vec_ok) return CATT_EINVAL;
-    const void* f = (var == CATT_VAR_VEC4) ? (const void*)row_thread_kernel<NMAT, EPI, true>
-                                           : (const void*)row_thread_kernel<NMAT, EPI, false>;
+    const void* f = var == CATT_VAR_VEC4     ? (const void*)row_thread_kernel<NMAT, EPI, 1>
+                    : var == CATT_VAR_BYPASS ? (const void*)row_thread_kernel<NMAT, EPI, 2>
+                                             : (const void*)row_thread_kernel<NMAT, EPI, 0>;
     size_t dyn = 0;
     catt_status st = prepare_launch(f, t, threads, 0, true, &a.t, &dyn);
     if (st != CATT_OK) return st;
     const int64_t grid = (a.M + threads - 1) / threads;
     if (var == CATT_VAR_VEC4)
-      row_thread_kernel<NMAT, EPI, true><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
+      row_thread_kernel<NMAT, EPI, 1><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
+    else if (var == CATT_VAR_BYPASS)
+      row_thread_kernel<NMAT, EPI, 2><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
     else
-      row_thread_kernel<NMAT, EPI, false><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
+      row_thread_kernel<NMAT, EPI, 0><<<dim3(unsigned(grid)), threads, dyn, s>>>(a);
     return after_launch();
   }
   if (var == CATT_VAR_COOP) {
@@ -540,22 +548,26 @@ const void* gemv_func(int loop, int variant, bool vec_ok) {
   if (row) {
     const int nmat = loop == CATT_K_GESUMMV ? 2 : 1;
     if (variant == CATT_VAR_STAGED) return row_tma_func(nmat);
+    const int vm = variant == CATT_VAR_VEC4 ? 1 : variant == CATT_VAR_BYPASS ? 2 : 0;
     if (loop == CATT_K_GESUMMV) {
-      if (variant == CATT_VAR_VEC4) return (const void*)row_thread_kernel<2, EPI_GESUMMV, true>;
       if (variant == CATT_VAR_COOP)
         return vec_ok ? row_warp_func<2, EPI_GESUMMV, true>(1) : row_warp_func<2, EPI_GESUMMV, false>(1);
-      return (const void*)row_thread_kernel<2, EPI_GESUMMV, false>;
+      return vm == 1 ? (const void*)row_thread_kernel<2, EPI_GESUMMV, 1>
+                     : vm == 2 ? (const void*)row_thread_kernel<2, EPI_GESUMMV, 2>
+                               : (const void*)row_thread_kernel<2, EPI_GESUMMV, 0>;
     }
     if (loop == CATT_K_MVT_1) {
-      if (variant == CATT_VAR_VEC4) return (const void*)row_thread_kernel<1, EPI_ACCUM, true>;
       if (variant == CATT_VAR_COOP)
         return vec_ok ? row_warp_func<1, EPI_ACCUM, true>(1) : row_warp_func<1, EPI_ACCUM, false>(1);
-      return (const void*)row_thread_kernel<1, EPI_ACCUM, false>;
+      return vm == 1 ? (const void*)row_thread_kernel<1, EPI_ACCUM, 1>
+                     : vm == 2 ? (const void*)row_thread_kernel<1, EPI_ACCUM, 2>
+                               : (const void*)row_thread_kernel<1, EPI_ACCUM, 0>;
     }
-    if (variant == CATT_VAR_VEC4) return (const void*)row_thread_kernel<1, EPI_STORE, true>;
     if (variant == CATT_VAR_COOP)
       return vec_ok ? row_warp_func<1, EPI_STORE, true>(1) : row_warp_func<1, EPI_STORE, false>(1);
-    return (const void*)row_thread_kernel<1, EPI_STORE, false>;
+    return vm == 1 ? (const void*)row_thread_kernel<1, EPI_STORE, 1>
+                   : vm == 2 ? (const void*)row_thread_kernel<1, EPI_STORE, 2>
+                             : (const void*)row_thread_kernel<1, EPI_STORE, 0>;
   }
   const bool acc = loop == CATT_K_MVT_2;
   if (variant == CATT_VAR_STAGED) return col_tma_func();

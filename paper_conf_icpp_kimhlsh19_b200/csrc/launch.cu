@@ -286,10 +286,11 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
     const bool two = loop == CATT_K_GESUMMV;
     out->n_loops = 1;
     out->extent[0] = M;
-    if (var == CATT_VAR_LITERAL) {
-      refs[n++] = mkref(N, 0, 1, 0, 4, 1, 0);                     // A[i*N + j]
+    if (var == CATT_VAR_LITERAL || var == CATT_VAR_BYPASS) {
+      const int32_t fa = var == CATT_VAR_BYPASS ? CATT_REF_NOT_L1 : 0;  // BYPASS: the rows skip L1
+      refs[n++] = mkref(N, 0, 1, 0, 4, 1, fa);                    // A[i*N + j]
       refs[n++] = mkref(0, 0, 1, 0, 4, 2, 0);                     // x[j]
-      if (two) refs[n++] = mkref(N, 0, 1, 0, 4, 3, 0);            // B[i*N + j]
+      if (two) refs[n++] = mkref(N, 0, 1, 0, 4, 3, fa);           // B[i*N + j]
       out->trip[0] = N;
       out->grid[0] = (M + threads - 1) / threads;
     } else if (var == CATT_VAR_VEC4) {

@@ -255,6 +255,25 @@ def test_syr2k_2048_sampled_rows():
         assert bits_equal(host(Cd)[rows], want), v
 
 
+def test_bypass_rows_equal_literal():
+    """BYPASS is the literal loop with L2-only loads: bit-identical results."""
+    m, n = 777, 301
+    A, B = si.matrix(2, m, n), si.matrix(3, m, n)
+    x, y0 = si.values(4, n), si.values(5, m)
+    for mode in (catt.ROWS_STORE, catt.ROWS_ACCUM, catt.ROWS_GESUMMV):
+        outs = []
+        for v in ("literal", "bypass"):
+            y, tmp = dev(y0), torch.empty(m, device="cuda")
+            catt.rows(dev(A), dev(x), y, mode, B=dev(B), tmp=tmp, alpha=1.5, beta=1.2, t=catt.Throttle(variant=v))
+            outs.append((host(y), host(tmp)))
+        assert bits_equal(outs[0][0], outs[1][0])
+        if mode == catt.ROWS_GESUMMV:
+            assert bits_equal(outs[0][1], outs[1][1])
+    t, r = catt.plan(catt.problem(catt.K_BICG_2, m=4096, n=4096), catt.Throttle(variant="bypass", carveout_kb=228),
+                     catt.paper_rule(catt.hw_query()))
+    assert r["flags"] == catt.FIT_NONE_NEEDED            # nothing of the divergent rows in L1
+
+
 # ------------------------------------------------------------------ GEMM (CI control)
 @pytest.mark.parametrize("variant", ["literal", "staged"])
 @pytest.mark.parametrize("ni,nj,nk", [(64, 64, 64), (130, 70, 37), (257, 129, 8), (1, 3, 2), (512, 512, 512),

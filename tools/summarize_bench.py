@@ -23,7 +23,7 @@ for f in sorted(glob.glob(os.path.join(sys.argv[1], "bench_*.json"))):
     for s in d.get("throttle_study") or []:
         print(f"      study {s['loop'][:40]:40s} cta {s['cta_threads']:4d} carve {s['carveout_kb']:3d}  B200 {s['catt']} "
               f"{s['catt_over_best']}x best  paper {s['catt_paper']} {s['paper_over_best']}x  full/best "
-              f"{round(s['full_ms'] / s['best_ms'], 3)}  best {s['best']}")
+              f"{round(s['full_ms'] / s['best_ms'], 3)}  best {s['best']}  bypass/best {s.get('bypass_over_best')}")
     for s in d.get("bftt_vs_catt") or []:
         print(f"      bftt  carve {s['carveout_kb']} catt {s['catt_ms']} ms  bftt {s['bftt_ms']} ms  "
               f"speedup {s['catt_speedup_over_bftt']}")
