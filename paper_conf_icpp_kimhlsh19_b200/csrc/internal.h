@@ -39,4 +39,7 @@ inline int cta_threads_or(const catt_throttle* t, int def) {
 }
 inline int variant_of(const catt_throttle* t) { return t ? t->variant : CATT_VAR_LITERAL; }
 
+// Tiled SYRK over the tiles on and above the diagonal only (k_syrk.cu).
+catt_status syrk_upper(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta, cudaStream_t s);
+
 }  // namespace catt

@@ -12,9 +12,11 @@
 // j2 the thread re-reads its whole column j1 (n rows apart), so the line it
 // reuses comes back only after n lines of its own: no throttle makes that fit
 // (the paper's "give up"), and the analyser reports CATT_FIT_UNRESOLVABLE.
-// STAGED: the same statistics kernel, then the columns transposed (32 x 32
-// tiles) and symmat = D^T D by the tiled SYRK kernel with alpha = 1, beta = 0:
-// each element is the same fmaf chain over i (fmaf is commutative),
+// STAGED: the columns transposed (32 x 32 tiles), the statistics a warp per
+// column (the same sequential order, lane 0), the centred data transposed
+// back, and symmat = D^T D by the tiled SYRK kernel with alpha = 1, beta = 0
+// over the upper tiles, mirrored into the lower triangle: each element is the
+// same fmaf chain over i (fmaf is commutative),
 // so the result is bit-identical to LITERAL; the diagonal is then set to 1.
 #include <cmath>
 #include <cstdint>
@@ -97,6 +99,59 @@ __global__ void __launch_bounds__(256) transpose32_kernel(const float* __restric
   }
 }
 
+// STAGED statistics on the transposed data (row j = column j, contiguous):
+// a warp per column stages the row in shared memory (coalesced), lane 0 runs
+// the two sequential sums in the same order and rounding as corr_stats_kernel,
+// then the whole warp writes the centred and scaled row back.
+constexpr int kStatWarps = 8;
+__global__ void __launch_bounds__(kStatWarps * 32) corr_stats_rows_kernel(float* rowsT, float* mean, float* stdv,
+                                                                         int64_t n, int64_t m) {
+  extern __shared__ float s_row[];  // [kStatWarps][n]
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t j = int64_t(blockIdx.x) * kStatWarps + w;
+  if (j >= m) return;
+  float* buf = s_row + int64_t(w) * n;
+  float* row = rowsT + j * n;
+  for (int64_t i = lane; i < n; i += 32) buf[i] = row[i];
+  __syncwarp();
+  const float fn = float(n), eps = 0.005f;
+  float mu = 0.0f, sd = 0.0f;
+  if (lane == 0) {
+    for (int64_t i = 0; i < n; ++i) mu = __fadd_rn(mu, buf[i]);
+    mu = __fdiv_rn(mu, fn);
+    for (int64_t i = 0; i < n; ++i) {
+      const float d = __fsub_rn(buf[i], mu);
+      sd = fmaf(d, d, sd);
+    }
+    sd = __fsqrt_rn(__fdiv_rn(sd, fn));
+    if (sd <= eps) sd = 1.0f;
+    mean[j] = mu;
+    stdv[j] = sd;
+  }
+  mu = __shfl_sync(0xffffffffu, mu, 0);
+  sd = __shfl_sync(0xffffffffu, sd, 0);
+  const float scale = __fmul_rn(__fsqrt_rn(fn), sd);
+  for (int64_t i = lane; i < n; i += 32) row[i] = __fdiv_rn(__fsub_rn(buf[i], mu), scale);
+}
+
+// symmat[i][j] = symmat[j][i] for i > j, through 32 x 32 tiles (the lower
+// triangle from the computed upper one)
+__global__ void __launch_bounds__(256) mirror_lower_kernel(float* symmat, int64_t m) {
+  if (blockIdx.x > blockIdx.y) return;  // destination tile (by, bx) must be on or below the diagonal
+  __shared__ float tile[32][33];
+  const int64_t di = int64_t(blockIdx.y) * 32, dj = int64_t(blockIdx.x) * 32;  // destination rows, columns
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  for (int r = ty; r < 32; r += 8) {  // source tile (dj, di): rows dj.., columns di..
+    const int64_t i = dj + r, j = di + tx;
+    if (i < m && j < m) tile[r][tx] = symmat[i * m + j];
+  }
+  __syncthreads();
+  for (int r = ty; r < 32; r += 8) {
+    const int64_t i = di + r, j = dj + tx;
+    if (i < m && j < m && i > j) symmat[i * m + j] = tile[tx][r];
+  }
+}
+
 __global__ void corr_diag_kernel(float* symmat, int64_t m) {
   const int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (j < m) symmat[j * m + j] = 1.0f;
@@ -120,10 +175,10 @@ extern "C" catt_status catt_corr(float* data, int64_t n, int64_t m, float* mean,
   const int var = variant_of(t);
   if (var != CATT_VAR_LITERAL && var != CATT_VAR_STAGED) return CATT_EINVAL;
   if (var == CATT_VAR_STAGED && !work) return CATT_EINVAL;
-  corr_stats_kernel<<<dim3(unsigned((m + 255) / 256)), 256, 0, s>>>(CorrStatsArgs{data, mean, stdv, n, m});
-  catt_status st = after_launch();
-  if (st != CATT_OK) return st;
+  catt_status st = CATT_OK;
   if (var == CATT_VAR_LITERAL) {
+    corr_stats_kernel<<<dim3(unsigned((m + 255) / 256)), 256, 0, s>>>(CorrStatsArgs{data, mean, stdv, n, m});
+    if ((st = after_launch()) != CATT_OK) return st;
     CorrArgs a{data, symmat, n, m, Throttle{}};
     const int threads = cta_threads_or(t, 256);
     size_t dyn = 0;
@@ -132,17 +187,28 @@ extern "C" catt_status catt_corr(float* data, int64_t n, int64_t m, float* mean,
     corr_thread_kernel<<<dim3(unsigned((m + threads - 1) / threads)), threads, dyn, s>>>(a);
     return after_launch();
   }
-  // STAGED: work = data^T (m x n), symmat = work work^T (alpha 1, beta 0), diagonal 1
-  const int64_t gy = (n + 31) / 32;
-  if (gy > 65535) return CATT_EINVAL;
-  transpose32_kernel<<<dim3(unsigned((m + 31) / 32), unsigned(gy)), 256, 0, s>>>(data, work, n, m);
-  st = after_launch();
-  if (st != CATT_OK) return st;
+  // STAGED: work = data^T (m x n); statistics and scaling on its rows; data =
+  // work^T (the centred data, as LITERAL leaves it); symmat = work work^T by
+  // the tiled SYRK (alpha 1, beta 0); diagonal 1
+  const int64_t gy = (n + 31) / 32, gx = (m + 31) / 32;
+  if (gy > 65535 || gx > 65535) return CATT_EINVAL;
+  const size_t srow = size_t(kStatWarps) * size_t(n) * 4;
+  if (srow > 200 * 1024) return CATT_EUNSUPPORTED;  // n > 6400 rows: use LITERAL
+  transpose32_kernel<<<dim3(unsigned(gx), unsigned(gy)), 256, 0, s>>>(data, work, n, m);
+  if ((st = after_launch()) != CATT_OK) return st;
+  if (srow > 48 * 1024 && cudaFuncSetAttribute((const void*)corr_stats_rows_kernel,
+                                               cudaFuncAttributeMaxDynamicSharedMemorySize, int(srow)) != cudaSuccess)
+    return after_launch();
+  corr_stats_rows_kernel<<<dim3(unsigned((m + kStatWarps - 1) / kStatWarps)), kStatWarps * 32, srow, s>>>(
+      work, mean, stdv, n, m);
+  if ((st = after_launch()) != CATT_OK) return st;
+  transpose32_kernel<<<dim3(unsigned(gy), unsigned(gx)), 256, 0, s>>>(work, data, m, n);
+  if ((st = after_launch()) != CATT_OK) return st;
   if (cudaMemsetAsync(symmat, 0, size_t(m) * size_t(m) * 4, s) != cudaSuccess) return after_launch();
-  catt_throttle staged{};
-  staged.variant = CATT_VAR_STAGED;
-  st = catt_syrk(work, symmat, m, n, 1.0f, 0.0f, &staged, stream);
+  st = syrk_upper(work, symmat, m, n, 1.0f, 0.0f, s);  // upper tiles only: symmat is symmetric
   if (st != CATT_OK) return st;
+  mirror_lower_kernel<<<dim3(unsigned(gx), unsigned(gx)), 256, 0, s>>>(symmat, m);
+  if ((st = after_launch()) != CATT_OK) return st;
   corr_diag_kernel<<<dim3(unsigned((m + 255) / 256)), 256, 0, s>>>(symmat, m);
   return after_launch();
 }

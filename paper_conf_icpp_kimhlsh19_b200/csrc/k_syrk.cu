@@ -98,8 +98,9 @@ __global__ void __launch_bounds__(1024, 2) syr2k_thread_kernel(Syr2kArgs a) {
 //   GEMM : 0 = alpha*a[i][k], 1 = b[k][j] (B is k-major: loaded without a transpose)
 // C is ni x nj (SYRK/SYR2K: ni = nj = n), the inner size is m.
 constexpr int MODE_SYRK = 0, MODE_SYR2K = 1, MODE_GEMM = 2;
-constexpr int BM = 128, TM = 8;
-constexpr int PITCH = BM + 4;  // transposed stage rows: 16-B aligned, store banks spread
+// TM x TM outputs per thread, 16 x 16 threads: TM = 8 -> 128 x 128 tiles,
+// TM = 4 -> 64 x 64 tiles (SYRK and GEMM only), for grids that would leave
+// most SMs idle with the large tile.
 
 struct TileArgs {
   const float* A;
@@ -110,25 +111,32 @@ struct TileArgs {
   int vec;  // m % 4 == 0 and A (SYR2K: and B) 16-B aligned: float4 loads along k
   int bvec; // GEMM: nj % 4 == 0 and B 16-B aligned: float4 loads of B rows
   int cvec; // nj % 4 == 0 and C 16-B aligned
+  int tri;  // SYRK only: compute the tiles on and above the diagonal (C symmetric; caller mirrors)
   Throttle t;
 };
 
-template <int MODE>
+template <int MODE, int TM>
 struct TileCfg {
+  static constexpr int BM = 16 * TM;            // tile edge
+  static constexpr int H = TM / 4;              // float4 groups per thread per dimension
+  static constexpr int GS = BM / H;             // group stride: rows {g*GS + 4t + r}
+  static constexpr int PITCH = BM + 4;          // transposed stage rows: 16-B aligned, store banks spread
   static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
-  static constexpr int KQ = BK / 4;            // float4 per stage row
-  static constexpr int NV = BM * KQ / 256;     // float4 per thread per array per stage
+  static constexpr int KQ = BK / 4;             // float4 per stage row
+  static constexpr int NV = BM * KQ / 256;      // float4 per thread per array per stage
+  static_assert(NV >= 1, "tile too small for the stage depth");
 };
 
-__device__ __forceinline__ int tile_off(int t, int r) { return r < 4 ? t * 4 + r : 64 + t * 4 + (r - 4); }
-
-template <int MODE, int MINB>
+template <int MODE, int MINB, int TM = 8>
 __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
   constexpr bool TWO = MODE == MODE_SYR2K, GEMM = MODE == MODE_GEMM;
-  using Cfg = TileCfg<MODE>;
-  constexpr int BK = Cfg::BK, NA = Cfg::NA, KQ = Cfg::KQ, NV = Cfg::NV;
+  using Cfg = TileCfg<MODE, TM>;
+  constexpr int BK = Cfg::BK, NA = Cfg::NA, KQ = Cfg::KQ, NV = Cfg::NV, BM = Cfg::BM, H = Cfg::H, GS = Cfg::GS;
+  constexpr int PITCH = Cfg::PITCH;
+  auto tile_off = [](int t, int r) { return (r / 4) * GS + t * 4 + (r % 4); };
   __shared__ __align__(16) float S[2][NA][BK][PITCH];
+  if (a.tri && blockIdx.x < blockIdx.y) return;  // strictly below the diagonal: mirrored by the caller
   cta_enter(a.t);
   const int tid = threadIdx.x;
   const int tx = tid & 15, ty = tid >> 4;
@@ -140,8 +148,8 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
   for (int r = 0; r < TM; ++r) {
     const int64_t gi = i0 + tile_off(ty, r);
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int64_t gj = j0 + 64 * h + tx * 4;
+    for (int h = 0; h < H; ++h) {
+      const int64_t gj = j0 + GS * h + tx * 4;
       if (a.cvec && gi < ni && gj + 3 < nj) {
         const float4 v = *reinterpret_cast<const float4*>(a.C + gi * nj + gj);
         c[r][4 * h] = __fmul_rn(v.x, a.beta);
@@ -170,7 +178,7 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 #pragma unroll
       for (int s = 0; s < NA; ++s) {
         if (GEMM && s == 1) {  // B rows k0 + kk, columns j0 + 4*c4 .. +3
-          const int kk = idx >> 5, c4 = idx & 31;
+          const int kk = idx / (BM / 4), c4 = idx % (BM / 4);
           const int64_t kb = k0 + kk, jb = j0 + 4 * c4;
           const float* Bp = a.B + kb * nj + jb;
           if (a.bvec && kb < m && jb + 3 < nj) {
@@ -208,7 +216,7 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
       for (int s = 0; s < NA; ++s) {
         float4 x = ld[s][v];
         if (GEMM && s == 1) {
-          *reinterpret_cast<float4*>(&S[buf][1][idx >> 5][4 * (idx & 31)]) = x;
+          *reinterpret_cast<float4*>(&S[buf][1][idx / (BM / 4)][4 * (idx % (BM / 4))]) = x;
           continue;
         }
         if (is_row(s)) {
@@ -230,8 +238,8 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
     for (int s = 0; s < NA; ++s) {
       const int t = is_row(s) ? ty : tx;
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const float4 v = *reinterpret_cast<const float4*>(&S[buf][s][kk][64 * h + t * 4]);
+      for (int h = 0; h < H; ++h) {
+        const float4 v = *reinterpret_cast<const float4*>(&S[buf][s][kk][GS * h + t * 4]);
         f[fb][s][4 * h] = v.x;
         f[fb][s][4 * h + 1] = v.y;
         f[fb][s][4 * h + 2] = v.z;
@@ -288,8 +296,8 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
     const int64_t gi = i0 + tile_off(ty, r);
     if (gi >= ni) continue;
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int64_t gj = j0 + 64 * h + tx * 4;
+    for (int h = 0; h < H; ++h) {
+      const int64_t gj = j0 + GS * h + tx * 4;
       if (a.cvec && gj + 3 < nj) {
         *reinterpret_cast<float4*>(a.C + gi * nj + gj) =
             make_float4(c[r][4 * h], c[r][4 * h + 1], c[r][4 * h + 2], c[r][4 * h + 3]);
@@ -320,20 +328,39 @@ static const void* tiled_func() {
   return tiled_minb(MODE == MODE_SYR2K) == 2 ? (const void*)tiled_kernel<MODE, 2> : (const void*)tiled_kernel<MODE, 1>;
 }
 
+// The 64 x 64 tile (SYRK, GEMM) when 128 x 128 tiles would not give every SM
+// a CTA; it keeps the same per-element order, so results are identical.
+template <int MODE>
+static bool small_tiles(int64_t ni, int64_t nj) {
+  if (MODE == MODE_SYR2K) return false;
+  static const int nsm = [] {
+    int d = 0, v = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    return v;
+  }();
+  return ((ni + 127) / 128) * ((nj + 127) / 128) < nsm;
+}
+
 template <int MODE>
 static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t s) {
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
+  const bool small = small_tiles<MODE>(a.ni, a.nj);
+  constexpr int TMs = MODE == MODE_SYR2K ? 8 : 4;  // SYR2K never takes the small tile (static_assert)
+  const void* f = small ? (const void*)tiled_kernel<MODE, 2, TMs> : tiled_func<MODE>();
   size_t dyn = 0;
-  catt_status st = prepare_launch(tiled_func<MODE>(), t, 256, 0, false, &a.t, &dyn);
+  catt_status st = prepare_launch(f, t, 256, 0, false, &a.t, &dyn);
   if (st != CATT_OK) return st;
-  const int64_t ty = (a.ni + BM - 1) / BM, tx = (a.nj + BM - 1) / BM;
+  const int64_t BMx = small ? 64 : 128;
+  const int64_t ty = (a.ni + BMx - 1) / BMx, tx = (a.nj + BMx - 1) / BMx;
   if (ty > 65535 || tx > (int64_t(1) << 31) - 1) return CATT_EINVAL;
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
   a.vec = (a.m % 4 == 0) && al(a.A) && (MODE != MODE_SYR2K || al(a.B));
   a.bvec = MODE == MODE_GEMM && (a.nj % 4 == 0) && al(a.B);
   a.cvec = (a.nj % 4 == 0) && al(a.C);
   const dim3 grid{unsigned(tx), unsigned(ty), 1u};
-  if (tiled_minb(MODE == MODE_SYR2K) == 2)
+  if (small)
+    tiled_kernel<MODE, 2, TMs><<<grid, 256, dyn, s>>>(a);
+  else if (tiled_minb(MODE == MODE_SYR2K) == 2)
     tiled_kernel<MODE, 2><<<grid, 256, dyn, s>>>(a);
   else
     tiled_kernel<MODE, 1><<<grid, 256, dyn, s>>>(a);
@@ -381,6 +408,13 @@ __global__ void __launch_bounds__(1024, 2) gemm_thread_kernel(GemmArgs a) {
   cta_exit(a.t);
 }
 
+// The upper tiles of C = beta C + alpha A A^T (tiles with column block >=
+// row block); elements below the diagonal inside diagonal tiles are computed
+// too. The caller mirrors the rest (CORR).
+catt_status syrk_upper(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta, cudaStream_t s) {
+  return launch_tiled<MODE_SYRK>(TileArgs{A, nullptr, C, n, n, m, alpha, beta, 0, 0, 0, 1, {}}, nullptr, s);
+}
+
 const void* gemm_func(int variant) {
   return variant == CATT_VAR_STAGED ? tiled_func<MODE_GEMM>() : (const void*)gemm_thread_kernel;
 }
@@ -409,7 +443,7 @@ extern "C" catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m,
     syrk_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_SYRK>(TileArgs{A, nullptr, C, n, n, m, alpha, beta, 0, 0, 0, {}}, t, s);
+  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_SYRK>(TileArgs{A, nullptr, C, n, n, m, alpha, beta, 0, 0, 0, 0, {}}, t, s);
   return CATT_EINVAL;
 }
 
@@ -433,7 +467,7 @@ extern "C" catt_status catt_syr2k(const float* A, const float* B, float* C, int6
     syr2k_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_SYR2K>(TileArgs{A, B, C, n, n, m, alpha, beta, 0, 0, 0, {}}, t, s);
+  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_SYR2K>(TileArgs{A, B, C, n, n, m, alpha, beta, 0, 0, 0, 0, {}}, t, s);
   return CATT_EINVAL;
 }
 
@@ -458,6 +492,6 @@ extern "C" catt_status catt_gemm(const float* A, const float* B, float* C, int64
     gemm_thread_kernel<<<grid, dim3(32, by), dyn, s>>>(a);
     return after_launch();
   }
-  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_GEMM>(TileArgs{A, B, C, ni, nj, nk, alpha, beta, 0, 0, 0, {}}, t, s);
+  if (var == CATT_VAR_STAGED) return launch_tiled<MODE_GEMM>(TileArgs{A, B, C, ni, nj, nk, alpha, beta, 0, 0, 0, 0, {}}, t, s);
   return CATT_EINVAL;
 }

@@ -277,7 +277,7 @@ def test_bypass_rows_equal_literal():
 # ------------------------------------------------------------------ GEMM (CI control)
 @pytest.mark.parametrize("variant", ["literal", "staged"])
 @pytest.mark.parametrize("ni,nj,nk", [(64, 64, 64), (130, 70, 37), (257, 129, 8), (1, 3, 2), (512, 512, 512),
-                                      (100, 130, 1)])
+                                      (100, 130, 1), (2048, 1200, 64)])   # the last: 128 x 128 tiles
 def test_gemm_exact(variant, ni, nj, nk):
     A, B, C = si.matrix(21, ni, nk), si.matrix(22, nk, nj), si.matrix(23, ni, nj)
     C_o = oracle.gemm(A, B, C, 1.5, 1.2)
