@@ -238,8 +238,10 @@ def test_guards_do_not_touch_paper_mode():
 def test_corr_gives_up_and_gemm_keeps_full_tlp():
     """CORR's footprint does not fit at any TLP (the reused line of
     data[i*m + j1] returns only after n rows), so CATT keeps the baseline;
-    Table 3 P:353 lists CORR #2 at (8,1) everywhere. P:397: the CI control
-    (GEMM) keeps baseline TLP."""
+    Table 3 P:353 lists CORR #2 at (8,1) everywhere. The union model (reading
+    R10: outer-loop reuse keeps the inner loop's lines) reproduces that row;
+    paper mode's per-warp Eq 8 sum does not (it throttles to (4,1) at 32 KB:
+    R15). P:397: the CI control (GEMM) keeps baseline TLP in both modes."""
     corr = catt.problem(catt.K_CORR, n=2048, k=2048)
     gemm = catt.problem(catt.K_GEMM, m=512, n=512, k=512)
     b200 = catt.hw_b200()
@@ -250,6 +252,8 @@ def test_corr_gives_up_and_gemm_keeps_full_tlp():
             assert (r["base_warps"], r["base_ctas"]) == (8, 1) and t.active_warps == 0 and t.active_ctas == 0
             t, r = catt.plan(gemm, catt.Throttle(carveout_kb=carve), hw)
             assert r["flags"] == catt.FIT_NONE_NEEDED and t.active_warps == 0 and t.active_ctas == 0
+            t, r = catt.plan(gemm, catt.Throttle(carveout_kb=carve), hw, mode=catt.MODE_PAPER)
+            assert r["flags"] == catt.FIT_NONE_NEEDED
     for carve in (8, 100, 228):   # B200 rule: the reused reference is coalesced -> guard, no throttle
         t, r = catt.plan(corr, catt.Throttle(carveout_kb=carve), b200)
         assert r["flags"] == catt.FIT_NONE_NEEDED | catt.FIT_GUARDED and t.active_warps == 0
