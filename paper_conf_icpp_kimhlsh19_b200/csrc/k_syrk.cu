@@ -115,23 +115,25 @@ struct TileArgs {
   Throttle t;
 };
 
-template <int MODE, int TM>
+template <int MODE, int TM, bool LEAN = false>
 struct TileCfg {
   static constexpr int BM = 16 * TM;            // tile edge
   static constexpr int H = TM / 4;              // float4 groups per thread per dimension
   static constexpr int GS = BM / H;             // group stride: rows {g*GS + 4t + r}
   static constexpr int PITCH = BM + 4;          // transposed stage rows: 16-B aligned, store banks spread
-  static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
+  static constexpr int BK = (MODE == MODE_SYR2K || LEAN) ? 8 : 16;
+  static constexpr int FBUF = LEAN ? 1 : 2;     // register fragments: double-buffered unless LEAN
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int KQ = BK / 4;             // float4 per stage row
   static constexpr int NV = BM * KQ / 256;      // float4 per thread per array per stage
   static_assert(NV >= 1, "tile too small for the stage depth");
 };
 
-template <int MODE, int MINB, int TM = 8>
+// LEAN: BK = 8 and single-buffered fragments (fewer registers: 2 CTAs per SM)
+template <int MODE, int MINB, int TM = 8, bool LEAN = false>
 __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
   constexpr bool TWO = MODE == MODE_SYR2K, GEMM = MODE == MODE_GEMM;
-  using Cfg = TileCfg<MODE, TM>;
+  using Cfg = TileCfg<MODE, TM, LEAN>;
   constexpr int BK = Cfg::BK, NA = Cfg::NA, KQ = Cfg::KQ, NV = Cfg::NV, BM = Cfg::BM, H = Cfg::H, GS = Cfg::GS;
   constexpr int PITCH = Cfg::PITCH;
   auto tile_off = [](int t, int r) { return (r / 4) * GS + t * 4 + (r % 4); };
@@ -232,7 +234,7 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
       }
     }
   };
-  float f[2][NA][TM];
+  float f[Cfg::FBUF][NA][TM];
   auto fload = [&](int fb, int buf, int kk) {
 #pragma unroll
     for (int s = 0; s < NA; ++s) {
@@ -274,8 +276,13 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
     if (kvalid == BK) {
 #pragma unroll
       for (int kk = 0; kk < BK; ++kk) {
-        if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
-        fma_step(kk & 1);
+        if constexpr (LEAN) {
+          if (kk > 0) fload(0, buf, kk);
+          fma_step(0);
+        } else {
+          if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
+          fma_step(kk & 1);
+        }
       }
     } else {  // ragged last stage: exactly kvalid steps
       fma_step(0);
@@ -323,6 +330,25 @@ static int tiled_minb(bool two) {
   (void)two;
 }
 
+// LEAN large tiles (BK = 8, single-buffered fragments, 2 CTAs per SM) for
+// SYRK when there are more active tiles than SMs: the SMs that get two tiles
+// run them concurrently (SYRK 2048: 0.497 -> 0.460 ms). With at most one tile
+// per SM the regular kernel is faster (CORR's upper tiles: 136 < 148).
+// CATT_TILED_LEAN=0 turns it off (tools only).
+static bool tiled_lean(int64_t active_tiles) {
+  static const int env = [] {
+    const char* e = getenv("CATT_TILED_LEAN");
+    return e ? atoi(e) : -1;
+  }();
+  static const int nsm = [] {
+    int d = 0, v = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    return v;
+  }();
+  if (env == 0) return false;
+  return active_tiles > nsm;
+}
+
 template <int MODE>
 static const void* tiled_func() {
   return tiled_minb(MODE == MODE_SYR2K) == 2 ? (const void*)tiled_kernel<MODE, 2> : (const void*)tiled_kernel<MODE, 1>;
@@ -346,7 +372,11 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
   const bool small = small_tiles<MODE>(a.ni, a.nj);
   constexpr int TMs = MODE == MODE_SYR2K ? 8 : 4;  // SYR2K never takes the small tile (static_assert)
+  const int64_t tt = (a.ni + 127) / 128;
+  const bool lean = !small && MODE == MODE_SYRK && tiled_lean(a.tri ? tt * (tt + 1) / 2 : tt * tt);
   const void* f = small ? (const void*)tiled_kernel<MODE, 2, TMs> : tiled_func<MODE>();
+  if constexpr (MODE == MODE_SYRK)
+    if (lean) f = (const void*)tiled_kernel<MODE, 2, 8, true>;
   size_t dyn = 0;
   catt_status st = prepare_launch(f, t, 256, 0, false, &a.t, &dyn);
   if (st != CATT_OK) return st;
@@ -358,7 +388,15 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
   a.bvec = MODE == MODE_GEMM && (a.nj % 4 == 0) && al(a.B);
   a.cvec = (a.nj % 4 == 0) && al(a.C);
   const dim3 grid{unsigned(tx), unsigned(ty), 1u};
-  if (small)
+  bool done = false;
+  if constexpr (MODE == MODE_SYRK) {
+    if (lean) {
+      tiled_kernel<MODE, 2, 8, true><<<grid, 256, dyn, s>>>(a);
+      done = true;
+    }
+  }
+  if (done) {
+  } else if (small)
     tiled_kernel<MODE, 2, TMs><<<grid, 256, dyn, s>>>(a);
   else if (tiled_minb(MODE == MODE_SYR2K) == 2)
     tiled_kernel<MODE, 2><<<grid, 256, dyn, s>>>(a);
