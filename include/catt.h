@@ -424,6 +424,12 @@ catt_status catt_kernel_attrs(const catt_problem* prob, const catt_throttle* t, 
 
 const char* catt_status_str(catt_status s);
 int catt_last_cuda_error(void);
+/* Diagnostics: the FUSED single-read kernel records, when the environment
+ * variable CATT_FUSED_TRACE is set at launch, six %globaltimer stamps per CTA
+ * (start, first stage landed, last stage consumed, column partials written,
+ * after the grid barrier, end) for CTAs < 1024. Copies the first n of the
+ * 6144 u64 values (CTA-major) to host memory `out` (synchronous). */
+catt_status catt_fused_trace(uint64_t* out, int32_t n);
 int catt_abi_version(void);
 
 #ifdef __cplusplus

@@ -176,6 +176,7 @@ def lib():
             "catt_fill_hash": [V, i64, u32, u64, i32, V],
             "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
             "catt_kernel_attrs": [P(Problem), T, P(i32), P(i32)],
+            "catt_fused_trace": [P(u64), i32],
             "catt_status_str": [ctypes.c_int],
             "catt_last_cuda_error": [],
             "catt_abi_version": [],
@@ -195,7 +196,7 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_gemm", "catt_corr", "catt_kmeans_assign",
             "catt_kmeans_acc_words", "catt_kmeans_transpose", "catt_kmeans_accumulate", "catt_kmeans_finalize",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
-            "catt_last_cuda_error", "catt_abi_version"]
+            "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace"]
 
 
 def _check(st: int, what: str):
@@ -416,6 +417,15 @@ def syr2k(A, B, C, alpha, beta, t: Optional[Throttle] = None):
     _check(lib().catt_syr2k(_dev(A, "A"), _dev(B, "B"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t),
                             _stream()), "catt_syr2k")
     return C
+
+
+def fused_trace(nctas):
+    """Phase timestamps (ns) of the last traced FUSED single-read launch
+    (CATT_FUSED_TRACE set at launch): array [nctas, 6] (catt_fused_trace)."""
+    import numpy as np
+    out = np.zeros(nctas * 6, dtype=np.uint64)
+    _check(lib().catt_fused_trace(out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), nctas * 6), "catt_fused_trace")
+    return out.reshape(nctas, 6)
 
 
 def kmeans_assign(feat, ld, npoints, nf, clusters, membership=None, t: Optional[Throttle] = None):

@@ -1,0 +1,27 @@
+// f32x2.cuh — packed fp32 pairs (sm_100a FFMA2 / FADD2). Each half is an
+// ordinary IEEE round-to-nearest fp32 operation, so a kernel that pairs two
+// independent chains computes bit-for-bit what two scalar chains compute.
+#pragma once
+#include <cstdint>
+
+namespace catt {
+
+__device__ __forceinline__ uint64_t f2_pack(float lo, float hi) {
+  return uint64_t(__float_as_uint(lo)) | (uint64_t(__float_as_uint(hi)) << 32);
+}
+__device__ __forceinline__ float f2_lo(uint64_t v) { return __uint_as_float(unsigned(v)); }
+__device__ __forceinline__ float f2_hi(uint64_t v) { return __uint_as_float(unsigned(v >> 32)); }
+// a - b per half
+__device__ __forceinline__ uint64_t f2_sub(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+// fmaf(a, b, c) per half
+__device__ __forceinline__ uint64_t f2_fma(uint64_t a, uint64_t b, uint64_t c) {
+  uint64_t d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+
+}  // namespace catt

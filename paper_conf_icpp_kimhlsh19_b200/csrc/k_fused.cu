@@ -27,6 +27,10 @@
 namespace catt {
 
 constexpr int kMaxDual = 4;
+constexpr int kTraceCtas = 1024, kTracePhases = 6;
+// per-CTA %globaltimer at: start, first stage landed, last stage consumed,
+// partials written, after the grid barrier, end (diagnostics only)
+__device__ unsigned long long g_fused_trace[kTraceCtas * kTracePhases];
 constexpr int kBandMax = 2048;  // rows per CTA whose xc / yr are staged in shared memory
 
 // Up to kMaxDual independent problems with the same column count N share one
@@ -44,6 +48,9 @@ struct FusedArgs {
   int row_acc[kMaxDual], col_acc[kMaxDual];
   int nprob;
   int bandcap;                // rows per CTA whose xc / yr fit the shared-memory band buffer (nd kernel)
+  int inter;                  // nd kernel: stage chunks dealt round robin over the problem's CTAs
+  int trace;                  // nd kernel: record phase timestamps per CTA (catt_fused_trace)
+  int fastbar;                // nd kernel: grid barrier by ordered atomics (grid_barrier_ordered)
   unsigned* gbar;             // grid barrier {count, generation}
   int64_t N;
 };
@@ -70,6 +77,30 @@ __device__ __forceinline__ void grid_barrier(unsigned* bar, unsigned nblocks) {
       while (vb[1] == gen) __nanosleep(64);
     }
     __threadfence();
+  }
+  __syncthreads();
+}
+
+// The same barrier with ordered atomics instead of separate fences: the
+// arrival is one acq_rel add (it publishes this CTA's earlier writes, which
+// __syncthreads made visible to thread 0), the last arriver resets the count
+// and bumps the generation with one release add, the others poll the
+// generation with acquire loads (no sleep: 148 pollers on one L2 line).
+__device__ __forceinline__ void grid_barrier_ordered(unsigned* bar, unsigned nblocks) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned gen, old;
+    asm volatile("ld.relaxed.gpu.u32 %0, [%1];" : "=r"(gen) : "l"(bar + 1) : "memory");
+    asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(old) : "l"(bar) : "memory");
+    if (old == nblocks - 1) {
+      asm volatile("st.relaxed.gpu.u32 [%0], 0;" ::"l"(bar) : "memory");
+      asm volatile("red.release.gpu.add.u32 [%0], 1;" ::"l"(bar + 1) : "memory");
+    } else {
+      unsigned cur;
+      do {
+        asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(cur) : "l"(bar + 1) : "memory");
+      } while (cur == gen);
+    }
   }
   __syncthreads();
 }
@@ -277,9 +308,18 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
   const int lb = int(blockIdx.x) - a.cta0[pi];
   const int64_t N = a.N, n4 = N >> 2, M = a.M[pi];
   const int64_t stage_bytes = int64_t(RPS) * N * 4;
-  const int64_t r0 = int64_t(lb) * a.band[pi], r1 = imin64(M, r0 + a.band[pi]);
-  const int64_t nst = r1 > r0 ? (r1 - r0 + RPS - 1) / RPS : 0;
+  // rows of stage c: a.inter = 0: the CTA's band [r0, r1) in order; a.inter = 1:
+  // chunks of RPS rows dealt round robin (chunk lb + c * Gp), so at any time
+  // all CTAs stream one narrow window of A
+  const int64_t Gp = a.cta0[pi + 1] - a.cta0[pi];
+  const int64_t r0 = a.inter ? 0 : int64_t(lb) * a.band[pi], r1 = a.inter ? M : imin64(M, r0 + a.band[pi]);
+  const int64_t nch = (M + RPS - 1) / RPS;
+  const int64_t nst = a.inter ? (nch > lb ? (nch - lb + Gp - 1) / Gp : 0) : (r1 > r0 ? (r1 - r0 + RPS - 1) / RPS : 0);
+  auto row0 = [&](int64_t c) { return a.inter ? (int64_t(lb) + c * Gp) * RPS : r0 + c * RPS; };
   const bool racc = a.row_acc[pi] != 0;
+  const bool tr = a.trace && blockIdx.x < kTraceCtas;
+  unsigned long long* trp = g_fused_trace + blockIdx.x * kTracePhases;
+  if (tr && threadIdx.x == 0) trp[0] = gtimer();
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       bar_init(&full[s], 1);
@@ -290,20 +330,23 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
   }
   auto issue = [&](int64_t c) {                                 // producer lane 0
     const int s = int(c % S);
-    const int64_t rows = imin64(RPS, r1 - (r0 + c * RPS));
+    const int64_t rows = imin64(RPS, r1 - row0(c));
     const uint32_t bytes = uint32_t(rows * N * 4);
     bar_expect_tx(&full[s], bytes);
-    bulk_1d(ring + int64_t(s) * stage_bytes, Ap + (r0 + c * RPS) * N, bytes, &full[s]);
+    bulk_1d(ring + int64_t(s) * stage_bytes, Ap + row0(c) * N, bytes, &full[s]);
   };
   __syncthreads();
   if (producer && lane == 0)
     for (int64_t c = 0; c < imin64(S, nst); ++c) issue(c);
   // the band's column weights and initial row values, all loads in flight at once
-  const bool inband = r1 - r0 <= BC;
+  // the CTA's column weights and initial row values (local row c * RPS + u),
+  // all loads in flight at once
+  const bool inband = nst * RPS <= BC;
   if (inband) {
-    for (int64_t i = threadIdx.x; i < r1 - r0; i += blockDim.x) {
-      bandbuf[i] = xc[r0 + i];
-      bandbuf[BC + i] = racc ? yr[r0 + i] : 0.0f;
+    for (int64_t i = threadIdx.x; i < nst * RPS; i += blockDim.x) {
+      const int64_t g = row0(i / RPS) + i % RPS;
+      bandbuf[i] = g < M ? xc[g] : 0.0f;
+      bandbuf[BC + i] = (racc && g < M) ? yr[g] : 0.0f;
     }
   }
   __syncthreads();
@@ -315,7 +358,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
     // row totals, then refill the consumed slot
     constexpr int RPP = 32 / NW;
     for (int64_t c = 0; c < nst; ++c) {
-      const int64_t i0 = r0 + c * RPS;
+      const int64_t i0 = row0(c);
       const int rows = int(imin64(RPS, r1 - i0));
       const int q = int(c % (2 * S));
       const float* rb = rowbuf + int64_t(q) * RPS * NW;
@@ -326,7 +369,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
 #pragma unroll
         for (int o = NW / 2; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
         if (lane % NW == 0 && u < rows) {
-          const float y0 = racc ? (inband ? bandbuf[BC + (i0 + u - r0)] : yr[i0 + u]) : 0.0f;
+          const float y0 = racc ? (inband ? bandbuf[BC + c * RPS + u] : yr[i0 + u]) : 0.0f;
           yr[i0 + u] = racc ? y0 + v : v;
         }
       }
@@ -351,10 +394,11 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
     for (int64_t c = 0; c < nst; ++c) {
       const int s = int(c % S);
       const int q = int(c % (2 * S));
-      const int64_t i0 = r0 + c * RPS;
+      const int64_t i0 = row0(c);
       const int rows = int(imin64(RPS, r1 - i0));
-      const float wl = lane < rows ? (inband ? bandbuf[i0 - r0 + lane] : xc[i0 + lane]) : 0.0f;
+      const float wl = lane < rows ? (inband ? bandbuf[c * RPS + lane] : xc[i0 + lane]) : 0.0f;
       bar_wait(&full[s], uint32_t((c / S) & 1));
+      if (tr && c == 0 && threadIdx.x == 0) trp[1] = gtimer();
       const float4* st = reinterpret_cast<const float4*>(ring + int64_t(s) * stage_bytes);
       float* rb = rowbuf + int64_t(q) * RPS * NW;
       for (int u0 = 0; u0 < rows; u0 += 4) {
@@ -412,6 +456,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
   // column partials -> workspace (the producer's acc is zero and unused);
   // grid barrier; fixed-tree column outputs
   float* part = a.part[pi] + int64_t(lb) * N;
+  if (tr && threadIdx.x == 0) trp[2] = gtimer();
   if (!producer) {
 #pragma unroll
     for (int t = 0; t < T; ++t) {
@@ -419,8 +464,15 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
       if (cc < n4) reinterpret_cast<float4*>(part)[cc] = acc[t];
     }
   }
-  __threadfence();
-  grid_barrier(a.gbar, gridDim.x);
+  if (a.fastbar) {
+    if (tr && threadIdx.x == 0) trp[3] = gtimer();
+    grid_barrier_ordered(a.gbar, gridDim.x);
+  } else {
+    __threadfence();
+    if (tr && threadIdx.x == 0) trp[3] = gtimer();
+    grid_barrier(a.gbar, gridDim.x);
+  }
+  if (tr && threadIdx.x == 0) trp[4] = gtimer();
   // column outputs in one round: chunks of CW = 32*L columns (L per lane,
   // chosen so every problem's chunks fit the grid); consumer warp w sums band
   // partials [w*gpw, (w+1)*gpw) in order, then the NW warp sums in warp order
@@ -467,6 +519,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
       __syncthreads();
     }
   }
+  if (tr && threadIdx.x == 0) trp[5] = gtimer();
 }
 
 namespace {
@@ -534,7 +587,7 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   const int64_t stage_target = (rps_env ? atoi(rps_env) : 64) * 1024;
   const int RPS = int(std::max<int64_t>(1, std::min<int64_t>(16, stage_target / row_bytes)));
   const char* budget_env = getenv("CATT_FUSED_SMEM_KB");
-  const int64_t budget = (budget_env ? atoi(budget_env) : 200) * 1024;
+  const int64_t budget = (budget_env ? atoi(budget_env) : 220) * 1024;
   // head: barriers in the first 1 KB, then the row partials (DEP: [RPS][NW+1];
   // single-read kernel: [S][RPS][NW], sized for up to 16 stages)
   DevCtx* ctx = nullptr;
@@ -599,6 +652,13 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   args.nprob = np;
   args.N = N;
   args.bandcap = bandcap;
+  {
+    const char* ie = getenv("CATT_FUSED_INTERLEAVE");
+    args.inter = nd ? (ie ? atoi(ie) != 0 : 1) : 0;
+    args.trace = nd && getenv("CATT_FUSED_TRACE") != nullptr;
+    const char* fb = getenv("CATT_FUSED_BARRIER");
+    args.fastbar = fb ? atoi(fb) != 0 : 1;
+  }
   int64_t given = 0;
   int cta = 0;
   for (int i = 0; i < np; ++i) {
@@ -668,6 +728,17 @@ const void* fused_func(bool dep) { return dep ? fused_fn<true>(16, 2) : fused_fn
 }  // namespace catt
 
 using namespace catt;
+
+extern "C" catt_status catt_fused_trace(uint64_t* out, int32_t n) {
+  if (!out || n < 0) return CATT_EINVAL;
+  const size_t bytes = size_t(std::min(n, kTraceCtas * kTracePhases)) * sizeof(uint64_t);
+  cudaError_t e = cudaMemcpyFromSymbol(out, g_fused_trace, bytes);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  return CATT_OK;
+}
 
 extern "C" catt_status catt_dual_group(const catt_dual_problem* probs, int32_t count, int32_t dependent,
                                        const catt_throttle* t, void* stream) {

@@ -15,6 +15,11 @@
 // registers: for f: v = feat[f*ld + p]; for c: d[c] = fmaf(v - C[c][f], ...).
 // Every (point, centre) pair still accumulates f = 0, 1, ... in order, so the
 // membership is bit-identical to LITERAL; no L1 reuse is needed.
+// COOP: a warp takes 128 consecutive points, a lane 4 of them: one 16-byte
+// L1-bypassing load per feature (512 B per warp request instead of 128 B),
+// FB features in flight per lane. The 4 points are two packed fp32 pairs, so
+// one FADD2 + one FFMA2 advance two (point, centre) chains; each half is the
+// scalar IEEE operation in the same order: bit-identical membership.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -23,6 +28,7 @@
 #include <cfloat>
 #include <cstdint>
 
+#include "f32x2.cuh"
 #include "internal.h"
 #include "tma.cuh"
 
@@ -162,6 +168,127 @@ __global__ void __launch_bounds__(256) kmeans_stream_kernel(KmArgs a) {
 }
 
 
+// COOP (see the header): centres duplicated into pairs (c, c) in shared
+// memory, [nf][KP] with KP = KMAX rounded up to 2, read as 16-byte
+// broadcasts; padding centres are +inf (never strictly nearer than FLT_MAX).
+// Persistent warps take 128-point groups g = warp id + i * (warps in grid);
+// the (group, feature batch) sequence is software-pipelined: the FB loads of
+// the next batch (possibly of the next group) are in flight while the current
+// batch is computed.
+template <int KMAX, int FB>
+__global__ void __launch_bounds__(256, 2) kmeans_coop_kernel(KmArgs a) {
+  constexpr int KP = (KMAX + 1) & ~1;
+  extern __shared__ __align__(16) unsigned char dyn_c[];
+  uint64_t* s_cd = reinterpret_cast<uint64_t*>(dyn_c);
+  const int nf = a.nf, k = a.k;
+  for (int q = threadIdx.x; q < nf * KP; q += blockDim.x) {
+    const int f = q / KP, c = q - f * KP;
+    const float v = c < k ? a.clusters[c * nf + f] : __int_as_float(0x7f800000);
+    s_cd[q] = f2_pack(v, v);
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t ngroups = (a.npoints + 127) / 128;
+  const int64_t gw = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int64_t TW = int64_t(gridDim.x) * (blockDim.x >> 5);
+  if (gw >= ngroups) return;
+  const int nb = (nf + FB - 1) / FB;                    // feature batches per group
+  const int64_t mine = (ngroups - gw + TW - 1) / TW;    // groups of this warp
+  const int64_t steps = mine * nb;                      // (group, batch) steps, software-pipelined
+  const int64_t ld = a.ld;
+  float4 cur[FB], nxt[FB];
+  // loads of step (group index gi: points from (gw + gi * TW) * 128, batch b)
+  auto load = [&](int64_t gi, int b, float4 (&v)[FB]) {
+    const int64_t p = (gw + gi * TW) * 128 + lane * 4;
+    const int f0 = b * FB;
+    const bool live = p < a.npoints;                    // p + 3 < ld: the 16-byte load stays inside row f
+    const float* src = a.feat + p + int64_t(f0) * ld;
+#pragma unroll
+    for (int u = 0; u < FB; ++u) {
+      v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (live && f0 + u < nf)
+        asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[u].x), "=f"(v[u].y), "=f"(v[u].z), "=f"(v[u].w)
+                     : "l"(src + int64_t(u) * ld));
+    }
+  };
+  uint64_t d01[KMAX], d23[KMAX];
+#pragma unroll
+  for (int c = 0; c < KMAX; ++c) d01[c] = d23[c] = 0ull;
+  load(0, 0, cur);
+  int64_t gi = 0;                                       // current group (of this warp) and batch
+  int b = 0;
+  for (int64_t j = 0; j < steps; ++j) {
+    const bool last = b == nb - 1;
+    if (j + 1 < steps) load(last ? gi + 1 : gi, last ? 0 : b + 1, nxt);
+    const int f0 = b * FB;
+#pragma unroll
+    for (int u = 0; u < FB; ++u) {
+      if (f0 + u < nf) {
+        const uint64_t v01 = f2_pack(cur[u].x, cur[u].y), v23 = f2_pack(cur[u].z, cur[u].w);
+        const ulonglong2* cf = reinterpret_cast<const ulonglong2*>(s_cd + (f0 + u) * KP);
+#pragma unroll
+        for (int q = 0; q < KP / 2; ++q) {
+          const ulonglong2 c2 = cf[q];
+          {
+            const uint64_t e01 = f2_sub(v01, c2.x), e23 = f2_sub(v23, c2.x);
+            d01[2 * q] = f2_fma(e01, e01, d01[2 * q]);
+            d23[2 * q] = f2_fma(e23, e23, d23[2 * q]);
+          }
+          if (2 * q + 1 < KMAX) {
+            const uint64_t e01 = f2_sub(v01, c2.y), e23 = f2_sub(v23, c2.y);
+            d01[2 * q + 1] = f2_fma(e01, e01, d01[2 * q + 1]);
+            d23[2 * q + 1] = f2_fma(e23, e23, d23[2 * q + 1]);
+          }
+        }
+      }
+    }
+    if (last) {                                          // group done: argmin of its 4 points per lane
+      const int64_t p = (gw + gi * TW) * 128 + lane * 4;
+      if (p < a.npoints) {
+        int idx[4];
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) {
+          int index = -1;
+          float best = FLT_MAX;
+#pragma unroll
+          for (int c = 0; c < KMAX; ++c) {
+            const float dv = jj == 0 ? f2_lo(d01[c]) : jj == 1 ? f2_hi(d01[c]) : jj == 2 ? f2_lo(d23[c]) : f2_hi(d23[c]);
+            if (dv < best) {
+              best = dv;
+              index = c;
+            }
+          }
+          idx[jj] = index;
+        }
+        int32_t* m = a.membership + p;
+        if (p + 3 < a.npoints && (reinterpret_cast<uintptr_t>(m) & 15u) == 0) {
+          *reinterpret_cast<int4*>(m) = make_int4(idx[0], idx[1], idx[2], idx[3]);
+        } else {
+#pragma unroll
+          for (int jj = 0; jj < 4; ++jj)
+            if (p + jj < a.npoints) m[jj] = idx[jj];
+        }
+      }
+#pragma unroll
+      for (int c = 0; c < KMAX; ++c) d01[c] = d23[c] = 0ull;
+      ++gi;
+      b = 0;
+    } else {
+      ++b;
+    }
+#pragma unroll
+    for (int u = 0; u < FB; ++u) cur[u] = nxt[u];
+  }
+}
+
+const void* kmeans_coop_fn(int k) {
+  if (k <= 2) return (const void*)kmeans_coop_kernel<2, 8>;
+  if (k <= 4) return (const void*)kmeans_coop_kernel<4, 8>;
+  if (k == 5) return (const void*)kmeans_coop_kernel<5, 8>;
+  return (const void*)kmeans_coop_kernel<8, 6>;
+}
+
 // STAGED: persistent CTAs; 2-D TMA copies of {256 points x nf features} tiles
 // (one request per tile) into an S-stage ring; thread t computes point
 // tile*256 + t from shared memory (column t of every feature row: conflict
@@ -269,6 +396,7 @@ int kmeans_tma_minb() {
 const void* kmeans_func(int variant, int nf) {
   (void)nf;
   if (variant == CATT_VAR_STAGED) return kmeans_tma_minb() == 2 ? kmeans_tma_fn<2>(8) : kmeans_tma_fn<1>(8);
+  if (variant == CATT_VAR_COOP) return kmeans_coop_fn(5);
   if (variant != CATT_VAR_REGS) return (const void*)kmeans_kernel<0>;
   return (const void*)kmeans_stream_kernel<8>;
 }
@@ -348,6 +476,35 @@ extern "C" catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t
   if (npoints == 0) return CATT_OK;
   const int var = variant_of(t);
   if (var == CATT_VAR_STAGED) return launch_kmeans_tma(feat, ld, npoints, nf, clusters, k, membership, t, stream);
+  if (var == CATT_VAR_COOP) {
+    // no L1-resident reference: nothing to throttle; 16-byte loads need ld % 4 == 0 and an aligned base
+    if (k > 8 || ld % 4 || (reinterpret_cast<uintptr_t>(feat) & 15u)) return CATT_EINVAL;
+    if (t && (t->active_warps || t->active_ctas || (t->cta_threads && t->cta_threads != 256))) return CATT_EINVAL;
+    const void* f = kmeans_coop_fn(k);
+    const int KP = ((k <= 2 ? 2 : k <= 4 ? 4 : k == 5 ? 5 : 8) + 1) & ~1;
+    const size_t dyn = size_t(nf) * KP * sizeof(uint64_t);
+    if (dyn > 48 * 1024 && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn)) != cudaSuccess)
+      return after_launch();
+    KmArgs a{feat, clusters, membership, ld, npoints, nf, k, Throttle{}};
+    DevCtx* ctx = nullptr;
+    catt_status st = dev_ctx(&ctx);
+    if (st != CATT_OK) return st;
+    int per_sm = 0;
+    cudaError_t oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, 256, dyn);
+    if (oe != cudaSuccess || per_sm < 1) {
+      record_cuda_error(oe == cudaSuccess ? cudaErrorInvalidConfiguration : oe);
+      return CATT_ECUDA;
+    }
+    const int64_t groups = (npoints + 127) / 128;       // persistent: at most one wave of CTAs
+    const unsigned grid = unsigned(std::min<int64_t>((groups + 7) / 8, int64_t(per_sm) * ctx->hw.num_sms));
+    void* args[] = {&a};
+    cudaError_t e = cudaLaunchKernel(f, dim3(grid), dim3(256), args, dyn, static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) {
+      record_cuda_error(e);
+      return CATT_ECUDA;
+    }
+    return after_launch();
+  }
   if (var != CATT_VAR_LITERAL && var != CATT_VAR_REGS) return CATT_EINVAL;
   const int threads = cta_threads_or(t, 256);
   if (var == CATT_VAR_REGS && (k > 32 || threads > 256)) return CATT_EINVAL;

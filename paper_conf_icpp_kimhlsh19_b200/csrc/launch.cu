@@ -492,6 +492,13 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->n_loops = 1;
       out->trip[0] = nf;
       refs[n++] = mkref(1, 0, ld, 0, 4, 1, CATT_REF_NOT_L1);       // TMA tiles in shared memory
+    } else if (var == CATT_VAR_COOP) {
+      out->grid[0] = (np + 4 * threads - 1) / (4 * threads);       // a lane = 4 points
+      out->extent[0] = (np + 3) / 4;
+      out->n_loops = 1;
+      out->trip[0] = nf;
+      refs[n++] = mkref(4, 0, ld, 0, 4, 1, CATT_REF_NOT_L1);       // 16-byte L1::no_allocate loads
+      dyn = nf * ((k + 1) & ~1) * 8;                               // centre pairs (c, c)
     } else {
       return CATT_EINVAL;
     }

@@ -326,18 +326,23 @@ def test_corr_2048_full_size():
 
 
 # ------------------------------------------------------------------ KMEANS
-@pytest.mark.parametrize("variant", ["literal", "regs", "staged"])
+@pytest.mark.parametrize("variant", ["literal", "regs", "staged", "coop"])
 @pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 4), (4099, 34, 5, 29), (257, 7, 3, 3), (300, 50, 12, 4),
-                                           (70000, 34, 5, 4)])
+                                           (70000, 34, 5, 4), (1, 3, 1, 3), (131, 34, 8, 1), (130, 9, 2, 2)])
 def test_kmeans_exact(variant, npts, nf, k, pad):
     ld = npts + pad
-    if variant == "staged" and ld % 4:
-        ld += 4 - ld % 4                                 # TMA rows need a 16-byte stride
+    if variant in ("staged", "coop") and ld % 4:
+        ld += 4 - ld % 4                                 # TMA rows / 16-byte loads need a 16-byte stride
+    if variant == "coop" and k > 8:
+        with pytest.raises(catt.CattError):
+            catt.kmeans_assign(dev(si.values(4, nf * ld)), ld, npts, nf, dev(np.zeros((k, nf), np.float32)),
+                               t=catt.Throttle(variant="coop"))
+        return
     feat = si.values(4, nf * ld)
     clusters = feat.reshape(nf, ld)[:, :k].T.copy()          # centres = first k points
     memb_o, _ = oracle.kmeans_assign(feat, ld, npts, nf, clusters)
     ts = [catt.Throttle(variant=variant)]
-    if variant != "staged":                              # staged has no L1 reuse to throttle
+    if variant not in ("staged", "coop"):                # staged / coop have no L1 reuse to throttle
         ts.append(catt.Throttle(variant=variant, active_warps=2, active_ctas=3))
     for t in ts:
         memb = catt.kmeans_assign(dev(feat), ld, npts, nf, dev(clusters), t=t)
@@ -373,7 +378,8 @@ def test_kmeans_rodinia_shape_full():
         memb_o, _ = oracle.kmeans_assign(fh, ld, npts, nf, clusters)
         hw = catt.hw_query()
         t, r = catt.plan(catt.problem(catt.K_KMEANS, m=npts, n=nf, k=k, ld=ld), catt.Throttle(), hw)
-        for tt in (catt.Throttle(), t, catt.Throttle(variant="regs"), catt.Throttle(variant="staged")):
+        for tt in (catt.Throttle(), t, catt.Throttle(variant="regs"), catt.Throttle(variant="staged"),
+                   catt.Throttle(variant="coop")):
             memb = catt.kmeans_assign(feat, ld, npts, nf, dev(clusters), t=tt)
             assert np.array_equal(host(memb), memb_o)
 
