@@ -171,12 +171,12 @@ __global__ void __launch_bounds__(256) kmeans_stream_kernel(KmArgs a) {
 // COOP (see the header): centres duplicated into pairs (c, c) in shared
 // memory, [nf][KP] with KP = KMAX rounded up to 2, read as 16-byte
 // broadcasts; padding centres are +inf (never strictly nearer than FLT_MAX).
-// Persistent warps take 128-point groups g = warp id + i * (warps in grid);
-// the (group, feature batch) sequence is software-pipelined: the FB loads of
-// the next batch (possibly of the next group) are in flight while the current
-// batch is computed.
+// One 128-point group per warp, FB features in flight per lane, register-lean
+// (4 CTAs of 256 threads per SM): on B200 this feature-major pattern streams
+// fastest with many warps and few loads each (tools/read_probe.cu fm-groups:
+// 32 warps/SM x 4 loads beat 16 x 8 and persistent software pipelining).
 template <int KMAX, int FB>
-__global__ void __launch_bounds__(256, 2) kmeans_coop_kernel(KmArgs a) {
+__global__ void __launch_bounds__(256, 4) kmeans_coop_kernel(KmArgs a) {
   constexpr int KP = (KMAX + 1) & ~1;
   extern __shared__ __align__(16) unsigned char dyn_c[];
   uint64_t* s_cd = reinterpret_cast<uint64_t*>(dyn_c);
@@ -188,44 +188,29 @@ __global__ void __launch_bounds__(256, 2) kmeans_coop_kernel(KmArgs a) {
   }
   __syncthreads();
   const int lane = threadIdx.x & 31;
-  const int64_t ngroups = (a.npoints + 127) / 128;
-  const int64_t gw = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  const int64_t TW = int64_t(gridDim.x) * (blockDim.x >> 5);
-  if (gw >= ngroups) return;
-  const int nb = (nf + FB - 1) / FB;                    // feature batches per group
-  const int64_t mine = (ngroups - gw + TW - 1) / TW;    // groups of this warp
-  const int64_t steps = mine * nb;                      // (group, batch) steps, software-pipelined
+  const int64_t g = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int64_t p = g * 128 + lane * 4;
+  if (p >= a.npoints) return;                        // p + 3 < ld: the 16-byte load stays inside row f
+  const float* __restrict__ src = a.feat + p;
   const int64_t ld = a.ld;
-  float4 cur[FB], nxt[FB];
-  // loads of step (group index gi: points from (gw + gi * TW) * 128, batch b)
-  auto load = [&](int64_t gi, int b, float4 (&v)[FB]) {
-    const int64_t p = (gw + gi * TW) * 128 + lane * 4;
-    const int f0 = b * FB;
-    const bool live = p < a.npoints;                    // p + 3 < ld: the 16-byte load stays inside row f
-    const float* src = a.feat + p + int64_t(f0) * ld;
-#pragma unroll
-    for (int u = 0; u < FB; ++u) {
-      v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (live && f0 + u < nf)
-        asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
-                     : "=f"(v[u].x), "=f"(v[u].y), "=f"(v[u].z), "=f"(v[u].w)
-                     : "l"(src + int64_t(u) * ld));
-    }
-  };
   uint64_t d01[KMAX], d23[KMAX];
 #pragma unroll
   for (int c = 0; c < KMAX; ++c) d01[c] = d23[c] = 0ull;
-  load(0, 0, cur);
-  int64_t gi = 0;                                       // current group (of this warp) and batch
-  int b = 0;
-  for (int64_t j = 0; j < steps; ++j) {
-    const bool last = b == nb - 1;
-    if (j + 1 < steps) load(last ? gi + 1 : gi, last ? 0 : b + 1, nxt);
-    const int f0 = b * FB;
+#pragma unroll 1
+  for (int f0 = 0; f0 < nf; f0 += FB) {
+    float4 v[FB];
+#pragma unroll
+    for (int u = 0; u < FB; ++u) {
+      v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (f0 + u < nf)
+        asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[u].x), "=f"(v[u].y), "=f"(v[u].z), "=f"(v[u].w)
+                     : "l"(src + int64_t(f0 + u) * ld));
+    }
 #pragma unroll
     for (int u = 0; u < FB; ++u) {
       if (f0 + u < nf) {
-        const uint64_t v01 = f2_pack(cur[u].x, cur[u].y), v23 = f2_pack(cur[u].z, cur[u].w);
+        const uint64_t v01 = f2_pack(v[u].x, v[u].y), v23 = f2_pack(v[u].z, v[u].w);
         const ulonglong2* cf = reinterpret_cast<const ulonglong2*>(s_cd + (f0 + u) * KP);
 #pragma unroll
         for (int q = 0; q < KP / 2; ++q) {
@@ -243,50 +228,37 @@ __global__ void __launch_bounds__(256, 2) kmeans_coop_kernel(KmArgs a) {
         }
       }
     }
-    if (last) {                                          // group done: argmin of its 4 points per lane
-      const int64_t p = (gw + gi * TW) * 128 + lane * 4;
-      if (p < a.npoints) {
-        int idx[4];
+  }
+  int idx[4];
 #pragma unroll
-        for (int jj = 0; jj < 4; ++jj) {
-          int index = -1;
-          float best = FLT_MAX;
+  for (int j = 0; j < 4; ++j) {
+    int index = -1;
+    float best = FLT_MAX;
 #pragma unroll
-          for (int c = 0; c < KMAX; ++c) {
-            const float dv = jj == 0 ? f2_lo(d01[c]) : jj == 1 ? f2_hi(d01[c]) : jj == 2 ? f2_lo(d23[c]) : f2_hi(d23[c]);
-            if (dv < best) {
-              best = dv;
-              index = c;
-            }
-          }
-          idx[jj] = index;
-        }
-        int32_t* m = a.membership + p;
-        if (p + 3 < a.npoints && (reinterpret_cast<uintptr_t>(m) & 15u) == 0) {
-          *reinterpret_cast<int4*>(m) = make_int4(idx[0], idx[1], idx[2], idx[3]);
-        } else {
-#pragma unroll
-          for (int jj = 0; jj < 4; ++jj)
-            if (p + jj < a.npoints) m[jj] = idx[jj];
-        }
+    for (int c = 0; c < KMAX; ++c) {
+      const float dv = j == 0 ? f2_lo(d01[c]) : j == 1 ? f2_hi(d01[c]) : j == 2 ? f2_lo(d23[c]) : f2_hi(d23[c]);
+      if (dv < best) {
+        best = dv;
+        index = c;
       }
-#pragma unroll
-      for (int c = 0; c < KMAX; ++c) d01[c] = d23[c] = 0ull;
-      ++gi;
-      b = 0;
-    } else {
-      ++b;
     }
+    idx[j] = index;
+  }
+  int32_t* m = a.membership + p;
+  if (p + 3 < a.npoints && (reinterpret_cast<uintptr_t>(m) & 15u) == 0) {
+    *reinterpret_cast<int4*>(m) = make_int4(idx[0], idx[1], idx[2], idx[3]);
+  } else {
 #pragma unroll
-    for (int u = 0; u < FB; ++u) cur[u] = nxt[u];
+    for (int j = 0; j < 4; ++j)
+      if (p + j < a.npoints) m[j] = idx[j];
   }
 }
 
 const void* kmeans_coop_fn(int k) {
-  if (k <= 2) return (const void*)kmeans_coop_kernel<2, 8>;
-  if (k <= 4) return (const void*)kmeans_coop_kernel<4, 8>;
-  if (k == 5) return (const void*)kmeans_coop_kernel<5, 8>;
-  return (const void*)kmeans_coop_kernel<8, 6>;
+  if (k <= 2) return (const void*)kmeans_coop_kernel<2, 4>;
+  if (k <= 4) return (const void*)kmeans_coop_kernel<4, 4>;
+  if (k == 5) return (const void*)kmeans_coop_kernel<5, 4>;
+  return (const void*)kmeans_coop_kernel<8, 2>;
 }
 
 // STAGED: persistent CTAs; 2-D TMA copies of {256 points x nf features} tiles
@@ -407,6 +379,23 @@ using namespace catt;
 
 namespace {
 
+}  // namespace
+
+namespace catt {
+// dynamic shared memory of the STAGED kernel: centres + S tile stages
+int64_t kmeans_tma_smem(int nf, int k) {
+  const int KMAX = k <= 4 ? 4 : k == 5 ? 5 : k <= 8 ? 8 : k <= 16 ? 16 : 32;
+  const int KP = (KMAX + 3) & ~3;
+  const int head = ((512 + ((nf * KP * 4 + 511) / 512) * 512 + 1023) / 1024) * 1024;
+  const int tile_bytes = nf * 256 * 4;
+  const int budget = (kmeans_tma_minb() == 2 ? 108 : 200) * 1024;
+  const int S = std::max(2, std::min(8, (budget - head) / tile_bytes));
+  return int64_t(head) + int64_t(S) * tile_bytes;
+}
+}  // namespace catt
+
+namespace {
+
 catt_status launch_kmeans_tma(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters,
                               int32_t k, int32_t* membership, const catt_throttle* t, void* stream) {
   if (k > 32 || nf > 256 || ld % 4 || (reinterpret_cast<uintptr_t>(feat) & 15u)) return CATT_EINVAL;
@@ -431,9 +420,8 @@ catt_status launch_kmeans_tma(const float* feat, int64_t ld, int64_t npoints, in
   const int KP = (KMAX + 3) & ~3;
   const int head = ((512 + ((nf * KP * 4 + 511) / 512) * 512 + 1023) / 1024) * 1024;
   const int minb = kmeans_tma_minb();
-  const int budget = (minb == 2 ? 108 : 200) * 1024;
-  const int S = std::max(2, std::min(8, (budget - head) / tile_bytes));
-  const size_t smem = size_t(head) + size_t(S) * tile_bytes;
+  const size_t smem = size_t(kmeans_tma_smem(nf, k));
+  const int S = int((int64_t(smem) - head) / tile_bytes);
   const void* f = minb == 2 ? kmeans_tma_fn<2>(k) : kmeans_tma_fn<1>(k);
   cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) {
@@ -486,17 +474,8 @@ extern "C" catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t
     if (dyn > 48 * 1024 && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn)) != cudaSuccess)
       return after_launch();
     KmArgs a{feat, clusters, membership, ld, npoints, nf, k, Throttle{}};
-    DevCtx* ctx = nullptr;
-    catt_status st = dev_ctx(&ctx);
-    if (st != CATT_OK) return st;
-    int per_sm = 0;
-    cudaError_t oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, 256, dyn);
-    if (oe != cudaSuccess || per_sm < 1) {
-      record_cuda_error(oe == cudaSuccess ? cudaErrorInvalidConfiguration : oe);
-      return CATT_ECUDA;
-    }
-    const int64_t groups = (npoints + 127) / 128;       // persistent: at most one wave of CTAs
-    const unsigned grid = unsigned(std::min<int64_t>((groups + 7) / 8, int64_t(per_sm) * ctx->hw.num_sms));
+    const int64_t groups = (npoints + 127) / 128;       // one group per warp
+    const unsigned grid = unsigned((groups + 7) / 8);
     void* args[] = {&a};
     cudaError_t e = cudaLaunchKernel(f, dim3(grid), dim3(256), args, dyn, static_cast<cudaStream_t>(stream));
     if (e != cudaSuccess) {

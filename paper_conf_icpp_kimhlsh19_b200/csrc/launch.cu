@@ -18,6 +18,7 @@ int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
 const void* syr2k_func(int variant);
 const void* kmeans_func(int variant, int nf);
+int64_t kmeans_tma_smem(int nf, int k);
 const void* kmeans_t_func(int variant);
 const void* corr_func(int variant);
 const void* gemm_func(int variant);
@@ -492,6 +493,8 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->n_loops = 1;
       out->trip[0] = nf;
       refs[n++] = mkref(1, 0, ld, 0, 4, 1, CATT_REF_NOT_L1);       // TMA tiles in shared memory
+      dyn = kmeans_tma_smem(int(nf), int(k));                       // centres + the tile ring (Eq 4 sizes the carveout)
+      out->grid[0] = std::min<int64_t>((np + 255) / 256, 2 * 148);  // persistent: at most 2 CTAs per SM
     } else if (var == CATT_VAR_COOP) {
       out->grid[0] = (np + 4 * threads - 1) / (4 * threads);       // a lane = 4 points
       out->extent[0] = (np + 3) / 4;
