@@ -118,14 +118,19 @@ typedef struct {
  * sizes per SM (ascending); l1d_bytes[i] the L1D capacity that option leaves
  * (measured on B200, see catt_hw_b200); carveout_pct[i] the
  * cudaFuncAttributePreferredSharedMemoryCarveout value that selects it.
- * min_warps_sm / divergent_lines are the B200 guards of union mode (0 = off;
- * DESIGN.md reading R18): a loop is throttled only if one of its reused
- * references touches >= divergent_lines lines per warp request, and never to
- * fewer than min_warps_sm active warps per SM. Paper mode ignores them. */
+ * min_warps_sm / divergent_lines / min_retouch / min_reuse_trip are the B200
+ * guards of union mode (0 = off; readings R18, R23): a loop is
+ * throttled only if one of its reused references touches >= divergent_lines
+ * lines per warp request, re-touches its line >= min_retouch times per thread
+ * (line / (|C_i| * elem_bytes), capped by the trip count; an outer-level reuse
+ * counts its trip count) and reuses in a loop of >= min_reuse_trip
+ * iterations; and never to fewer than min_warps_sm active warps per SM.
+ * Paper mode ignores them. */
 typedef struct {
   int32_t num_sms, max_warps_sm, max_ctas_sm, regs_sm, reg_alloc_unit, warp_size;
   int32_t smem_alloc_unit, reserved_smem_cta, line_bytes, n_carveouts;
   int32_t min_warps_sm, divergent_lines;
+  int32_t min_retouch, min_reuse_trip;
   int32_t carveout_kb[CATT_MAX_CARVEOUTS];
   int32_t carveout_pct[CATT_MAX_CARVEOUTS];
   int64_t l1d_bytes[CATT_MAX_CARVEOUTS];
@@ -430,6 +435,7 @@ int catt_last_cuda_error(void);
  * after the grid barrier, end) for CTAs < 1024. Copies the first n of the
  * 6144 u64 values (CTA-major) to host memory `out` (synchronous). */
 catt_status catt_fused_trace(uint64_t* out, int32_t n);
+/* ABI revision of this header: 2 (catt_hw gained min_retouch, min_reuse_trip). */
 int catt_abi_version(void);
 
 #ifdef __cplusplus

@@ -30,6 +30,9 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
       every (a, m) pair by active warps per SM descending, ties -> fewer CTAs
       of more warps (a per-SM cap is cheap on B200); none below min_warps_sm;
       if none at or above it fits, the most throttled one that respects it.
+      R23 adds two conditions on that divergent reference: it re-touches its
+      line >= min_retouch times per thread and its reuse loop runs >=
+      min_reuse_trip iterations (retouches(), reuse_trip()).
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -181,6 +184,24 @@ def has_locality(ref: Ref, trips: Sequence[int], line: int) -> bool:
     return any(abs(ref.c_iter[k]) * ref.elem_bytes < line and trips[k] >= 2 for k in range(len(trips)))
 
 
+def _reuse_levels(ref: Ref, trips: Sequence[int], line: int):
+    return [k for k in range(len(trips)) if abs(ref.c_iter[k]) * ref.elem_bytes < line and trips[k] >= 2]
+
+
+def retouches(ref: Ref, trips: Sequence[int], line: int) -> int:
+    """R23: how many times one thread touches a line of the reference before
+    leaving it: line / (|C_i| * e) consecutive iterations, capped by the trip
+    count; an outer-level reuse (C_i = 0) re-touches once per iteration of that
+    level. Maximum over the reuse levels (0 without reuse)."""
+    return max([trips[k] if ref.c_iter[k] == 0 else min(trips[k], line // (abs(ref.c_iter[k]) * ref.elem_bytes))
+                for k in _reuse_levels(ref, trips, line)] or [0])
+
+
+def reuse_trip(ref: Ref, trips: Sequence[int], line: int) -> int:
+    """R23: the longest trip count among the loops that carry the reuse."""
+    return max([trips[k] for k in _reuse_levels(ref, trips, line)] or [0])
+
+
 def _window(ref: Ref, trips: Sequence[int], line: int):
     """Iteration vectors whose lines the warp retains until the reuse, as a
     function of the phase k of the innermost loop (Eq 6; R10, R11).
@@ -271,8 +292,10 @@ class Model:
             per_ref = [len(_lines(r, gids00, it0, self.line)) for r in self.refs]
             self.lines_per_warp_iter = sum(per_ref)
             div = hw.get("divergent_lines", 0)
-            self.divergent = div <= 0 or any(
-                n >= div for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line))
+            rt, rtrip = hw.get("min_retouch", 0), hw.get("min_reuse_trip", 0)
+            self.divergent = (div <= 0 and rt <= 0 and rtrip <= 0) or any(
+                n >= div and retouches(r, loop.trips, self.line) >= rt and reuse_trip(r, loop.trips, self.line) >= rtrip
+                for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line))
             self.reuse_span = len(self.retained(0, 0, 0))
 
     def retained(self, b: int, w: int, k: int):
@@ -323,7 +346,8 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
 
     if M.fits(full) or not M.locality:
         return done(W, T, full, FIT_NONE_NEEDED)
-    guards = not M.paper and (hw.get("min_warps_sm", 0) > 0 or hw.get("divergent_lines", 0) > 0)
+    guards = not M.paper and any(hw.get(key, 0) > 0 for key in ("min_warps_sm", "divergent_lines", "min_retouch",
+                                                                  "min_reuse_trip"))
     if guards:
         # B200 rule (R18, R19): memory-divergent loops only; all (a, m) with a | W,
         # m <= T, by warps per SM descending, ties -> larger a (fewer CTAs);

@@ -61,12 +61,13 @@ class Hw(ctypes.Structure):
                 ("smem_alloc_unit", ctypes.c_int32), ("reserved_smem_cta", ctypes.c_int32),
                 ("line_bytes", ctypes.c_int32), ("n_carveouts", ctypes.c_int32),
                 ("min_warps_sm", ctypes.c_int32), ("divergent_lines", ctypes.c_int32),
+                ("min_retouch", ctypes.c_int32), ("min_reuse_trip", ctypes.c_int32),
                 ("carveout_kb", ctypes.c_int32 * MAX_CARVEOUTS), ("carveout_pct", ctypes.c_int32 * MAX_CARVEOUTS),
                 ("l1d_bytes", ctypes.c_int64 * MAX_CARVEOUTS)]
 
     def as_dict(self):
         n = self.n_carveouts
-        d = {f: getattr(self, f) for f, _ in self._fields_[:12]}
+        d = {f: getattr(self, f) for f, _ in self._fields_[:14]}
         d["carveout_kb"] = list(self.carveout_kb[:n])
         d["carveout_pct"] = list(self.carveout_pct[:n])
         d["l1d_bytes"] = list(self.l1d_bytes[:n])
@@ -75,7 +76,7 @@ class Hw(ctypes.Structure):
     @classmethod
     def from_dict(cls, d):
         h = cls()
-        for f, _ in cls._fields_[:12]:
+        for f, _ in cls._fields_[:14]:
             if f in d:
                 setattr(h, f, d[f])
         n = len(d["carveout_kb"])
@@ -219,6 +220,8 @@ def paper_rule(hw: Hw) -> Hw:
     h = Hw.from_dict(hw.as_dict())
     h.min_warps_sm = 0
     h.divergent_lines = 0
+    h.min_retouch = 0
+    h.min_reuse_trip = 0
     return h
 
 

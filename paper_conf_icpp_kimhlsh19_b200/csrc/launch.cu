@@ -631,4 +631,4 @@ extern "C" const char* catt_status_str(catt_status s) {
 }
 
 extern "C" int catt_last_cuda_error(void) { return g_last_err; }
-extern "C" int catt_abi_version(void) { return 1; }
+extern "C" int catt_abi_version(void) { return 2; }

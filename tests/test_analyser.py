@@ -24,14 +24,14 @@ def test_library_loads_and_exports_every_declared_symbol():
     assert declared == set(catt.catt.EXPORTED)
     for name in declared:
         assert hasattr(L, name), name
-    assert L.catt_abi_version() == 1
+    assert L.catt_abi_version() == 2
 
 
 def test_struct_layouts_match_header():
     # sizes of the C structs (x86-64 ABI) as the header defines them
     assert ctypes.sizeof(catt.Ref) == 3 * 8 + 4 * 8 + 8 + 4 * 4
     assert ctypes.sizeof(catt.Throttle) == 8 * 4 + 8
-    assert ctypes.sizeof(catt.Hw) == 12 * 4 + 16 * 4 * 2 + 16 * 8
+    assert ctypes.sizeof(catt.Hw) == 14 * 4 + 16 * 4 * 2 + 16 * 8
     assert ctypes.sizeof(catt.FootprintResult) == 6 * 8 + 6 * 4
 
 
@@ -90,6 +90,7 @@ def _rand_hw(rnd):
                 max_ctas_sm=rnd.choice([4, 8, 32]), regs_sm=65536, reg_alloc_unit=256, warp_size=32,
                 smem_alloc_unit=rnd.choice([128, 256]), reserved_smem_cta=rnd.choice([0, 1024]), line_bytes=128,
                 min_warps_sm=rnd.choice([0, 0, 4, 16]), divergent_lines=rnd.choice([0, 0, 2, 8]),
+                min_retouch=rnd.choice([0, 0, 4, 16]), min_reuse_trip=rnd.choice([0, 0, 8, 30]),
                 carveout_kb=carve, l1d_bytes=[rnd.randint(1, 200) * 128 for _ in carve])
 
 
@@ -226,7 +227,7 @@ def test_guards_do_not_touch_paper_mode():
     paper mode is the printed rule."""
     g = json.load(open(os.path.join(GOLDEN, "table3_paper_mode.json")))
     hw = catt.hw_titanv()
-    hw.min_warps_sm, hw.divergent_lines = 16, 8
+    hw.min_warps_sm, hw.divergent_lines, hw.min_retouch, hw.min_reuse_trip = 16, 8, 16, 128
     for c in g["cases"]:
         refs = [dict(c_gid=(ct, 0, 0), c_iter=(ci,), array_id=k) for k, (ct, ci) in enumerate(c["refs"])]
         d, keep = catt.make_desc(refs, (40960,), (c["block"], 1, 1), (c["grid"], 1, 1), mode=catt.MODE_PAPER,
@@ -259,3 +260,64 @@ def test_corr_gives_up_and_gemm_keeps_full_tlp():
         assert r["flags"] == catt.FIT_NONE_NEEDED | catt.FIT_GUARDED and t.active_warps == 0
         t, r = catt.plan(gemm, catt.Throttle(carveout_kb=carve, cta_threads=1024), b200)
         assert r["flags"] == catt.FIT_NONE_NEEDED
+
+
+def _thread_lines(ref, trips, line, gid=0):
+    """Line index sequence one thread walks (loops nested outer -> inner)."""
+    import itertools
+    seq = []
+    for it in itertools.product(*[range(t) for t in trips]):
+        idx = ref.base + ref.c_gid[0] * gid + sum(c * i for c, i in zip(ref.c_iter, it))
+        seq.append((idx * ref.elem_bytes) // line)
+    return seq
+
+
+@pytest.mark.parametrize("c_iter,e,trips,want", [((1,), 4, (100,), 32), ((4,), 4, (64,), 8), ((1,), 16, (40,), 8),
+                                                 ((2,), 8, (9,), 8), ((1,), 4, (20,), 20), ((33,), 4, (10,), 0),
+                                                 ((32,), 4, (10,), 0), ((0, 64), 4, (5, 34), 5),
+                                                 ((64, 1), 4, (3, 50), 32)])
+def test_retouches_and_reuse_trip_against_traces(c_iter, e, trips, want):
+    """R23 (retouches / reuse_trip) against brute force on the address trace
+    of one thread, line-aligned base: with reuse in the innermost loop, the
+    longest run of consecutive iterations on one line; with reuse only at an
+    outer level (C_i = 0, the inner loop leaves the line every iteration), the
+    number of visits of a line; and the trip count of the reuse loop."""
+    ref = fp.Ref(c_gid=(4096, 0, 0), c_iter=c_iter, base=0, elem_bytes=e)
+    seq = _thread_lines(ref, trips, 128)
+    inner_reuse = abs(c_iter[-1]) * e < 128 and trips[-1] >= 2
+    outer_reuse = len(trips) > 1 and c_iter[0] == 0 and trips[0] >= 2
+    if inner_reuse:
+        runs = best = 1
+        for a, b in zip(seq, seq[1:]):
+            runs = runs + 1 if a == b else 1
+            best = max(best, runs)
+        brute = best
+    elif outer_reuse:
+        brute = max(seq.count(x) for x in set(seq))
+    else:
+        brute = 0
+    assert brute == want
+    assert fp.retouches(ref, trips, 128) == want
+    levels = [k for k, c in enumerate(c_iter) if abs(c) * e < 128 and trips[k] >= 2]
+    assert fp.reuse_trip(ref, trips, 128) == (trips[levels[-1]] if levels else 0)
+
+
+def test_r23_guards_vec4_and_short_trip():
+    """R23 on the library's own loops (B200 table): the scalar row loop of BICG
+    at a contended launch is throttled; the same loop with 16-byte steps (8
+    re-touches per line) and the KM transpose (a 34-iteration reuse loop) are
+    not; with the R23 terms off both are throttled again (the R18 rule)."""
+    b200 = catt.hw_b200()
+    assert (b200.min_retouch, b200.min_reuse_trip) == (16, 128)
+    old = catt.Hw.from_dict(b200.as_dict())
+    old.min_retouch, old.min_reuse_trip = 0, 0
+    rows = catt.problem(catt.K_BICG_2, m=4096, n=4096)
+    tr = catt.problem(catt.K_KMEANS_T, m=494020, n=34, ld=494020)
+    launch = dict(cta_threads=1024, carveout_kb=196)
+    t, r = catt.plan(rows, catt.Throttle(variant="literal", **launch), b200)
+    assert t.active_warps and t.active_warps < r["base_warps"]
+    for prob, var in ((rows, "vec4"), (tr, "literal")):
+        t, r = catt.plan(prob, catt.Throttle(variant=var, **launch), b200)
+        assert r["flags"] == catt.FIT_NONE_NEEDED | catt.FIT_GUARDED and t.active_warps == 0 and t.active_ctas == 0
+        t, r = catt.plan(prob, catt.Throttle(variant=var, **launch), old)
+        assert t.active_warps or t.active_ctas

@@ -1,0 +1,129 @@
+"""Second held-out throttle study (after R23 was fixed): loops and launches
+used neither to fit R18/R19 nor to choose R23's thresholds. For each launch:
+every (a, m) of the literal loop, timed cold (L2 flushed: write + clean read),
+median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
+of the paper's rule are recorded BEFORE the timings (--predict prints them
+without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
+them. Writes gpurun_out/heldout2_study.json.
+usage: python tools/heldout2_study.py [--predict]"""
+import json
+import os
+import statistics
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_kimhlsh19_b200 as catt  # noqa: E402
+
+P = catt.problem
+CASES = [
+    # KM transpose (Rodinia invert_mapping) at other feature counts: trip 16 / 64 / 128 / 256
+    ("kmeans transpose nf=16", P(catt.K_KMEANS_T, m=262144, n=16, ld=262144), "literal", [(256, 16), (256, 228), (1024, 196)]),
+    ("kmeans transpose nf=64", P(catt.K_KMEANS_T, m=262144, n=64, ld=262144), "literal", [(256, 16), (256, 228), (1024, 196)]),
+    ("kmeans transpose nf=128", P(catt.K_KMEANS_T, m=262144, n=128, ld=262144), "literal", [(256, 16), (256, 228), (1024, 196)]),
+    ("kmeans transpose nf=256", P(catt.K_KMEANS_T, m=131072, n=256, ld=131072), "literal", [(256, 16), (1024, 196)]),
+    # VEC4 row loops (8 re-touches per line) at launches not studied before
+    ("mvt1 vec4", P(catt.K_MVT_1, n=4096), "vec4", [(1024, 228), (512, 196), (1024, 132)]),
+    ("gesummv vec4", P(catt.K_GESUMMV, n=8192), "vec4", [(1024, 196), (256, 228)]),
+    # scalar row loops with short rows: trip 96 (< 128) and 256
+    ("bicg2 literal n=96", P(catt.K_BICG_2, m=262144, n=96), "literal", [(1024, 196), (1024, 228), (256, 228)]),
+    ("bicg2 literal n=256", P(catt.K_BICG_2, m=131072, n=256), "literal", [(1024, 196), (1024, 228), (256, 228)]),
+]
+
+
+def picks(prob, var, cta, carve):
+    b200 = catt.hw_query() if catt_gpu() else catt.hw_b200()
+    r18 = catt.Hw.from_dict(b200.as_dict())
+    r18.min_retouch, r18.min_reuse_trip = 0, 0
+    out = {}
+    for name, hw in (("b200", b200), ("r18", r18), ("paper", catt.paper_rule(b200))):
+        launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var)
+        t, r = catt.plan(prob, launch, hw)
+        W, T = r["base_warps"], r["base_ctas"]
+        out[name] = [t.active_warps or W, t.active_ctas or T]
+        out["base"], out["carveout_kb"] = [W, T], r["carveout_kb"]
+        out["footprint"], out["l1d_lines"] = r["footprint_lines_full"], r["l1d_bytes"] // 128
+    return out
+
+
+def catt_gpu():
+    try:
+        import torch
+        return torch.cuda.is_available()
+    except Exception:
+        return False
+
+
+def main():
+    predict = "--predict" in sys.argv
+    if predict:
+        for name, prob, var, launches in CASES:
+            for cta, carve in launches:
+                print(name, cta, carve, picks(prob, var, cta, carve))
+        return
+    import torch
+    dev = torch.device("cuda")
+    flush_buf = torch.empty(64 * 1024 * 1024, dtype=torch.int32, device=dev)
+    clean_buf = torch.zeros(64 * 1024 * 1024, dtype=torch.int32, device=dev)
+
+    def med(fn, reps):
+        ts = []
+        for r in range(reps + 1):
+            flush_buf.zero_()
+            clean_buf.sum()
+            torch.cuda._sleep(400_000)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            torch.cuda.synchronize()
+            if r:
+                ts.append(a.elapsed_time(b))
+        return statistics.median(ts)
+
+    res = []
+    for name, prob, var, launches in CASES:
+        if prob.loop == catt.K_KMEANS_T:
+            npts, nf, ld = prob.m, prob.n, prob.ld
+            pm = torch.empty(npts * nf, device=dev)
+            catt.fill_hash(pm, 41)
+            fm = torch.empty(nf * ld, device=dev)
+            make = lambda th: (lambda: catt.kmeans_transpose(pm, npts, nf, fm, ld, t=th))
+        elif prob.loop == catt.K_GESUMMV:
+            n = prob.n
+            A = torch.empty(n, n, device=dev); catt.fill_hash(A, 5)
+            B = torch.empty(n, n, device=dev); catt.fill_hash(B, 105)
+            x = torch.empty(n, device=dev); catt.fill_hash(x, 205)
+            y, tmp = torch.empty(n, device=dev), torch.empty(n, device=dev)
+            make = lambda th: (lambda: catt.rows(A, x, y, catt.ROWS_GESUMMV, B=B, tmp=tmp, alpha=1.5, beta=1.2, t=th))
+        else:
+            m = prob.m if prob.loop == catt.K_BICG_2 else prob.n
+            n = prob.n
+            A = torch.empty(m, n, device=dev); catt.fill_hash(A, 2)
+            x = torch.empty(n, device=dev); catt.fill_hash(x, 102)
+            y = torch.empty(m, device=dev)
+            mode = catt.ROWS_ACCUM if prob.loop == catt.K_MVT_1 else catt.ROWS_STORE
+            make = lambda th: (lambda: catt.rows(A, x, y, mode, t=th))
+        for cta, carve in launches:
+            pk = picks(prob, var, cta, carve)
+            W, T = pk["base"]
+            launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var)
+            times = {}
+            for a in [d for d in range(W, 0, -1) if W % d == 0]:
+                for m in range(T, 0, -1):
+                    th = launch.copy(active_warps=a, active_ctas=m if m < T else 0)
+                    times[(a, m)] = med(make(th), 3)
+            best = min(times, key=times.get)
+            row = dict(loop=name, prob=dict(loop=prob.loop, m=prob.m, n=prob.n, k=prob.k, ld=prob.ld), variant=var,
+                       cta=cta, carveout_kb=carve, base=[W, T], footprint=pk["footprint"], l1d_lines=pk["l1d_lines"],
+                       b200=pk["b200"], r18=pk["r18"], paper=pk["paper"], best=list(best),
+                       best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
+                       **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3) for k in ("b200", "r18", "paper")},
+                       swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
+            print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
+            res.append(row)
+    os.makedirs("gpurun_out", exist_ok=True)
+    json.dump(res, open("gpurun_out/heldout2_study.json", "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,111 @@
+"""Re-plan every stored throttle sweep under a rule and score the pick.
+
+Each stored sweep row (profiles/**: bench.py throttle_study rows, held-out
+studies) has the time of every (a, m) at one launch. The problem of each loop
+name is rebuilt here, the analyser (catt_plan, no GPU) picks (a, m) under the
+rule, and the pick's time is divided by the best swept time.
+
+usage: python tools/rule_replay.py [--rule b200|r18|paper] [--set final|heldout|heldout2|all] [-v]
+  b200  = the library's B200 table (R18 + R19 + R23)
+  r18   = the same with the R23 terms off (the round-1 rule as fitted)
+  paper = guards off (the paper's Eq 9 as printed)
+"""
+import argparse
+import glob
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_kimhlsh19_b200 as catt  # noqa: E402
+
+P = catt.problem
+# loop name -> (problem, variant), for the files of each set
+LOOPS = {
+    ("final", "bicg2 q=A p (literal, row per thread)"): (P(catt.K_BICG_2, m=4096, n=4096), "literal"),
+    ("final", "gesummv (literal, row per thread)"): (P(catt.K_GESUMMV, n=8192), "literal"),
+    ("final", "kmeans assign (literal, feature-major)"): (P(catt.K_KMEANS, m=494020, n=34, k=5, ld=494020), "literal"),
+    ("final", "kmeans transpose (literal, point-major -> feature-major)"):
+        (P(catt.K_KMEANS_T, m=494020, n=34, ld=494020), "literal"),
+    ("final", "syrk (literal, 2-D block 32 x 8)"): (P(catt.K_SYRK, n=2048, k=2048), "literal"),
+    ("final", "syr2k (literal, 2-D block 32 x 8)"): (P(catt.K_SYR2K, n=2048, k=2048), "literal"),
+    ("final", "corr loop (literal, thread per column j1)"): (P(catt.K_CORR, n=2048, k=2048), "literal"),
+    ("final", "gemm (literal, 2-D block 32 x 8)"): (P(catt.K_GEMM, m=512, n=512, k=512), "literal"),
+    ("heldout", "syrk2048 literal"): (P(catt.K_SYRK, n=2048, k=2048), "literal"),
+    ("heldout", "mvt1 literal"): (P(catt.K_MVT_1, n=4096), "literal"),
+    ("heldout", "bicg2 vec4"): (P(catt.K_BICG_2, m=4096, n=4096), "vec4"),
+    ("heldout", "kmeans ld=494048"): (P(catt.K_KMEANS, m=494020, n=34, k=5, ld=494048), "literal"),
+}
+FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["profiles/r1/heldout_study.json"],
+         "heldout2": sorted(glob.glob("profiles/r1q/heldout2_study.json"))}
+ATAX = {"bench_atax.json": P(catt.K_ATAX_1, m=65536, n=16384), "bench_atax256.json": P(catt.K_ATAX_1, m=256, n=256)}
+
+
+def rows_of(f):
+    txt = open(f).read().strip()
+    d = json.loads(txt) if txt.startswith("[") else json.loads(txt.splitlines()[-1])
+    return d if isinstance(d, list) else (d.get("throttle_study") or [])
+
+
+def problem_of(s, f, r):
+    if "prob" in r:                                   # rows that carry their problem (heldout2 and later)
+        return P(r["prob"]["loop"], **{k: v for k, v in r["prob"].items() if k != "loop"}), r.get("variant", "literal")
+    if r["loop"].startswith("atax1"):
+        return ATAX[os.path.basename(f)], "literal"
+    return LOOPS[(s, r["loop"])]
+
+
+def rule_hw(name):
+    hw = catt.hw_b200()
+    if name == "r18":
+        hw.min_retouch, hw.min_reuse_trip = 0, 0
+    elif name == "paper":
+        hw = catt.paper_rule(hw)
+    return hw
+
+
+def replay(rule, sets, verbose):
+    hw = rule_hw(rule)
+    out = []
+    for s in sets:
+        for f in FILES[s]:
+            for r in rows_of(f):
+                if "swept" not in r:
+                    continue
+                prob, var = problem_of(s, f, r)
+                cta = r.get("cta_threads", r.get("cta"))
+                launch = catt.Throttle(cta_threads=cta, carveout_kb=r["carveout_kb"], variant=var)
+                t, res = catt.plan(prob, launch, hw)
+                W, T = res["base_warps"], res["base_ctas"]
+                if [W, T] != list(r["base"]):
+                    raise SystemExit(f"base mismatch {r['loop']} {cta} {r['carveout_kb']}: {W, T} vs {r['base']}")
+                sw = dict(r["swept"]) if isinstance(r["swept"], list) else r["swept"]
+                best = min(sw.values())
+                pick = (t.active_warps or W, t.active_ctas or T)
+                q = sw[f"{pick[0]},{pick[1]}"] / best
+                full = sw[f"{W},{T}"] / best
+                out.append((s, r["loop"], cta, r["carveout_kb"], pick, q, full))
+                if verbose:
+                    print(f"{s:8s} {r['loop'][:40]:40s} cta {cta:5d} carve {r['carveout_kb']:3d}  pick {pick}  "
+                          f"{q:.3f}x best  full {full:.3f}x")
+    return out
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--rule", default="b200", choices=["b200", "r18", "paper"])
+    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "all"])
+    ap.add_argument("-v", action="store_true")
+    a = ap.parse_args()
+    sets = ["final", "heldout", "heldout2"] if a.set == "all" else [a.set]
+    res = replay(a.rule, sets, a.v)
+    for s in sets:
+        rs = [x for x in res if x[0] == s]
+        if not rs:
+            continue
+        within = sum(1 for x in rs if x[5] <= 1.05)
+        contended = [x for x in rs if x[6] > 1.05]
+        beats = sum(1 for x in contended if x[5] < x[6] / 1.0)
+        print(f"[{a.rule}] {s}: {within}/{len(rs)} within 5% of best swept; worst {max(x[5] for x in rs):.3f}x; "
+              f"launches where some throttle beats full TLP by >5%: {len(contended)}, pick beats full TLP on "
+              f"{beats} of them")
