@@ -106,6 +106,7 @@ if __name__ == "__main__":
         within = sum(1 for x in rs if x[5] <= 1.05)
         contended = [x for x in rs if x[6] > 1.05]
         beats = sum(1 for x in contended if x[5] < x[6] / 1.0)
+        slower = sum(1 for x in rs if x[5] > 1.05 * x[6])
         print(f"[{a.rule}] {s}: {within}/{len(rs)} within 5% of best swept; worst {max(x[5] for x in rs):.3f}x; "
               f"launches where some throttle beats full TLP by >5%: {len(contended)}, pick beats full TLP on "
-              f"{beats} of them")
+              f"{beats} of them; pick >5% slower than full TLP on {slower}")
