@@ -32,7 +32,9 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
       if none at or above it fits, the most throttled one that respects it.
       R23 adds two conditions on that divergent reference: it re-touches its
       line >= min_retouch times per thread and its reuse loop runs >=
-      min_reuse_trip iterations (retouches(), reuse_trip()).
+      min_reuse_trip iterations (retouches(), reuse_trip()). R24: no throttle
+      when stores and loads without reuse exceed max_stream_pct % of a lane's
+      bytes per iteration.
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -293,9 +295,18 @@ class Model:
             self.lines_per_warp_iter = sum(per_ref)
             div = hw.get("divergent_lines", 0)
             rt, rtrip = hw.get("min_retouch", 0), hw.get("min_reuse_trip", 0)
-            self.divergent = (div <= 0 and rt <= 0 and rtrip <= 0) or any(
+            self.divergent = (div <= 0 and rt <= 0 and rtrip <= 0 and hw.get("max_stream_pct", 0) <= 0) or any(
                 n >= div and retouches(r, loop.trips, self.line) >= rt and reuse_trip(r, loop.trips, self.line) >= rtrip
                 for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line))
+            # R24: bytes per lane and iteration of streams L1 cannot serve again
+            pct = hw.get("max_stream_pct", 0)
+            if pct > 0:
+                mem = [r for r in loop.refs if not (r.flags & REF_NOT_L1)]
+                total = sum(r.elem_bytes for r in mem)
+                stream = sum(r.elem_bytes for r in mem
+                             if (r.flags & REF_STORE) or not has_locality(r, loop.trips, self.line))
+                if 100 * stream > pct * total:
+                    self.divergent = False
             self.reuse_span = len(self.retained(0, 0, 0))
 
     def retained(self, b: int, w: int, k: int):
@@ -347,7 +358,7 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
     if M.fits(full) or not M.locality:
         return done(W, T, full, FIT_NONE_NEEDED)
     guards = not M.paper and any(hw.get(key, 0) > 0 for key in ("min_warps_sm", "divergent_lines", "min_retouch",
-                                                                  "min_reuse_trip"))
+                                                                  "min_reuse_trip", "max_stream_pct"))
     if guards:
         # B200 rule (R18, R19): memory-divergent loops only; all (a, m) with a | W,
         # m <= T, by warps per SM descending, ties -> larger a (fewer CTAs);

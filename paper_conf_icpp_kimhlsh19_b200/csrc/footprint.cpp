@@ -224,7 +224,7 @@ class Model {
     // (>= divergent_lines lines per warp request), re-touches its line often
     // enough (>= min_retouch times per thread) and keeps reusing for long
     // enough (a reuse loop of >= min_reuse_trip iterations)
-    divergent_ = hw_.divergent_lines <= 0 && hw_.min_retouch <= 0 && hw_.min_reuse_trip <= 0;
+    divergent_ = hw_.divergent_lines <= 0 && hw_.min_retouch <= 0 && hw_.min_reuse_trip <= 0 && hw_.max_stream_pct <= 0;
     for (const catt_ref& r : refs_) {
       std::unordered_set<uint64_t> s;
       add_lines(r, g00, it0, d_.n_loops, line_, &s);
@@ -242,6 +242,22 @@ class Model {
       if (reuse && int64_t(s.size()) >= hw_.divergent_lines && retouch >= hw_.min_retouch &&
           rtrip >= hw_.min_reuse_trip)
         divergent_ = true;
+    }
+    // R24: no throttle when more than max_stream_pct % of a lane's bytes per
+    // iteration belong to streams L1 cannot serve again (stores, loads
+    // without reuse): those need the memory-level parallelism a throttle removes
+    if (hw_.max_stream_pct > 0) {
+      int64_t total = 0, stream = 0;
+      for (int i = 0; i < d_.n_refs; ++i) {
+        const catt_ref& r = d_.refs[i];
+        if (r.flags & CATT_REF_NOT_L1) continue;
+        total += r.elem_bytes;
+        bool reuse = false;
+        for (int k = 0; k < d_.n_loops; ++k)
+          if (iabs(r.c_iter[k]) * r.elem_bytes < line_ && d_.trip[k] >= 2) reuse = true;
+        if ((r.flags & CATT_REF_STORE) || !reuse) stream += r.elem_bytes;
+      }
+      if (100 * stream > int64_t(hw_.max_stream_pct) * total) divergent_ = false;
     }
     reuse_span_ = int64_t(retained(0, 0, 0).size());
     return CATT_OK;
@@ -331,7 +347,8 @@ catt_status validate(const catt_loop_desc* d, const catt_hw* hw) {
   if (hw->warp_size != 32 || hw->num_sms < 1 || hw->max_warps_sm < 1 || hw->max_ctas_sm < 1) return CATT_EINVAL;
   if (hw->line_bytes < 4 || hw->n_carveouts < 1 || hw->n_carveouts > CATT_MAX_CARVEOUTS) return CATT_EINVAL;
   if (hw->smem_alloc_unit < 1 || hw->reg_alloc_unit < 1 || hw->regs_sm < 1) return CATT_EINVAL;
-  if (hw->min_warps_sm < 0 || hw->divergent_lines < 0 || hw->min_retouch < 0 || hw->min_reuse_trip < 0)
+  if (hw->min_warps_sm < 0 || hw->divergent_lines < 0 || hw->min_retouch < 0 || hw->min_reuse_trip < 0 ||
+      hw->max_stream_pct < 0 || hw->max_stream_pct > 100)
     return CATT_EINVAL;
   for (int i = 1; i < hw->n_carveouts; ++i)
     if (hw->carveout_kb[i] <= hw->carveout_kb[i - 1]) return CATT_EINVAL;
@@ -373,7 +390,8 @@ extern "C" catt_status catt_footprint(const catt_loop_desc* desc, const catt_hw*
   if (M.fits(full) || !M.locality_) return done(W, T, full, CATT_FIT_NONE_NEEDED);
   const bool paper = desc->mode == CATT_MODE_PAPER;
   const bool guards =
-      !paper && (hw->min_warps_sm > 0 || hw->divergent_lines > 0 || hw->min_retouch > 0 || hw->min_reuse_trip > 0);
+      !paper && (hw->min_warps_sm > 0 || hw->divergent_lines > 0 || hw->min_retouch > 0 || hw->min_reuse_trip > 0 ||
+                 hw->max_stream_pct > 0);
   if (guards) {
     // B200 rule (R18, R19): only memory-divergent loops; every (a, m) pair
     // with a | W, m <= T, by active warps per SM descending, ties -> fewer
@@ -460,12 +478,15 @@ extern "C" catt_status catt_hw_b200(catt_hw* out) {
   out->min_warps_sm = 8;
   out->divergent_lines = 8;
   // R23 (round 1, after the final pass): a throttle must be paid for by
-  // enough reuse. A thread re-touches its line >= 16 times (VEC4's 16-byte
-  // steps give 8: full TLP measured 1.23x faster than the guarded pick) and
-  // the reuse loop runs >= 128 iterations (the KM transpose's 34-iteration
-  // feature loop: full TLP 1.26-1.31x faster than the floor pick).
+  // enough reuse: a thread re-touches its line >= 16 times (VEC4's 16-byte
+  // steps give 8: full TLP measured 1.23x faster than the guarded pick).
+  // R23's reuse-trip term (>= 128 iterations) is off since R24: held-out
+  // study 2 (profiles/r1q/) showed short scalar rows (96 iterations) gain
+  // 1.3x from a throttle while the KM transpose loses at every trip count
+  // (16 .. 256); what sets the transpose apart is its store stream (R24).
   out->min_retouch = 16;
-  out->min_reuse_trip = 128;
+  out->min_reuse_trip = 0;
+  out->max_stream_pct = 25;
   // Shared-memory options (KB) and the carveout percentage that selects each
   // (percent of the 228 KB maximum; the driver rounds up to the next option).
   // L1D capacity per option, measured on B200 by the Fig 3-style sweep

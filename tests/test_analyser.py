@@ -31,7 +31,7 @@ def test_struct_layouts_match_header():
     # sizes of the C structs (x86-64 ABI) as the header defines them
     assert ctypes.sizeof(catt.Ref) == 3 * 8 + 4 * 8 + 8 + 4 * 4
     assert ctypes.sizeof(catt.Throttle) == 8 * 4 + 8
-    assert ctypes.sizeof(catt.Hw) == 14 * 4 + 16 * 4 * 2 + 16 * 8
+    assert ctypes.sizeof(catt.Hw) == 16 * 4 + 16 * 4 * 2 + 16 * 8
     assert ctypes.sizeof(catt.FootprintResult) == 6 * 8 + 6 * 4
 
 
@@ -91,6 +91,7 @@ def _rand_hw(rnd):
                 smem_alloc_unit=rnd.choice([128, 256]), reserved_smem_cta=rnd.choice([0, 1024]), line_bytes=128,
                 min_warps_sm=rnd.choice([0, 0, 4, 16]), divergent_lines=rnd.choice([0, 0, 2, 8]),
                 min_retouch=rnd.choice([0, 0, 4, 16]), min_reuse_trip=rnd.choice([0, 0, 8, 30]),
+                max_stream_pct=rnd.choice([0, 0, 25, 60]),
                 carveout_kb=carve, l1d_bytes=[rnd.randint(1, 200) * 128 for _ in carve])
 
 
@@ -302,15 +303,19 @@ def test_retouches_and_reuse_trip_against_traces(c_iter, e, trips, want):
     assert fp.reuse_trip(ref, trips, 128) == (trips[levels[-1]] if levels else 0)
 
 
-def test_r23_guards_vec4_and_short_trip():
-    """R23 on the library's own loops (B200 table): the scalar row loop of BICG
-    at a contended launch is throttled; the same loop with 16-byte steps (8
-    re-touches per line) and the KM transpose (a 34-iteration reuse loop) are
-    not; with the R23 terms off both are throttled again (the R18 rule)."""
+def test_r23_r24_guard_vec4_and_store_stream():
+    """R23/R24 on the library's own loops (B200 table): the scalar row loop of
+    BICG at a contended launch is throttled, also with 96-element rows; the
+    same loop with 16-byte steps (8 re-touches per line, R23) and the KM
+    transpose (half of its bytes are the store stream out[f*ld + p], R24) are
+    not; with both terms off both are throttled again (the R18 rule)."""
     b200 = catt.hw_b200()
-    assert (b200.min_retouch, b200.min_reuse_trip) == (16, 128)
+    assert (b200.min_retouch, b200.min_reuse_trip, b200.max_stream_pct) == (16, 0, 25)
     old = catt.Hw.from_dict(b200.as_dict())
-    old.min_retouch, old.min_reuse_trip = 0, 0
+    old.min_retouch, old.min_reuse_trip, old.max_stream_pct = 0, 0, 0
+    t, r = catt.plan(catt.problem(catt.K_BICG_2, m=262144, n=96), catt.Throttle(cta_threads=1024, carveout_kb=196),
+                     b200)
+    assert t.active_warps or t.active_ctas
     rows = catt.problem(catt.K_BICG_2, m=4096, n=4096)
     tr = catt.problem(catt.K_KMEANS_T, m=494020, n=34, ld=494020)
     launch = dict(cta_threads=1024, carveout_kb=196)
@@ -321,3 +326,30 @@ def test_r23_guards_vec4_and_short_trip():
         assert r["flags"] == catt.FIT_NONE_NEEDED | catt.FIT_GUARDED and t.active_warps == 0 and t.active_ctas == 0
         t, r = catt.plan(prob, catt.Throttle(variant=var, **launch), old)
         assert t.active_warps or t.active_ctas
+
+
+def test_r24_stream_fraction_on_synthetic_loops():
+    """R24 against its definition on hand-made loops: a divergent reused load
+    plus a coalesced store of the same width is 50 % stream (guarded at 25 %,
+    throttled at 60 %); adding a second reused load makes it 33 %; a NOT_L1
+    store does not count."""
+    hw = catt.hw_b200()
+    hw.max_stream_pct = 25
+    loose = catt.Hw.from_dict(hw.as_dict())
+    loose.max_stream_pct = 60
+
+    def plan(refs, h):
+        d, keep = catt.make_desc(refs, (4096,), (256, 1, 1), (4096, 1, 1), force_carveout_kb=228)
+        return catt.footprint(d, h)
+
+    load = dict(c_gid=(4096, 0, 0), c_iter=(1,), array_id=0)
+    store = dict(c_gid=(1, 0, 0), c_iter=(65536,), array_id=1, flags=catt.REF_STORE)
+    load2 = dict(c_gid=(4096, 0, 0), c_iter=(1,), array_id=2)
+    r = plan([load, store], hw)
+    assert r["flags"] & catt.FIT_GUARDED and r["active_warps"] == r["base_warps"]
+    r = plan([load, store], loose)
+    assert r["active_warps"] * r["active_ctas"] < r["base_warps"] * r["base_ctas"]     # throttled
+    r = plan([load, load2, store], hw)
+    assert r["flags"] & catt.FIT_GUARDED                      # 33 % > 25 %
+    r = plan([load, load2, dict(store, flags=catt.REF_STORE | catt.REF_NOT_L1)], hw)
+    assert r["active_warps"] * r["active_ctas"] < r["base_warps"] * r["base_ctas"]

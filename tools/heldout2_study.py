@@ -5,7 +5,7 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict]"""
+usage: python tools/heldout2_study.py [--predict] [--set3]   (--set3: the third held-out set, after R24)"""
 import json
 import os
 import statistics
@@ -29,13 +29,27 @@ CASES = [
     ("bicg2 literal n=256", P(catt.K_BICG_2, m=131072, n=256), "literal", [(1024, 196), (1024, 228), (256, 228)]),
 ]
 
+# Third held-out set (after R24 was fixed on the second): new shapes and launches
+CASES3 = [
+    ("kmeans transpose nf=34 512thr", P(catt.K_KMEANS_T, m=494020, n=34, ld=494020), "literal", [(512, 16), (512, 196)]),
+    ("kmeans transpose nf=96", P(catt.K_KMEANS_T, m=262144, n=96, ld=262144), "literal", [(256, 100), (512, 228)]),
+    ("atax1 literal n=192", P(catt.K_ATAX_1, m=131072, n=192), "literal", [(1024, 196), (512, 228)]),
+    ("mvt1 literal n=2048", P(catt.K_MVT_1, n=2048), "literal", [(512, 196), (1024, 228)]),
+    ("bicg2 literal n=512", P(catt.K_BICG_2, m=65536, n=512), "literal", [(512, 228), (1024, 132)]),
+    ("bicg2 vec4 n=96", P(catt.K_BICG_2, m=262144, n=96), "vec4", [(1024, 196)]),
+    ("syr2k literal 1024", P(catt.K_SYR2K, n=1024, k=1024), "literal", [(512, 196), (128, 228)]),
+    ("syrk literal 1024", P(catt.K_SYRK, n=1024, k=1024), "literal", [(512, 228), (128, 164)]),
+]
+
 
 def picks(prob, var, cta, carve):
     b200 = catt.hw_query() if catt_gpu() else catt.hw_b200()
     r18 = catt.Hw.from_dict(b200.as_dict())
-    r18.min_retouch, r18.min_reuse_trip = 0, 0
+    r18.min_retouch, r18.min_reuse_trip, r18.max_stream_pct = 0, 0, 0
+    r23 = catt.Hw.from_dict(r18.as_dict())
+    r23.min_retouch, r23.min_reuse_trip = 16, 128
     out = {}
-    for name, hw in (("b200", b200), ("r18", r18), ("paper", catt.paper_rule(b200))):
+    for name, hw in (("b200", b200), ("r23", r23), ("r18", r18), ("paper", catt.paper_rule(b200))):
         launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var)
         t, r = catt.plan(prob, launch, hw)
         W, T = r["base_warps"], r["base_ctas"]
@@ -55,8 +69,10 @@ def catt_gpu():
 
 def main():
     predict = "--predict" in sys.argv
+    third = "--set3" in sys.argv
+    cases = CASES3 if third else CASES
     if predict:
-        for name, prob, var, launches in CASES:
+        for name, prob, var, launches in cases:
             for cta, carve in launches:
                 print(name, cta, carve, picks(prob, var, cta, carve))
         return
@@ -81,13 +97,22 @@ def main():
         return statistics.median(ts)
 
     res = []
-    for name, prob, var, launches in CASES:
+    for name, prob, var, launches in cases:
         if prob.loop == catt.K_KMEANS_T:
             npts, nf, ld = prob.m, prob.n, prob.ld
             pm = torch.empty(npts * nf, device=dev)
             catt.fill_hash(pm, 41)
             fm = torch.empty(nf * ld, device=dev)
             make = lambda th: (lambda: catt.kmeans_transpose(pm, npts, nf, fm, ld, t=th))
+        elif prob.loop in (catt.K_SYRK, catt.K_SYR2K):
+            n = prob.n
+            A = torch.empty(n, n, device=dev); catt.fill_hash(A, 6)
+            B2 = torch.empty(n, n, device=dev); catt.fill_hash(B2, 8)
+            C = torch.empty(n, n, device=dev); catt.fill_hash(C, 106)
+            if prob.loop == catt.K_SYRK:
+                make = lambda th: (lambda: catt.syrk(A, C, 1.5, 1.2, t=th))
+            else:
+                make = lambda th: (lambda: catt.syr2k(A, B2, C, 1.5, 1.2, t=th))
         elif prob.loop == catt.K_GESUMMV:
             n = prob.n
             A = torch.empty(n, n, device=dev); catt.fill_hash(A, 5)
@@ -96,7 +121,7 @@ def main():
             y, tmp = torch.empty(n, device=dev), torch.empty(n, device=dev)
             make = lambda th: (lambda: catt.rows(A, x, y, catt.ROWS_GESUMMV, B=B, tmp=tmp, alpha=1.5, beta=1.2, t=th))
         else:
-            m = prob.m if prob.loop == catt.K_BICG_2 else prob.n
+            m = prob.m if prob.loop in (catt.K_BICG_2, catt.K_ATAX_1) else prob.n
             n = prob.n
             A = torch.empty(m, n, device=dev); catt.fill_hash(A, 2)
             x = torch.empty(n, device=dev); catt.fill_hash(x, 102)
@@ -115,14 +140,15 @@ def main():
             best = min(times, key=times.get)
             row = dict(loop=name, prob=dict(loop=prob.loop, m=prob.m, n=prob.n, k=prob.k, ld=prob.ld), variant=var,
                        cta=cta, carveout_kb=carve, base=[W, T], footprint=pk["footprint"], l1d_lines=pk["l1d_lines"],
-                       b200=pk["b200"], r18=pk["r18"], paper=pk["paper"], best=list(best),
+                       b200=pk["b200"], r23=pk["r23"], r18=pk["r18"], paper=pk["paper"], best=list(best),
                        best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
-                       **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3) for k in ("b200", "r18", "paper")},
+                       **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3)
+                          for k in ("b200", "r23", "r18", "paper")},
                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    json.dump(res, open("gpurun_out/heldout2_study.json", "w"), indent=1)
+    json.dump(res, open("gpurun_out/heldout3_study.json" if third else "gpurun_out/heldout2_study.json", "w"), indent=1)
 
 
 if __name__ == "__main__":

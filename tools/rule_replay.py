@@ -5,9 +5,10 @@ studies) has the time of every (a, m) at one launch. The problem of each loop
 name is rebuilt here, the analyser (catt_plan, no GPU) picks (a, m) under the
 rule, and the pick's time is divided by the best swept time.
 
-usage: python tools/rule_replay.py [--rule b200|r18|paper] [--set final|heldout|heldout2|all] [-v]
-  b200  = the library's B200 table (R18 + R19 + R23)
-  r18   = the same with the R23 terms off (the round-1 rule as fitted)
+usage: python tools/rule_replay.py [--rule b200|r23|r18|paper] [--set final|heldout|heldout2|heldout3|all] [-v]
+  b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24)
+  r23   = R18 + R19 + R23 (re-touch and reuse-trip terms), as held-out study 2 tested it
+  r18   = the new terms off (the round-1 rule as fitted)
   paper = guards off (the paper's Eq 9 as printed)
 """
 import argparse
@@ -37,7 +38,8 @@ LOOPS = {
     ("heldout", "kmeans ld=494048"): (P(catt.K_KMEANS, m=494020, n=34, k=5, ld=494048), "literal"),
 }
 FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["profiles/r1/heldout_study.json"],
-         "heldout2": sorted(glob.glob("profiles/r1q/heldout2_study.json"))}
+         "heldout2": sorted(glob.glob("profiles/r1q/heldout2_study.json")),
+         "heldout3": sorted(glob.glob("profiles/r1q/heldout3_study.json"))}
 ATAX = {"bench_atax.json": P(catt.K_ATAX_1, m=65536, n=16384), "bench_atax256.json": P(catt.K_ATAX_1, m=256, n=256)}
 
 
@@ -58,7 +60,9 @@ def problem_of(s, f, r):
 def rule_hw(name):
     hw = catt.hw_b200()
     if name == "r18":
-        hw.min_retouch, hw.min_reuse_trip = 0, 0
+        hw.min_retouch, hw.min_reuse_trip, hw.max_stream_pct = 0, 0, 0
+    elif name == "r23":                        # as pre-registered for held-out study 2
+        hw.min_retouch, hw.min_reuse_trip, hw.max_stream_pct = 16, 128, 0
     elif name == "paper":
         hw = catt.paper_rule(hw)
     return hw
@@ -93,11 +97,11 @@ def replay(rule, sets, verbose):
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("--rule", default="b200", choices=["b200", "r18", "paper"])
-    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "all"])
+    ap.add_argument("--rule", default="b200", choices=["b200", "r23", "r18", "paper"])
+    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
-    sets = ["final", "heldout", "heldout2"] if a.set == "all" else [a.set]
+    sets = ["final", "heldout", "heldout2", "heldout3"] if a.set == "all" else [a.set]
     res = replay(a.rule, sets, a.v)
     for s in sets:
         rs = [x for x in res if x[0] == s]
