@@ -7,7 +7,9 @@
 namespace catt {
 
 __device__ __forceinline__ uint64_t f2_pack(float lo, float hi) {
-  return uint64_t(__float_as_uint(lo)) | (uint64_t(__float_as_uint(hi)) << 32);
+  uint64_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
 }
 __device__ __forceinline__ float f2_lo(uint64_t v) { return __uint_as_float(unsigned(v)); }
 __device__ __forceinline__ float f2_hi(uint64_t v) { return __uint_as_float(unsigned(v >> 32)); }
@@ -15,6 +17,18 @@ __device__ __forceinline__ float f2_hi(uint64_t v) { return __uint_as_float(unsi
 __device__ __forceinline__ uint64_t f2_sub(uint64_t a, uint64_t b) {
   uint64_t d;
   asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+// a + b per half
+__device__ __forceinline__ uint64_t f2_add(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+// a * b per half
+__device__ __forceinline__ uint64_t f2_mul(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
   return d;
 }
 // fmaf(a, b, c) per half

@@ -14,6 +14,7 @@
 #include <cstdlib>
 #include <cstdint>
 
+#include "f32x2.cuh"
 #include "internal.h"
 
 namespace catt {
@@ -249,16 +250,30 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
       }
     }
   };
+  // the accumulators as packed pairs (c[r][2p], c[r][2p+1]): one FFMA2 (SYR2K:
+  // FMUL2 + FFMA2 + FADD2) advances two outputs; the row operand is a
+  // broadcast (ptxas folds it into the .F32 operand form), and each half is
+  // the scalar IEEE operation, so the result stays bit-identical
+  uint64_t cp[TM][TM / 2];
+#pragma unroll
+  for (int r = 0; r < TM; ++r)
+#pragma unroll
+    for (int p = 0; p < TM / 2; ++p) cp[r][p] = f2_pack(c[r][2 * p], c[r][2 * p + 1]);
   auto fma_step = [&](int fb) {
 #pragma unroll
-    for (int r = 0; r < TM; ++r)
+    for (int r = 0; r < TM; ++r) {
+      const uint64_t ar = f2_pack(f[fb][0][r], f[fb][0][r]);
 #pragma unroll
-      for (int q = 0; q < TM; ++q) {
-        if constexpr (TWO)
-          c[r][q] = __fadd_rn(c[r][q], fmaf(f[fb][0][r], f[fb][1][q], __fmul_rn(f[fb][2][r], f[fb][3][q])));
-        else
-          c[r][q] = fmaf(f[fb][0][r], f[fb][1][q], c[r][q]);
+      for (int p = 0; p < TM / 2; ++p) {
+        const uint64_t bq = f2_pack(f[fb][1][2 * p], f[fb][1][2 * p + 1]);
+        if constexpr (TWO) {
+          const uint64_t pr = f2_mul(f2_pack(f[fb][2][r], f[fb][2][r]), f2_pack(f[fb][3][2 * p], f[fb][3][2 * p + 1]));
+          cp[r][p] = f2_add(cp[r][p], f2_fma(ar, bq, pr));
+        } else {
+          cp[r][p] = f2_fma(ar, bq, cp[r][p]);
+        }
       }
+    }
   };
 
   const int64_t ktiles = (m + BK - 1) / BK;
@@ -299,6 +314,13 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
   }
 
 #pragma unroll
+  for (int r = 0; r < TM; ++r)
+#pragma unroll
+    for (int p = 0; p < TM / 2; ++p) {
+      c[r][2 * p] = f2_lo(cp[r][p]);
+      c[r][2 * p + 1] = f2_hi(cp[r][p]);
+    }
+#pragma unroll
   for (int r = 0; r < TM; ++r) {
     const int64_t gi = i0 + tile_off(ty, r);
     if (gi >= ni) continue;
@@ -330,11 +352,11 @@ static int tiled_minb(bool two) {
   (void)two;
 }
 
-// LEAN large tiles (BK = 8, single-buffered fragments, 2 CTAs per SM) for
-// SYRK when there are more active tiles than SMs: the SMs that get two tiles
-// run them concurrently (SYRK 2048: 0.497 -> 0.460 ms). With at most one tile
-// per SM the regular kernel is faster (CORR's upper tiles: 136 < 148).
-// CATT_TILED_LEAN=0 turns it off (tools only).
+// LEAN large tiles (BK = 8, single-buffered fragments, 2 CTAs per SM): with
+// scalar FFMA they beat one CTA per SM when tiles outnumber SMs (SYRK 2048:
+// 0.497 -> 0.460 ms); since the inner product runs as FFMA2 the regular
+// kernel is faster (0.441 ms; LEAN 0.466 ms, 44 bytes of spills at 128
+// registers), so LEAN is off unless CATT_TILED_LEAN=1 (tools only).
 static bool tiled_lean(int64_t active_tiles) {
   static const int env = [] {
     const char* e = getenv("CATT_TILED_LEAN");
@@ -345,7 +367,7 @@ static bool tiled_lean(int64_t active_tiles) {
     if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
     return v;
   }();
-  if (env == 0) return false;
+  if (env != 1) return false;
   return active_tiles > nsm;
 }
 
@@ -364,6 +386,11 @@ static bool small_tiles(int64_t ni, int64_t nj) {
     if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
     return v;
   }();
+  static const int force = [] {
+    const char* e = getenv("CATT_TILED_SMALL");  // 0 / 1: force the tile size (tools only)
+    return e ? atoi(e) : -1;
+  }();
+  if (force == 0 || force == 1) return force == 1;
   return ((ni + 127) / 128) * ((nj + 127) / 128) < nsm;
 }
 
