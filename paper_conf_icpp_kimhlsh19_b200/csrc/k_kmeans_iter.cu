@@ -24,6 +24,7 @@
 #include <cstdint>
 #include <cstring>
 
+#include "f32x2.cuh"
 #include "internal.h"
 #include "tma.cuh"
 
@@ -230,21 +231,25 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
     int c = -1, rank = 0, changed = 0;
     if (p < a.npoints) {
       const float* f0 = a.feat + p;
-      float d[KMAX];
+      // partial distances as packed pairs of centres (d[2p], d[2p+1]): one
+      // FADD2 + one FFMA2 per pair, the point's value broadcast; each half is
+      // the scalar IEEE operation (same order, bit-identical decisions)
+      constexpr int KH = (KMAX + 1) / 2;
+      uint64_t dp[KH];
 #pragma unroll
-      for (int cc = 0; cc < KMAX; ++cc) d[cc] = 0.0f;
+      for (int h = 0; h < KH; ++h) dp[h] = 0ull;
       auto feature = [&](int f, float v) {
         tile[f * KTP + t] = v;
         const float4* cf = reinterpret_cast<const float4*>(s_ct + f * KP);
+        const uint64_t vv = f2_pack(v, v);
 #pragma unroll
         for (int q = 0; q < KP / 4; ++q) {
           const float4 c4 = cf[q];
-          const float cv[4] = {c4.x, c4.y, c4.z, c4.w};
 #pragma unroll
-          for (int j = 0; j < 4; ++j)
+          for (int j = 0; j < 4; j += 2)
             if (4 * q + j < KMAX) {
-              const float diff = v - cv[j];
-              d[4 * q + j] = fmaf(diff, diff, d[4 * q + j]);
+              const uint64_t e = f2_sub(vv, j == 0 ? f2_pack(c4.x, c4.y) : f2_pack(c4.z, c4.w));
+              dp[(4 * q + j) / 2] = f2_fma(e, e, dp[(4 * q + j) / 2]);
             }
         }
       };
@@ -273,11 +278,13 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
       }
       float best = FLT_MAX;
 #pragma unroll
-      for (int cc = 0; cc < KMAX; ++cc)
-        if (d[cc] < best) {
-          best = d[cc];
+      for (int cc = 0; cc < KMAX; ++cc) {
+        const float dc = (cc & 1) ? f2_hi(dp[cc / 2]) : f2_lo(dp[cc / 2]);
+        if (dc < best) {
+          best = dc;
           c = cc;
         }
+      }
       changed = old != c;  // c = -1: every distance NaN or >= FLT_MAX (as catt_kmeans_assign)
       a.memb[p] = c;
       if (c >= 0) rank = atomicAdd(&s_cnt[c], 1);

@@ -378,8 +378,12 @@ def test_kmeans_rodinia_shape_full():
         memb_o, _ = oracle.kmeans_assign(fh, ld, npts, nf, clusters)
         hw = catt.hw_query()
         t, r = catt.plan(catt.problem(catt.K_KMEANS, m=npts, n=nf, k=k, ld=ld), catt.Throttle(), hw)
+        # the bench's launch: STAGED planned by CATT (Eq 4 -> the 228 KB carveout, 2 CTAs per SM)
+        tb, _ = catt.plan(catt.problem(catt.K_KMEANS, m=npts, n=nf, k=k, ld=ld),
+                          catt.Throttle(cta_threads=256, variant="staged"), hw)
+        assert tb.carveout_kb == 228
         for tt in (catt.Throttle(), t, catt.Throttle(variant="regs"), catt.Throttle(variant="staged"),
-                   catt.Throttle(variant="coop")):
+                   catt.Throttle(variant="coop"), tb):
             memb = catt.kmeans_assign(feat, ld, npts, nf, dev(clusters), t=tt)
             assert np.array_equal(host(memb), memb_o)
 
