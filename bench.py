@@ -564,6 +564,15 @@ class Atax(Workload):
         mat = rows * n * 4
         self.study = dict(name="atax1 tmp=A x (literal, row per thread)", prob=catt.problem(catt.K_ATAX_1, m=rows, n=n),
                           A=self.A, x=self.x, y=self.tmp, launches=[(1024, 196), (256, 228)])
+        if var == "fused_peer":
+            # the A^T partials all-reduced inside the fused kernel through peer
+            # memory: no NCCL call, one launch per step
+            from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+            self.peer = cdist.peer_setup(n)
+            self.loops = [Loop("atax fused + peer all-reduce",
+                               lambda: cdist.atax_rowshard_peer(self.A, self.x, self.peer, self.tmp, self.y),
+                               mat + 4 * 2 * (rows + n), "fused")]
+            return
         if var == "fused":
             tf = self.plan("atax fused", catt.problem(catt.K_ATAX_1, m=rows, n=n), catt.Throttle(variant="fused"))
             self.loops = [Loop("atax fused", lambda: catt.dual(self.A, self.x, self.tmp, self.y, dependent=True, t=tf),
@@ -580,7 +589,7 @@ class Atax(Workload):
                            mat + 4 * (rows + n), "cols")]
 
     def collective(self):
-        if self.world > 1:
+        if self.world > 1 and self.variant != "fused_peer":   # fused_peer reduces inside its kernel
             import torch.distributed as dist
             dist.all_reduce(self.y)
 

@@ -431,6 +431,34 @@ catt_status catt_kernel_attrs(const catt_problem* prob, const catt_throttle* t, 
 
 const char* catt_status_str(catt_status s);
 int catt_last_cuda_error(void);
+/* ------------------------------------------------------------ multi-GPU
+ * Row-sharded ATAX with the A^T partial sums all-reduced inside the fused
+ * kernel through peer memory (the row-sharded step of 8(e)
+ * with NCCL's all-reduce replaced by stores into the other ranks' buffers
+ * over NVLink). One process per GPU; world <= 8 ranks of one NVLink domain.
+ *
+ * catt_peer_create allocates this rank's buffer (receive slots and flags for
+ * n columns, cudaMalloc, owned by the object) and writes its CUDA IPC handle
+ * (CATT_PEER_HANDLE_BYTES bytes) to host memory `handle`. The caller ships
+ * the handles between ranks (e.g. all_gather_object) and calls
+ * catt_peer_open once per other rank. catt_atax_peer then computes, on every
+ * rank g, tmp_g = A_g x (rows of this shard, m x n row-major) and the full
+ * y = sum over ranks of A_g^T tmp_g, summed in rank order in the kernel, so
+ * every rank holds bit-identical y. All ranks must call it in the same order
+ * with equal shapes (equal shards give equal grids); each call is one launch
+ * on `stream`, asynchronous. A wait for a peer longer than 10 s makes the
+ * kernel give up; catt_peer_check (synchronous) reports it. Results: within
+ * 1e-5 of fp64, bit-exact on exact-dyadic inputs (the FUSED bar). Errors: CATT_EINVAL (arguments, a peer not opened, grids over
+ * 1024 CTAs), CATT_ECUDA (IPC or launch), CATT_EUNSUPPORTED (n > 16384). */
+enum { CATT_PEER_HANDLE_BYTES = 64 };
+typedef struct catt_peer catt_peer;
+catt_status catt_peer_create(int32_t world, int32_t rank, int64_t n, catt_peer** out, void* handle);
+catt_status catt_peer_open(catt_peer* p, int32_t peer_rank, const void* handle);
+catt_status catt_peer_check(catt_peer* p, int32_t* timed_out);
+catt_status catt_peer_destroy(catt_peer* p);
+catt_status catt_atax_peer(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n, catt_peer* p,
+                           void* stream);
+
 /* Diagnostics: the FUSED single-read kernel records, when the environment
  * variable CATT_FUSED_TRACE is set at launch, six %globaltimer stamps per CTA
  * (start, first stage landed, last stage consumed, column partials written,

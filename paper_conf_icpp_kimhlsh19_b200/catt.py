@@ -25,6 +25,7 @@ MODE_UNION, MODE_PAPER = 0, 1
 FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE, FIT_GUARDED = 1, 2, 4, 8, 16
 VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED, VAR_BYPASS = 0, 1, 2, 3, 4, 5, 6
 ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
+PEER_HANDLE_BYTES = 64
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
 (K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K,
@@ -179,6 +180,11 @@ def lib():
             "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
             "catt_kernel_attrs": [P(Problem), T, P(i32), P(i32)],
             "catt_fused_trace": [P(u64), i32],
+            "catt_peer_create": [i32, i32, i64, P(V), V],
+            "catt_peer_open": [V, i32, V],
+            "catt_peer_check": [V, P(i32)],
+            "catt_peer_destroy": [V],
+            "catt_atax_peer": [V, V, V, V, i64, i64, V, V],
             "catt_status_str": [ctypes.c_int],
             "catt_last_cuda_error": [],
             "catt_abi_version": [],
@@ -198,7 +204,8 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_gemm", "catt_corr", "catt_kmeans_assign",
             "catt_kmeans_acc_words", "catt_kmeans_transpose", "catt_kmeans_accumulate", "catt_kmeans_finalize",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
-            "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace"]
+            "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
+            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer"]
 
 
 def _check(st: int, what: str):
@@ -422,6 +429,45 @@ def syr2k(A, B, C, alpha, beta, t: Optional[Throttle] = None):
     _check(lib().catt_syr2k(_dev(A, "A"), _dev(B, "B"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t),
                             _stream()), "catt_syr2k")
     return C
+
+
+class Peer:
+    """This rank's peer-memory all-reduce state (catt_peer_*): create, ship
+    `handle` (bytes) to the other ranks, `open` theirs, then `atax_peer`."""
+
+    def __init__(self, world, rank, n):
+        self.ptr = ctypes.c_void_p()
+        buf = ctypes.create_string_buffer(PEER_HANDLE_BYTES)
+        _check(lib().catt_peer_create(world, rank, n, ctypes.byref(self.ptr), buf), "catt_peer_create")
+        self.handle = buf.raw
+        self.world, self.rank, self.n = world, rank, n
+
+    def open(self, peer_rank, handle: bytes):
+        buf = ctypes.create_string_buffer(handle, PEER_HANDLE_BYTES)
+        _check(lib().catt_peer_open(self.ptr, peer_rank, buf), "catt_peer_open")
+
+    def timed_out(self) -> bool:
+        v = ctypes.c_int32()
+        _check(lib().catt_peer_check(self.ptr, ctypes.byref(v)), "catt_peer_check")
+        return bool(v.value)
+
+    def close(self):
+        if self.ptr:
+            _check(lib().catt_peer_destroy(self.ptr), "catt_peer_destroy")
+            self.ptr = ctypes.c_void_p()
+
+
+def atax_peer(A_g, x, peer: Peer, tmp_g=None, y=None):
+    """Row-sharded ATAX step with the A^T partials all-reduced inside the fused
+    kernel through peer memory (catt_atax_peer): tmp_g = A_g x, y = sum over
+    ranks of A_g^T tmp_g (identical on every rank). Returns (tmp_g, y)."""
+    torch = _torch()
+    m, n = A_g.shape
+    tmp_g = torch.empty(m, device=A_g.device) if tmp_g is None else tmp_g
+    y = torch.empty(n, device=A_g.device) if y is None else y
+    _check(lib().catt_atax_peer(_dev(A_g, "A"), _dev(x, "x"), _dev(tmp_g, "tmp"), _dev(y, "y"), m, n, peer.ptr,
+                                _stream()), "catt_atax_peer")
+    return tmp_g, y
 
 
 def fused_trace(nctas):

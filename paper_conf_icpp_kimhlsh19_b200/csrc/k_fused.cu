@@ -18,6 +18,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstdlib>
+#include <cstring>
 
 #include <cooperative_groups.h>
 
@@ -27,6 +28,8 @@
 namespace catt {
 
 constexpr int kMaxDual = 4;
+constexpr int kMaxPeers = 8;      // ranks of one NVLink / NVSwitch domain
+constexpr int kPeerCtas = 1024;   // flag slots per (parity, source rank)
 constexpr int kTraceCtas = 1024, kTracePhases = 6;
 // per-CTA %globaltimer at: start, first stage landed, last stage consumed,
 // partials written, after the grid barrier, end (diagnostics only)
@@ -53,6 +56,13 @@ struct FusedArgs {
   int fastbar;                // nd kernel: grid barrier by ordered atomics (grid_barrier_ordered)
   unsigned* gbar;             // grid barrier {count, generation}
   int64_t N;
+  // DEP kernel, row-sharded ATAX (catt_atax_peer): the column outputs are
+  // all-reduced across ranks through peer memory inside this kernel
+  float* peer_recv[kMaxPeers];       // rank p's receive buffer [2 parities][world][N] (IPC-mapped)
+  unsigned* peer_flag[kMaxPeers];    // rank p's flags [2][world][kPeerCtas]
+  unsigned* peer_err;                // this rank's error word (a wait timed out)
+  int world, rank;                   // world = 0: no peer reduction
+  unsigned epoch;                    // launch number, equal on every rank
 };
 
 __device__ __forceinline__ float4 ld_stream4(const float4* p) {
@@ -103,6 +113,64 @@ __device__ __forceinline__ void grid_barrier_ordered(unsigned* bar, unsigned nbl
     }
   }
   __syncthreads();
+}
+
+// Peer-memory all-reduce of the column outputs (row-sharded ATAX): every CTA
+// has stored its columns' partials into slot [par][rank] of every rank's
+// receive buffer (plain stores through the IPC-mapped pointers, over NVLink
+// between GPUs). Then: system-scope fence, and thread 0 publishes epoch in
+// flag [par][rank][cta] of every rank (release). The CTA waits for flag
+// [par][g][cta] == epoch from every source g (acquire; the chunk -> CTA map
+// is the same on every rank: equal shards, equal grids), and sums the slots
+// in rank order: every rank gets bit-identical outputs. par = epoch & 1
+// double-buffers slots and flags, so a rank one launch ahead never
+// overwrites data still being read (it cannot get two launches ahead: its
+// next wait needs this rank's next flags). A wait longer than 10 s sets
+// *peer_err and gives up instead of hanging the GPU.
+template <int NW>
+__device__ void peer_allreduce(const FusedArgs& a) {
+  const int64_t N = a.N;
+  const unsigned par = a.epoch & 1u;
+  __threadfence_system();
+  __syncthreads();
+  __shared__ int s_ok;
+  if (threadIdx.x == 0) {
+    for (int p = 0; p < a.world; ++p) {
+      unsigned* f = a.peer_flag[p] + (int64_t(par) * a.world + a.rank) * kPeerCtas + blockIdx.x;
+      asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(a.epoch) : "memory");
+    }
+    int ok = 1;
+    const unsigned long long t0 = gtimer();
+    unsigned* mine = a.peer_flag[a.rank];
+    for (int g = 0; g < a.world && ok; ++g) {
+      const unsigned* f = mine + (int64_t(par) * a.world + g) * kPeerCtas + blockIdx.x;
+      unsigned v;
+      while (true) {
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+        if (v == a.epoch) break;
+        if (gtimer() - t0 > 10000000000ull) {
+          atomicExch(a.peer_err, 1u);
+          ok = 0;
+          break;
+        }
+        __nanosleep(100);
+      }
+    }
+    s_ok = ok;
+  }
+  __syncthreads();
+  if (!s_ok) return;
+  const float* recv = a.peer_recv[a.rank] + int64_t(par) * a.world * N;
+  const int64_t chunks = (N + 31) / 32;
+  for (int64_t ch = blockIdx.x; ch < chunks; ch += gridDim.x) {
+    const int64_t j = ch * 32 + (threadIdx.x & 31);
+    if ((threadIdx.x >> 5) == 0 && j < N) {
+      float tot = __ldcg(recv + j);
+      for (int g = 1; g < a.world; ++g) tot += __ldcg(recv + int64_t(g) * N + j);
+      if (a.col_acc[0]) tot = a.yc[0][j] + tot;
+      a.yc[0][j] = tot;
+    }
+  }
 }
 
 // DEP = true: ATAX (the column loop's vector is the row loop's result).
@@ -267,12 +335,19 @@ __global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS,
       if (warp == 0 && j < N) {
         float tot = red[0][lane];
         for (int w = 1; w < NW; ++w) tot += red[w][lane];
-        if (a.col_acc[q]) tot = a.yc[q][j] + tot;
-        a.yc[q][j] = tot;
+        if (a.world > 0) {
+          // this rank's partial of column j, stored into every rank's slot [par][rank]
+          const int64_t slot = (int64_t(a.epoch & 1u) * a.world + a.rank) * N + j;
+          for (int p = 0; p < a.world; ++p) a.peer_recv[p][slot] = tot;
+        } else {
+          if (a.col_acc[q]) tot = a.yc[q][j] + tot;
+          a.yc[q][j] = tot;
+        }
       }
       __syncthreads();
     }
   }
+  if (a.world > 0) peer_allreduce<NW>(a);
 }
 
 // Independent pair (BICG, MVT: the column weights xc are inputs), one read
@@ -559,8 +634,31 @@ struct DualProblem {
   int row_acc, col_acc;
 };
 
+}  // namespace catt
+
+// A rank's peer-reduction state (catt_peer_*): one cudaMalloc holding
+// [receive slots: 2 x world x n floats][flags: 2 x world x kPeerCtas u32][error word],
+// exported by a CUDA IPC handle; the peers' buffers opened from theirs.
+struct catt_peer {
+  int world = 0, rank = 0;
+  int64_t n = 0;
+  void* base = nullptr;
+  size_t bytes = 0;
+  float* recv[catt::kMaxPeers] = {};
+  unsigned* flag[catt::kMaxPeers] = {};
+  void* opened[catt::kMaxPeers] = {};
+  unsigned epoch = 0;
+  unsigned* err = nullptr;
+};
+
+namespace catt {
+
+struct PeerLaunch {
+  catt_peer* p;
+};
+
 catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t N, const catt_throttle* t,
-                               cudaStream_t s) {
+                               cudaStream_t s, const PeerLaunch* peer = nullptr) {
   if (np < 1 || np > kMaxDual || N <= 0 || N % 4) return CATT_EINVAL;
   int64_t Mtot = 0;
   for (int i = 0; i < np; ++i) {
@@ -680,6 +778,20 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   }
   args.cta0[np] = cta;
   if (cta > slots) return CATT_EUNSUPPORTED;                 // cannot be co-resident for the grid barrier
+  if (peer) {
+    catt_peer* P = peer->p;
+    if (!dep || np != 1 || CL != 1 || cta > kPeerCtas || P->n != N) return CATT_EINVAL;
+    for (int r = 0; r < P->world; ++r)
+      if (!P->recv[r] || !P->flag[r]) return CATT_EINVAL;       // a peer not opened yet
+    args.world = P->world;
+    args.rank = P->rank;
+    args.epoch = ++P->epoch;
+    args.peer_err = P->err;
+    for (int r = 0; r < P->world; ++r) {
+      args.peer_recv[r] = P->recv[r];
+      args.peer_flag[r] = P->flag[r];
+    }
+  }
   float* work = nullptr;
   unsigned* gbar = nullptr;
   size_t need = 0;
@@ -728,6 +840,88 @@ const void* fused_func(bool dep) { return dep ? fused_fn<true>(16, 2) : fused_fn
 }  // namespace catt
 
 using namespace catt;
+
+namespace {
+size_t peer_layout(int world, int64_t n, size_t* flag_off, size_t* err_off) {
+  *flag_off = ((size_t(2) * world * size_t(n) * sizeof(float) + 255) / 256) * 256;
+  *err_off = *flag_off + size_t(2) * world * kPeerCtas * sizeof(unsigned);
+  return *err_off + 256;
+}
+}  // namespace
+
+extern "C" catt_status catt_peer_create(int32_t world, int32_t rank, int64_t n, catt_peer** out, void* handle) {
+  if (!out || !handle || world < 1 || world > kMaxPeers || rank < 0 || rank >= world || n < 1) return CATT_EINVAL;
+  catt_peer* p = new catt_peer();
+  p->world = world;
+  p->rank = rank;
+  p->n = n;
+  size_t foff = 0, eoff = 0;
+  p->bytes = peer_layout(world, n, &foff, &eoff);
+  cudaError_t e = cudaMalloc(&p->base, p->bytes);
+  if (e == cudaSuccess) e = cudaMemset(p->base, 0, p->bytes);
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(static_cast<cudaIpcMemHandle_t*>(handle), p->base);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    if (p->base) cudaFree(p->base);
+    delete p;
+    return e == cudaErrorMemoryAllocation ? CATT_ENOMEM : CATT_ECUDA;
+  }
+  char* b = static_cast<char*>(p->base);
+  p->recv[rank] = reinterpret_cast<float*>(b);
+  p->flag[rank] = reinterpret_cast<unsigned*>(b + foff);
+  p->err = reinterpret_cast<unsigned*>(b + eoff);
+  *out = p;
+  return CATT_OK;
+}
+
+extern "C" catt_status catt_peer_open(catt_peer* p, int32_t peer_rank, const void* handle) {
+  if (!p || !handle || peer_rank < 0 || peer_rank >= p->world) return CATT_EINVAL;
+  if (peer_rank == p->rank) return CATT_OK;                  // own buffer: nothing to open
+  if (p->opened[peer_rank]) return CATT_EINVAL;
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  void* q = nullptr;
+  cudaError_t e = cudaIpcOpenMemHandle(&q, h, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  size_t foff = 0, eoff = 0;
+  peer_layout(p->world, p->n, &foff, &eoff);
+  p->opened[peer_rank] = q;
+  p->recv[peer_rank] = static_cast<float*>(q);
+  p->flag[peer_rank] = reinterpret_cast<unsigned*>(static_cast<char*>(q) + foff);
+  return CATT_OK;
+}
+
+extern "C" catt_status catt_peer_check(catt_peer* p, int32_t* timed_out) {
+  if (!p || !timed_out) return CATT_EINVAL;
+  unsigned v = 0;
+  cudaError_t e = cudaMemcpy(&v, p->err, sizeof(v), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  *timed_out = int32_t(v != 0);
+  return CATT_OK;
+}
+
+extern "C" catt_status catt_peer_destroy(catt_peer* p) {
+  if (!p) return CATT_EINVAL;
+  for (int r = 0; r < kMaxPeers; ++r)
+    if (p->opened[r]) cudaIpcCloseMemHandle(p->opened[r]);
+  if (p->base) cudaFree(p->base);
+  delete p;
+  return CATT_OK;
+}
+
+extern "C" catt_status catt_atax_peer(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n,
+                                      catt_peer* p, void* stream) {
+  if (!A || !x || !tmp || !y || !p || m < 1 || n < 1) return CATT_EINVAL;
+  DualProblem pr{A, x, nullptr, tmp, y, m, 0, 0};
+  PeerLaunch pl{p};
+  return launch_fused_group(true, &pr, 1, n, nullptr, static_cast<cudaStream_t>(stream), &pl);
+}
 
 extern "C" catt_status catt_fused_trace(uint64_t* out, int32_t n) {
   if (!out || n < 0) return CATT_EINVAL;

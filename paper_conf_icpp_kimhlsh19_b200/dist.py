@@ -77,6 +77,30 @@ def atax_rowshard(A_g, x, tmp_g=None, y=None, k1=None, k2=None, group=None, ops=
     return tmp_g, y
 
 
+def peer_setup(n, group=None):
+    """This rank's catt.Peer for n columns: its CUDA IPC
+    handle goes to every rank of the group (all_gather_object) and the other
+    ranks' buffers are opened. One per (group, n); reuse it for every step."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = _rank(group)
+    peer = catt.Peer(world, rank, n)
+    if world > 1:
+        handles = [None] * world
+        dist.all_gather_object(handles, (rank, peer.handle), group=group)
+        for r, h in handles:
+            if r != rank:
+                peer.open(r, h)
+    return peer
+
+
+def atax_rowshard_peer(A_g, x, peer, tmp_g=None, y=None):
+    """tmp_g = A_g x; y = sum over ranks of A_g^T tmp_g, with the sum done
+    inside the fused kernel through peer memory (no NCCL call): one launch
+    per step on every rank, y bit-identical on all ranks."""
+    return catt.atax_peer(A_g, x, peer, tmp_g, y)
+
+
 def bicg_rowshard(A_g, p, r_g, q_g=None, s=None, k1=None, k2=None, group=None, ops=CudaOps):
     """s = sum over ranks of A_g^T r_g (k1); q_g = A_g p (k2)."""
     import torch

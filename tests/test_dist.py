@@ -260,3 +260,51 @@ def test_rowshard_single_rank_nccl():
         assert np.array_equal(q.cpu().numpy(), q_o) and np.array_equal(s.cpu().numpy(), s_o)
     finally:
         dist.destroy_process_group()
+
+
+class _FakePeer:
+    """Stands in for catt.Peer on CPU: records which handles were opened."""
+
+    def __init__(self, world, rank, n):
+        self.world, self.rank, self.n = world, rank, n
+        self.handle = bytes([rank]) * catt_mod.PEER_HANDLE_BYTES
+        self.opened = {}
+
+    def open(self, r, h):
+        assert r not in self.opened
+        self.opened[r] = h
+
+
+def _peer_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        orig = catt_mod.Peer
+        catt_mod.Peer = _FakePeer
+        try:
+            p = cdist.peer_setup(4096)
+        finally:
+            catt_mod.Peer = orig
+        q.put((rank, p.world, p.rank, sorted(p.opened), {r: h[0] for r, h in p.opened.items()}))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_peer_setup_exchanges_handles_world3_gloo():
+    """Host side of the fused peer all-reduce (f4): every rank creates one
+    peer object and opens every other rank's IPC handle exactly once (its own
+    never), over a gloo group of 3 processes."""
+    world, port = 3, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_peer_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    assert all(p.exitcode == 0 for p in procs)
+    for rank, w, r, opened, first_bytes in res:
+        assert (w, r) == (world, rank)
+        assert opened == [x for x in range(world) if x != rank]
+        assert all(first_bytes[x] == x for x in opened)          # the handle of rank x came from rank x
