@@ -58,6 +58,7 @@ def _rank_main(rank, world, port, m, n, steps, out_dir):
         tmp, y = cdist.atax_rowshard_peer(Ag, xd, peer)
         torch.cuda.synchronize()
         ys.append(y.cpu().numpy().copy())
+    os.environ["CATT_FUSED_NO_SMALL"] = "1"          # the plain fused kernel at every shape (the peer path's tree)
     tmp_p, y_p = catt.atax(Ag, xd, k1=catt.Throttle(variant="fused"))     # this rank's partial, no exchange
     torch.cuda.synchronize()
     np.save(os.path.join(out_dir, f"y{rank}.npy"), np.stack(ys))
