@@ -195,6 +195,7 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
   float* tile = reinterpret_cast<float*>(dyn + L.tile);                // [nf][KTP]
   __shared__ int s_cnt[KMAX], s_start[KMAX + 1], s_tot[KMAX];
   __shared__ unsigned short s_idx[KT];
+  __shared__ unsigned char s_cid[KT];                                    // centre of each sorted entry
   const int t = threadIdx.x, lane = t & 31, w = t >> 5;
   // a padded centre at +inf is never strictly nearer than FLT_MAX: same decisions
   for (int q = t; q < nf * KP; q += KT) {
@@ -303,13 +304,16 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
       }
     }
     __syncthreads();
-    if (c >= 0) s_idx[s_start[c] + rank] = static_cast<unsigned short>(t);
+    if (c >= 0) {
+      s_idx[s_start[c] + rank] = static_cast<unsigned short>(t);
+      s_cid[s_start[c] + rank] = static_cast<unsigned char>(c);
+    }
     __syncthreads();
     // phase 2: warp w owns sorted entries [32w, 32w + 32). Group g holds
     // features [32g, 32g + 32); a group with fg < 32 features (the last one)
     // spreads its lanes as fg features x (32/fg) sub-chunks of fg entries.
-    // The centre of a sorted segment is warp-uniform, so acc[g][cc] has a
-    // static index.
+    // The centres met by a lane's range are consecutive in the sorted order
+    // (s_cid of its first and last entry bound them).
 #pragma unroll
     for (int g = 0; g < FB; ++g) {
       const int rem = nf - 32 * g;
@@ -320,7 +324,10 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
         const bool fok = fl < rem;
         const float* row = tile + (32 * g + fl) * KTP;
         u128* mine = s_acc + (w * FB + g) * k * 32 + lane;
-        for (int cc = 0; cc < k; ++cc) {
+        // only the centres whose segments meet [s_lo, s_hi) (usually one or two)
+        const int e1 = min(s_hi, s_start[k]);
+        const int c0 = s_lo < e1 ? int(s_cid[s_lo]) : k, c1 = s_lo < e1 ? int(s_cid[e1 - 1]) : -1;
+        for (int cc = c0; cc <= c1; ++cc) {
           const int lo = max(s_start[cc], s_lo), hi = fok ? min(s_start[cc + 1], s_hi) : lo;
           if (lo < hi) mine[cc * 32] += segment_sum(row, s_idx, lo, hi, inexact);
         }
