@@ -323,15 +323,19 @@ class KmeansIter(Workload):
         self.memb = torch.full((self.np_,), -1, dtype=torch.int32, device=dev)
         self.acc = torch.zeros(catt.kmeans_acc_words(self.k, self.nf), dtype=torch.int64, device=dev)
         nbytes = self.np_ * self.nf * 4 + 8 * self.np_ + self.k * self.nf * 4
-        self.loops = [Loop("kmeans assign+sums", lambda: catt.kmeans_accumulate(
-                               self.feat, self.ld, self.np_, self.nf, self.clusters, self.memb, self.acc),
-                           nbytes, "kmeans_acc"),
-                      Loop("kmeans finalize", lambda: catt.kmeans_finalize(self.acc, self.clusters),
-                           self.acc.numel() * 8 * 2 + self.k * self.nf * 4, "kmeans_fin")]
-        if world > 1:                    # the iteration's one exchange: integer sums, between the two kernels
+        if world == 1:                   # one launch: the last CTA rounds the centres (catt_kmeans_step)
+            self.loops = [Loop("kmeans iteration (one launch)", lambda: catt.kmeans_step(
+                                   self.feat, self.ld, self.np_, self.nf, self.clusters, self.memb, self.acc),
+                               nbytes + self.k * self.nf * 4, "kmeans_acc")]
+        else:                            # the iteration's one exchange: integer sums, between the two kernels
             import torch.distributed as dist
-            self.loops.insert(1, Loop("kmeans all-reduce of the sums", lambda: dist.all_reduce(self.acc),
-                                      self.acc.numel() * 8, "collective"))
+            self.loops = [Loop("kmeans assign+sums", lambda: catt.kmeans_accumulate(
+                                   self.feat, self.ld, self.np_, self.nf, self.clusters, self.memb, self.acc),
+                               nbytes, "kmeans_acc"),
+                          Loop("kmeans all-reduce of the sums", lambda: dist.all_reduce(self.acc),
+                               self.acc.numel() * 8, "collective"),
+                          Loop("kmeans finalize", lambda: catt.kmeans_finalize(self.acc, self.clusters),
+                               self.acc.numel() * 8 * 2 + self.k * self.nf * 4, "kmeans_fin")]
         # the KM transpose loop (Rodinia invert_mapping), CATT-planned and studied
         self.pm = torch.empty(self.np_ * self.nf, device=dev)
         catt.fill_hash(self.pm, si.sub_seed(si.SEED_KMEANS, 3))

@@ -359,8 +359,16 @@ catt_status catt_kmeans_accumulate(const float* feat, int64_t ld, int64_t npoint
 catt_status catt_kmeans_finalize(int64_t* acc, int32_t k, int32_t nf, float* clusters, int64_t* stats,
                                  int32_t zero_acc, void* stream);
 
+/* One k-means iteration on one GPU in ONE launch: catt_kmeans_accumulate,
+ * then (the last CTA to finish, after every CTA's exact sums are in acc) the
+ * work of catt_kmeans_finalize with zero_acc = 1. Bit-identical to the two
+ * calls. stats (device int64[3], may be NULL) as in catt_kmeans_finalize.
+ * Not for sharded runs: there the sums are all-reduced between the two. */
+catt_status catt_kmeans_step(const float* feat, int64_t ld, int64_t npoints, int32_t nf, float* clusters, int32_t k,
+                             int32_t* membership, int64_t* acc, int64_t* stats, void* stream);
+
 /* The k-means loop on one GPU: membership := -1, then up to max_iter
- * iterations of accumulate + finalize; stops after the first iteration whose
+ * iterations of catt_kmeans_step (one launch each); stops after the first iteration whose
  * delta <= max_changes. clusters (k x nf, in: initial centres, out: final).
  * ws: device int64 workspace of catt_kmeans_acc_words(k, nf) + 4 words.
  * Iterations are queued without host round trips (a device-side done flag

@@ -171,6 +171,7 @@ def lib():
             "catt_kmeans_transpose": [V, V, i64, i32, i64, T, V],
             "catt_kmeans_accumulate": [V, i64, i64, i32, V, i32, V, V, V],
             "catt_kmeans_finalize": [V, i32, i32, V, V, i32, V],
+            "catt_kmeans_step": [V, i64, i64, i32, V, i32, V, V, V, V],
             "catt_kmeans": [V, i64, i64, i32, V, i32, V, i32, i64, V, P(i32), V],
             "catt_rows": [V, V, V, V, V, i64, i64, f32, f32, i32, T, V],
             "catt_dual": [V, V, V, V, V, i64, i64, i32, i32, i32, T, V],
@@ -203,6 +204,7 @@ def lib():
 EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint", "catt_kernel_desc", "catt_plan",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_gemm", "catt_corr", "catt_kmeans_assign",
             "catt_kmeans_acc_words", "catt_kmeans_transpose", "catt_kmeans_accumulate", "catt_kmeans_finalize",
+            "catt_kmeans_step",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
             "catt_peer_check", "catt_peer_destroy", "catt_atax_peer"]
@@ -545,6 +547,18 @@ def kmeans_finalize(acc, clusters, stats=None, zero_acc=True):
     sp = _dev(stats, "stats", torch.int64) if stats is not None else None
     _check(lib().catt_kmeans_finalize(_dev(acc, "acc", torch.int64), k, nf, _dev(clusters, "clusters"), sp,
                                       int(bool(zero_acc)), _stream()), "catt_kmeans_finalize")
+    return clusters
+
+
+def kmeans_step(feat, ld, npoints, nf, clusters, membership, acc, stats=None):
+    """One k-means iteration in one launch (catt_kmeans_step): accumulate, then
+    the last CTA rounds the new centres into clusters and zeroes acc."""
+    torch = _torch()
+    k = clusters.shape[0]
+    sp = _dev(stats, "stats", torch.int64) if stats is not None else None
+    _check(lib().catt_kmeans_step(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"), k,
+                                  _dev(membership, "membership", torch.int32), _dev(acc, "acc", torch.int64), sp,
+                                  _stream()), "catt_kmeans_step")
     return clusters
 
 

@@ -164,7 +164,18 @@ struct AccArgs {
   const long long* done;  // nullable: skip the pass when *done != 0
   int64_t ld, npoints;
   int nf, k;
+  // fused finalize (catt_kmeans_step, the single-GPU loop): the last CTA to
+  // finish rounds the new centres; fin_ctr = nullptr: accumulate only
+  unsigned* fin_ctr;
+  float* clusters_out;
+  long long* stats;
+  long long* ctrl;
+  int max_iter;
+  long long max_changes;
 };
+
+__device__ void finalize_body(unsigned long long* acc, int k, int nf, float* clusters, long long* stats, int zero,
+                              long long* ctrl, int max_iter, long long max_changes);
 
 // Dynamic shared memory: {mbarrier | centres [nf][KP] | TMA stage [nf][256]
 // (TMA only) | tile [nf][KTP] | 128-bit accumulators}.
@@ -356,6 +367,24 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
   if (t < k && s_tot[t]) atomicAdd(a.acc + K4 + t, (unsigned long long)s_tot[t]);
   if (t == 0 && delta) atomicAdd(a.acc + K4 + k, (unsigned long long)delta);
   if (inexact) atomicAdd(a.acc + K4 + k + 1, (unsigned long long)inexact);
+  if (a.fin_ctr) {
+    // last-CTA finalize: this CTA's sums are published (fence) before its
+    // arrival; the CTA that arrives last sees every CTA's sums (acq_rel)
+    __shared__ int s_last;
+    __threadfence();
+    __syncthreads();
+    if (t == 0) {
+      unsigned prev;
+      asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(prev) : "l"(a.fin_ctr) : "memory");
+      s_last = prev == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (s_last) {
+      __threadfence();
+      finalize_body(a.acc, k, nf, a.clusters_out, a.stats, 1, a.ctrl, a.max_iter, a.max_changes);
+      if (t == 0) *a.fin_ctr = 0u;                               // ready for the next launch
+    }
+  }
 }
 
 // round-to-nearest-even of (S * 2^-64) / cnt, S a signed 128-bit integer
@@ -395,6 +424,12 @@ __global__ void __launch_bounds__(1024) km_finalize_kernel(unsigned long long* a
                                                            long long* stats, int zero, long long* ctrl, int max_iter,
                                                            long long max_changes) {
   if (ctrl && ctrl[0]) return;
+  finalize_body(acc, k, nf, clusters, stats, zero, ctrl, max_iter, max_changes);
+}
+
+// the finalize of one CTA (any block size): new centres, stats, loop control, zeroing
+__device__ void finalize_body(unsigned long long* acc, int k, int nf, float* clusters, long long* stats, int zero,
+                              long long* ctrl, int max_iter, long long max_changes) {
   const int K4 = k * nf * 4, t = threadIdx.x;
   for (int q = t; q < k * nf; q += blockDim.x) {
     const int c = q / nf;
@@ -444,8 +479,17 @@ const void* acc_fn() {
   return (const void*)km_accumulate_kernel<KMAX, FB, TMA>;
 }
 
+struct FinArgs {
+  float* clusters;
+  long long* stats;
+  long long* ctrl;
+  int max_iter;
+  long long max_changes;
+};
+
 catt_status acc_launch(const float* feat, int64_t ld, int64_t npoints, int32_t nf, const float* clusters, int32_t k,
-                       int32_t* memb, int64_t* acc, const long long* done, cudaStream_t s) {
+                       int32_t* memb, int64_t* acc, const long long* done, cudaStream_t s,
+                       const FinArgs* fin = nullptr) {
   // TMA needs a 16-B aligned base and a row stride that is a multiple of 16 B;
   // otherwise the general form (per-thread loads, centres padded to 16)
   const bool tma = (reinterpret_cast<uintptr_t>(feat) & 15u) == 0 && ld % 4 == 0 && encode_fn() != nullptr;
@@ -493,7 +537,16 @@ catt_status acc_launch(const float* feat, int64_t ld, int64_t npoints, int32_t n
   }
   const int64_t tiles = (npoints + KT - 1) / KT;
   const int grid = int(std::min<int64_t>(tiles, int64_t(per_sm) * ctx->hw.num_sms));
-  AccArgs a{feat, clusters, memb, reinterpret_cast<unsigned long long*>(acc), done, ld, npoints, nf, k};
+  AccArgs a{feat, clusters, memb, reinterpret_cast<unsigned long long*>(acc), done, ld, npoints, nf, k,
+            nullptr, nullptr, nullptr, nullptr, 0, 0};
+  if (fin) {
+    a.fin_ctr = ctx->gbar + 8;                                    // a counter word beside the grid barrier
+    a.clusters_out = fin->clusters;
+    a.stats = fin->stats;
+    a.ctrl = fin->ctrl;
+    a.max_iter = fin->max_iter;
+    a.max_changes = fin->max_changes;
+  }
   void* args[] = {&map, &a};
   e = cudaLaunchKernel(f, dim3(unsigned(grid)), dim3(KT), args, smem, s);
   if (e != cudaSuccess) {
@@ -556,6 +609,20 @@ extern "C" catt_status catt_kmeans_accumulate(const float* feat, int64_t ld, int
   return acc_launch(feat, ld, npoints, nf, clusters, k, membership, acc, nullptr, static_cast<cudaStream_t>(stream));
 }
 
+extern "C" catt_status catt_kmeans_step(const float* feat, int64_t ld, int64_t npoints, int32_t nf, float* clusters,
+                                        int32_t k, int32_t* membership, int64_t* acc, int64_t* stats, void* stream) {
+  if (!acc_args_ok(ld, npoints, nf, k) || !acc || !clusters) return CATT_EINVAL;
+  if (npoints > 0 && (!feat || !membership)) return CATT_EINVAL;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (npoints == 0) {
+    km_finalize_kernel<<<1, 1024, 0, s>>>(reinterpret_cast<unsigned long long*>(acc), k, nf, clusters,
+                                          reinterpret_cast<long long*>(stats), 1, nullptr, 0, 0);
+    return after_launch();
+  }
+  FinArgs fin{clusters, reinterpret_cast<long long*>(stats), nullptr, 0, 0};
+  return acc_launch(feat, ld, npoints, nf, clusters, k, membership, acc, nullptr, s, &fin);
+}
+
 extern "C" catt_status catt_kmeans_finalize(int64_t* acc, int32_t k, int32_t nf, float* clusters, int64_t* stats,
                                             int32_t zero_acc, void* stream) {
   if (!acc || !clusters || k < 1 || nf < 1 || k > 16 || nf > 64) return CATT_EINVAL;
@@ -584,13 +651,15 @@ extern "C" catt_status catt_kmeans(const float* feat, int64_t ld, int64_t npoint
   constexpr int kBatch = 4;  // iterations queued between host checks of the device-side done flag
   for (int it = 0; it < max_iter; it += kBatch) {
     for (int j = 0; j < kBatch && it + j < max_iter; ++j) {
-      if (npoints > 0) {
-        catt_status st = acc_launch(feat, ld, npoints, nf, clusters, k, membership, ws, ctrl, s);
+      if (npoints > 0) {                                           // one launch per iteration
+        FinArgs fin{clusters, nullptr, ctrl, max_iter, max_changes};
+        catt_status st = acc_launch(feat, ld, npoints, nf, clusters, k, membership, ws, ctrl, s, &fin);
         if (st != CATT_OK) return st;
+      } else {
+        km_finalize_kernel<<<1, 1024, 0, s>>>(reinterpret_cast<unsigned long long*>(ws), k, nf, clusters, nullptr, 1,
+                                              ctrl, max_iter, max_changes);
+        if (after_launch() != CATT_OK) return CATT_ECUDA;
       }
-      km_finalize_kernel<<<1, 1024, 0, s>>>(reinterpret_cast<unsigned long long*>(ws), k, nf, clusters, nullptr, 1,
-                                            ctrl, max_iter, max_changes);
-      if (after_launch() != CATT_OK) return CATT_ECUDA;
     }
     e = cudaMemcpyAsync(host_ctrl, ctrl, sizeof(host_ctrl), cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);

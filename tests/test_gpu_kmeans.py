@@ -204,3 +204,34 @@ def test_invalid_arguments():
                                memb, acc)                                                        # nf > 64
     with pytest.raises(catt.CattError):
         catt.kmeans_transpose(feat, 10, 4, feat, 5, t=catt.Throttle(variant="coop"))             # ld < npoints
+
+
+@pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 4), (70001, 34, 5, 29), (300, 50, 12, 4), (257, 7, 3, 3)])
+def test_step_equals_accumulate_then_finalize(npts, nf, k, pad):
+    """catt_kmeans_step (one launch, last-CTA finalize) is bit-identical to
+    catt_kmeans_accumulate + catt_kmeans_finalize, over two iterations (the
+    second checks that the step left acc zeroed and its counter reset)."""
+    ld = npts + pad + (-(npts + pad)) % 4
+    feat = si.values(4, nf * ld)
+    cl0 = feat.reshape(nf, ld)[:, :k].T.copy()
+    F = dev(feat)
+    runs = []
+    for fused in (False, True):
+        C = dev(cl0)
+        memb = torch.full((npts,), -1, dtype=torch.int32, device="cuda")
+        acc = torch.zeros(catt.kmeans_acc_words(k, nf), dtype=torch.int64, device="cuda")
+        stats = torch.zeros(3, dtype=torch.int64, device="cuda")
+        out = []
+        for _ in range(2):
+            if fused:
+                catt.kmeans_step(F, ld, npts, nf, C, memb, acc, stats)
+            else:
+                catt.kmeans_accumulate(F, ld, npts, nf, C, memb, acc)
+                catt.kmeans_finalize(acc, C, stats)
+            torch.cuda.synchronize()
+            out.append((host(C).copy(), host(memb).copy(), host(stats).copy(), host(acc).copy()))
+        runs.append(out)
+    for (c0, m0, s0, a0), (c1, m1, s1, a1) in zip(*runs):
+        assert np.array_equal(c0.view(np.uint32), c1.view(np.uint32))
+        assert np.array_equal(m0, m1) and np.array_equal(s0, s1) and np.array_equal(a0, a1)
+        assert not a1.any()
