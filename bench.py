@@ -572,6 +572,8 @@ class Atax(Workload):
             # the A^T partials all-reduced inside the fused kernel through peer
             # memory: no NCCL call, one launch per step
             from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+            self.desc = ("ATAX 65536x16384 fp32 row-sharded, A^T partials all-reduced inside the fused kernel "
+                         "through peer memory (configs[4], SURVEY 8(f) f4)")
             self.peer = cdist.peer_setup(n)
             self.loops = [Loop("atax fused + peer all-reduce",
                                lambda: cdist.atax_rowshard_peer(self.A, self.x, self.peer, self.tmp, self.y),
