@@ -17,6 +17,7 @@ struct DevCtx {
   unsigned* gbar = nullptr;   // grid barrier {count, generation} of the fused kernels (inside the same allocation)
   float* work = nullptr;      // fused kernels' column partials, grown on demand
   size_t work_bytes = 0;
+  unsigned arrive_total[4] = {};  // FUSED single-read kernel: expected per-problem arrival counts (gbar + 32)
 };
 
 // Per-device context of the current device (hardware table, CTA-cap counters).

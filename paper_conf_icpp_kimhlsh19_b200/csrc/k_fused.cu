@@ -54,6 +54,9 @@ struct FusedArgs {
   int inter;                  // nd kernel: stage chunks dealt round robin over the problem's CTAs
   int trace;                  // nd kernel: record phase timestamps per CTA (catt_fused_trace)
   int fastbar;                // nd kernel: grid barrier by ordered atomics (grid_barrier_ordered)
+  int redpf;                  // nd kernel: column reduction issues a warp's band loads together
+  unsigned* arrive;           // nd kernel, fastbar 2: per-problem monotonic arrival counters
+  unsigned arrive_target[kMaxDual];  // counter value once every CTA of problem p has arrived
   unsigned* gbar;             // grid barrier {count, generation}
   int64_t N;
   // DEP kernel, row-sharded ATAX (catt_atax_peer): the column outputs are
@@ -539,7 +542,13 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
       if (cc < n4) reinterpret_cast<float4*>(part)[cc] = acc[t];
     }
   }
-  if (a.fastbar) {
+  if (a.fastbar == 2) {
+    // split arrival: one release add on this problem's counter, no last
+    // arriver; a CTA waits below only for the problem whose columns it sums
+    __syncthreads();
+    if (tr && threadIdx.x == 0) trp[3] = gtimer();
+    if (threadIdx.x == 0) asm volatile("red.release.gpu.add.u32 [%0], 1;" ::"l"(a.arrive + pi) : "memory");
+  } else if (a.fastbar) {
     if (tr && threadIdx.x == 0) trp[3] = gtimer();
     grid_barrier_ordered(a.gbar, gridDim.x);
   } else {
@@ -565,15 +574,54 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
       const int64_t gpw = (G + NW - 1) / NW;
       const int64_t b0 = warp * gpw, b1 = imin64(G, b0 + gpw);
       const float* pq = a.part[q];
+      // MVT's x2 (in/out) is an input until this chunk writes it: fetch it
+      // before waiting
+      float y0[LMAX];
+#pragma unroll
+      for (int l = 0; l < LMAX; ++l) {
+        const int64_t j = ch * CW + l * 32 + lane;
+        y0[l] = (warp == 0 && a.col_acc[q] && l < L && j < N) ? a.yc[q][j] : 0.0f;
+      }
+      if (a.fastbar == 2) {
+        if (threadIdx.x == 0) {
+          unsigned cur;
+          do {
+            asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(cur) : "l"(a.arrive + q) : "memory");
+          } while (int(cur - a.arrive_target[q]) < 0);
+          if (tr && gch == blockIdx.x) trp[4] = gtimer();
+        }
+        __syncthreads();
+      }
       if (!producer) {
         float sum[LMAX];
 #pragma unroll
         for (int l = 0; l < LMAX; ++l) sum[l] = 0.0f;
-        for (int64_t b = b0; b < b1; ++b) {
+        if (a.redpf) {
+          // all of the warp's band partials in flight at once (one L2 round
+          // trip instead of gpw), then added in band order as before
+          constexpr int BP = 8;
+          for (int64_t bb = b0; bb < b1; bb += BP) {
+            float v[BP][LMAX];
 #pragma unroll
-          for (int l = 0; l < LMAX; ++l) {
-            const int64_t j = ch * CW + l * 32 + lane;
-            if (l < L && j < N) sum[l] += pq[b * N + j];
+            for (int u = 0; u < BP; ++u)
+#pragma unroll
+              for (int l = 0; l < LMAX; ++l) {
+                const int64_t j = ch * CW + l * 32 + lane;
+                v[u][l] = (bb + u < b1 && l < L && j < N) ? pq[(bb + u) * N + j] : 0.0f;
+              }
+#pragma unroll
+            for (int u = 0; u < BP; ++u)
+#pragma unroll
+              for (int l = 0; l < LMAX; ++l)
+                if (bb + u < b1) sum[l] += v[u][l];
+          }
+        } else {
+          for (int64_t b = b0; b < b1; ++b) {
+#pragma unroll
+            for (int l = 0; l < LMAX; ++l) {
+              const int64_t j = ch * CW + l * 32 + lane;
+              if (l < L && j < N) sum[l] += pq[b * N + j];
+            }
           }
         }
 #pragma unroll
@@ -586,7 +634,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
           if (j < N) {
             float tot = red[0][l * 32 + lane];
             for (int w = 1; w < NW; ++w) tot += red[w][l * 32 + lane];
-            if (a.col_acc[q]) tot = a.yc[q][j] + tot;
+            if (a.col_acc[q]) tot = y0[l] + tot;
             a.yc[q][j] = tot;
           }
         }
@@ -868,7 +916,9 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
     args.inter = nd ? (ie ? atoi(ie) != 0 : 1) : 0;
     args.trace = nd && getenv("CATT_FUSED_TRACE") != nullptr;
     const char* fb = getenv("CATT_FUSED_BARRIER");
-    args.fastbar = fb ? atoi(fb) != 0 : 1;
+    args.fastbar = fb ? atoi(fb) : 2;
+    const char* rp = getenv("CATT_FUSED_REDPF");
+    args.redpf = rp ? atoi(rp) != 0 : 1;
   }
   int64_t given = 0;
   int cta = 0;
@@ -917,6 +967,20 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
     off += size_t((args.cta0[i + 1] - args.cta0[i]) / CL) * size_t(N);
   }
   args.gbar = gbar;
+  // per-problem arrival counters (fastbar 2) live after the {count,
+  // generation} pair, on their own 128-byte line; the host tracks their
+  // running totals and commits them only when the launch went in
+  args.arrive = gbar + 32;
+  {
+    // a captured launch would replay stale targets: graphs get the
+    // self-resetting barrier
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (args.fastbar == 2 && (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone)) {
+      cudaGetLastError();
+      args.fastbar = 1;
+    }
+  }
+  for (int i = 0; i < np; ++i) args.arrive_target[i] = ctx->arrive_total[i] + unsigned(args.cta0[i + 1] - args.cta0[i]);
   int rps = RPS, stages = S;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(unsigned(cta), 1, 1);
@@ -938,7 +1002,10 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
     record_cuda_error(e);
     return CATT_ECUDA;
   }
-  return after_launch();
+  st = after_launch();
+  if (st == CATT_OK && nd && args.fastbar == 2)
+    for (int i = 0; i < np; ++i) ctx->arrive_total[i] = args.arrive_target[i];
+  return st;
 }
 
 catt_status launch_fused(bool dep, const float* A, const float* xr, const float* xc, float* yr, float* yc, int64_t M,

@@ -581,3 +581,84 @@ def test_dual_group_bicg_and_mvt_in_one_launch(shapes):
     catt.dual_group(probs)
     for YR, YC, q, s in want:
         assert bits_equal(host(YR), q) and bits_equal(host(YC), s)
+
+
+def _dual_case(shapes, seed0):
+    probs, want = [], []
+    for k, (m, n) in enumerate(shapes):
+        A = si.matrix(seed0 + k, m, n, si.MODE_DYADIC)
+        xr, xc = si.values(seed0 + 10 + k, n, mode=si.MODE_DYADIC), si.values(seed0 + 20 + k, m, mode=si.MODE_DYADIC)
+        yr0, yc0 = si.values(seed0 + 30 + k, m, mode=si.MODE_DYADIC), si.values(seed0 + 40 + k, n, mode=si.MODE_DYADIC)
+        acc = k % 2 == 1
+        YR, YC = dev(yr0), dev(yc0)
+        probs.append(dict(A=dev(A), xr=dev(xr), xc=dev(xc), yr=YR, yc=YC, row_accumulate=acc, col_accumulate=acc))
+        q, s = oracle.bicg(A, xr, xc)
+        if acc:
+            q = (yr0.astype(np.float64) + q).astype(np.float32)
+            s = (yc0.astype(np.float64) + s).astype(np.float32)
+        want.append((YR, YC, yr0, yc0, q, s))
+    return probs, want
+
+
+@pytest.mark.parametrize("barrier", ["0", "1", "2"])
+def test_dual_group_barrier_modes_repeated(barrier, monkeypatch):
+    """Every grid-barrier form of the single-read fused kernel (0: fenced
+    count/generation, 1: ordered atomics, 2: per-problem monotonic arrival
+    counters with host-tracked targets, the default) over repeated launches
+    whose groups change shape (so the per-problem CTA counts, and with them
+    the arrival targets, change between launches): bit-exact every time."""
+    monkeypatch.setenv("CATT_FUSED_BARRIER", barrier)
+    cases = [_dual_case([(4096, 4096), (4096, 4096)], 300), _dual_case([(33, 64), (5000, 64), (7, 64)], 400),
+             _dual_case([(1000, 132), (300, 132)], 500)]
+    for rep in range(7):
+        probs, want = cases[rep % 3]
+        for p, (YR, YC, yr0, yc0, _, _) in zip(probs, want):
+            YR.copy_(dev(yr0))
+            YC.copy_(dev(yc0))
+        catt.dual_group(probs)
+        for YR, YC, _, _, q, s in want:
+            assert bits_equal(host(YR), q) and bits_equal(host(YC), s), (barrier, rep)
+
+
+def test_dual_group_uniform_same_bits_every_barrier(monkeypatch):
+    """The barrier form changes only when the partials are read, never the
+    order they are added in: uniform (inexact) inputs give the same bits."""
+    n = 2048
+    A, B = dev(si.matrix(71, n, n)), dev(si.matrix(72, n, n))
+    v = [dev(si.values(80 + i, n)) for i in range(8)]
+    outs = []
+    for barrier in ("0", "1", "2"):
+        monkeypatch.setenv("CATT_FUSED_BARRIER", barrier)
+        yr1, yc1, yr2, yc2 = (torch.zeros(n, device="cuda") for _ in range(4))
+        catt.dual_group([dict(A=A, xr=v[0], xc=v[1], yr=yr1, yc=yc1), dict(A=B, xr=v[2], xc=v[3], yr=yr2, yc=yc2)])
+        outs.append([host(t) for t in (yr1, yc1, yr2, yc2)])
+    for o in outs[1:]:
+        for a_, b_ in zip(outs[0], o):
+            assert bits_equal(a_, b_)
+
+
+def test_dual_group_graph_capture_replays():
+    """A captured grouped launch falls back to the self-resetting barrier (the
+    arrival targets of the default form are host-tracked and would go stale
+    in a replay): three replays with new inputs are bit-exact."""
+    probs, want = _dual_case([(4096, 4096), (4096, 4096)], 600)
+    catt.dual_group(probs)                      # grows the workspace outside the capture
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        catt.dual_group(probs)
+    for rep in range(3):
+        for p, (YR, YC, yr0, yc0, _, _) in zip(probs, want):
+            YR.copy_(dev(yr0))
+            YC.copy_(dev(yc0))
+        g.replay()
+        torch.cuda.synchronize()
+        for YR, YC, _, _, q, s in want:
+            assert bits_equal(host(YR), q) and bits_equal(host(YC), s), rep
+    catt.dual_group(probs)                      # the default form after a capture still agrees
+    for p, (YR, YC, yr0, yc0, _, _) in zip(probs, want):
+        YR.copy_(dev(yr0))
+        YC.copy_(dev(yc0))
+    catt.dual_group(probs)
+    for YR, YC, _, _, q, s in want:
+        assert bits_equal(host(YR), q) and bits_equal(host(YC), s)
