@@ -385,7 +385,10 @@ class Gesummv(Workload):
         self.loops = [Loop("gesummv", lambda: catt.rows(self.A, self.x, self.y, catt.ROWS_GESUMMV, self.B, self.tmp,
                                                          1.5, 1.2, t), 2 * n * n * 4 + 12 * n, "rows")]
         self.study = dict(name="gesummv (literal, row per thread)", prob=catt.problem(catt.K_GESUMMV, n=n),
-                          gesummv=True, launches=[(1024, 0), (1024, 196), (256, 196), (256, 228)])
+                          gesummv=True, launches=[(1024, 0), (1024, 196), (256, 196), (256, 228),
+                                                  # CTA- vs warp-level on SM partitions (SURVEY 8(d) [3]):
+                                                  # 32 CTAs on 8 SMs = 4 per SM, on 16 SMs = 2 per SM
+                                                  (256, 8, 8), (256, 196, 8), (256, 228, 8), (256, 228, 16)])
 
     def inputs(self):
         return [self.A, self.B, self.x]
@@ -700,42 +703,62 @@ def throttle_study(catt, torch, w, flush):
 
     out = []
     S = w.study
-    paper_hw = catt.paper_rule(hw)
-    for cta, carve in S["launches"]:
-        launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
-        t, r = catt.plan(S["prob"], launch, hw)               # B200 rule (guards on)
-        tp, rp = catt.plan(S["prob"], launch, paper_hw)       # the paper's Eq 9 rule
-        W, T = r["base_warps"], r["base_ctas"]
-        cands = []
-        for a in [d for d in range(W, 0, -1) if W % d == 0]:
-            for m in range(T, 0, -1):
-                cands.append((a, m))
-        times = {}
-        for a, m in cands:
-            th = launch.copy(active_warps=a, active_ctas=m if m < T else 0)
-            times[(a, m)] = med(study_fn(catt, w, th), S.get("reps", 5))
-        pick = (t.active_warps or W, t.active_ctas or T)
-        pick_p = (tp.active_warps or W, tp.active_ctas or T)
-        best = min(times, key=times.get)
-        # the bypass alternative: the same literal row loop with L2-only
-        # matrix loads at full TLP (row-loop studies only)
-        byp = None
-        if not S.get("fn") and not S.get("kmeans"):
-            byp = med(study_fn(catt, w, launch.copy(variant=catt.VAR_BYPASS)), S.get("reps", 5))
-        out.append(dict(loop=S["name"], cta_threads=cta, carveout_kb=r["carveout_kb"], base=[W, T],
-                        footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
-                        contended=rp["flags"] != catt.FIT_NONE_NEEDED,
-                        catt=list(pick), catt_rule=catt.FLAG_NAMES.get(r["flags"], r["flags"]),
-                        catt_ms=round(times[pick], 4),
-                        catt_paper=list(pick_p), catt_paper_ms=round(times[pick_p], 4),
-                        full_ms=round(times[(W, T)], 4), best=list(best), best_ms=round(times[best], 4),
-                        catt_over_best=round(times[pick] / times[best], 3),
-                        catt_over_full=round(times[pick] / times[(W, T)], 3),
-                        paper_over_best=round(times[pick_p] / times[best], 3),
-                        bypass_ms=round(byp, 4) if byp is not None else None,
-                        bypass_over_best=round(byp / times[best], 3) if byp is not None else None,
-                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()}))
+    parts = {}
+    import contextlib
+    for spec in S["launches"]:
+        cta, carve = spec[0], spec[1]
+        # a third entry: run on an SM partition of that many SMs (green
+        # context), planned with num_sms = the partition's SM count
+        sms = spec[2] if len(spec) > 2 else 0
+        if sms and sms not in parts:
+            parts[sms] = catt.SmPartition(sms)
+        part = parts.get(sms)
+        hw_l = part.hw(hw) if part else hw
+        with (torch.cuda.stream(part.stream) if part else contextlib.nullcontext()):
+            row = _study_launch(catt, w, S, cta, carve, hw_l, med)
+        if part:
+            row["sm_partition"] = part.sms
+        out.append(row)
+    for p in parts.values():
+        p.close()
     return out
+
+
+def _study_launch(catt, w, S, cta, carve, hw, med):
+    paper_hw = catt.paper_rule(hw)
+    launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
+    t, r = catt.plan(S["prob"], launch, hw)               # B200 rule (guards on)
+    tp, rp = catt.plan(S["prob"], launch, paper_hw)       # the paper's Eq 9 rule
+    W, T = r["base_warps"], r["base_ctas"]
+    cands = []
+    for a in [d for d in range(W, 0, -1) if W % d == 0]:
+        for m in range(T, 0, -1):
+            cands.append((a, m))
+    times = {}
+    for a, m in cands:
+        th = launch.copy(active_warps=a, active_ctas=m if m < T else 0)
+        times[(a, m)] = med(study_fn(catt, w, th), S.get("reps", 5))
+    pick = (t.active_warps or W, t.active_ctas or T)
+    pick_p = (tp.active_warps or W, tp.active_ctas or T)
+    best = min(times, key=times.get)
+    # the bypass alternative: the same literal row loop with L2-only
+    # matrix loads at full TLP (row-loop studies only)
+    byp = None
+    if not S.get("fn") and not S.get("kmeans"):
+        byp = med(study_fn(catt, w, launch.copy(variant=catt.VAR_BYPASS)), S.get("reps", 5))
+    return dict(loop=S["name"], cta_threads=cta, carveout_kb=r["carveout_kb"], base=[W, T],
+                    footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
+                    contended=rp["flags"] != catt.FIT_NONE_NEEDED,
+                    catt=list(pick), catt_rule=catt.FLAG_NAMES.get(r["flags"], r["flags"]),
+                    catt_ms=round(times[pick], 4),
+                    catt_paper=list(pick_p), catt_paper_ms=round(times[pick_p], 4),
+                    full_ms=round(times[(W, T)], 4), best=list(best), best_ms=round(times[best], 4),
+                    catt_over_best=round(times[pick] / times[best], 3),
+                    catt_over_full=round(times[pick] / times[(W, T)], 3),
+                    paper_over_best=round(times[pick_p] / times[best], 3),
+                    bypass_ms=round(byp, 4) if byp is not None else None,
+                    bypass_over_best=round(byp / times[best], 3) if byp is not None else None,
+                    swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
 
 
 def app_study(catt, torch, w, flush):

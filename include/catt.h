@@ -467,6 +467,21 @@ catt_status catt_peer_destroy(catt_peer* p);
 catt_status catt_atax_peer(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n, catt_peer* p,
                            void* stream);
 
+/* ------------------------------------------------------------ SM partition
+ * A stream whose kernels run on a partition of the device's SMs (a CUDA green
+ * context, driver 12.4+). SURVEY 8(d) [3]: CTA-level throttling (Fig 5,
+ * P:295-322) needs several co-resident CTAs per SM, which GESUMMV 8192's 32
+ * CTAs of 256 threads only get on a few SMs; the partition reproduces the
+ * paper's #TB_SM > 1 regime (Eq 3) on B200. `min_sms` is rounded up by
+ * the driver to its partition granularity; *sms_out receives the partition's
+ * SM count (plan with catt_hw.num_sms = *sms_out). The stream is owned by the
+ * library until catt_sm_partition_destroy; device memory of the primary
+ * context is usable on it. Errors: CATT_EINVAL (min_sms < 1 or above the
+ * device's count, null outputs), CATT_EUNSUPPORTED (driver without green
+ * contexts), CATT_ECUDA (driver call failed). */
+catt_status catt_sm_partition_create(int device, int32_t min_sms, void** stream_out, int32_t* sms_out);
+catt_status catt_sm_partition_destroy(void* stream);
+
 /* Diagnostics: the FUSED single-read kernel records, when the environment
  * variable CATT_FUSED_TRACE is set at launch, six %globaltimer stamps per CTA
  * (start, first stage landed, last stage consumed, column partials written,

@@ -189,6 +189,8 @@ def lib():
             "catt_status_str": [ctypes.c_int],
             "catt_last_cuda_error": [],
             "catt_abi_version": [],
+            "catt_sm_partition_create": [ctypes.c_int, i32, P(V), P(i32)],
+            "catt_sm_partition_destroy": [V],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -207,7 +209,8 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_kmeans_step",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
-            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer"]
+            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_sm_partition_create",
+            "catt_sm_partition_destroy"]
 
 
 def _check(st: int, what: str):
@@ -591,3 +594,36 @@ def calibrate_l1(device: int, pct: int, kb_list):
     out = (ctypes.c_float * n)()
     _check(lib().catt_calibrate_l1(device, pct, kb, n, out), "catt_calibrate_l1")
     return list(out)
+
+
+class SmPartition:
+    """A stream on a partition of >= min_sms SMs (catt_sm_partition_create, a
+    CUDA green context). `stream` is a torch ExternalStream: inside
+    `with torch.cuda.stream(p.stream):` every catt launch runs on the
+    partition. `sms` is the partition's SM count; `hw(base)` is the hardware
+    table to plan with (num_sms = sms, Eq 3's ceil(grid / #SM) bound)."""
+
+    def __init__(self, min_sms: int, device: int = 0):
+        h, n = ctypes.c_void_p(), ctypes.c_int32()
+        _check(lib().catt_sm_partition_create(device, min_sms, ctypes.byref(h), ctypes.byref(n)),
+               "catt_sm_partition_create")
+        self._h, self.sms = h, n.value
+        self.stream = _torch().cuda.ExternalStream(h.value, device=_torch().device("cuda", device))
+
+    def hw(self, base: "Hw") -> "Hw":
+        h = Hw()
+        ctypes.memmove(ctypes.byref(h), ctypes.byref(base), ctypes.sizeof(Hw))
+        h.num_sms = self.sms
+        return h
+
+    def close(self):
+        if self._h is not None:
+            self.stream.synchronize()
+            _check(lib().catt_sm_partition_destroy(self._h), "catt_sm_partition_destroy")
+            self._h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()

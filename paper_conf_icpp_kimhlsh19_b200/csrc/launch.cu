@@ -5,6 +5,9 @@
 #include <cstdint>
 #include <cstring>
 #include <mutex>
+#include <vector>
+
+#include <cuda.h>
 
 #include "internal.h"
 
@@ -632,3 +635,101 @@ extern "C" const char* catt_status_str(catt_status s) {
 
 extern "C" int catt_last_cuda_error(void) { return g_last_err; }
 extern "C" int catt_abi_version(void) { return 2; }
+
+// ------------------------------------------------------------ SM partition
+// Green context of >= min_sms SMs and a non-blocking stream in it (catt.h).
+// Driver entry points through the runtime (no -lcuda link).
+namespace {
+struct GreenApi {
+  bool ok = false;
+  CUresult (*devGet)(CUdevice*, int) = nullptr;
+  CUresult (*getRes)(CUdevice, CUdevResource*, CUdevResourceType) = nullptr;
+  CUresult (*split)(CUdevResource*, unsigned*, const CUdevResource*, CUdevResource*, unsigned, unsigned) = nullptr;
+  CUresult (*genDesc)(CUdevResourceDesc*, CUdevResource*, unsigned) = nullptr;
+  CUresult (*create)(CUgreenCtx*, CUdevResourceDesc, CUdevice, unsigned) = nullptr;
+  CUresult (*destroy)(CUgreenCtx) = nullptr;
+  CUresult (*streamCreate)(CUstream*, CUgreenCtx, unsigned, int) = nullptr;
+  CUresult (*streamDestroy)(CUstream) = nullptr;
+};
+template <typename F>
+bool entry(const char* name, F* out) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  *out = reinterpret_cast<F>(p);
+  return true;
+}
+const GreenApi& green_api() {
+  static GreenApi g = [] {
+    GreenApi a;
+    a.ok = entry("cuDeviceGet", &a.devGet) && entry("cuDeviceGetDevResource", &a.getRes) &&
+           entry("cuDevSmResourceSplitByCount", &a.split) && entry("cuDevResourceGenerateDesc", &a.genDesc) &&
+           entry("cuGreenCtxCreate", &a.create) && entry("cuGreenCtxDestroy", &a.destroy) &&
+           entry("cuGreenCtxStreamCreate", &a.streamCreate) && entry("cuStreamDestroy", &a.streamDestroy);
+    return a;
+  }();
+  return g;
+}
+std::mutex g_green_mu;
+std::vector<std::pair<CUstream, CUgreenCtx>> g_green;
+}  // namespace
+
+extern "C" catt_status catt_sm_partition_create(int device, int32_t min_sms, void** stream_out, int32_t* sms_out) {
+  if (!stream_out || !sms_out || min_sms < 1) return CATT_EINVAL;
+  const GreenApi& g = green_api();
+  if (!g.ok) return CATT_EUNSUPPORTED;
+  int nsm = 0;
+  cudaError_t e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  if (min_sms > nsm) return CATT_EINVAL;
+  e = cudaFree(nullptr);  // the primary context is active before the green one (cuGreenCtxCreate note)
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  CUdevice dev;
+  CUdevResource all{}, part{};
+  CUdevResourceDesc desc;
+  CUgreenCtx gc = nullptr;
+  CUstream st = nullptr;
+  unsigned ngroups = 1;
+  if (g.devGet(&dev, device) != CUDA_SUCCESS || g.getRes(dev, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS ||
+      g.split(&part, &ngroups, &all, nullptr, 0, unsigned(min_sms)) != CUDA_SUCCESS || ngroups < 1 ||
+      g.genDesc(&desc, &part, 1) != CUDA_SUCCESS || g.create(&gc, desc, dev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS)
+    return CATT_ECUDA;
+  if (g.streamCreate(&st, gc, CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS) {
+    g.destroy(gc);
+    return CATT_ECUDA;
+  }
+  {
+    std::lock_guard<std::mutex> lk(g_green_mu);
+    g_green.push_back({st, gc});
+  }
+  *stream_out = reinterpret_cast<void*>(st);
+  *sms_out = int32_t(part.sm.smCount);
+  return CATT_OK;
+}
+
+extern "C" catt_status catt_sm_partition_destroy(void* stream) {
+  const GreenApi& g = green_api();
+  if (!g.ok) return CATT_EUNSUPPORTED;
+  CUgreenCtx gc = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_green_mu);
+    for (size_t i = 0; i < g_green.size(); ++i)
+      if (reinterpret_cast<void*>(g_green[i].first) == stream) {
+        gc = g_green[i].second;
+        g_green.erase(g_green.begin() + long(i));
+        break;
+      }
+  }
+  if (!gc) return CATT_EINVAL;
+  const bool ok = g.streamDestroy(reinterpret_cast<CUstream>(stream)) == CUDA_SUCCESS;
+  return (g.destroy(gc) == CUDA_SUCCESS && ok) ? CATT_OK : CATT_ECUDA;
+}

@@ -662,3 +662,44 @@ def test_dual_group_graph_capture_replays():
     catt.dual_group(probs)
     for YR, YC, _, _, q, s in want:
         assert bits_equal(host(YR), q) and bits_equal(host(YC), s)
+
+
+# ------------------------------------------------------------------ SM partition (green context)
+@pytest.mark.parametrize("min_sms", [8, 16])
+def test_sm_partition_confines_ctas_and_keeps_results(min_sms):
+    """catt_sm_partition_create: launches on the partition's stream run on at
+    most `sms` distinct SMs (residency probe %smid), plan with num_sms = sms
+    gives the multi-CTA-per-SM base of Eq 3 (SURVEY 8(d) [3]: GESUMMV's 32
+    CTAs at 4 / 2 per SM), a CTA cap is enforced there, and results are the
+    literal loop's (bit-exact to seq-fmaf)."""
+    with catt.SmPartition(min_sms) as part:
+        assert min_sms <= part.sms < 148
+        hw = part.hw(catt.hw_query())
+        assert hw.num_sms == part.sms
+        n = 8192
+        t, r = catt.plan(catt.problem(catt.K_GESUMMV, n=n), catt.Throttle(cta_threads=256, carveout_kb=8,
+                                                                          variant="literal"), hw)
+        assert r["base_ctas"] == min(8, -(-32 // part.sms))
+        m, nn = 64 * 256, 256                                   # 64 CTAs of 256 rows
+        A = torch.empty(m * nn, device="cuda")
+        catt.fill_hash(A, 1)
+        x = torch.ones(nn, device="cuda")
+        probe = torch.zeros((m // 256) * 8 * 3, dtype=torch.int64, device="cuda")
+        with torch.cuda.stream(part.stream):
+            tmp, y = catt.atax(A.view(m, nn), x, k1=catt.Throttle(active_ctas=2, probe=probe.data_ptr()))
+        part.stream.synchronize()
+        rec = host(probe).astype(np.int64).reshape(-1, 3)
+        sms = set(int(s) for s in rec[rec[:, 2] > 0, 0])
+        assert 1 <= len(sms) <= part.sms
+        mw, mc = _concurrency(rec, 8)
+        assert mc <= 2
+        Ah = oracle.fill(1, m * nn).reshape(m, nn)
+        tmp_o, y_o = oracle.atax(Ah, np.ones(nn, dtype=np.float32))
+        assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y), y_o)
+
+
+def test_sm_partition_errors():
+    with pytest.raises(catt.CattError):
+        catt.SmPartition(0)
+    with pytest.raises(catt.CattError):
+        catt.SmPartition(10_000)
