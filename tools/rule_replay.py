@@ -5,13 +5,14 @@ studies) has the time of every (a, m) at one launch. The problem of each loop
 name is rebuilt here, the analyser (catt_plan, no GPU) picks (a, m) under the
 rule, and the pick's time is divided by the best swept time.
 
-usage: python tools/rule_replay.py [--rule b200|r23|r18|paper] [--set final|heldout|heldout2|heldout3|all] [-v]
+usage: python tools/rule_replay.py [--rule b200|r23|r18|paper] [--set final|heldout|heldout2|heldout3|partition|all] [-v]
   b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24)
   r23   = R18 + R19 + R23 (re-touch and reuse-trip terms), as held-out study 2 tested it
   r18   = the new terms off (the round-1 rule as fitted)
   paper = guards off (the paper's Eq 9 as printed)
 """
 import argparse
+import ctypes
 import glob
 import json
 import os
@@ -32,6 +33,7 @@ LOOPS = {
     ("final", "syr2k (literal, 2-D block 32 x 8)"): (P(catt.K_SYR2K, n=2048, k=2048), "literal"),
     ("final", "corr loop (literal, thread per column j1)"): (P(catt.K_CORR, n=2048, k=2048), "literal"),
     ("final", "gemm (literal, 2-D block 32 x 8)"): (P(catt.K_GEMM, m=512, n=512, k=512), "literal"),
+    ("partition", "gesummv (literal, row per thread)"): (P(catt.K_GESUMMV, n=8192), "literal"),
     ("heldout", "syrk2048 literal"): (P(catt.K_SYRK, n=2048, k=2048), "literal"),
     ("heldout", "mvt1 literal"): (P(catt.K_MVT_1, n=4096), "literal"),
     ("heldout", "bicg2 vec4"): (P(catt.K_BICG_2, m=4096, n=4096), "vec4"),
@@ -39,7 +41,10 @@ LOOPS = {
 }
 FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["profiles/r1/heldout_study.json"],
          "heldout2": sorted(glob.glob("profiles/r1q/heldout2_study.json")),
-         "heldout3": sorted(glob.glob("profiles/r1q/heldout3_study.json"))}
+         "heldout3": sorted(glob.glob("profiles/r1q/heldout3_study.json")),
+         # GESUMMV on SM partitions of 8 / 16 SMs (4 / 2 CTAs per SM), measured
+         # after R24 was fixed: the CTA-level regime (SURVEY 8(d) [3])
+         "partition": ["profiles/r1g/bench_gesummv.json"]}
 ATAX = {"bench_atax.json": P(catt.K_ATAX_1, m=65536, n=16384), "bench_atax256.json": P(catt.K_ATAX_1, m=256, n=256)}
 
 
@@ -76,10 +81,17 @@ def replay(rule, sets, verbose):
             for r in rows_of(f):
                 if "swept" not in r:
                     continue
+                if (s == "partition") != ("sm_partition" in r):
+                    continue
                 prob, var = problem_of(s, f, r)
                 cta = r.get("cta_threads", r.get("cta"))
                 launch = catt.Throttle(cta_threads=cta, carveout_kb=r["carveout_kb"], variant=var)
-                t, res = catt.plan(prob, launch, hw)
+                hw_l = hw
+                if "sm_partition" in r:
+                    hw_l = catt.Hw()
+                    ctypes.memmove(ctypes.byref(hw_l), ctypes.byref(hw), ctypes.sizeof(catt.Hw))
+                    hw_l.num_sms = r["sm_partition"]
+                t, res = catt.plan(prob, launch, hw_l)
                 W, T = res["base_warps"], res["base_ctas"]
                 if [W, T] != list(r["base"]):
                     raise SystemExit(f"base mismatch {r['loop']} {cta} {r['carveout_kb']}: {W, T} vs {r['base']}")
@@ -98,10 +110,10 @@ def replay(rule, sets, verbose):
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--rule", default="b200", choices=["b200", "r23", "r18", "paper"])
-    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "all"])
+    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "partition", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
-    sets = ["final", "heldout", "heldout2", "heldout3"] if a.set == "all" else [a.set]
+    sets = ["final", "heldout", "heldout2", "heldout3", "partition"] if a.set == "all" else [a.set]
     res = replay(a.rule, sets, a.v)
     for s in sets:
         rs = [x for x in res if x[0] == s]
