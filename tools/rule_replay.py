@@ -126,3 +126,12 @@ if __name__ == "__main__":
         print(f"[{a.rule}] {s}: {within}/{len(rs)} within 5% of best swept; worst {max(x[5] for x in rs):.3f}x; "
               f"launches where some throttle beats full TLP by >5%: {len(contended)}, pick beats full TLP on "
               f"{beats} of them; pick >5% slower than full TLP on {slower}")
+    # the paper's headline form (P:7: speedup over the baseline's full TLP and
+    # over the best static throttle), as geometric means over the launches
+    import math
+    gm = lambda v: math.exp(sum(math.log(x) for x in v) / len(v)) if v else float("nan")
+    cont = [x for x in res if x[6] > 1.05]
+    print(f"[{a.rule}] geomean over {len(res)} launches: speedup over full TLP {gm([x[6] / x[5] for x in res]):.3f}x, "
+          f"pick / best swept {gm([x[5] for x in res]):.3f}x; over the {len(cont)} launches where full TLP is >5% "
+          f"off the best: speedup over full TLP {gm([x[6] / x[5] for x in cont]):.3f}x "
+          f"(best swept: {gm([x[6] for x in cont]):.3f}x)")
