@@ -188,6 +188,21 @@ class BicgMvt(Workload):
         mat = rows * n * 4
         acc2 = rank == 0                 # x2 = x2 + sum_g A_g^T y2_g: only rank 0 adds the initial x2
         P = catt.problem
+        if var == "fused_peer":
+            # the grouped single-read launch with s and x2 all-reduced inside
+            # the kernel through peer memory: no NCCL
+            # call; x2's initial value is replicated and added after the sum
+            from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+            self.desc = ("BICG and MVT 4096x4096 fp32 per rank, row-sharded, column partials all-reduced inside "
+                         "the fused kernel through peer memory (configs[1] weak-scaled, SURVEY 8(f) f4)")
+            self.peer = cdist.peer_setup(2 * n)
+            group = [dict(A=self.Ab, xr=self.p, xc=self.r, yr=self.q, yc=self.s),
+                     dict(A=self.Am, xr=self.y1, xc=self.y2, yr=self.x1, yc=self.x2, row_accumulate=True,
+                          col_accumulate=True)]
+            self.loops = [Loop("bicg+mvt fused + peer all-reduce", lambda: cdist.bicg_mvt_rowshard_peer(group, self.peer),
+                               mat + 4 * 2 * (rows + n) + mat + 4 * (3 * rows + 3 * n), "fused")]
+            self.study = None
+            return
         if var in ("fused", "fused1"):
             # both loops of each application in one pass over A (A read once);
             # "fused" also groups BICG and MVT into one launch (one 128 MiB
@@ -247,7 +262,7 @@ class BicgMvt(Workload):
             launches=[(1024, 196), (1024, 228), (1024, 132)])
 
     def collective(self):
-        if self.world > 1:
+        if self.world > 1 and self.variant != "fused_peer":   # fused_peer reduces inside its kernel
             import torch.distributed as dist
             dist.all_reduce(self.s)
             dist.all_reduce(self.x2)

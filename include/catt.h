@@ -482,6 +482,18 @@ catt_status catt_atax_peer(const float* A, const float* x, float* tmp, float* y,
 catt_status catt_sm_partition_create(int device, int32_t min_sms, void** stream_out, int32_t* sms_out);
 catt_status catt_sm_partition_destroy(void* stream);
 
+/* Row-sharded BICG / MVT (any group of independent single-read problems, as
+ * catt_dual_group with dependent = 0) with every problem's column outputs
+ * all-reduced across ranks inside the kernel through the same peer memory
+ * (s = sum over ranks of A_g^T r_g, x2 = x2 + sum over ranks of
+ * A_g^T y2_g). On rank g each problem holds the rank's rows A_g (m x n); row
+ * outputs (q, x1) stay rank-local; column outputs are summed over ranks in
+ * rank order and then, for col_accumulate, added to the initial value (which
+ * must be the same on every rank), so every rank holds bit-identical columns.
+ * `p` must have been created with n = problems' n x count. Same calling rules,
+ * asynchrony, give-up and error codes as catt_atax_peer. */
+catt_status catt_dual_group_peer(const catt_dual_problem* probs, int32_t count, catt_peer* p, void* stream);
+
 /* Diagnostics: the FUSED single-read kernel records, when the environment
  * variable CATT_FUSED_TRACE is set at launch, six %globaltimer stamps per CTA
  * (start, first stage landed, last stage consumed, column partials written,

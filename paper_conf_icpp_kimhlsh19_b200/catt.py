@@ -186,6 +186,7 @@ def lib():
             "catt_peer_check": [V, P(i32)],
             "catt_peer_destroy": [V],
             "catt_atax_peer": [V, V, V, V, i64, i64, V, V],
+            "catt_dual_group_peer": [P(DualProblem), i32, V, V],
             "catt_status_str": [ctypes.c_int],
             "catt_last_cuda_error": [],
             "catt_abi_version": [],
@@ -209,7 +210,7 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_kmeans_step",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
-            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_sm_partition_create",
+            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_dual_group_peer", "catt_sm_partition_create",
             "catt_sm_partition_destroy"]
 
 
@@ -410,6 +411,11 @@ def dual(A, xr, yr, yc, xc=None, row_accumulate=False, col_accumulate=False, dep
 def dual_group(problems, dependent=False, t: Optional[Throttle] = None):
     """Grouped catt_dual: problems = [dict(A=, xr=, yr=, yc=, xc=None, row_accumulate=False,
     col_accumulate=False)], same column count, one launch."""
+    arr = _dual_array(problems)
+    _check(lib().catt_dual_group(arr, len(problems), int(bool(dependent)), _tp(t), _stream()), "catt_dual_group")
+
+
+def _dual_array(problems):
     arr = (DualProblem * len(problems))()
     for i, p in enumerate(problems):
         m, n = p["A"].shape
@@ -417,7 +423,17 @@ def dual_group(problems, dependent=False, t: Optional[Throttle] = None):
                              _dev(p["xc"], "xc").value if p.get("xc") is not None else None,
                              _dev(p["yr"], "yr").value, _dev(p["yc"], "yc").value, m, n,
                              int(bool(p.get("row_accumulate"))), int(bool(p.get("col_accumulate"))))
-    _check(lib().catt_dual_group(arr, len(problems), int(bool(dependent)), _tp(t), _stream()), "catt_dual_group")
+    return arr
+
+
+def dual_group_peer(problems, peer: "Peer"):
+    """Row-sharded grouped BICG / MVT step (catt_dual_group_peer): each
+    problem's A is this rank's rows; the column outputs yc are summed over
+    ranks inside the kernel (peer memory, rank order, then the initial value
+    for col_accumulate) and are bit-identical on every rank; yr stays local.
+    `peer` holds n x len(problems) columns."""
+    arr = _dual_array(problems)
+    _check(lib().catt_dual_group_peer(arr, len(problems), peer.ptr, _stream()), "catt_dual_group_peer")
 
 
 def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):

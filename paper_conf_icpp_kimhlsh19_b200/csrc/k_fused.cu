@@ -66,6 +66,7 @@ struct FusedArgs {
   unsigned* peer_err;                // this rank's error word (a wait timed out)
   int world, rank;                   // world = 0: no peer reduction
   unsigned epoch;                    // launch number, equal on every rank
+  int fence_all;                     // peer_flags: every thread fences (diagnostics)
 };
 
 __device__ __forceinline__ float4 ld_stream4(const float4* p) {
@@ -130,14 +131,18 @@ __device__ __forceinline__ void grid_barrier_ordered(unsigned* bar, unsigned nbl
 // overwrites data still being read (it cannot get two launches ahead: its
 // next wait needs this rank's next flags). A wait longer than 10 s sets
 // *peer_err and gives up instead of hanging the GPU.
-template <int NW>
-__device__ void peer_allreduce(const FusedArgs& a) {
-  const int64_t N = a.N;
+// The flag half of it: publish this CTA's partials, wait for the same CTA
+// index of every rank. Returns false (every thread) after a 10 s give-up.
+__device__ bool peer_flags(const FusedArgs& a) {
   const unsigned par = a.epoch & 1u;
-  __threadfence_system();
+  // the CTA's partial stores are ordered before thread 0's system-scope fence
+  // by the barrier (release cumulativity), so one fence per CTA publishes
+  // them (CATT_PEER_FENCE_ALL: every thread fences, the earlier form)
+  if (a.fence_all) __threadfence_system();
   __syncthreads();
   __shared__ int s_ok;
   if (threadIdx.x == 0) {
+    if (!a.fence_all) __threadfence_system();
     for (int p = 0; p < a.world; ++p) {
       unsigned* f = a.peer_flag[p] + (int64_t(par) * a.world + a.rank) * kPeerCtas + blockIdx.x;
       asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(a.epoch) : "memory");
@@ -162,7 +167,14 @@ __device__ void peer_allreduce(const FusedArgs& a) {
     s_ok = ok;
   }
   __syncthreads();
-  if (!s_ok) return;
+  return s_ok != 0;
+}
+
+template <int NW>
+__device__ void peer_allreduce(const FusedArgs& a) {
+  const int64_t N = a.N;
+  const unsigned par = a.epoch & 1u;
+  if (!peer_flags(a)) return;
   const float* recv = a.peer_recv[a.rank] + int64_t(par) * a.world * N;
   const int64_t chunks = (N + 31) / 32;
   for (int64_t ch = blockIdx.x; ch < chunks; ch += gridDim.x) {
@@ -634,12 +646,41 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
           if (j < N) {
             float tot = red[0][l * 32 + lane];
             for (int w = 1; w < NW; ++w) tot += red[w][l * 32 + lane];
-            if (a.col_acc[q]) tot = y0[l] + tot;
-            a.yc[q][j] = tot;
+            if (a.world > 0) {
+              // row-sharded (catt_dual_group_peer): this rank's partial of
+              // column j of problem q into slot [par][rank] of every rank
+              const int64_t slot = (int64_t(a.epoch & 1u) * a.world + a.rank) * (N * a.nprob) + int64_t(q) * N + j;
+              for (int p = 0; p < a.world; ++p) a.peer_recv[p][slot] = tot;
+            } else {
+              if (a.col_acc[q]) tot = y0[l] + tot;
+              a.yc[q][j] = tot;
+            }
           }
         }
       }
       __syncthreads();
+    }
+    if (a.world > 0 && peer_flags(a)) {
+      // the same chunks again: every rank's partials in rank order, then the
+      // initial value (MVT's x2, replicated on every rank): bit-identical
+      // outputs on every rank
+      const int64_t NP = N * a.nprob;
+      const float* recv = a.peer_recv[a.rank] + int64_t(a.epoch & 1u) * a.world * NP;
+      for (int64_t gch = blockIdx.x; gch < chunks * a.nprob; gch += gridDim.x) {
+        const int q = int(gch / chunks);
+        const int64_t ch = gch % chunks;
+        if (warp == 0)
+          for (int l = 0; l < L; ++l) {
+            const int64_t j = ch * CW + l * 32 + lane;
+            if (j < N) {
+              const int64_t c = int64_t(q) * N + j;
+              float tot = __ldcg(recv + c);
+              for (int g = 1; g < a.world; ++g) tot += __ldcg(recv + int64_t(g) * NP + c);
+              if (a.col_acc[q]) tot = a.yc[q][j] + tot;
+              a.yc[q][j] = tot;
+            }
+          }
+      }
     }
   }
   if (tr && threadIdx.x == 0) trp[5] = gtimer();
@@ -943,12 +984,15 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
   if (cta > slots) return CATT_EUNSUPPORTED;                 // cannot be co-resident for the grid barrier
   if (peer) {
     catt_peer* P = peer->p;
-    if (!dep || np != 1 || CL != 1 || cta > kPeerCtas || P->n != N) return CATT_EINVAL;
+    // ATAX (DEP): one problem; the single-read kernel: any group, the peer
+    // buffer holding every problem's columns
+    if ((dep && np != 1) || (!dep && !nd) || CL != 1 || cta > kPeerCtas || P->n != N * np) return CATT_EINVAL;
     for (int r = 0; r < P->world; ++r)
       if (!P->recv[r] || !P->flag[r]) return CATT_EINVAL;       // a peer not opened yet
     args.world = P->world;
     args.rank = P->rank;
     args.epoch = ++P->epoch;
+    args.fence_all = getenv("CATT_PEER_FENCE_ALL") != nullptr;
     args.peer_err = P->err;
     for (int r = 0; r < P->world; ++r) {
       args.peer_recv[r] = P->recv[r];
@@ -1126,6 +1170,21 @@ extern "C" catt_status catt_dual_group(const catt_dual_problem* probs, int32_t c
     pr[i] = DualProblem{q.A, q.xr, q.xc, q.yr, q.yc, q.m, q.row_accumulate != 0, q.col_accumulate != 0};
   }
   return launch_fused_group(dependent != 0, pr, count, N, t, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" catt_status catt_dual_group_peer(const catt_dual_problem* probs, int32_t count, catt_peer* p,
+                                            void* stream) {
+  if (!probs || !p || count < 1 || count > kMaxDual) return CATT_EINVAL;
+  DualProblem pr[kMaxDual];
+  const int64_t N = probs[0].n;
+  for (int i = 0; i < count; ++i) {
+    const catt_dual_problem& q = probs[i];
+    if (q.n != N || q.m < 1 || !q.A || !q.xr || !q.xc || !q.yr || !q.yc) return CATT_EINVAL;
+    pr[i] = DualProblem{q.A, q.xr, q.xc, q.yr, q.yc, q.m, q.row_accumulate != 0, q.col_accumulate != 0};
+  }
+  if (getenv("CATT_FUSED_ND") != nullptr) return CATT_EINVAL;  // the peer form is the single-read kernel's
+  PeerLaunch pl{p};
+  return launch_fused_group(false, pr, count, N, nullptr, static_cast<cudaStream_t>(stream), &pl);
 }
 
 extern "C" catt_status catt_dual(const float* A, const float* xr, const float* xc, float* yr, float* yc, int64_t m,

@@ -101,6 +101,15 @@ def atax_rowshard_peer(A_g, x, peer, tmp_g=None, y=None):
     return catt.atax_peer(A_g, x, peer, tmp_g, y)
 
 
+def bicg_mvt_rowshard_peer(problems, peer):
+    """The grouped single-read step (catt_dual_group_peer) on this rank's rows
+    of every problem: row outputs local, column outputs (BICG's s, MVT's x2)
+    summed over ranks inside the kernel through peer memory (no NCCL call),
+    bit-identical on all ranks. `peer` from peer_setup(n * len(problems))."""
+    catt.dual_group_peer(problems, peer)
+    return problems
+
+
 def bicg_rowshard(A_g, p, r_g, q_g=None, s=None, k1=None, k2=None, group=None, ops=CudaOps):
     """s = sum over ranks of A_g^T r_g (k1); q_g = A_g p (k2)."""
     import torch

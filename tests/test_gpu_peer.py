@@ -1,5 +1,6 @@
-"""Row-sharded ATAX with the A^T partials all-reduced inside the fused kernel
-through peer memory (catt_atax_peer). This run has one GPU,
+"""Row-sharded ATAX (catt_atax_peer) and BICG + MVT (catt_dual_group_peer) with
+the A^T partials all-reduced inside the fused kernel through peer memory
+(SURVEY 8(e), 8(f) f4). This run has one GPU,
 so the two ranks are two processes on cuda:0 whose buffers are mapped into
 each other by CUDA IPC, exactly as on an NVLink box (where the stores cross
 NVLink). Exact-dyadic inputs make every summation order bit-identical, each
@@ -129,3 +130,120 @@ def test_atax_peer_processes_share_one_gpu(tmp_path, world, m, n):
         tmp = np.load(tmp_path / f"tmp{r}.npy")
         assert np.array_equal(tmp, np.load(tmp_path / f"tmpp{r}.npy"))
         assert _relerr(tmp, t64[r * rows:(r + 1) * rows]) <= TOL
+
+
+# ------------------------------------------------------------------ BICG + MVT (catt_dual_group_peer)
+def _bm_problem(m, n):
+    A = si.matrix(si.SEED_BICG, m, n)
+    B = si.matrix(si.SEED_MVT, m, n)
+    p, r = si.values(si.sub_seed(si.SEED_BICG, 1), n), si.values(si.sub_seed(si.SEED_BICG, 2), m)
+    y1, y2 = si.values(si.sub_seed(si.SEED_MVT, 1), n), si.values(si.sub_seed(si.SEED_MVT, 2), m)
+    x1, x2 = si.values(si.sub_seed(si.SEED_MVT, 3), m), si.values(si.sub_seed(si.SEED_MVT, 4), n)
+    return A, B, p, r, y1, y2, x1, x2
+
+
+def _bm_group(torch, A, B, p, r, y1, y2, x1, x2, lo, hi, acc=True):
+    T = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    q, s = torch.empty(hi - lo, device="cuda"), torch.empty(A.shape[1], device="cuda")
+    X1, X2 = T(x1[lo:hi]), T(x2 if acc else np.zeros_like(x2))
+    return [dict(A=T(A[lo:hi]), xr=T(p), xc=T(r[lo:hi]), yr=q, yc=s),
+            dict(A=T(B[lo:hi]), xr=T(y1), xc=T(y2[lo:hi]), yr=X1, yc=X2, row_accumulate=True,
+                 col_accumulate=acc)]
+
+
+def _bm_rank_main(rank, world, port, m, n, steps, out_dir):
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+    import paper_conf_icpp_kimhlsh19_b200 as catt
+    A, B, p, r, y1, y2, x1, x2 = _bm_problem(m, n)
+    rows = m // world
+    lo, hi = rank * rows, (rank + 1) * rows
+    peer = cdist.peer_setup(2 * n)
+    outs = []
+    for _ in range(steps):
+        g = _bm_group(torch, A, B, p, r, y1, y2, x1, x2, lo, hi)
+        cdist.bicg_mvt_rowshard_peer(g, peer)
+        torch.cuda.synchronize()
+        outs.append([t.cpu().numpy().copy() for t in (g[0]["yr"], g[0]["yc"], g[1]["yr"], g[1]["yc"])])
+    part = _bm_group(torch, A, B, p, r, y1, y2, x1, x2, lo, hi, acc=False)   # this rank's partials, no exchange
+    catt.dual_group(part)
+    torch.cuda.synchronize()
+    for k, name in enumerate(("q", "s", "x1", "x2")):
+        np.save(os.path.join(out_dir, f"{name}{rank}.npy"), np.stack([o[k] for o in outs]))
+    np.save(os.path.join(out_dir, f"ps{rank}.npy"), part[0]["yc"].cpu().numpy())
+    np.save(os.path.join(out_dir, f"px2{rank}.npy"), part[1]["yc"].cpu().numpy())
+    np.save(os.path.join(out_dir, f"err{rank}.npy"), np.array([peer.timed_out()]))
+    dist.barrier()
+    peer.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+def test_bicg_mvt_peer_single_rank_equals_grouped_launch():
+    import torch
+    import paper_conf_icpp_kimhlsh19_b200 as catt
+    m, n = 900, 1028
+    args = _bm_problem(m, n)
+    ref = _bm_group(torch, *args, 0, m)
+    catt.dual_group(ref)
+    peer = catt.Peer(1, 0, 2 * n)
+    try:
+        for _ in range(3):                                   # both buffer parities
+            g = _bm_group(torch, *args, 0, m)
+            catt.dual_group_peer(g, peer)
+            torch.cuda.synchronize()
+            for a, b in zip(g, ref):
+                assert np.array_equal(a["yr"].cpu().numpy(), b["yr"].cpu().numpy())
+                assert np.array_equal(a["yc"].cpu().numpy(), b["yc"].cpu().numpy())
+        assert not peer.timed_out()
+        with pytest.raises(catt.CattError):                  # the buffer must hold both problems' columns
+            catt.dual_group_peer(_bm_group(torch, *args, 0, m), catt.Peer(1, 0, n))
+    finally:
+        peer.close()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world,m,n", [(2, 4096, 4096), (3, 771, 260), (2, 1024, 16384)])
+def test_bicg_mvt_peer_processes_share_one_gpu(tmp_path, world, m, n):
+    """The default bench step, row-sharded: s and x2 bit-identical on every
+    rank and launch, equal to the rank-order fp32 sum of the ranks' partials
+    (x2: then added to its initial value), within 1e-5 of the fp64 oracle;
+    q and x1 are the ranks' rows of the oracle's."""
+    import torch.multiprocessing as mp
+    import oracle
+    m -= m % world
+    ctx = mp.get_context("spawn")
+    port = _free_port()
+    procs = [ctx.Process(target=_bm_rank_main, args=(r, world, port, m, n, 3, str(tmp_path))) for r in range(world)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=240)
+    alive = [p for p in procs if p.is_alive()]
+    for p in alive:
+        p.kill()
+    assert not alive, "a rank hung"
+    assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
+    A, B, p, r, y1, y2, x1, x2 = _bm_problem(m, n)
+    q64, s64 = oracle.bicg(A, p, r, mode=oracle.SEQ_F64)
+    b1, b2 = oracle.bicg(B, y1, y2, mode=oracle.SEQ_F64)      # MVT's products (A need not be square here)
+    x164, x264 = x1.astype(np.float64) + b1, x2.astype(np.float64) + b2
+    ws, wx2 = np.load(tmp_path / "ps0.npy"), np.load(tmp_path / "px20.npy")
+    for g in range(1, world):
+        ws = (ws + np.load(tmp_path / f"ps{g}.npy")).astype(np.float32)
+        wx2 = (wx2 + np.load(tmp_path / f"px2{g}.npy")).astype(np.float32)
+    wx2 = (x2 + wx2).astype(np.float32)
+    assert _relerr(ws, s64) <= TOL and _relerr(wx2, x264) <= TOL
+    rows = m // world
+    for g in range(world):
+        assert not np.load(tmp_path / f"err{g}.npy")[0]
+        for s_, x2_ in zip(np.load(tmp_path / f"s{g}.npy"), np.load(tmp_path / f"x2{g}.npy")):
+            assert np.array_equal(s_, ws) and np.array_equal(x2_, wx2)
+        for q_ in np.load(tmp_path / f"q{g}.npy"):
+            assert _relerr(q_, q64[g * rows:(g + 1) * rows]) <= TOL
+        for x1_ in np.load(tmp_path / f"x1{g}.npy"):
+            assert _relerr(x1_, x164[g * rows:(g + 1) * rows]) <= TOL
