@@ -112,14 +112,64 @@ __global__ void __launch_bounds__(kStatWarps * 32) corr_stats_rows_kernel(float*
   if (j >= m) return;
   float* buf = s_row + int64_t(w) * n;
   float* row = rowsT + j * n;
-  for (int64_t i = lane; i < n; i += 32) buf[i] = row[i];
+  {
+    // the row into shared memory with 16 loads in flight per lane
+    int64_t i = lane;
+    for (; i + 32 * 15 < n; i += 32 * 16) {
+      float v[16];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) v[u] = row[i + 32 * u];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) buf[i + 32 * u] = v[u];
+    }
+    for (; i < n; i += 32) buf[i] = row[i];
+  }
   __syncwarp();
   const float fn = float(n), eps = 0.005f;
   float mu = 0.0f, sd = 0.0f;
   if (lane == 0) {
-    for (int64_t i = 0; i < n; ++i) mu = __fadd_rn(mu, buf[i]);
+    // the same two sequential chains; the loads go 32 values ahead of the
+    // adds (8 x LDS.128 per batch when the rows are 16-byte aligned), so each
+    // chain runs at the add latency rather than the load latency
+    int64_t i = 0;
+    if ((n & 3) == 0) {
+      const float4* b4 = reinterpret_cast<const float4*>(buf);
+      for (; i + 32 <= n; i += 32) {
+        float4 v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = b4[i / 4 + u];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          mu = __fadd_rn(mu, v[u].x);
+          mu = __fadd_rn(mu, v[u].y);
+          mu = __fadd_rn(mu, v[u].z);
+          mu = __fadd_rn(mu, v[u].w);
+        }
+      }
+    }
+    for (; i < n; ++i) mu = __fadd_rn(mu, buf[i]);
     mu = __fdiv_rn(mu, fn);
-    for (int64_t i = 0; i < n; ++i) {
+    i = 0;
+    if ((n & 3) == 0) {
+      const float4* b4 = reinterpret_cast<const float4*>(buf);
+      for (; i + 32 <= n; i += 32) {
+        float4 v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = b4[i / 4 + u];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          float d = __fsub_rn(v[u].x, mu);
+          sd = fmaf(d, d, sd);
+          d = __fsub_rn(v[u].y, mu);
+          sd = fmaf(d, d, sd);
+          d = __fsub_rn(v[u].z, mu);
+          sd = fmaf(d, d, sd);
+          d = __fsub_rn(v[u].w, mu);
+          sd = fmaf(d, d, sd);
+        }
+      }
+    }
+    for (; i < n; ++i) {
       const float d = __fsub_rn(buf[i], mu);
       sd = fmaf(d, d, sd);
     }
