@@ -5,7 +5,8 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict] [--set3]   (--set3: the third held-out set, after R24)"""
+usage: python tools/heldout2_study.py [--predict] [--set3|--set4]   (--set3: the third held-out set, after
+R24; --set4: the fourth, testing the candidate R25)"""
 import json
 import os
 import statistics
@@ -41,6 +42,19 @@ CASES3 = [
     ("syrk literal 1024", P(catt.K_SYRK, n=1024, k=1024), "literal", [(512, 228), (128, 164)]),
 ]
 
+# Fourth held-out set (after R24; tests the candidate R25 before it enters the
+# library): launches of 512- and 1024-thread CTAs where R25 (TLP floor of 16
+# warps per SM for CTAs of >= 16 warps, 8 otherwise) and the library's rule
+# pick differently, plus four where they agree
+CASES4 = [
+    ("gesummv literal 8192", P(catt.K_GESUMMV, n=8192), "literal", [(1024, 228), (512, 196), (512, 228), (512, 100)]),
+    ("atax1 literal 65536x16384", P(catt.K_ATAX_1, m=65536, n=16384), "literal", [(512, 196), (1024, 228), (512, 228)]),
+    ("mvt1 literal 8192", P(catt.K_MVT_1, n=8192), "literal", [(1024, 196), (1024, 228), (512, 228), (1024, 132)]),
+    ("bicg2 literal m=131072 n=128", P(catt.K_BICG_2, m=131072, n=128), "literal", [(1024, 196), (512, 228), (1024, 164)]),
+    ("bicg2 literal m=32768 n=1024", P(catt.K_BICG_2, m=32768, n=1024), "literal", [(1024, 228), (512, 196)]),
+    ("syr2k literal 1024 wide", P(catt.K_SYR2K, n=1024, k=1024), "literal", [(1024, 228)]),
+]
+
 
 def picks(prob, var, cta, carve):
     b200 = catt.hw_query() if catt_gpu() else catt.hw_b200()
@@ -49,7 +63,9 @@ def picks(prob, var, cta, carve):
     r23 = catt.Hw.from_dict(r18.as_dict())
     r23.min_retouch, r23.min_reuse_trip = 16, 128
     out = {}
-    for name, hw in (("b200", b200), ("r23", r23), ("r18", r18), ("paper", catt.paper_rule(b200))):
+    r25 = catt.Hw.from_dict(b200.as_dict())
+    r25.min_warps_sm = 16 if cta // 32 >= 16 else 8
+    for name, hw in (("b200", b200), ("r23", r23), ("r18", r18), ("paper", catt.paper_rule(b200)), ("r25", r25)):
         launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var)
         t, r = catt.plan(prob, launch, hw)
         W, T = r["base_warps"], r["base_ctas"]
@@ -70,7 +86,8 @@ def catt_gpu():
 def main():
     predict = "--predict" in sys.argv
     third = "--set3" in sys.argv
-    cases = CASES3 if third else CASES
+    fourth = "--set4" in sys.argv
+    cases = CASES4 if fourth else CASES3 if third else CASES
     if predict:
         for name, prob, var, launches in cases:
             for cta, carve in launches:
@@ -143,12 +160,14 @@ def main():
                        b200=pk["b200"], r23=pk["r23"], r18=pk["r18"], paper=pk["paper"], best=list(best),
                        best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
                        **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3)
-                          for k in ("b200", "r23", "r18", "paper")},
+                          for k in ("b200", "r23", "r18", "paper", "r25")},
+                       r25=pk["r25"],
                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    json.dump(res, open("gpurun_out/heldout3_study.json" if third else "gpurun_out/heldout2_study.json", "w"), indent=1)
+    out = "heldout4" if fourth else "heldout3" if third else "heldout2"
+    json.dump(res, open(f"gpurun_out/{out}_study.json", "w"), indent=1)
 
 
 if __name__ == "__main__":
