@@ -32,7 +32,12 @@
  *   - An unresolvable footprint is a result flag, not an error.
  *   - fp32 row-major matrices; inputs and outputs must not alias.
  *   - CTA caps that use the per-SM counters assume capped kernels on one
- *     device do not run concurrently on different streams.
+ *     device do not run concurrently on different streams. The same holds
+ *     for FUSED launches (catt_dual*, catt_atax_peer): they share the
+ *     device's workspace and its grid-barrier / arrival-counter words, whose
+ *     expected values the library tracks per device in launch order (a
+ *     stream-captured single-read launch uses the self-resetting barrier
+ *     instead, so CUDA graphs replay correctly).
  */
 #ifndef CATT_H
 #define CATT_H
