@@ -586,6 +586,8 @@ class Atax(Workload):
         mat = rows * n * 4
         self.study = dict(name="atax1 tmp=A x (literal, row per thread)", prob=catt.problem(catt.K_ATAX_1, m=rows, n=n),
                           A=self.A, x=self.x, y=self.tmp, launches=[(1024, 196), (256, 228)])
+        # both loops in one kernel, a throttle per loop
+        self.kernel_study = dict(m=4096, n=4096, launches=[(1024, 196), (1024, 228), (512, 196)])
         if var == "fused_peer":
             # the A^T partials all-reduced inside the fused kernel through peer
             # memory: no NCCL call, one launch per step
@@ -832,6 +834,66 @@ def app_study(catt, torch, w, flush):
     return out
 
 
+def kernel_study(catt, torch, w, flush):
+    """Per-loop throttles inside ONE kernel: ATAX's two literal
+    loops in one cooperative kernel (catt_atax_onekernel). CATT gives each
+    loop its own warp gate (a1, a2) and the kernel one CTA cap m (the
+    tighter of the loops' caps); BFTT is the best single (a, m) for both
+    loops; the sweep covers every (a1, a2, m)."""
+    S = getattr(w, "kernel_study", None)
+    if not S:
+        return None
+    import seeded_inputs as si
+    mm, nn = S["m"], S["n"]
+    A = torch.empty(mm, nn, device="cuda")
+    catt.fill_hash(A, si.SEED_ATAX, offset=0)
+    x = torch.empty(nn, device="cuda")
+    catt.fill_hash(x, si.sub_seed(si.SEED_ATAX, 1))
+    tmp, y = torch.empty(mm, device="cuda"), torch.empty(nn, device="cuda")
+
+    def med(fn, reps=3):
+        ts = []
+        for _ in range(reps + 1):
+            flush()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        ts = sorted(ts[1:])
+        return ts[len(ts) // 2]
+
+    out = []
+    P = catt.problem
+    for cta, carve in S["launches"]:
+        launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
+        t1, r1 = catt.plan(P(catt.K_ATAX_1, m=mm, n=nn), launch, w.hw)
+        t2, r2 = catt.plan(P(catt.K_ATAX_2, m=mm, n=nn), launch, w.hw)
+        W = cta // 32
+        T = min(r1["base_ctas"], r2["base_ctas"])
+        divs = [d for d in range(W, 0, -1) if W % d == 0]
+        times = {}
+        for m in range(T, 0, -1):
+            for a1 in divs:
+                for a2 in divs:
+                    k1 = launch.copy(active_warps=a1, active_ctas=m if m < T else 0)
+                    k2 = catt.Throttle(active_warps=a2, active_ctas=m if m < T else 0)
+                    times[(a1, a2, m)] = med(lambda k1=k1, k2=k2: catt.atax_onekernel(A, x, tmp, y, k1=k1, k2=k2))
+        pick = (t1.active_warps or W, t2.active_warps or W, min(t1.active_ctas or T, t2.active_ctas or T))
+        bftt = min(((a, a, m) for a in divs for m in range(1, T + 1)), key=lambda k: times[k])
+        best = min(times, key=times.get)
+        full = (W, W, T)
+        out.append(dict(kernel=f"ATAX {mm}x{nn}, both literal loops in one kernel", cta_threads=cta, carveout_kb=carve,
+                        catt=list(pick), catt_ms=round(times[pick], 4), bftt=list(bftt), bftt_ms=round(times[bftt], 4),
+                        full_ms=round(times[full], 4), best=list(best), best_ms=round(times[best], 4),
+                        catt_speedup_over_bftt=round(times[bftt] / times[pick], 4),
+                        catt_speedup_over_full=round(times[full] / times[pick], 4),
+                        catt_over_best=round(times[pick] / times[best], 4),
+                        swept={f"{a1},{a2},{m}": round(v, 4) for (a1, a2, m), v in times.items()}))
+    return out
+
+
 def ncu_traffic(workload):
     """DRAM bytes per launch of the workload's dominant kernel from the committed ncu summary."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -1006,10 +1068,11 @@ def main():
         e2e = {"value": round(total_bytes / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(e2e_ms, 4),
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
 
-    study = app = None
+    study = app = kst = None
     if rank == 0 and not args.no_study:
         study = throttle_study(catt, torch, w, flush)
         app = app_study(catt, torch, w, flush)
+        kst = kernel_study(catt, torch, w, flush)
 
     # ---- roofline of the dominant loop
     dom = max((i for i in range(len(w.loops)) if w.loops[i].kind != "collective"), key=lambda i: loop_ms[i])
@@ -1109,6 +1172,7 @@ def main():
             "clocks": clk,
             "throttle_study": study,
             "bftt_vs_catt": app,
+            "per_loop_in_one_kernel": kst,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

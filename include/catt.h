@@ -263,6 +263,20 @@ catt_status catt_plan(const catt_problem* prob, const catt_throttle* launch, con
 catt_status catt_atax(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n,
                       const catt_throttle* k1, const catt_throttle* k2, void* stream);
 
+/* ATAX's two literal loops in ONE kernel with a warp-level throttle per loop
+ * (throttling applied "to individual loops in a kernel"; PF#1's
+ * loops take different factors): loop 1 (thread per row, tmp = A x) runs
+ * under k1->active_warps, then a grid barrier, then loop 2 (thread per
+ * column, y = A^T tmp) under k2->active_warps. The CTA size, carveout, CTA
+ * cap (one decision for the whole kernel; applied around each loop)
+ * and probe come from k1; k2 may only set active_warps and gate (a k2
+ * cta_threads or active_ctas that differs from k1's is CATT_EINVAL). LITERAL
+ * only; cooperative launch of ceil(max(m, n) / cta_threads) CTAs, which must
+ * all be resident (CATT_EUNSUPPORTED otherwise). Results bit-exact to the
+ * sequential oracle, as catt_atax's literal loops. */
+catt_status catt_atax_onekernel(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n,
+                                const catt_throttle* k1, const catt_throttle* k2, void* stream);
+
 /* BICG (Table 2, Table 3): s = A^T r (loop 1, k1) and q = A p
  * (loop 2, k2). A is nx x ny; p[ny], r[nx], q[nx], s[ny]; q, s overwritten. */
 catt_status catt_bicg(const float* A, const float* p, const float* r, float* q, float* s, int64_t nx, int64_t ny,

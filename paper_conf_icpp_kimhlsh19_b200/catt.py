@@ -187,6 +187,7 @@ def lib():
             "catt_peer_destroy": [V],
             "catt_atax_peer": [V, V, V, V, i64, i64, V, V],
             "catt_dual_group_peer": [P(DualProblem), i32, V, V],
+            "catt_atax_onekernel": [V, V, V, V, i64, i64, T, T, V],
             "catt_status_str": [ctypes.c_int],
             "catt_last_cuda_error": [],
             "catt_abi_version": [],
@@ -210,7 +211,7 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_kmeans_step",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
-            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_dual_group_peer", "catt_sm_partition_create",
+            "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_dual_group_peer", "catt_atax_onekernel", "catt_sm_partition_create",
             "catt_sm_partition_destroy"]
 
 
@@ -348,6 +349,19 @@ def atax(A, x, tmp=None, y=None, k1: Optional[Throttle] = None, k2: Optional[Thr
     y = torch.empty(n, device=A.device) if y is None else y
     _check(lib().catt_atax(_dev(A, "A"), _dev(x, "x"), _dev(tmp, "tmp"), _dev(y, "y"), m, n, _tp(k1), _tp(k2),
                            _stream()), "catt_atax")
+    return tmp, y
+
+
+def atax_onekernel(A, x, tmp=None, y=None, k1: Optional[Throttle] = None, k2: Optional[Throttle] = None):
+    """Both ATAX loops in one literal kernel, a warp throttle per loop
+    (catt_atax_onekernel): k1 = the launch and loop 1's gate, k2 = loop 2's
+    gate. Returns (tmp, y)."""
+    torch = _torch()
+    m, n = A.shape
+    tmp = torch.empty(m, device=A.device) if tmp is None else tmp
+    y = torch.empty(n, device=A.device) if y is None else y
+    _check(lib().catt_atax_onekernel(_dev(A, "A"), _dev(x, "x"), _dev(tmp, "tmp"), _dev(y, "y"), m, n, _tp(k1),
+                                     _tp(k2), _stream()), "catt_atax_onekernel")
     return tmp, y
 
 

@@ -259,6 +259,50 @@ __global__ void __launch_bounds__(1024, 2) col_thread_kernel(ColArgs a) {
   cta_exit(a.t);
 }
 
+// ---------------------------------------------------------------- ATAX in one literal kernel
+// Both ATAX loops in ONE kernel with a throttle per loop (throttling
+// "even within a kernel", applied "to individual loops"; PF#1's loops
+// get different factors): loop 1 (thread per row: tmp[i] = sum_j A[i][j]
+// x[j], memory-divergent) under warp gate t1, a grid barrier (cooperative
+// launch), loop 2 (thread per column: y[j] = sum_i A[i][j] tmp[i],
+// coalesced) under warp gate t2. The CTA-level cap is one decision for the
+// whole kernel, entered and left around each loop. Results are the
+// literal loops' (bit-exact to seq-fmaf).
+__global__ void __launch_bounds__(1024, 2) atax_onekernel_kernel(RowArgs r, Throttle t2) {
+  namespace cg = cooperative_groups;
+  __shared__ int slots;
+  gate_init(&slots, r.t);
+  __syncthreads();
+  const int64_t g = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  cta_enter(r.t);
+  throttled(r.t, &slots, [&]() {
+    if (g >= r.M) return;
+    const int64_t N = r.N;
+    const float* __restrict__ ar = r.A + g * N;
+    float acc = 0.0f;
+#pragma unroll 2
+    for (int64_t j = 0; j < N; ++j) acc = fmaf(ar[j], r.x[j], acc);
+    r.y[g] = acc;                                             // tmp
+  });
+  cta_exit(r.t);
+  __threadfence();
+  cg::this_grid().sync();
+  gate_init(&slots, t2);
+  __syncthreads();
+  cta_enter(t2);
+  throttled(t2, &slots, [&]() {
+    if (g >= r.N) return;
+    const int64_t N = r.N, M = r.M;
+    const float* __restrict__ tmp = r.y;
+    float acc = 0.0f;
+    const float* p = r.A + g;
+#pragma unroll 2
+    for (int64_t i = 0; i < M; ++i, p += N) acc = fmaf(*p, tmp[i], acc);
+    r.tmp[g] = acc;                                           // y
+  });
+  cta_exit(t2);
+}
+
 // ---------------------------------------------------------------- column, CTA per 32-column block (COOP)
 // Lane l owns column c0 + l; warp w sums rows w, w + NW, ...; the NW partial
 // sums are then added in warp order (deterministic).
@@ -624,6 +668,54 @@ extern "C" catt_status catt_atax(const float* A, const float* x, float* tmp, flo
   catt_status st = launch_row(A, nullptr, x, tmp, nullptr, m, n, 0.f, 0.f, EPI_STORE, k1, s);  // tmp = A x
   if (st != CATT_OK) return st;
   return launch_col(A, tmp, y, m, n, EPI_STORE, k2, s);                                        // y = A^T tmp
+}
+
+extern "C" catt_status catt_atax_onekernel(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n,
+                                           const catt_throttle* k1, const catt_throttle* k2, void* stream) {
+  if (check_common(m, n) != CATT_OK || m < 1 || n < 1 || !A || !x || !tmp || !y) return CATT_EINVAL;
+  if ((k1 && k1->variant != CATT_VAR_LITERAL) || (k2 && k2->variant != CATT_VAR_LITERAL)) return CATT_EINVAL;
+  const int threads = cta_threads_or(k1, 256);
+  // one launch: k2 may only choose its warp gate; CTA size, carveout, CTA
+  // cap and probe are the kernel's (k1's)
+  catt_throttle c2 = k1 ? *k1 : catt_throttle{};
+  if (!k1) {
+    c2.carveout_kb = -1;
+  }
+  if (k2) {
+    if ((k2->cta_threads && k2->cta_threads != threads) || (k2->active_ctas && k2->active_ctas != c2.active_ctas))
+      return CATT_EINVAL;
+    c2.active_warps = k2->active_warps;
+    c2.gate = k2->gate;
+  } else {
+    c2.active_warps = 0;
+  }
+  c2.probe = nullptr;
+  const void* f = (const void*)atax_onekernel_kernel;
+  RowArgs r{A, nullptr, x, tmp, y, m, n, 0.f, 0.f, Throttle{}};
+  Throttle t2{};
+  size_t dyn = 0, dyn2 = 0;
+  catt_status st = prepare_launch(f, k1, threads, 0, true, &r.t, &dyn);
+  if (st != CATT_OK) return st;
+  st = prepare_launch(f, &c2, threads, 0, true, &t2, &dyn2);
+  if (st != CATT_OK) return st;
+  int occ = 0;
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f, threads, dyn);
+  DevCtx* ctx = nullptr;
+  if ((st = dev_ctx(&ctx)) != CATT_OK) return st;
+  const int64_t grid = (std::max(m, n) + threads - 1) / threads;
+  if (e != cudaSuccess || occ < 1) {
+    record_cuda_error(e == cudaSuccess ? cudaErrorInvalidConfiguration : e);
+    return CATT_ECUDA;
+  }
+  if (grid > int64_t(occ) * ctx->hw.num_sms) return CATT_EUNSUPPORTED;  // the grid barrier needs every CTA resident
+  void* args[] = {&r, &t2};
+  e = cudaLaunchCooperativeKernel(f, dim3(unsigned(grid)), dim3(unsigned(threads)), args, dyn,
+                                  static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  return after_launch();
 }
 
 extern "C" catt_status catt_bicg(const float* A, const float* p, const float* r, float* q, float* s_out,

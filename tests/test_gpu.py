@@ -703,3 +703,32 @@ def test_sm_partition_errors():
         catt.SmPartition(0)
     with pytest.raises(catt.CattError):
         catt.SmPartition(10_000)
+
+
+# ------------------------------------------------------------------ ATAX in one kernel, a throttle per loop
+@pytest.mark.parametrize("m,n,k1,k2", [
+    (1000, 700, catt.Throttle(), catt.Throttle()),
+    (4096, 260, catt.Throttle(cta_threads=1024, active_warps=8, carveout_kb=196), catt.Throttle()),
+    (513, 2049, catt.Throttle(cta_threads=256, active_warps=2, carveout_kb=228), catt.Throttle(active_warps=8)),
+    (3000, 3000, catt.Throttle(cta_threads=256, active_warps=4, active_ctas=1, carveout_kb=228),
+     catt.Throttle(active_warps=1, active_ctas=1)),
+    (777, 1500, catt.Throttle(cta_threads=512, active_warps=4, gate=catt.GATE_BARRIER), catt.Throttle(active_warps=2)),
+], ids=repr)
+def test_atax_onekernel_per_loop_throttles_exact(m, n, k1, k2):
+    """Both literal loops in one cooperative kernel, each under its own warp
+    gate, the CTA cap for the whole kernel: bit-exact
+    to the sequential oracle whatever the throttles."""
+    A, x = si.matrix(1, m, n), si.values(101, n)
+    tmp_o, y_o = oracle.atax(A, x)
+    tmp, y = catt.atax_onekernel(dev(A), dev(x), k1=k1, k2=k2)
+    assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y), y_o)
+
+
+def test_atax_onekernel_rejects_a_second_launch_shape():
+    A, x = dev(si.matrix(1, 64, 64)), dev(si.values(101, 64))
+    with pytest.raises(catt.CattError):                      # loop 2 cannot change the CTA size
+        catt.atax_onekernel(A, x, k1=catt.Throttle(cta_threads=256), k2=catt.Throttle(cta_threads=512))
+    with pytest.raises(catt.CattError):                      # nor the kernel's CTA cap (P:357)
+        catt.atax_onekernel(A, x, k1=catt.Throttle(active_ctas=2), k2=catt.Throttle(active_ctas=1))
+    with pytest.raises(catt.CattError):                      # LITERAL only
+        catt.atax_onekernel(A, x, k1=catt.Throttle(variant="coop"))
