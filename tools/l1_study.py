@@ -31,6 +31,7 @@ for name in names:
     if not rows:
         continue
     w = bench.WORKLOADS[name](catt, torch, 0, 1, None)
+    parts = {}
     for r in rows:
         W, T = r["base"]
         launch = catt.Throttle(cta_threads=r["cta_threads"], carveout_kb=r["carveout_kb"], variant="literal")
@@ -38,7 +39,17 @@ for name in names:
         for label, (a, m) in picks:
             th = launch.copy(active_warps=a, active_ctas=m if m < T else 0)
             fn = bench.study_fn(catt, w, th)
-            cases.append((name, r["loop"], r["cta_threads"], r["carveout_kb"], label, [a, m], fn))
+            sms = r.get("sm_partition")
+            if sms:                                    # the row was measured on an SM partition (green context)
+                if sms not in parts:
+                    parts[sms] = catt.SmPartition(sms)
+
+                def fn(f=fn, p=parts[sms]):
+                    with torch.cuda.stream(p.stream):
+                        f()
+                    p.stream.synchronize()
+            cases.append((name, r["loop"] + (f" [{sms} SMs]" if sms else ""), r["cta_threads"], r["carveout_kb"],
+                          label, [a, m], fn))
     del w
     torch.cuda.empty_cache()
 torch.cuda.synchronize()
