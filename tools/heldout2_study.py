@@ -5,8 +5,8 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict] [--set3|--set4]   (--set3: the third held-out set, after
-R24; --set4: the fourth, testing the candidate R25)"""
+usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5]   (--set3: the third held-out set, after
+R24; --set4: the fourth, testing the candidate R25; --set5: the fifth, new shapes)"""
 import json
 import os
 import statistics
@@ -55,6 +55,23 @@ CASES4 = [
     ("syr2k literal 1024 wide", P(catt.K_SYR2K, n=1024, k=1024), "literal", [(1024, 228)]),
 ]
 
+# Fifth held-out set (no rule change under test): loop shapes and launches of
+# every literal family not studied before -- KMEANS assign at other feature /
+# centre counts, CTAs of 384, 640 and 768 threads (W = 12, 20, 24: divisors
+# that are not powers of two), other matrix sizes -- to check that the
+# library's rule generalises
+CASES5 = [
+    ("kmeans assign nf=16 k=8", P(catt.K_KMEANS, m=262144, n=16, k=8, ld=262144), "literal", [(256, 100), (512, 228)]),
+    ("kmeans assign nf=64 k=4", P(catt.K_KMEANS, m=131072, n=64, k=4, ld=131072), "literal", [(256, 32), (1024, 196)]),
+    ("atax1 literal 32768x2048", P(catt.K_ATAX_1, m=32768, n=2048), "literal", [(256, 196), (768, 228)]),
+    ("gesummv literal 4096", P(catt.K_GESUMMV, n=4096), "literal", [(384, 196), (1024, 100)]),
+    ("mvt1 literal 6000", P(catt.K_MVT_1, n=6000), "literal", [(512, 164), (256, 132)]),
+    ("syrk literal 1536", P(catt.K_SYRK, n=1536, k=1536), "literal", [(256, 196), (1024, 100)]),
+    ("syr2k literal 768", P(catt.K_SYR2K, n=768, k=768), "literal", [(256, 228)]),
+    ("bicg2 literal m=65536 n=384", P(catt.K_BICG_2, m=65536, n=384), "literal", [(640, 196)]),
+    ("kmeans transpose nf=48", P(catt.K_KMEANS_T, m=262144, n=48, ld=262144), "literal", [(256, 64), (384, 228)]),
+]
+
 
 def picks(prob, var, cta, carve):
     b200 = catt.hw_query() if catt_gpu() else catt.hw_b200()
@@ -87,7 +104,8 @@ def main():
     predict = "--predict" in sys.argv
     third = "--set3" in sys.argv
     fourth = "--set4" in sys.argv
-    cases = CASES4 if fourth else CASES3 if third else CASES
+    fifth = "--set5" in sys.argv
+    cases = CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
     if predict:
         for name, prob, var, launches in cases:
             for cta, carve in launches:
@@ -115,7 +133,14 @@ def main():
 
     res = []
     for name, prob, var, launches in cases:
-        if prob.loop == catt.K_KMEANS_T:
+        if prob.loop == catt.K_KMEANS:
+            npts, nf, ld, kc = prob.m, prob.n, prob.ld, prob.k
+            fm = torch.empty(nf * ld, device=dev)
+            catt.fill_hash(fm, 44)
+            cl = fm.view(nf, ld)[:, :kc].t().contiguous()          # centres = the first k points
+            memb = torch.empty(npts, dtype=torch.int32, device=dev)
+            make = lambda th: (lambda: catt.kmeans_assign(fm, ld, npts, nf, cl, memb, t=th))
+        elif prob.loop == catt.K_KMEANS_T:
             npts, nf, ld = prob.m, prob.n, prob.ld
             pm = torch.empty(npts * nf, device=dev)
             catt.fill_hash(pm, 41)
@@ -166,7 +191,7 @@ def main():
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    out = "heldout4" if fourth else "heldout3" if third else "heldout2"
+    out = "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
     json.dump(res, open(f"gpurun_out/{out}_study.json", "w"), indent=1)
 
 
