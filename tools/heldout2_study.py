@@ -5,8 +5,9 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5]   (--set3: the third held-out set, after
-R24; --set4: the fourth, testing the candidate R25; --set5: the fifth, new shapes)"""
+usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5|--set6]   (--set3: the third held-out set, after
+R24; --set4: the fourth, testing the candidate R25; --set5: the fifth, new shapes; --set6: the sixth, testing
+the candidate R26)"""
 import json
 import os
 import statistics
@@ -72,6 +73,27 @@ CASES5 = [
     ("kmeans transpose nf=48", P(catt.K_KMEANS_T, m=262144, n=48, ld=262144), "literal", [(256, 64), (384, 228)]),
 ]
 
+# Sixth held-out set: tests the candidate R26 (the TLP floor is the largest
+# warp count per SM not above 8 that the launch can reach, a | W times m <= T;
+# the library's floor of 8 rounds up to W when W = 12, 20 or 28), at CTAs of
+# 384, 640, 768 and 896 threads; six launches where the two rules differ and
+# six where they agree
+CASES6 = [
+    ("gesummv literal 4096", P(catt.K_GESUMMV, n=4096), "literal", [(384, 228), (384, 132)]),
+    ("atax1 literal 65536x2048", P(catt.K_ATAX_1, m=65536, n=2048), "literal", [(384, 196), (384, 228)]),
+    ("mvt1 literal 6000 w12", P(catt.K_MVT_1, n=6000), "literal", [(384, 196)]),
+    ("bicg2 literal m=65536 n=1024", P(catt.K_BICG_2, m=65536, n=1024), "literal", [(640, 228)]),
+    ("gesummv literal 8192 w20", P(catt.K_GESUMMV, n=8192), "literal", [(640, 196), (384, 196)]),
+    ("atax1 literal 32768x2048 w24", P(catt.K_ATAX_1, m=32768, n=2048), "literal", [(768, 196)]),
+    ("mvt1 literal 8192 w28", P(catt.K_MVT_1, n=8192), "literal", [(896, 196), (896, 228)]),
+    ("bicg2 literal m=131072 n=128 w12", P(catt.K_BICG_2, m=131072, n=128), "literal", [(384, 228)]),
+]
+
+
+def r26_floor(W, T):
+    """R26's TLP floor: the largest a * m <= 8 with a | W and m <= T."""
+    return max(a * m for a in range(1, W + 1) if W % a == 0 for m in range(1, T + 1) if a * m <= 8)
+
 
 def picks(prob, var, cta, carve):
     b200 = catt.hw_query() if catt_gpu() else catt.hw_b200()
@@ -82,7 +104,11 @@ def picks(prob, var, cta, carve):
     out = {}
     r25 = catt.Hw.from_dict(b200.as_dict())
     r25.min_warps_sm = 16 if cta // 32 >= 16 else 8
-    for name, hw in (("b200", b200), ("r23", r23), ("r18", r18), ("paper", catt.paper_rule(b200)), ("r25", r25)):
+    r26 = catt.Hw.from_dict(b200.as_dict())
+    _, base = catt.plan(prob, catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var), b200)
+    r26.min_warps_sm = r26_floor(base["base_warps"], base["base_ctas"])
+    for name, hw in (("b200", b200), ("r23", r23), ("r18", r18), ("paper", catt.paper_rule(b200)), ("r25", r25),
+                     ("r26", r26)):
         launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var)
         t, r = catt.plan(prob, launch, hw)
         W, T = r["base_warps"], r["base_ctas"]
@@ -105,7 +131,8 @@ def main():
     third = "--set3" in sys.argv
     fourth = "--set4" in sys.argv
     fifth = "--set5" in sys.argv
-    cases = CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
+    sixth = "--set6" in sys.argv
+    cases = CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
     if predict:
         for name, prob, var, launches in cases:
             for cta, carve in launches:
@@ -185,13 +212,13 @@ def main():
                        b200=pk["b200"], r23=pk["r23"], r18=pk["r18"], paper=pk["paper"], best=list(best),
                        best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
                        **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3)
-                          for k in ("b200", "r23", "r18", "paper", "r25")},
-                       r25=pk["r25"],
+                          for k in ("b200", "r23", "r18", "paper", "r25", "r26")},
+                       r25=pk["r25"], r26=pk["r26"],
                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    out = "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
+    out = "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
     json.dump(res, open(f"gpurun_out/{out}_study.json", "w"), indent=1)
 
 
