@@ -5,9 +5,9 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5|--set6]   (--set3: the third held-out set, after
+usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5|--set6|--set7]   (--set3: the third held-out set, after
 R24; --set4: the fourth, testing the candidate R25; --set5: the fifth, new shapes; --set6: the sixth, testing
-the candidate R26)"""
+the candidate R26; --set7: the seventh, testing the candidate R27)"""
 import json
 import os
 import statistics
@@ -89,6 +89,33 @@ CASES6 = [
     ("bicg2 literal m=131072 n=128 w12", P(catt.K_BICG_2, m=131072, n=128), "literal", [(384, 228)]),
 ]
 
+# Seventh held-out set: tests the candidate R27 (in the floor fallback -- no
+# pair at or above the TLP floor fits -- cap whole CTAs, (W, m) with the
+# smallest m such that floor <= W m <= 2 floor, when such an m exists, instead
+# of gating warps down to the floor), fitted on stored sweeps where it changed
+# 10 picks and lost none; new shapes at 320- to 512-thread CTAs
+CASES7 = [
+    ("gesummv literal 6144", P(catt.K_GESUMMV, n=6144), "literal", [(512, 228), (512, 196), (320, 196)]),
+    ("mvt1 literal 5120", P(catt.K_MVT_1, n=5120), "literal", [(512, 228), (512, 196)]),
+    ("atax1 literal 131072x1024", P(catt.K_ATAX_1, m=131072, n=1024), "literal", [(384, 228), (512, 228), (384, 196)]),
+    ("bicg2 literal m=98304 n=768", P(catt.K_BICG_2, m=98304, n=768), "literal", [(512, 228), (1024, 196)]),
+    ("atax1 literal 49152x4096", P(catt.K_ATAX_1, m=49152, n=4096), "literal", [(512, 228), (320, 228)]),
+    ("bicg2 literal m=131072 n=256 w12", P(catt.K_BICG_2, m=131072, n=256), "literal", [(384, 228)]),
+]
+
+
+def r27_pick(prob, launch, hw):
+    """R27 applied to the library's pick (see CASES7)."""
+    t, r = catt.plan(prob, launch, hw)
+    W, T = r["base_warps"], r["base_ctas"]
+    pick = [t.active_warps or W, t.active_ctas or T]
+    if (r["flags"] & catt.FIT_GUARDED) and pick != [W, T] and r["footprint_bytes"] > r["l1d_bytes"]:
+        floor = hw.min_warps_sm
+        ms = [m for m in range(1, T + 1) if floor <= W * m <= 2 * floor]
+        if ms:
+            pick = [W, min(ms)]
+    return pick
+
 
 def r26_floor(W, T):
     """R26's TLP floor: the largest a * m <= 8 with a | W and m <= T."""
@@ -115,6 +142,7 @@ def picks(prob, var, cta, carve):
         out[name] = [t.active_warps or W, t.active_ctas or T]
         out["base"], out["carveout_kb"] = [W, T], r["carveout_kb"]
         out["footprint"], out["l1d_lines"] = r["footprint_lines_full"], r["l1d_bytes"] // 128
+    out["r27"] = r27_pick(prob, catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var), b200)
     return out
 
 
@@ -132,7 +160,8 @@ def main():
     fourth = "--set4" in sys.argv
     fifth = "--set5" in sys.argv
     sixth = "--set6" in sys.argv
-    cases = CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
+    seventh = "--set7" in sys.argv
+    cases = CASES7 if seventh else CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
     if predict:
         for name, prob, var, launches in cases:
             for cta, carve in launches:
@@ -212,13 +241,13 @@ def main():
                        b200=pk["b200"], r23=pk["r23"], r18=pk["r18"], paper=pk["paper"], best=list(best),
                        best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
                        **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3)
-                          for k in ("b200", "r23", "r18", "paper", "r25", "r26")},
-                       r25=pk["r25"], r26=pk["r26"],
+                          for k in ("b200", "r23", "r18", "paper", "r25", "r26", "r27")},
+                       r25=pk["r25"], r26=pk["r26"], r27=pk["r27"],
                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    out = "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
+    out = "heldout7" if seventh else "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
     json.dump(res, open(f"gpurun_out/{out}_study.json", "w"), indent=1)
 
 
