@@ -132,12 +132,16 @@ typedef struct {
  * iterations; and never to fewer than min_warps_sm active warps per SM.
  * max_stream_pct (R24; 0 = off, <= 100): no throttle when more than that
  * percentage of a lane's bytes per iteration are streams L1 cannot serve
- * again (stores, loads without reuse). Paper mode ignores them. */
+ * again (stores, loads without reuse). cta_fallback (R27; 0 = off): when
+ * nothing at or above min_warps_sm fits and an SM holds several CTAs (T >= 2),
+ * cap whole CTAs -- (W, m) with the smallest m such that min_warps_sm <= W m
+ * <= 2 min_warps_sm -- instead of gating warps down to the floor. Paper mode
+ * ignores them. */
 typedef struct {
   int32_t num_sms, max_warps_sm, max_ctas_sm, regs_sm, reg_alloc_unit, warp_size;
   int32_t smem_alloc_unit, reserved_smem_cta, line_bytes, n_carveouts;
   int32_t min_warps_sm, divergent_lines;
-  int32_t min_retouch, min_reuse_trip, max_stream_pct, reserved_;
+  int32_t min_retouch, min_reuse_trip, max_stream_pct, cta_fallback;
   int32_t carveout_kb[CATT_MAX_CARVEOUTS];
   int32_t carveout_pct[CATT_MAX_CARVEOUTS];
   int64_t l1d_bytes[CATT_MAX_CARVEOUTS];
@@ -519,7 +523,8 @@ catt_status catt_dual_group_peer(const catt_dual_problem* probs, int32_t count, 
  * after the grid barrier, end) for CTAs < 1024. Copies the first n of the
  * 6144 u64 values (CTA-major) to host memory `out` (synchronous). */
 catt_status catt_fused_trace(uint64_t* out, int32_t n);
-/* ABI revision of this header: 2 (catt_hw gained min_retouch, min_reuse_trip, max_stream_pct). */
+/* ABI revision of this header: 3 (catt_hw's last reserved word became
+ * cta_fallback; 2 added min_retouch, min_reuse_trip, max_stream_pct). */
 int catt_abi_version(void);
 
 #ifdef __cplusplus

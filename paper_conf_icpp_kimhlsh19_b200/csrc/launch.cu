@@ -634,7 +634,7 @@ extern "C" const char* catt_status_str(catt_status s) {
 }
 
 extern "C" int catt_last_cuda_error(void) { return g_last_err; }
-extern "C" int catt_abi_version(void) { return 2; }
+extern "C" int catt_abi_version(void) { return 3; }
 
 // ------------------------------------------------------------ SM partition
 // Green context of >= min_sms SMs and a non-blocking stream in it (catt.h).

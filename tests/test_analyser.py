@@ -24,7 +24,7 @@ def test_library_loads_and_exports_every_declared_symbol():
     assert declared == set(catt.catt.EXPORTED)
     for name in declared:
         assert hasattr(L, name), name
-    assert L.catt_abi_version() == 2
+    assert L.catt_abi_version() == 3
 
 
 def test_struct_layouts_match_header():
@@ -91,7 +91,7 @@ def _rand_hw(rnd):
                 smem_alloc_unit=rnd.choice([128, 256]), reserved_smem_cta=rnd.choice([0, 1024]), line_bytes=128,
                 min_warps_sm=rnd.choice([0, 0, 4, 16]), divergent_lines=rnd.choice([0, 0, 2, 8]),
                 min_retouch=rnd.choice([0, 0, 4, 16]), min_reuse_trip=rnd.choice([0, 0, 8, 30]),
-                max_stream_pct=rnd.choice([0, 0, 25, 60]),
+                max_stream_pct=rnd.choice([0, 0, 25, 60]), cta_fallback=rnd.choice([0, 1]),
                 carveout_kb=carve, l1d_bytes=[rnd.randint(1, 200) * 128 for _ in carve])
 
 
@@ -353,3 +353,28 @@ def test_r24_stream_fraction_on_synthetic_loops():
     assert r["flags"] & catt.FIT_GUARDED                      # 33 % > 25 %
     r = plan([load, load2, dict(store, flags=catt.REF_STORE | catt.REF_NOT_L1)], hw)
     assert r["active_warps"] * r["active_ctas"] < r["base_warps"] * r["base_ctas"]
+
+
+def test_r27_cta_fallback():
+    """R27 on the library's own loops (B200 table): when nothing at or above
+    the 8-warp floor fits and an SM holds several CTAs, the fallback caps whole
+    CTAs -- (W, m), the smallest m with 8 <= W m <= 16 -- instead of gating
+    warps to the floor; with one CTA per SM, or with R27 off, the fallback is
+    the most throttled pair at the floor (R18). Held-out sets 6 and 7
+    (profiles/r1h6, r1h7): (12, 1) measured best where (4, 2) was 1.23-1.40x."""
+    b200 = catt.hw_b200()
+    assert b200.cta_fallback == 1
+    off = catt.Hw.from_dict(b200.as_dict())
+    off.cta_fallback = 0
+    cases = [  # problem, CTA threads, carveout, base, R27 pick, R18 pick
+        (catt.problem(catt.K_ATAX_1, m=131072, n=1024), 384, 228, (12, 3), (12, 1), (4, 2)),
+        (catt.problem(catt.K_ATAX_1, m=131072, n=1024), 512, 228, (16, 2), (16, 1), (8, 1)),
+        (catt.problem(catt.K_GESUMMV, n=6144), 512, 228, (16, 1), (8, 1), (8, 1)),      # T = 1: unchanged
+    ]
+    for prob, cta, carve, base, want, want_off in cases:
+        for hw, w in ((b200, want), (off, want_off)):
+            t, r = catt.plan(prob, catt.Throttle(cta_threads=cta, carveout_kb=carve), hw)
+            W, T = r["base_warps"], r["base_ctas"]
+            assert (W, T) == base
+            assert (t.active_warps or W, t.active_ctas or T) == w
+            assert r["flags"] & catt.FIT_GUARDED
