@@ -5,9 +5,10 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5|--set6|--set7]   (--set3: the third held-out set, after
+usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5|--set6|--set7|--set8]   (--set3: the third held-out set, after
 R24; --set4: the fourth, testing the candidate R25; --set5: the fifth, new shapes; --set6: the sixth, testing
-the candidate R26; --set7: the seventh, testing the candidate R27)"""
+the candidate R26; --set7: the seventh, testing the candidate R27; --set8: the
+eighth, R27 as adopted)"""
 import json
 import os
 import statistics
@@ -103,6 +104,19 @@ CASES7 = [
     ("bicg2 literal m=131072 n=256 w12", P(catt.K_BICG_2, m=131072, n=256), "literal", [(384, 228)]),
 ]
 
+# Eighth held-out set: the library's rule (with R27 for T >= 2) against the
+# same rule without R27, on launches with several CTAs per SM where the floor
+# fallback applies and W = 12 or 16 (the only CTA sizes where the two differ
+# under the 8-warp floor); recorded before measuring
+CASES8 = [
+    ("bicg2 literal m=163840 n=512", P(catt.K_BICG_2, m=163840, n=512), "literal", [(512, 228), (384, 228)]),
+    ("bicg2 literal m=131072 n=512 w12", P(catt.K_BICG_2, m=131072, n=512), "literal", [(384, 196), (384, 228)]),
+    ("atax1 literal 196608x256", P(catt.K_ATAX_1, m=196608, n=256), "literal", [(512, 196), (384, 228), (512, 228)]),
+    ("bicg2 literal m=262144 n=128", P(catt.K_BICG_2, m=262144, n=128), "literal", [(512, 164), (512, 228)]),
+    ("atax1 literal 131072x640", P(catt.K_ATAX_1, m=131072, n=640), "literal", [(512, 196), (512, 228)]),
+    ("bicg2 literal m=98304 n=1024 w12", P(catt.K_BICG_2, m=98304, n=1024), "literal", [(384, 228)]),
+]
+
 
 def r27_pick(prob, launch, hw):
     """R27 applied to the library's pick (see CASES7)."""
@@ -131,11 +145,13 @@ def picks(prob, var, cta, carve):
     out = {}
     r25 = catt.Hw.from_dict(b200.as_dict())
     r25.min_warps_sm = 16 if cta // 32 >= 16 else 8
+    r24 = catt.Hw.from_dict(b200.as_dict())
+    r24.cta_fallback = 0
     r26 = catt.Hw.from_dict(b200.as_dict())
     _, base = catt.plan(prob, catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var), b200)
     r26.min_warps_sm = r26_floor(base["base_warps"], base["base_ctas"])
     for name, hw in (("b200", b200), ("r23", r23), ("r18", r18), ("paper", catt.paper_rule(b200)), ("r25", r25),
-                     ("r26", r26)):
+                     ("r26", r26), ("r24", r24)):
         launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var)
         t, r = catt.plan(prob, launch, hw)
         W, T = r["base_warps"], r["base_ctas"]
@@ -161,7 +177,8 @@ def main():
     fifth = "--set5" in sys.argv
     sixth = "--set6" in sys.argv
     seventh = "--set7" in sys.argv
-    cases = CASES7 if seventh else CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
+    eighth = "--set8" in sys.argv
+    cases = CASES8 if eighth else CASES7 if seventh else CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
     if predict:
         for name, prob, var, launches in cases:
             for cta, carve in launches:
@@ -241,13 +258,13 @@ def main():
                        b200=pk["b200"], r23=pk["r23"], r18=pk["r18"], paper=pk["paper"], best=list(best),
                        best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
                        **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3)
-                          for k in ("b200", "r23", "r18", "paper", "r25", "r26", "r27")},
-                       r25=pk["r25"], r26=pk["r26"], r27=pk["r27"],
+                          for k in ("b200", "r23", "r18", "paper", "r25", "r26", "r27", "r24")},
+                       r25=pk["r25"], r26=pk["r26"], r27=pk["r27"], r24=pk["r24"],
                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    out = "heldout7" if seventh else "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
+    out = "heldout8" if eighth else "heldout7" if seventh else "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
     json.dump(res, open(f"gpurun_out/{out}_study.json", "w"), indent=1)
 
 
