@@ -5,7 +5,7 @@ median of `reps`; the picks of the B200 rule (R18+R19+R23), of R18 alone and
 of the paper's rule are recorded BEFORE the timings (--predict prints them
 without a GPU). Rows carry their problem, so tools/rule_replay.py can re-plan
 them. Writes gpurun_out/heldout2_study.json.
-usage: python tools/heldout2_study.py [--predict] [--set3|--set4|--set5|--set6|--set7|--set8]   (--set3: the third held-out set, after
+usage: python tools/heldout2_study.py [--predict] [--set3|...|--set9]   (--set3: the third held-out set, after
 R24; --set4: the fourth, testing the candidate R25; --set5: the fifth, new shapes; --set6: the sixth, testing
 the candidate R26; --set7: the seventh, testing the candidate R27; --set8: the
 eighth, R27 as adopted)"""
@@ -117,6 +117,34 @@ CASES8 = [
     ("bicg2 literal m=98304 n=1024 w12", P(catt.K_BICG_2, m=98304, n=1024), "literal", [(384, 228)]),
 ]
 
+# Ninth held-out set: tests the candidate R28 (one CTA per SM, 8 < W < 16, W
+# even: the TLP floor becomes W / 2 instead of rounding up to W -- the W = 12
+# misses of held-out sets 5 and 6, where 6 warps were best) at CTAs of 320,
+# 384 and 448 threads (W = 10, 12, 14)
+CASES9 = [
+    ("gesummv literal 6144 w10", P(catt.K_GESUMMV, n=6144), "literal", [(320, 228)]),
+    ("mvt1 literal 8192 w10", P(catt.K_MVT_1, n=8192), "literal", [(320, 196)]),
+    ("atax1 literal 16384x4096 w10", P(catt.K_ATAX_1, m=16384, n=4096), "literal", [(320, 228)]),
+    ("bicg2 literal m=32768 n=2048 w10", P(catt.K_BICG_2, m=32768, n=2048), "literal", [(320, 196)]),
+    ("gesummv literal 6144 w12", P(catt.K_GESUMMV, n=6144), "literal", [(384, 196)]),
+    ("mvt1 literal 8192 w12", P(catt.K_MVT_1, n=8192), "literal", [(384, 228)]),
+    ("bicg2 literal m=40960 n=1024 w12", P(catt.K_BICG_2, m=40960, n=1024), "literal", [(384, 196)]),
+    ("gesummv literal 6144 w14", P(catt.K_GESUMMV, n=6144), "literal", [(448, 228)]),
+    ("atax1 literal 32768x1024 w14", P(catt.K_ATAX_1, m=32768, n=1024), "literal", [(448, 196)]),
+    ("mvt1 literal 6000 w14", P(catt.K_MVT_1, n=6000), "literal", [(448, 228)]),
+]
+
+
+def r28_pick(prob, launch, hw):
+    """The library's rule with R28 (see CASES9)."""
+    t, r = catt.plan(prob, launch, hw)
+    W, T = r["base_warps"], r["base_ctas"]
+    if T == 1 and 8 < W < 16 and W % 2 == 0:
+        h = catt.Hw.from_dict(hw.as_dict())
+        h.min_warps_sm = W // 2
+        t, r = catt.plan(prob, launch, h)
+    return [t.active_warps or W, t.active_ctas or T]
+
 
 def r27_pick(prob, launch, hw):
     """R27 applied to the library's pick (see CASES7)."""
@@ -159,6 +187,7 @@ def picks(prob, var, cta, carve):
         out["base"], out["carveout_kb"] = [W, T], r["carveout_kb"]
         out["footprint"], out["l1d_lines"] = r["footprint_lines_full"], r["l1d_bytes"] // 128
     out["r27"] = r27_pick(prob, catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var), b200)
+    out["r28"] = r28_pick(prob, catt.Throttle(cta_threads=cta, carveout_kb=carve, variant=var), b200)
     return out
 
 
@@ -178,7 +207,8 @@ def main():
     sixth = "--set6" in sys.argv
     seventh = "--set7" in sys.argv
     eighth = "--set8" in sys.argv
-    cases = CASES8 if eighth else CASES7 if seventh else CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
+    ninth = "--set9" in sys.argv
+    cases = CASES9 if ninth else CASES8 if eighth else CASES7 if seventh else CASES6 if sixth else CASES5 if fifth else CASES4 if fourth else CASES3 if third else CASES
     if predict:
         for name, prob, var, launches in cases:
             for cta, carve in launches:
@@ -258,13 +288,13 @@ def main():
                        b200=pk["b200"], r23=pk["r23"], r18=pk["r18"], paper=pk["paper"], best=list(best),
                        best_ms=round(times[best], 4), full_ms=round(times[(W, T)], 4),
                        **{f"{k}_over_best": round(times[tuple(pk[k])] / times[best], 3)
-                          for k in ("b200", "r23", "r18", "paper", "r25", "r26", "r27", "r24")},
-                       r25=pk["r25"], r26=pk["r26"], r27=pk["r27"], r24=pk["r24"],
+                          for k in ("b200", "r23", "r18", "paper", "r25", "r26", "r27", "r24", "r28")},
+                       r25=pk["r25"], r26=pk["r26"], r27=pk["r27"], r24=pk["r24"], r28=pk["r28"],
                        swept={f"{a},{m}": round(v, 4) for (a, m), v in times.items()})
             print(json.dumps({k: v for k, v in row.items() if k != "swept"}), flush=True)
             res.append(row)
     os.makedirs("gpurun_out", exist_ok=True)
-    out = "heldout8" if eighth else "heldout7" if seventh else "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
+    out = "heldout9" if ninth else "heldout8" if eighth else "heldout7" if seventh else "heldout6" if sixth else "heldout5" if fifth else "heldout4" if fourth else "heldout3" if third else "heldout2"
     json.dump(res, open(f"gpurun_out/{out}_study.json", "w"), indent=1)
 
 
