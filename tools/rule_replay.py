@@ -5,7 +5,7 @@ studies) has the time of every (a, m) at one launch. The problem of each loop
 name is rebuilt here, the analyser (catt_plan, no GPU) picks (a, m) under the
 rule, and the pick's time is divided by the best swept time.
 
-usage: python tools/rule_replay.py [--rule b200|r24|r23|r18|paper] [--set final|heldout|heldout2|heldout3|heldout4|heldout5|heldout6|heldout7|heldout8|partition|all] [-v]
+usage: python tools/rule_replay.py [--rule b200|r24|r23|r18|paper] [--set final|heldout|heldout2|heldout3|heldout4|heldout5|heldout6|heldout7|heldout8|heldout9|partition|all] [-v]
   b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24 + R27)
   r24   = the same without R27 (the floor fallback gates warps also with several CTAs per SM)
   r23   = R18 + R19 + R23 (re-touch and reuse-trip terms), as held-out study 2 tested it
@@ -53,6 +53,8 @@ FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["p
          "heldout7": ["profiles/r1h7/heldout7_study.json"],
          # several CTAs per SM, W = 12 / 16: R27 as adopted, pre-registered
          "heldout8": ["profiles/r1h8/heldout8_study.json"],
+         # one CTA per SM at W = 10 / 12 / 14, measured to test the candidate R28 (not adopted)
+         "heldout9": ["profiles/r1h9/heldout9_study.json"],
          # GESUMMV on SM partitions of 8 / 16 SMs (4 / 2 CTAs per SM), measured
          # after R24 was fixed: the CTA-level regime (SURVEY 8(d) [3])
          "partition": ["profiles/r1g/bench_gesummv.json"]}
@@ -123,10 +125,10 @@ def replay(rule, sets, verbose):
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--rule", default="b200", choices=["b200", "r24", "r23", "r18", "paper"])
-    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "partition", "all"])
+    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
-    sets = ["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "partition"] if a.set == "all" else [a.set]
+    sets = ["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition"] if a.set == "all" else [a.set]
     res = replay(a.rule, sets, a.v)
     for s in sets:
         rs = [x for x in res if x[0] == s]
