@@ -116,13 +116,16 @@ struct TileArgs {
   Throttle t;
 };
 
-template <int MODE, int TM, bool LEAN = false>
+template <int MODE, int TM, bool LEAN = false, bool DEEP = false>
 struct TileCfg {
   static constexpr int BM = 16 * TM;            // tile edge
   static constexpr int H = TM / 4;              // float4 groups per thread per dimension
   static constexpr int GS = BM / H;             // group stride: rows {g*GS + 4t + r}
   static constexpr int PITCH = BM + 4;          // transposed stage rows: 16-B aligned, store banks spread
-  static constexpr int BK = (MODE == MODE_SYR2K || LEAN) ? 8 : 16;
+  // DEEP: BK = 32 (SYR2K: 16) in dynamic shared memory, half the stage
+  // barriers and global-load phases per k
+  static constexpr int BK = DEEP ? ((MODE == MODE_SYR2K) ? 16 : 32) : (MODE == MODE_SYR2K || LEAN) ? 8 : 16;
+  static constexpr size_t SBYTES = size_t(2) * (MODE == MODE_SYR2K ? 4 : 2) * BK * PITCH * 4;
   static constexpr int FBUF = LEAN ? 1 : 2;     // register fragments: double-buffered unless LEAN
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int KQ = BK / 4;             // float4 per stage row
@@ -131,14 +134,21 @@ struct TileCfg {
 };
 
 // LEAN: BK = 8 and single-buffered fragments (fewer registers: 2 CTAs per SM)
-template <int MODE, int MINB, int TM = 8, bool LEAN = false>
+template <int MODE, int MINB, int TM = 8, bool LEAN = false, bool DEEP = false>
 __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
   constexpr bool TWO = MODE == MODE_SYR2K, GEMM = MODE == MODE_GEMM;
-  using Cfg = TileCfg<MODE, TM, LEAN>;
+  using Cfg = TileCfg<MODE, TM, LEAN, DEEP>;
   constexpr int BK = Cfg::BK, NA = Cfg::NA, KQ = Cfg::KQ, NV = Cfg::NV, BM = Cfg::BM, H = Cfg::H, GS = Cfg::GS;
   constexpr int PITCH = Cfg::PITCH;
   auto tile_off = [](int t, int r) { return (r / 4) * GS + t * 4 + (r % 4); };
-  __shared__ __align__(16) float S[2][NA][BK][PITCH];
+  float (*S)[NA][BK][PITCH];
+  if constexpr (DEEP) {
+    extern __shared__ __align__(16) float tiled_dyn[];
+    S = reinterpret_cast<float (*)[NA][BK][PITCH]>(tiled_dyn);
+  } else {
+    __shared__ __align__(16) float S_st[2][NA][BK][PITCH];
+    S = S_st;
+  }
   if (a.tri && blockIdx.x < blockIdx.y) return;  // strictly below the diagonal: mirrored by the caller
   cta_enter(a.t);
   const int tid = threadIdx.x;
@@ -421,6 +431,28 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
       tiled_kernel<MODE, 2, 8, true><<<grid, 256, dyn, s>>>(a);
       done = true;
     }
+  }
+  // DEEP stages (BK = 32 / 16): measured faster for SYR2K (1.123 -> 1.101 ms
+  // at 2048^2) and slower for SYRK (0.439 -> 0.470 ms) and CORR
+  // (profiles/r1deep/); CATT_TILED_DEEP=0/1 overrides (tools only)
+  static const int deep_env = [] {
+    const char* e = getenv("CATT_TILED_DEEP");
+    return e ? atoi(e) : -1;
+  }();
+  const bool deep = deep_env >= 0 ? deep_env == 1 : MODE == MODE_SYR2K;
+  if (!done && deep && !small && tiled_minb(MODE == MODE_SYR2K) == 1) {
+    const void* fd = (const void*)tiled_kernel<MODE, 1, 8, false, true>;
+    constexpr size_t sb = TileCfg<MODE, 8, false, true>::SBYTES;
+    size_t dyn2 = 0;
+    st = prepare_launch(fd, t, 256, sb, false, &a.t, &dyn2);
+    if (st != CATT_OK) return st;
+    cudaError_t e = cudaFuncSetAttribute(fd, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn2));
+    if (e != cudaSuccess) {
+      record_cuda_error(e);
+      return CATT_ECUDA;
+    }
+    tiled_kernel<MODE, 1, 8, false, true><<<grid, 256, dyn2, s>>>(a);
+    done = true;
   }
   if (done) {
   } else if (small)
