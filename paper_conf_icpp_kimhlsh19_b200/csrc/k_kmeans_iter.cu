@@ -22,6 +22,7 @@
 #include <algorithm>
 #include <cfloat>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 
 #include "f32x2.cuh"
@@ -172,6 +173,7 @@ struct AccArgs {
   long long* ctrl;
   int max_iter;
   long long max_changes;
+  int fence_all;  // every thread fences before the arrival (CATT_KM_FENCE_ALL; the earlier form)
 };
 
 __device__ void finalize_body(unsigned long long* acc, int k, int nf, float* clusters, long long* stats, int zero,
@@ -368,12 +370,15 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
   if (t == 0 && delta) atomicAdd(a.acc + K4 + k, (unsigned long long)delta);
   if (inexact) atomicAdd(a.acc + K4 + k + 1, (unsigned long long)inexact);
   if (a.fin_ctr) {
-    // last-CTA finalize: this CTA's sums are published (fence) before its
-    // arrival; the CTA that arrives last sees every CTA's sums (acq_rel)
+    // last-CTA finalize: this CTA's sums are published before its arrival
+    // (the barrier orders every thread's atomics before thread 0's fence and
+    // acq_rel arrival, the cooperative-groups grid-sync pattern); the CTA
+    // that arrives last sees every CTA's sums (acq_rel)
     __shared__ int s_last;
-    __threadfence();
+    if (a.fence_all) __threadfence();
     __syncthreads();
     if (t == 0) {
+      __threadfence();
       unsigned prev;
       asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(prev) : "l"(a.fin_ctr) : "memory");
       s_last = prev == gridDim.x - 1;
@@ -538,7 +543,7 @@ catt_status acc_launch(const float* feat, int64_t ld, int64_t npoints, int32_t n
   const int64_t tiles = (npoints + KT - 1) / KT;
   const int grid = int(std::min<int64_t>(tiles, int64_t(per_sm) * ctx->hw.num_sms));
   AccArgs a{feat, clusters, memb, reinterpret_cast<unsigned long long*>(acc), done, ld, npoints, nf, k,
-            nullptr, nullptr, nullptr, nullptr, 0, 0};
+            nullptr, nullptr, nullptr, nullptr, 0, 0, getenv("CATT_KM_FENCE_ALL") != nullptr};
   if (fin) {
     a.fin_ctr = ctx->gbar + 8;                                    // a counter word beside the grid barrier
     a.clusters_out = fin->clusters;
