@@ -1,7 +1,7 @@
 #!/bin/bash
 # full GPU suite + smoke + default bench line (consistency check after changes)
 export PYTHONPATH=.
-O=gpurun_out/r1chk3; mkdir -p $O
+O=gpurun_out/r1chk4; mkdir -p $O
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1; echo "smoke rc=$?" >> $O/smoke.txt
 timeout 1800 python -m pytest tests -m gpu -q > $O/pytest_gpu.txt 2>&1; echo "rc=$?" >> $O/pytest_gpu.txt
 timeout 900 python bench.py > $O/bench_default.json 2> $O/bench_default.err
