@@ -347,7 +347,7 @@ catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t npoints, i
  * (256-point shared-memory tiles, coalesced; no throttle). Bit-exact copy.
  *
  * Exact centroid sums. acc is a device int64 array of
- * catt_kmeans_acc_words(k, nf) = 4*k*nf + k + 2 words:
+ * catt_kmeans_acc_words(k, nf) = 4*k*nf + k + 3 words:
  *   acc[(c*nf + f)*4 + l], l < 4  limbs of the sum, over the points assigned to
  *                                 c, of feature f as the two's-complement
  *                                 128-bit integer v = x * 2^64. Each 128-bit
@@ -360,6 +360,11 @@ catt_status catt_kmeans_assign(const float* feat, int64_t ld, int64_t npoints, i
  *   acc[4*k*nf + k + 1]           inexact: feature values not representable
  *                                 (non-zero bits below 2^-64, |x| >= 2^31,
  *                                 subnormal, inf, NaN); 0 means S is exact
+ *   acc[4*k*nf + k + 2]           arrival counter of catt_kmeans_step's last-CTA
+ *                                 finalize (0 between launches; the launch that
+ *                                 uses it resets it). Kept in the caller's acc
+ *                                 so concurrent steps on different acc arrays
+ *                                 (streams) never share a counter.
  * All limbs are integer sums, so adding acc arrays (e.g. an integer
  * all-reduce across GPUs, each holding a shard of the points) gives exactly
  * the acc of the whole point set. Limits: nf <= 64, k <= 16, npoints < 2^31. */
@@ -386,7 +391,8 @@ catt_status catt_kmeans_finalize(int64_t* acc, int32_t k, int32_t nf, float* clu
  * then (the last CTA to finish, after every CTA's exact sums are in acc) the
  * work of catt_kmeans_finalize with zero_acc = 1. Bit-identical to the two
  * calls. stats (device int64[3], may be NULL) as in catt_kmeans_finalize.
- * Not for sharded runs: there the sums are all-reduced between the two. */
+ * Not for sharded runs: there the sums are all-reduced between the two.
+ * Concurrent steps (different streams) must use different acc arrays. */
 catt_status catt_kmeans_step(const float* feat, int64_t ld, int64_t npoints, int32_t nf, float* clusters, int32_t k,
                              int32_t* membership, int64_t* acc, int64_t* stats, void* stream);
 
@@ -460,6 +466,18 @@ catt_status catt_calibrate_l1(int device, int32_t pct, const int32_t* kb, int32_
 /* Number of registers / static shared bytes of the kernel a loop+launch uses. */
 catt_status catt_kernel_attrs(const catt_problem* prob, const catt_throttle* t, int32_t* regs, int32_t* static_smem);
 
+/* Eq 1-3 as the CUDA runtime computes it, for pinning the
+ * analyser's a1 step: cudaOccupancyMaxActiveBlocksPerMultiprocessor for the
+ * kernel a loop+launch uses, with that launch's CTA size and dynamic shared
+ * memory plus `extra_dyn_smem` bytes (a Fig 5 style pad), evaluated at the
+ * largest shared-memory carveout (Eq 1 divides the maximum shared memory; the
+ * function's carveout preference is restored afterwards). No grid bound.
+ * *ctas_per_sm receives the count; *dyn_smem (may be NULL) the dynamic bytes
+ * used. Synchronous, no launch. EINVAL on bad arguments, ECUDA on a runtime
+ * error. */
+catt_status catt_kernel_occupancy(const catt_problem* prob, const catt_throttle* t, int64_t extra_dyn_smem,
+                                  int32_t* ctas_per_sm, int64_t* dyn_smem);
+
 const char* catt_status_str(catt_status s);
 int catt_last_cuda_error(void);
 /* ------------------------------------------------------------ multi-GPU
@@ -478,7 +496,12 @@ int catt_last_cuda_error(void);
  * every rank holds bit-identical y. All ranks must call it in the same order
  * with equal shapes (equal shards give equal grids); each call is one launch
  * on `stream`, asynchronous. A wait for a peer longer than 10 s makes the
- * kernel give up; catt_peer_check (synchronous) reports it. Results: within
+ * kernel give up; a peer whose launch has another grid size (shards of
+ * different row counts below the co-resident CTA count) is detected at its
+ * first flag and the kernel gives up too (its column outputs are then
+ * undefined). catt_peer_check (synchronous) reports the error word:
+ * *timed_out = 0 (none), 1 (a wait timed out), 2 (grid mismatch between
+ * ranks); the word stays set until the peer object is destroyed. Results: within
  * 1e-5 of fp64, bit-exact on exact-dyadic inputs (the FUSED bar). Errors: CATT_EINVAL (arguments, a peer not opened, grids over
  * 1024 CTAs), CATT_ECUDA (IPC or launch), CATT_EUNSUPPORTED (n > 16384). */
 enum { CATT_PEER_HANDLE_BYTES = 64 };
@@ -523,8 +546,9 @@ catt_status catt_dual_group_peer(const catt_dual_problem* probs, int32_t count, 
  * after the grid barrier, end) for CTAs < 1024. Copies the first n of the
  * 6144 u64 values (CTA-major) to host memory `out` (synchronous). */
 catt_status catt_fused_trace(uint64_t* out, int32_t n);
-/* ABI revision of this header: 3 (catt_hw's last reserved word became
- * cta_fallback; 2 added min_retouch, min_reuse_trip, max_stream_pct). */
+/* ABI revision of this header: 4 (added catt_kernel_occupancy; 3: catt_hw's
+ * last reserved word became cta_fallback; 2 added min_retouch,
+ * min_reuse_trip, max_stream_pct). */
 int catt_abi_version(void);
 
 #ifdef __cplusplus

@@ -19,6 +19,13 @@ row starts in) do not count (reading R12).
 
 An event is one warp-level memory instruction: a tuple of (line, thread id)
 pairs, one per active lane.
+
+`program(b, w)` is the same loop body with every access labelled: a list of
+(instruction, is_store, bytes per lane, lanes) where lanes is the event tuple.
+It follows the kernels' source order (csrc/k_gemv.cu row_thread_kernel: x[j],
+then A[i*N + j], then B[i*N + j]) and includes the stores, which L1 does not
+keep (write-through, no allocate) and `events` therefore leaves out. The
+B200 decision rule's inputs are measured on it (oracle/b200_rule.py).
 """
 from __future__ import annotations
 
@@ -73,6 +80,20 @@ class RowKernel(Kernel):
                 ev.append(tuple((_line("x", j), i) for i in rows))
         return ev
 
+    def program(self, b, w):
+        rows = [i for i in (b * self.threads + t for t in self.lanes(b, w)) if i < self.M]
+        out = []
+        if not rows:
+            return out
+        nb = 4 * self.vec
+        for j in range(0, self.N, self.vec):
+            if self.with_tmp:
+                out.append(("tmp", False, 4, tuple((_line("tmp", i), i) for i in rows)))
+            out.append(("x", False, nb, tuple((_line("x", j), i) for i in rows)))
+            for X in self.matrices:
+                out.append((X, False, nb, tuple((_line(X, i * self.N + j), i) for i in rows)))
+        return out
+
 
 class ColKernel(Kernel):
     """Thread j owns column j (j < N):  for i < M: acc += A[i*N + j] * v[i]."""
@@ -93,6 +114,14 @@ class ColKernel(Kernel):
             ev.append(tuple((_line("A", i * self.N + j), j) for j in cols))
             ev.append(tuple((_line("v", i), j) for j in cols))
         return ev
+
+    def program(self, b, w):
+        cols = [j for j in (b * self.threads + t for t in self.lanes(b, w)) if j < self.N]
+        out = []
+        for i in range(self.M if cols else 0):
+            out.append(("A", False, 4, tuple((_line("A", i * self.N + j), j) for j in cols)))
+            out.append(("v", False, 4, tuple((_line("v", i), j) for j in cols)))
+        return out
 
 
 class SyrkKernel(Kernel):
@@ -123,6 +152,24 @@ class SyrkKernel(Kernel):
             ev.append(tuple((_line("a", j * self.Mk + k), (i, j)) for i, j in th))
         return ev
 
+    def _ij(self, b, w):
+        bx, by = b % self.gx, b // self.gx
+        th = []
+        for t in self.lanes(b, w):
+            tx, ty = t % self.bdim[0], t // self.bdim[0]
+            i, j = by * self.bdim[1] + ty, bx * self.bdim[0] + tx
+            if i < self.N and j < self.N:
+                th.append((i, j))
+        return th
+
+    def program(self, b, w):
+        th = self._ij(b, w)
+        out = []
+        for k in range(self.Mk if th else 0):
+            out.append(("a_i", False, 4, tuple((_line("a", i * self.Mk + k), (i, j)) for i, j in th)))
+            out.append(("a_j", False, 4, tuple((_line("a", j * self.Mk + k), (i, j)) for i, j in th)))
+        return out
+
 
 class Syr2kKernel(SyrkKernel):
     """PolyBench/GPU syr2k, block (32, 8), same thread map as syrk; for k < Mk:
@@ -143,6 +190,15 @@ class Syr2kKernel(SyrkKernel):
             for X, row in (("a", 0), ("b", 0), ("b", 1), ("a", 1)):
                 ev.append(tuple((_line(X, (i, j)[row] * self.Mk + k), (i, j)) for i, j in th))
         return ev
+
+    def program(self, b, w):
+        th = self._ij(b, w)
+        out = []
+        for k in range(self.Mk if th else 0):
+            for X, row in (("a", 0), ("b", 0), ("b", 1), ("a", 1)):
+                out.append((f"{X}_{'ij'[row]}", False, 4,
+                            tuple((_line(X, (i, j)[row] * self.Mk + k), (i, j)) for i, j in th)))
+        return out
 
 
 class GemmKernel(Kernel):
@@ -173,6 +229,20 @@ class GemmKernel(Kernel):
             ev.append(tuple((_line("b", k * self.nj + j), (i, j)) for i, j in th))
         return ev
 
+    def program(self, b, w):
+        bx, by = b % self.gx, b // self.gx
+        th = []
+        for t in self.lanes(b, w):
+            tx, ty = t % self.bdim[0], t // self.bdim[0]
+            i, j = by * self.bdim[1] + ty, bx * self.bdim[0] + tx
+            if i < self.ni and j < self.nj:
+                th.append((i, j))
+        out = []
+        for k in range(self.nk if th else 0):
+            out.append(("a", False, 4, tuple((_line("a", i * self.nk + k), (i, j)) for i, j in th)))
+            out.append(("b", False, 4, tuple((_line("b", k * self.nj + j), (i, j)) for i, j in th)))
+        return out
+
 
 class KmeansKernel(Kernel):
     """Rodinia kmeansPoint, feature-major: thread p (p < npoints):
@@ -195,6 +265,64 @@ class KmeansKernel(Kernel):
             for f in range(self.nf):
                 ev.append(tuple((_line("F", f * self.ld + p), p) for p in pts))
         return ev
+
+    def program(self, b, w):
+        return [("F", False, 4, ev) for ev in self.events(b, w)]
+
+
+class TransposeKernel(Kernel):
+    """Rodinia invert_mapping (KM's other loop, csrc/k_kmeans_iter.cu LITERAL):
+    thread p (p < npoints): for f < nf: out[f*ld + p] = in[p*nf + f]."""
+
+    def __init__(self, npoints, nf, ld, cta):
+        self.npoints, self.nf, self.ld = npoints, nf, ld
+        self.threads = cta
+        self.W = (cta + 31) // 32
+        self.nblocks = (npoints + cta - 1) // cta
+
+    def program(self, b, w):
+        pts = [p for p in (b * self.threads + t for t in self.lanes(b, w)) if p < self.npoints]
+        out = []
+        for f in range(self.nf if pts else 0):
+            out.append(("in", False, 4, tuple((_line("in", p * self.nf + f), p) for p in pts)))
+            out.append(("out", True, 4, tuple((_line("out", f * self.ld + p), p) for p in pts)))
+        return out
+
+    def events(self, b, w):
+        return [lanes for _, st, _, lanes in self.program(b, w) if not st]
+
+
+class CorrKernel(Kernel):
+    """PolyBench/GPU correlation, the thread-per-column loop (csrc/k_corr.cu
+    corr_thread_kernel): thread j1 (j1 < m): for j2 in j1+1 .. m-1: for i < n:
+    s += data[i*m + j1] * data[i*m + j2]; then symmat[j1*m + j2] = s and
+    symmat[j2*m + j1] = s. Lane j1 starts its j2 loop at j1 + 1, so the warp's
+    lanes are at different j2 in the same step."""
+
+    def __init__(self, m, n, cta):
+        self.m, self.n = m, n
+        self.threads = cta
+        self.W = (cta + 31) // 32
+        self.nblocks = (m + cta - 1) // cta
+
+    def program(self, b, w):
+        cols = [j for j in (b * self.threads + t for t in self.lanes(b, w)) if j < self.m]
+        out = []
+        if not cols:
+            return out
+        # the lanes run the j2 loop in lockstep from their own start: at step
+        # q lane j1 is at j2 = j1 + 1 + q, and is done once j2 reaches m
+        for q in range(self.m - min(cols) - 1):
+            act = [(j1, j1 + 1 + q) for j1 in cols if j1 + 1 + q < self.m]
+            for i in range(self.n):
+                out.append(("d_j1", False, 4, tuple((_line("d", i * self.m + j1), j1) for j1, j2 in act)))
+                out.append(("d_j2", False, 4, tuple((_line("d", i * self.m + j2), j1) for j1, j2 in act)))
+            out.append(("sym_12", True, 4, tuple((_line("sym", j1 * self.m + j2), j1) for j1, j2 in act)))
+            out.append(("sym_21", True, 4, tuple((_line("sym", j2 * self.m + j1), j1) for j1, j2 in act)))
+        return out
+
+    def events(self, b, w):
+        return [lanes for _, st, _, lanes in self.program(b, w) if not st]
 
 
 def simulate(kernel: Kernel, sm_blocks: Sequence[int], a: int, m: int, capacity: int) -> Dict:

@@ -180,6 +180,7 @@ def lib():
             "catt_fill_hash": [V, i64, u32, u64, i32, V],
             "catt_calibrate_l1": [ctypes.c_int, i32, P(i32), i32, P(f32)],
             "catt_kernel_attrs": [P(Problem), T, P(i32), P(i32)],
+            "catt_kernel_occupancy": [P(Problem), T, i64, P(i32), P(i64)],
             "catt_fused_trace": [P(u64), i32],
             "catt_peer_create": [i32, i32, i64, P(V), V],
             "catt_peer_open": [V, i32, V],
@@ -209,7 +210,8 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_atax", "catt_bicg", "catt_mvt", "catt_gesummv", "catt_syrk", "catt_syr2k", "catt_gemm", "catt_corr", "catt_kmeans_assign",
             "catt_kmeans_acc_words", "catt_kmeans_transpose", "catt_kmeans_accumulate", "catt_kmeans_finalize",
             "catt_kmeans_step",
-            "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs", "catt_status_str",
+            "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs",
+            "catt_kernel_occupancy", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
             "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_dual_group_peer", "catt_atax_onekernel", "catt_sm_partition_create",
             "catt_sm_partition_destroy"]
@@ -318,20 +320,43 @@ def kernel_attrs(prob: Problem, launch: Optional[Throttle] = None) -> Tuple[int,
     return regs.value, smem.value
 
 
+def kernel_occupancy(prob: Problem, launch: Optional[Throttle] = None, extra_dyn_smem: int = 0) -> Tuple[int, int]:
+    """cudaOccupancyMaxActiveBlocksPerMultiprocessor for the loop's kernel at the
+    largest carveout (catt_kernel_occupancy). Returns (CTAs per SM, dynamic bytes)."""
+    n, dyn = ctypes.c_int32(), ctypes.c_int64()
+    _check(lib().catt_kernel_occupancy(ctypes.byref(prob), ctypes.byref(launch) if launch else None,
+                                       int(extra_dyn_smem), ctypes.byref(n), ctypes.byref(dyn)),
+           "catt_kernel_occupancy")
+    return n.value, dyn.value
+
+
 # ------------------------------------------------------------------ device calls
 def _torch():
     import torch
     return torch
 
 
-def _dev(t, name, dtype=None):
+def _dev(t, name, dtype=None, n=0):
+    """Device pointer of t after the checks the C ABI cannot make: a contiguous
+    CUDA tensor of `dtype` on the current device with at least n elements
+    (the extent the entry point reads or writes; an undersized buffer would be
+    read or written out of bounds)."""
     torch = _torch()
     dtype = dtype or torch.float32
     if not isinstance(t, torch.Tensor) or not t.is_cuda:
         raise CattError(f"{name}: expected a CUDA tensor")
     if t.dtype != dtype or not t.is_contiguous():
         raise CattError(f"{name}: expected a contiguous {dtype} tensor")
+    if t.device.index != torch.cuda.current_device():
+        raise CattError(f"{name}: tensor on cuda:{t.device.index}, current device is cuda:{torch.cuda.current_device()}")
+    if t.numel() < n:
+        raise CattError(f"{name}: {t.numel()} elements, the call needs {n}")
     return ctypes.c_void_p(t.data_ptr())
+
+
+def _fm(ld, npoints, nf):
+    """Elements a feature-major [nf][ld] array must hold to reach point npoints - 1 of feature nf - 1."""
+    return (nf - 1) * ld + npoints if npoints > 0 and nf > 0 else 0
 
 
 def _stream():
@@ -348,7 +373,7 @@ def atax(A, x, tmp=None, y=None, k1: Optional[Throttle] = None, k2: Optional[Thr
     m, n = A.shape
     tmp = torch.empty(m, device=A.device) if tmp is None else tmp
     y = torch.empty(n, device=A.device) if y is None else y
-    _check(lib().catt_atax(_dev(A, "A"), _dev(x, "x"), _dev(tmp, "tmp"), _dev(y, "y"), m, n, _tp(k1), _tp(k2),
+    _check(lib().catt_atax(_dev(A, "A", n=m * n), _dev(x, "x", n=n), _dev(tmp, "tmp", n=m), _dev(y, "y", n=n), m, n, _tp(k1), _tp(k2),
                            _stream()), "catt_atax")
     return tmp, y
 
@@ -361,7 +386,7 @@ def atax_onekernel(A, x, tmp=None, y=None, k1: Optional[Throttle] = None, k2: Op
     m, n = A.shape
     tmp = torch.empty(m, device=A.device) if tmp is None else tmp
     y = torch.empty(n, device=A.device) if y is None else y
-    _check(lib().catt_atax_onekernel(_dev(A, "A"), _dev(x, "x"), _dev(tmp, "tmp"), _dev(y, "y"), m, n, _tp(k1),
+    _check(lib().catt_atax_onekernel(_dev(A, "A", n=m * n), _dev(x, "x", n=n), _dev(tmp, "tmp", n=m), _dev(y, "y", n=n), m, n, _tp(k1),
                                      _tp(k2), _stream()), "catt_atax_onekernel")
     return tmp, y
 
@@ -372,7 +397,7 @@ def bicg(A, p, r, q=None, s=None, k1: Optional[Throttle] = None, k2: Optional[Th
     nx, ny = A.shape
     q = torch.empty(nx, device=A.device) if q is None else q
     s = torch.empty(ny, device=A.device) if s is None else s
-    _check(lib().catt_bicg(_dev(A, "A"), _dev(p, "p"), _dev(r, "r"), _dev(q, "q"), _dev(s, "s"), nx, ny,
+    _check(lib().catt_bicg(_dev(A, "A", n=nx * ny), _dev(p, "p", n=ny), _dev(r, "r", n=nx), _dev(q, "q", n=nx), _dev(s, "s", n=ny), nx, ny,
                            _tp(k1), _tp(k2), _stream()), "catt_bicg")
     return q, s
 
@@ -380,7 +405,7 @@ def bicg(A, p, r, q=None, s=None, k1: Optional[Throttle] = None, k2: Optional[Th
 def mvt(A, y1, y2, x1, x2, k1: Optional[Throttle] = None, k2: Optional[Throttle] = None):
     """x1 += A y1, x2 += A^T y2, in place (catt_mvt). Returns (x1, x2)."""
     n = A.shape[0]
-    _check(lib().catt_mvt(_dev(A, "A"), _dev(y1, "y1"), _dev(y2, "y2"), _dev(x1, "x1"), _dev(x2, "x2"), n,
+    _check(lib().catt_mvt(_dev(A, "A", n=n * n), _dev(y1, "y1", n=n), _dev(y2, "y2", n=n), _dev(x1, "x1", n=n), _dev(x2, "x2", n=n), n,
                           _tp(k1), _tp(k2), _stream()), "catt_mvt")
     return x1, x2
 
@@ -391,7 +416,7 @@ def gesummv(A, B, x, alpha, beta, y=None, tmp=None, t: Optional[Throttle] = None
     n = A.shape[0]
     y = torch.empty(n, device=A.device) if y is None else y
     tmp = torch.empty(n, device=A.device) if tmp is None else tmp
-    _check(lib().catt_gesummv(_dev(A, "A"), _dev(B, "B"), _dev(x, "x"), _dev(y, "y"), _dev(tmp, "tmp"), n,
+    _check(lib().catt_gesummv(_dev(A, "A", n=n * n), _dev(B, "B", n=n * n), _dev(x, "x", n=n), _dev(y, "y", n=n), _dev(tmp, "tmp", n=n), n,
                               float(alpha), float(beta), _tp(t), _stream()), "catt_gesummv")
     return y, tmp
 
@@ -399,8 +424,8 @@ def gesummv(A, B, x, alpha, beta, y=None, tmp=None, t: Optional[Throttle] = None
 def rows(A, x, y, mode=ROWS_STORE, B=None, tmp=None, alpha=0.0, beta=0.0, t: Optional[Throttle] = None):
     """One row loop (catt_rows): y = A x (STORE), y += A x (ACCUM), or GESUMMV."""
     m, n = A.shape
-    _check(lib().catt_rows(_dev(A, "A"), _dev(B, "B") if B is not None else None, _dev(x, "x"), _dev(y, "y"),
-                           _dev(tmp, "tmp") if tmp is not None else None, m, n, float(alpha), float(beta), mode,
+    _check(lib().catt_rows(_dev(A, "A", n=m * n), _dev(B, "B", n=m * n) if B is not None else None, _dev(x, "x", n=n), _dev(y, "y", n=m),
+                           _dev(tmp, "tmp", n=m) if tmp is not None else None, m, n, float(alpha), float(beta), mode,
                            _tp(t), _stream()), "catt_rows")
     return y
 
@@ -408,7 +433,7 @@ def rows(A, x, y, mode=ROWS_STORE, B=None, tmp=None, alpha=0.0, beta=0.0, t: Opt
 def cols(A, v, y, accumulate=False, t: Optional[Throttle] = None):
     """One column loop (catt_cols): y (+)= A^T v."""
     m, n = A.shape
-    _check(lib().catt_cols(_dev(A, "A"), _dev(v, "v"), _dev(y, "y"), m, n, int(bool(accumulate)), _tp(t),
+    _check(lib().catt_cols(_dev(A, "A", n=m * n), _dev(v, "v", n=m), _dev(y, "y", n=n), m, n, int(bool(accumulate)), _tp(t),
                            _stream()), "catt_cols")
     return y
 
@@ -417,8 +442,8 @@ def dual(A, xr, yr, yc, xc=None, row_accumulate=False, col_accumulate=False, dep
          t: Optional[Throttle] = None):
     """Both loops in one pass over A (catt_dual): yr (+)= A xr; yc (+)= A^T (yr if dependent else xc)."""
     m, n = A.shape
-    _check(lib().catt_dual(_dev(A, "A"), _dev(xr, "xr"), _dev(xc, "xc") if xc is not None else None, _dev(yr, "yr"),
-                           _dev(yc, "yc"), m, n, int(bool(row_accumulate)), int(bool(col_accumulate)),
+    _check(lib().catt_dual(_dev(A, "A", n=m * n), _dev(xr, "xr", n=n), _dev(xc, "xc", n=m) if xc is not None else None, _dev(yr, "yr", n=m),
+                           _dev(yc, "yc", n=n), m, n, int(bool(row_accumulate)), int(bool(col_accumulate)),
                            int(bool(dependent)), _tp(t), _stream()), "catt_dual")
     return yr, yc
 
@@ -434,9 +459,9 @@ def _dual_array(problems):
     arr = (DualProblem * len(problems))()
     for i, p in enumerate(problems):
         m, n = p["A"].shape
-        arr[i] = DualProblem(_dev(p["A"], "A").value, _dev(p["xr"], "xr").value,
-                             _dev(p["xc"], "xc").value if p.get("xc") is not None else None,
-                             _dev(p["yr"], "yr").value, _dev(p["yc"], "yc").value, m, n,
+        arr[i] = DualProblem(_dev(p["A"], "A", n=m * n).value, _dev(p["xr"], "xr", n=n).value,
+                             _dev(p["xc"], "xc", n=m).value if p.get("xc") is not None else None,
+                             _dev(p["yr"], "yr", n=m).value, _dev(p["yc"], "yc", n=n).value, m, n,
                              int(bool(p.get("row_accumulate"))), int(bool(p.get("col_accumulate"))))
     return arr
 
@@ -454,7 +479,7 @@ def dual_group_peer(problems, peer: "Peer"):
 def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):
     """C = beta C + alpha A A^T in place (catt_syrk). Returns C."""
     n, m = A.shape
-    _check(lib().catt_syrk(_dev(A, "A"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t), _stream()),
+    _check(lib().catt_syrk(_dev(A, "A", n=n * m), _dev(C, "C", n=n * n), n, m, float(alpha), float(beta), _tp(t), _stream()),
            "catt_syrk")
     return C
 
@@ -462,7 +487,7 @@ def syrk(A, C, alpha, beta, t: Optional[Throttle] = None):
 def syr2k(A, B, C, alpha, beta, t: Optional[Throttle] = None):
     """C = beta C + alpha (A B^T + B A^T) in place (catt_syr2k). Returns C."""
     n, m = A.shape
-    _check(lib().catt_syr2k(_dev(A, "A"), _dev(B, "B"), _dev(C, "C"), n, m, float(alpha), float(beta), _tp(t),
+    _check(lib().catt_syr2k(_dev(A, "A", n=n * m), _dev(B, "B", n=n * m), _dev(C, "C", n=n * n), n, m, float(alpha), float(beta), _tp(t),
                             _stream()), "catt_syr2k")
     return C
 
@@ -482,10 +507,14 @@ class Peer:
         buf = ctypes.create_string_buffer(handle, PEER_HANDLE_BYTES)
         _check(lib().catt_peer_open(self.ptr, peer_rank, buf), "catt_peer_open")
 
-    def timed_out(self) -> bool:
+    def error(self) -> int:
+        """catt_peer_check's error word: 0 none, 1 a wait timed out, 2 the ranks launched different grids."""
         v = ctypes.c_int32()
         _check(lib().catt_peer_check(self.ptr, ctypes.byref(v)), "catt_peer_check")
-        return bool(v.value)
+        return v.value
+
+    def timed_out(self) -> bool:
+        return self.error() != 0
 
     def close(self):
         if self.ptr:
@@ -501,7 +530,7 @@ def atax_peer(A_g, x, peer: Peer, tmp_g=None, y=None):
     m, n = A_g.shape
     tmp_g = torch.empty(m, device=A_g.device) if tmp_g is None else tmp_g
     y = torch.empty(n, device=A_g.device) if y is None else y
-    _check(lib().catt_atax_peer(_dev(A_g, "A"), _dev(x, "x"), _dev(tmp_g, "tmp"), _dev(y, "y"), m, n, peer.ptr,
+    _check(lib().catt_atax_peer(_dev(A_g, "A", n=m * n), _dev(x, "x", n=n), _dev(tmp_g, "tmp", n=m), _dev(y, "y", n=n), m, n, peer.ptr,
                                 _stream()), "catt_atax_peer")
     return tmp_g, y
 
@@ -520,8 +549,9 @@ def kmeans_assign(feat, ld, npoints, nf, clusters, membership=None, t: Optional[
     torch = _torch()
     k = clusters.shape[0]
     membership = torch.empty(npoints, dtype=torch.int32, device=feat.device) if membership is None else membership
-    _check(lib().catt_kmeans_assign(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"), k,
-                                    _dev(membership, "membership", torch.int32), _tp(t), _stream()),
+    _check(lib().catt_kmeans_assign(_dev(feat, "feat", n=_fm(ld, npoints, nf)), ld, npoints, nf,
+                                    _dev(clusters, "clusters", n=k * nf), k,
+                                    _dev(membership, "membership", torch.int32, npoints), _tp(t), _stream()),
            "catt_kmeans_assign")
     return membership
 
@@ -530,7 +560,7 @@ def gemm(A, B, C, alpha, beta, t: Optional[Throttle] = None):
     """C = beta C + alpha A B in place (catt_gemm). Returns C."""
     ni, nk = A.shape
     nj = B.shape[1]
-    _check(lib().catt_gemm(_dev(A, "A"), _dev(B, "B"), _dev(C, "C"), ni, nj, nk, float(alpha), float(beta), _tp(t),
+    _check(lib().catt_gemm(_dev(A, "A", n=ni * nk), _dev(B, "B", n=nk * nj), _dev(C, "C", n=ni * nj), ni, nj, nk, float(alpha), float(beta), _tp(t),
                            _stream()), "catt_gemm")
     return C
 
@@ -548,8 +578,9 @@ def corr(data, mean=None, stdv=None, symmat=None, work=None, t: Optional[Throttl
     staged = t is not None and t.variant == VAR_STAGED
     if staged and work is None:
         work = mk(n * m)
-    wp = _dev(work, "work") if work is not None else None
-    _check(lib().catt_corr(_dev(data, "data"), n, m, _dev(mean, "mean"), _dev(stdv, "stdv"), _dev(symmat, "symmat"),
+    wp = _dev(work, "work", n=n * m) if work is not None else None
+    _check(lib().catt_corr(_dev(data, "data", n=n * m), n, m, _dev(mean, "mean", n=m), _dev(stdv, "stdv", n=m),
+                           _dev(symmat, "symmat", n=m * m),
                            wp, _tp(t), _stream()), "catt_corr")
     return symmat, mean, stdv
 
@@ -561,7 +592,7 @@ def kmeans_acc_words(k: int, nf: int) -> int:
 
 def kmeans_transpose(feat_pm, npoints, nf, out, ld, t: Optional[Throttle] = None):
     """out[f*ld + p] = feat_pm[p*nf + f] (catt_kmeans_transpose). Returns out."""
-    _check(lib().catt_kmeans_transpose(_dev(feat_pm, "in"), _dev(out, "out"), npoints, nf, ld, _tp(t), _stream()),
+    _check(lib().catt_kmeans_transpose(_dev(feat_pm, "in", n=npoints * nf), _dev(out, "out", n=_fm(ld, npoints, nf)), npoints, nf, ld, _tp(t), _stream()),
            "catt_kmeans_transpose")
     return out
 
@@ -569,17 +600,20 @@ def kmeans_transpose(feat_pm, npoints, nf, out, ld, t: Optional[Throttle] = None
 def kmeans_accumulate(feat, ld, npoints, nf, clusters, membership, acc):
     """Assignment + exact centroid sums into acc (catt_kmeans_accumulate)."""
     torch = _torch()
-    _check(lib().catt_kmeans_accumulate(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"),
-                                        clusters.shape[0], _dev(membership, "membership", torch.int32),
-                                        _dev(acc, "acc", torch.int64), _stream()), "catt_kmeans_accumulate")
+    _check(lib().catt_kmeans_accumulate(_dev(feat, "feat", n=_fm(ld, npoints, nf)), ld, npoints, nf,
+                                        _dev(clusters, "clusters", n=clusters.shape[0] * nf),
+                                        clusters.shape[0], _dev(membership, "membership", torch.int32, npoints),
+                                        _dev(acc, "acc", torch.int64, kmeans_acc_words(clusters.shape[0], nf)), _stream()),
+           "catt_kmeans_accumulate")
 
 
 def kmeans_finalize(acc, clusters, stats=None, zero_acc=True):
     """clusters := exact means from acc (catt_kmeans_finalize)."""
     torch = _torch()
     k, nf = clusters.shape
-    sp = _dev(stats, "stats", torch.int64) if stats is not None else None
-    _check(lib().catt_kmeans_finalize(_dev(acc, "acc", torch.int64), k, nf, _dev(clusters, "clusters"), sp,
+    sp = _dev(stats, "stats", torch.int64, 3) if stats is not None else None
+    _check(lib().catt_kmeans_finalize(_dev(acc, "acc", torch.int64, kmeans_acc_words(k, nf)), k, nf,
+                                      _dev(clusters, "clusters", n=k * nf), sp,
                                       int(bool(zero_acc)), _stream()), "catt_kmeans_finalize")
     return clusters
 
@@ -589,9 +623,11 @@ def kmeans_step(feat, ld, npoints, nf, clusters, membership, acc, stats=None):
     the last CTA rounds the new centres into clusters and zeroes acc."""
     torch = _torch()
     k = clusters.shape[0]
-    sp = _dev(stats, "stats", torch.int64) if stats is not None else None
-    _check(lib().catt_kmeans_step(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"), k,
-                                  _dev(membership, "membership", torch.int32), _dev(acc, "acc", torch.int64), sp,
+    sp = _dev(stats, "stats", torch.int64, 3) if stats is not None else None
+    _check(lib().catt_kmeans_step(_dev(feat, "feat", n=_fm(ld, npoints, nf)), ld, npoints, nf,
+                                  _dev(clusters, "clusters", n=k * nf), k,
+                                  _dev(membership, "membership", torch.int32, npoints),
+                                  _dev(acc, "acc", torch.int64, kmeans_acc_words(k, nf)), sp,
                                   _stream()), "catt_kmeans_step")
     return clusters
 
@@ -606,9 +642,11 @@ def kmeans(feat, ld, npoints, nf, clusters, membership=None, max_iter=500, max_c
     if ws is None:
         ws = torch.empty(kmeans_acc_words(k, nf) + 4, dtype=torch.int64, device=feat.device)
     it = ctypes.c_int32(0)
-    _check(lib().catt_kmeans(_dev(feat, "feat"), ld, npoints, nf, _dev(clusters, "clusters"), k,
-                             _dev(membership, "membership", torch.int32), max_iter, max_changes,
-                             _dev(ws, "ws", torch.int64), ctypes.byref(it), _stream()), "catt_kmeans")
+    _check(lib().catt_kmeans(_dev(feat, "feat", n=_fm(ld, npoints, nf)), ld, npoints, nf,
+                             _dev(clusters, "clusters", n=k * nf), k,
+                             _dev(membership, "membership", torch.int32, npoints), max_iter, max_changes,
+                             _dev(ws, "ws", torch.int64, kmeans_acc_words(k, nf) + 4), ctypes.byref(it), _stream()),
+           "catt_kmeans")
     return membership, it.value
 
 

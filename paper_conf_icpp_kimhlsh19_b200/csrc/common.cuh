@@ -49,11 +49,20 @@ __device__ __forceinline__ long long linear_cta() {
   return blockIdx.x + (long long)gridDim.x * (blockIdx.y + (long long)gridDim.y * blockIdx.z);
 }
 
+// The SM counter a CTA took in cta_enter, kept for cta_exit: %smid may change
+// during execution (e.g. after preemption), so cta_exit must not read it again.
+__device__ __forceinline__ unsigned& cta_slot() {
+  __shared__ unsigned slot;
+  return slot;
+}
+
 // CTA-level entry: one thread waits for a slot on its SM's counter.
 __device__ __forceinline__ void cta_enter(const Throttle& t) {
   if (t.cta_cap <= 0) return;
   if (linear_tid() == 0) {
-    int* c = t.sm_counter + smid();
+    const unsigned sm = smid();
+    cta_slot() = sm;
+    int* c = t.sm_counter + sm;
     unsigned ns = 64;
     while (true) {
       int v = atomicAdd(c, 1);
@@ -72,7 +81,7 @@ __device__ __forceinline__ void cta_exit(const Throttle& t) {
   __syncthreads();
   if (linear_tid() == 0) {
     __threadfence();
-    atomicSub(t.sm_counter + smid(), 1);
+    atomicSub(t.sm_counter + cta_slot(), 1);
   }
 }
 

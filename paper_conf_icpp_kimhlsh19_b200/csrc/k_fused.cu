@@ -130,11 +130,16 @@ __device__ __forceinline__ void grid_barrier_ordered(unsigned* bar, unsigned nbl
 // double-buffers slots and flags, so a rank one launch ahead never
 // overwrites data still being read (it cannot get two launches ahead: its
 // next wait needs this rank's next flags). A wait longer than 10 s sets
-// *peer_err and gives up instead of hanging the GPU.
+// *peer_err (1) and gives up instead of hanging the GPU; a source rank that
+// launched another grid (unequal shards) sets it to 2 at once.
 // The flag half of it: publish this CTA's partials, wait for the same CTA
 // index of every rank. Returns false (every thread) after a 10 s give-up.
 __device__ bool peer_flags(const FusedArgs& a) {
   const unsigned par = a.epoch & 1u;
+  // the flag carries the launch's grid size beside the epoch: the chunk ->
+  // CTA map is a function of the grid, so a rank whose grid differs (unequal
+  // shards of fewer rows than CTAs) is detected instead of summed silently
+  const unsigned tag = (a.epoch << 11) | (gridDim.x & 0x7FFu);
   // the CTA's partial stores are ordered before thread 0's system-scope fence
   // by the barrier (release cumulativity), so one fence per CTA publishes
   // them (CATT_PEER_FENCE_ALL: every thread fences, the earlier form)
@@ -145,7 +150,7 @@ __device__ bool peer_flags(const FusedArgs& a) {
     if (!a.fence_all) __threadfence_system();
     for (int p = 0; p < a.world; ++p) {
       unsigned* f = a.peer_flag[p] + (int64_t(par) * a.world + a.rank) * kPeerCtas + blockIdx.x;
-      asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(a.epoch) : "memory");
+      asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(tag) : "memory");
     }
     int ok = 1;
     const unsigned long long t0 = gtimer();
@@ -155,9 +160,14 @@ __device__ bool peer_flags(const FusedArgs& a) {
       unsigned v;
       while (true) {
         asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
-        if (v == a.epoch) break;
-        if (gtimer() - t0 > 10000000000ull) {
-          atomicExch(a.peer_err, 1u);
+        if (v == tag) break;
+        if ((v >> 11) == (tag >> 11)) {                 // this launch, another grid
+          atomicExch(a.peer_err, 2u);
+          ok = 0;
+          break;
+        }
+        if (*reinterpret_cast<volatile unsigned*>(a.peer_err) != 0u || gtimer() - t0 > 10000000000ull) {
+          atomicCAS(a.peer_err, 0u, 1u);                // another CTA's verdict stands
           ok = 0;
           break;
         }
@@ -415,7 +425,10 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
       bar_init(&full[s], 1);
       bar_init(&empty[s], NW);
     }
-    for (int s = 0; s < 2 * S; ++s) bar_init(&part_full[s], NW);
+    // every lane that writes a row partial (lanes 0, 8, 16, 24 of each
+    // consumer warp) arrives itself: its write is ordered before the
+    // producer's read by its own release-arrive / the producer's acquire-wait
+    for (int s = 0; s < 2 * S; ++s) bar_init(&part_full[s], NW * 4);
     fence_barrier_init();
   }
   auto issue = [&](int64_t c) {                                 // producer lane 0
@@ -536,11 +549,9 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
         const int r = lane >> 3;
         if ((lane & 7) == 0 && u0 + r < rows) rb[(u0 + r) * NW + warp] = f;
       }
+      if ((lane & 7) == 0) bar_arrive(&part_full[q]);
       __syncwarp();
-      if (lane == 0) {
-        bar_arrive(&part_full[q]);
-        bar_arrive(&empty[s]);
-      }
+      if (lane == 0) bar_arrive(&empty[s]);
     }
   }
   // column partials -> workspace (the producer's acc is zero and unused);
@@ -1126,7 +1137,7 @@ extern "C" catt_status catt_peer_check(catt_peer* p, int32_t* timed_out) {
     record_cuda_error(e);
     return CATT_ECUDA;
   }
-  *timed_out = int32_t(v != 0);
+  *timed_out = int32_t(v);
   return CATT_OK;
 }
 

@@ -545,7 +545,9 @@ catt_status acc_launch(const float* feat, int64_t ld, int64_t npoints, int32_t n
   AccArgs a{feat, clusters, memb, reinterpret_cast<unsigned long long*>(acc), done, ld, npoints, nf, k,
             nullptr, nullptr, nullptr, nullptr, 0, 0, getenv("CATT_KM_FENCE_ALL") != nullptr};
   if (fin) {
-    a.fin_ctr = ctx->gbar + 8;                                    // a counter word beside the grid barrier
+    // the arrival counter is the last word of the caller's acc (catt.h), so
+    // steps on different acc arrays never share it
+    a.fin_ctr = reinterpret_cast<unsigned*>(acc + catt_kmeans_acc_words(k, nf) - 1);
     a.clusters_out = fin->clusters;
     a.stats = fin->stats;
     a.ctrl = fin->ctrl;
@@ -569,7 +571,7 @@ bool acc_args_ok(int64_t ld, int64_t npoints, int32_t nf, int32_t k) {
 
 extern "C" int64_t catt_kmeans_acc_words(int32_t k, int32_t nf) {
   if (k < 1 || nf < 1) return 0;
-  return int64_t(k) * nf * 4 + k + 2;
+  return int64_t(k) * nf * 4 + k + 3;
 }
 
 extern "C" catt_status catt_kmeans_transpose(const float* in, float* out, int64_t npoints, int32_t nf, int64_t ld,

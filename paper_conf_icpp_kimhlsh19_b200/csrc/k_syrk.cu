@@ -404,6 +404,18 @@ static bool small_tiles(int64_t ni, int64_t nj) {
   return ((ni + 127) / 128) * ((nj + 127) / 128) < nsm;
 }
 
+// DEEP stages (BK = 32 / 16): measured faster for SYR2K (1.123 -> 1.101 ms
+// at 2048^2) and slower for SYRK (0.439 -> 0.470 ms) and CORR
+// (profiles/r1deep/); CATT_TILED_DEEP=0/1 overrides (tools only)
+template <int MODE>
+static bool tiled_deep() {
+  static const int deep_env = [] {
+    const char* e = getenv("CATT_TILED_DEEP");
+    return e ? atoi(e) : -1;
+  }();
+  return deep_env >= 0 ? deep_env == 1 : MODE == MODE_SYR2K;
+}
+
 template <int MODE>
 static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t s) {
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
@@ -432,24 +444,25 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
       done = true;
     }
   }
-  // DEEP stages (BK = 32 / 16): measured faster for SYR2K (1.123 -> 1.101 ms
-  // at 2048^2) and slower for SYRK (0.439 -> 0.470 ms) and CORR
-  // (profiles/r1deep/); CATT_TILED_DEEP=0/1 overrides (tools only)
-  static const int deep_env = [] {
-    const char* e = getenv("CATT_TILED_DEEP");
-    return e ? atoi(e) : -1;
-  }();
-  const bool deep = deep_env >= 0 ? deep_env == 1 : MODE == MODE_SYR2K;
-  if (!done && deep && !small && tiled_minb(MODE == MODE_SYR2K) == 1) {
+  if (!done && tiled_deep<MODE>() && !small && tiled_minb(MODE == MODE_SYR2K) == 1) {
     const void* fd = (const void*)tiled_kernel<MODE, 1, 8, false, true>;
     constexpr size_t sb = TileCfg<MODE, 8, false, true>::SBYTES;
-    size_t dyn2 = 0;
-    st = prepare_launch(fd, t, 256, sb, false, &a.t, &dyn2);
-    if (st != CATT_OK) return st;
-    cudaError_t e = cudaFuncSetAttribute(fd, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn2));
+    // the dynamic-size attribute first, so prepare_launch's occupancy query
+    // (for a CTA cap) sees the kernel as it will run
+    cudaError_t e = cudaFuncSetAttribute(fd, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sb));
     if (e != cudaSuccess) {
       record_cuda_error(e);
       return CATT_ECUDA;
+    }
+    size_t dyn2 = 0;
+    st = prepare_launch(fd, t, 256, sb, false, &a.t, &dyn2);
+    if (st != CATT_OK) return st;
+    if (dyn2 > sb) {                                           // a Fig 5 pad on top
+      e = cudaFuncSetAttribute(fd, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn2));
+      if (e != cudaSuccess) {
+        record_cuda_error(e);
+        return CATT_ECUDA;
+      }
     }
     tiled_kernel<MODE, 1, 8, false, true><<<grid, 256, dyn2, s>>>(a);
     done = true;
@@ -468,8 +481,16 @@ const void* syrk_func(int variant) {
   return variant == CATT_VAR_STAGED ? tiled_func<MODE_SYRK>() : (const void*)syrk_thread_kernel;
 }
 
+// the kernel a large (128 x 128 tile) STAGED SYR2K launch runs, and its
+// dynamic shared memory (catt_kernel_desc / catt_plan describe this kernel)
 const void* syr2k_func(int variant) {
-  return variant == CATT_VAR_STAGED ? tiled_func<MODE_SYR2K>() : (const void*)syr2k_thread_kernel;
+  if (variant != CATT_VAR_STAGED) return (const void*)syr2k_thread_kernel;
+  if (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) return (const void*)tiled_kernel<MODE_SYR2K, 1, 8, false, true>;
+  return tiled_func<MODE_SYR2K>();
+}
+
+int64_t syr2k_staged_dyn() {
+  return (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) ? int64_t(TileCfg<MODE_SYR2K, 8, false, true>::SBYTES) : 0;
 }
 
 // ---------------------------------------------------------------- GEMM

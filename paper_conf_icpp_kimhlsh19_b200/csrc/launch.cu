@@ -20,6 +20,7 @@ int row_tma_stage_bytes(int nmat, int rows, int boxes);
 int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
 const void* syr2k_func(int variant);
+int64_t syr2k_staged_dyn();
 const void* kmeans_func(int variant, int nf);
 int64_t kmeans_tma_smem(int nf, int k);
 const void* kmeans_t_func(int variant);
@@ -265,6 +266,47 @@ extern "C" catt_status catt_kernel_attrs(const catt_problem* prob, const catt_th
   return CATT_OK;
 }
 
+extern "C" catt_status catt_kernel_occupancy(const catt_problem* prob, const catt_throttle* t, int64_t extra_dyn_smem,
+                                             int32_t* ctas_per_sm, int64_t* dyn_smem) {
+  if (!prob || !ctas_per_sm || extra_dyn_smem < 0) return CATT_EINVAL;
+  catt_ref refs[8];
+  catt_loop_desc d;
+  catt_status st = catt_kernel_desc(prob, t, CATT_MODE_UNION, &d, refs, 8);
+  if (st != CATT_OK) return st;
+  const void* func = loop_func(*prob, variant_of(t));
+  cudaFuncAttributes fa;
+  cudaError_t e = cudaFuncGetAttributes(&fa, func);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  const int64_t dyn = int64_t(d.smem_per_cta) - int64_t(fa.sharedSizeBytes) + extra_dyn_smem;
+  if (dyn < 0) return CATT_EINVAL;
+  const int threads = d.block[0] * d.block[1] * d.block[2];
+  if (dyn > fa.maxDynamicSharedSizeBytes) {
+    e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn));
+    if (e != cudaSuccess) {
+      record_cuda_error(e);
+      return CATT_ECUDA;
+    }
+  }
+  e = cudaFuncSetAttribute(func, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  int n = 0;
+  if (e == cudaSuccess)
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessorWithFlags(&n, func, threads, size_t(dyn),
+                                                               cudaOccupancyDisableCachingOverride);
+  const cudaError_t e2 = cudaFuncSetAttribute(func, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                              fa.preferredShmemCarveout);
+  if (e == cudaSuccess) e = e2;
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  *ctas_per_sm = n;
+  if (dyn_smem) *dyn_smem = dyn;
+  return CATT_OK;
+}
+
 extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_throttle* t, int32_t mode,
                                         catt_loop_desc* out, catt_ref* refs, int32_t cap) {
   if (!prob || !out || !refs || cap < 8) return CATT_EINVAL;
@@ -414,6 +456,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->grid[0] = (N + 127) / 128;
       out->grid[1] = (N + 127) / 128;
       refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);
+      dyn = syr2k_staged_dyn();                                    // the DEEP stages (dynamic shared memory)
     } else {
       return CATT_EINVAL;
     }
@@ -634,7 +677,7 @@ extern "C" const char* catt_status_str(catt_status s) {
 }
 
 extern "C" int catt_last_cuda_error(void) { return g_last_err; }
-extern "C" int catt_abi_version(void) { return 3; }
+extern "C" int catt_abi_version(void) { return 4; }
 
 // ------------------------------------------------------------ SM partition
 // Green context of >= min_sms SMs and a non-blocking stream in it (catt.h).

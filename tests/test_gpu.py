@@ -467,15 +467,28 @@ def _concurrency(rec, W):
 
 
 @pytest.mark.parametrize("t,want", [
-    (catt.Throttle(), (8, 8)),
-    (catt.Throttle(active_warps=2), (2, 8)),
-    (catt.Throttle(active_warps=4, gate=catt.GATE_BARRIER), (4, 8)),
-    (catt.Throttle(active_warps=1, active_ctas=3), (1, 3)),
+    (catt.Throttle(carveout_kb=16), (8, 8)),
+    (catt.Throttle(active_warps=2, carveout_kb=16), (2, 8)),
+    (catt.Throttle(active_warps=4, gate=catt.GATE_BARRIER, carveout_kb=16), (4, 8)),
+    (catt.Throttle(active_warps=1, active_ctas=3, carveout_kb=16), (1, 3)),
     (catt.Throttle(active_ctas=2, cap=catt.CAP_SMEM_PAD, carveout_kb=64), (8, 2)),
+    (catt.Throttle(carveout_kb=8), (8, 7)),
 ], ids=repr)
 def test_residency_probe_enforces_throttle(t, want):
+    """a6 (Fig 4/5) and a1 (Eq 1-4): the measured concurrency equals the
+    throttle -- warps per CTA inside the loop and CTAs per SM inside the loop.
+    Full TLP co-schedules exactly T CTAs: 8 at the carveout Eq 4 picks (16 KB
+    for 8 CTAs of 1 KB reserved + 16 B), and 7 when the launch forces the 8 KB
+    option (7 x 1152 B fit, 8 do not) -- the model's T for that carveout."""
     # long rows so CTAs overlap in time; 148 SMs x 8 CTAs x 256 rows x 2 waves
     m, n = 148 * 8 * 256 * 2, 512
+    prob = catt.problem(catt.K_ATAX_1, m=m, n=n)
+    _, r = catt.plan(prob, catt.Throttle(carveout_kb=t.carveout_kb), catt.hw_query())
+    if t.cap != catt.CAP_SMEM_PAD:
+        assert r["base_ctas"] == {16: 8, 8: 7}[t.carveout_kb]       # the model's T at this carveout
+    if t.carveout_kb == 16 and not t.active_ctas:
+        _, r0 = catt.plan(prob, catt.Throttle(), catt.hw_query())
+        assert r0["carveout_kb"] == 16                     # Eq 4's own pick
     A = torch.empty(m * n, device="cuda")
     catt.fill_hash(A, 1)
     x = torch.ones(n, device="cuda")
@@ -486,20 +499,53 @@ def test_residency_probe_enforces_throttle(t, want):
     mw, mc = _concurrency(host(probe).astype(np.int64), 8)
     assert mw <= want[0] and mc <= want[1]
     assert mw == want[0]                                   # the slots are actually used
-    assert mc >= min(want[1], 2)
+    assert mc == want[1]                                   # ... and so are the CTA slots: T (or the cap) co-resident
 
 
-def test_plan_on_device_matches_occupancy_api():
+P_ = catt.problem
+OCC_CASES = [   # (problem, launch, extra dynamic smem): register-, smem-, warp- and CTA-slot-limited launches
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(), 0),                              # 8 warps: #TB_HW
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(cta_threads=384), 0),               # 12 warps: 64 // 12
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(cta_threads=1024), 0),
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(cta_threads=32), 0),                # 32-CTA slot limit
+    (P_(catt.K_ATAX_1, m=1 << 22, n=4096), catt.Throttle(variant="staged"), 0),              # row_tma: >= 128 regs + ring
+    (P_(catt.K_ATAX_1, m=1 << 22, n=4096), catt.Throttle(variant="staged", cta_threads=64), 0),
+    (P_(catt.K_GESUMMV, n=1 << 20), catt.Throttle(variant="staged"), 0),
+    (P_(catt.K_ATAX_2, m=4096, n=1 << 22), catt.Throttle(variant="staged"), 0),
+    (P_(catt.K_SYRK, n=16384, k=2048), catt.Throttle(variant="staged"), 0),                 # tiled: 128+ regs
+    (P_(catt.K_SYR2K, n=16384, k=2048), catt.Throttle(variant="staged"), 0),
+    (P_(catt.K_GEMM, m=16384, n=16384, k=512), catt.Throttle(variant="staged"), 0),
+    (P_(catt.K_KMEANS, m=494020 * 8, n=34, k=5, ld=494020 * 8), catt.Throttle(variant="staged"), 0),   # ~106 KB ring
+    (P_(catt.K_KMEANS, m=494020 * 8, n=34, k=5, ld=494020 * 8), catt.Throttle(), 0),
+    (P_(catt.K_KMEANS_T, m=494020 * 8, n=34, ld=494020 * 8), catt.Throttle(variant="coop"), 0),
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(), 100 * 1024),                     # Fig 5 pads: 2, 3, 5 CTAs
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(), 70 * 1024),
+    (P_(catt.K_ATAX_1, m=1 << 22, n=256), catt.Throttle(), 40 * 1024),
+]
+
+
+@pytest.mark.parametrize("prob,launch,pad", OCC_CASES, ids=[f"{c[0].loop}-{c[1]!r}-{c[2]}" for c in OCC_CASES])
+def test_occupancy_model_matches_cuda_occupancy_api(prob, launch, pad):
+    """a1 pin (Eq 1-3, the B200 arm of reading R9): the analyser's
+    #TB_SM from the kernel's real registers and shared memory equals what the
+    CUDA runtime computes for the same kernel, CTA size and dynamic shared
+    memory at the largest carveout (Eq 1 divides the maximum shared memory);
+    the grids are large enough that ceil(grid / #SM) does not bind."""
     hw = catt.hw_query()
     assert hw.num_sms == 148
-    for prob, launch in [(catt.problem(catt.K_ATAX_1, m=1 << 20, n=256), catt.Throttle()),
-                         (catt.problem(catt.K_KMEANS, m=494020, n=34, k=5, ld=494020), catt.Throttle()),
-                         (catt.problem(catt.K_SYRK, n=2048, k=2048), catt.Throttle())]:
-        d, keep = catt.kernel_desc(prob, launch)
-        regs, smem = catt.kernel_attrs(prob, launch)
-        assert d.regs_per_thread == regs and regs <= 32      # full TLP is not register-limited
-        t, r = catt.plan(prob, launch, hw)
-        assert r["base_ctas"] == 8
+    api, dyn = catt.kernel_occupancy(prob, launch, pad)
+    d, keep = catt.kernel_desc(prob, launch)
+    regs, ssm = catt.kernel_attrs(prob, launch)
+    assert d.regs_per_thread == regs
+    assert d.smem_per_cta + pad == ssm + dyn
+    d.smem_per_cta += pad
+    r = catt.footprint(d, hw)
+    grid = d.grid[0] * d.grid[1] * d.grid[2]
+    # persistent kernels size their grid to the occupancy: there the grid bound
+    # (R8) equals it; everywhere else the grid is large enough not to bind
+    want = min(api, -(-grid // 148))
+    assert r["base_ctas"] == want, dict(api=api, regs=regs, smem=ssm, dyn=dyn, threads=d.block[0] * d.block[1],
+                                        grid=grid, model=r["base_ctas"])
 
 
 # ------------------------------------------------------------------ FUSED (both loops in one pass)

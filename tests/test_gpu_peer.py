@@ -247,3 +247,67 @@ def test_bicg_mvt_peer_processes_share_one_gpu(tmp_path, world, m, n):
             assert _relerr(q_, q64[g * rows:(g + 1) * rows]) <= TOL
         for x1_ in np.load(tmp_path / f"x1{g}.npy"):
             assert _relerr(x1_, x164[g * rows:(g + 1) * rows]) <= TOL
+
+
+# ------------------------------------------------------------------ unequal shards
+def _uneven_rank_main(rank, world, port, rows, n, out_dir):
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+    m = sum(rows)
+    A, x = _problem(m, n, si.MODE_UNIFORM)
+    lo = sum(rows[:rank])
+    Ag = torch.from_numpy(np.ascontiguousarray(A[lo:lo + rows[rank]])).cuda()
+    peer = cdist.peer_setup(n)
+    tmp, y = cdist.atax_rowshard_peer(Ag, torch.from_numpy(x).cuda(), peer)
+    torch.cuda.synchronize()
+    np.save(os.path.join(out_dir, f"y{rank}.npy"), y.cpu().numpy())
+    np.save(os.path.join(out_dir, f"err{rank}.npy"), np.array([peer.error()]))
+    dist.barrier()
+    peer.close()
+    dist.destroy_process_group()
+
+
+def _run_uneven(tmp_path, rows, n):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    port = _free_port()
+    procs = [ctx.Process(target=_uneven_rank_main, args=(r, len(rows), port, rows, n, str(tmp_path)))
+             for r in range(len(rows))]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=240)
+    alive = [p for p in procs if p.is_alive()]
+    for p in alive:
+        p.kill()
+    assert not alive, "a rank hung"
+    assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
+    return [int(np.load(tmp_path / f"err{r}.npy")[0]) for r in range(len(rows))]
+
+
+@pytest.mark.gpu
+def test_atax_peer_unequal_shards_equal_grids(tmp_path):
+    """Shards of 1025 and 1024 rows launch the same grid (one CTA per SM):
+    the exchange is valid and y is the oracle's on both ranks."""
+    import oracle
+    rows, n = [1025, 1024], 1028
+    errs = _run_uneven(tmp_path, rows, n)
+    assert errs == [0, 0]
+    A, x = _problem(sum(rows), n, si.MODE_UNIFORM)
+    _, y64 = oracle.atax(A, x, mode=oracle.SEQ_F64)
+    y0, y1 = np.load(tmp_path / "y0.npy"), np.load(tmp_path / "y1.npy")
+    assert np.array_equal(y0, y1) and _relerr(y0, y64) <= TOL
+
+
+@pytest.mark.gpu
+def test_atax_peer_grid_mismatch_is_reported_not_hung(tmp_path):
+    """shards of 100 and 101 rows launch grids of 100 and 101 CTAs,
+    whose chunk -> CTA maps differ. Both ranks must report the mismatch
+    (catt_peer_check = 2, or 1 where a CTA had no partner) within the test's
+    time limit instead of summing stale slots."""
+    errs = _run_uneven(tmp_path, [100, 101], 1028)
+    assert all(e in (1, 2) for e in errs) and 2 in errs, errs

@@ -1,0 +1,60 @@
+#!/bin/bash
+# One parameterised runner for gpurun calls (replaces round 1's r1*.sh):
+#   /usr/local/graft/bin/gpurun --timeout S -- 'bash tools/gpu_jobs.sh <job> [<job> ...]'
+# Every job writes under gpurun_out/$TAG/ (TAG defaults to the job list).
+# Jobs:
+#   smoke     __graft_entry__.smoke()
+#   tests     pytest -m gpu (all)
+#   occ       the occupancy-API and residency-probe tests only
+#   sanitize  compute-sanitizer memcheck / racecheck / synccheck on tools/sanitize_cases.py
+#   bench     default bench line (+ the reference arm)
+#   benchall  every workload's bench line
+#   launches  ncu launch list of the default bench (gpu__time_duration)
+#   ncu       ncu --set full of the default bench's dominant kernel
+#   sass      per-kernel SASS opcode summary of libcatt.so
+export PYTHONPATH=.
+TAG=${TAG:-$(echo "$@" | tr ' ' '_')}
+O=gpurun_out/$TAG
+mkdir -p $O
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw,temperature.gpu --format=csv > $O/nvsmi.txt 2>&1
+CS="compute-sanitizer --kernel-name kns=catt --print-limit 50 --error-exitcode 9"
+for job in "$@"; do
+  case $job in
+    smoke)
+      timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1; echo "rc=$?" >> $O/smoke.txt ;;
+    tests)
+      timeout 2400 python -m pytest tests -m gpu -q -x > $O/pytest_gpu.txt 2>&1; echo "rc=$?" >> $O/pytest_gpu.txt ;;
+    occ)
+      timeout 600 python -m pytest tests/test_gpu.py -m gpu -q -k "occupancy or residency" > $O/pytest_occ.txt 2>&1; echo "rc=$?" >> $O/pytest_occ.txt ;;
+    sanitize)
+      S=$O/sanitizer; mkdir -p $S
+      timeout 1500 $CS --tool memcheck python tools/sanitize_cases.py > $S/memcheck_all.txt 2>&1; echo "rc=$?" >> $S/memcheck_all.txt
+      timeout 1200 $CS --tool synccheck python tools/sanitize_cases.py > $S/synccheck_all.txt 2>&1; echo "rc=$?" >> $S/synccheck_all.txt
+      for c in gate_sem gate_barrier cta_counter smem_pad staged coop fused fused_graph onekernel kmeans km_iter tiles; do
+        timeout 900 $CS --tool racecheck --racecheck-report analysis python tools/sanitize_cases.py $c > $S/racecheck_$c.txt 2>&1; echo "rc=$?" >> $S/racecheck_$c.txt
+      done
+      timeout 900 python -m torch.distributed.run --nnodes 1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 \
+        --no-python $CS --tool memcheck python tools/sanitize_cases.py peer > $S/memcheck_peer.txt 2>&1; echo "rc=$?" >> $S/memcheck_peer.txt
+      timeout 900 python -m torch.distributed.run --nnodes 1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29534 \
+        --no-python $CS --tool racecheck python tools/sanitize_cases.py peer > $S/racecheck_peer.txt 2>&1; echo "rc=$?" >> $S/racecheck_peer.txt
+      ;;
+    bench)
+      timeout 1200 python bench.py > $O/bench.json 2> $O/bench.err; echo "rc=$?" >> $O/bench.err
+      timeout 900 python bench.py --impl reference --steps 3 --warmup 3 > $O/bench_reference.json 2> $O/bench_reference.err ;;
+    benchall)
+      for w in atax bicg_mvt kmeans kmeans_iter gesummv syrk syr2k corr gemm atax256; do
+        timeout 1500 python bench.py --workload $w > $O/bench_$w.json 2> $O/bench_$w.err
+      done ;;
+    launches)
+      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv \
+        python bench.py --steps 2 --warmup 3 --no-study --no-e2e --cpu-seconds 0 > $O/launches.log 2>&1 ;;
+    ncu)
+      timeout 900 ncu --set full --clock-control none --import-source on -k regex:${NCU_KERNEL:-fused} -s 3 -c 1 -o $O/ncu_default -f \
+        python bench.py --steps 1 --warmup 3 --no-study --no-e2e --cpu-seconds 0 > $O/ncu_default.log 2>&1 ;;
+    sass)
+      python tools/sass_summary.py paper_conf_icpp_kimhlsh19_b200/libcatt.so > $O/sass_summary.txt 2>&1 ;;
+    *)
+      echo "unknown job $job" >> $O/errors.txt ;;
+  esac
+done
+ls -la $O > $O/ls.txt
