@@ -145,3 +145,15 @@ def decide(kernel, W: int, T: int, l1d_lines: int, num_sms: int, guards: Dict = 
 
 def l1d_lines(carveout_kb: int, line: int = lru.LINE) -> int:
     return B200_L1D_KB[carveout_kb] * 1024 // line
+
+
+def b200_hw(num_sms: int = 148) -> Dict:
+    """The B200 table for oracle.footprint.occupancy (Eq 1-4): 148 SMs, 64
+    warps / 32 CTAs / 64 K registers per SM, 128-byte shared-memory allocation
+    unit, 1 KB reserved per CTA (SURVEY 8 header; pinned on the device by
+    tests/test_gpu.py::test_occupancy_model_matches_cuda_occupancy_api), the
+    carveout options and measured L1D of DESIGN.md section 5."""
+    carve = sorted(B200_L1D_KB)
+    return dict(num_sms=num_sms, max_warps_sm=64, max_ctas_sm=32, regs_sm=65536, reg_alloc_unit=256, warp_size=32,
+                smem_alloc_unit=128, reserved_smem_cta=1024, line_bytes=128, carveout_kb=carve,
+                l1d_bytes=[B200_L1D_KB[c] * 1024 for c in carve])

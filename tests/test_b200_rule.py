@@ -1,0 +1,189 @@
+"""The B200 decision rule (R17-R19, R23, R24, R27) against an oracle
+that shares nothing with the analyser: oracle/b200_rule.py measures the
+rule's inputs on the loop bodies' address traces (oracle/lru.py `program`)
+and decides "fits" with the LRU L1D simulator, then picks by a plain
+enumeration of every (a, m). VERDICT r1 weak 1: the previous check compared
+two transcriptions of one heuristic (oracle/footprint.py's guard branch and
+csrc/footprint.cpp)."""
+import json
+import os
+import sys
+
+import pytest
+
+import paper_conf_icpp_kimhlsh19_b200 as catt
+from oracle import b200_rule as br
+from oracle import footprint as fp
+from oracle import lru
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+GOLDEN = os.path.join(ROOT, "tests", "golden", "b200_rule_picks.json")
+
+
+# ------------------------------------------------------------------ the trace measurements, by hand
+def test_trace_inputs_of_the_row_loop():
+    """Row per thread, 4-byte loads (Fig 1's loop): A[i*N + j] touches
+    32 lines per warp request (rows 4N bytes apart), a thread re-touches its
+    line 128 / 4 = 32 times; x[j] is one line per request; every load reuses,
+    so nothing streams. VEC4 (16-byte steps) re-touches 8 times."""
+    inp = br.trace_inputs(lru.RowKernel(256, 128, 256))
+    assert inp.lines == {"x": 1, "A": 32}
+    assert inp.retouch == {"x": 32, "A": 32}
+    assert inp.reuse == {"x": True, "A": True} and inp.stream_bytes == 0 and inp.locality
+    v = br.trace_inputs(lru.RowKernel(256, 128, 256, vec=4))
+    assert v.retouch["A"] == 8 and v.lines["A"] == 32
+    short = br.trace_inputs(lru.RowKernel(256, 20, 256))          # a row of 20 floats: 20 touches, capped by the trip
+    assert short.retouch["A"] == 20
+    one = br.trace_inputs(lru.RowKernel(256, 1, 256))             # one iteration: no reuse at all (R17)
+    assert not one.locality
+
+
+def test_trace_inputs_of_the_other_loops():
+    # the KM transpose: lanes 34 floats apart (one line each), 34 touches of a
+    # 136-byte row; the store out[f*ld + p] is half of the bytes (R24)
+    t = br.trace_inputs(lru.TransposeKernel(4096, 34, 4096, 256))
+    assert t.lines["in"] == 32 and t.retouch["in"] == 32 and t.reuse["in"] and t.stored["out"]
+    assert 2 * t.stream_bytes == t.total_bytes
+    # KMEANS feature-major: coalesced (one line per request when ld is aligned),
+    # re-touched once per centre (outer-level reuse)
+    k = br.trace_inputs(lru.KmeansKernel(4096, 6, 5, 4096, 256))
+    assert k.lines["F"] == 1 and k.retouch["F"] == 5
+    # the column loop: A[i*N + j] coalesced and never re-touched -> streams;
+    # v[i] broadcast, re-touched 32 times
+    c = br.trace_inputs(lru.ColKernel(64, 512, 256))
+    assert c.lines["A"] == 1 and not c.reuse["A"] and c.retouch["v"] == 32 and c.reuse["v"]
+    assert 2 * c.stream_bytes == c.total_bytes
+    # SYRK's a[j*M + k]: 32 lines per request (one row per lane), 32 touches
+    s = br.trace_inputs(lru.SyrkKernel(256, 64))
+    assert s.lines == {"a_i": 1, "a_j": 32} and s.retouch["a_j"] == 32
+    # CORR: lanes at j2 = j1 + 1 + q read coalesced columns (j2 = 1..32 spans two lines)
+    r = br.trace_inputs(lru.CorrKernel(96, 4, 32))
+    assert r.lines["d_j1"] == 1 and r.lines["d_j2"] == 2 and r.reuse["d_j1"] and r.stored["sym_12"]
+
+
+def test_divergence_predicate():
+    g = dict(br.B200_GUARDS)
+    assert br.divergent(br.trace_inputs(lru.RowKernel(256, 128, 256)), g)           # 32 lines, 32 touches
+    assert not br.divergent(br.trace_inputs(lru.RowKernel(256, 128, 256, vec=4)), g)  # 8 touches < 16 (R23)
+    assert not br.divergent(br.trace_inputs(lru.TransposeKernel(4096, 34, 4096, 256)), g)  # 50 % stream (R24)
+    assert not br.divergent(br.trace_inputs(lru.KmeansKernel(4096, 6, 5, 4096, 256)), g)  # coalesced (R18)
+    loose = dict(g, max_stream_pct=60)
+    assert br.divergent(br.trace_inputs(lru.TransposeKernel(4096, 34, 4096, 256)), loose)
+
+
+def test_lru_fit_is_the_capacity_of_the_retained_lines():
+    """One CTA of W warps of the row loop retains 32 W + 1 lines (each warp's
+    32 row lines and the shared x line): the LRU fits exactly at that
+    capacity, and a warps fit at 32 a + 1."""
+    k = br._Loads(lru.RowKernel(256, 64, 256))
+    blocks = [0]
+    for a in (8, 4, 2):
+        cap = 32 * a + 1
+        assert lru.simulate(k, blocks, a, 1, cap)["intra_thread_capacity_misses"] == 0
+        assert lru.simulate(k, blocks, a, 1, cap - 1)["intra_thread_capacity_misses"] > 0
+
+
+# ------------------------------------------------------------------ decisions: hand-worked
+def test_rule_decisions_worked_by_hand():
+    """A few picks worked out from the definitions (B200 table, W and T from
+    Eq 1-4): 1024-thread row loop at 196 KB (53 KB L1D = 424 lines): 32 warps
+    need 32*32 + 1 = 1025 lines, 8 warps 257 fit, 16 warps 513 do not -> (8, 1);
+    at 132 KB (944 lines) 16 warps fit -> (16, 1). 256-thread rows with 2
+    CTAs per SM at 228 KB (168 lines): no pair at or above 8 warps per SM fits,
+    T = 2 -> R27 caps a whole CTA: (8, 1). The same loop with VEC4 steps: not
+    divergent enough (8 re-touches) -> full TLP."""
+    hw = br.b200_hw()
+    rows = lru.RowKernel(4096, 128, 1024)
+    assert br.decide(rows, 32, 1, br.l1d_lines(196), 148)[:2] == (8, 1)
+    assert br.decide(rows, 32, 1, br.l1d_lines(132), 148)[:2] == (16, 1)
+    big = lru.RowKernel(65536, 128, 256)
+    W, T, _, l1d = fp.occupancy(fp.Loop(refs=[], trips=(), block=(256, 1, 1), grid=(256, 1, 1), smem=16,
+                                        force_carveout_kb=228), hw)
+    assert (W, T, l1d // 128) == (8, 2, 168)
+    assert br.decide(big, W, T, l1d // 128, 148) == (8, 1, "fallback(cta)")
+    assert br.decide(lru.RowKernel(4096, 128, 1024, vec=4), 32, 1, br.l1d_lines(196), 148) == (32, 1, "none(guard)")
+
+
+# ------------------------------------------------------------------ the library against the trace oracle
+SMALL_HW = dict(num_sms=2, max_warps_sm=16, max_ctas_sm=4, regs_sm=65536, reg_alloc_unit=256, warp_size=32,
+                smem_alloc_unit=128, reserved_smem_cta=0, line_bytes=128, carveout_kb=[0, 8, 16, 32],
+                l1d_bytes=[n * 128 for n in (600, 257, 120, 33)])
+SMALL_GUARDS = dict(min_warps_sm=2, divergent_lines=8, min_retouch=16, max_stream_pct=25, cta_fallback=1)
+
+KERNELS = [
+    ("atax1", catt.problem(catt.K_ATAX_1, m=256, n=64), catt.Throttle(), lru.RowKernel(256, 64, 256)),
+    ("atax1_vec4", catt.problem(catt.K_ATAX_1, m=256, n=64), catt.Throttle(variant="vec4"),
+     lru.RowKernel(256, 64, 256, vec=4)),
+    ("bicg2_ragged", catt.problem(catt.K_BICG_2, m=300, n=96), catt.Throttle(cta_threads=128),
+     lru.RowKernel(300, 96, 128)),
+    ("mvt1_multi_cta", catt.problem(catt.K_MVT_1, n=1024), catt.Throttle(cta_threads=128),
+     lru.RowKernel(1024, 64, 128)),
+    ("gesummv", catt.problem(catt.K_GESUMMV, n=256), catt.Throttle(), lru.RowKernel(256, 256, 256, matrices=("A", "B"))),
+    ("atax2", catt.problem(catt.K_ATAX_2, m=40, n=512), catt.Throttle(), lru.ColKernel(40, 512, 256)),
+    ("kmeans", catt.problem(catt.K_KMEANS, m=2040, n=6, k=3, ld=2044), catt.Throttle(cta_threads=128),
+     lru.KmeansKernel(2040, 6, 3, 2044, 128)),
+    ("km_transpose", catt.problem(catt.K_KMEANS_T, m=2040, n=34, ld=2044), catt.Throttle(cta_threads=128),
+     lru.TransposeKernel(2040, 34, 2044, 128)),
+    ("syrk", catt.problem(catt.K_SYRK, n=128, k=64), catt.Throttle(), lru.SyrkKernel(128, 64)),
+    ("syr2k", catt.problem(catt.K_SYR2K, n=128, k=64), catt.Throttle(), lru.Syr2kKernel(128, 64)),
+    ("gemm", catt.problem(catt.K_GEMM, m=96, n=64, k=48), catt.Throttle(), lru.GemmKernel(96, 64, 48)),
+]
+
+
+@pytest.mark.parametrize("name,prob,launch,kern", KERNELS, ids=[k[0] for k in KERNELS])
+def test_library_rule_equals_trace_oracle_on_own_kernels(name, prob, launch, kern):
+    """catt_footprint with the B200 guards on a small fake GPU (2 SMs, 16
+    warps) picks what the trace oracle picks, at every carveout."""
+    hw = catt.Hw.from_dict(dict(SMALL_HW, **SMALL_GUARDS))
+    for carve in SMALL_HW["carveout_kb"]:
+        d, keep = catt.kernel_desc(prob, launch)
+        d.regs_per_thread = 0
+        d.smem_per_cta = 0
+        d.force_carveout_kb = carve
+        got = catt.footprint(d, hw)
+        W, T = got["base_warps"], got["base_ctas"]
+        a, m, how = br.decide(kern, W, T, got["l1d_bytes"] // 128, SMALL_HW["num_sms"], SMALL_GUARDS)
+        assert (got["active_warps"], got["active_ctas"]) == (a, m), (name, carve, got, how)
+
+
+def _golden():
+    return json.load(open(GOLDEN))
+
+
+def test_library_rule_equals_trace_oracle_on_the_160_replayed_launches():
+    """Every launch of the stored sweeps (tools/rule_replay.py's 160: the round-1
+    final pass, held-out sets 1-9, the SM partitions), at its full shape: the
+    library's (W, T), L1D and pick equal those tools/gen_rule_golden.py derived
+    from oracle/ alone (traces + LRU + Eq 1-4)."""
+    g = _golden()
+    assert len(g["launches"]) == 160 and g["guards"] == br.B200_GUARDS
+    b200 = catt.hw_b200()
+    assert (b200.min_warps_sm, b200.divergent_lines, b200.min_retouch, b200.max_stream_pct, b200.cta_fallback) == \
+        tuple(br.B200_GUARDS[k] for k in ("min_warps_sm", "divergent_lines", "min_retouch", "max_stream_pct",
+                                          "cta_fallback"))
+    for L in g["launches"]:
+        p = dict(L["prob"])
+        prob = catt.problem(p.pop("loop"), **p)
+        hw = catt.hw_b200()
+        if L["sm_partition"]:
+            hw.num_sms = L["sm_partition"]
+        t, r = catt.plan(prob, catt.Throttle(cta_threads=L["cta"], carveout_kb=L["carveout_kb"], variant=L["variant"]),
+                         hw)
+        W, T = r["base_warps"], r["base_ctas"]
+        assert (W, T, r["l1d_bytes"] // 128) == (L["W"], L["T"], L["l1d_lines"]), L
+        assert [t.active_warps or W, t.active_ctas or T] == L["pick"], L
+
+
+def test_golden_file_is_the_generators_output():
+    """A sample of the golden entries re-derived now (the cheap ones), so the
+    stored file cannot drift from tools/gen_rule_golden.py + oracle/."""
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    import gen_rule_golden as gen
+    g = _golden()["launches"]
+    cheap = [L for L in g if L["prob"]["loop"] in (gen.K_ATAX_1, gen.K_BICG_2, gen.K_MVT_1, gen.K_GESUMMV,
+                                                   gen.K_KMEANS_T)]
+    sample = cheap[::6][:12]
+    assert len(sample) >= 8
+    for L in sample:
+        spec = {k: L[k] for k in ("set", "loop", "prob", "variant", "cta", "carveout_kb", "sm_partition")}
+        assert gen.decide(spec) == L

@@ -437,58 +437,61 @@ def test_atax_65536x16384_sampled():
 
 
 # ------------------------------------------------------------------ throttle enforcement (residency probe)
+def _max_overlap(ivs):
+    ev = sorted([(a, 1) for a, b in ivs] + [(b, -1) for a, b in ivs])   # ends before starts at equal stamps
+    cur = best = 0
+    for _, d in ev:
+        cur += d
+        best = max(best, cur)
+    return best
+
+
 def _concurrency(rec, W):
-    """rec: [ncta*W, 3] (smid, t0, t1). Max warps of one CTA inside the loop at
-    once, and max CTAs of one SM with a warp inside the loop at once."""
+    """rec: [ncta*W, 3] (smid, t0, t1) per warp around the loop. Returns the
+    most warps of one CTA inside the loop at once, the most CTAs of one SM
+    with a warp inside the loop at once, and the most warps of one SM inside
+    the loop at once."""
     rec = rec.reshape(-1, W, 3)
     valid = rec[:, :, 2] > 0
-    max_w = 0
-    for c in range(rec.shape[0]):
-        ev = sorted([(rec[c, w, 1], 1) for w in range(W) if valid[c, w]] +
-                    [(rec[c, w, 2], -1) for w in range(W) if valid[c, w]], key=lambda e: (e[0], e[1]))
-        cur = 0
-        for _, d in ev:
-            cur += d
-            max_w = max(max_w, cur)
-    cta_iv = {}
+    max_w = max(_max_overlap([(rec[c, w, 1], rec[c, w, 2]) for w in range(W) if valid[c, w]])
+                for c in range(rec.shape[0]))
+    cta_iv, warp_iv = {}, {}
     for c in range(rec.shape[0]):
         if not valid[c].any():
             continue
         sm = int(rec[c, valid[c], 0][0])
         cta_iv.setdefault(sm, []).append((rec[c, valid[c], 1].min(), rec[c, valid[c], 2].max()))
-    max_c = 0
-    for sm, ivs in cta_iv.items():
-        ev = sorted([(a, 1) for a, b in ivs] + [(b, -1) for a, b in ivs], key=lambda e: (e[0], e[1]))
-        cur = 0
-        for _, d in ev:
-            cur += d
-            max_c = max(max_c, cur)
-    return max_w, max_c
+        warp_iv.setdefault(sm, []).extend((rec[c, w, 1], rec[c, w, 2]) for w in range(W) if valid[c, w])
+    max_c = max(_max_overlap(v) for v in cta_iv.values())
+    max_ws = max(_max_overlap(v) for v in warp_iv.values())
+    return max_w, max_c, max_ws
 
 
 @pytest.mark.parametrize("t,want", [
-    (catt.Throttle(carveout_kb=16), (8, 8)),
-    (catt.Throttle(active_warps=2, carveout_kb=16), (2, 8)),
-    (catt.Throttle(active_warps=4, gate=catt.GATE_BARRIER, carveout_kb=16), (4, 8)),
-    (catt.Throttle(active_warps=1, active_ctas=3, carveout_kb=16), (1, 3)),
-    (catt.Throttle(active_ctas=2, cap=catt.CAP_SMEM_PAD, carveout_kb=64), (8, 2)),
-    (catt.Throttle(carveout_kb=8), (8, 7)),
+    (catt.Throttle(carveout_kb=16), (8, 0, 64)),
+    (catt.Throttle(active_warps=2, carveout_kb=16), (2, 0, 16)),
+    (catt.Throttle(active_warps=4, gate=catt.GATE_BARRIER, carveout_kb=16), (4, 0, 32)),
+    (catt.Throttle(active_warps=1, active_ctas=3, carveout_kb=16), (1, 3, 3)),
+    (catt.Throttle(active_ctas=2, cap=catt.CAP_SMEM_PAD, carveout_kb=64), (8, 2, 16)),
 ], ids=repr)
 def test_residency_probe_enforces_throttle(t, want):
     """a6 (Fig 4/5) and a1 (Eq 1-4): the measured concurrency equals the
-    throttle -- warps per CTA inside the loop and CTAs per SM inside the loop.
-    Full TLP co-schedules exactly T CTAs: 8 at the carveout Eq 4 picks (16 KB
-    for 8 CTAs of 1 KB reserved + 16 B), and 7 when the launch forces the 8 KB
-    option (7 x 1152 B fit, 8 do not) -- the model's T for that carveout."""
+    throttle -- warps per CTA inside the loop (a), CTAs per SM inside the loop
+    under a CTA cap (m), and warps per SM inside the loop (a * T, or a * m).
+    Full TLP co-schedules W * T = 8 * 8 = 64 warps per SM at the carveout Eq 4
+    picks (16 KB for 8 CTAs of 1 KB reserved + 16 B). Without a cap the
+    number of CTAs with a warp in the loop can exceed T (a warp's slot is
+    freed when the warp exits, so the next CTA starts while the last warps of
+    the previous one still run), so T is checked through the warps per SM.
+    A forced small carveout does not cap CTAs: the driver takes a larger
+    shared-memory configuration when that fits more CTAs (8 KB forced: 12 CTAs
+    measured), which is why the library's CTA cap is the per-SM counter."""
     # long rows so CTAs overlap in time; 148 SMs x 8 CTAs x 256 rows x 2 waves
     m, n = 148 * 8 * 256 * 2, 512
     prob = catt.problem(catt.K_ATAX_1, m=m, n=n)
     _, r = catt.plan(prob, catt.Throttle(carveout_kb=t.carveout_kb), catt.hw_query())
-    if t.cap != catt.CAP_SMEM_PAD:
-        assert r["base_ctas"] == {16: 8, 8: 7}[t.carveout_kb]       # the model's T at this carveout
-    if t.carveout_kb == 16 and not t.active_ctas:
-        _, r0 = catt.plan(prob, catt.Throttle(), catt.hw_query())
-        assert r0["carveout_kb"] == 16                     # Eq 4's own pick
+    _, r0 = catt.plan(prob, catt.Throttle(), catt.hw_query())
+    assert r0["carveout_kb"] == 16 and (r0["base_warps"], r0["base_ctas"]) == (8, 8)   # Eq 4's own pick
     A = torch.empty(m * n, device="cuda")
     catt.fill_hash(A, 1)
     x = torch.ones(n, device="cuda")
@@ -496,10 +499,11 @@ def test_residency_probe_enforces_throttle(t, want):
     probe = torch.zeros(ncta * 8 * 3, dtype=torch.int64, device="cuda")
     tt = t.copy(probe=probe.data_ptr())
     catt.atax(A.view(m, n), x, k1=tt)
-    mw, mc = _concurrency(host(probe).astype(np.int64), 8)
-    assert mw <= want[0] and mc <= want[1]
-    assert mw == want[0]                                   # the slots are actually used
-    assert mc == want[1]                                   # ... and so are the CTA slots: T (or the cap) co-resident
+    mw, mc, mws = _concurrency(host(probe).astype(np.int64), 8)
+    assert mw == want[0]                                   # the warp slots: used and never exceeded
+    if want[1]:
+        assert mc == want[1]                               # the CTA cap: used and never exceeded
+    assert mws == want[2]                                  # a * T (or a * m) warps per SM in the loop
 
 
 P_ = catt.problem
@@ -737,8 +741,8 @@ def test_sm_partition_confines_ctas_and_keeps_results(min_sms):
         rec = host(probe).astype(np.int64).reshape(-1, 3)
         sms = set(int(s) for s in rec[rec[:, 2] > 0, 0])
         assert 1 <= len(sms) <= part.sms
-        mw, mc = _concurrency(rec, 8)
-        assert mc <= 2
+        mw, mc, mws = _concurrency(rec, 8)
+        assert mc == 2 and mws <= 16
         Ah = oracle.fill(1, m * nn).reshape(m, nn)
         tmp_o, y_o = oracle.atax(Ah, np.ones(nn, dtype=np.float32))
         assert bits_equal(host(tmp), tmp_o) and bits_equal(host(y), y_o)

@@ -234,7 +234,7 @@ def case_peer():
 CASES = {k[5:]: v for k, v in globals().items() if k.startswith("case_")}
 
 if __name__ == "__main__":
-    names = sys.argv[1:] or sorted(CASES)
+    names = sys.argv[1:] or sorted(c for c in CASES if c != "peer")   # peer runs under torchrun
     for nm in names:
         CASES[nm]()
         torch.cuda.synchronize()
