@@ -1,17 +1,24 @@
 #!/usr/bin/env python3
 """bench.py — the CATT hot path on B200, one JSON line.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload bicg_mvt|kmeans|gesummv|syrk|atax256|atax]
-                    [--variant coop|staged|vec4|literal] [--impl reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload atax|bicg_mvt|kmeans|gesummv|syrk|atax256|...]
+                    [--variant fused|fused_peer|coop|staged|vec4|literal] [--impl reference] [--no-l1]
 
 A step is one pass of the whole hot path over one batch: the CATT analysis of
 every loop (host, microseconds), then every loop of the workload launched with
 its CATT throttle through the C ABI (catt_rows / catt_cols / catt_kmeans_assign
 / catt_syrk), plus the NCCL all-reduce of the A^T partials when N > 1.
-Default workload = BASELINE.json configs[1]: BICG and MVT 4096 x 4096 fp32
-(four loops: s = A^T r, q = A p, x1 += A y1, x2 += A^T y2). Multi-GPU is weak
-scaling: every rank owns 4096 more rows of a (4096 N) x 4096 matrix; the two
-A^T partials are all-reduced (the only exchange the path has).
+Default workload = BASELINE.json configs[4], the largest configuration and the
+scaling one: ATAX 65536 x 16384 fp32 (tmp = A x, y = A^T tmp), rows sharded
+over the N ranks (16384 x 65536 / N rows each at N > 1), the A^T partials
+all-reduced by NCCL (the only exchange the path has). At N = 1 it is the whole
+4 GiB matrix on one B200. `--workload bicg_mvt` is configs[1] (BICG and MVT
+4096 x 4096, weak-scaled over ranks).
+
+After the timed region (N = 1): the throttle study of the workload's literal
+loop (CATT pick, paper rule, full TLP, every swept (a, m)), and the L1 hit
+rate and DRAM bytes of each pick from an ncu subprocess (the metric's other
+half).
 
 `value` = algorithmic bytes of the step (all ranks) / device time (max over
 ranks), GB/s. L2 is flushed (256 MiB write) before every timed step.
@@ -43,7 +50,7 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
-    p.add_argument("--workload", default="bicg_mvt",
+    p.add_argument("--workload", default="atax",
                    choices=["bicg_mvt", "kmeans", "kmeans_iter", "gesummv", "syrk", "syr2k", "corr", "gemm", "atax256", "atax"])
     p.add_argument("--variant", default=None,
                    help="fused (default for bicg_mvt/atax), fused1, coop, staged, vec4, literal, regs (kmeans)")
@@ -53,6 +60,8 @@ def parse():
     p.add_argument("--flush-order", default="flush_sleep", choices=["flush_sleep", "sleep_flush"],
                    help="order of the L2 flush and the enqueue-cover GPU sleep before each timed step")
     p.add_argument("--cpu-seconds", type=float, default=8.0, help="CPU-oracle sample budget")
+    p.add_argument("--no-l1", action="store_true", help="skip the ncu L1-hit-rate pass over the study picks")
+    p.add_argument("--l1-child", default=None, help=argparse.SUPPRESS)   # internal: the ncu-profiled launches
     return p.parse_args()
 
 
@@ -125,9 +134,10 @@ class ClockSampler:
 
 # ------------------------------------------------------------------ workloads
 class Loop:
-    def __init__(self, name, fn, nbytes, kind, prob=None, launch=None):
+    def __init__(self, name, fn, nbytes, kind, prob=None, launch=None, plans=None):
         self.name, self.fn, self.nbytes, self.kind = name, fn, nbytes, kind
         self.prob, self.launch = prob, launch
+        self.plans = plans or [name]          # keys of Workload.plans behind this launch
 
 
 class Workload:
@@ -143,13 +153,20 @@ class Workload:
         self.plans = {}
 
     def plan(self, key, prob, launch):
-        """The CATT analysis (a1-a5) for one loop; returns the throttle to launch with."""
-        t0 = time.perf_counter()
-        t, r = self.catt.plan(prob, launch, self.hw)
+        """The CATT analysis (a1-a5) for one loop; returns the throttle to
+        launch with. analysis_us = the median of 21 analyses (catt_plan: the
+        kernel's attributes, the descriptor, Eq 1-9), first_us = the first
+        (it also queries the device); the paper reports 1-2 s."""
+        ts = []
+        for _ in range(21):
+            t0 = time.perf_counter()
+            t, r = self.catt.plan(prob, launch, self.hw)
+            ts.append(1e6 * (time.perf_counter() - t0))
         self.plans[key] = dict(throttle=[t.active_warps or r["base_warps"], t.active_ctas or r["base_ctas"]],
                                base=[r["base_warps"], r["base_ctas"]], flags=self.catt.FLAG_NAMES[r["flags"]],
                                footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
-                               carveout_kb=r["carveout_kb"], analysis_us=round(1e6 * (time.perf_counter() - t0), 1))
+                               carveout_kb=r["carveout_kb"], analysis_us=round(statistics.median(ts), 1),
+                               analysis_first_us=round(ts[0], 1))
         return t
 
     def collective(self):
@@ -216,7 +233,7 @@ class BicgMvt(Workload):
                          dict(A=self.Am, xr=self.y1, xc=self.y2, yr=self.x1, yc=self.x2, row_accumulate=True,
                               col_accumulate=acc2)]
                 self.loops = [Loop("bicg+mvt fused (one launch)", lambda: catt.dual_group(group, t=tf),
-                                   bicg_b + mvt_b, "fused")]
+                                   bicg_b + mvt_b, "fused", plans=["bicg fused", "mvt fused"])]
             else:
                 self.loops = [
                     Loop("bicg fused", lambda: catt.dual(self.Ab, self.p, self.q, self.s, xc=self.r, t=tf),
@@ -585,7 +602,7 @@ class Atax(Workload):
         var = self.variant
         mat = rows * n * 4
         self.study = dict(name="atax1 tmp=A x (literal, row per thread)", prob=catt.problem(catt.K_ATAX_1, m=rows, n=n),
-                          A=self.A, x=self.x, y=self.tmp, launches=[(1024, 196), (256, 228)])
+                          A=self.A, x=self.x, y=self.tmp, launches=[(256, 228), (256, 196), (1024, 196)])
         # both loops in one kernel, a throttle per loop
         self.kernel_study = dict(m=4096, n=4096, launches=[(1024, 196), (1024, 228), (512, 196)])
         if var == "fused_peer":
@@ -744,7 +761,11 @@ def throttle_study(catt, torch, w, flush):
 def _study_launch(catt, w, S, cta, carve, hw, med):
     paper_hw = catt.paper_rule(hw)
     launch = catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
-    t, r = catt.plan(S["prob"], launch, hw)               # B200 rule (guards on)
+    ts = []
+    for _ in range(11):                                   # the analysis' latency (1-2 s per application)
+        t0 = time.perf_counter()
+        t, r = catt.plan(S["prob"], launch, hw)           # B200 rule (guards on)
+        ts.append(1e6 * (time.perf_counter() - t0))
     tp, rp = catt.plan(S["prob"], launch, paper_hw)       # the paper's Eq 9 rule
     W, T = r["base_warps"], r["base_ctas"]
     cands = []
@@ -764,6 +785,7 @@ def _study_launch(catt, w, S, cta, carve, hw, med):
     if not S.get("fn") and not S.get("kmeans"):
         byp = med(study_fn(catt, w, launch.copy(variant=catt.VAR_BYPASS)), S.get("reps", 5))
     return dict(loop=S["name"], cta_threads=cta, carveout_kb=r["carveout_kb"], base=[W, T],
+                    analysis_us=round(statistics.median(ts), 1),
                     footprint_lines=r["footprint_lines_full"], l1d_lines=r["l1d_bytes"] // 128,
                     contended=rp["flags"] != catt.FIT_NONE_NEEDED,
                     catt=list(pick), catt_rule=catt.FLAG_NAMES.get(r["flags"], r["flags"]),
@@ -894,6 +916,88 @@ def kernel_study(catt, torch, w, flush):
     return out
 
 
+NCU_L1_METRICS = ("l1tex__t_sector_hit_rate.pct", "dram__bytes_read.sum", "dram__bytes_write.sum",
+                  "gpu__time_duration.sum")
+
+
+def l1_spec(study):
+    """The launches the ncu pass profiles: each study row's CATT pick, paper
+    pick, full TLP and best swept throttle (duplicates once)."""
+    spec = []
+    for i, row in enumerate(study or []):
+        if row.get("sm_partition"):
+            continue                          # ncu cannot profile a green-context launch
+        roles = {}
+        for role, am in (("catt", row["catt"]), ("paper", row["catt_paper"]), ("full", row["base"]),
+                         ("best", row["best"])):
+            roles.setdefault(tuple(am), []).append(role)
+        for (a, m), rl in roles.items():
+            spec.append(dict(row=i, cta=row["cta_threads"], carve=row["carveout_kb"], a=a, m=m, T=row["base"][1],
+                             roles=rl))
+    return spec
+
+
+def l1_child(args, catt, torch, w):
+    """--l1-child: launch the study loop once per spec entry between
+    cudaProfilerStart/Stop (ncu --profile-from-start off sees only these)."""
+    spec = json.loads(args.l1_child)
+    fns = []
+    for e in spec:
+        th = catt.Throttle(cta_threads=e["cta"], carveout_kb=e["carve"], variant="literal", active_warps=e["a"],
+                           active_ctas=e["m"] if e["m"] < e["T"] else 0)
+        fns.append(study_fn(catt, w, th))
+    torch.cuda.synchronize()
+    torch.cuda.profiler.start()
+    for f in fns:
+        f()
+    torch.cuda.synchronize()
+    torch.cuda.profiler.stop()
+    return 0
+
+
+def l1_pass(args, study):
+    """The L1 half of the metric (Fig 6): ncu's L1 sector hit
+    rate, DRAM bytes and duration of the study loop at each pick, one cold
+    launch each (ncu flushes the caches before every profiled kernel), in a
+    subprocess after the timed region. Adds row["l1"][role] to the study rows."""
+    import csv
+    import io
+    import shutil
+    spec = l1_spec(study)
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not spec or not os.path.exists(ncu):
+        return {"status": "skipped", "why": "no study launches" if not spec else "ncu not found"}
+    cmd = [ncu, "--profile-from-start", "off", "--metrics", ",".join(NCU_L1_METRICS), "--csv", "--print-units", "base",
+           sys.executable, os.path.join(ROOT, "bench.py"), "--workload", args.workload, "--l1-child", json.dumps(spec)]
+    if args.variant:
+        cmd += ["--variant", args.variant]
+    t0 = time.perf_counter()
+    try:
+        out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    except Exception as ex:                   # pragma: no cover
+        return {"status": "failed", "why": str(ex)[:200]}
+    rows = [r for r in csv.reader(io.StringIO("\n".join(l for l in out.stdout.splitlines() if l.startswith('"'))))]
+    if not rows:
+        return {"status": "failed", "rc": out.returncode, "why": (out.stderr or out.stdout)[-300:]}
+    head = rows[0]
+    ci = {k: head.index(k) for k in ("ID", "Kernel Name", "Metric Name", "Metric Value")}
+    per = {}
+    for r in rows[1:]:
+        per.setdefault(int(r[ci["ID"]]), {})[r[ci["Metric Name"]]] = float(r[ci["Metric Value"]].replace(",", ""))
+    ids = sorted(per)
+    if len(ids) != len(spec):
+        return {"status": "failed", "why": f"{len(ids)} profiled kernels for {len(spec)} launches"}
+    for e, k in zip(spec, ids):
+        m = per[k]
+        res = {"throttle": [e["a"], e["m"]], "l1_hit_pct": round(m["l1tex__t_sector_hit_rate.pct"], 2),
+               "dram_bytes": int(m["dram__bytes_read.sum"] + m["dram__bytes_write.sum"]),
+               "ncu_us": round(m["gpu__time_duration.sum"] / 1e3, 1)}
+        for role in e["roles"]:
+            study[e["row"]].setdefault("l1", {})[role] = res
+    return {"status": "ok", "launches": len(spec), "seconds": round(time.perf_counter() - t0, 1),
+            "metrics": list(NCU_L1_METRICS), "cache_control": "all (ncu default: caches flushed before each kernel)"}
+
+
 def ncu_traffic(workload):
     """DRAM bytes per launch of the workload's dominant kernel from the committed ncu summary."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -936,8 +1040,19 @@ def run_reference(args):
         nbytes = npts * nf * 4 + npts * 4
         cfg = Kmeans.desc
         sample = "the full assign step per step"
+    elif wl == "atax":
+        # configs[4]: the oracle on a bounded sample of the 65536 x 16384 matrix
+        # (its first 2048 rows, all 16384 columns: 128 MiB, the same generator
+        # and seed as the GPU arm), tmp = A x and y = A^T tmp per step
+        rows, n = 2048, 16384
+        A = oracle.fill(si.SEED_ATAX_SHARDED, rows * n).reshape(rows, n)
+        x = oracle.fill(si.sub_seed(si.SEED_ATAX_SHARDED, 1), n)
+        step = lambda: oracle.atax(A, x)
+        nbytes = rows * n * 4 + 4 * (2 * n + rows)
+        cfg = Atax.desc
+        sample = f"ATAX on the first {rows} of the 65536 rows (x 16384 columns) per step"
     else:
-        print(json.dumps({"impl": "reference", "unavailable": f"reference arm implemented for bicg_mvt and kmeans, not {wl}"}))
+        print(json.dumps({"impl": "reference", "unavailable": f"reference arm implemented for atax, bicg_mvt and kmeans, not {wl}"}))
         return 0
     for _ in range(max(args.warmup, 1)):
         step()
@@ -980,6 +1095,9 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as dist
+        # NCCL's own report of the communicator (ranks, NVLink / NVLS paths)
+        # lands in stderr for the driver's rank check
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
         if share:
             dist.init_process_group("gloo")
         else:
@@ -987,9 +1105,13 @@ def main():
         barrier = lambda: dist.barrier()
     else:
         barrier = lambda: None
+    log(f"bench: rank {rank} of world {world} on cuda:{local} ({torch.cuda.get_device_name(local)}), "
+        f"workload {args.workload}")
     import paper_conf_icpp_kimhlsh19_b200 as catt
 
     w = WORKLOADS[args.workload](catt, torch, rank, world, args.variant)
+    if args.l1_child:
+        return l1_child(args, catt, torch, w)
     # L2 flush between steps: write 256 MiB (> 126 MB L2), then read another
     # 256 MiB so the lines left in L2 are clean (a write-only flush leaves
     # ~126 MB of dirty lines whose write-back would land in the timed region)
@@ -1068,11 +1190,13 @@ def main():
         e2e = {"value": round(total_bytes / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(e2e_ms, 4),
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
 
-    study = app = kst = None
+    study = app = kst = l1 = None
     if rank == 0 and not args.no_study:
         study = throttle_study(catt, torch, w, flush)
         app = app_study(catt, torch, w, flush)
         kst = kernel_study(catt, torch, w, flush)
+        if world == 1 and not args.no_l1:
+            l1 = l1_pass(args, study)
 
     # ---- roofline of the dominant loop
     dom = max((i for i in range(len(w.loops)) if w.loops[i].kind != "collective"), key=lambda i: loop_ms[i])
@@ -1091,6 +1215,20 @@ def main():
         roof = {"bound": "hbm", "kernel": lp.name, "achieved": round(ach, 2), "peak": peak, "unit": "GB/s",
                 "frac": round(ach / peak, 4), "traffic": ncu_traffic(w.name) if w.variant == type(w).variant else None,
                 "peak_source": f"{peak_src} (MEASURED_PEAKS.json hbm_gbs)" if peak_src == "measured" else "fallback"}
+
+    # ---- the dominant loop's rate on every rank (max-over-ranks timing above
+    # is the job's; this is each GPU's own roofline)
+    if world > 1:
+        import torch.distributed as dist
+        mine = torch.tensor([loop_ms[dom]], device="cuda", dtype=torch.float64)
+        allr = [torch.zeros_like(mine) for _ in range(world)]
+        dist.all_gather(allr, mine)
+        roof["per_rank"] = []
+        for r_, t_ in enumerate(allr):
+            ms_r = float(t_.item())
+            a_r = (w.flops / (ms_r * 1e-3) / 1e12) if roof["unit"] == "TFLOP/s" else lp.nbytes / (ms_r * 1e-3) / 1e9
+            roof["per_rank"].append({"rank": r_, "ms": round(ms_r, 5), "achieved": round(a_r, 2),
+                                     "frac": round(a_r / roof["peak"], 4)})
 
     # ---- context: a plain device copy moving the same bytes as the dominant
     # loop, timed the same way (flush, queued events). At 64 MiB a single
@@ -1151,6 +1289,19 @@ def main():
                 cpu_bytes = step_bytes * min(w.rows, 8192) / w.rows
             cpu = {"value": round(cpu_bytes / sec / 1e9, 3), "unit": "GB/s", "cores": oracle.num_threads(),
                    "kind": "oracle", "sample": f"{reps} x one oracle step ({w.name}), {1e3 * sec:.1f} ms each"}
+            # the same oracle on one host thread (SURVEY 8(d) oracle timing (i))
+            nthr = oracle.num_threads()
+            oracle.set_num_threads(1)
+            try:
+                reps1, t0 = 0, time.perf_counter()
+                while reps1 < 1 or time.perf_counter() - t0 < args.cpu_seconds / 2:
+                    w.cpu_oracle_step(oracle, host)
+                    reps1 += 1
+                sec1 = (time.perf_counter() - t0) / reps1
+            finally:
+                oracle.set_num_threads(nthr)
+            cpu["single_thread"] = {"value": round(cpu_bytes / sec1 / 1e9, 3), "unit": "GB/s", "cores": 1,
+                                    "sample": f"{reps1} x the same step, {1e3 * sec1:.1f} ms each"}
         except Exception as ex:                     # pragma: no cover
             cpu = {"value": None, "unit": "GB/s", "cores": None, "kind": "oracle", "sample": f"failed: {ex}"}
 
@@ -1163,13 +1314,19 @@ def main():
                        "rows_per_rank": getattr(w, "rows", None), "parallelism": f"row-shard x{world}"},
             "loops": {lp.name: {"ms": round(loop_ms[i], 5),
                                 "gbs": round(lp.nbytes / (loop_ms[i] * 1e-3) / 1e9, 1),
-                                "plan": w.plans.get(lp.name)} for i, lp in enumerate(w.loops)},
+                                "plan": [dict(w.plans[k], loop=k) for k in lp.plans if k in w.plans] or None}
+                      for i, lp in enumerate(w.loops)},
+            "analysis_us": max([p_["analysis_us"] for p_ in w.plans.values()] +
+                               [r_.get("analysis_us", 0) for r_ in (study or [])] or [None]),
             "collective_ms": round(statistics.mean(coll), 5) if world > 1 else 0.0,
             "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": len(w.loops) * args.steps,
             "clocks": clk,
+            "l1_hit_pct": ({role: study[0]["l1"][role]["l1_hit_pct"] for role in ("catt", "paper", "full", "best")
+                            if role in study[0].get("l1", {})} if study and l1 and l1.get("status") == "ok" else None),
+            "l1_pass": l1,
             "throttle_study": study,
             "bftt_vs_catt": app,
             "per_loop_in_one_kernel": kst,
