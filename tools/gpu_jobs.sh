@@ -12,6 +12,7 @@
 #   launches  ncu launch list of the default bench (gpu__time_duration)
 #   ncu       ncu --set full of the default bench's dominant kernel
 #   sass      per-kernel SASS opcode summary of libcatt.so
+#   mcprobe   NVLS multicast support with one visible GPU (tools/multicast_probe)
 export PYTHONPATH=.
 TAG=${TAG:-$(echo "$@" | tr ' ' '_')}
 O=gpurun_out/$TAG
@@ -26,10 +27,13 @@ for job in "$@"; do
       timeout 2400 python -m pytest tests -m gpu -q -x > $O/pytest_gpu.txt 2>&1; echo "rc=$?" >> $O/pytest_gpu.txt ;;
     occ)
       timeout 600 python -m pytest tests/test_gpu.py -m gpu -q -k "occupancy or residency" > $O/pytest_occ.txt 2>&1; echo "rc=$?" >> $O/pytest_occ.txt ;;
-    sanitize)
+    sanitize|sanitize_mem)
       S=$O/sanitizer; mkdir -p $S
       timeout 1500 $CS --tool memcheck python tools/sanitize_cases.py > $S/memcheck_all.txt 2>&1; echo "rc=$?" >> $S/memcheck_all.txt
       timeout 1200 $CS --tool synccheck python tools/sanitize_cases.py > $S/synccheck_all.txt 2>&1; echo "rc=$?" >> $S/synccheck_all.txt
+      # initcheck without the kernel filter: torch's fills (zeros) must be seen as writes
+      timeout 1500 compute-sanitizer --print-limit 50 --error-exitcode 9 --tool initcheck python tools/sanitize_cases.py > $S/initcheck_all.txt 2>&1; echo "rc=$?" >> $S/initcheck_all.txt
+      [ $job = sanitize_mem ] && continue
       for c in gate_sem gate_barrier cta_counter smem_pad staged coop fused fused_graph onekernel kmeans km_iter tiles; do
         timeout 900 $CS --tool racecheck --racecheck-report analysis python tools/sanitize_cases.py $c > $S/racecheck_$c.txt 2>&1; echo "rc=$?" >> $S/racecheck_$c.txt
       done
@@ -51,6 +55,9 @@ for job in "$@"; do
     ncu)
       timeout 900 ncu --set full --clock-control none --import-source on -k regex:${NCU_KERNEL:-fused} -s 3 -c 1 -o $O/ncu_default -f \
         python bench.py --steps 1 --warmup 3 --no-study --no-e2e --cpu-seconds 0 > $O/ncu_default.log 2>&1 ;;
+    mcprobe)
+      nvidia-smi topo -m > $O/topo.txt 2>&1
+      timeout 120 ./tools/multicast_probe > $O/multicast_probe.txt 2>&1; echo "rc=$?" >> $O/multicast_probe.txt ;;
     sass)
       python tools/sass_summary.py paper_conf_icpp_kimhlsh19_b200/libcatt.so > $O/sass_summary.txt 2>&1 ;;
     *)
