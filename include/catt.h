@@ -135,13 +135,18 @@ typedef struct {
  * again (stores, loads without reuse). cta_fallback (R27; 0 = off): when
  * nothing at or above min_warps_sm fits and an SM holds several CTAs (T >= 2),
  * cap whole CTAs -- (W, m) with the smallest m such that min_warps_sm <= W m
- * <= 2 min_warps_sm -- instead of gating warps down to the floor. Paper mode
- * ignores them. */
+ * <= 2 min_warps_sm -- instead of gating warps down to the floor.
+ * stream_floor (R29; 0 = off): with one CTA per SM (T = 1) and S >= 2
+ * memory-divergent reused loads (each meeting the divergent_lines /
+ * min_retouch / min_reuse_trip terms), the floor is ceil(min_warps_sm / S):
+ * S streams per warp keep as many lines in flight as S times the warps.
+ * Paper mode ignores them. */
 typedef struct {
   int32_t num_sms, max_warps_sm, max_ctas_sm, regs_sm, reg_alloc_unit, warp_size;
   int32_t smem_alloc_unit, reserved_smem_cta, line_bytes, n_carveouts;
   int32_t min_warps_sm, divergent_lines;
   int32_t min_retouch, min_reuse_trip, max_stream_pct, cta_fallback;
+  int32_t stream_floor, reserved_;
   int32_t carveout_kb[CATT_MAX_CARVEOUTS];
   int32_t carveout_pct[CATT_MAX_CARVEOUTS];
   int64_t l1d_bytes[CATT_MAX_CARVEOUTS];
@@ -220,7 +225,8 @@ enum {
   CATT_K_KMEANS_T = 10, /* KM transpose: out[f*ld + p] = in[p*nf + f]          */
   CATT_K_CORR = 11,   /* CORR loop: symmat[j1][j2] = sum_i d[i][j1] d[i][j2]   */
   CATT_K_GEMM = 12,   /* C = beta C + alpha A B, 2-D block 32 x 8 (CI control) */
-  CATT_K_COUNT = 13
+  CATT_K_ROWS3 = 13,  /* y = A x + B x + C x, thread per row (three divergent streams; rule studies) */
+  CATT_K_COUNT = 14
 };
 
 /* Problem sizes: ATAX/BICG m x n (rows, cols); MVT/GESUMMV n (m ignored);
@@ -417,11 +423,17 @@ catt_status catt_kmeans(const float* feat, int64_t ld, int64_t npoints, int32_t 
  *   mode CATT_ROWS_ACCUM:   y[i] = y[i] + sum_j A[i*n + j] * x[j]   (y in/out)
  *   mode CATT_ROWS_GESUMMV: tmp[i] = sum_j A[i*n+j] x[j];
  *                           y[i] = alpha*tmp[i] + beta*sum_j B[i*n+j] x[j]
- * B and tmp are used only by CATT_ROWS_GESUMMV (else may be NULL).
+ *   mode CATT_ROWS_SUM3:    y[i] = (sA + sB) + sC, sX = sum_j X[i*n + j] * x[j]
+ *                           each by fmaf in j order; B holds the m x n matrices
+ *                           B and C back to back (2 m n floats); LITERAL only.
+ *                           Three memory-divergent streams per thread: the
+ *                           loop the decision-rule studies use (DESIGN R29).
+ * B and tmp are used only by CATT_ROWS_GESUMMV (B also by CATT_ROWS_SUM3;
+ * else may be NULL).
  * Column loop (ATAX#2, BICG#1, MVT#2; coalesced): for j < n,
  *   y[j] = (accumulate ? y[j] : 0) + sum_i A[i*n + j] * v[i].
  * A is m x n row-major in both. */
-enum { CATT_ROWS_STORE = 0, CATT_ROWS_ACCUM = 1, CATT_ROWS_GESUMMV = 2 };
+enum { CATT_ROWS_STORE = 0, CATT_ROWS_ACCUM = 1, CATT_ROWS_GESUMMV = 2, CATT_ROWS_SUM3 = 3 };
 catt_status catt_rows(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t m, int64_t n,
                       float alpha, float beta, int32_t mode, const catt_throttle* t, void* stream);
 catt_status catt_cols(const float* A, const float* v, float* y, int64_t m, int64_t n, int32_t accumulate,
@@ -546,7 +558,8 @@ catt_status catt_dual_group_peer(const catt_dual_problem* probs, int32_t count, 
  * after the grid barrier, end) for CTAs < 1024. Copies the first n of the
  * 6144 u64 values (CTA-major) to host memory `out` (synchronous). */
 catt_status catt_fused_trace(uint64_t* out, int32_t n);
-/* ABI revision of this header: 4 (added catt_kernel_occupancy; 3: catt_hw's
+/* ABI revision of this header: 5 (catt_hw.stream_floor + reserved_,
+ * CATT_K_ROWS3, CATT_ROWS_SUM3; 4 added catt_kernel_occupancy; 3: catt_hw's
  * last reserved word became cta_fallback; 2 added min_retouch,
  * min_reuse_trip, max_stream_pct). */
 int catt_abi_version(void);

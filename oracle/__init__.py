@@ -52,6 +52,7 @@ def lib():
         L.orc_bicg.argtypes = [ctypes.c_int, f32p, f32p, f32p, f32p, f32p, i64, i64]
         L.orc_mvt.argtypes = [ctypes.c_int, f32p, f32p, f32p, f32p, f32p, i64]
         L.orc_gesummv.argtypes = [ctypes.c_int, f32p, f32p, f32p, f32p, f32p, i64, ctypes.c_float, ctypes.c_float]
+        L.orc_rows3.argtypes = [ctypes.c_int, f32p, f32p, f32p, f32p, f32p, i64, i64]
         L.orc_syrk.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float]
         L.orc_syrk_rows.argtypes = [ctypes.c_int, f32p, f32p, i64, i64, ctypes.c_float, ctypes.c_float,
                                     ctypes.POINTER(ctypes.c_int64), i64, f32p]
@@ -130,6 +131,16 @@ def gesummv(A, B, x, alpha, beta, mode=SEQ_FMAF):
     y, tmp = np.empty(n, np.float32), np.empty(n, np.float32)
     lib().orc_gesummv(mode, _p(A), _p(B), _p(x), _p(y), _p(tmp), n, alpha, beta)
     return y, tmp
+
+
+def rows3(A, B, C, x, mode=SEQ_FMAF):
+    """y = (A x + B x) + C x, each product an fmaf chain in j order (the
+    three-stream row loop, DESIGN R29)."""
+    A, B, C, x = _f32(A), _f32(B), _f32(C), _f32(x)
+    m, n = A.shape
+    y = np.empty(m, np.float32)
+    lib().orc_rows3(mode, _p(A), _p(B), _p(C), _p(x), _p(y), m, n)
+    return y
 
 
 def syrk(A, C, alpha, beta, mode=SEQ_FMAF):

@@ -23,7 +23,9 @@ The rule (readings R17-R19, R23, R24, R27), restated on traces:
                   bytes of the loop body (R24)
   divergent       some reused load has lines >= divergent_lines and retouch >=
                   min_retouch, and 100 * stream <= max_stream_pct * total (R18,
-                  R23, R24)
+                  R23, R24); S = the number of such loads
+  floor           min_warps_sm, or ceil(min_warps_sm / S) when stream_floor is on,
+                  T = 1 and S >= 2 (R29)
   fits(a, m)      zero intra-thread capacity misses when a warps per CTA and m
                   CTAs per SM run SM 0's first T CTAs through an LRU of the L1D's
                   lines (R12)
@@ -50,7 +52,8 @@ from . import lru
 
 # DESIGN.md R18 (floor 8 warps/SM, >= 8 lines per request), R23 (>= 16
 # re-touches), R24 (<= 25 % stream bytes), R27 (CTA fallback on)
-B200_GUARDS = dict(min_warps_sm=8, divergent_lines=8, min_retouch=16, max_stream_pct=25, cta_fallback=1)
+B200_GUARDS = dict(min_warps_sm=8, divergent_lines=8, min_retouch=16, max_stream_pct=25, cta_fallback=1,
+                   stream_floor=0)
 # shared-memory options (KB) and the L1D each leaves (KB, measured)
 B200_L1D_KB = {0: 218, 8: 218, 16: 218, 32: 218, 64: 186, 100: 150, 132: 118, 164: 86, 196: 53, 228: 21}
 
@@ -93,10 +96,14 @@ def trace_inputs(kernel, line: int = lru.LINE) -> TraceInputs:
                        total_bytes=sum(nbytes.values()))
 
 
+def divergent_loads(inp: TraceInputs, guards: Dict) -> int:
+    """How many reused loads are memory-divergent (R18, R23): the streams of R29."""
+    return sum(1 for i in inp.lines if inp.reuse[i] and not inp.stored[i] and inp.lines[i] >= guards["divergent_lines"]
+               and inp.retouch[i] >= guards["min_retouch"])
+
+
 def divergent(inp: TraceInputs, guards: Dict) -> bool:
-    hot = any(inp.reuse[i] and not inp.stored[i] and inp.lines[i] >= guards["divergent_lines"]
-              and inp.retouch[i] >= guards["min_retouch"] for i in inp.lines)
-    return hot and 100 * inp.stream_bytes <= guards["max_stream_pct"] * inp.total_bytes
+    return divergent_loads(inp, guards) > 0 and 100 * inp.stream_bytes <= guards["max_stream_pct"] * inp.total_bytes
 
 
 class _Loads(lru.Kernel):
@@ -126,6 +133,9 @@ def decide(kernel, W: int, T: int, l1d_lines: int, num_sms: int, guards: Dict = 
     if not divergent(inp, guards):
         return W, T, "none(guard)"
     floor = guards["min_warps_sm"]
+    S = divergent_loads(inp, guards)
+    if guards.get("stream_floor", 0) and T == 1 and S >= 2:          # R29: S streams per warp
+        floor = -(-floor // S)
     admissible = [(a, m) for a in range(1, W + 1) if W % a == 0 for m in range(1, T + 1)
                   if (a, m) != (W, T) and a * m >= floor]
     if not admissible:

@@ -36,7 +36,9 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
       when stores and loads without reuse exceed max_stream_pct % of a lane's
       bytes per iteration. R27 (hw key cta_fallback): when that fallback is
       taken and an SM holds several CTAs (T >= 2), cap whole CTAs instead --
-      (W, m), the smallest m with floor <= W m <= 2 floor.
+      (W, m), the smallest m with floor <= W m <= 2 floor. R29 (hw key
+      stream_floor): with T = 1 and S >= 2 such divergent reused loads, the
+      floor is ceil(min_warps_sm / S).
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -271,6 +273,7 @@ class Model:
         self.line = hw["line_bytes"]
         self.paper = loop.mode == MODE_PAPER
         self.divergent = True
+        self.streams = 0
         # contention is measured only "for loops where cache locality presents"
         self.locality = any(has_locality(r, loop.trips, self.line) for r in loop.refs
                             if not (r.flags & REF_NOT_L1))
@@ -297,9 +300,10 @@ class Model:
             self.lines_per_warp_iter = sum(per_ref)
             div = hw.get("divergent_lines", 0)
             rt, rtrip = hw.get("min_retouch", 0), hw.get("min_reuse_trip", 0)
-            self.divergent = (div <= 0 and rt <= 0 and rtrip <= 0 and hw.get("max_stream_pct", 0) <= 0) or any(
-                n >= div and retouches(r, loop.trips, self.line) >= rt and reuse_trip(r, loop.trips, self.line) >= rtrip
-                for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line))
+            hot = [n >= div and retouches(r, loop.trips, self.line) >= rt and reuse_trip(r, loop.trips, self.line) >= rtrip
+                   for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line)]
+            self.streams = sum(hot)                   # R29: memory-divergent reused loads
+            self.divergent = (div <= 0 and rt <= 0 and rtrip <= 0 and hw.get("max_stream_pct", 0) <= 0) or any(hot)
             # R24: bytes per lane and iteration of streams L1 cannot serve again
             pct = hw.get("max_stream_pct", 0)
             if pct > 0:
@@ -368,6 +372,8 @@ def analyse(loop: Loop, hw: Dict) -> Dict:
         if not M.divergent:
             return done(W, T, full, FIT_NONE_NEEDED | FIT_GUARDED)
         floor_w = hw.get("min_warps_sm", 0)
+        if hw.get("stream_floor", 0) > 0 and T == 1 and M.streams >= 2:     # R29
+            floor_w = _ceil_div(floor_w, M.streams)
         cands = [(a, m) for a in range(W, 0, -1) if W % a == 0 for m in range(T, 0, -1)
                  if (a, m) != (W, T) and a * m >= floor_w]
         cands.sort(key=lambda am: (-am[0] * am[1], -am[0]))

@@ -190,6 +190,36 @@ int orc_gesummv(int mode, const float* A, const float* B, const float* x, float*
   return 0;
 }
 
+/* ---------------------------------------------------------------- three-matrix row loop
+ * y[i] = (sum_j A[i][j] x[j] + sum_j B[i][j] x[j]) + sum_j C[i][j] x[j]: the
+ * row loop with three memory-divergent streams per thread (not a PolyBench
+ * kernel; the decision-rule studies' vehicle, DESIGN reading R29). Each sum
+ * is its own fmaf chain in j order, as GESUMMV's two are (P:110-131 row form). */
+int orc_rows3(int mode, const float* A, const float* B, const float* C, const float* x, float* y, int64_t m,
+              int64_t n) {
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < m; ++i) {
+    if (mode == ORC_SEQ_FMAF) {
+      float a = 0.0f, b = 0.0f, c = 0.0f;
+      for (int64_t j = 0; j < n; ++j) {
+        a = fmaf(A[i * n + j], x[j], a);
+        b = fmaf(B[i * n + j], x[j], b);
+        c = fmaf(C[i * n + j], x[j], c);
+      }
+      y[i] = (a + b) + c;
+    } else {
+      double a = 0.0, b = 0.0, c = 0.0;
+      for (int64_t j = 0; j < n; ++j) {
+        a += (double)A[i * n + j] * (double)x[j];
+        b += (double)B[i * n + j] * (double)x[j];
+        c += (double)C[i * n + j] * (double)x[j];
+      }
+      y[i] = (float)((a + b) + c);
+    }
+  }
+  return 0;
+}
+
 /* ---------------------------------------------------------------- SYRK
  * PolyBench/GPU syrk (Table 2; CI group), A is n x m, C is n x n in/out,
  * full square (no triangle), 2-D thread block over (i, j):

@@ -24,12 +24,12 @@ REF_IRREGULAR, REF_STORE, REF_NOT_L1 = 1, 2, 4
 MODE_UNION, MODE_PAPER = 0, 1
 FIT_NONE_NEEDED, FIT_WARP, FIT_CTA, FIT_UNRESOLVABLE, FIT_GUARDED = 1, 2, 4, 8, 16
 VAR_LITERAL, VAR_VEC4, VAR_STAGED, VAR_COOP, VAR_REGS, VAR_FUSED, VAR_BYPASS = 0, 1, 2, 3, 4, 5, 6
-ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV = 0, 1, 2
+ROWS_STORE, ROWS_ACCUM, ROWS_GESUMMV, ROWS_SUM3 = 0, 1, 2, 3
 PEER_HANDLE_BYTES = 64
 GATE_SEMAPHORE, GATE_BARRIER = 0, 1
 CAP_SM_COUNTER, CAP_SMEM_PAD = 0, 1
 (K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K,
- K_KMEANS_T, K_CORR, K_GEMM) = range(13)
+ K_KMEANS_T, K_CORR, K_GEMM, K_ROWS3) = range(14)
 
 VARIANTS = {"literal": VAR_LITERAL, "vec4": VAR_VEC4, "staged": VAR_STAGED, "coop": VAR_COOP, "regs": VAR_REGS,
             "fused": VAR_FUSED, "bypass": VAR_BYPASS}
@@ -64,12 +64,13 @@ class Hw(ctypes.Structure):
                 ("min_warps_sm", ctypes.c_int32), ("divergent_lines", ctypes.c_int32),
                 ("min_retouch", ctypes.c_int32), ("min_reuse_trip", ctypes.c_int32),
                 ("max_stream_pct", ctypes.c_int32), ("cta_fallback", ctypes.c_int32),
+                ("stream_floor", ctypes.c_int32), ("reserved_", ctypes.c_int32),
                 ("carveout_kb", ctypes.c_int32 * MAX_CARVEOUTS), ("carveout_pct", ctypes.c_int32 * MAX_CARVEOUTS),
                 ("l1d_bytes", ctypes.c_int64 * MAX_CARVEOUTS)]
 
     def as_dict(self):
         n = self.n_carveouts
-        d = {f: getattr(self, f) for f, _ in self._fields_[:16]}
+        d = {f: getattr(self, f) for f, _ in self._fields_[:17]}
         d["carveout_kb"] = list(self.carveout_kb[:n])
         d["carveout_pct"] = list(self.carveout_pct[:n])
         d["l1d_bytes"] = list(self.l1d_bytes[:n])
@@ -78,7 +79,7 @@ class Hw(ctypes.Structure):
     @classmethod
     def from_dict(cls, d):
         h = cls()
-        for f, _ in cls._fields_[:16]:
+        for f, _ in cls._fields_[:17]:
             if f in d:
                 setattr(h, f, d[f])
         n = len(d["carveout_kb"])
@@ -241,6 +242,7 @@ def paper_rule(hw: Hw) -> Hw:
     h.min_reuse_trip = 0
     h.max_stream_pct = 0
     h.cta_fallback = 0
+    h.stream_floor = 0
     return h
 
 
@@ -422,9 +424,11 @@ def gesummv(A, B, x, alpha, beta, y=None, tmp=None, t: Optional[Throttle] = None
 
 
 def rows(A, x, y, mode=ROWS_STORE, B=None, tmp=None, alpha=0.0, beta=0.0, t: Optional[Throttle] = None):
-    """One row loop (catt_rows): y = A x (STORE), y += A x (ACCUM), or GESUMMV."""
+    """One row loop (catt_rows): y = A x (STORE), y += A x (ACCUM), GESUMMV, or
+    SUM3 (y = A x + B x + C x with B holding B and C back to back)."""
     m, n = A.shape
-    _check(lib().catt_rows(_dev(A, "A", n=m * n), _dev(B, "B", n=m * n) if B is not None else None, _dev(x, "x", n=n), _dev(y, "y", n=m),
+    nb = (2 if mode == ROWS_SUM3 else 1) * m * n
+    _check(lib().catt_rows(_dev(A, "A", n=m * n), _dev(B, "B", n=nb) if B is not None else None, _dev(x, "x", n=n), _dev(y, "y", n=m),
                            _dev(tmp, "tmp", n=m) if tmp is not None else None, m, n, float(alpha), float(beta), mode,
                            _tp(t), _stream()), "catt_rows")
     return y

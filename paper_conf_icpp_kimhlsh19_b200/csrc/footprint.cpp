@@ -240,8 +240,10 @@ class Model {
           rtrip = std::max(rtrip, d_.trip[k]);
         }
       if (reuse && int64_t(s.size()) >= hw_.divergent_lines && retouch >= hw_.min_retouch &&
-          rtrip >= hw_.min_reuse_trip)
+          rtrip >= hw_.min_reuse_trip) {
         divergent_ = true;
+        ++streams_;                    // R29: one more memory-divergent reused load
+      }
     }
     // R24: no throttle when more than max_stream_pct % of a lane's bytes per
     // iteration belong to streams L1 cannot serve again (stores, loads
@@ -310,6 +312,7 @@ class Model {
 
   bool locality_ = false;
   bool divergent_ = true;  // some reused reference is memory-divergent (B200 guard)
+  int32_t streams_ = 0;    // how many (R29)
   int64_t lines_per_warp_iter_ = 0, reuse_span_ = 0;
 
  private:
@@ -348,7 +351,7 @@ catt_status validate(const catt_loop_desc* d, const catt_hw* hw) {
   if (hw->line_bytes < 4 || hw->n_carveouts < 1 || hw->n_carveouts > CATT_MAX_CARVEOUTS) return CATT_EINVAL;
   if (hw->smem_alloc_unit < 1 || hw->reg_alloc_unit < 1 || hw->regs_sm < 1) return CATT_EINVAL;
   if (hw->min_warps_sm < 0 || hw->divergent_lines < 0 || hw->min_retouch < 0 || hw->min_reuse_trip < 0 ||
-      hw->max_stream_pct < 0 || hw->max_stream_pct > 100)
+      hw->max_stream_pct < 0 || hw->max_stream_pct > 100 || hw->stream_floor < 0)
     return CATT_EINVAL;
   for (int i = 1; i < hw->n_carveouts; ++i)
     if (hw->carveout_kb[i] <= hw->carveout_kb[i - 1]) return CATT_EINVAL;
@@ -398,7 +401,10 @@ extern "C" catt_status catt_footprint(const catt_loop_desc* desc, const catt_hw*
     // CTAs with more warps each; never below min_warps_sm; if nothing at or
     // above the floor fits, the most throttled pair that respects it.
     if (!M.divergent_) return done(W, T, full, CATT_FIT_NONE_NEEDED | CATT_FIT_GUARDED);
-    const int32_t floor_w = std::max(0, hw->min_warps_sm);
+    int32_t floor_w = std::max(0, hw->min_warps_sm);
+    // R29: with one CTA per SM, S divergent streams per warp keep the lines
+    // in flight of S times as many warps: the floor scales by 1/S
+    if (hw->stream_floor > 0 && T == 1 && M.streams_ >= 2) floor_w = (floor_w + M.streams_ - 1) / M.streams_;
     std::vector<std::pair<int32_t, int32_t>> cands;
     for (int32_t a = W; a >= 1; --a) {
       if (W % a) continue;

@@ -22,11 +22,11 @@
 
 namespace catt {
 
-enum { EPI_STORE = 0, EPI_ACCUM = 1, EPI_GESUMMV = 2 };
+enum { EPI_STORE = 0, EPI_ACCUM = 1, EPI_GESUMMV = 2, EPI_SUM3 = 3 };
 
 struct RowArgs {
   const float* A;
-  const float* B;   // second matrix (GESUMMV) or nullptr
+  const float* B;   // second matrix (GESUMMV), the second and third back to back (SUM3), or nullptr
   const float* x;
   float* y;         // output (EPI_ACCUM: in/out)
   float* tmp;       // GESUMMV: A x
@@ -59,8 +59,10 @@ __device__ __forceinline__ float ld_na(const float* p) {
 }
 
 template <int NMAT, int EPI>
-__device__ __forceinline__ void row_epilogue(const RowArgs& a, int64_t i, float acc, float acc2) {
-  if (EPI == EPI_GESUMMV) {
+__device__ __forceinline__ void row_epilogue(const RowArgs& a, int64_t i, float acc, float acc2, float acc3 = 0.0f) {
+  if (EPI == EPI_SUM3) {
+    a.y[i] = __fadd_rn(__fadd_rn(acc, acc2), acc3);
+  } else if (EPI == EPI_GESUMMV) {
     a.tmp[i] = acc;
     a.y[i] = __fmaf_rn(a.alpha, acc, __fmul_rn(a.beta, acc2));
   } else {
@@ -74,8 +76,9 @@ __device__ __forceinline__ void row_epilogue(const RowArgs& a, int64_t i, float 
 // only, so the divergent rows never occupy L1; the alternative to throttling
 // that the paper discusses as related work)
 template <int NMAT, int EPI, int VM>
-__global__ void __launch_bounds__(1024, (NMAT == 2 && VM == 1) ? 1 : 2) row_thread_kernel(RowArgs a) {
+__global__ void __launch_bounds__(1024, (NMAT >= 2 && VM == 1) ? 1 : 2) row_thread_kernel(RowArgs a) {
   constexpr bool VEC = VM == 1, BYPASS = VM == 2;
+  static_assert(NMAT < 3 || VM == 0, "the 3-matrix row loop is literal only");
   __shared__ int slots;
   gate_init(&slots, a.t);
   __syncthreads();
@@ -85,16 +88,18 @@ __global__ void __launch_bounds__(1024, (NMAT == 2 && VM == 1) ? 1 : 2) row_thre
     if (i >= a.M) return;
     const int64_t N = a.N;
     const float* __restrict__ ar = a.A + i * N;
-    const float* __restrict__ br = (NMAT == 2) ? a.B + i * N : nullptr;
+    const float* __restrict__ br = (NMAT >= 2) ? a.B + i * N : nullptr;
+    const float* __restrict__ cr = (NMAT == 3) ? a.B + a.M * N + i * N : nullptr;
     const float* __restrict__ x = a.x;
     float acc = (EPI == EPI_ACCUM) ? a.y[i] : 0.0f;
-    float acc2 = 0.0f;
+    float acc2 = 0.0f, acc3 = 0.0f;
     if (!VEC) {
 #pragma unroll 2
       for (int64_t j = 0; j < N; ++j) {
         const float xv = x[j];
         acc = fmaf(BYPASS ? __ldcg(ar + j) : ar[j], xv, acc);
-        if (NMAT == 2) acc2 = fmaf(BYPASS ? __ldcg(br + j) : br[j], xv, acc2);
+        if (NMAT >= 2) acc2 = fmaf(BYPASS ? __ldcg(br + j) : br[j], xv, acc2);
+        if (NMAT == 3) acc3 = fmaf(cr[j], xv, acc3);
       }
     } else {
       const float4* __restrict__ a4 = reinterpret_cast<const float4*>(ar);
@@ -118,7 +123,7 @@ __global__ void __launch_bounds__(1024, (NMAT == 2 && VM == 1) ? 1 : 2) row_thre
         }
       }
     }
-    row_epilogue<NMAT, EPI>(a, i, acc, acc2);
+    row_epilogue<NMAT, EPI>(a, i, acc, acc2, acc3);
   });
   cta_exit(a.t);
 }
@@ -465,6 +470,20 @@ void row_warp_launch(int S, unsigned grid, size_t dyn, cudaStream_t s, const Row
   }
 }
 
+// the 3-matrix row loop (CATT_ROWS_SUM3): literal only, for the decision-rule
+// studies (three divergent streams per thread)
+catt_status launch_row3(RowArgs a, const catt_throttle* t, cudaStream_t s) {
+  if (a.M == 0) return CATT_OK;
+  if (variant_of(t) != CATT_VAR_LITERAL) return CATT_EINVAL;
+  const int threads = cta_threads_or(t, 256);
+  const void* f = (const void*)row_thread_kernel<3, EPI_SUM3, 0>;
+  size_t dyn = 0;
+  catt_status st = prepare_launch(f, t, threads, 0, true, &a.t, &dyn);
+  if (st != CATT_OK) return st;
+  row_thread_kernel<3, EPI_SUM3, 0><<<dim3(unsigned((a.M + threads - 1) / threads)), threads, dyn, s>>>(a);
+  return after_launch();
+}
+
 template <int NMAT, int EPI>
 catt_status launch_row_t(RowArgs a, const catt_throttle* t, cudaStream_t s) {
   const int var = variant_of(t);
@@ -588,6 +607,7 @@ const void* col_tma_func();
 
 // Kernel instance a loop + variant launches (for attributes / descriptors).
 const void* gemv_func(int loop, int variant, bool vec_ok) {
+  if (loop == CATT_K_ROWS3) return (const void*)row_thread_kernel<3, EPI_SUM3, 0>;
   const bool row = loop == CATT_K_ATAX_1 || loop == CATT_K_BICG_2 || loop == CATT_K_MVT_1 || loop == CATT_K_GESUMMV;
   if (row) {
     const int nmat = loop == CATT_K_GESUMMV ? 2 : 1;
@@ -623,6 +643,7 @@ const void* gemv_func(int loop, int variant, bool vec_ok) {
 catt_status launch_row(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t M, int64_t N,
                        float alpha, float beta, int epi, const catt_throttle* t, cudaStream_t s) {
   RowArgs a{A, B, x, y, tmp, M, N, alpha, beta, Throttle{}};
+  if (epi == EPI_SUM3) return launch_row3(a, t, s);
   if (epi == EPI_GESUMMV) return launch_row_t<2, EPI_GESUMMV>(a, t, s);
   if (epi == EPI_ACCUM) return launch_row_t<1, EPI_ACCUM>(a, t, s);
   return launch_row_t<1, EPI_STORE>(a, t, s);
@@ -755,9 +776,10 @@ extern "C" catt_status catt_gesummv(const float* A, const float* B, const float*
 extern "C" catt_status catt_rows(const float* A, const float* B, const float* x, float* y, float* tmp, int64_t m,
                                  int64_t n, float alpha, float beta, int32_t mode, const catt_throttle* t,
                                  void* stream) {
-  if (check_common(m, n) != CATT_OK || mode < CATT_ROWS_STORE || mode > CATT_ROWS_GESUMMV) return CATT_EINVAL;
+  if (check_common(m, n) != CATT_OK || mode < CATT_ROWS_STORE || mode > CATT_ROWS_SUM3) return CATT_EINVAL;
   if ((m * n > 0 && !A) || (n > 0 && !x) || (m > 0 && !y)) return CATT_EINVAL;
   if (mode == CATT_ROWS_GESUMMV && ((m * n > 0 && !B) || (m > 0 && !tmp))) return CATT_EINVAL;
+  if (mode == CATT_ROWS_SUM3 && m * n > 0 && !B) return CATT_EINVAL;
   return launch_row(A, B, x, y, tmp, m, n, alpha, beta, mode, t, static_cast<cudaStream_t>(stream));
 }
 

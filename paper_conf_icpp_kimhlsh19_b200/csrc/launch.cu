@@ -230,7 +230,8 @@ int default_threads(int loop, int variant) {
 }
 
 bool is_row(int loop) {
-  return loop == CATT_K_ATAX_1 || loop == CATT_K_BICG_2 || loop == CATT_K_MVT_1 || loop == CATT_K_GESUMMV;
+  return loop == CATT_K_ATAX_1 || loop == CATT_K_BICG_2 || loop == CATT_K_MVT_1 || loop == CATT_K_GESUMMV ||
+         loop == CATT_K_ROWS3;
 }
 bool is_col(int loop) { return loop == CATT_K_ATAX_2 || loop == CATT_K_BICG_1 || loop == CATT_K_MVT_2; }
 
@@ -329,14 +330,16 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
     const int64_t M = (loop == CATT_K_MVT_1 || loop == CATT_K_GESUMMV) ? prob->n : prob->m;
     const int64_t N = prob->n;
     if (M < 1 || N < 1) return CATT_EINVAL;
-    const bool two = loop == CATT_K_GESUMMV;
+    const bool two = loop == CATT_K_GESUMMV, three = loop == CATT_K_ROWS3;
+    if (three && var != CATT_VAR_LITERAL) return CATT_EINVAL;
     out->n_loops = 1;
     out->extent[0] = M;
     if (var == CATT_VAR_LITERAL || var == CATT_VAR_BYPASS) {
       const int32_t fa = var == CATT_VAR_BYPASS ? CATT_REF_NOT_L1 : 0;  // BYPASS: the rows skip L1
       refs[n++] = mkref(N, 0, 1, 0, 4, 1, fa);                    // A[i*N + j]
       refs[n++] = mkref(0, 0, 1, 0, 4, 2, 0);                     // x[j]
-      if (two) refs[n++] = mkref(N, 0, 1, 0, 4, 3, fa);           // B[i*N + j]
+      if (two || three) refs[n++] = mkref(N, 0, 1, 0, 4, 3, fa);  // B[i*N + j]
+      if (three) refs[n++] = mkref(N, 0, 1, 0, 4, 4, fa);         // C[i*N + j]
       out->trip[0] = N;
       out->grid[0] = (M + threads - 1) / threads;
     } else if (var == CATT_VAR_VEC4) {
@@ -677,7 +680,7 @@ extern "C" const char* catt_status_str(catt_status s) {
 }
 
 extern "C" int catt_last_cuda_error(void) { return g_last_err; }
-extern "C" int catt_abi_version(void) { return 4; }
+extern "C" int catt_abi_version(void) { return 5; }
 
 // ------------------------------------------------------------ SM partition
 // Green context of >= min_sms SMs and a non-blocking stream in it (catt.h).

@@ -24,14 +24,14 @@ def test_library_loads_and_exports_every_declared_symbol():
     assert declared == set(catt.catt.EXPORTED)
     for name in declared:
         assert hasattr(L, name), name
-    assert L.catt_abi_version() == 4
+    assert L.catt_abi_version() == 5
 
 
 def test_struct_layouts_match_header():
     # sizes of the C structs (x86-64 ABI) as the header defines them
     assert ctypes.sizeof(catt.Ref) == 3 * 8 + 4 * 8 + 8 + 4 * 4
     assert ctypes.sizeof(catt.Throttle) == 8 * 4 + 8
-    assert ctypes.sizeof(catt.Hw) == 16 * 4 + 16 * 4 * 2 + 16 * 8
+    assert ctypes.sizeof(catt.Hw) == 18 * 4 + 16 * 4 * 2 + 16 * 8
     assert ctypes.sizeof(catt.FootprintResult) == 6 * 8 + 6 * 4
 
 
@@ -92,6 +92,7 @@ def _rand_hw(rnd):
                 min_warps_sm=rnd.choice([0, 0, 4, 16]), divergent_lines=rnd.choice([0, 0, 2, 8]),
                 min_retouch=rnd.choice([0, 0, 4, 16]), min_reuse_trip=rnd.choice([0, 0, 8, 30]),
                 max_stream_pct=rnd.choice([0, 0, 25, 60]), cta_fallback=rnd.choice([0, 1]),
+                stream_floor=rnd.choice([0, 1]),
                 carveout_kb=carve, l1d_bytes=[rnd.randint(1, 200) * 128 for _ in carve])
 
 

@@ -128,6 +128,23 @@ def test_gesummv(variant, n):
         assert bits_equal(host(y), y_o) and bits_equal(host(tmp), t_o)
 
 
+@pytest.mark.parametrize("m,n,t", [(130, 70, catt.Throttle()), (1000, 96, catt.Throttle(active_warps=2)),
+                                   (700, 257, catt.Throttle(cta_threads=384, active_warps=3, carveout_kb=228)),
+                                   (148 * 256 * 2 + 5, 64, catt.Throttle(active_ctas=1))])
+def test_rows3_literal_bit_exact(m, n, t):
+    """The three-stream row loop (CATT_ROWS_SUM3, DESIGN R29) through catt_rows,
+    throttled or not: bit-exact to the oracle's fmaf chains."""
+    A, BC, x = si.matrix(5, m, n), si.matrix(105, 2 * m, n), si.values(205, n)
+    y_o = oracle.rows3(A, BC[:m], BC[m:], x)
+    y = torch.empty(m, device="cuda")
+    catt.rows(dev(A), dev(x), y, catt.ROWS_SUM3, B=dev(BC), t=t)
+    assert bits_equal(host(y), y_o)
+    with pytest.raises(catt.CattError):                   # literal only
+        catt.rows(dev(A), dev(x), y, catt.ROWS_SUM3, B=dev(BC), t=catt.Throttle(variant="coop"))
+    with pytest.raises(catt.CattError):                   # B must hold both matrices
+        catt.rows(dev(A), dev(x), y, catt.ROWS_SUM3, B=dev(BC[:m]), t=t)
+
+
 @pytest.mark.parametrize("n", [64, 1024])
 def test_coop_bit_exact_on_dyadic_inputs(n):
     A, p, r = (si.matrix(9, n, n, DYADIC), si.values(19, n, mode=DYADIC), si.values(29, n, mode=DYADIC))

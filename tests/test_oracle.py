@@ -144,6 +144,28 @@ def test_gesummv_vs_numpy_and_special_cases():
     assert _rel(ya, 1.2 * (B64 @ x)) < n * 2.0 ** -24
 
 
+def test_rows3_vs_numpy_and_special_cases():
+    """The three-stream row loop (DESIGN R29): numpy float64 within 3n u; with
+    B = C = 0 it is BICG's q = A p bit for bit (the same fmaf chain, then +0
+    twice); on exact-dyadic inputs it equals numpy exactly; swapping the
+    order of A and C (a wrong stream) changes the rounding."""
+    m, n = 90, 170
+    A, B, C = si.matrix(5, m, n), si.matrix(105, m, n), si.matrix(305, m, n)
+    x = si.values(205, n)
+    y = oracle.rows3(A, B, C, x)
+    ref = (A.astype(np.float64) @ x + B.astype(np.float64) @ x) + C.astype(np.float64) @ x
+    assert _rel(y, ref) < 3 * n * 2.0 ** -24
+    assert _rel(oracle.rows3(A, B, C, x, mode=oracle.SEQ_F64), ref) < 2.0 ** -23
+    z = np.zeros_like(A)
+    q, _ = oracle.bicg(A, x, np.zeros(m, np.float32))
+    assert np.array_equal(oracle.rows3(A, z, z, x), q)
+    D = si.MODE_DYADIC
+    Ad, Bd, Cd, xd = si.matrix(6, m, n, D), si.matrix(7, m, n, D), si.matrix(8, m, n, D), si.values(9, n, mode=D)
+    want = (Ad.astype(np.float64) @ xd + Bd.astype(np.float64) @ xd) + Cd.astype(np.float64) @ xd
+    assert np.array_equal(oracle.rows3(Ad, Bd, Cd, xd), want.astype(np.float32))
+    assert not np.array_equal(oracle.rows3(C, B, A, x), y)
+
+
 def test_syrk_vs_numpy_and_symmetry():
     n, m = 70, 45
     A = si.matrix(6, n, m)

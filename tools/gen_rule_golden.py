@@ -30,8 +30,9 @@ from oracle import lru  # noqa: E402
 
 # catt.h CATT_K_* (ABI constants)
 K_ATAX_1, K_ATAX_2, K_BICG_1, K_BICG_2, K_MVT_1, K_MVT_2, K_GESUMMV, K_SYRK, K_KMEANS, K_SYR2K, K_KMEANS_T, K_CORR, \
-    K_GEMM = range(13)
-ROWS = (K_ATAX_1, K_BICG_2, K_MVT_1, K_GESUMMV)
+    K_GEMM, K_ROWS3 = range(14)
+ROWS = (K_ATAX_1, K_BICG_2, K_MVT_1, K_GESUMMV, K_ROWS3)
+MATS = {K_GESUMMV: ("A", "B"), K_ROWS3: ("A", "B", "C")}
 
 LOOPS = {  # (set, loop name) -> (problem, variant) for the sweep rows that do not carry their problem
     ("final", "bicg2 q=A p (literal, row per thread)"): (dict(loop=K_BICG_2, m=4096, n=4096), "literal"),
@@ -95,7 +96,7 @@ def shape(L):
         M = p["n"] if loop in (K_MVT_1, K_GESUMMV) else p["m"]
         N = p["n"]
         vec = 4 if var == "vec4" else 1
-        k = lru.RowKernel(M, _short(N), cta, vec=vec, matrices=("A", "B") if loop == K_GESUMMV else ("A",))
+        k = lru.RowKernel(M, _short(N), cta, vec=vec, matrices=MATS.get(loop, ("A",)))
         block, grid = (cta, 1, 1), (math.ceil(M / cta), 1, 1)
     elif loop in (K_SYRK, K_SYR2K, K_GEMM):
         by = cta // 32

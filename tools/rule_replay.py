@@ -7,6 +7,7 @@ rule, and the pick's time is divided by the best swept time.
 
 usage: python tools/rule_replay.py [--rule b200|r24|r23|r18|paper] [--set final|heldout|heldout2|heldout3|heldout4|heldout5|heldout6|heldout7|heldout8|heldout9|partition|all] [-v]
   b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24 + R27)
+  r29   = b200 + the divergent-streams TLP floor (R29, tested on held-out study 10)
   r24   = the same without R27 (the floor fallback gates warps also with several CTAs per SM)
   r23   = R18 + R19 + R23 (re-touch and reuse-trip terms), as held-out study 2 tested it
   r18   = the new terms off (the round-1 rule as fitted)
@@ -83,6 +84,8 @@ def rule_hw(name):
         hw.min_retouch, hw.min_reuse_trip, hw.max_stream_pct, hw.cta_fallback = 16, 128, 0, 0
     elif name == "r24":                        # the library's rule before R27
         hw.cta_fallback = 0
+    elif name == "r29":                        # + the divergent-streams floor (held-out study 10)
+        hw.stream_floor = 1
     elif name == "paper":
         hw = catt.paper_rule(hw)
     return hw
@@ -124,7 +127,7 @@ def replay(rule, sets, verbose):
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("--rule", default="b200", choices=["b200", "r24", "r23", "r18", "paper"])
+    ap.add_argument("--rule", default="b200", choices=["b200", "r29", "r24", "r23", "r18", "paper"])
     ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
