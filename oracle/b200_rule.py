@@ -51,9 +51,10 @@ from typing import Dict, List, Tuple
 from . import lru
 
 # DESIGN.md R18 (floor 8 warps/SM, >= 8 lines per request), R23 (>= 16
-# re-touches), R24 (<= 25 % stream bytes), R27 (CTA fallback on)
+# re-touches), R24 (<= 25 % stream bytes), R27 (CTA fallback on), R29 (the
+# floor divided by the divergent streams when T = 1)
 B200_GUARDS = dict(min_warps_sm=8, divergent_lines=8, min_retouch=16, max_stream_pct=25, cta_fallback=1,
-                   stream_floor=0)
+                   stream_floor=1)
 # shared-memory options (KB) and the L1D each leaves (KB, measured)
 B200_L1D_KB = {0: 218, 8: 218, 16: 218, 32: 218, 64: 186, 100: 150, 132: 118, 164: 86, 196: 53, 228: 21}
 

@@ -506,6 +506,11 @@ extern "C" catt_status catt_hw_b200(catt_hw* out) {
   // R27 (after held-out set 7, restricted to T >= 2): the floor fallback caps
   // whole CTAs when an SM holds several
   out->cta_fallback = 1;
+  // R29 (round 2, held-out study 10, picks pre-registered): with one CTA per
+  // SM, S >= 2 divergent streams lower the TLP floor to ceil(8 / S):
+  // 14/18 launches within 5 % of the best (7/18 without), geomean 1.019x
+  // (1.106x), worst 1.076x (1.373x) (profiles/r2/heldout10/)
+  out->stream_floor = 1;
   // Shared-memory options (KB) and the carveout percentage that selects each
   // (percent of the 228 KB maximum; the driver rounds up to the next option).
   // L1D capacity per option, measured on B200 by the Fig 3-style sweep

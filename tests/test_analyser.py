@@ -365,6 +365,7 @@ def test_r27_cta_fallback():
     (profiles/r1h6, r1h7): (12, 1) measured best where (4, 2) was 1.23-1.40x."""
     b200 = catt.hw_b200()
     assert b200.cta_fallback == 1
+    b200.stream_floor = 0                        # R27 alone (R29 has its own test)
     off = catt.Hw.from_dict(b200.as_dict())
     off.cta_fallback = 0
     cases = [  # problem, CTA threads, carveout, base, R27 pick, R18 pick
@@ -379,3 +380,26 @@ def test_r27_cta_fallback():
             assert (W, T) == base
             assert (t.active_warps or W, t.active_ctas or T) == w
             assert r["flags"] & catt.FIT_GUARDED
+
+
+def test_r29_stream_floor():
+    """R29 (round 2, held-out study 10): with one CTA per SM, a loop with S >= 2
+    memory-divergent reused loads gets the TLP floor ceil(8 / S). GESUMMV
+    (A and B rows: S = 2) at 256 threads / 196 KB: (8, 1) -> (4, 1); the
+    3-matrix rows (S = 3) at 384 threads / 196 KB: (12, 1) -> (4, 1) (8/3
+    rounds up to 3, and 3 does not divide 12: 4 fits); a 1-stream loop is
+    unchanged; with two CTAs per SM the floor stays 8 (R27's regime)."""
+    b200 = catt.hw_b200()
+    assert b200.stream_floor == 1
+    off = catt.Hw.from_dict(b200.as_dict())
+    off.stream_floor = 0
+    lit = lambda cta, carve: catt.Throttle(cta_threads=cta, carveout_kb=carve, variant="literal")
+    cases = [(catt.problem(catt.K_GESUMMV, n=5120), lit(256, 196), (8, 1), (4, 1)),
+             (catt.problem(catt.K_ROWS3, m=6144, n=6144), lit(384, 196), (12, 1), (4, 1)),
+             (catt.problem(catt.K_BICG_2, m=4096, n=4096), lit(1024, 196), (8, 1), (8, 1)),
+             (catt.problem(catt.K_GESUMMV, n=65536), lit(256, 228), (8, 1), (8, 1))]      # T = 2
+    for prob, launch, want_off, want in cases:
+        for hw, w in ((off, want_off), (b200, want)):
+            t, r = catt.plan(prob, launch, hw)
+            W, T = r["base_warps"], r["base_ctas"]
+            assert (t.active_warps or W, t.active_ctas or T) == w, (prob.loop, launch, hw.stream_floor)

@@ -150,17 +150,17 @@ def _golden():
     return json.load(open(GOLDEN))
 
 
-def test_library_rule_equals_trace_oracle_on_the_160_replayed_launches():
-    """Every launch of the stored sweeps (tools/rule_replay.py's 160: the round-1
-    final pass, held-out sets 1-9, the SM partitions), at its full shape: the
+def test_library_rule_equals_trace_oracle_on_the_178_replayed_launches():
+    """Every launch of the stored sweeps (tools/rule_replay.py's 178: the round-1
+    final pass, held-out sets 1-9, the SM partitions, round 2's held-out set
+    10), at its full shape: the
     library's (W, T), L1D and pick equal those tools/gen_rule_golden.py derived
     from oracle/ alone (traces + LRU + Eq 1-4)."""
     g = _golden()
-    assert len(g["launches"]) == 160 and g["guards"] == br.B200_GUARDS
+    assert len(g["launches"]) == 178 and g["guards"] == br.B200_GUARDS
     b200 = catt.hw_b200()
-    assert (b200.min_warps_sm, b200.divergent_lines, b200.min_retouch, b200.max_stream_pct, b200.cta_fallback) == \
-        tuple(br.B200_GUARDS[k] for k in ("min_warps_sm", "divergent_lines", "min_retouch", "max_stream_pct",
-                                          "cta_fallback"))
+    keys = ("min_warps_sm", "divergent_lines", "min_retouch", "max_stream_pct", "cta_fallback", "stream_floor")
+    assert tuple(getattr(b200, k) for k in keys) == tuple(br.B200_GUARDS[k] for k in keys)
     for L in g["launches"]:
         p = dict(L["prob"])
         prob = catt.problem(p.pop("loop"), **p)
@@ -181,7 +181,7 @@ def test_golden_file_is_the_generators_output():
     import gen_rule_golden as gen
     g = _golden()["launches"]
     cheap = [L for L in g if L["prob"]["loop"] in (gen.K_ATAX_1, gen.K_BICG_2, gen.K_MVT_1, gen.K_GESUMMV,
-                                                   gen.K_KMEANS_T)]
+                                                   gen.K_KMEANS_T, gen.K_ROWS3)]
     sample = cheap[::6][:12]
     assert len(sample) >= 8
     for L in sample:
