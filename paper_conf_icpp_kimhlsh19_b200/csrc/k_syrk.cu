@@ -16,6 +16,7 @@
 
 #include "f32x2.cuh"
 #include "internal.h"
+#include "tma.cuh"
 
 namespace catt {
 
@@ -350,6 +351,293 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
   cta_exit(a.t);
 }
 
+// ---------------------------------------------------------------- tiled, two CTAs per SM (round 2)
+// T2: the tile, the per-thread 8 x 8 outputs and the per-element order of
+// tiled_kernel (so the result is bit-identical to it, to LITERAL and to the
+// oracle), rebuilt for two co-resident CTAs per SM (<= 128 registers: 4
+// warps per SM sub-partition instead of 2):
+//  * one elected thread streams each stage's row blocks [128 rows][BK k] of
+//    A (and B) global -> shared with TMA into a 3-stage raw ring (mbarrier
+//    completion; zero fill past n and m), so no thread holds staging
+//    registers or computes addresses (tiled_kernel's register staging held it
+//    at 182 registers, one CTA per SM);
+//  * after computing stage kt, the CTA transposes raw stage kt+1 into the
+//    k-major fragment buffer [k][row] (double-buffered), applying
+//    alpha * a[i][k] with the literal kernel's rounding on the way; one CTA
+//    barrier per stage. The buffer has no padding: row groups of 4 are
+//    XOR-swizzled by k so that the transposing stores and the float4 fragment
+//    reads are both free of bank conflicts;
+//  * a warp owns 4 ty x 8 tx threads (tiled_kernel: 2 x 16), so each
+//    half-warp's float4 fragment read touches 2 row words or 8 column words
+//    (at most 128 B): one shared-memory wavefront each.
+// Needs m % 4 == 0 and 16-byte aligned A (B): the TMA row stride. Otherwise
+// (and with CATT_TILED_T2=0) tiled_kernel runs.
+template <int MODE>
+struct T2Cfg {
+  static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
+  static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
+  static constexpr int NS = 3;                                   // raw TMA stages
+  static constexpr int RAW_FLOATS = NA * 128 * BK;                // one raw stage
+  static constexpr int T_FLOATS = NA * BK * 128;                  // one transposed stage
+  static constexpr int SWZ = 128 / BK;                            // XOR step per 4 k (8 or 16 floats)
+  static constexpr int FBUF = MODE == MODE_SYR2K ? 1 : 2;
+  static constexpr size_t SBYTES = size_t(NS) * RAW_FLOATS * 4 + size_t(2) * T_FLOATS * 4 + 64;
+};
+
+template <int MODE>
+__global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ CUtensorMap mapA,
+                                                       const __grid_constant__ CUtensorMap mapB, TileArgs a) {
+  static_assert(MODE != MODE_GEMM, "T2 covers SYRK and SYR2K");
+  constexpr bool TWO = MODE == MODE_SYR2K;
+  using Cfg = T2Cfg<MODE>;
+  constexpr int BK = Cfg::BK, NA = Cfg::NA, NS = Cfg::NS, TM = 8, SWZ = Cfg::SWZ;
+  extern __shared__ __align__(128) float t2_dyn[];
+  float* raw = t2_dyn;                                                    // [NS][NA][128][BK]
+  float (*T)[NA][BK][128] = reinterpret_cast<float (*)[NA][BK][128]>(t2_dyn + NS * Cfg::RAW_FLOATS);
+  uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::RAW_FLOATS + 2 * Cfg::T_FLOATS);
+
+  // tile of this CTA: a linear index over the computed tiles (tri: the upper
+  // triangle by rows, so no CTA slot is spent on an empty tile)
+  const int nt = int((a.ni + 127) / 128);
+  int by, bx;
+  if (a.tri) {
+    int rem = int(blockIdx.x);
+    by = 0;
+    while (rem >= nt - by) rem -= nt - by, ++by;
+    bx = by + rem;
+  } else {
+    by = int(blockIdx.x) / nt;
+    bx = int(blockIdx.x) % nt;
+  }
+  cta_enter(a.t);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tx = (warp & 1) * 8 + (lane & 7), ty = (warp >> 1) * 4 + (lane >> 3);
+  const int64_t i0 = int64_t(by) * 128, j0 = int64_t(bx) * 128;
+  const int64_t n = a.ni, m = a.m;
+  const int64_t ktiles = (m + BK - 1) / BK;
+
+  // stage array s: 0 = alpha*a[i][k], 1 = a[j][k] (SYR2K: b[j][k]), 2 = alpha*b[i][k], 3 = a[j][k]
+  auto tma = [&](int64_t kt) {  // one elected thread
+    float* dst = raw + int(kt % NS) * Cfg::RAW_FLOATS;
+    uint64_t* bar = &full[kt % NS];
+    bar_expect_tx(bar, uint32_t(Cfg::RAW_FLOATS * 4));
+    const int32_t k0 = int32_t(kt * BK);
+#pragma unroll
+    for (int s = 0; s < NA; ++s) {
+      const CUtensorMap* mp = (s == 0 || s == 3 || (!TWO && s == 1)) ? &mapA : &mapB;
+      const int32_t r0 = int32_t((s == 0 || s == 2) ? i0 : j0);
+      tma_2d(dst + s * 128 * BK, mp, k0, r0, bar);
+    }
+  };
+  if (tid == 0) {
+    for (int s = 0; s < NS; ++s) bar_init(&full[s], 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  if (tid == 0)
+    for (int64_t kt = 0; kt < NS && kt < ktiles; ++kt) tma(kt);
+
+  // raw stage kt -> T[kt & 1]: thread t moves float4 idx = t + 256u, (row = idx / (BK/4), k4 = idx % (BK/4))
+  auto transpose = [&](int64_t kt) {
+    bar_wait(&full[kt % NS], uint32_t((kt / NS) & 1));
+    const float* src = raw + int(kt % NS) * Cfg::RAW_FLOATS;
+    const int buf = int(kt & 1);
+#pragma unroll
+    for (int s = 0; s < NA; ++s) {
+      const bool row_side = s == 0 || s == 2;
+#pragma unroll
+      for (int u = 0; u < 128 * BK / 4 / 256; ++u) {
+        const int idx = tid + 256 * u;
+        const int row = idx / (BK / 4), k4 = idx % (BK / 4);
+        float4 v = *reinterpret_cast<const float4*>(src + s * 128 * BK + row * BK + 4 * k4);
+        if (row_side) {
+          v.x = __fmul_rn(a.alpha, v.x);
+          v.y = __fmul_rn(a.alpha, v.y);
+          v.z = __fmul_rn(a.alpha, v.z);
+          v.w = __fmul_rn(a.alpha, v.w);
+        }
+        const int pr = row ^ (k4 * SWZ);
+        T[buf][s][4 * k4 + 0][pr] = v.x;
+        T[buf][s][4 * k4 + 1][pr] = v.y;
+        T[buf][s][4 * k4 + 2][pr] = v.z;
+        T[buf][s][4 * k4 + 3][pr] = v.w;
+      }
+    }
+  };
+
+  // beta * C into the accumulators (pairs along j), while the first stages land
+  uint64_t cp[TM][TM / 2];
+  const bool cvec = a.cvec;
+#pragma unroll
+  for (int r = 0; r < TM; ++r) {
+    const int64_t gi = i0 + (r / 4) * 64 + ty * 4 + (r % 4);
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int64_t gj = j0 + 64 * h + tx * 4;
+      float c4[4];
+      if (cvec && gi < n && gj + 3 < n) {
+        const float4 v = *reinterpret_cast<const float4*>(a.C + gi * n + gj);
+        c4[0] = v.x, c4[1] = v.y, c4[2] = v.z, c4[3] = v.w;
+      } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) c4[q] = (gi < n && gj + q < n) ? a.C[gi * n + gj + q] : 0.0f;
+      }
+      cp[r][2 * h] = f2_pack(__fmul_rn(c4[0], a.beta), __fmul_rn(c4[1], a.beta));
+      cp[r][2 * h + 1] = f2_pack(__fmul_rn(c4[2], a.beta), __fmul_rn(c4[3], a.beta));
+    }
+  }
+
+  float f[Cfg::FBUF][NA][TM];
+  auto fload = [&](int fb, int buf, int kk) {
+    const int sw = (kk >> 2) * SWZ;
+#pragma unroll
+    for (int s = 0; s < NA; ++s) {
+      const int t = (s == 0 || s == 2) ? ty : tx;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const float4 v = *reinterpret_cast<const float4*>(&T[buf][s][kk][(64 * h + t * 4) ^ sw]);
+        f[fb][s][4 * h] = v.x;
+        f[fb][s][4 * h + 1] = v.y;
+        f[fb][s][4 * h + 2] = v.z;
+        f[fb][s][4 * h + 3] = v.w;
+      }
+    }
+  };
+  auto fma_step = [&](int fb) {
+#pragma unroll
+    for (int r = 0; r < TM; ++r) {
+      const uint64_t ar = f2_pack(f[fb][0][r], f[fb][0][r]);
+#pragma unroll
+      for (int p = 0; p < TM / 2; ++p) {
+        const uint64_t bq = f2_pack(f[fb][1][2 * p], f[fb][1][2 * p + 1]);
+        if constexpr (TWO) {
+          const uint64_t pr = f2_mul(f2_pack(f[fb][2][r], f[fb][2][r]), f2_pack(f[fb][3][2 * p], f[fb][3][2 * p + 1]));
+          cp[r][p] = f2_add(cp[r][p], f2_fma(ar, bq, pr));
+        } else {
+          cp[r][p] = f2_fma(ar, bq, cp[r][p]);
+        }
+      }
+    }
+  };
+
+  if (ktiles > 0) {
+    transpose(0);
+    __syncthreads();
+    if (tid == 0 && NS < ktiles) tma(NS);  // raw slot 0 is free
+  }
+  for (int64_t kt = 0; kt < ktiles; ++kt) {
+    const int buf = int(kt & 1);
+    const int kvalid = int(imin64(BK, m - kt * BK));
+    if (kvalid == BK) {
+      fload(0, buf, 0);
+#pragma unroll
+      for (int kk = 0; kk < BK; ++kk) {
+        if constexpr (Cfg::FBUF == 2) {
+          if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
+          fma_step(kk & 1);
+        } else {
+          if (kk > 0) fload(0, buf, kk);
+          fma_step(0);
+        }
+      }
+    } else {  // ragged last stage: exactly kvalid steps
+      for (int kk = 0; kk < kvalid; ++kk) {
+        fload(0, buf, kk);
+        fma_step(0);
+      }
+    }
+    if (kt + 1 < ktiles) {
+      // T[buf ^ 1] was last read in stage kt - 1, before the previous barrier
+      transpose(kt + 1);
+      __syncthreads();  // stage kt + 1 transposed; raw slot (kt + 1) % NS consumed
+      if (tid == 0 && kt + 1 + NS < ktiles) tma(kt + 1 + NS);
+    }
+  }
+
+#pragma unroll
+  for (int r = 0; r < TM; ++r) {
+    const int64_t gi = i0 + (r / 4) * 64 + ty * 4 + (r % 4);
+    if (gi >= n) continue;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int64_t gj = j0 + 64 * h + tx * 4;
+      const float c0 = f2_lo(cp[r][2 * h]), c1 = f2_hi(cp[r][2 * h]);
+      const float c2 = f2_lo(cp[r][2 * h + 1]), c3 = f2_hi(cp[r][2 * h + 1]);
+      if (cvec && gj + 3 < n) {
+        *reinterpret_cast<float4*>(a.C + gi * n + gj) = make_float4(c0, c1, c2, c3);
+      } else {
+        const float cv[4] = {c0, c1, c2, c3};
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (gj + q < n) a.C[gi * n + gj + q] = cv[q];
+      }
+    }
+  }
+  cta_exit(a.t);
+}
+
+// T2 is the default for the 128 x 128 SYRK / SYR2K tiles; CATT_TILED_T2=0
+// restores tiled_kernel (tools only, for A/B timing).
+static bool tiled_t2() {
+  static const int env = [] {
+    const char* e = getenv("CATT_TILED_T2");
+    return e ? atoi(e) : 1;
+  }();
+  return env != 0;
+}
+
+// rows x cols fp32, row-major, box {BK cols, 128 rows}, zero fill out of range
+static bool t2_map(CUtensorMap* mp, const float* base, int64_t rows, int64_t cols, int bk) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  const cuuint64_t dims[2] = {cuuint64_t(cols), cuuint64_t(rows)};
+  const cuuint64_t strides[1] = {cuuint64_t(cols) * 4};
+  const cuuint32_t box[2] = {cuuint32_t(bk), 128u};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(mp, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <int MODE>
+static bool t2_ok(const TileArgs& a) {
+  auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
+  return tiled_t2() && a.m > 0 && a.m % 4 == 0 && a.m < (int64_t(1) << 31) && a.ni < (int64_t(1) << 31) && al(a.A) &&
+         (MODE != MODE_SYR2K || al(a.B));
+}
+
+template <int MODE>
+static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s) {
+  const void* f = (const void*)tile2_kernel<MODE>;
+  constexpr size_t sb = T2Cfg<MODE>::SBYTES;
+  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sb));
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    return CATT_ECUDA;
+  }
+  size_t dyn = 0;
+  catt_status st = prepare_launch(f, t, 256, sb, false, &a.t, &dyn);
+  if (st != CATT_OK) return st;
+  if (dyn > sb) {  // a Fig 5 pad on top
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn));
+    if (e != cudaSuccess) {
+      record_cuda_error(e);
+      return CATT_ECUDA;
+    }
+  }
+  CUtensorMap ma, mb;
+  if (!t2_map(&ma, a.A, a.ni, a.m, T2Cfg<MODE>::BK) ||
+      !t2_map(&mb, MODE == MODE_SYR2K ? a.B : a.A, a.ni, a.m, T2Cfg<MODE>::BK))
+    return CATT_ECUDA;
+  const int64_t nt = (a.ni + 127) / 128;
+  const int64_t tiles = a.tri ? nt * (nt + 1) / 2 : nt * nt;
+  if (tiles > (int64_t(1) << 31) - 1) return CATT_EINVAL;
+  auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
+  a.cvec = (a.nj % 4 == 0) && al(a.C);
+  tile2_kernel<MODE><<<unsigned(tiles), 256, dyn, s>>>(ma, mb, a);
+  return after_launch();
+}
+
 // Register budget per kernel: MINB = 1 (up to 255 registers, one 256-thread
 // CTA per SM) or 2 (128 registers). CATT_TILED_MINB overrides (tools only).
 static int tiled_minb(bool two) {
@@ -420,6 +708,8 @@ template <int MODE>
 static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t s) {
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
   const bool small = small_tiles<MODE>(a.ni, a.nj);
+  if constexpr (MODE != MODE_GEMM)
+    if (!small && t2_ok<MODE>(a)) return launch_t2<MODE>(a, t, s);
   constexpr int TMs = MODE == MODE_SYR2K ? 8 : 4;  // SYR2K never takes the small tile (static_assert)
   const int64_t tt = (a.ni + 127) / 128;
   const bool lean = !small && MODE == MODE_SYRK && tiled_lean(a.tri ? tt * (tt + 1) / 2 : tt * tt);
@@ -477,19 +767,24 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
   return after_launch();
 }
 
+// the kernel a large (128 x 128 tile) STAGED launch runs, and its dynamic
+// shared memory (catt_kernel_desc / catt_plan describe this kernel)
 const void* syrk_func(int variant) {
-  return variant == CATT_VAR_STAGED ? tiled_func<MODE_SYRK>() : (const void*)syrk_thread_kernel;
+  if (variant != CATT_VAR_STAGED) return (const void*)syrk_thread_kernel;
+  return tiled_t2() ? (const void*)tile2_kernel<MODE_SYRK> : tiled_func<MODE_SYRK>();
 }
 
-// the kernel a large (128 x 128 tile) STAGED SYR2K launch runs, and its
-// dynamic shared memory (catt_kernel_desc / catt_plan describe this kernel)
+int64_t syrk_staged_dyn() { return tiled_t2() ? int64_t(T2Cfg<MODE_SYRK>::SBYTES) : 0; }
+
 const void* syr2k_func(int variant) {
   if (variant != CATT_VAR_STAGED) return (const void*)syr2k_thread_kernel;
+  if (tiled_t2()) return (const void*)tile2_kernel<MODE_SYR2K>;
   if (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) return (const void*)tiled_kernel<MODE_SYR2K, 1, 8, false, true>;
   return tiled_func<MODE_SYR2K>();
 }
 
 int64_t syr2k_staged_dyn() {
+  if (tiled_t2()) return int64_t(T2Cfg<MODE_SYR2K>::SBYTES);
   return (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) ? int64_t(TileCfg<MODE_SYR2K, 8, false, true>::SBYTES) : 0;
 }
 

@@ -21,6 +21,7 @@ int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant);
 const void* syr2k_func(int variant);
 int64_t syr2k_staged_dyn();
+int64_t syrk_staged_dyn();
 const void* kmeans_func(int variant, int nf);
 int64_t kmeans_tma_smem(int nf, int k);
 const void* kmeans_t_func(int variant);
@@ -434,6 +435,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->grid[0] = (N + 127) / 128;
       out->grid[1] = (N + 127) / 128;
       refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);                     // staged through shared memory
+      dyn = syrk_staged_dyn();                                     // the T2 stage ring (dynamic shared memory)
     } else {
       return CATT_EINVAL;
     }
@@ -473,6 +475,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->grid[0] = (Mc + 127) / 128;
       out->grid[1] = (Mc + 127) / 128;
       refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);
+      dyn = syrk_staged_dyn();
       goto done_refs;
     }
     if (var != CATT_VAR_LITERAL) return CATT_EINVAL;

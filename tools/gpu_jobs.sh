@@ -11,6 +11,8 @@
 #   benchall  every workload's bench line
 #   launches  ncu launch list of the default bench (gpu__time_duration)
 #   ncu       ncu --set full of the default bench's dominant kernel
+#   tiles     FP32 tile kernels: bit-exact tests, T2 vs tiled_kernel timing, FFMA2 peak probe
+#   ncutile   ncu --set full of one tile kernel (NCU_KERNEL, TILE_ONLY)
 #   sass      per-kernel SASS opcode summary of libcatt.so
 #   mcprobe   NVLS multicast support with one visible GPU (tools/multicast_probe)
 export PYTHONPATH=.
@@ -58,6 +60,15 @@ for job in "$@"; do
     mcprobe)
       nvidia-smi topo -m > $O/topo.txt 2>&1
       timeout 120 ./tools/multicast_probe > $O/multicast_probe.txt 2>&1; echo "rc=$?" >> $O/multicast_probe.txt ;;
+    tiles)
+      timeout 300 python -m pytest tests/test_gpu.py -m gpu -q -k "syrk or syr2k or corr or gemm" > $O/pytest_tiles.txt 2>&1; echo "rc=$?" >> $O/pytest_tiles.txt
+      for v in 0 1; do
+        CATT_TILED_T2=$v timeout 300 python tools/tile_bench.py > $O/tile_bench_t2_$v.json 2> $O/tile_bench_t2_$v.err
+      done
+      [ -x tools/ffma_probe ] && timeout 120 ./tools/ffma_probe > $O/ffma_probe.txt 2>&1 ;;
+    ncutile)
+      timeout 600 ncu --set full --clock-control none --import-source on -k regex:${NCU_KERNEL:-tile2} -s 1 -c 1 -o $O/ncu_tile -f \
+        python tools/tile_bench.py --reps 1 --only ${TILE_ONLY:-syrk} > $O/ncu_tile.log 2>&1 ;;
     sass)
       python tools/sass_summary.py paper_conf_icpp_kimhlsh19_b200/libcatt.so > $O/sass_summary.txt 2>&1 ;;
     *)
