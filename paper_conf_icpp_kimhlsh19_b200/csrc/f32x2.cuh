@@ -38,4 +38,16 @@ __device__ __forceinline__ uint64_t f2_fma(uint64_t a, uint64_t b, uint64_t c) {
   return d;
 }
 
+// c = fmaf(a, b, c) per half, accumulating in place: the tied operand keeps
+// the accumulator in one register pair across an unrolled loop (with separate
+// in/out operands ptxas rotated accumulators between pairs and paid ~50
+// IMAD.MOV / MOV per stage, on the FMA pipe, to restore them)
+__device__ __forceinline__ void f2_fma_acc(uint64_t& c, uint64_t a, uint64_t b) {
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(c) : "l"(a), "l"(b));
+}
+// c = c + a per half, in place
+__device__ __forceinline__ void f2_add_acc(uint64_t& c, uint64_t a) {
+  asm("add.rn.f32x2 %0, %0, %1;" : "+l"(c) : "l"(a));
+}
+
 }  // namespace catt

@@ -512,9 +512,9 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
         const uint64_t bq = f2_pack(f[fb][1][2 * p], f[fb][1][2 * p + 1]);
         if constexpr (TWO) {
           const uint64_t pr = f2_mul(f2_pack(f[fb][2][r], f[fb][2][r]), f2_pack(f[fb][3][2 * p], f[fb][3][2 * p + 1]));
-          cp[r][p] = f2_add(cp[r][p], f2_fma(ar, bq, pr));
+          f2_add_acc(cp[r][p], f2_fma(ar, bq, pr));
         } else {
-          cp[r][p] = f2_fma(ar, bq, cp[r][p]);
+          f2_fma_acc(cp[r][p], ar, bq);
         }
       }
     }
@@ -525,24 +525,20 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
     __syncthreads();
     if (tid == 0 && NS < ktiles) tma(NS);  // raw slot 0 is free
   }
-  for (int64_t kt = 0; kt < ktiles; ++kt) {
+  // full stages in a loop of their own (one register assignment for the
+  // accumulators: a ragged branch inside the loop made ptxas insert ~50
+  // accumulator moves per stage), then the ragged last stage
+  const int64_t kfull = m / BK;
+  for (int64_t kt = 0; kt < kfull; ++kt) {
     const int buf = int(kt & 1);
-    const int kvalid = int(imin64(BK, m - kt * BK));
-    if (kvalid == BK) {
-      fload(0, buf, 0);
+    fload(0, buf, 0);
 #pragma unroll
-      for (int kk = 0; kk < BK; ++kk) {
-        if constexpr (Cfg::FBUF == 2) {
-          if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
-          fma_step(kk & 1);
-        } else {
-          if (kk > 0) fload(0, buf, kk);
-          fma_step(0);
-        }
-      }
-    } else {  // ragged last stage: exactly kvalid steps
-      for (int kk = 0; kk < kvalid; ++kk) {
-        fload(0, buf, kk);
+    for (int kk = 0; kk < BK; ++kk) {
+      if constexpr (Cfg::FBUF == 2) {
+        if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
+        fma_step(kk & 1);
+      } else {
+        if (kk > 0) fload(0, buf, kk);
         fma_step(0);
       }
     }
@@ -551,6 +547,14 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
       transpose(kt + 1);
       __syncthreads();  // stage kt + 1 transposed; raw slot (kt + 1) % NS consumed
       if (tid == 0 && kt + 1 + NS < ktiles) tma(kt + 1 + NS);
+    }
+  }
+  if (kfull < ktiles) {  // exactly m % BK steps
+    const int buf = int(kfull & 1);
+    const int kvalid = int(m - kfull * BK);
+    for (int kk = 0; kk < kvalid; ++kk) {
+      fload(0, buf, kk);
+      fma_step(0);
     }
   }
 
