@@ -12,6 +12,7 @@
 // break the 1e-5 bar, BASELINE north_star). SYR2K (below) shares the tiled
 // kernel; its literal kernel is the paper's 2-D CS loop.
 #include <cstdlib>
+#include <mutex>
 #include <cstdint>
 
 #include "f32x2.cuh"
@@ -355,46 +356,45 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 // T2: the tile, the per-thread 8 x 8 outputs and the per-element order of
 // tiled_kernel (so the result is bit-identical to it, to LITERAL and to the
 // oracle), rebuilt for two co-resident CTAs per SM (<= 128 registers: 4
-// warps per SM sub-partition instead of 2):
-//  * one elected thread streams each stage's row blocks [128 rows][BK k] of
-//    A (and B) global -> shared with TMA into a 3-stage raw ring (mbarrier
-//    completion; zero fill past n and m), so no thread holds staging
-//    registers or computes addresses (tiled_kernel's register staging held it
-//    at 182 registers, one CTA per SM);
-//  * after computing stage kt, the CTA transposes raw stage kt+1 into the
-//    k-major fragment buffer [k][row] (double-buffered), applying
-//    alpha * a[i][k] with the literal kernel's rounding on the way; one CTA
-//    barrier per stage. The buffer has no padding: row groups of 4 are
-//    XOR-swizzled by k so that the transposing stores and the float4 fragment
-//    reads are both free of bank conflicts;
-//  * a warp owns 4 ty x 8 tx threads (tiled_kernel: 2 x 16), so each
-//    half-warp's float4 fragment read touches 2 row words or 8 column words
-//    (at most 128 B): one shared-memory wavefront each.
-// Needs m % 4 == 0 and 16-byte aligned A (B): the TMA row stride. Otherwise
-// (and with CATT_TILED_T2=0) tiled_kernel runs.
+// warps per SM sub-partition instead of 2) and for a barrier-free main loop:
+//  * a prep kernel writes the operands k-major once per call, A^T and
+//    (alpha A)^T (SYR2K: also B^T and (alpha B)^T), into a stream-ordered
+//    workspace; alpha * a[i][k] is the literal kernel's rounding, so nothing
+//    changes numerically. This replaces tiled_kernel's per-stage transpose
+//    through registers (what held it at 182 registers, one CTA per SM);
+//  * one elected thread streams [BK k][128 rows] boxes of the k-major
+//    operands global -> shared with TMA into an NS-stage ring (zero fill past
+//    n and m); every warp waits on the stage's full mbarrier, computes its
+//    BK steps and arrives on the stage's empty mbarrier, and the elected
+//    thread refills a stage once all 8 warps released it: no CTA barrier in
+//    the k loop;
+//  * a warp owns 4 ty x 8 tx threads; a float4 fragment read costs 2
+//    shared-memory wavefronts for the row operand (<= 2 distinct words per
+//    quarter-warp: merged) and 4 for the column operand (tools/lds_probe.cu).
 template <int MODE>
 struct T2Cfg {
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
-  static constexpr int NS = 3;                                   // raw TMA stages
-  static constexpr int RAW_FLOATS = NA * 128 * BK;                // one raw stage
-  static constexpr int T_FLOATS = NA * BK * 128;                  // one transposed stage
-  static constexpr int SWZ = 128 / BK;                            // XOR step per 4 k (8 or 16 floats)
+  static constexpr int NS = 4;                                   // ring stages
+  static constexpr int STAGE_FLOATS = NA * BK * 128;
   static constexpr int FBUF = MODE == MODE_SYR2K ? 1 : 2;
-  static constexpr size_t SBYTES = size_t(NS) * RAW_FLOATS * 4 + size_t(2) * T_FLOATS * 4 + 64;
+  static constexpr size_t SBYTES = size_t(NS) * STAGE_FLOATS * 4 + 2 * NS * 8;
+};
+
+struct T2Maps {
+  CUtensorMap m[4];  // per stage array: the k-major operand it is loaded from
 };
 
 template <int MODE>
-__global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ CUtensorMap mapA,
-                                                       const __grid_constant__ CUtensorMap mapB, TileArgs a) {
+__global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T2Maps maps, TileArgs a) {
   static_assert(MODE != MODE_GEMM, "T2 covers SYRK and SYR2K");
   constexpr bool TWO = MODE == MODE_SYR2K;
   using Cfg = T2Cfg<MODE>;
-  constexpr int BK = Cfg::BK, NA = Cfg::NA, NS = Cfg::NS, TM = 8, SWZ = Cfg::SWZ;
+  constexpr int BK = Cfg::BK, NA = Cfg::NA, NS = Cfg::NS, TM = 8;
   extern __shared__ __align__(128) float t2_dyn[];
-  float* raw = t2_dyn;                                                    // [NS][NA][128][BK]
-  float (*T)[NA][BK][128] = reinterpret_cast<float (*)[NA][BK][128]>(t2_dyn + NS * Cfg::RAW_FLOATS);
-  uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::RAW_FLOATS + 2 * Cfg::T_FLOATS);
+  float (*T)[NA][BK][128] = reinterpret_cast<float (*)[NA][BK][128]>(t2_dyn);  // [NS] stages
+  uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
+  uint64_t* empty = full + NS;
 
   // tile of this CTA: a linear index over the computed tiles (tri: the upper
   // triangle by rows, so no CTA slot is spent on an empty tile)
@@ -417,53 +417,24 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
   const int64_t ktiles = (m + BK - 1) / BK;
 
   // stage array s: 0 = alpha*a[i][k], 1 = a[j][k] (SYR2K: b[j][k]), 2 = alpha*b[i][k], 3 = a[j][k]
-  auto tma = [&](int64_t kt) {  // one elected thread
-    float* dst = raw + int(kt % NS) * Cfg::RAW_FLOATS;
-    uint64_t* bar = &full[kt % NS];
-    bar_expect_tx(bar, uint32_t(Cfg::RAW_FLOATS * 4));
+  auto tma = [&](int64_t kt) {  // the elected thread
+    const int slot = int(kt % NS);
+    bar_expect_tx(&full[slot], uint32_t(Cfg::STAGE_FLOATS * 4));
     const int32_t k0 = int32_t(kt * BK);
 #pragma unroll
-    for (int s = 0; s < NA; ++s) {
-      const CUtensorMap* mp = (s == 0 || s == 3 || (!TWO && s == 1)) ? &mapA : &mapB;
-      const int32_t r0 = int32_t((s == 0 || s == 2) ? i0 : j0);
-      tma_2d(dst + s * 128 * BK, mp, k0, r0, bar);
-    }
+    for (int s = 0; s < NA; ++s)
+      tma_2d(&T[slot][s][0][0], &maps.m[s], int32_t((s == 0 || s == 2) ? i0 : j0), k0, &full[slot]);
   };
   if (tid == 0) {
-    for (int s = 0; s < NS; ++s) bar_init(&full[s], 1);
+    for (int s = 0; s < NS; ++s) {
+      bar_init(&full[s], 1);
+      bar_init(&empty[s], 8);
+    }
     fence_barrier_init();
   }
   __syncthreads();
   if (tid == 0)
     for (int64_t kt = 0; kt < NS && kt < ktiles; ++kt) tma(kt);
-
-  // raw stage kt -> T[kt & 1]: thread t moves float4 idx = t + 256u, (row = idx / (BK/4), k4 = idx % (BK/4))
-  auto transpose = [&](int64_t kt) {
-    bar_wait(&full[kt % NS], uint32_t((kt / NS) & 1));
-    const float* src = raw + int(kt % NS) * Cfg::RAW_FLOATS;
-    const int buf = int(kt & 1);
-#pragma unroll
-    for (int s = 0; s < NA; ++s) {
-      const bool row_side = s == 0 || s == 2;
-#pragma unroll
-      for (int u = 0; u < 128 * BK / 4 / 256; ++u) {
-        const int idx = tid + 256 * u;
-        const int row = idx / (BK / 4), k4 = idx % (BK / 4);
-        float4 v = *reinterpret_cast<const float4*>(src + s * 128 * BK + row * BK + 4 * k4);
-        if (row_side) {
-          v.x = __fmul_rn(a.alpha, v.x);
-          v.y = __fmul_rn(a.alpha, v.y);
-          v.z = __fmul_rn(a.alpha, v.z);
-          v.w = __fmul_rn(a.alpha, v.w);
-        }
-        const int pr = row ^ (k4 * SWZ);
-        T[buf][s][4 * k4 + 0][pr] = v.x;
-        T[buf][s][4 * k4 + 1][pr] = v.y;
-        T[buf][s][4 * k4 + 2][pr] = v.z;
-        T[buf][s][4 * k4 + 3][pr] = v.w;
-      }
-    }
-  };
 
   // beta * C into the accumulators (pairs along j), while the first stages land
   uint64_t cp[TM][TM / 2];
@@ -488,14 +459,13 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
   }
 
   float f[Cfg::FBUF][NA][TM];
-  auto fload = [&](int fb, int buf, int kk) {
-    const int sw = (kk >> 2) * SWZ;
+  auto fload = [&](int fb, int slot, int kk) {
 #pragma unroll
     for (int s = 0; s < NA; ++s) {
       const int t = (s == 0 || s == 2) ? ty : tx;
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const float4 v = *reinterpret_cast<const float4*>(&T[buf][s][kk][(64 * h + t * 4) ^ sw]);
+        const float4 v = *reinterpret_cast<const float4*>(&T[slot][s][kk][64 * h + t * 4]);
         f[fb][s][4 * h] = v.x;
         f[fb][s][4 * h + 1] = v.y;
         f[fb][s][4 * h + 2] = v.z;
@@ -519,41 +489,42 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
       }
     }
   };
+  // the warp is done reading stage kt's slot; the elected thread refills the
+  // slot of the stage before (released by every warp by now, in practice)
+  auto release = [&](int64_t kt) {
+    __syncwarp();
+    if (lane == 0) bar_arrive(&empty[kt % NS]);
+    if (tid == 0 && kt >= 1 && kt - 1 + NS < ktiles) {
+      bar_wait(&empty[(kt - 1) % NS], uint32_t(((kt - 1) / NS) & 1));
+      tma(kt - 1 + NS);
+    }
+  };
 
-  if (ktiles > 0) {
-    transpose(0);
-    __syncthreads();
-    if (tid == 0 && NS < ktiles) tma(NS);  // raw slot 0 is free
-  }
   // full stages in a loop of their own (one register assignment for the
-  // accumulators: a ragged branch inside the loop made ptxas insert ~50
-  // accumulator moves per stage), then the ragged last stage
+  // accumulators), then the ragged last stage
   const int64_t kfull = m / BK;
   for (int64_t kt = 0; kt < kfull; ++kt) {
-    const int buf = int(kt & 1);
-    fload(0, buf, 0);
+    const int slot = int(kt % NS);
+    bar_wait(&full[slot], uint32_t((kt / NS) & 1));
+    fload(0, slot, 0);
 #pragma unroll
     for (int kk = 0; kk < BK; ++kk) {
       if constexpr (Cfg::FBUF == 2) {
-        if (kk + 1 < BK) fload((kk + 1) & 1, buf, kk + 1);
+        if (kk + 1 < BK) fload((kk + 1) & 1, slot, kk + 1);
         fma_step(kk & 1);
       } else {
-        if (kk > 0) fload(0, buf, kk);
+        if (kk > 0) fload(0, slot, kk);
         fma_step(0);
       }
     }
-    if (kt + 1 < ktiles) {
-      // T[buf ^ 1] was last read in stage kt - 1, before the previous barrier
-      transpose(kt + 1);
-      __syncthreads();  // stage kt + 1 transposed; raw slot (kt + 1) % NS consumed
-      if (tid == 0 && kt + 1 + NS < ktiles) tma(kt + 1 + NS);
-    }
+    release(kt);
   }
   if (kfull < ktiles) {  // exactly m % BK steps
-    const int buf = int(kfull & 1);
+    const int slot = int(kfull % NS);
+    bar_wait(&full[slot], uint32_t((kfull / NS) & 1));
     const int kvalid = int(m - kfull * BK);
     for (int kk = 0; kk < kvalid; ++kk) {
-      fload(0, buf, kk);
+      fload(0, slot, kk);
       fma_step(0);
     }
   }
@@ -580,6 +551,30 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ C
   cta_exit(a.t);
 }
 
+// k-major copies of X (n x m, row-major): Xt[k][i] = X[i][k] and, when aXt is
+// given, aXt[k][i] = alpha * X[i][k] (the literal kernel's rounding). Rows of
+// the copies have pitch ld (a multiple of 4 floats: the TMA stride).
+__global__ void __launch_bounds__(256) t2_prep_kernel(const float* __restrict__ X, float* __restrict__ Xt,
+                                                      float* __restrict__ aXt, int64_t n, int64_t m, int64_t ld,
+                                                      float alpha) {
+  __shared__ float tile[32][33];
+  const int64_t i0 = int64_t(blockIdx.x) * 32, k0 = int64_t(blockIdx.y) * 32;
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  for (int r = ty; r < 32; r += 8) {
+    const int64_t i = i0 + r, k = k0 + tx;
+    tile[r][tx] = (i < n && k < m) ? X[i * m + k] : 0.0f;
+  }
+  __syncthreads();
+  for (int r = ty; r < 32; r += 8) {
+    const int64_t k = k0 + r, i = i0 + tx;
+    if (k < m && i < n) {
+      const float v = tile[tx][r];
+      Xt[k * ld + i] = v;
+      if (aXt) aXt[k * ld + i] = __fmul_rn(alpha, v);
+    }
+  }
+}
+
 // T2 is the default for the 128 x 128 SYRK / SYR2K tiles; CATT_TILED_T2=0
 // restores tiled_kernel (tools only, for A/B timing).
 static bool tiled_t2() {
@@ -590,24 +585,22 @@ static bool tiled_t2() {
   return env != 0;
 }
 
-// rows x cols fp32, row-major, box {BK cols, 128 rows}, zero fill out of range
-static bool t2_map(CUtensorMap* mp, const float* base, int64_t rows, int64_t cols, int bk) {
+// a k-major operand: m rows (k) x n columns, pitch ld; box {128 columns, BK rows}
+static bool t2_map(CUtensorMap* mp, const float* base, int64_t n, int64_t m, int64_t ld, int bk) {
   auto fn = encode_fn();
   if (!fn) return false;
-  const cuuint64_t dims[2] = {cuuint64_t(cols), cuuint64_t(rows)};
-  const cuuint64_t strides[1] = {cuuint64_t(cols) * 4};
-  const cuuint32_t box[2] = {cuuint32_t(bk), 128u};
+  const cuuint64_t dims[2] = {cuuint64_t(n), cuuint64_t(m)};
+  const cuuint64_t strides[1] = {cuuint64_t(ld) * 4};
+  const cuuint32_t box[2] = {128u, cuuint32_t(bk)};
   const cuuint32_t estr[2] = {1, 1};
   return fn(mp, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
-            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 template <int MODE>
 static bool t2_ok(const TileArgs& a) {
-  auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
-  return tiled_t2() && a.m > 0 && a.m % 4 == 0 && a.m < (int64_t(1) << 31) && a.ni < (int64_t(1) << 31) && al(a.A) &&
-         (MODE != MODE_SYR2K || al(a.B));
+  return tiled_t2() && a.m > 0 && a.m < (int64_t(1) << 31) && a.ni < (int64_t(1) << 31);
 }
 
 template <int MODE>
@@ -629,17 +622,59 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
       return CATT_ECUDA;
     }
   }
-  CUtensorMap ma, mb;
-  if (!t2_map(&ma, a.A, a.ni, a.m, T2Cfg<MODE>::BK) ||
-      !t2_map(&mb, MODE == MODE_SYR2K ? a.B : a.A, a.ni, a.m, T2Cfg<MODE>::BK))
+  const int64_t n = a.ni, m = a.m, ld = (n + 3) / 4 * 4;
+  const bool scale = a.alpha != 1.0f;  // alpha * x == x exactly: (alpha A)^T is A^T
+  const int nsrc = MODE == MODE_SYR2K ? 2 : 1;
+  const int64_t per = m * ld;          // floats per k-major copy
+  const size_t bytes = size_t(per) * 4 * size_t(nsrc * (scale ? 2 : 1));
+  // the workspace: stream-ordered, so concurrent launches on other streams get their own
+  static std::once_flag pool_once;
+  std::call_once(pool_once, [] {
+    int d = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&d) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, d) == cudaSuccess) {
+      uint64_t keep = UINT64_MAX;  // keep freed blocks for the next call
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+  });
+  float* ws = nullptr;
+  e = cudaMallocAsync(reinterpret_cast<void**>(&ws), bytes, s);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
     return CATT_ECUDA;
-  const int64_t nt = (a.ni + 127) / 128;
+  }
+  // copies: A^T, [(alpha A)^T], SYR2K: B^T, [(alpha B)^T]
+  float* At = ws;
+  float* aAt = scale ? ws + per : At;
+  float* Bt = MODE == MODE_SYR2K ? ws + per * (scale ? 2 : 1) : nullptr;
+  float* aBt = MODE == MODE_SYR2K ? (scale ? Bt + per : Bt) : nullptr;
+  const dim3 pg(unsigned((n + 31) / 32), unsigned((m + 31) / 32));
+  if (pg.y > 65535) {
+    cudaFreeAsync(ws, s);
+    return CATT_EINVAL;
+  }
+  t2_prep_kernel<<<pg, 256, 0, s>>>(a.A, At, scale ? aAt : nullptr, n, m, ld, a.alpha);
+  if (MODE == MODE_SYR2K) t2_prep_kernel<<<pg, 256, 0, s>>>(a.B, Bt, scale ? aBt : nullptr, n, m, ld, a.alpha);
+  T2Maps maps{};
+  const float* src[4] = {aAt, MODE == MODE_SYR2K ? Bt : At, aBt, At};
+  bool ok = true;
+  for (int q = 0; q < T2Cfg<MODE>::NA; ++q) ok = ok && t2_map(&maps.m[q], src[q], n, m, ld, T2Cfg<MODE>::BK);
+  if (!ok) {
+    cudaFreeAsync(ws, s);
+    return CATT_ECUDA;
+  }
+  const int64_t nt = (n + 127) / 128;
   const int64_t tiles = a.tri ? nt * (nt + 1) / 2 : nt * nt;
-  if (tiles > (int64_t(1) << 31) - 1) return CATT_EINVAL;
+  if (tiles > (int64_t(1) << 31) - 1) {
+    cudaFreeAsync(ws, s);
+    return CATT_EINVAL;
+  }
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
   a.cvec = (a.nj % 4 == 0) && al(a.C);
-  tile2_kernel<MODE><<<unsigned(tiles), 256, dyn, s>>>(ma, mb, a);
-  return after_launch();
+  tile2_kernel<MODE><<<unsigned(tiles), 256, dyn, s>>>(maps, a);
+  const catt_status ls = after_launch();
+  cudaFreeAsync(ws, s);
+  return ls;
 }
 
 // Register budget per kernel: MINB = 1 (up to 255 registers, one 256-thread
