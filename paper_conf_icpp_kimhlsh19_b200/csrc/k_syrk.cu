@@ -11,6 +11,7 @@
 // bit-identical to LITERAL. FP32 CUDA-core bound (no tensor cores: TF32 would
 // break the 1e-5 bar, BASELINE north_star). SYR2K (below) shares the tiled
 // kernel; its literal kernel is the paper's 2-D CS loop.
+#include <algorithm>
 #include <cstdlib>
 #include <mutex>
 #include <cstdint>
@@ -371,80 +372,84 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 //  * a warp owns 4 ty x 8 tx threads; a float4 fragment read costs 2
 //    shared-memory wavefronts for the row operand (<= 2 distinct words per
 //    quarter-warp: merged) and 4 for the column operand (tools/lds_probe.cu).
+// Tiles are 64 x 256 or 48 x 256 (8 x 8 or 6 x 8 outputs per thread, warp w
+// = row group w, lane = column group): the row blocks mix both heights so
+// that the tile count fills the 2 x #SM CTA slots in one wave (2048 on 148
+// SMs: 17 blocks of 64 and 20 of 48 rows x 8 strips = 296 tiles; 128 x 128
+// tiles gave 256 = 1.73 per SM, i.e. SMs with one tile idle half the time).
+// The row operand is then a broadcast in every warp (2 wavefronts per float4
+// read), the column operand 32 distinct words (4).
 template <int MODE>
 struct T2Cfg {
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
+  static constexpr int NP = NA / 2;                               // row-side (and column-side) arrays
   static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
   static constexpr int NS = 4;                                   // ring stages
-  static constexpr int STAGE_FLOATS = NA * BK * 128;
+  static constexpr int RB = 64, CB = 256;                        // row box, column strip
+  static constexpr int ROW_FLOATS = BK * RB, COL_FLOATS = BK * CB;
+  static constexpr int STAGE_FLOATS = NP * (ROW_FLOATS + COL_FLOATS);
   static constexpr int FBUF = MODE == MODE_SYR2K ? 1 : 2;
   static constexpr size_t SBYTES = size_t(NS) * STAGE_FLOATS * 4 + 2 * NS * 8;
 };
 
 struct T2Maps {
-  CUtensorMap m[4];  // per stage array: the k-major operand it is loaded from
+  CUtensorMap m[4];  // per stage array (row-side first): the k-major operand it is loaded from
 };
 
-template <int MODE>
-__global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T2Maps maps, TileArgs a) {
-  static_assert(MODE != MODE_GEMM, "T2 covers SYRK and SYR2K");
+struct T2Geo {
+  int cs;            // column strips
+  int x;             // row blocks of 64 rows (the first x); the rest have 48
+  int rbs;           // row blocks
+  int tri;           // compute only tiles reaching the diagonal or above (all blocks 64 rows)
+};
+
+__device__ __forceinline__ int64_t t2_row0(const T2Geo& g, int rb) {
+  return rb < g.x ? int64_t(64) * rb : int64_t(64) * g.x + int64_t(48) * (rb - g.x);
+}
+
+// One tile: RH rows per thread (8: a 64-row block, 6: a 48-row block).
+template <int MODE, int RH>
+__device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* empty, const T2Maps& maps,
+                                        const TileArgs& a, int64_t i0, int64_t j0) {
   constexpr bool TWO = MODE == MODE_SYR2K;
   using Cfg = T2Cfg<MODE>;
-  constexpr int BK = Cfg::BK, NA = Cfg::NA, NS = Cfg::NS, TM = 8;
-  extern __shared__ __align__(128) float t2_dyn[];
-  float (*T)[NA][BK][128] = reinterpret_cast<float (*)[NA][BK][128]>(t2_dyn);  // [NS] stages
-  uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
-  uint64_t* empty = full + NS;
-
-  // tile of this CTA: a linear index over the computed tiles (tri: the upper
-  // triangle by rows, so no CTA slot is spent on an empty tile)
-  const int nt = int((a.ni + 127) / 128);
-  int by, bx;
-  if (a.tri) {
-    int rem = int(blockIdx.x);
-    by = 0;
-    while (rem >= nt - by) rem -= nt - by, ++by;
-    bx = by + rem;
-  } else {
-    by = int(blockIdx.x) / nt;
-    bx = int(blockIdx.x) % nt;
-  }
-  cta_enter(a.t);
+  constexpr int BK = Cfg::BK, NP = Cfg::NP, NS = Cfg::NS, RBX = Cfg::RB, CBX = Cfg::CB;
+  // stage layout: NP row arrays [BK][64], then NP column arrays [BK][256]
+  auto rowp = [&](int slot, int s, int kk) { return sm + slot * Cfg::STAGE_FLOATS + s * Cfg::ROW_FLOATS + kk * RBX; };
+  auto colp = [&](int slot, int s, int kk) {
+    return sm + slot * Cfg::STAGE_FLOATS + NP * Cfg::ROW_FLOATS + s * Cfg::COL_FLOATS + kk * CBX;
+  };
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int tx = (warp & 1) * 8 + (lane & 7), ty = (warp >> 1) * 4 + (lane >> 3);
-  const int64_t i0 = int64_t(by) * 128, j0 = int64_t(bx) * 128;
+  const int ty = warp, tx = lane;
   const int64_t n = a.ni, m = a.m;
   const int64_t ktiles = (m + BK - 1) / BK;
+  // rows of this thread: r < 4: ty*4 + r; r >= 4: 32 + ty*(RH - 4) + r - 4
+  auto row_of = [&](int r) { return r < 4 ? ty * 4 + r : 32 + ty * (RH - 4) + (r - 4); };
 
-  // stage array s: 0 = alpha*a[i][k], 1 = a[j][k] (SYR2K: b[j][k]), 2 = alpha*b[i][k], 3 = a[j][k]
+  // row-side stage arrays: alpha*a[i][k] (SYR2K: then alpha*b[i][k]); column-side: a[j][k]
+  // (SYR2K: b[j][k], then a[j][k]); maps in the same order
   auto tma = [&](int64_t kt) {  // the elected thread
     const int slot = int(kt % NS);
     bar_expect_tx(&full[slot], uint32_t(Cfg::STAGE_FLOATS * 4));
     const int32_t k0 = int32_t(kt * BK);
 #pragma unroll
-    for (int s = 0; s < NA; ++s)
-      tma_2d(&T[slot][s][0][0], &maps.m[s], int32_t((s == 0 || s == 2) ? i0 : j0), k0, &full[slot]);
-  };
-  if (tid == 0) {
-    for (int s = 0; s < NS; ++s) {
-      bar_init(&full[s], 1);
-      bar_init(&empty[s], 8);
+    for (int s = 0; s < NP; ++s) {
+      tma_2d(rowp(slot, s, 0), &maps.m[s], int32_t(i0), k0, &full[slot]);
+      tma_2d(colp(slot, s, 0), &maps.m[NP + s], int32_t(j0), k0, &full[slot]);
     }
-    fence_barrier_init();
-  }
-  __syncthreads();
+  };
   if (tid == 0)
     for (int64_t kt = 0; kt < NS && kt < ktiles; ++kt) tma(kt);
 
   // beta * C into the accumulators (pairs along j), while the first stages land
-  uint64_t cp[TM][TM / 2];
+  uint64_t cp[RH][4];
   const bool cvec = a.cvec;
 #pragma unroll
-  for (int r = 0; r < TM; ++r) {
-    const int64_t gi = i0 + (r / 4) * 64 + ty * 4 + (r % 4);
+  for (int r = 0; r < RH; ++r) {
+    const int64_t gi = i0 + row_of(r);
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-      const int64_t gj = j0 + 64 * h + tx * 4;
+      const int64_t gj = j0 + 128 * h + tx * 4;
       float c4[4];
       if (cvec && gi < n && gj + 3 < n) {
         const float4 v = *reinterpret_cast<const float4*>(a.C + gi * n + gj);
@@ -458,30 +463,37 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
     }
   }
 
-  float f[Cfg::FBUF][NA][TM];
+  float fr[Cfg::FBUF][NP][RH], fc[Cfg::FBUF][NP][8];
   auto fload = [&](int fb, int slot, int kk) {
 #pragma unroll
-    for (int s = 0; s < NA; ++s) {
-      const int t = (s == 0 || s == 2) ? ty : tx;
+    for (int s = 0; s < NP; ++s) {
+      const float* rp = rowp(slot, s, kk);
+      const float4 v0 = *reinterpret_cast<const float4*>(rp + ty * 4);
+      fr[fb][s][0] = v0.x, fr[fb][s][1] = v0.y, fr[fb][s][2] = v0.z, fr[fb][s][3] = v0.w;
+      if constexpr (RH == 8) {
+        const float4 v1 = *reinterpret_cast<const float4*>(rp + 32 + ty * 4);
+        fr[fb][s][4] = v1.x, fr[fb][s][5] = v1.y, fr[fb][s][6] = v1.z, fr[fb][s][7] = v1.w;
+      } else {
+        const float2 v1 = *reinterpret_cast<const float2*>(rp + 32 + ty * 2);
+        fr[fb][s][4] = v1.x, fr[fb][s][5] = v1.y;
+      }
+      const float* cq = colp(slot, s, kk);
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const float4 v = *reinterpret_cast<const float4*>(&T[slot][s][kk][64 * h + t * 4]);
-        f[fb][s][4 * h] = v.x;
-        f[fb][s][4 * h + 1] = v.y;
-        f[fb][s][4 * h + 2] = v.z;
-        f[fb][s][4 * h + 3] = v.w;
+        const float4 v = *reinterpret_cast<const float4*>(cq + 128 * h + tx * 4);
+        fc[fb][s][4 * h] = v.x, fc[fb][s][4 * h + 1] = v.y, fc[fb][s][4 * h + 2] = v.z, fc[fb][s][4 * h + 3] = v.w;
       }
     }
   };
   auto fma_step = [&](int fb) {
 #pragma unroll
-    for (int r = 0; r < TM; ++r) {
-      const uint64_t ar = f2_pack(f[fb][0][r], f[fb][0][r]);
+    for (int r = 0; r < RH; ++r) {
+      const uint64_t ar = f2_pack(fr[fb][0][r], fr[fb][0][r]);
 #pragma unroll
-      for (int p = 0; p < TM / 2; ++p) {
-        const uint64_t bq = f2_pack(f[fb][1][2 * p], f[fb][1][2 * p + 1]);
-        if constexpr (TWO) {
-          const uint64_t pr = f2_mul(f2_pack(f[fb][2][r], f[fb][2][r]), f2_pack(f[fb][3][2 * p], f[fb][3][2 * p + 1]));
+      for (int p = 0; p < 4; ++p) {
+        const uint64_t bq = f2_pack(fc[fb][0][2 * p], fc[fb][0][2 * p + 1]);
+        if constexpr (TWO) {  // fmaf(alpha*a_ik, b_jk, (alpha*b_ik) * a_jk), then c + s (R20)
+          const uint64_t pr = f2_mul(f2_pack(fr[fb][1][r], fr[fb][1][r]), f2_pack(fc[fb][1][2 * p], fc[fb][1][2 * p + 1]));
           f2_add_acc(cp[r][p], f2_fma(ar, bq, pr));
         } else {
           f2_fma_acc(cp[r][p], ar, bq);
@@ -530,12 +542,12 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
   }
 
 #pragma unroll
-  for (int r = 0; r < TM; ++r) {
-    const int64_t gi = i0 + (r / 4) * 64 + ty * 4 + (r % 4);
+  for (int r = 0; r < RH; ++r) {
+    const int64_t gi = i0 + row_of(r);
     if (gi >= n) continue;
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-      const int64_t gj = j0 + 64 * h + tx * 4;
+      const int64_t gj = j0 + 128 * h + tx * 4;
       const float c0 = f2_lo(cp[r][2 * h]), c1 = f2_hi(cp[r][2 * h]);
       const float c2 = f2_lo(cp[r][2 * h + 1]), c3 = f2_hi(cp[r][2 * h + 1]);
       if (cvec && gj + 3 < n) {
@@ -547,6 +559,53 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
           if (gj + q < n) a.C[gi * n + gj + q] = cv[q];
       }
     }
+  }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T2Maps maps, TileArgs a, T2Geo g) {
+  static_assert(MODE != MODE_GEMM, "T2 covers SYRK and SYR2K");
+  using Cfg = T2Cfg<MODE>;
+  constexpr int NS = Cfg::NS;
+  extern __shared__ __align__(128) float t2_dyn[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
+  uint64_t* empty = full + NS;
+  // the tile: 64-row blocks first (spread one per SM by the block scheduler),
+  // then 48-row blocks; tri: the tiles that reach the diagonal, by row block
+  int rb, cs;
+  if (g.tri) {
+    int rem = int(blockIdx.x);
+    rb = 0;
+    while (true) {
+      const int lo = int((int64_t(64) * rb) / 256);  // first strip with an element j >= i
+      if (rem < g.cs - lo) {
+        cs = lo + rem;
+        break;
+      }
+      rem -= g.cs - lo;
+      ++rb;
+    }
+  } else {
+    rb = int(blockIdx.x) / g.cs;
+    cs = int(blockIdx.x) % g.cs;
+  }
+  cta_enter(a.t);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < NS; ++s) {
+      bar_init(&full[s], 1);
+      bar_init(&empty[s], 8);
+    }
+    fence_barrier_init();
+  }
+  __syncthreads();
+  const int64_t i0 = t2_row0(g, rb), j0 = int64_t(cs) * Cfg::CB;
+  if constexpr (MODE == MODE_SYR2K) {  // 64-row blocks only: two tile bodies spill at 128 registers
+    t2_tile<MODE, 8>(t2_dyn, full, empty, maps, a, i0, j0);
+  } else {
+    if (rb < g.x)
+      t2_tile<MODE, 8>(t2_dyn, full, empty, maps, a, i0, j0);
+    else
+      t2_tile<MODE, 6>(t2_dyn, full, empty, maps, a, i0, j0);
   }
   cta_exit(a.t);
 }
@@ -585,13 +644,44 @@ static bool tiled_t2() {
   return env != 0;
 }
 
-// a k-major operand: m rows (k) x n columns, pitch ld; box {128 columns, BK rows}
-static bool t2_map(CUtensorMap* mp, const float* base, int64_t n, int64_t m, int64_t ld, int bk) {
+// Row blocks for n rows: enough blocks of 64 and 48 rows that the tile count
+// (x 256-column strips) fills the 2 x #SM CTA slots in one wave, as many 64s
+// as needed to cover n; when n needs more than that, all blocks are 64 rows.
+static T2Geo t2_geometry(int64_t n, bool tri, bool only64) {
+  static const int nsm = [] {
+    int d = 0, v = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    return v;
+  }();
+  T2Geo g{};
+  g.cs = int((n + 255) / 256);
+  g.tri = tri ? 1 : 0;
+  const int64_t r64 = (n + 63) / 64;
+  if (tri || only64) {
+    g.rbs = g.x = int(r64);
+    return g;
+  }
+  const int64_t want = std::max<int64_t>(1, (2 * int64_t(nsm)) / g.cs);  // row blocks for one full wave
+  if (want <= r64 || 48 * want < n - 63) {  // 64-row blocks already fill (or exceed) the wave
+    g.rbs = g.x = int(r64);
+    return g;
+  }
+  // want blocks: x of 64 rows and want - x of 48, 64 x + 48 (want - x) >= n
+  const int64_t need = n - 48 * want;
+  g.x = int(need <= 0 ? 0 : (need + 15) / 16);
+  g.rbs = int(want);
+  // drop trailing 48-row blocks that lie wholly past n
+  while (g.rbs > g.x && 64 * int64_t(g.x) + 48 * int64_t(g.rbs - 1 - g.x) >= n) --g.rbs;
+  return g;
+}
+
+// a k-major operand: m rows (k) x n columns, pitch ld; box {bw columns, BK rows}
+static bool t2_map(CUtensorMap* mp, const float* base, int64_t n, int64_t m, int64_t ld, int bw, int bk) {
   auto fn = encode_fn();
   if (!fn) return false;
   const cuuint64_t dims[2] = {cuuint64_t(n), cuuint64_t(m)};
   const cuuint64_t strides[1] = {cuuint64_t(ld) * 4};
-  const cuuint32_t box[2] = {128u, cuuint32_t(bk)};
+  const cuuint32_t box[2] = {cuuint32_t(bw), cuuint32_t(bk)};
   const cuuint32_t estr[2] = {1, 1};
   return fn(mp, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -655,23 +745,33 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   }
   t2_prep_kernel<<<pg, 256, 0, s>>>(a.A, At, scale ? aAt : nullptr, n, m, ld, a.alpha);
   if (MODE == MODE_SYR2K) t2_prep_kernel<<<pg, 256, 0, s>>>(a.B, Bt, scale ? aBt : nullptr, n, m, ld, a.alpha);
+  // stage arrays, row side then column side: SYRK {(alpha A)^T} {A^T};
+  // SYR2K {(alpha A)^T, (alpha B)^T} {B^T, A^T}
   T2Maps maps{};
-  const float* src[4] = {aAt, MODE == MODE_SYR2K ? Bt : At, aBt, At};
+  using Cfg = T2Cfg<MODE>;
+  const float* src[4];
+  if (MODE == MODE_SYR2K) {
+    src[0] = aAt, src[1] = aBt, src[2] = Bt, src[3] = At;
+  } else {
+    src[0] = aAt, src[1] = At, src[2] = src[3] = nullptr;
+  }
   bool ok = true;
-  for (int q = 0; q < T2Cfg<MODE>::NA; ++q) ok = ok && t2_map(&maps.m[q], src[q], n, m, ld, T2Cfg<MODE>::BK);
+  for (int q = 0; q < Cfg::NA; ++q)
+    ok = ok && t2_map(&maps.m[q], src[q], n, m, ld, q < Cfg::NP ? Cfg::RB : Cfg::CB, Cfg::BK);
   if (!ok) {
     cudaFreeAsync(ws, s);
     return CATT_ECUDA;
   }
-  const int64_t nt = (n + 127) / 128;
-  const int64_t tiles = a.tri ? nt * (nt + 1) / 2 : nt * nt;
+  const T2Geo g = t2_geometry(n, a.tri != 0, MODE == MODE_SYR2K);
+  int64_t tiles = 0;
+  for (int rb = 0; rb < g.rbs; ++rb) tiles += g.tri ? g.cs - (int64_t(64) * rb) / 256 : g.cs;
   if (tiles > (int64_t(1) << 31) - 1) {
     cudaFreeAsync(ws, s);
     return CATT_EINVAL;
   }
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
   a.cvec = (a.nj % 4 == 0) && al(a.C);
-  tile2_kernel<MODE><<<unsigned(tiles), 256, dyn, s>>>(maps, a);
+  tile2_kernel<MODE><<<unsigned(tiles), 256, dyn, s>>>(maps, a, g);
   const catt_status ls = after_launch();
   cudaFreeAsync(ws, s);
   return ls;
