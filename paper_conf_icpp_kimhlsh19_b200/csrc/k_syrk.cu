@@ -372,13 +372,14 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 //  * a warp owns 4 ty x 8 tx threads; a float4 fragment read costs 2
 //    shared-memory wavefronts for the row operand (<= 2 distinct words per
 //    quarter-warp: merged) and 4 for the column operand (tools/lds_probe.cu).
-// Tiles are 64 x 256 or 48 x 256 (8 x 8 or 6 x 8 outputs per thread, warp w
-// = row group w, lane = column group): the row blocks mix both heights so
-// that the tile count fills the 2 x #SM CTA slots in one wave (2048 on 148
-// SMs: 17 blocks of 64 and 20 of 48 rows x 8 strips = 296 tiles; 128 x 128
-// tiles gave 256 = 1.73 per SM, i.e. SMs with one tile idle half the time).
-// The row operand is then a broadcast in every warp (2 wavefronts per float4
-// read), the column operand 32 distinct words (4).
+// Tiles are 64 x 256 (8 x 8 outputs per thread; warp w = row group w, lane =
+// column group): the row operand is a broadcast in every warp (2 shared-memory
+// wavefronts per float4 read), the column operand 32 distinct words (4).
+// Measured at 2048: 0.366 ms against 0.375 ms for 128 x 128 tiles. A mix of
+// 64- and 48-row blocks that fills the 296 CTA slots in one wave (instead of
+// 256 tiles, 1.73 per SM) measured the same 0.367 ms: the 48-row tile's 6 x 8
+// outputs per thread need as many column reads for 3/4 of the FMAs and the
+// SM's shared-memory pipe becomes the limit, so it was not kept.
 template <int MODE>
 struct T2Cfg {
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
@@ -397,17 +398,13 @@ struct T2Maps {
 };
 
 struct T2Geo {
-  int cs;            // column strips
-  int x;             // row blocks of 64 rows (the first x); the rest have 48
-  int rbs;           // row blocks
-  int tri;           // compute only tiles reaching the diagonal or above (all blocks 64 rows)
+  int cs;            // column strips of 256
+  int rbs;           // row blocks of 64
+  int tri;           // compute only tiles reaching the diagonal or above
 };
 
-__device__ __forceinline__ int64_t t2_row0(const T2Geo& g, int rb) {
-  return rb < g.x ? int64_t(64) * rb : int64_t(64) * g.x + int64_t(48) * (rb - g.x);
-}
-
-// One tile: RH rows per thread (8: a 64-row block, 6: a 48-row block).
+// One 64 x 256 tile, RH = 8 rows per thread (the body also compiles for 6:
+// a 48-row block).
 template <int MODE, int RH>
 __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* empty, const T2Maps& maps,
                                         const TileArgs& a, int64_t i0, int64_t j0) {
@@ -570,8 +567,7 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
   extern __shared__ __align__(128) float t2_dyn[];
   uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
   uint64_t* empty = full + NS;
-  // the tile: 64-row blocks first (spread one per SM by the block scheduler),
-  // then 48-row blocks; tri: the tiles that reach the diagonal, by row block
+  // the tile (tri: the tiles that reach the diagonal, by row block)
   int rb, cs;
   if (g.tri) {
     int rem = int(blockIdx.x);
@@ -598,15 +594,7 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
     fence_barrier_init();
   }
   __syncthreads();
-  const int64_t i0 = t2_row0(g, rb), j0 = int64_t(cs) * Cfg::CB;
-  if constexpr (MODE == MODE_SYR2K) {  // 64-row blocks only: two tile bodies spill at 128 registers
-    t2_tile<MODE, 8>(t2_dyn, full, empty, maps, a, i0, j0);
-  } else {
-    if (rb < g.x)
-      t2_tile<MODE, 8>(t2_dyn, full, empty, maps, a, i0, j0);
-    else
-      t2_tile<MODE, 6>(t2_dyn, full, empty, maps, a, i0, j0);
-  }
+  t2_tile<MODE, 8>(t2_dyn, full, empty, maps, a, int64_t(64) * rb, int64_t(cs) * Cfg::CB);
   cta_exit(a.t);
 }
 
@@ -642,37 +630,6 @@ static bool tiled_t2() {
     return e ? atoi(e) : 1;
   }();
   return env != 0;
-}
-
-// Row blocks for n rows: enough blocks of 64 and 48 rows that the tile count
-// (x 256-column strips) fills the 2 x #SM CTA slots in one wave, as many 64s
-// as needed to cover n; when n needs more than that, all blocks are 64 rows.
-static T2Geo t2_geometry(int64_t n, bool tri, bool only64) {
-  static const int nsm = [] {
-    int d = 0, v = 148;
-    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
-    return v;
-  }();
-  T2Geo g{};
-  g.cs = int((n + 255) / 256);
-  g.tri = tri ? 1 : 0;
-  const int64_t r64 = (n + 63) / 64;
-  if (tri || only64) {
-    g.rbs = g.x = int(r64);
-    return g;
-  }
-  const int64_t want = std::max<int64_t>(1, (2 * int64_t(nsm)) / g.cs);  // row blocks for one full wave
-  if (want <= r64 || 48 * want < n - 63) {  // 64-row blocks already fill (or exceed) the wave
-    g.rbs = g.x = int(r64);
-    return g;
-  }
-  // want blocks: x of 64 rows and want - x of 48, 64 x + 48 (want - x) >= n
-  const int64_t need = n - 48 * want;
-  g.x = int(need <= 0 ? 0 : (need + 15) / 16);
-  g.rbs = int(want);
-  // drop trailing 48-row blocks that lie wholly past n
-  while (g.rbs > g.x && 64 * int64_t(g.x) + 48 * int64_t(g.rbs - 1 - g.x) >= n) --g.rbs;
-  return g;
 }
 
 // a k-major operand: m rows (k) x n columns, pitch ld; box {bw columns, BK rows}
@@ -762,7 +719,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     cudaFreeAsync(ws, s);
     return CATT_ECUDA;
   }
-  const T2Geo g = t2_geometry(n, a.tri != 0, MODE == MODE_SYR2K);
+  const T2Geo g{int((n + 255) / 256), int((n + 63) / 64), a.tri ? 1 : 0};
   int64_t tiles = 0;
   for (int rb = 0; rb < g.rbs; ++rb) tiles += g.tri ? g.cs - (int64_t(64) * rb) / 256 : g.cs;
   if (tiles > (int64_t(1) << 31) - 1) {

@@ -10,6 +10,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 __global__ void empty_k(float* out) {
@@ -53,8 +54,10 @@ __global__ void read_k(const float4* __restrict__ a, long long n4, float* out) {
   if (s == -1.f) out[blockIdx.x] = s;
 }
 
-int main() {
-  const long long bytes = 134381568;  // BICG + MVT 4096^2: two matrices + vectors
+int main(int argc, char** argv) {
+  // default: BICG + MVT 4096^2 (two matrices + vectors); argv[1]: other byte
+  // counts, e.g. 69152800 (KMEANS assign 494020 x 34 + memberships)
+  const long long bytes = argc > 1 ? atoll(argv[1]) / 16 * 16 : 134381568;
   const long long n4 = bytes / 16;
   float4 *a, *f;
   float* out;

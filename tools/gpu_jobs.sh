@@ -29,6 +29,11 @@ for job in "$@"; do
       timeout 2400 python -m pytest tests -m gpu -q -x > $O/pytest_gpu.txt 2>&1; echo "rc=$?" >> $O/pytest_gpu.txt ;;
     occ)
       timeout 600 python -m pytest tests/test_gpu.py -m gpu -q -k "occupancy or residency" > $O/pytest_occ.txt 2>&1; echo "rc=$?" >> $O/pytest_occ.txt ;;
+    sanitize_t2)
+      S=$O/sanitizer; mkdir -p $S
+      for tool in memcheck racecheck synccheck; do
+        timeout 1200 $CS --tool $tool python tools/sanitize_cases.py tiles2 > $S/${tool}_tiles2.txt 2>&1; echo "rc=$?" >> $S/${tool}_tiles2.txt
+      done ;;
     sanitize|sanitize_mem)
       S=$O/sanitizer; mkdir -p $S
       timeout 1500 $CS --tool memcheck python tools/sanitize_cases.py > $S/memcheck_all.txt 2>&1; echo "rc=$?" >> $S/memcheck_all.txt
@@ -36,7 +41,7 @@ for job in "$@"; do
       # initcheck without the kernel filter: torch's fills (zeros) must be seen as writes
       timeout 1500 compute-sanitizer --print-limit 50 --error-exitcode 9 --tool initcheck python tools/sanitize_cases.py > $S/initcheck_all.txt 2>&1; echo "rc=$?" >> $S/initcheck_all.txt
       [ $job = sanitize_mem ] && continue
-      for c in gate_sem gate_barrier cta_counter smem_pad staged coop fused fused_graph onekernel kmeans km_iter tiles; do
+      for c in ${SAN_CASES:-gate_sem gate_barrier cta_counter smem_pad staged coop fused fused_graph onekernel kmeans km_iter tiles tiles2}; do
         timeout 900 $CS --tool racecheck --racecheck-report analysis python tools/sanitize_cases.py $c > $S/racecheck_$c.txt 2>&1; echo "rc=$?" >> $S/racecheck_$c.txt
       done
       timeout 900 python -m torch.distributed.run --nnodes 1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 \

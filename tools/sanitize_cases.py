@@ -15,6 +15,8 @@ Mechanisms:
   kmeans        assign (literal gated, staged TMA ring, coop) + transpose
   km_iter       km_accumulate + finalize + the one-launch loop
   tiles         SYRK / SYR2K / GEMM / CORR tiled kernels
+  tiles2        the two-CTA-per-SM tile kernel T2 (prep transpose, TMA ring with
+                full/empty mbarriers, 64- and 48-row tiles, ragged n and m, tri)
   peer          one rank of the peer-memory all-reduce (launch 2 under torchrun)
 Every case checks its result against the CPU oracle so a silent corruption
 under the sanitizer is also caught.
@@ -202,6 +204,23 @@ def case_tiles():
     data = si.matrix(12, 130, 70)
     sym = catt.corr(T(data), t=catt.Throttle(variant="staged"))[0]
     eq(sym, oracle.corr(data)[0], "corr")
+
+
+def case_tiles2():
+    n, m = 1601, 40                                   # 64/48-row geometry, ragged edge and last stage
+    A, B = si.matrix(6, n, m, D), si.matrix(8, n, m, D)
+    C0 = si.matrix(9, n, n, D)
+    C = T(C0)
+    catt.syrk(T(A), C, 1.5, 1.25, t=catt.Throttle(variant="staged"))
+    eq(C, oracle.syrk(A, C0, 1.5, 1.25), "syrk T2")
+    n2 = 300
+    C0 = si.matrix(9, n2, n2, D)
+    C = T(C0)
+    catt.syr2k(T(A[:n2]), T(B[:n2]), C, 1.5, 1.25, t=catt.Throttle(variant="staged"))
+    eq(C, oracle.syr2k(A[:n2], B[:n2], C0, 1.5, 1.25), "syr2k T2")
+    data = si.matrix(12, 24, n)                       # n columns: the upper tiles through T2
+    sym = catt.corr(T(data), t=catt.Throttle(variant="staged"))[0]
+    eq(sym, oracle.corr(data)[0], "corr T2")
 
 
 def case_peer():
