@@ -726,6 +726,26 @@ def test_dual_group_barrier_modes_repeated(barrier, monkeypatch):
             assert bits_equal(host(YR), q) and bits_equal(host(YC), s), (barrier, rep)
 
 
+def test_dual_group_default_launch_uniform_vs_f64_oracle():
+    """The bench's default configs[1] launch as it runs there: BICG and MVT
+    4096^2 in one grouped single-read launch, on uniform (inexact) inputs,
+    every output element within 1e-5 of the fp64 sequential oracle (the
+    dyadic tests above pin the order; this pins the arithmetic on the
+    distribution the bench uses)."""
+    n = 4096
+    Ab, Am = si.matrix(si.SEED_BICG, n, n), si.matrix(si.SEED_MVT, n, n)
+    p, r = si.values(102, n), si.values(202, n)
+    y1, y2, x1, x2 = (si.values(s, n) for s in (103, 203, 104, 204))
+    q, s_ = torch.zeros(n, device="cuda"), torch.zeros(n, device="cuda")
+    X1, X2 = dev(x1), dev(x2)
+    catt.dual_group([dict(A=dev(Ab), xr=dev(p), xc=dev(r), yr=q, yc=s_),
+                     dict(A=dev(Am), xr=dev(y1), xc=dev(y2), yr=X1, yc=X2, row_accumulate=True, col_accumulate=True)])
+    q64, s64 = oracle.bicg(Ab, p, r, mode=oracle.SEQ_F64)
+    x1_64, x2_64 = oracle.mvt(Am, y1, y2, x1, x2, mode=oracle.SEQ_F64)
+    assert relerr(host(q), q64) <= TOL and relerr(host(s_), s64) <= TOL
+    assert relerr(host(X1), x1_64) <= TOL and relerr(host(X2), x2_64) <= TOL
+
+
 def test_dual_group_uniform_same_bits_every_barrier(monkeypatch):
     """The barrier form changes only when the partials are read, never the
     order they are added in: uniform (inexact) inputs give the same bits."""
