@@ -128,6 +128,8 @@ def mvt(a, y1, y2, x1, x2, mode=SEQ_FMAF):
 def gesummv(A, B, x, alpha, beta, mode=SEQ_FMAF):
     A, B, x = _f32(A), _f32(B), _f32(x)
     n = A.shape[0]
+    if A.shape != (n, n) or B.shape != (n, n) or x.shape != (n,):   # the C loop assumes square n x n
+        raise ValueError(f"gesummv: A {A.shape}, B {B.shape}, x {x.shape}: need n x n, n x n, n")
     y, tmp = np.empty(n, np.float32), np.empty(n, np.float32)
     lib().orc_gesummv(mode, _p(A), _p(B), _p(x), _p(y), _p(tmp), n, alpha, beta)
     return y, tmp

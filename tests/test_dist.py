@@ -308,3 +308,113 @@ def test_peer_setup_exchanges_handles_world3_gloo():
         assert (w, r) == (world, rank)
         assert opened == [x for x in range(world) if x != rank]
         assert all(first_bytes[x] == x for x in opened)          # the handle of rank x came from rank x
+
+
+def _cuda_worker(rank, world, port, mode, q):
+    """The row-sharded and point-sharded paths through the CUDA kernels
+    (CudaOps, libcatt.so) in world processes that share cuda:0, with gloo
+    collectives on the CUDA tensors (NCCL needs one GPU per rank; this run
+    has one GPU)."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        C = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+        H = lambda t: (torch.cuda.synchronize(), t.cpu().numpy())[1]
+        m, n = 4099, 1024                               # ragged: 2050 + 2049 rows, several CTAs per rank
+        A = si.matrix(7, m, n, mode=mode)
+        x, p = si.values(8, n, mode=mode), si.values(9, n, mode=mode)
+        r = si.values(10, m, mode=mode)
+        lo, hi = cdist.row_range(m, world, rank)
+        tmp_g, y = cdist.atax_rowshard(C(A[lo:hi]), C(x))
+        q_g, s = cdist.bicg_rowshard(C(A[lo:hi]), C(p), C(r[lo:hi]))
+        sq = si.matrix(12, n, n, mode=mode)
+        lo2, hi2 = cdist.row_range(n, world, rank)
+        x1, x2 = si.values(13, n, mode=mode), C(si.values(14, n, mode=mode))
+        y1, y2s = si.values(15, n, mode=mode), si.values(16, n, mode=mode)
+        x1_g, x2 = cdist.mvt_rowshard(C(sq[lo2:hi2]), C(y1), C(y2s[lo2:hi2]), C(x1[lo2:hi2]), x2)
+        ng = 1027                                        # GESUMMV is square: 514 + 513 rows
+        Ag, Bg, xg = si.matrix(18, ng, ng, mode=mode), si.matrix(17, ng, ng, mode=mode), si.values(19, ng, mode=mode)
+        lo4, hi4 = cdist.row_range(ng, world, rank)
+        yg, tg = cdist.gesummv_rowshard(C(Ag[lo4:hi4]), C(Bg[lo4:hi4]), C(xg), 1.5, 1.25)
+        npts, nf, k = 3001, 6, 3                        # k-means, point-sharded, exact sums
+        feat = si.values(21, nf * npts)
+        lo3, hi3 = cdist.row_range(npts, world, rank)
+        shard = np.concatenate([feat[f * npts + lo3:f * npts + hi3] for f in range(nf)])
+        init = np.stack([feat[f * npts:f * npts + k] for f in range(nf)], axis=1)
+        cl = C(init)
+        memb, it = cdist.kmeans_pointshard(C(shard), hi3 - lo3, hi3 - lo3, nf, cl, max_iter=8)
+        q.put((rank, lo, hi, H(tmp_g), H(y), H(q_g), H(s), H(x1_g), H(x2), H(yg), H(tg), H(memb), H(cl), int(it)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", [si.MODE_DYADIC, si.MODE_UNIFORM])
+def test_rowshard_world2_cuda_kernels_gloo(mode):
+    """§8(e) at world 2 through the CUDA kernels: ATAX / BICG / MVT / GESUMMV
+    row-sharded and KMEANS point-sharded, every rank's outputs against the
+    oracle: row outputs bit-exact; the all-reduced column outputs bit-exact to
+    the per-shard oracle partials summed in fp32 (and, uniform inputs, within
+    1e-5 of the unsharded fp64 oracle); k-means bit-identical to the
+    unsharded oracle loop."""
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_cuda_worker, args=(r, world, port, mode, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = sorted([q.get(timeout=300) for _ in range(world)], key=lambda t: t[0])
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    m, n = 4099, 1024
+    A = si.matrix(7, m, n, mode=mode)
+    x, p = si.values(8, n, mode=mode), si.values(9, n, mode=mode)
+    r = si.values(10, m, mode=mode)
+    sq = si.matrix(12, n, n, mode=mode)
+    mv = (sq, si.values(15, n, mode=mode), si.values(16, n, mode=mode), si.values(13, n, mode=mode),
+          si.values(14, n, mode=mode))
+    ng = 1027
+    tmp_o, y_o = oracle.atax(A, x)
+    q_o, s_o = oracle.bicg(A, p, r)
+    x1_o, x2_o = oracle.mvt(*mv)
+    yg_o, tg_o = oracle.gesummv(si.matrix(18, ng, ng, mode=mode), si.matrix(17, ng, ng, mode=mode),
+                                si.values(19, ng, mode=mode), 1.5, 1.25)
+    cat = lambda i: np.concatenate([t[i] for t in res])
+    # row outputs: each rank's rows, sequential per row in every variant the default plan picks
+    assert np.array_equal(cat(3), tmp_o) and np.array_equal(cat(9), yg_o) and np.array_equal(cat(10), tg_o)
+    assert np.array_equal(cat(5), q_o) and np.array_equal(cat(7), x1_o)
+    for t in res:                                     # the all-reduced outputs are replicated
+        for i in (4, 6, 8):
+            assert np.array_equal(t[i], res[0][i])
+    # the all-reduced outputs: each rank's partial is its shard's sequential
+    # column loop (the oracle on the shard), and the world-2 SUM is one fp32
+    # add of the two partials: bit-exact in both modes
+    T = torch.from_numpy
+    parts = {"y": [], "s": [], "x2": []}
+    for g in range(2):
+        lo, hi = cdist.row_range(m, 2, g)
+        tmp_g, _ = oracle.atax(A[lo:hi], x)
+        parts["y"].append(OracleOps.cols(T(A[lo:hi].copy()), T(tmp_g), torch.empty(n), False).numpy())
+        parts["s"].append(OracleOps.cols(T(A[lo:hi].copy()), T(r[lo:hi].copy()), torch.empty(n), False).numpy())
+        lo2, hi2 = cdist.row_range(n, 2, g)
+        x2_init = mv[4].copy() if g == 0 else np.zeros(n, np.float32)
+        parts["x2"].append(OracleOps.cols(T(sq[lo2:hi2].copy()), T(mv[2][lo2:hi2].copy()), T(x2_init), g == 0).numpy())
+    for key, i in (("y", 4), ("s", 6), ("x2", 8)):
+        want = (parts[key][0] + parts[key][1]).astype(np.float32)
+        assert np.array_equal(res[0][i], want), key
+    if mode == si.MODE_UNIFORM:                       # and within the 1e-5 bar of fp64
+        _, y64 = oracle.atax(A, x, mode=oracle.SEQ_F64)
+        _, s64 = oracle.bicg(A, p, r, mode=oracle.SEQ_F64)
+        _, x2_64 = oracle.mvt(*mv, mode=oracle.SEQ_F64)
+        for got, ref in ((res[0][4], y64), (res[0][6], s64), (res[0][8], x2_64)):
+            assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-5
+    from oracle import kmeans as okm
+    npts, nf, k = 3001, 6, 3
+    feat = si.values(21, nf * npts)
+    init = np.stack([feat[f * npts:f * npts + k] for f in range(nf)], axis=1)
+    cl_o, memb_o, it_o, _ = okm.kmeans(feat, npts, npts, nf, init, max_iter=8)
+    assert np.array_equal(cat(11), memb_o)
+    for t in res:
+        assert np.array_equal(t[12], cl_o) and t[13] == it_o
