@@ -207,10 +207,10 @@ __global__ void corr_diag_kernel(float* symmat, int64_t m) {
   if (j < m) symmat[j * m + j] = 1.0f;
 }
 
-const void* syrk_func(int variant);
+const void* syrk_func(int variant, int64_t n, bool tri);
 
-const void* corr_func(int variant) {
-  return variant == CATT_VAR_STAGED ? syrk_func(CATT_VAR_STAGED) : (const void*)corr_thread_kernel;
+const void* corr_func(int variant, int64_t m) {
+  return variant == CATT_VAR_STAGED ? syrk_func(CATT_VAR_STAGED, m, true) : (const void*)corr_thread_kernel;
 }
 
 }  // namespace catt

@@ -380,13 +380,20 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 // 256 tiles, 1.73 per SM) measured the same 0.367 ms: the 48-row tile's 6 x 8
 // outputs per thread need as many column reads for 3/4 of the FMAs and the
 // SM's shared-memory pipe becomes the limit, so it was not kept.
-template <int MODE>
+// RH rows per thread: 8 (64-row tiles, two CTAs per SM, <= 128 registers).
+// The template also builds RH = 15 (120-row tiles, one CTA per SM, 222
+// registers: 15 x 8 outputs per thread cut the shared-memory wavefronts per
+// FMA by 0.6x, and 2048 rows make 144 tiles for 148 SMs); measured slower at
+// every size (2048: 0.379 vs 0.357 ms; 4096: 1.65 vs 1.15 ms; one CTA of 8
+// warps per SM does not keep the FMA pipe busy), so only RH = 8 is launched.
+template <int MODE, int RH = 8>
 struct T2Cfg {
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int NP = NA / 2;                               // row-side (and column-side) arrays
   static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
-  static constexpr int NS = 4;                                   // ring stages
-  static constexpr int RB = 64, CB = 256;                        // row box, column strip
+  static constexpr int MINB = RH > 8 ? 1 : 2;                    // CTAs per SM
+  static constexpr int NS = RH > 8 ? 6 : 4;                      // ring stages
+  static constexpr int RB = 8 * RH, CB = 256;                    // row box, column strip
   static constexpr int ROW_FLOATS = BK * RB, COL_FLOATS = BK * CB;
   static constexpr int STAGE_FLOATS = NP * (ROW_FLOATS + COL_FLOATS);
   static constexpr int FBUF = MODE == MODE_SYR2K ? 1 : 2;
@@ -399,19 +406,20 @@ struct T2Maps {
 
 struct T2Geo {
   int cs;            // column strips of 256
-  int rbs;           // row blocks of 64
+  int rbs;           // row blocks of 8 * RH rows
   int tri;           // compute only tiles reaching the diagonal or above
 };
 
-// One 64 x 256 tile, RH = 8 rows per thread (the body also compiles for 6:
-// a 48-row block).
+// One (8 RH) x 256 tile, RH rows per thread: rows {32 g + 4 ty + r} for the
+// G = RH / 4 full groups, then {32 G + (RH % 4) ty + r} (ty = warp).
 template <int MODE, int RH>
 __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* empty, const T2Maps& maps,
                                         const TileArgs& a, int64_t i0, int64_t j0) {
   constexpr bool TWO = MODE == MODE_SYR2K;
-  using Cfg = T2Cfg<MODE>;
+  using Cfg = T2Cfg<MODE, RH>;
   constexpr int BK = Cfg::BK, NP = Cfg::NP, NS = Cfg::NS, RBX = Cfg::RB, CBX = Cfg::CB;
-  // stage layout: NP row arrays [BK][64], then NP column arrays [BK][256]
+  constexpr int G = RH / 4, RR = RH % 4;
+  // stage layout: NP row arrays [BK][8 RH], then NP column arrays [BK][256]
   auto rowp = [&](int slot, int s, int kk) { return sm + slot * Cfg::STAGE_FLOATS + s * Cfg::ROW_FLOATS + kk * RBX; };
   auto colp = [&](int slot, int s, int kk) {
     return sm + slot * Cfg::STAGE_FLOATS + NP * Cfg::ROW_FLOATS + s * Cfg::COL_FLOATS + kk * CBX;
@@ -420,8 +428,7 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
   const int ty = warp, tx = lane;
   const int64_t n = a.ni, m = a.m;
   const int64_t ktiles = (m + BK - 1) / BK;
-  // rows of this thread: r < 4: ty*4 + r; r >= 4: 32 + ty*(RH - 4) + r - 4
-  auto row_of = [&](int r) { return r < 4 ? ty * 4 + r : 32 + ty * (RH - 4) + (r - 4); };
+  auto row_of = [&](int r) { return r < 4 * G ? 32 * (r / 4) + 4 * ty + (r % 4) : 32 * G + RR * ty + (r - 4 * G); };
 
   // row-side stage arrays: alpha*a[i][k] (SYR2K: then alpha*b[i][k]); column-side: a[j][k]
   // (SYR2K: b[j][k], then a[j][k]); maps in the same order
@@ -465,14 +472,17 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
 #pragma unroll
     for (int s = 0; s < NP; ++s) {
       const float* rp = rowp(slot, s, kk);
-      const float4 v0 = *reinterpret_cast<const float4*>(rp + ty * 4);
-      fr[fb][s][0] = v0.x, fr[fb][s][1] = v0.y, fr[fb][s][2] = v0.z, fr[fb][s][3] = v0.w;
-      if constexpr (RH == 8) {
-        const float4 v1 = *reinterpret_cast<const float4*>(rp + 32 + ty * 4);
-        fr[fb][s][4] = v1.x, fr[fb][s][5] = v1.y, fr[fb][s][6] = v1.z, fr[fb][s][7] = v1.w;
+#pragma unroll
+      for (int g = 0; g < G; ++g) {
+        const float4 v = *reinterpret_cast<const float4*>(rp + 32 * g + ty * 4);
+        fr[fb][s][4 * g] = v.x, fr[fb][s][4 * g + 1] = v.y, fr[fb][s][4 * g + 2] = v.z, fr[fb][s][4 * g + 3] = v.w;
+      }
+      if constexpr (RR == 2) {
+        const float2 v = *reinterpret_cast<const float2*>(rp + 32 * G + ty * 2);
+        fr[fb][s][4 * G] = v.x, fr[fb][s][4 * G + 1] = v.y;
       } else {
-        const float2 v1 = *reinterpret_cast<const float2*>(rp + 32 + ty * 2);
-        fr[fb][s][4] = v1.x, fr[fb][s][5] = v1.y;
+#pragma unroll
+        for (int q = 0; q < RR; ++q) fr[fb][s][4 * G + q] = rp[32 * G + RR * ty + q];
       }
       const float* cq = colp(slot, s, kk);
 #pragma unroll
@@ -559,10 +569,11 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
   }
 }
 
-template <int MODE>
-__global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T2Maps maps, TileArgs a, T2Geo g) {
+template <int MODE, int RH>
+__global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __grid_constant__ T2Maps maps, TileArgs a,
+                                                                      T2Geo g) {
   static_assert(MODE != MODE_GEMM, "T2 covers SYRK and SYR2K");
-  using Cfg = T2Cfg<MODE>;
+  using Cfg = T2Cfg<MODE, RH>;
   constexpr int NS = Cfg::NS;
   extern __shared__ __align__(128) float t2_dyn[];
   uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
@@ -573,7 +584,7 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
     int rem = int(blockIdx.x);
     rb = 0;
     while (true) {
-      const int lo = int((int64_t(64) * rb) / 256);  // first strip with an element j >= i
+      const int lo = int((int64_t(Cfg::RB) * rb) / 256);  // first strip with an element j >= i
       if (rem < g.cs - lo) {
         cs = lo + rem;
         break;
@@ -594,7 +605,7 @@ __global__ void __launch_bounds__(256, 2) tile2_kernel(const __grid_constant__ T
     fence_barrier_init();
   }
   __syncthreads();
-  t2_tile<MODE, 8>(t2_dyn, full, empty, maps, a, int64_t(64) * rb, int64_t(cs) * Cfg::CB);
+  t2_tile<MODE, RH>(t2_dyn, full, empty, maps, a, int64_t(Cfg::RB) * rb, int64_t(cs) * Cfg::CB);
   cta_exit(a.t);
 }
 
@@ -650,10 +661,16 @@ static bool t2_ok(const TileArgs& a) {
   return tiled_t2() && a.m > 0 && a.m < (int64_t(1) << 31) && a.ni < (int64_t(1) << 31);
 }
 
-template <int MODE>
+static int64_t t2_tiles(const T2Geo& g, int rb_rows) {
+  int64_t tiles = 0;
+  for (int rb = 0; rb < g.rbs; ++rb) tiles += g.tri ? g.cs - (int64_t(rb_rows) * rb) / 256 : g.cs;
+  return tiles;
+}
+
+template <int MODE, int RH>
 static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s) {
-  const void* f = (const void*)tile2_kernel<MODE>;
-  constexpr size_t sb = T2Cfg<MODE>::SBYTES;
+  const void* f = (const void*)tile2_kernel<MODE, RH>;
+  constexpr size_t sb = T2Cfg<MODE, RH>::SBYTES;
   cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sb));
   if (e != cudaSuccess) {
     record_cuda_error(e);
@@ -705,7 +722,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   // stage arrays, row side then column side: SYRK {(alpha A)^T} {A^T};
   // SYR2K {(alpha A)^T, (alpha B)^T} {B^T, A^T}
   T2Maps maps{};
-  using Cfg = T2Cfg<MODE>;
+  using Cfg = T2Cfg<MODE, RH>;
   const float* src[4];
   if (MODE == MODE_SYR2K) {
     src[0] = aAt, src[1] = aBt, src[2] = Bt, src[3] = At;
@@ -719,16 +736,15 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     cudaFreeAsync(ws, s);
     return CATT_ECUDA;
   }
-  const T2Geo g{int((n + 255) / 256), int((n + 63) / 64), a.tri ? 1 : 0};
-  int64_t tiles = 0;
-  for (int rb = 0; rb < g.rbs; ++rb) tiles += g.tri ? g.cs - (int64_t(64) * rb) / 256 : g.cs;
+  const T2Geo g{int((n + 255) / 256), int((n + Cfg::RB - 1) / Cfg::RB), a.tri ? 1 : 0};
+  const int64_t tiles = t2_tiles(g, Cfg::RB);
   if (tiles > (int64_t(1) << 31) - 1) {
     cudaFreeAsync(ws, s);
     return CATT_EINVAL;
   }
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
   a.cvec = (a.nj % 4 == 0) && al(a.C);
-  tile2_kernel<MODE><<<unsigned(tiles), 256, dyn, s>>>(maps, a, g);
+  tile2_kernel<MODE, RH><<<unsigned(tiles), 256, dyn, s>>>(maps, a, g);
   const catt_status ls = after_launch();
   cudaFreeAsync(ws, s);
   return ls;
@@ -805,7 +821,7 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
   const bool small = small_tiles<MODE>(a.ni, a.nj);
   if constexpr (MODE != MODE_GEMM)
-    if (!small && t2_ok<MODE>(a)) return launch_t2<MODE>(a, t, s);
+    if (!small && t2_ok<MODE>(a)) return launch_t2<MODE, 8>(a, t, s);
   constexpr int TMs = MODE == MODE_SYR2K ? 8 : 4;  // SYR2K never takes the small tile (static_assert)
   const int64_t tt = (a.ni + 127) / 128;
   const bool lean = !small && MODE == MODE_SYRK && tiled_lean(a.tri ? tt * (tt + 1) / 2 : tt * tt);
@@ -865,22 +881,27 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
 
 // the kernel a large (128 x 128 tile) STAGED launch runs, and its dynamic
 // shared memory (catt_kernel_desc / catt_plan describe this kernel)
-const void* syrk_func(int variant) {
+const void* syrk_func(int variant, int64_t n, bool tri) {
   if (variant != CATT_VAR_STAGED) return (const void*)syrk_thread_kernel;
-  return tiled_t2() ? (const void*)tile2_kernel<MODE_SYRK> : tiled_func<MODE_SYRK>();
+  if (!tiled_t2()) return tiled_func<MODE_SYRK>();
+  return (const void*)tile2_kernel<MODE_SYRK, 8>;
+  (void)n, (void)tri;
 }
 
-int64_t syrk_staged_dyn() { return tiled_t2() ? int64_t(T2Cfg<MODE_SYRK>::SBYTES) : 0; }
+int64_t syrk_staged_dyn(int64_t n, bool tri) {
+  (void)n, (void)tri;
+  return tiled_t2() ? int64_t(T2Cfg<MODE_SYRK, 8>::SBYTES) : 0;
+}
 
 const void* syr2k_func(int variant) {
   if (variant != CATT_VAR_STAGED) return (const void*)syr2k_thread_kernel;
-  if (tiled_t2()) return (const void*)tile2_kernel<MODE_SYR2K>;
+  if (tiled_t2()) return (const void*)tile2_kernel<MODE_SYR2K, 8>;
   if (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) return (const void*)tiled_kernel<MODE_SYR2K, 1, 8, false, true>;
   return tiled_func<MODE_SYR2K>();
 }
 
 int64_t syr2k_staged_dyn() {
-  if (tiled_t2()) return int64_t(T2Cfg<MODE_SYR2K>::SBYTES);
+  if (tiled_t2()) return int64_t(T2Cfg<MODE_SYR2K, 8>::SBYTES);
   return (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) ? int64_t(TileCfg<MODE_SYR2K, 8, false, true>::SBYTES) : 0;
 }
 
