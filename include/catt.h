@@ -525,6 +525,25 @@ catt_status catt_peer_destroy(catt_peer* p);
 catt_status catt_atax_peer(const float* A, const float* x, float* tmp, float* y, int64_t m, int64_t n, catt_peer* p,
                            void* stream);
 
+/* The same peer state over memory the caller maps (the
+ * NVSwitch form): symmetric memory in which every rank's buffer is mapped
+ * into every process (e.g. torch.distributed._symmetric_memory
+ * `buffer_ptrs`), optionally with a multicast alias of those buffers bound
+ * to an NVLS multicast object (`multicast_ptr`). bases[r] is rank r's buffer
+ * as mapped in this process, each catt_peer_bytes(world, n) bytes, 256-byte
+ * aligned and zero-filled before the first launch; the caller keeps them
+ * mapped until catt_peer_destroy (the library frees nothing of them).
+ * mc_base: the multicast alias (256-byte aligned) or NULL. With mc_base
+ * each column partial and each flag is one multimem.st (the NVSwitch
+ * replicates it to every rank) instead of one store per rank; without it
+ * the kernel stores to every rank through bases[] as with CUDA IPC. The sums
+ * are read from this rank's own buffer in rank order either way, so results
+ * are the same bits as catt_peer_create's. catt_peer_open is not used
+ * (CATT_EINVAL). Errors: CATT_EINVAL (arguments, misaligned bases). */
+int64_t catt_peer_bytes(int32_t world, int64_t n);
+catt_status catt_peer_create_mapped(int32_t world, int32_t rank, int64_t n, void* const* bases, void* mc_base,
+                                    catt_peer** out);
+
 /* ------------------------------------------------------------ SM partition
  * A stream whose kernels run on a partition of the device's SMs (a CUDA green
  * context, driver 12.4+). SURVEY 8(d) [3]: CTA-level throttling (Fig 5,

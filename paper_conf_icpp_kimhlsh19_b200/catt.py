@@ -185,6 +185,7 @@ def lib():
             "catt_fused_trace": [P(u64), i32],
             "catt_peer_create": [i32, i32, i64, P(V), V],
             "catt_peer_open": [V, i32, V],
+            "catt_peer_create_mapped": [i32, i32, i64, P(V), V, P(V)],
             "catt_peer_check": [V, P(i32)],
             "catt_peer_destroy": [V],
             "catt_atax_peer": [V, V, V, V, i64, i64, V, V],
@@ -203,6 +204,8 @@ def lib():
         L.catt_status_str.restype = ctypes.c_char_p
         L.catt_kmeans_acc_words.argtypes = [i32, i32]
         L.catt_kmeans_acc_words.restype = ctypes.c_int64
+        L.catt_peer_bytes.argtypes = [i32, i64]
+        L.catt_peer_bytes.restype = ctypes.c_int64
         _lib = L
     return _lib
 
@@ -214,6 +217,7 @@ EXPORTED = ["catt_hw_query", "catt_hw_b200", "catt_hw_titanv", "catt_footprint",
             "catt_kmeans", "catt_rows", "catt_cols", "catt_dual", "catt_dual_group", "catt_fill_hash", "catt_calibrate_l1", "catt_kernel_attrs",
             "catt_kernel_occupancy", "catt_status_str",
             "catt_last_cuda_error", "catt_abi_version", "catt_fused_trace", "catt_peer_create", "catt_peer_open",
+            "catt_peer_bytes", "catt_peer_create_mapped",
             "catt_peer_check", "catt_peer_destroy", "catt_atax_peer", "catt_dual_group_peer", "catt_atax_onekernel", "catt_sm_partition_create",
             "catt_sm_partition_destroy"]
 
@@ -500,12 +504,34 @@ class Peer:
     """This rank's peer-memory all-reduce state (catt_peer_*): create, ship
     `handle` (bytes) to the other ranks, `open` theirs, then `atax_peer`."""
 
-    def __init__(self, world, rank, n):
+    def __init__(self, world, rank, n, _mapped=None):
         self.ptr = ctypes.c_void_p()
+        self.world, self.rank, self.n = world, rank, n
+        self.multicast = False
+        if _mapped is not None:                      # Peer.mapped
+            bases, mc, self._keep = _mapped
+            arr = (ctypes.c_void_p * world)(*bases)
+            _check(lib().catt_peer_create_mapped(world, rank, n, arr, ctypes.c_void_p(mc or None), ctypes.byref(self.ptr)),
+                   "catt_peer_create_mapped")
+            self.handle = None
+            self.multicast = bool(mc)
+            return
         buf = ctypes.create_string_buffer(PEER_HANDLE_BYTES)
         _check(lib().catt_peer_create(world, rank, n, ctypes.byref(self.ptr), buf), "catt_peer_create")
         self.handle = buf.raw
-        self.world, self.rank, self.n = world, rank, n
+
+    @staticmethod
+    def nbytes(world, n) -> int:
+        """Bytes of one rank's peer buffer (catt_peer_bytes)."""
+        return int(lib().catt_peer_bytes(world, n))
+
+    @classmethod
+    def mapped(cls, world, rank, n, bases, multicast_ptr=0, keep=None):
+        """Peer state over caller-mapped memory (catt_peer_create_mapped):
+        bases[r] = rank r's buffer as mapped here (symmetric memory), each
+        Peer.nbytes(world, n) bytes, zero-filled; multicast_ptr = the NVLS
+        multicast alias or 0. `keep` is held so the mapping outlives the peer."""
+        return cls(world, rank, n, _mapped=(list(bases), multicast_ptr, keep))
 
     def open(self, peer_rank, handle: bytes):
         buf = ctypes.create_string_buffer(handle, PEER_HANDLE_BYTES)

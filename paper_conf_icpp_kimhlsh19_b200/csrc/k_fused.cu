@@ -63,6 +63,8 @@ struct FusedArgs {
   // all-reduced across ranks through peer memory inside this kernel
   float* peer_recv[kMaxPeers];       // rank p's receive buffer [2 parities][world][N] (IPC-mapped)
   unsigned* peer_flag[kMaxPeers];    // rank p's flags [2][world][kPeerCtas]
+  float* mc_recv;                    // multicast alias of every rank's receive buffer (NVLS), or null
+  unsigned* mc_flag;                 // multicast alias of every rank's flags, or null
   unsigned* peer_err;                // this rank's error word (a wait timed out)
   int world, rank;                   // world = 0: no peer reduction
   unsigned epoch;                    // launch number, equal on every rank
@@ -134,6 +136,23 @@ __device__ __forceinline__ void grid_barrier_ordered(unsigned* bar, unsigned nbl
 // launched another grid (unequal shards) sets it to 2 at once.
 // The flag half of it: publish this CTA's partials, wait for the same CTA
 // index of every rank. Returns false (every thread) after a 10 s give-up.
+// One store that lands in every rank's copy of a buffer bound to a multicast
+// object (NVSwitch NVLS): replaces the world per-peer stores.
+__device__ __forceinline__ void mc_st_f32(float* p, float v) {
+  asm volatile("multimem.st.relaxed.sys.global.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+__device__ __forceinline__ void mc_st_release_u32(unsigned* p, unsigned v) {
+  asm volatile("multimem.st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+// this rank's partial of one column into slot `slot` of every rank's receive buffer
+__device__ __forceinline__ void peer_put(const FusedArgs& a, int64_t slot, float v) {
+  if (a.mc_recv) {
+    mc_st_f32(a.mc_recv + slot, v);
+  } else {
+    for (int p = 0; p < a.world; ++p) a.peer_recv[p][slot] = v;
+  }
+}
+
 __device__ bool peer_flags(const FusedArgs& a) {
   const unsigned par = a.epoch & 1u;
   // the flag carries the launch's grid size beside the epoch: the chunk ->
@@ -148,9 +167,12 @@ __device__ bool peer_flags(const FusedArgs& a) {
   __shared__ int s_ok;
   if (threadIdx.x == 0) {
     if (!a.fence_all) __threadfence_system();
-    for (int p = 0; p < a.world; ++p) {
-      unsigned* f = a.peer_flag[p] + (int64_t(par) * a.world + a.rank) * kPeerCtas + blockIdx.x;
-      asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(tag) : "memory");
+    const int64_t fo = (int64_t(par) * a.world + a.rank) * kPeerCtas + blockIdx.x;
+    if (a.mc_flag) {
+      mc_st_release_u32(a.mc_flag + fo, tag);
+    } else {
+      for (int p = 0; p < a.world; ++p)
+        asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(a.peer_flag[p] + fo), "r"(tag) : "memory");
     }
     int ok = 1;
     const unsigned long long t0 = gtimer();
@@ -363,7 +385,7 @@ __global__ void __launch_bounds__(NW * 32, 1) fused_kernel(FusedArgs a, int RPS,
         if (a.world > 0) {
           // this rank's partial of column j, stored into every rank's slot [par][rank]
           const int64_t slot = (int64_t(a.epoch & 1u) * a.world + a.rank) * N + j;
-          for (int p = 0; p < a.world; ++p) a.peer_recv[p][slot] = tot;
+          peer_put(a, slot, tot);
         } else {
           if (a.col_acc[q]) tot = a.yc[q][j] + tot;
           a.yc[q][j] = tot;
@@ -661,7 +683,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) fused_nd_kernel(FusedArgs a,
               // row-sharded (catt_dual_group_peer): this rank's partial of
               // column j of problem q into slot [par][rank] of every rank
               const int64_t slot = (int64_t(a.epoch & 1u) * a.world + a.rank) * (N * a.nprob) + int64_t(q) * N + j;
-              for (int p = 0; p < a.world; ++p) a.peer_recv[p][slot] = tot;
+              peer_put(a, slot, tot);
             } else {
               if (a.col_acc[q]) tot = y0[l] + tot;
               a.yc[q][j] = tot;
@@ -852,8 +874,10 @@ catt_status launch_atax_small(const DualProblem& p, int64_t N, cudaStream_t s) {
 struct catt_peer {
   int world = 0, rank = 0;
   int64_t n = 0;
-  void* base = nullptr;
+  void* base = nullptr;              // own allocation (catt_peer_create), else null
   size_t bytes = 0;
+  float* mc_recv = nullptr;          // catt_peer_create_mapped with a multicast alias
+  unsigned* mc_flag = nullptr;
   float* recv[catt::kMaxPeers] = {};
   unsigned* flag[catt::kMaxPeers] = {};
   void* opened[catt::kMaxPeers] = {};
@@ -1005,6 +1029,8 @@ catt_status launch_fused_group(bool dep, const DualProblem* pr, int np, int64_t 
     args.epoch = ++P->epoch;
     args.fence_all = getenv("CATT_PEER_FENCE_ALL") != nullptr;
     args.peer_err = P->err;
+    args.mc_recv = P->mc_recv;
+    args.mc_flag = P->mc_flag;
     for (int r = 0; r < P->world; ++r) {
       args.peer_recv[r] = P->recv[r];
       args.peer_flag[r] = P->flag[r];
@@ -1109,9 +1135,42 @@ extern "C" catt_status catt_peer_create(int32_t world, int32_t rank, int64_t n, 
   return CATT_OK;
 }
 
+extern "C" int64_t catt_peer_bytes(int32_t world, int64_t n) {
+  if (world < 1 || world > kMaxPeers || n < 1) return -1;
+  size_t foff = 0, eoff = 0;
+  return int64_t(peer_layout(world, n, &foff, &eoff));
+}
+
+extern "C" catt_status catt_peer_create_mapped(int32_t world, int32_t rank, int64_t n, void* const* bases, void* mc_base,
+                                               catt_peer** out) {
+  if (!out || !bases || world < 1 || world > kMaxPeers || rank < 0 || rank >= world || n < 1) return CATT_EINVAL;
+  for (int r = 0; r < world; ++r)
+    if (!bases[r] || (reinterpret_cast<uintptr_t>(bases[r]) & 255u)) return CATT_EINVAL;
+  if (reinterpret_cast<uintptr_t>(mc_base) & 255u) return CATT_EINVAL;
+  catt_peer* p = new catt_peer();
+  p->world = world;
+  p->rank = rank;
+  p->n = n;
+  size_t foff = 0, eoff = 0;
+  p->bytes = peer_layout(world, n, &foff, &eoff);
+  for (int r = 0; r < world; ++r) {
+    char* b = static_cast<char*>(bases[r]);
+    p->recv[r] = reinterpret_cast<float*>(b);
+    p->flag[r] = reinterpret_cast<unsigned*>(b + foff);
+  }
+  p->err = reinterpret_cast<unsigned*>(static_cast<char*>(bases[rank]) + eoff);
+  if (mc_base) {
+    p->mc_recv = static_cast<float*>(mc_base);
+    p->mc_flag = reinterpret_cast<unsigned*>(static_cast<char*>(mc_base) + foff);
+  }
+  *out = p;
+  return CATT_OK;
+}
+
 extern "C" catt_status catt_peer_open(catt_peer* p, int32_t peer_rank, const void* handle) {
   if (!p || !handle || peer_rank < 0 || peer_rank >= p->world) return CATT_EINVAL;
   if (peer_rank == p->rank) return CATT_OK;                  // own buffer: nothing to open
+  if (!p->base) return CATT_EINVAL;                          // mapped by the caller (catt_peer_create_mapped)
   if (p->opened[peer_rank]) return CATT_EINVAL;
   cudaIpcMemHandle_t h;
   std::memcpy(&h, handle, sizeof(h));

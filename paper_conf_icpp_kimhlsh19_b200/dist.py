@@ -94,6 +94,29 @@ def peer_setup(n, group=None):
     return peer
 
 
+def peer_setup_symmetric(n, group=None):
+    """This rank's catt.Peer over PyTorch symmetric memory (SURVEY 8(f) f4,
+    the NVSwitch form): every rank's buffer mapped into every process, and,
+    where the device and driver support NVLS multicast, a multicast alias so
+    the in-kernel all-reduce stores each partial once (multimem.st) instead
+    of once per rank. Falls back to per-rank stores through the mapped
+    buffers when there is no multicast (peer.multicast tells which). Needs an
+    initialised process group (NCCL) with one GPU per rank."""
+    import torch
+    import torch.distributed as dist
+    import torch.distributed._symmetric_memory as symm
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    nb = catt.Peer.nbytes(world, n)
+    buf = symm.empty(nb, dtype=torch.uint8, device=torch.device("cuda", torch.cuda.current_device()))
+    buf.zero_()
+    h = symm.rendezvous(buf, group if group is not None else dist.group.WORLD)
+    torch.cuda.synchronize()
+    h.barrier()
+    mc = int(h.multicast_ptr) if getattr(h, "has_multicast_support", lambda: False)() else 0
+    return catt.Peer.mapped(world, rank, n, [int(p) for p in h.buffer_ptrs], mc, keep=(buf, h))
+
+
 def atax_rowshard_peer(A_g, x, peer, tmp_g=None, y=None):
     """tmp_g = A_g x; y = sum over ranks of A_g^T tmp_g, with the sum done
     inside the fused kernel through peer memory (no NCCL call): one launch

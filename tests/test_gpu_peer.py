@@ -311,3 +311,90 @@ def test_atax_peer_grid_mismatch_is_reported_not_hung(tmp_path):
     time limit instead of summing stale slots."""
     errs = _run_uneven(tmp_path, [100, 101], 1028)
     assert all(e in (1, 2) for e in errs) and 2 in errs, errs
+
+
+# ------------------------------------------------------------------ caller-mapped (symmetric) peer memory
+@pytest.mark.gpu
+def test_peer_mapped_buffer_equals_grouped_launch():
+    """catt_peer_create_mapped over a plain device buffer (one rank, no
+    multicast alias): the per-rank store path through caller-mapped memory,
+    bit-identical to the grouped launch on every launch (both parities); the
+    argument checks of the mapped form."""
+    import torch
+    import paper_conf_icpp_kimhlsh19_b200 as catt
+    m, n = 900, 1028
+    args = _bm_problem(m, n)
+    ref = _bm_group(torch, *args, 0, m)
+    catt.dual_group(ref)
+    nb = catt.Peer.nbytes(1, 2 * n)
+    assert nb > 2 * 2 * n * 4
+    buf = torch.zeros(nb, dtype=torch.uint8, device="cuda")
+    peer = catt.Peer.mapped(1, 0, 2 * n, [buf.data_ptr()], 0, keep=buf)
+    try:
+        assert not peer.multicast
+        for _ in range(3):
+            g = _bm_group(torch, *args, 0, m)
+            catt.dual_group_peer(g, peer)
+            torch.cuda.synchronize()
+            for a, b in zip(g, ref):
+                assert np.array_equal(a["yr"].cpu().numpy(), b["yr"].cpu().numpy())
+                assert np.array_equal(a["yc"].cpu().numpy(), b["yc"].cpu().numpy())
+        assert not peer.timed_out()
+        with pytest.raises(catt.CattError):                  # no IPC handles to open on a mapped peer
+            peer.open(0, bytes(catt.PEER_HANDLE_BYTES))
+    finally:
+        peer.close()
+    with pytest.raises(catt.CattError):                      # misaligned base
+        catt.Peer.mapped(1, 0, 2 * n, [buf.data_ptr() + 4], 0)
+    assert catt.Peer.nbytes(0, n) < 0 and catt.Peer.nbytes(1, 0) < 0
+
+
+def _symm_worker(port, m, n, q):
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
+        import paper_conf_icpp_kimhlsh19_b200 as catt
+        args = _bm_problem(m, n)
+        ref = _bm_group(torch, *args, 0, m)
+        catt.dual_group(ref)
+        try:
+            peer = cdist.peer_setup_symmetric(2 * n)
+        except Exception as e:                               # symmetric memory unavailable here
+            q.put(("skip", f"{type(e).__name__}: {e}"))
+            return
+        ok = True
+        for _ in range(3):
+            g = _bm_group(torch, *args, 0, m)
+            catt.dual_group_peer(g, peer)
+            torch.cuda.synchronize()
+            for a, b in zip(g, ref):
+                ok &= np.array_equal(a["yr"].cpu().numpy(), b["yr"].cpu().numpy())
+                ok &= np.array_equal(a["yc"].cpu().numpy(), b["yc"].cpu().numpy())
+        ok &= not peer.timed_out()
+        mc = peer.multicast
+        peer.close()
+        q.put(("ok" if ok else "mismatch", f"multicast={mc}"))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+def test_peer_over_torch_symmetric_memory_single_rank():
+    """dist.peer_setup_symmetric (the NVSwitch form, §8(f) f4) at world 1:
+    PyTorch symmetric memory as the peer buffer, the multicast alias when the
+    device offers one (this one-GPU box does not: the per-rank path runs),
+    results bit-identical to the grouped launch."""
+    import multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    pr = ctx.Process(target=_symm_worker, args=(_free_port(), 900, 1028, q))
+    pr.start()
+    status, info = q.get(timeout=300)
+    pr.join(timeout=60)
+    if status == "skip":
+        pytest.skip(f"torch symmetric memory unavailable: {info}")
+    assert status == "ok" and pr.exitcode == 0, info

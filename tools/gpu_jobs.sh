@@ -13,6 +13,7 @@
 #   ncu       ncu --set full of the default bench's dominant kernel
 #   tiles     FP32 tile kernels: bit-exact tests, T2 vs tiled_kernel timing, FFMA2 peak probe
 #   ncutile   ncu --set full of one tile kernel (NCU_KERNEL, TILE_ONLY)
+#   ncut2     ncu --set full of the T2 tile kernel for syrk / syr2k / corr (details csv)
 #   sass      per-kernel SASS opcode summary of libcatt.so
 #   mcprobe   NVLS multicast support with one visible GPU (tools/multicast_probe)
 export PYTHONPATH=.
@@ -74,6 +75,12 @@ for job in "$@"; do
     ncutile)
       timeout 600 ncu --set full --clock-control none --import-source on -k regex:${NCU_KERNEL:-tile2} -s 1 -c 1 -o $O/ncu_tile -f \
         python tools/tile_bench.py --reps 1 --only ${TILE_ONLY:-syrk} > $O/ncu_tile.log 2>&1 ;;
+    ncut2)
+      for w in syrk syr2k corr; do
+        timeout 600 ncu --set full --clock-control none --import-source on -k regex:tile2 -s 1 -c 1 -o $O/ncu_t2_$w -f \
+          python tools/tile_bench.py --reps 1 --only $w > $O/ncu_t2_$w.log 2>&1
+        ncu -i $O/ncu_t2_$w.ncu-rep --page details --csv > $O/ncu_t2_${w}_details.csv 2>/dev/null
+      done ;;
     sass)
       python tools/sass_summary.py paper_conf_icpp_kimhlsh19_b200/libcatt.so > $O/sass_summary.txt 2>&1 ;;
     *)
