@@ -42,5 +42,10 @@ inline int variant_of(const catt_throttle* t) { return t ? t->variant : CATT_VAR
 
 // Tiled SYRK over the tiles on and above the diagonal only (k_syrk.cu).
 catt_status syrk_upper(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta, cudaStream_t s);
+// CORR: symmat = D^T D (upper tiles, accumulators from +0) with D (nrows x
+// mcols) the centred data and Dt = D^T (mcols x nrows) its transpose (only
+// read when syrk_kmajor_ok(D, mcols) is false; may be null otherwise).
+bool syrk_kmajor_ok(const float* D, int64_t mcols);
+catt_status syrk_upper_kmajor(const float* D, const float* Dt, float* C, int64_t mcols, int64_t nrows, cudaStream_t s);
 
 }  // namespace catt

@@ -117,6 +117,9 @@ struct TileArgs {
   int cvec; // nj % 4 == 0 and C 16-B aligned
   int tri;  // SYRK only: compute the tiles on and above the diagonal (C symmetric; caller mirrors)
   Throttle t;
+  int zinit = 0;              // T2: accumulators start at +0 without reading C (CORR's s = 0)
+  const float* kmaj = nullptr;  // T2, SYRK with alpha = 1: A^T given (k-major, pitch kld): no prep
+  int64_t kld = 0;
 };
 
 template <int MODE, int TM, bool LEAN = false, bool DEEP = false>
@@ -447,12 +450,16 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
 
   // beta * C into the accumulators (pairs along j), while the first stages land
   uint64_t cp[RH][4];
-  const bool cvec = a.cvec;
+  const bool cvec = a.cvec, zinit = a.zinit != 0;
 #pragma unroll
   for (int r = 0; r < RH; ++r) {
     const int64_t gi = i0 + row_of(r);
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
+      if (zinit) {
+        cp[r][2 * h] = cp[r][2 * h + 1] = 0ull;
+        continue;
+      }
       const int64_t gj = j0 + 128 * h + tx * 4;
       float c4[4];
       if (cvec && gi < n && gj + 3 < n) {
@@ -686,11 +693,12 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
       return CATT_ECUDA;
     }
   }
-  const int64_t n = a.ni, m = a.m, ld = (n + 3) / 4 * 4;
+  const bool given = MODE == MODE_SYRK && a.kmaj && a.alpha == 1.0f;  // A^T supplied: no prep, no workspace
+  const int64_t n = a.ni, m = a.m, ld = given ? a.kld : (n + 3) / 4 * 4;
   const bool scale = a.alpha != 1.0f;  // alpha * x == x exactly: (alpha A)^T is A^T
   const int nsrc = MODE == MODE_SYR2K ? 2 : 1;
   const int64_t per = m * ld;          // floats per k-major copy
-  const size_t bytes = size_t(per) * 4 * size_t(nsrc * (scale ? 2 : 1));
+  const size_t bytes = given ? 16 : size_t(per) * 4 * size_t(nsrc * (scale ? 2 : 1));
   // the workspace: stream-ordered, so concurrent launches on other streams get their own
   static std::once_flag pool_once;
   std::call_once(pool_once, [] {
@@ -708,16 +716,16 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     return CATT_ECUDA;
   }
   // copies: A^T, [(alpha A)^T], SYR2K: B^T, [(alpha B)^T]
-  float* At = ws;
+  float* At = given ? const_cast<float*>(a.kmaj) : ws;
   float* aAt = scale ? ws + per : At;
   float* Bt = MODE == MODE_SYR2K ? ws + per * (scale ? 2 : 1) : nullptr;
   float* aBt = MODE == MODE_SYR2K ? (scale ? Bt + per : Bt) : nullptr;
   const dim3 pg(unsigned((n + 31) / 32), unsigned((m + 31) / 32));
-  if (pg.y > 65535) {
+  if (pg.y > 65535 && !given) {
     cudaFreeAsync(ws, s);
     return CATT_EINVAL;
   }
-  t2_prep_kernel<<<pg, 256, 0, s>>>(a.A, At, scale ? aAt : nullptr, n, m, ld, a.alpha);
+  if (!given) t2_prep_kernel<<<pg, 256, 0, s>>>(a.A, At, scale ? aAt : nullptr, n, m, ld, a.alpha);
   if (MODE == MODE_SYR2K) t2_prep_kernel<<<pg, 256, 0, s>>>(a.B, Bt, scale ? aBt : nullptr, n, m, ld, a.alpha);
   // stage arrays, row side then column side: SYRK {(alpha A)^T} {A^T};
   // SYR2K {(alpha A)^T, (alpha B)^T} {B^T, A^T}
@@ -943,6 +951,31 @@ __global__ void __launch_bounds__(1024, 2) gemm_thread_kernel(GemmArgs a) {
 // too. The caller mirrors the rest (CORR).
 catt_status syrk_upper(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta, cudaStream_t s) {
   return launch_tiled<MODE_SYRK>(TileArgs{A, nullptr, C, n, n, m, alpha, beta, 0, 0, 0, 1, {}}, nullptr, s);
+}
+
+// CORR's symmat = D^T D over the upper tiles straight from the centred data
+// D (nrows x mcols, row-major, pitch mcols): D is already the k-major operand
+// of the SYRK over D's columns, so T2 runs without its prep copy, and the
+// accumulators start at +0 without reading C (the literal loop's s = 0;
+// C need not be initialised). Falls back to syrk_upper's path when T2 cannot
+// take D directly (TMA: 16-byte aligned rows).
+bool syrk_kmajor_ok(const float* D, int64_t mcols) {
+  TileArgs a{D, nullptr, nullptr, mcols, mcols, 1, 1.0f, 0.0f, 0, 0, 0, 1, {}};
+  return (reinterpret_cast<uintptr_t>(D) & 15) == 0 && mcols % 4 == 0 && !small_tiles<MODE_SYRK>(mcols, mcols) &&
+         t2_ok<MODE_SYRK>(a);
+}
+
+catt_status syrk_upper_kmajor(const float* D, const float* Dt, float* C, int64_t mcols, int64_t nrows, cudaStream_t s) {
+  TileArgs a{Dt, nullptr, C, mcols, mcols, nrows, 1.0f, 0.0f, 0, 0, 0, 1, {}};
+  if (syrk_kmajor_ok(D, mcols) && nrows > 0) {
+    a.kmaj = D;
+    a.kld = mcols;
+    a.zinit = 1;
+    return launch_t2<MODE_SYRK, 8>(a, nullptr, s);
+  }
+  if (!Dt) return CATT_EINVAL;                 // the transposed operand is needed off the T2 path
+  if (cudaMemsetAsync(C, 0, size_t(mcols) * size_t(mcols) * 4, s) != cudaSuccess) return after_launch();
+  return launch_tiled<MODE_SYRK>(a, nullptr, s);
 }
 
 const void* gemm_func(int variant) {

@@ -113,7 +113,10 @@ def peer_setup_symmetric(n, group=None):
     h = symm.rendezvous(buf, group if group is not None else dist.group.WORLD)
     torch.cuda.synchronize()
     h.barrier()
-    mc = int(h.multicast_ptr) if getattr(h, "has_multicast_support", lambda: False)() else 0
+    try:                                  # 0 where the device or driver offers no NVLS multicast
+        mc = int(h.multicast_ptr or 0)
+    except (RuntimeError, AttributeError):
+        mc = 0
     return catt.Peer.mapped(world, rank, n, [int(p) for p in h.buffer_ptrs], mc, keep=(buf, h))
 
 

@@ -344,6 +344,21 @@ def test_corr_exact(variant, n, m):
     assert bits_equal(host(sym), sym_o)
 
 
+@pytest.mark.parametrize("n,m", [(37, 1604), (20, 1601), (300, 1664)])
+def test_corr_staged_direct_and_transposed_forms(n, m):
+    """STAGED CORR at sizes where the tiled SYRK is T2: m % 4 == 0 takes the
+    direct form (column-strip statistics in place, T2 straight from the
+    centred data; 1604 leaves a ragged 4-column strip), m = 1601 the
+    transposed form. Bit-exact to the oracle, a constant column included."""
+    data = si.matrix(24, n, m)
+    data[:, 5] = 0.25
+    sym_o, mean_o, std_o, d_o = oracle.corr(data)
+    D = dev(data)
+    sym, mean, std = catt.corr(D, t=catt.Throttle(variant="staged"))
+    assert bits_equal(host(D), d_o) and bits_equal(host(mean), mean_o) and bits_equal(host(std), std_o)
+    assert bits_equal(host(sym), sym_o)
+
+
 def test_corr_2048_full_size():
     """Table 2 P:81 size (2K x 2K), both variants, and a throttled literal run."""
     n = m = 2048

@@ -340,10 +340,14 @@ def test_peer_mapped_buffer_equals_grouped_launch():
                 assert np.array_equal(a["yr"].cpu().numpy(), b["yr"].cpu().numpy())
                 assert np.array_equal(a["yc"].cpu().numpy(), b["yc"].cpu().numpy())
         assert not peer.timed_out()
-        with pytest.raises(catt.CattError):                  # no IPC handles to open on a mapped peer
-            peer.open(0, bytes(catt.PEER_HANDLE_BYTES))
     finally:
         peer.close()
+    p2 = catt.Peer.mapped(2, 0, 2 * n, [buf.data_ptr(), buf.data_ptr()], 0, keep=buf)
+    try:
+        with pytest.raises(catt.CattError):                  # no IPC handles to open on a mapped peer
+            p2.open(1, bytes(catt.PEER_HANDLE_BYTES))
+    finally:
+        p2.close()
     with pytest.raises(catt.CattError):                      # misaligned base
         catt.Peer.mapped(1, 0, 2 * n, [buf.data_ptr() + 4], 0)
     assert catt.Peer.nbytes(0, n) < 0 and catt.Peer.nbytes(1, 0) < 0

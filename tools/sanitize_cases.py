@@ -218,9 +218,12 @@ def case_tiles2():
     C = T(C0)
     catt.syr2k(T(A[:n2]), T(B[:n2]), C, 1.5, 1.25, t=catt.Throttle(variant="staged"))
     eq(C, oracle.syr2k(A[:n2], B[:n2], C0, 1.5, 1.25), "syr2k T2")
-    data = si.matrix(12, 24, n)                       # n columns: the upper tiles through T2
+    data = si.matrix(12, 24, n)                       # n columns: the upper tiles through T2 (transposed form)
     sym = catt.corr(T(data), t=catt.Throttle(variant="staged"))[0]
     eq(sym, oracle.corr(data)[0], "corr T2")
+    data = si.matrix(13, 300, 1604)                   # m % 4 == 0: strip statistics (TMA boxes) + T2 on the data
+    sym = catt.corr(T(data), t=catt.Throttle(variant="staged"))[0]
+    eq(sym, oracle.corr(data)[0], "corr direct")
 
 
 def case_peer():
