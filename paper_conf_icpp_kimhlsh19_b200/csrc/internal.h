@@ -46,6 +46,10 @@ catt_status syrk_upper(const float* A, float* C, int64_t n, int64_t m, float alp
 // mcols) the centred data and Dt = D^T (mcols x nrows) its transpose (only
 // read when syrk_kmajor_ok(D, mcols) is false; may be null otherwise).
 bool syrk_kmajor_ok(const float* D, int64_t mcols);
-catt_status syrk_upper_kmajor(const float* D, const float* Dt, float* C, int64_t mcols, int64_t nrows, cudaStream_t s);
+// mirror_diag (T2 path only): the kernel also writes the lower triangle and
+// a unit diagonal (CORR's symmat in one pass); the caller checks
+// syrk_kmajor_ok first and otherwise mirrors itself.
+catt_status syrk_upper_kmajor(const float* D, const float* Dt, float* C, int64_t mcols, int64_t nrows, cudaStream_t s,
+                              bool mirror_diag = false);
 
 }  // namespace catt

@@ -358,12 +358,8 @@ extern "C" catt_status catt_corr(float* data, int64_t n, int64_t m, float* mean,
     corr_stats_strip_kernel<<<dim3(unsigned((m + kStripCols - 1) / kStripCols)), 256, sstrip, s>>>(smap, data, mean, stdv,
                                                                                                   n, m);
     if ((st = after_launch()) != CATT_OK) return st;
-    st = syrk_upper_kmajor(data, nullptr, symmat, m, n, s);
-    if (st != CATT_OK) return st;
-    mirror_lower_kernel<<<dim3(unsigned(gx), unsigned(gx)), 256, 0, s>>>(symmat, m);
-    if ((st = after_launch()) != CATT_OK) return st;
-    corr_diag_kernel<<<dim3(unsigned((m + 255) / 256)), 256, 0, s>>>(symmat, m);
-    return after_launch();
+    // the whole symmat in one launch: upper tiles, their mirror, diagonal 1
+    return syrk_upper_kmajor(data, nullptr, symmat, m, n, s, true);
   }
   // STAGED, transposed form: work = data^T (m x n); statistics and scaling on
   // its rows; data = work^T (the centred data, as LITERAL leaves it); symmat

@@ -118,6 +118,7 @@ struct TileArgs {
   int tri;  // SYRK only: compute the tiles on and above the diagonal (C symmetric; caller mirrors)
   Throttle t;
   int zinit = 0;              // T2: accumulators start at +0 without reading C (CORR's s = 0)
+  int mirror = 0;             // T2, tri: write C[i][j] and C[j][i] for j > i, C[i][i] = 1 (CORR's symmat)
   const float* kmaj = nullptr;  // T2, SYRK with alpha = 1: A^T given (k-major, pitch kld): no prep
   int64_t kld = 0;
 };
@@ -564,6 +565,21 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
       const int64_t gj = j0 + 128 * h + tx * 4;
       const float c0 = f2_lo(cp[r][2 * h]), c1 = f2_hi(cp[r][2 * h]);
       const float c2 = f2_lo(cp[r][2 * h + 1]), c3 = f2_hi(cp[r][2 * h + 1]);
+      if (a.mirror) {
+        // CORR: only the upper elements (j > i) and the unit diagonal here;
+        // the lower triangle below, through shared memory
+        const float cv[4] = {c0, c1, c2, c3};
+        if (gj > gi && gj + 3 < n) {
+          *reinterpret_cast<float4*>(a.C + gi * n + gj) = make_float4(c0, c1, c2, c3);
+        } else {
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const int64_t j = gj + q;
+            if (j < n && j >= gi) a.C[gi * n + j] = j == gi ? 1.0f : cv[q];
+          }
+        }
+        continue;
+      }
       if (cvec && gj + 3 < n) {
         *reinterpret_cast<float4*>(a.C + gi * n + gj) = make_float4(c0, c1, c2, c3);
       } else {
@@ -571,6 +587,34 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
 #pragma unroll
         for (int q = 0; q < 4; ++q)
           if (gj + q < n) a.C[gi * n + gj + q] = cv[q];
+      }
+    }
+  }
+  if (a.mirror) {
+    // the lower triangle: C[j][i] = C[i][j] for j > i, the tile staged
+    // transposed through the (now idle) stage ring so each warp writes whole
+    // 64-float row segments of C^T (coalesced). Every stage was consumed
+    // (each warp waited on it), so after the barrier the ring is free.
+    constexpr int TP = CBX + 1;                  // [8 RH rows][256 cols], odd pitch: row writes and column reads conflict-free
+    static_assert(8 * RH * TP <= NS * Cfg::STAGE_FLOATS, "the staged tile must fit the ring");
+    __syncthreads();
+    float* tt = sm;
+#pragma unroll
+    for (int r = 0; r < RH; ++r)
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const float v = (q & 1) ? f2_hi(cp[r][2 * h + q / 2]) : f2_lo(cp[r][2 * h + q / 2]);
+          tt[row_of(r) * TP + 128 * h + tx * 4 + q] = v;
+        }
+    __syncthreads();
+    for (int c = warp; c < CBX; c += 8) {
+      const int64_t j = j0 + c;
+      if (j >= n) break;
+      for (int r = lane; r < 8 * RH; r += 32) {
+        const int64_t i = i0 + r;
+        if (i < n && j > i) a.C[j * n + i] = tt[r * TP + c];
       }
     }
   }
@@ -612,6 +656,10 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
     fence_barrier_init();
   }
   __syncthreads();
+  // launched as a programmatic dependent of the kernel that wrote the
+  // operands (the prep copies; CORR's statistics): everything above overlapped
+  // its tail; wait for its completion (and memory) before reading A or C
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   t2_tile<MODE, RH>(t2_dyn, full, empty, maps, a, int64_t(Cfg::RB) * rb, int64_t(cs) * Cfg::CB);
   cta_exit(a.t);
 }
@@ -622,6 +670,7 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
 __global__ void __launch_bounds__(256) t2_prep_kernel(const float* __restrict__ X, float* __restrict__ Xt,
                                                       float* __restrict__ aXt, int64_t n, int64_t m, int64_t ld,
                                                       float alpha) {
+  asm volatile("griddepcontrol.launch_dependents;");  // the tile kernel may start its prologue
   __shared__ float tile[32][33];
   const int64_t i0 = int64_t(blockIdx.x) * 32, k0 = int64_t(blockIdx.y) * 32;
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
@@ -752,8 +801,27 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   }
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
   a.cvec = (a.nj % 4 == 0) && al(a.C);
-  tile2_kernel<MODE, RH><<<unsigned(tiles), 256, dyn, s>>>(maps, a, g);
-  const catt_status ls = after_launch();
+  // programmatic dependent launch after the prep copies: the kernel's
+  // prologue overlaps their tail (griddepcontrol.wait inside). Not for the
+  // upper-triangle grid (CORR, one tile per SM): CTAs launched early land two
+  // per SM on the SMs the previous kernel leaves free, which doubled the
+  // makespan (0.216 -> 0.382 ms)
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(unsigned(tiles));
+  cfg.blockDim = dim3(256);
+  cfg.dynamicSmemBytes = dyn;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = a.tri ? 0 : 1;
+  e = cudaLaunchKernelEx(&cfg, tile2_kernel<MODE, RH>, maps, a, g);
+  if (e != cudaSuccess) {
+    record_cuda_error(e);
+    cudaGetLastError();
+  }
+  const catt_status ls = e != cudaSuccess ? CATT_ECUDA : after_launch();
   cudaFreeAsync(ws, s);
   return ls;
 }
@@ -965,12 +1033,14 @@ bool syrk_kmajor_ok(const float* D, int64_t mcols) {
          t2_ok<MODE_SYRK>(a);
 }
 
-catt_status syrk_upper_kmajor(const float* D, const float* Dt, float* C, int64_t mcols, int64_t nrows, cudaStream_t s) {
+catt_status syrk_upper_kmajor(const float* D, const float* Dt, float* C, int64_t mcols, int64_t nrows, cudaStream_t s,
+                              bool mirror_diag) {
   TileArgs a{Dt, nullptr, C, mcols, mcols, nrows, 1.0f, 0.0f, 0, 0, 0, 1, {}};
   if (syrk_kmajor_ok(D, mcols) && nrows > 0) {
     a.kmaj = D;
     a.kld = mcols;
     a.zinit = 1;
+    a.mirror = mirror_diag ? 1 : 0;
     return launch_t2<MODE_SYRK, 8>(a, nullptr, s);
   }
   if (!Dt) return CATT_EINVAL;                 // the transposed operand is needed off the T2 path
