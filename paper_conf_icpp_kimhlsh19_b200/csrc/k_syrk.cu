@@ -410,15 +410,20 @@ struct T2Maps {
 
 struct T2Geo {
   int cs;            // column strips of 256
-  int rbs;           // row blocks of 8 * RH rows
-  int tri;           // compute only tiles reaching the diagonal or above
+  int rbs;           // tri: row blocks of 8 * RH rows
+  int tri;           // compute only tiles reaching the diagonal or above (8 warps per tile)
+  int q;             // otherwise: CTAs per strip, each 8-row warp units of the strip's rows:
+  int uw, ux;        // uw units each, the first ux CTAs one more (<= 8: one unit per warp)
 };
 
-// One (8 RH) x 256 tile, RH rows per thread: rows {32 g + 4 ty + r} for the
-// G = RH / 4 full groups, then {32 G + (RH % 4) ty + r} (ty = warp).
+// One (RH W) x 256 tile computed by its first W warps (W <= 8), RH rows per
+// thread: rows {4 W g + 4 ty + r} for the G = RH / 4 full groups, then
+// {4 W G + (RH % 4) ty + r} (ty = warp). Fewer active warps make a shorter
+// tile at the same 8 x 8 outputs (and shared-memory cost) per thread, which
+// is how the grid balances the SMs' work (launch_t2).
 template <int MODE, int RH>
 __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* empty, const T2Maps& maps,
-                                        const TileArgs& a, int64_t i0, int64_t j0) {
+                                        const TileArgs& a, int64_t i0, int64_t j0, int W) {
   constexpr bool TWO = MODE == MODE_SYR2K;
   using Cfg = T2Cfg<MODE, RH>;
   constexpr int BK = Cfg::BK, NP = Cfg::NP, NS = Cfg::NS, RBX = Cfg::RB, CBX = Cfg::CB;
@@ -432,7 +437,8 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
   const int ty = warp, tx = lane;
   const int64_t n = a.ni, m = a.m;
   const int64_t ktiles = (m + BK - 1) / BK;
-  auto row_of = [&](int r) { return r < 4 * G ? 32 * (r / 4) + 4 * ty + (r % 4) : 32 * G + RR * ty + (r - 4 * G); };
+  const int gs = 4 * W;  // row group stride
+  auto row_of = [&](int r) { return r < 4 * G ? gs * (r / 4) + 4 * ty + (r % 4) : gs * G + RR * ty + (r - 4 * G); };
 
   // row-side stage arrays: alpha*a[i][k] (SYR2K: then alpha*b[i][k]); column-side: a[j][k]
   // (SYR2K: b[j][k], then a[j][k]); maps in the same order
@@ -448,6 +454,7 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
   };
   if (tid == 0)
     for (int64_t kt = 0; kt < NS && kt < ktiles; ++kt) tma(kt);
+  if (warp >= W) return;  // an idle warp of a short tile (not with a.mirror: W == 8 there)
 
   // beta * C into the accumulators (pairs along j), while the first stages land
   uint64_t cp[RH][4];
@@ -482,15 +489,15 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
       const float* rp = rowp(slot, s, kk);
 #pragma unroll
       for (int g = 0; g < G; ++g) {
-        const float4 v = *reinterpret_cast<const float4*>(rp + 32 * g + ty * 4);
+        const float4 v = *reinterpret_cast<const float4*>(rp + gs * g + ty * 4);
         fr[fb][s][4 * g] = v.x, fr[fb][s][4 * g + 1] = v.y, fr[fb][s][4 * g + 2] = v.z, fr[fb][s][4 * g + 3] = v.w;
       }
       if constexpr (RR == 2) {
-        const float2 v = *reinterpret_cast<const float2*>(rp + 32 * G + ty * 2);
+        const float2 v = *reinterpret_cast<const float2*>(rp + gs * G + ty * 2);
         fr[fb][s][4 * G] = v.x, fr[fb][s][4 * G + 1] = v.y;
       } else {
 #pragma unroll
-        for (int q = 0; q < RR; ++q) fr[fb][s][4 * G + q] = rp[32 * G + RR * ty + q];
+        for (int q = 0; q < RR; ++q) fr[fb][s][4 * G + q] = rp[gs * G + RR * ty + q];
       }
       const float* cq = colp(slot, s, kk);
 #pragma unroll
@@ -629,11 +636,12 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
   extern __shared__ __align__(128) float t2_dyn[];
   uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
   uint64_t* empty = full + NS;
-  // the tile (tri: the tiles that reach the diagonal, by row block)
-  int rb, cs;
+  // the tile. tri: the 8-warp tiles that reach the diagonal, by row block;
+  // otherwise CTA k of strip cs owns warp units [k uw + min(k, ux), +W)
+  int cs, W;
+  int64_t i0;
   if (g.tri) {
-    int rem = int(blockIdx.x);
-    rb = 0;
+    int rem = int(blockIdx.x), rb = 0;
     while (true) {
       const int lo = int((int64_t(Cfg::RB) * rb) / 256);  // first strip with an element j >= i
       if (rem < g.cs - lo) {
@@ -643,15 +651,19 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
       rem -= g.cs - lo;
       ++rb;
     }
+    W = 8;
+    i0 = int64_t(Cfg::RB) * rb;
   } else {
-    rb = int(blockIdx.x) / g.cs;
-    cs = int(blockIdx.x) % g.cs;
+    cs = int(blockIdx.x) / g.q;
+    const int k = int(blockIdx.x) % g.q;
+    W = g.uw + (k < g.ux ? 1 : 0);
+    i0 = int64_t(RH) * (int64_t(k) * g.uw + min(k, g.ux));
   }
   cta_enter(a.t);
   if (threadIdx.x == 0) {
     for (int s = 0; s < NS; ++s) {
       bar_init(&full[s], 1);
-      bar_init(&empty[s], 8);
+      bar_init(&empty[s], unsigned(W));
     }
     fence_barrier_init();
   }
@@ -660,7 +672,7 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
   // operands (the prep copies; CORR's statistics): everything above overlapped
   // its tail; wait for its completion (and memory) before reading A or C
   asm volatile("griddepcontrol.wait;" ::: "memory");
-  t2_tile<MODE, RH>(t2_dyn, full, empty, maps, a, int64_t(Cfg::RB) * rb, int64_t(cs) * Cfg::CB);
+  t2_tile<MODE, RH>(t2_dyn, full, empty, maps, a, i0, int64_t(cs) * Cfg::CB, W);
   cta_exit(a.t);
 }
 
@@ -715,6 +727,31 @@ static bool t2_map(CUtensorMap* mp, const float* base, int64_t n, int64_t m, int
 template <int MODE>
 static bool t2_ok(const TileArgs& a) {
   return tiled_t2() && a.m > 0 && a.m < (int64_t(1) << 31) && a.ni < (int64_t(1) << 31);
+}
+
+// Tiles for an n x n output. tri: 8-warp tiles of 8 RH rows. Otherwise each
+// 256-column strip's rows are dealt as 8-row warp units to q CTAs, q chosen
+// so that the grid fills the 2 x #SM CTA slots (one wave) with at most 8
+// units per CTA: 2048 on 148 SMs gives 37 CTAs per strip of 7 or 6 units
+// (56 or 48 rows), so the busiest SM has 14 units of work where 64-row
+// tiles gave it 16 (256 tiles in 296 slots).
+static T2Geo t2_geometry(int64_t n, bool tri, int rh) {
+  static const int nsm = [] {
+    int d = 0, v = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    return v;
+  }();
+  T2Geo g{};
+  g.cs = int((n + 255) / 256);
+  g.tri = tri ? 1 : 0;
+  g.rbs = int((n + 8 * rh - 1) / (8 * rh));
+  const int64_t units = (n + rh - 1) / rh;                  // warp units of rh rows
+  const int64_t per_strip = std::max<int64_t>(1, (2 * int64_t(nsm)) / g.cs);
+  const int64_t q = std::max((units + 7) / 8, std::min(units, per_strip));
+  g.q = int(q);
+  g.uw = int(units / q);
+  g.ux = int(units % q);
+  return g;
 }
 
 static int64_t t2_tiles(const T2Geo& g, int rb_rows) {
@@ -793,8 +830,8 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     cudaFreeAsync(ws, s);
     return CATT_ECUDA;
   }
-  const T2Geo g{int((n + 255) / 256), int((n + Cfg::RB - 1) / Cfg::RB), a.tri ? 1 : 0};
-  const int64_t tiles = t2_tiles(g, Cfg::RB);
+  const T2Geo g = t2_geometry(n, a.tri != 0, RH);
+  const int64_t tiles = a.tri ? t2_tiles(g, Cfg::RB) : int64_t(g.cs) * g.q;
   if (tiles > (int64_t(1) << 31) - 1) {
     cudaFreeAsync(ws, s);
     return CATT_EINVAL;
