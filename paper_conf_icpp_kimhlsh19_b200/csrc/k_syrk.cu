@@ -404,6 +404,10 @@ struct T2Cfg {
   static constexpr size_t SBYTES = size_t(NS) * STAGE_FLOATS * 4 + 2 * NS * 8;
 };
 
+#ifndef T2_PAIR_OUTER
+#define T2_PAIR_OUTER 1
+#endif
+
 struct T2Maps {
   CUtensorMap m[4];  // per stage array (row-side first): the k-major operand it is loaded from
 };
@@ -508,6 +512,32 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
     }
   };
   auto fma_step = [&](int fb) {
+    // column pair outer: its two registers stay in the operand reuse cache
+    // across the RH instructions that use them (SYRK 0.359 -> 0.348 ms)
+    if constexpr (!TWO && T2_PAIR_OUTER) {
+#pragma unroll
+      for (int p = 0; p < 4; ++p) {
+        const uint64_t bq = f2_pack(fc[fb][0][2 * p], fc[fb][0][2 * p + 1]);
+#pragma unroll
+        for (int r = 0; r < RH; ++r) f2_fma_acc(cp[r][p], f2_pack(fr[fb][0][r], fr[fb][0][r]), bq);
+      }
+      return;
+    }
+    if constexpr (TWO && T2_PAIR_OUTER) {  // SYR2K: the same, each op kind grouped over r
+#pragma unroll
+      for (int p = 0; p < 4; ++p) {
+        const uint64_t bq = f2_pack(fc[fb][0][2 * p], fc[fb][0][2 * p + 1]);
+        const uint64_t aq = f2_pack(fc[fb][1][2 * p], fc[fb][1][2 * p + 1]);
+        uint64_t pr[RH];
+#pragma unroll
+        for (int r = 0; r < RH; ++r) pr[r] = f2_mul(f2_pack(fr[fb][1][r], fr[fb][1][r]), aq);
+#pragma unroll
+        for (int r = 0; r < RH; ++r) pr[r] = f2_fma(f2_pack(fr[fb][0][r], fr[fb][0][r]), bq, pr[r]);
+#pragma unroll
+        for (int r = 0; r < RH; ++r) f2_add_acc(cp[r][p], pr[r]);
+      }
+      return;
+    }
 #pragma unroll
     for (int r = 0; r < RH; ++r) {
       const uint64_t ar = f2_pack(fr[fb][0][r], fr[fb][0][r]);
