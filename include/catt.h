@@ -304,7 +304,13 @@ catt_status catt_gesummv(const float* A, const float* B, const float* x, float* 
 
 /* SYRK (Table 2): C = beta*C + alpha*A*A^T over the full n x n square.
  * A is n x m; C in/out. LITERAL = 2-D block 32 x (cta_threads/32), one thread
- * per C element; STAGED = shared-memory tiles, register blocking, same k order. */
+ * per C element; STAGED = shared-memory tiles, register blocking, same k order.
+ * STAGED with at least one tile per SM (T2) first writes A^T
+ * and (alpha*A)^T (one copy when alpha == 1) into a workspace taken from the
+ * device's default memory pool, stream-ordered on `stream` (cudaMallocAsync,
+ * released by cudaFreeAsync after the launch; the pool keeps it for reuse):
+ * 2*n*m floats. If that allocation fails the library runs its round-1 tiled
+ * kernel instead, which needs no workspace (same results, slower). */
 catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alpha, float beta,
                       const catt_throttle* t, void* stream);
 
@@ -313,7 +319,8 @@ catt_status catt_syrk(const float* A, float* C, int64_t n, int64_t m, float alph
  * C in/out. Per element, k ascending: p = alpha*a_ik, q = alpha*b_ik,
  * s = fmaf(p, b_jk, q*a_jk), c = c + s (every intermediate rounded; DESIGN.md
  * R20). LITERAL = 2-D block 32 x (cta_threads/32); STAGED = shared-memory
- * tiles with the same order. */
+ * tiles with the same order; its workspace as catt_syrk's with B too:
+ * 4*n*m floats (2*n*m when alpha == 1). */
 catt_status catt_syr2k(const float* A, const float* B, float* C, int64_t n, int64_t m, float alpha, float beta,
                        const catt_throttle* t, void* stream);
 

@@ -828,8 +828,8 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   float* ws = nullptr;
   e = cudaMallocAsync(reinterpret_cast<void**>(&ws), bytes, s);
   if (e != cudaSuccess) {
-    record_cuda_error(e);
-    return CATT_ECUDA;
+    cudaGetLastError();                // not sticky: the caller falls back to tiled_kernel
+    return e == cudaErrorMemoryAllocation ? CATT_ENOMEM : (record_cuda_error(e), CATT_ECUDA);
   }
   // copies: A^T, [(alpha A)^T], SYR2K: B^T, [(alpha B)^T]
   float* At = given ? const_cast<float*>(a.kmaj) : ws;
@@ -964,7 +964,10 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
   if (t && t->cta_threads != 0 && t->cta_threads != 256) return CATT_EINVAL;
   const bool small = small_tiles<MODE>(a.ni, a.nj);
   if constexpr (MODE != MODE_GEMM)
-    if (!small && t2_ok<MODE>(a)) return launch_t2<MODE, 8>(a, t, s);
+    if (!small && t2_ok<MODE>(a)) {
+      const catt_status st = launch_t2<MODE, 8>(a, t, s);
+      if (st != CATT_ENOMEM) return st;  // no room for the k-major copies: the round-1 kernel below
+    }
   constexpr int TMs = MODE == MODE_SYR2K ? 8 : 4;  // SYR2K never takes the small tile (static_assert)
   const int64_t tt = (a.ni + 127) / 128;
   const bool lean = !small && MODE == MODE_SYRK && tiled_lean(a.tri ? tt * (tt + 1) / 2 : tt * tt);
