@@ -384,6 +384,12 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 // 256 tiles, 1.73 per SM) measured the same 0.367 ms: the 48-row tile's 6 x 8
 // outputs per thread need as many column reads for 3/4 of the FMAs and the
 // SM's shared-memory pipe becomes the limit, so it was not kept.
+#ifndef T2_NS
+#define T2_NS 4
+#endif
+#ifndef T2_BK
+#define T2_BK 16
+#endif
 // RH rows per thread: 8 (64-row tiles, two CTAs per SM, <= 128 registers).
 // The template also builds RH = 15 (120-row tiles, one CTA per SM, 222
 // registers: 15 x 8 outputs per thread cut the shared-memory wavefronts per
@@ -394,9 +400,9 @@ template <int MODE, int RH = 8>
 struct T2Cfg {
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int NP = NA / 2;                               // row-side (and column-side) arrays
-  static constexpr int BK = MODE == MODE_SYR2K ? 8 : 16;
+  static constexpr int BK = MODE == MODE_SYR2K ? 8 : T2_BK;
   static constexpr int MINB = RH > 8 ? 1 : 2;                    // CTAs per SM
-  static constexpr int NS = RH > 8 ? 6 : 4;                      // ring stages
+  static constexpr int NS = RH > 8 ? 6 : T2_NS;                  // ring stages
   static constexpr int RB = 8 * RH, CB = 256;                    // row box, column strip
   static constexpr int ROW_FLOATS = BK * RB, COL_FLOATS = BK * CB;
   static constexpr int STAGE_FLOATS = NP * (ROW_FLOATS + COL_FLOATS);
@@ -627,7 +633,7 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
       }
     }
   }
-  if (a.mirror) {
+  if constexpr (MODE == MODE_SYRK) if (a.mirror) {
     // the lower triangle: C[j][i] = C[i][j] for j > i, the tile staged
     // transposed through the (now idle) stage ring so each warp writes whole
     // 64-float row segments of C^T (coalesced). Every stage was consumed
