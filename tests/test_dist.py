@@ -9,7 +9,6 @@ GPU (1 device): the same functions through the CUDA kernels with a
 single-rank NCCL group.
 """
 import os
-import socket
 
 import numpy as np
 import pytest
@@ -116,16 +115,18 @@ class OracleKmeansOps:
 
 
 def _free_port():
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
-    return port
+    """A fresh rendezvous file for init_method="file://..." (a TCP port picked
+    here could be taken by another process before the ranks bind it)."""
+    import tempfile
+    return os.path.join(tempfile.mkdtemp(prefix="catt_pg_"), "store")
+
+
+def _init(store):
+    return "file://" + store
 
 
 def _worker(rank, world, port, mode, q):
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     try:
         m, n = 301, 96                                  # ragged: 151 + 150 rows
         A = si.matrix(7, m, n, mode=mode)
@@ -189,8 +190,7 @@ def test_rowshard_world2_gloo(mode):
 
 
 def _km_worker(rank, world, port, q):
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     try:
         npts, nf, k = 301, 6, 3
         feat = si.values(21, nf * npts)                  # uniform, feature-major, ld = npts
@@ -239,8 +239,7 @@ def test_row_range_partitions():
 @pytest.mark.gpu
 def test_rowshard_single_rank_nccl():
     """The product path (CUDA kernels + NCCL) on a one-rank group."""
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(_free_port()))
-    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    dist.init_process_group("nccl", init_method=_init(_free_port()), rank=0, world_size=1, device_id=torch.device("cuda", 0))
     try:
         m, n = 1000, 256
         A = si.matrix(7, m, n, mode=si.MODE_DYADIC)
@@ -276,8 +275,7 @@ class _FakePeer:
 
 
 def _peer_worker(rank, world, port, q):
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     try:
         orig = catt_mod.Peer
         catt_mod.Peer = _FakePeer
@@ -315,9 +313,8 @@ def _cuda_worker(rank, world, port, mode, q):
     (CudaOps, libcatt.so) in world processes that share cuda:0, with gloo
     collectives on the CUDA tensors (NCCL needs one GPU per rank; this run
     has one GPU)."""
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     torch.cuda.set_device(0)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     try:
         C = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
         H = lambda t: (torch.cuda.synchronize(), t.cpu().numpy())[1]

@@ -9,7 +9,6 @@ parities), equal bit for bit to the rank-order fp32 sum of the per-rank
 partials that the plain fused kernel computes, and within the 1e-5 bar of the
 fp64 oracle (ATAX's A^T tmp is not exact in fp32 even on dyadic inputs)."""
 import os
-import socket
 import sys
 
 import numpy as np
@@ -28,11 +27,14 @@ def _relerr(got, want):
 
 
 def _free_port():
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
-    return port
+    """A fresh rendezvous file for init_method="file://..." (a TCP port picked
+    here could be taken by another process before the ranks bind it)."""
+    import tempfile
+    return os.path.join(tempfile.mkdtemp(prefix="catt_pg_"), "store")
+
+
+def _init(store):
+    return "file://" + store
 
 
 def _problem(m, n, mode):
@@ -44,8 +46,7 @@ def _problem(m, n, mode):
 def _rank_main(rank, world, port, m, n, steps, out_dir):
     import torch
     import torch.distributed as dist
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     torch.cuda.set_device(0)
     from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
     import paper_conf_icpp_kimhlsh19_b200 as catt
@@ -154,8 +155,7 @@ def _bm_group(torch, A, B, p, r, y1, y2, x1, x2, lo, hi, acc=True):
 def _bm_rank_main(rank, world, port, m, n, steps, out_dir):
     import torch
     import torch.distributed as dist
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     torch.cuda.set_device(0)
     from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
     import paper_conf_icpp_kimhlsh19_b200 as catt
@@ -253,8 +253,7 @@ def test_bicg_mvt_peer_processes_share_one_gpu(tmp_path, world, m, n):
 def _uneven_rank_main(rank, world, port, rows, n, out_dir):
     import torch
     import torch.distributed as dist
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=_init(port), rank=rank, world_size=world)
     torch.cuda.set_device(0)
     from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
     m = sum(rows)
@@ -356,9 +355,8 @@ def test_peer_mapped_buffer_equals_grouped_launch():
 def _symm_worker(port, m, n, q):
     import torch
     import torch.distributed as dist
-    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     torch.cuda.set_device(0)
-    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    dist.init_process_group("nccl", init_method=_init(port), rank=0, world_size=1, device_id=torch.device("cuda", 0))
     try:
         from paper_conf_icpp_kimhlsh19_b200 import dist as cdist
         import paper_conf_icpp_kimhlsh19_b200 as catt
