@@ -145,6 +145,7 @@ class Workload:
     name = ""
     desc = ""
     variant = "coop"
+    scaling = "weak"          # every rank's work is fixed as N grows (the JSON line's "scaling")
 
     def __init__(self, catt, torch, rank, world, variant):
         self.catt, self.torch, self.rank, self.world = catt, torch, rank, world
@@ -591,6 +592,7 @@ class Atax(Workload):
         super().__init__(catt, torch, rank, world, variant)
         import seeded_inputs as si
         rows = m // world if m >= 1024 else m          # configs[4]: the global matrix is split across ranks
+        self.scaling = "strong" if m >= 1024 else "weak"  # the 65536 x 16384 total is fixed as N grows
         self.m, self.n, self.rows = m, n, rows
         dev = torch.device("cuda")
         seed = si.SEED_ATAX_SHARDED if m >= 1024 else si.SEED_ATAX
@@ -1065,7 +1067,8 @@ def run_reference(args):
     gbs = nbytes / (ms * 1e-3) / 1e9
     cores = oracle.num_threads()
     line = {"metric": METRIC, "value": round(gbs, 3), "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
+            "scaling": "strong" if args.workload == "atax" else "weak",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded counter hash)",
             "config": {"workload": cfg, "l2": "n/a (CPU)"}, "impl": "reference",
             "cpu_baseline": {"value": round(gbs, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
@@ -1308,7 +1311,7 @@ def main():
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": w.scaling,
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded counter hash, generated on device)",
             "config": {"workload": w.desc, "variant": w.variant, "l2": "flushed before every step (256 MiB write, then 256 MiB clean read)", "flush_order": args.flush_order,
                        "rows_per_rank": getattr(w, "rows", None), "parallelism": f"row-shard x{world}"},
