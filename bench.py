@@ -1194,7 +1194,7 @@ def main():
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
 
     study = app = kst = l1 = None
-    if rank == 0 and not args.no_study:
+    if rank == 0 and world == 1 and not args.no_study:   # N > 1 (SCALE runs): the studies are per-GPU, done at N = 1
         study = throttle_study(catt, torch, w, flush)
         app = app_study(catt, torch, w, flush)
         kst = kernel_study(catt, torch, w, flush)
