@@ -193,7 +193,7 @@ __global__ void __launch_bounds__(kStatWarps * 32) corr_stats_rows_kernel(float*
 // batch ahead of the adds), and the whole CTA writes the centred and scaled
 // strip back in place. No transposes: the centred data is then the k-major
 // operand of the SYRK (syrk_upper_kmajor).
-constexpr int kStripCols = 16, kStripBox = 256, kStripMaxBoxes = 16;
+constexpr int kStripCols = 8, kStripBox = 256, kStripMaxBoxes = 16;  // 8 columns: 25 us at 2048 (16: 28, 4: 31)
 __global__ void __launch_bounds__(256) corr_stats_strip_kernel(const __grid_constant__ CUtensorMap map, float* data,
                                                                float* mean, float* stdv, int64_t n, int64_t m) {
   extern __shared__ __align__(128) float s_strip[];  // [n rounded to boxes][kStripCols]
@@ -261,9 +261,10 @@ __global__ void __launch_bounds__(256) corr_stats_strip_kernel(const __grid_cons
   __syncthreads();
   // write-back: float4 of 4 columns per thread (m % 4 == 0 on this path)
   const int q4 = (nc + 3) / 4;
-  for (int64_t e = t; e < n * 4; e += 256) {
-    const int64_t i = e / 4;
-    const int c4 = int(e % 4);
+  constexpr int R4 = kStripCols / 4;  // float4 per strip row
+  for (int64_t e = t; e < n * R4; e += 256) {
+    const int64_t i = e / R4;
+    const int c4 = int(e % R4);
     if (c4 < q4) {
       const float4 v = *reinterpret_cast<const float4*>(s_strip + i * kStripCols + 4 * c4);
       float4 o;
