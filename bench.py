@@ -38,6 +38,9 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "kernel runtime & L1 hit rate: CATT throttle vs full-TLP vs best swept, HBM GB/s"
+# FP32 FMA throughput measured on this pool's B200 (tools/ffma_probe.cu, 1965 MHz):
+# the ALU roofline reports its fraction beside the derived 148 x 128 x 2 x clock peak
+FP32_MEASURED_TFLOPS = 72.3
 FALLBACK_HBM_GBS = 6650.0
 
 
@@ -1212,7 +1215,11 @@ def main():
         ach = w.flops / (loop_ms[dom] * 1e-3) / 1e12
         roof = {"bound": "alu", "kernel": lp.name, "achieved": round(ach, 3), "peak": round(peak_t, 3),
                 "unit": "TFLOP/s", "frac": round(ach / peak_t, 4), "traffic": ncu_traffic(w.name) if w.variant == type(w).variant else None,
-                "peak_source": f"derived: 148 SM x 128 FP32 lanes x 2 x {clk_mhz:.0f} MHz (median under load)"}
+                "peak_source": f"derived: 148 SM x 128 FP32 lanes x 2 x {clk_mhz:.0f} MHz (median under load)",
+                # the highest FP32 FMA rate measured on this pool's B200 (tools/ffma_probe.cu:
+                # independent FFMA chains, 512-thread CTAs, 1965 MHz; profiles/r2/tiles/ffma_probe.txt)
+                "measured_peak": FP32_MEASURED_TFLOPS, "frac_of_measured": round(ach / FP32_MEASURED_TFLOPS, 4),
+                "measured_peak_source": "tools/ffma_probe.cu, profiles/r2/tiles/ffma_probe.txt"}
     else:
         ach = lp.nbytes / (loop_ms[dom] * 1e-3) / 1e9
         roof = {"bound": "hbm", "kernel": lp.name, "achieved": round(ach, 2), "peak": peak, "unit": "GB/s",
