@@ -820,7 +820,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   const bool scale = a.alpha != 1.0f;  // alpha * x == x exactly: (alpha A)^T is A^T
   const int nsrc = MODE == MODE_SYR2K ? 2 : 1;
   const int64_t per = m * ld;          // floats per k-major copy
-  const size_t bytes = given ? 16 : size_t(per) * 4 * size_t(nsrc * (scale ? 2 : 1));
+  const size_t bytes = size_t(per) * 4 * size_t(nsrc * (scale ? 2 : 1));
   // the workspace: stream-ordered, so concurrent launches on other streams get their own
   static std::once_flag pool_once;
   std::call_once(pool_once, [] {
@@ -832,7 +832,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     }
   });
   float* ws = nullptr;
-  e = cudaMallocAsync(reinterpret_cast<void**>(&ws), bytes, s);
+  e = given ? cudaSuccess : cudaMallocAsync(reinterpret_cast<void**>(&ws), bytes, s);  // nothing to copy when A^T is given
   if (e != cudaSuccess) {
     cudaGetLastError();                // not sticky: the caller falls back to tiled_kernel
     return e == cudaErrorMemoryAllocation ? CATT_ENOMEM : (record_cuda_error(e), CATT_ECUDA);
@@ -844,7 +844,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   float* aBt = MODE == MODE_SYR2K ? (scale ? Bt + per : Bt) : nullptr;
   const dim3 pg(unsigned((n + 31) / 32), unsigned((m + 31) / 32));
   if (pg.y > 65535 && !given) {
-    cudaFreeAsync(ws, s);
+    if (ws) cudaFreeAsync(ws, s);
     return CATT_EINVAL;
   }
   if (!given) t2_prep_kernel<<<pg, 256, 0, s>>>(a.A, At, scale ? aAt : nullptr, n, m, ld, a.alpha);
@@ -863,13 +863,13 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   for (int q = 0; q < Cfg::NA; ++q)
     ok = ok && t2_map(&maps.m[q], src[q], n, m, ld, q < Cfg::NP ? Cfg::RB : Cfg::CB, Cfg::BK);
   if (!ok) {
-    cudaFreeAsync(ws, s);
+    if (ws) cudaFreeAsync(ws, s);
     return CATT_ECUDA;
   }
   const T2Geo g = t2_geometry(n, a.tri != 0, RH);
   const int64_t tiles = a.tri ? t2_tiles(g, Cfg::RB) : int64_t(g.cs) * g.q;
   if (tiles > (int64_t(1) << 31) - 1) {
-    cudaFreeAsync(ws, s);
+    if (ws) cudaFreeAsync(ws, s);
     return CATT_EINVAL;
   }
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
@@ -895,7 +895,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     cudaGetLastError();
   }
   const catt_status ls = e != cudaSuccess ? CATT_ECUDA : after_launch();
-  cudaFreeAsync(ws, s);
+  if (ws) cudaFreeAsync(ws, s);
   return ls;
 }
 

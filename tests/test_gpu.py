@@ -228,6 +228,22 @@ def test_syrk_staged_large_tiles(n, m, t):
     assert bits_equal(host(Cd), C_o)
 
 
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.5), (1.5, 0.0), (-0.75, 1.0)])
+def test_syrk_syr2k_staged_alpha_beta_forms(alpha, beta):
+    """T2 with alpha == 1 (one k-major copy serves both operands), beta == 0
+    and a negative alpha, SYRK and SYR2K, ragged n and m: bit-exact."""
+    n, m = 1601, 37
+    A, B, C = si.matrix(6, n, m), si.matrix(8, n, m), si.matrix(106, n, n)
+    Cd = dev(C)
+    catt.syrk(dev(A), Cd, alpha, beta, t=catt.Throttle(variant="staged"))
+    assert bits_equal(host(Cd), oracle.syrk(A, C, alpha, beta))
+    n2 = 300
+    C2 = si.matrix(208, n2, n2)
+    Cd = dev(C2)
+    catt.syr2k(dev(A[:n2]), dev(B[:n2]), Cd, alpha, beta, t=catt.Throttle(variant="staged"))
+    assert bits_equal(host(Cd), oracle.syr2k(A[:n2], B[:n2], C2, alpha, beta))
+
+
 def test_syrk_throttled():
     A, C = si.matrix(6, 96, 64), si.matrix(106, 96, 96)
     C_o = oracle.syrk(A, C, 1.5, 1.2)
