@@ -715,10 +715,22 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
 // k-major copies of X (n x m, row-major): Xt[k][i] = X[i][k] and, when aXt is
 // given, aXt[k][i] = alpha * X[i][k] (the literal kernel's rounding). Rows of
 // the copies have pitch ld (a multiple of 4 floats: the TMA stride).
-__global__ void __launch_bounds__(256) t2_prep_kernel(const float* __restrict__ X, float* __restrict__ Xt,
-                                                      float* __restrict__ aXt, int64_t n, int64_t m, int64_t ld,
-                                                      float alpha, int vec) {
+struct PrepSrc {
+  const float* X;   // n x m, row-major
+  float* Xt;        // m x ld: X^T
+  float* aXt;       // m x ld: (alpha X)^T, or null
+  int vec;          // float4 loads of X (m % 4 == 0, 16-byte aligned)
+};
+
+// blockIdx.z selects the matrix (SYR2K copies A and B in one launch)
+__global__ void __launch_bounds__(256) t2_prep_kernel(PrepSrc s0, PrepSrc s1, int64_t n, int64_t m, int64_t ld,
+                                                      float alpha) {
   asm volatile("griddepcontrol.launch_dependents;");  // the tile kernel may start its prologue
+  const PrepSrc& src = blockIdx.z ? s1 : s0;
+  const float* __restrict__ X = src.X;
+  float* __restrict__ Xt = src.Xt;
+  float* __restrict__ aXt = src.aXt;
+  const int vec = src.vec;
   // 64 (i) x 64 (k) tiles; float4 reads along k when vec (m % 4 == 0, X
   // 16-byte aligned), float4 writes along i (ld % 4 == 0). 32 x 32 scalar
   // tiles ran at ~3 TB/s (16 us per 2048^2 matrix).
@@ -877,8 +889,12 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     if (ws) cudaFreeAsync(ws, s);
     return CATT_EINVAL;
   }
-  if (!given) t2_prep_kernel<<<pg, 256, 0, s>>>(a.A, At, scale ? aAt : nullptr, n, m, ld, a.alpha, vecA);
-  if (MODE == MODE_SYR2K) t2_prep_kernel<<<pg, 256, 0, s>>>(a.B, Bt, scale ? aBt : nullptr, n, m, ld, a.alpha, vecB);
+  if (!given) {
+    const PrepSrc pa{a.A, At, scale ? aAt : nullptr, vecA};
+    const PrepSrc pb{a.B, Bt, scale ? aBt : nullptr, vecB};
+    const dim3 pg2(pg.x, pg.y, MODE == MODE_SYR2K ? 2u : 1u);
+    t2_prep_kernel<<<pg2, 256, 0, s>>>(pa, pb, n, m, ld, a.alpha);
+  }
   // stage arrays, row side then column side: SYRK {(alpha A)^T} {A^T};
   // SYR2K {(alpha A)^T, (alpha B)^T} {B^T, A^T}
   T2Maps maps{};
