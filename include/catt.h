@@ -140,13 +140,17 @@ typedef struct {
  * memory-divergent reused loads (each meeting the divergent_lines /
  * min_retouch / min_reuse_trip terms), the floor is ceil(min_warps_sm / S):
  * S streams per warp keep as many lines in flight as S times the warps.
+ * private_streams (R32; 0 = off): a memory-divergent reused load whose first
+ * warp request touches the same lines in warp 1 as in warp 0 of CTA 0 (the
+ * lines are shared by the CTA's warps, e.g. SYRK's a[j][k] in a 32 x 8 block)
+ * counts neither as divergent nor as a stream.
  * Paper mode ignores them. */
 typedef struct {
   int32_t num_sms, max_warps_sm, max_ctas_sm, regs_sm, reg_alloc_unit, warp_size;
   int32_t smem_alloc_unit, reserved_smem_cta, line_bytes, n_carveouts;
   int32_t min_warps_sm, divergent_lines;
   int32_t min_retouch, min_reuse_trip, max_stream_pct, cta_fallback;
-  int32_t stream_floor, reserved_;
+  int32_t stream_floor, private_streams;
   int32_t carveout_kb[CATT_MAX_CARVEOUTS];
   int32_t carveout_pct[CATT_MAX_CARVEOUTS];
   int64_t l1d_bytes[CATT_MAX_CARVEOUTS];
@@ -584,7 +588,8 @@ catt_status catt_dual_group_peer(const catt_dual_problem* probs, int32_t count, 
  * after the grid barrier, end) for CTAs < 1024. Copies the first n of the
  * 6144 u64 values (CTA-major) to host memory `out` (synchronous). */
 catt_status catt_fused_trace(uint64_t* out, int32_t n);
-/* ABI revision of this header: 5 (catt_hw.stream_floor + reserved_,
+/* ABI revision of this header: 6 (catt_hw.reserved_ became private_streams);
+ * 5 (catt_hw.stream_floor + reserved_,
  * CATT_K_ROWS3, CATT_ROWS_SUM3; 4 added catt_kernel_occupancy; 3: catt_hw's
  * last reserved word became cta_fallback; 2 added min_retouch,
  * min_reuse_trip, max_stream_pct). */

@@ -64,13 +64,13 @@ class Hw(ctypes.Structure):
                 ("min_warps_sm", ctypes.c_int32), ("divergent_lines", ctypes.c_int32),
                 ("min_retouch", ctypes.c_int32), ("min_reuse_trip", ctypes.c_int32),
                 ("max_stream_pct", ctypes.c_int32), ("cta_fallback", ctypes.c_int32),
-                ("stream_floor", ctypes.c_int32), ("reserved_", ctypes.c_int32),
+                ("stream_floor", ctypes.c_int32), ("private_streams", ctypes.c_int32),
                 ("carveout_kb", ctypes.c_int32 * MAX_CARVEOUTS), ("carveout_pct", ctypes.c_int32 * MAX_CARVEOUTS),
                 ("l1d_bytes", ctypes.c_int64 * MAX_CARVEOUTS)]
 
     def as_dict(self):
         n = self.n_carveouts
-        d = {f: getattr(self, f) for f, _ in self._fields_[:17]}
+        d = {f: getattr(self, f) for f, _ in self._fields_[:18]}
         d["carveout_kb"] = list(self.carveout_kb[:n])
         d["carveout_pct"] = list(self.carveout_pct[:n])
         d["l1d_bytes"] = list(self.l1d_bytes[:n])
@@ -79,7 +79,7 @@ class Hw(ctypes.Structure):
     @classmethod
     def from_dict(cls, d):
         h = cls()
-        for f, _ in cls._fields_[:17]:
+        for f, _ in cls._fields_[:18]:
             if f in d:
                 setattr(h, f, d[f])
         n = len(d["carveout_kb"])
@@ -247,6 +247,7 @@ def paper_rule(hw: Hw) -> Hw:
     h.max_stream_pct = 0
     h.cta_fallback = 0
     h.stream_floor = 0
+    h.private_streams = 0
     return h
 
 

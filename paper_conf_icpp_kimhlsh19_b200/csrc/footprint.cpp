@@ -239,7 +239,16 @@ class Model {
           retouch = std::max(retouch, per_line);
           rtrip = std::max(rtrip, d_.trip[k]);
         }
-      if (reuse && int64_t(s.size()) >= hw_.divergent_lines && retouch >= hw_.min_retouch &&
+      // R32: a divergent load whose lines every warp of the CTA requests too
+      // (warp 1 touches the same lines as warp 0) is served to the CTA's
+      // warps by one fill: it does not make the loop divergent
+      bool cta_shared = false;
+      if (hw_.private_streams > 0 && o_.W >= 2 && int64_t(s.size()) >= hw_.divergent_lines) {
+        std::unordered_set<uint64_t> s1;
+        add_lines(r, lane_gids(d_, 0, 1, hw_.warp_size), it0, d_.n_loops, line_, &s1);
+        cta_shared = s1 == s;
+      }
+      if (reuse && !cta_shared && int64_t(s.size()) >= hw_.divergent_lines && retouch >= hw_.min_retouch &&
           rtrip >= hw_.min_reuse_trip) {
         divergent_ = true;
         ++streams_;                    // R29: one more memory-divergent reused load
@@ -351,7 +360,7 @@ catt_status validate(const catt_loop_desc* d, const catt_hw* hw) {
   if (hw->line_bytes < 4 || hw->n_carveouts < 1 || hw->n_carveouts > CATT_MAX_CARVEOUTS) return CATT_EINVAL;
   if (hw->smem_alloc_unit < 1 || hw->reg_alloc_unit < 1 || hw->regs_sm < 1) return CATT_EINVAL;
   if (hw->min_warps_sm < 0 || hw->divergent_lines < 0 || hw->min_retouch < 0 || hw->min_reuse_trip < 0 ||
-      hw->max_stream_pct < 0 || hw->max_stream_pct > 100 || hw->stream_floor < 0)
+      hw->max_stream_pct < 0 || hw->max_stream_pct > 100 || hw->stream_floor < 0 || hw->private_streams < 0)
     return CATT_EINVAL;
   for (int i = 1; i < hw->n_carveouts; ++i)
     if (hw->carveout_kb[i] <= hw->carveout_kb[i - 1]) return CATT_EINVAL;

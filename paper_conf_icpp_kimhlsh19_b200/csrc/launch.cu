@@ -683,7 +683,7 @@ extern "C" const char* catt_status_str(catt_status s) {
 }
 
 extern "C" int catt_last_cuda_error(void) { return g_last_err; }
-extern "C" int catt_abi_version(void) { return 5; }
+extern "C" int catt_abi_version(void) { return 6; }
 
 // ------------------------------------------------------------ SM partition
 // Green context of >= min_sms SMs and a non-blocking stream in it (catt.h).

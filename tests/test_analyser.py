@@ -24,7 +24,7 @@ def test_library_loads_and_exports_every_declared_symbol():
     assert declared == set(catt.catt.EXPORTED)
     for name in declared:
         assert hasattr(L, name), name
-    assert L.catt_abi_version() == 5
+    assert L.catt_abi_version() == 6
 
 
 def test_struct_layouts_match_header():

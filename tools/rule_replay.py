@@ -7,6 +7,7 @@ rule, and the pick's time is divided by the best swept time.
 
 usage: python tools/rule_replay.py [--rule b200|r24|r23|r18|paper] [--set final|heldout|heldout2|heldout3|heldout4|heldout5|heldout6|heldout7|heldout8|heldout9|partition|all] [-v]
   b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24 + R27 + R29)
+  r32   = b200 + the candidate R32 (a divergent load shared by the CTA's warps is not a stream)
   r27   = the round-1 rule (b200 without R29's divergent-streams floor)
   r24   = the same without R27 (the floor fallback gates warps also with several CTAs per SM)
   r23   = R18 + R19 + R23 (re-touch and reuse-trip terms), as held-out study 2 tested it
@@ -80,6 +81,9 @@ def problem_of(s, f, r):
 
 def rule_hw(name):
     hw = catt.hw_b200()
+    if name == "r32":                          # candidate: CTA-shared divergent loads do not count (R32)
+        hw.private_streams = 1
+        return hw
     if name != "b200":
         hw.stream_floor = 0                    # every older rule predates R29
     if name == "r18":
@@ -131,7 +135,7 @@ def replay(rule, sets, verbose):
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("--rule", default="b200", choices=["b200", "r27", "r24", "r23", "r18", "paper"])
+    ap.add_argument("--rule", default="b200", choices=["b200", "r32", "r27", "r24", "r23", "r18", "paper"])
     ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
