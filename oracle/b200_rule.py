@@ -21,9 +21,12 @@ The rule (readings R17-R19, R23, R24, R27), restated on traces:
   retouch(I)      the most touches one thread makes to one line with I (R23)
   stream          bytes of stores and of loads without reuse over all traced
                   bytes of the loop body (R24)
+  shared(I)       warp 1 of CTA 0 requests exactly warp 0's lines with I's
+                  first access (the CTA's warps share I's lines; R32)
   divergent       some reused load has lines >= divergent_lines and retouch >=
-                  min_retouch, and 100 * stream <= max_stream_pct * total (R18,
-                  R23, R24); S = the number of such loads
+                  min_retouch (and, when private_streams is on, is not shared),
+                  and 100 * stream <= max_stream_pct * total (R18, R23, R24,
+                  R32); S = the number of such loads
   floor           min_warps_sm, or ceil(min_warps_sm / S) when stream_floor is on,
                   T = 1 and S >= 2 (R29)
   fits(a, m)      zero intra-thread capacity misses when a warps per CTA and m
@@ -52,9 +55,10 @@ from . import lru
 
 # DESIGN.md R18 (floor 8 warps/SM, >= 8 lines per request), R23 (>= 16
 # re-touches), R24 (<= 25 % stream bytes), R27 (CTA fallback on), R29 (the
-# floor divided by the divergent streams when T = 1)
+# floor divided by the divergent streams when T = 1), R32 (loads shared by
+# the CTA's warps are not streams; a candidate, off until adopted)
 B200_GUARDS = dict(min_warps_sm=8, divergent_lines=8, min_retouch=16, max_stream_pct=25, cta_fallback=1,
-                   stream_floor=1)
+                   stream_floor=1, private_streams=0)
 # shared-memory options (KB) and the L1D each leaves (KB, measured)
 B200_L1D_KB = {0: 218, 8: 218, 16: 218, 32: 218, 64: 186, 100: 150, 132: 118, 164: 86, 196: 53, 228: 21}
 
@@ -67,6 +71,7 @@ class TraceInputs:
     stored: Dict[str, bool]
     stream_bytes: int
     total_bytes: int
+    shared: Dict[str, bool]
 
     @property
     def locality(self) -> bool:
@@ -93,14 +98,24 @@ def trace_inputs(kernel, line: int = lru.LINE) -> TraceInputs:
         retouch[instr] = max(retouch[instr], c)
     reuse = {i: retouch[i] >= 2 for i in first}
     stream = sum(nbytes[i] for i in first if stored[i] or not reuse[i])
+    # R32: the first request of each instruction in warp 1 of the same CTA
+    first1: Dict[str, set] = {}
+    for instr, _, _, lanes in (kernel.program(0, 1) if kernel.W >= 2 else []):
+        if instr not in first1:
+            first1[instr] = {ln for ln, _ in lanes}
+    first0: Dict[str, set] = {}
+    for instr, _, _, lanes in prog:
+        if instr not in first0:
+            first0[instr] = {ln for ln, _ in lanes}
+    shared = {i: i in first1 and first1[i] == first0[i] for i in first}
     return TraceInputs(reuse=reuse, lines=first, retouch=retouch, stored=stored, stream_bytes=stream,
-                       total_bytes=sum(nbytes.values()))
+                       total_bytes=sum(nbytes.values()), shared=shared)
 
 
 def divergent_loads(inp: TraceInputs, guards: Dict) -> int:
     """How many reused loads are memory-divergent (R18, R23): the streams of R29."""
     return sum(1 for i in inp.lines if inp.reuse[i] and not inp.stored[i] and inp.lines[i] >= guards["divergent_lines"]
-               and inp.retouch[i] >= guards["min_retouch"])
+               and inp.retouch[i] >= guards["min_retouch"] and not (guards.get("private_streams", 0) and inp.shared[i]))
 
 
 def divergent(inp: TraceInputs, guards: Dict) -> bool:

@@ -38,7 +38,9 @@ Steps, in the paper's order and notation (DESIGN.md lists every reading R1..R17)
       taken and an SM holds several CTAs (T >= 2), cap whole CTAs instead --
       (W, m), the smallest m with floor <= W m <= 2 floor. R29 (hw key
       stream_floor): with T = 1 and S >= 2 such divergent reused loads, the
-      floor is ceil(min_warps_sm / S).
+      floor is ceil(min_warps_sm / S). R32 (hw key private_streams): a load
+      whose first request lines are the same in warp 1 as in warp 0 of CTA 0
+      (shared by the CTA's warps) is neither divergent nor a stream.
 
 Units: footprints are in cache lines; "fits" means lines*line_bytes <= L1D
 bytes (throttle iff strictly larger, P:239 R5).
@@ -300,8 +302,13 @@ class Model:
             self.lines_per_warp_iter = sum(per_ref)
             div = hw.get("divergent_lines", 0)
             rt, rtrip = hw.get("min_retouch", 0), hw.get("min_reuse_trip", 0)
-            hot = [n >= div and retouches(r, loop.trips, self.line) >= rt and reuse_trip(r, loop.trips, self.line) >= rtrip
-                   for r, n in zip(self.refs, per_ref) if has_locality(r, loop.trips, self.line)]
+            # R32 (hw key private_streams): a load whose lines warp 1 requests
+            # exactly as warp 0 does is shared by the CTA's warps, not a stream
+            gids01 = _lane_gids(loop, 0, 1, hw["warp_size"]) if (hw.get("private_streams", 0) > 0 and self.W >= 2) else None
+            shared = [gids01 is not None and n >= div and _lines(r, gids01, it0, self.line) == _lines(r, gids00, it0, self.line)
+                      for r, n in zip(self.refs, per_ref)]
+            hot = [n >= div and not sh and retouches(r, loop.trips, self.line) >= rt and reuse_trip(r, loop.trips, self.line) >= rtrip
+                   for r, n, sh in zip(self.refs, per_ref, shared) if has_locality(r, loop.trips, self.line)]
             self.streams = sum(hot)                   # R29: memory-divergent reused loads
             self.divergent = (div <= 0 and rt <= 0 and rtrip <= 0 and hw.get("max_stream_pct", 0) <= 0) or any(hot)
             # R24: bytes per lane and iteration of streams L1 cannot serve again

@@ -92,7 +92,7 @@ def _rand_hw(rnd):
                 min_warps_sm=rnd.choice([0, 0, 4, 16]), divergent_lines=rnd.choice([0, 0, 2, 8]),
                 min_retouch=rnd.choice([0, 0, 4, 16]), min_reuse_trip=rnd.choice([0, 0, 8, 30]),
                 max_stream_pct=rnd.choice([0, 0, 25, 60]), cta_fallback=rnd.choice([0, 1]),
-                stream_floor=rnd.choice([0, 1]),
+                stream_floor=rnd.choice([0, 1]), private_streams=rnd.choice([0, 1]),
                 carveout_kb=carve, l1d_bytes=[rnd.randint(1, 200) * 128 for _ in carve])
 
 

@@ -56,6 +56,12 @@ def test_trace_inputs_of_the_other_loops():
     # SYRK's a[j*M + k]: 32 lines per request (one row per lane), 32 touches
     s = br.trace_inputs(lru.SyrkKernel(256, 64))
     assert s.lines == {"a_i": 1, "a_j": 32} and s.retouch["a_j"] == 32
+    # ... and a[j*M + k] is the same 32 lines for every warp of the 32 x 8
+    # block (warps differ in i only), a[i*M + k] is not (R32)
+    assert s.shared == {"a_i": False, "a_j": True}
+    s2 = br.trace_inputs(lru.Syr2kKernel(256, 64))
+    assert s2.shared == {"a_i": False, "b_i": False, "b_j": True, "a_j": True}
+    assert br.trace_inputs(lru.RowKernel(256, 128, 256)).shared == {"x": True, "A": False}   # lanes are rows
     # CORR: lanes at j2 = j1 + 1 + q read coalesced columns (j2 = 1..32 spans two lines)
     r = br.trace_inputs(lru.CorrKernel(96, 4, 32))
     assert r.lines["d_j1"] == 1 and r.lines["d_j2"] == 2 and r.reuse["d_j1"] and r.stored["sym_12"]
@@ -69,6 +75,13 @@ def test_divergence_predicate():
     assert not br.divergent(br.trace_inputs(lru.KmeansKernel(4096, 6, 5, 4096, 256)), g)  # coalesced (R18)
     loose = dict(g, max_stream_pct=60)
     assert br.divergent(br.trace_inputs(lru.TransposeKernel(4096, 34, 4096, 256)), loose)
+    # R32: SYRK's one divergent load is shared by the CTA's warps; SYR2K has two
+    syrk, syr2k = br.trace_inputs(lru.SyrkKernel(256, 64)), br.trace_inputs(lru.Syr2kKernel(256, 64))
+    off, on = dict(g, private_streams=0), dict(g, private_streams=1)
+    assert br.divergent_loads(syrk, off) == 1 and br.divergent_loads(syr2k, off) == 2
+    assert br.divergent_loads(syrk, on) == 0 and not br.divergent(syr2k, on)
+    rows = br.trace_inputs(lru.RowKernel(256, 128, 256))
+    assert br.divergent_loads(rows, on) == br.divergent_loads(rows, off) == 1
 
 
 def test_lru_fit_is_the_capacity_of_the_retained_lines():
@@ -130,11 +143,14 @@ KERNELS = [
 ]
 
 
+@pytest.mark.parametrize("private", [0, 1], ids=["r32off", "r32on"])
 @pytest.mark.parametrize("name,prob,launch,kern", KERNELS, ids=[k[0] for k in KERNELS])
-def test_library_rule_equals_trace_oracle_on_own_kernels(name, prob, launch, kern):
+def test_library_rule_equals_trace_oracle_on_own_kernels(name, prob, launch, kern, private):
     """catt_footprint with the B200 guards on a small fake GPU (2 SMs, 16
-    warps) picks what the trace oracle picks, at every carveout."""
-    hw = catt.Hw.from_dict(dict(SMALL_HW, **SMALL_GUARDS))
+    warps) picks what the trace oracle picks, at every carveout, with R32
+    (private_streams) off and on."""
+    guards = dict(SMALL_GUARDS, private_streams=private)
+    hw = catt.Hw.from_dict(dict(SMALL_HW, **guards))
     for carve in SMALL_HW["carveout_kb"]:
         d, keep = catt.kernel_desc(prob, launch)
         d.regs_per_thread = 0
@@ -142,7 +158,7 @@ def test_library_rule_equals_trace_oracle_on_own_kernels(name, prob, launch, ker
         d.force_carveout_kb = carve
         got = catt.footprint(d, hw)
         W, T = got["base_warps"], got["base_ctas"]
-        a, m, how = br.decide(kern, W, T, got["l1d_bytes"] // 128, SMALL_HW["num_sms"], SMALL_GUARDS)
+        a, m, how = br.decide(kern, W, T, got["l1d_bytes"] // 128, SMALL_HW["num_sms"], guards)
         assert (got["active_warps"], got["active_ctas"]) == (a, m), (name, carve, got, how)
 
 
@@ -157,9 +173,10 @@ def test_library_rule_equals_trace_oracle_on_the_178_replayed_launches():
     library's (W, T), L1D and pick equal those tools/gen_rule_golden.py derived
     from oracle/ alone (traces + LRU + Eq 1-4)."""
     g = _golden()
-    assert len(g["launches"]) == 178 and g["guards"] == br.B200_GUARDS
+    assert len(g["launches"]) == 178 and dict({"private_streams": 0}, **g["guards"]) == br.B200_GUARDS
     b200 = catt.hw_b200()
-    keys = ("min_warps_sm", "divergent_lines", "min_retouch", "max_stream_pct", "cta_fallback", "stream_floor")
+    keys = ("min_warps_sm", "divergent_lines", "min_retouch", "max_stream_pct", "cta_fallback", "stream_floor",
+            "private_streams")
     assert tuple(getattr(b200, k) for k in keys) == tuple(br.B200_GUARDS[k] for k in keys)
     for L in g["launches"]:
         p = dict(L["prob"])
