@@ -9,7 +9,7 @@ rule is measured on the loop body's address trace (oracle/lru.py `program`,
 written from the kernels' source loops), and "fits" is the LRU L1D simulator's
 verdict, not a footprint formula.
 
-The rule (readings R17-R19, R23, R24, R27), restated on traces:
+The rule (readings R17-R19, R23, R24, R27, R29, R32), restated on traces:
 
   reuse(I)        instruction I has same-thread locality: one thread touches one
                   line with I in two different iterations (Eq 6's intent,
@@ -56,9 +56,9 @@ from . import lru
 # DESIGN.md R18 (floor 8 warps/SM, >= 8 lines per request), R23 (>= 16
 # re-touches), R24 (<= 25 % stream bytes), R27 (CTA fallback on), R29 (the
 # floor divided by the divergent streams when T = 1), R32 (loads shared by
-# the CTA's warps are not streams; a candidate, off until adopted)
+# the CTA's warps are not streams)
 B200_GUARDS = dict(min_warps_sm=8, divergent_lines=8, min_retouch=16, max_stream_pct=25, cta_fallback=1,
-                   stream_floor=1, private_streams=0)
+                   stream_floor=1, private_streams=1)
 # shared-memory options (KB) and the L1D each leaves (KB, measured)
 B200_L1D_KB = {0: 218, 8: 218, 16: 218, 32: 218, 64: 186, 100: 150, 132: 118, 164: 86, 196: 53, 228: 21}
 

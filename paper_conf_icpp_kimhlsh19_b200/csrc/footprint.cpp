@@ -520,6 +520,11 @@ extern "C" catt_status catt_hw_b200(catt_hw* out) {
   // 14/18 launches within 5 % of the best (7/18 without), geomean 1.019x
   // (1.106x), worst 1.076x (1.373x) (profiles/r2/heldout10/)
   out->stream_floor = 1;
+  // R32 (round 2, held-out study 11, picks pre-registered): a divergent load
+  // whose lines every warp of the CTA shares (SYRK/SYR2K's a[j][k]) is not a
+  // stream: 14/17 launches within 5 % of the best (10/17 without), geomean
+  // 1.016x (1.089x), worst 1.089x (1.359x) (profiles/r2/heldout11/)
+  out->private_streams = 1;
   // Shared-memory options (KB) and the carveout percentage that selects each
   // (percent of the 228 KB maximum; the driver rounds up to the next option).
   // L1D capacity per option, measured on B200 by the Fig 3-style sweep

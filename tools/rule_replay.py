@@ -6,8 +6,8 @@ name is rebuilt here, the analyser (catt_plan, no GPU) picks (a, m) under the
 rule, and the pick's time is divided by the best swept time.
 
 usage: python tools/rule_replay.py [--rule b200|r24|r23|r18|paper] [--set final|heldout|heldout2|heldout3|heldout4|heldout5|heldout6|heldout7|heldout8|heldout9|partition|all] [-v]
-  b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24 + R27 + R29)
-  r32   = b200 + the candidate R32 (a divergent load shared by the CTA's warps is not a stream)
+  b200  = the library's B200 table (R18 + R19 + R23 re-touch term + R24 + R27 + R29 + R32)
+  r29   = b200 without R32 (a divergent load shared by the CTA's warps is not a stream)
   r27   = the round-1 rule (b200 without R29's divergent-streams floor)
   r24   = the same without R27 (the floor fallback gates warps also with several CTAs per SM)
   r23   = R18 + R19 + R23 (re-touch and reuse-trip terms), as held-out study 2 tested it
@@ -61,7 +61,9 @@ FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["p
          # after R24 was fixed: the CTA-level regime (SURVEY 8(d) [3])
          "partition": ["profiles/r1g/bench_gesummv.json"],
          # round 2: 2- and 3-stream rows at T = 1, testing the candidate R29 (adopted)
-         "heldout10": ["profiles/r2/heldout10/heldout10_study.json"]}
+         "heldout10": ["profiles/r2/heldout10/heldout10_study.json"],
+         # round 2: SYRK / SYR2K 2-D blocks, testing the candidate R32 (adopted)
+         "heldout11": ["profiles/r2/heldout11/heldout11_study.json"]}
 ATAX = {"bench_atax.json": P(catt.K_ATAX_1, m=65536, n=16384), "bench_atax256.json": P(catt.K_ATAX_1, m=256, n=256)}
 
 
@@ -81,8 +83,10 @@ def problem_of(s, f, r):
 
 def rule_hw(name):
     hw = catt.hw_b200()
-    if name == "r32":                          # candidate: CTA-shared divergent loads do not count (R32)
-        hw.private_streams = 1
+    if name == "b200":
+        return hw
+    hw.private_streams = 0                     # every older rule predates R32
+    if name == "r29":                          # the library's rule before R32
         return hw
     if name != "b200":
         hw.stream_floor = 0                    # every older rule predates R29
@@ -135,11 +139,11 @@ def replay(rule, sets, verbose):
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("--rule", default="b200", choices=["b200", "r32", "r27", "r24", "r23", "r18", "paper"])
-    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "all"])
+    ap.add_argument("--rule", default="b200", choices=["b200", "r29", "r27", "r24", "r23", "r18", "paper"])
+    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "heldout11", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
-    sets = ["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10"] if a.set == "all" else [a.set]
+    sets = ["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "heldout11"] if a.set == "all" else [a.set]
     res = replay(a.rule, sets, a.v)
     for s in sets:
         rs = [x for x in res if x[0] == s]
