@@ -380,10 +380,15 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 // column group): the row operand is a broadcast in every warp (2 shared-memory
 // wavefronts per float4 read), the column operand 32 distinct words (4).
 // Measured at 2048: 0.366 ms against 0.375 ms for 128 x 128 tiles. A mix of
-// 64- and 48-row blocks that fills the 296 CTA slots in one wave (instead of
-// 256 tiles, 1.73 per SM) measured the same 0.367 ms: the 48-row tile's 6 x 8
-// outputs per thread need as many column reads for 3/4 of the FMAs and the
-// SM's shared-memory pipe becomes the limit, so it was not kept.
+// 64- and 48-row CTAs that fills the 296 CTA slots in one wave measured the
+// same 0.367 ms (round 2, early): which CTAs share an SM is not under the
+// kernel's control, and two 64-row CTAs on one SM still load each
+// sub-partition with 4 units. The work per sub-partition is what sets the
+// time once the grid is one wave (a warp runs on sub-partition warp % 4; two
+// warps per sub-partition issue FFMA2 as fast as four, tools/warp_rate_probe):
+// the mixed 56-row tile (kMixRows) mixes within the CTA instead, 8 + 6 rows
+// per sub-partition from every CTA, and took SYRK 2048 from 0.342 to 0.327 ms
+// and SYR2K from 0.976 to 0.916 ms, bit-identical (t2_use_mix picks it).
 #ifndef T2_NS
 #define T2_NS 4
 #endif
@@ -396,14 +401,14 @@ __global__ void __launch_bounds__(256, MINB) tiled_kernel(TileArgs a) {
 // FMA by 0.6x, and 2048 rows make 144 tiles for 148 SMs); measured slower at
 // every size (2048: 0.379 vs 0.357 ms; 4096: 1.65 vs 1.15 ms; one CTA of 8
 // warps per SM does not keep the FMA pipe busy), so only RH = 8 is launched.
-template <int MODE, int RH = 8>
+template <int MODE, int RH = 8, int RBOX = 8 * RH>
 struct T2Cfg {
   static constexpr int NA = MODE == MODE_SYR2K ? 4 : 2;
   static constexpr int NP = NA / 2;                               // row-side (and column-side) arrays
   static constexpr int BK = MODE == MODE_SYR2K ? 8 : T2_BK;
   static constexpr int MINB = RH > 8 ? 1 : 2;                    // CTAs per SM
   static constexpr int NS = RH > 8 ? 6 : T2_NS;                  // ring stages
-  static constexpr int RB = 8 * RH, CB = 256;                    // row box, column strip
+  static constexpr int RB = RBOX, CB = 256;                       // row box, column strip
   static constexpr int ROW_FLOATS = BK * RB, COL_FLOATS = BK * CB;
   static constexpr int STAGE_FLOATS = NP * (ROW_FLOATS + COL_FLOATS);
   static constexpr int FBUF = MODE == MODE_SYR2K ? 1 : 2;
@@ -426,16 +431,27 @@ struct T2Geo {
   int uw, ux;        // uw units each, the first ux CTAs one more (<= 8: one unit per warp)
 };
 
+// The mixed tile (tile2_mix_kernel): 56 rows, warps 0-3 take 8 rows each and
+// warps 4-7 take 6. A warp runs on sub-partition (warp % 4), so every CTA
+// gives each sub-partition 8 + 6 rows of work, wherever the CTA lands. With
+// whole 8-row units a 2048-row SYRK has 13.8 units per SM, and the busiest of
+// the four sub-partitions carries 4 of them (two CTAs of 7 active warps: one
+// sub-partition gets 2 units, the others 4); the mixed tile carries 3.5.
+constexpr int kMixRows = 56;
+
 // One (RH W) x 256 tile computed by its first W warps (W <= 8), RH rows per
 // thread: rows {4 W g + 4 ty + r} for the G = RH / 4 full groups, then
 // {4 W G + (RH % 4) ty + r} (ty = warp). Fewer active warps make a shorter
 // tile at the same 8 x 8 outputs (and shared-memory cost) per thread, which
 // is how the grid balances the SMs' work (launch_t2).
-template <int MODE, int RH>
+// MIX (the 56-row tile): this warp's RH rows start at row wrow of the tile,
+// contiguous (8: two float4 groups; 6: one float4 and one float2 group,
+// whichever order keeps both aligned).
+template <int MODE, int RH, int RBOX = 8 * RH, bool MIX = false>
 __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* empty, const T2Maps& maps,
-                                        const TileArgs& a, int64_t i0, int64_t j0, int W) {
+                                        const TileArgs& a, int64_t i0, int64_t j0, int W, int wrow = 0) {
   constexpr bool TWO = MODE == MODE_SYR2K;
-  using Cfg = T2Cfg<MODE, RH>;
+  using Cfg = T2Cfg<MODE, RH, RBOX>;
   constexpr int BK = Cfg::BK, NP = Cfg::NP, NS = Cfg::NS, RBX = Cfg::RB, CBX = Cfg::CB;
   constexpr int G = RH / 4, RR = RH % 4;
   // stage layout: NP row arrays [BK][8 RH], then NP column arrays [BK][256]
@@ -448,7 +464,28 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
   const int64_t n = a.ni, m = a.m;
   const int64_t ktiles = (m + BK - 1) / BK;
   const int gs = 4 * W;  // row group stride
-  auto row_of = [&](int r) { return r < 4 * G ? gs * (r / 4) + 4 * ty + (r % 4) : gs * G + RR * ty + (r - 4 * G); };
+  // tile row of the warp's float4 group g (rows off4(g) .. +3) and of its
+  // remaining RR rows (off2() ..); the uniform tile interleaves the warps'
+  // groups, the mixed tile gives each warp contiguous rows
+  int m4a = 0, m4b = 0, m2 = 0;
+  if constexpr (MIX) {
+    static_assert(RH == 8 || RH == 6, "the mixed tile has 8- and 6-row warps");
+    if constexpr (RH == 8) {
+      m4a = wrow, m4b = wrow + 4;
+    } else {
+      const bool lo = (wrow & 3) == 0;
+      m4a = lo ? wrow : wrow + 2, m2 = lo ? wrow + 4 : wrow;
+    }
+  }
+  auto off4 = [&](int g) {
+    if constexpr (MIX) return g == 0 ? m4a : m4b;
+    else return gs * g + 4 * ty;
+  };
+  auto off2 = [&]() {
+    if constexpr (MIX) return m2;
+    else return gs * G + RR * ty;
+  };
+  auto row_of = [&](int r) { return r < 4 * G ? off4(r / 4) + (r % 4) : off2() + (r - 4 * G); };
 
   // row-side stage arrays: alpha*a[i][k] (SYR2K: then alpha*b[i][k]); column-side: a[j][k]
   // (SYR2K: b[j][k], then a[j][k]); maps in the same order
@@ -499,15 +536,15 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
       const float* rp = rowp(slot, s, kk);
 #pragma unroll
       for (int g = 0; g < G; ++g) {
-        const float4 v = *reinterpret_cast<const float4*>(rp + gs * g + ty * 4);
+        const float4 v = *reinterpret_cast<const float4*>(rp + off4(g));
         fr[fb][s][4 * g] = v.x, fr[fb][s][4 * g + 1] = v.y, fr[fb][s][4 * g + 2] = v.z, fr[fb][s][4 * g + 3] = v.w;
       }
       if constexpr (RR == 2) {
-        const float2 v = *reinterpret_cast<const float2*>(rp + gs * G + ty * 2);
+        const float2 v = *reinterpret_cast<const float2*>(rp + off2());
         fr[fb][s][4 * G] = v.x, fr[fb][s][4 * G + 1] = v.y;
       } else {
 #pragma unroll
-        for (int q = 0; q < RR; ++q) fr[fb][s][4 * G + q] = rp[gs * G + RR * ty + q];
+        for (int q = 0; q < RR; ++q) fr[fb][s][4 * G + q] = rp[off2() + q];
       }
       const float* cq = colp(slot, s, kk);
 #pragma unroll
@@ -530,6 +567,8 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
       return;
     }
     if constexpr (TWO && T2_PAIR_OUTER) {  // SYR2K: the same, each op kind grouped over r
+      // (grouping 4 rows at a time spills less at 128 registers but measured
+      // slower: 0.976 -> 1.010 ms uniform, equal in the mixed tile)
 #pragma unroll
       for (int p = 0; p < 4; ++p) {
         const uint64_t bq = f2_pack(fc[fb][0][2 * p], fc[fb][0][2 * p + 1]);
@@ -633,7 +672,7 @@ __device__ __forceinline__ void t2_tile(float* sm, uint64_t* full, uint64_t* emp
       }
     }
   }
-  if constexpr (MODE == MODE_SYRK) if (a.mirror) {
+  if constexpr (MODE == MODE_SYRK && !MIX) if (a.mirror) {
     // the lower triangle: C[j][i] = C[i][j] for j > i, the tile staged
     // transposed through the (now idle) stage ring so each warp writes whole
     // 64-float row segments of C^T (coalesced). Every stage was consumed
@@ -709,6 +748,41 @@ __global__ void __launch_bounds__(256, (RH > 8 ? 1 : 2)) tile2_kernel(const __gr
   // its tail; wait for its completion (and memory) before reading A or C
   asm volatile("griddepcontrol.wait;" ::: "memory");
   t2_tile<MODE, RH>(t2_dyn, full, empty, maps, a, i0, int64_t(cs) * Cfg::CB, W);
+  cta_exit(a.t);
+}
+
+// The mixed 56-row tile (kMixRows): CTA k of strip cs owns rows [56 k, 56 k + 56).
+template <int MODE>
+__global__ void __launch_bounds__(256, 2) tile2_mix_kernel(const __grid_constant__ T2Maps maps, TileArgs a, T2Geo g) {
+  using Cfg = T2Cfg<MODE, 8, kMixRows>;
+  static_assert(sizeof(T2Cfg<MODE, 6, kMixRows>) > 0 && T2Cfg<MODE, 6, kMixRows>::STAGE_FLOATS == Cfg::STAGE_FLOATS &&
+                    T2Cfg<MODE, 6, kMixRows>::NS == Cfg::NS && T2Cfg<MODE, 6, kMixRows>::BK == Cfg::BK,
+                "both warp kinds read one stage ring");
+  constexpr int NS = Cfg::NS;
+  extern __shared__ __align__(128) float t2_dyn[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(t2_dyn + NS * Cfg::STAGE_FLOATS);
+  uint64_t* empty = full + NS;
+  const int cs = int(blockIdx.x) / g.q, k = int(blockIdx.x) % g.q;
+  const int64_t i0 = int64_t(kMixRows) * k;
+  auto wrow = [](int w) { return w < 4 ? 8 * w : 32 + 6 * (w - 4); };
+  int W = 0;  // warps with a row inside the matrix (rows ascend with the warp)
+  for (int w = 0; w < 8; ++w)
+    if (i0 + wrow(w) < a.ni) W = w + 1;
+  cta_enter(a.t);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < NS; ++s) {
+      bar_init(&full[s], 1);
+      bar_init(&empty[s], unsigned(W));
+    }
+    fence_barrier_init();
+  }
+  __syncthreads();
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  const int warp = int(threadIdx.x) >> 5;
+  if (warp < 4)
+    t2_tile<MODE, 8, kMixRows, true>(t2_dyn, full, empty, maps, a, i0, int64_t(cs) * Cfg::CB, W, wrow(warp));
+  else
+    t2_tile<MODE, 6, kMixRows, true>(t2_dyn, full, empty, maps, a, i0, int64_t(cs) * Cfg::CB, W, wrow(warp));
   cta_exit(a.t);
 }
 
@@ -836,10 +910,37 @@ static int64_t t2_tiles(const T2Geo& g, int rb_rows) {
   return tiles;
 }
 
-template <int MODE, int RH>
+// The mixed 56-row tile instead of whole 8-row units: when both grids fit one
+// wave, when it lowers the busiest sub-partition's load (in 8-row units:
+// per CTA ceil(W / 4) of its W active warps, 1.75 for the mixed tile; two
+// CTAs per SM when the grid exceeds the SMs). CATT_T2_MIX=0/1 overrides
+// (tools only).
+static bool t2_use_mix(int64_t n, bool tri) {
+  static const int env = [] {
+    const char* e = getenv("CATT_T2_MIX");
+    return e ? atoi(e) : -1;
+  }();
+  static const int nsm = [] {
+    int d = 0, v = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    return v;
+  }();
+  if (tri) return false;
+  if (env == 0 || env == 1) return env == 1;
+  const T2Geo g = t2_geometry(n, false, 8);
+  const int64_t gu = int64_t(g.cs) * g.q, gm = int64_t(g.cs) * ((n + kMixRows - 1) / kMixRows);
+  if (gu > 2 * nsm || gm > 2 * nsm) return false;
+  const int wmax = g.uw + (g.ux > 0 ? 1 : 0);
+  const double lu = (gu > nsm ? 2 : 1) * double((wmax + 3) / 4);
+  const double lm = (gm > nsm ? 2 : 1) * 1.75;
+  return lm < lu;
+}
+
+template <int MODE, int RH, int RBOX = 8 * RH>
 static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s) {
-  const void* f = (const void*)tile2_kernel<MODE, RH>;
-  constexpr size_t sb = T2Cfg<MODE, RH>::SBYTES;
+  constexpr bool MIX = RBOX != 8 * RH;
+  const void* f = MIX ? (const void*)tile2_mix_kernel<MODE> : (const void*)tile2_kernel<MODE, RH>;
+  constexpr size_t sb = T2Cfg<MODE, RH, RBOX>::SBYTES;
   cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(sb));
   if (e != cudaSuccess) {
     record_cuda_error(e);
@@ -898,7 +999,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   // stage arrays, row side then column side: SYRK {(alpha A)^T} {A^T};
   // SYR2K {(alpha A)^T, (alpha B)^T} {B^T, A^T}
   T2Maps maps{};
-  using Cfg = T2Cfg<MODE, RH>;
+  using Cfg = T2Cfg<MODE, RH, RBOX>;
   const float* src[4];
   if (MODE == MODE_SYR2K) {
     src[0] = aAt, src[1] = aBt, src[2] = Bt, src[3] = At;
@@ -912,7 +1013,8 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
     if (ws) cudaFreeAsync(ws, s);
     return CATT_ECUDA;
   }
-  const T2Geo g = t2_geometry(n, a.tri != 0, RH);
+  T2Geo g = t2_geometry(n, a.tri != 0, RH);
+  if (MIX) g.q = int((n + kMixRows - 1) / kMixRows), g.uw = g.ux = 0;
   const int64_t tiles = a.tri ? t2_tiles(g, Cfg::RB) : int64_t(g.cs) * g.q;
   if (tiles > (int64_t(1) << 31) - 1) {
     if (ws) cudaFreeAsync(ws, s);
@@ -935,7 +1037,10 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = a.tri ? 0 : 1;
-  e = cudaLaunchKernelEx(&cfg, tile2_kernel<MODE, RH>, maps, a, g);
+  if constexpr (MIX)
+    e = cudaLaunchKernelEx(&cfg, tile2_mix_kernel<MODE>, maps, a, g);
+  else
+    e = cudaLaunchKernelEx(&cfg, tile2_kernel<MODE, RH>, maps, a, g);
   if (e != cudaSuccess) {
     record_cuda_error(e);
     cudaGetLastError();
@@ -1017,7 +1122,8 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
   const bool small = small_tiles<MODE>(a.ni, a.nj);
   if constexpr (MODE != MODE_GEMM)
     if (!small && t2_ok<MODE>(a)) {
-      const catt_status st = launch_t2<MODE, 8>(a, t, s);
+      const catt_status st = (!a.mirror && t2_use_mix(a.ni, a.tri != 0)) ? launch_t2<MODE, 8, kMixRows>(a, t, s)
+                                                                          : launch_t2<MODE, 8>(a, t, s);
       if (st != CATT_ENOMEM) return st;  // no room for the k-major copies: the round-1 kernel below
     }
   constexpr int TMs = MODE == MODE_SYR2K ? 8 : 4;  // SYR2K never takes the small tile (static_assert)
@@ -1082,24 +1188,25 @@ static catt_status launch_tiled(TileArgs a, const catt_throttle* t, cudaStream_t
 const void* syrk_func(int variant, int64_t n, bool tri) {
   if (variant != CATT_VAR_STAGED) return (const void*)syrk_thread_kernel;
   if (!tiled_t2()) return tiled_func<MODE_SYRK>();
+  if (t2_use_mix(n, tri)) return (const void*)tile2_mix_kernel<MODE_SYRK>;
   return (const void*)tile2_kernel<MODE_SYRK, 8>;
-  (void)n, (void)tri;
 }
 
 int64_t syrk_staged_dyn(int64_t n, bool tri) {
-  (void)n, (void)tri;
-  return tiled_t2() ? int64_t(T2Cfg<MODE_SYRK, 8>::SBYTES) : 0;
+  if (!tiled_t2()) return 0;
+  return t2_use_mix(n, tri) ? int64_t(T2Cfg<MODE_SYRK, 8, kMixRows>::SBYTES) : int64_t(T2Cfg<MODE_SYRK, 8>::SBYTES);
 }
 
-const void* syr2k_func(int variant) {
+const void* syr2k_func(int variant, int64_t n) {
   if (variant != CATT_VAR_STAGED) return (const void*)syr2k_thread_kernel;
-  if (tiled_t2()) return (const void*)tile2_kernel<MODE_SYR2K, 8>;
+  if (tiled_t2()) return t2_use_mix(n, false) ? (const void*)tile2_mix_kernel<MODE_SYR2K> : (const void*)tile2_kernel<MODE_SYR2K, 8>;
   if (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) return (const void*)tiled_kernel<MODE_SYR2K, 1, 8, false, true>;
   return tiled_func<MODE_SYR2K>();
 }
 
-int64_t syr2k_staged_dyn() {
-  if (tiled_t2()) return int64_t(T2Cfg<MODE_SYR2K, 8>::SBYTES);
+int64_t syr2k_staged_dyn(int64_t n) {
+  if (tiled_t2())
+    return t2_use_mix(n, false) ? int64_t(T2Cfg<MODE_SYR2K, 8, kMixRows>::SBYTES) : int64_t(T2Cfg<MODE_SYR2K, 8>::SBYTES);
   return (tiled_deep<MODE_SYR2K>() && tiled_minb(true) == 1) ? int64_t(TileCfg<MODE_SYR2K, 8, false, true>::SBYTES) : 0;
 }
 

@@ -19,8 +19,8 @@ int col_tma_stages(int cols, int rows_per_stage);
 int row_tma_stage_bytes(int nmat, int rows, int boxes);
 int col_tma_stage_bytes(int cols, int rows_per_stage);
 const void* syrk_func(int variant, int64_t n, bool tri);
-const void* syr2k_func(int variant);
-int64_t syr2k_staged_dyn();
+const void* syr2k_func(int variant, int64_t n);
+int64_t syr2k_staged_dyn(int64_t n);
 int64_t syrk_staged_dyn(int64_t n, bool tri);
 const void* kmeans_func(int variant, int nf);
 int64_t kmeans_tma_smem(int nf, int k);
@@ -240,7 +240,7 @@ const void* loop_func(const catt_problem& p, int variant) {
   if (variant == CATT_VAR_FUSED && (is_row(p.loop) || is_col(p.loop))) return fused_func(p.loop == CATT_K_ATAX_1 || p.loop == CATT_K_ATAX_2);
   if (is_row(p.loop) || is_col(p.loop)) return gemv_func(p.loop, variant, true);
   if (p.loop == CATT_K_SYRK) return syrk_func(variant, p.n, false);
-  if (p.loop == CATT_K_SYR2K) return syr2k_func(variant);
+  if (p.loop == CATT_K_SYR2K) return syr2k_func(variant, p.n);
   if (p.loop == CATT_K_KMEANS_T) return kmeans_t_func(variant);
   if (p.loop == CATT_K_CORR) return corr_func(variant, p.n);
   if (p.loop == CATT_K_GEMM) return gemm_func(variant);
@@ -461,7 +461,7 @@ extern "C" catt_status catt_kernel_desc(const catt_problem* prob, const catt_thr
       out->grid[0] = (N + 127) / 128;
       out->grid[1] = (N + 127) / 128;
       refs[n++] = mkref(0, 0, 1, 0, 4, 1, NL);
-      dyn = syr2k_staged_dyn();                                    // the DEEP stages (dynamic shared memory)
+      dyn = syr2k_staged_dyn(N);                                    // the DEEP stages (dynamic shared memory)
     } else {
       return CATT_EINVAL;
     }

@@ -228,6 +228,21 @@ def test_syrk_staged_large_tiles(n, m, t):
     assert bits_equal(host(Cd), C_o)
 
 
+@pytest.mark.parametrize("n,m", [(1001, 33), (1800, 21)])
+def test_syrk_syr2k_mixed_tile_ragged(n, m):
+    """The mixed 56-row T2 tile (warps 0-3: 8 rows, 4-7: 6 rows; chosen at
+    these sizes by t2_use_mix): the last CTA of a strip holds 49 (n = 1001:
+    seven warps active, the seventh partly) or 8 rows (n = 1800: one warp),
+    with a ragged last k stage. SYRK and SYR2K bit-exact."""
+    A, B, C = si.matrix(6, n, m), si.matrix(8, n, m), si.matrix(106, n, n)
+    Cd = dev(C)
+    catt.syrk(dev(A), Cd, 1.5, 1.2, t=catt.Throttle(variant="staged"))
+    assert bits_equal(host(Cd), oracle.syrk(A, C, 1.5, 1.2))
+    Cd = dev(C)
+    catt.syr2k(dev(A), dev(B), Cd, 1.5, 1.2, t=catt.Throttle(variant="staged"))
+    assert bits_equal(host(Cd), oracle.syr2k(A, B, C, 1.5, 1.2))
+
+
 @pytest.mark.parametrize("alpha,beta", [(1.0, 0.5), (1.5, 0.0), (-0.75, 1.0)])
 def test_syrk_syr2k_staged_alpha_beta_forms(alpha, beta):
     """T2 with alpha == 1 (one k-major copy serves both operands), beta == 0

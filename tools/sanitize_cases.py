@@ -207,12 +207,23 @@ def case_tiles():
 
 
 def case_tiles2():
-    n, m = 1601, 40                                   # 64/48-row geometry, ragged edge and last stage
+    n, m = 1601, 40                                   # the mixed 56-row tile, ragged edge and last stage
     A, B = si.matrix(6, n, m, D), si.matrix(8, n, m, D)
     C0 = si.matrix(9, n, n, D)
     C = T(C0)
     catt.syrk(T(A), C, 1.5, 1.25, t=catt.Throttle(variant="staged"))
-    eq(C, oracle.syrk(A, C0, 1.5, 1.25), "syrk T2")
+    eq(C, oracle.syrk(A, C0, 1.5, 1.25), "syrk T2 (mixed tile)")
+    n1 = 1001                                         # SYR2K through the mixed tile: 7 warps in the last CTA
+    C0 = si.matrix(9, n1, n1, D)
+    C = T(C0)
+    catt.syr2k(T(A[:n1]), T(B[:n1]), C, 1.5, 1.25, t=catt.Throttle(variant="staged"))
+    eq(C, oracle.syr2k(A[:n1], B[:n1], C0, 1.5, 1.25), "syr2k T2 (mixed tile)")
+    n3, m3 = 2200, 8                                  # more than one wave: the uniform 64-row tile
+    A3 = si.matrix(7, n3, m3, D)
+    C0 = si.matrix(9, n3, n3, D)
+    C = T(C0)
+    catt.syrk(T(A3), C, 1.5, 1.25, t=catt.Throttle(variant="staged"))
+    eq(C, oracle.syrk(A3, C0, 1.5, 1.25), "syrk T2 (uniform tile)")
     n2 = 300
     C0 = si.matrix(9, n2, n2, D)
     C = T(C0)
