@@ -196,6 +196,7 @@ __global__ void __launch_bounds__(kStatWarps * 32) corr_stats_rows_kernel(float*
 constexpr int kStripCols = 8, kStripBox = 256, kStripMaxBoxes = 16;  // 8 columns: 25 us at 2048 (16: 28, 4: 31)
 __global__ void __launch_bounds__(256) corr_stats_strip_kernel(const __grid_constant__ CUtensorMap map, float* data,
                                                                float* mean, float* stdv, int64_t n, int64_t m) {
+  asm volatile("griddepcontrol.launch_dependents;");  // the symmat tile kernel may become resident early
   extern __shared__ __align__(128) float s_strip[];  // [n rounded to boxes][kStripCols]
   __shared__ float s_mu[kStripCols], s_scale[kStripCols];
   __shared__ __align__(8) uint64_t s_bar[kStripMaxBoxes];

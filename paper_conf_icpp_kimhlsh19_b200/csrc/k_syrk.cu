@@ -1027,6 +1027,32 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   // upper-triangle grid (CORR, one tile per SM): CTAs launched early land two
   // per SM on the SMs the previous kernel leaves free, which doubled the
   // makespan (0.216 -> 0.382 ms)
+  // The upper-triangle grid can still follow its producer (CORR's statistics)
+  // programmatically when it has at most one tile per SM: a dynamic
+  // shared-memory request above half the SM's keeps the early CTAs one per SM
+  static const int tri_pdl = [] {
+    const char* e = getenv("CATT_T2_TRI_PDL");
+    return e ? atoi(e) : 1;
+  }();
+  static const int nsm_l = [] {
+    int d = 0, v = 148;
+    if (cudaGetDevice(&d) == cudaSuccess) cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    return v;
+  }();
+  bool pdl = !a.tri;
+  if (a.tri && tri_pdl && tiles <= nsm_l && !(t && t->active_ctas > 0)) {
+    constexpr size_t half = 116 * 1024;  // > 228 KB / 2
+    if (dyn < half) {
+      e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, int(half));
+      if (e != cudaSuccess) {
+        record_cuda_error(e);
+        if (ws) cudaFreeAsync(ws, s);
+        return CATT_ECUDA;
+      }
+      dyn = half;
+    }
+    pdl = true;
+  }
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(unsigned(tiles));
   cfg.blockDim = dim3(256);
@@ -1036,7 +1062,7 @@ static catt_status launch_t2(TileArgs a, const catt_throttle* t, cudaStream_t s)
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = a.tri ? 0 : 1;
+  cfg.numAttrs = pdl ? 1 : 0;
   if constexpr (MIX)
     e = cudaLaunchKernelEx(&cfg, tile2_mix_kernel<MODE>, maps, a, g);
   else
