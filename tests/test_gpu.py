@@ -232,8 +232,9 @@ def test_syrk_staged_large_tiles(n, m, t):
 def test_syrk_syr2k_mixed_tile_ragged(n, m):
     """The mixed 56-row T2 tile (warps 0-3: 8 rows, 4-7: 6 rows; chosen at
     these sizes by t2_use_mix): the last CTA of a strip holds 49 (n = 1001:
-    seven warps active, the seventh partly) or 8 rows (n = 1800: one warp),
-    with a ragged last k stage. SYRK and SYR2K bit-exact."""
+    seven warps active, the seventh partly; SYR2K, SYRK takes the 64 x 64
+    small tile there) or 8 rows (n = 1800: one warp), with a ragged last k
+    stage. SYRK and SYR2K bit-exact."""
     A, B, C = si.matrix(6, n, m), si.matrix(8, n, m), si.matrix(106, n, n)
     Cd = dev(C)
     catt.syrk(dev(A), Cd, 1.5, 1.2, t=catt.Throttle(variant="staged"))
