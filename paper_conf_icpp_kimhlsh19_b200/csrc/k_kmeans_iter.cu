@@ -359,11 +359,15 @@ __global__ void __launch_bounds__(KT, 2) km_accumulate_kernel(const __grid_const
     for (int ww = 0; ww < KT / 32; ++ww)
       for (int l = fl; l < 32; l += fg) s += s_acc[((ww * FB + g) * k + cc) * 32 + l];
     if (s != 0) {
+      // only the non-zero chunks: the 296 CTAs add into the same k * nf * 4
+      // words at the end, so every atomic saved shortens the contended tail
+      // (values in [2^-9, 1) leave chunk 0 and chunk 3 zero)
       unsigned long long* limb = a.acc + int64_t(q) * 4;
-      atomicAdd(limb + 0, (unsigned long long)uint32_t(s));
-      atomicAdd(limb + 1, (unsigned long long)uint32_t(s >> 32));
-      atomicAdd(limb + 2, (unsigned long long)uint32_t(s >> 64));
-      atomicAdd(limb + 3, (unsigned long long)(long long)int32_t(uint32_t(s >> 96)));
+      const uint32_t c0 = uint32_t(s), c1 = uint32_t(s >> 32), c2 = uint32_t(s >> 64), c3 = uint32_t(s >> 96);
+      if (c0) atomicAdd(limb + 0, (unsigned long long)c0);
+      if (c1) atomicAdd(limb + 1, (unsigned long long)c1);
+      if (c2) atomicAdd(limb + 2, (unsigned long long)c2);
+      if (c3) atomicAdd(limb + 3, (unsigned long long)(long long)int32_t(c3));
     }
   }
   if (t < k && s_tot[t]) atomicAdd(a.acc + K4 + t, (unsigned long long)s_tot[t]);
