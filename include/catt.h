@@ -247,7 +247,10 @@ typedef struct {
 /* Device properties + the L1D table of catt_hw_b200 (CATT_ENODEV without a GPU). */
 catt_status catt_hw_query(int device, catt_hw* out);
 /* B200 (sm_100a, 148 SMs) with the L1D capacities measured per carveout option
- * by the Fig 3-style footprint sweep (profiles/round1_probe_hw.txt). No GPU needed. */
+ * by the Fig 3-style footprint sweep (profiles/round1_probe_hw.txt), and the
+ * B200 rule on: min_warps_sm 8, divergent_lines 8, min_retouch 16,
+ * min_reuse_trip 0, max_stream_pct 25, cta_fallback 1, stream_floor 1,
+ * private_streams 1 (R18-R32). No GPU needed. */
 catt_status catt_hw_b200(catt_hw* out);
 /* Titan V, the paper's GPU: Table 1, 64 warps/SM, shared
  * memory options 0/8/16/32/64/96 KB with L1D = 128 KB - option. */
