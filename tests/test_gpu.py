@@ -244,6 +244,22 @@ def test_syrk_syr2k_mixed_tile_ragged(n, m):
     assert bits_equal(host(Cd), oracle.syr2k(A, B, C, 1.5, 1.2))
 
 
+def test_t2_geometry_sweep_bit_exact():
+    """Sizes around the switch between the mixed 56-row tile and the uniform
+    64-row tile (one wave vs several, t2_use_mix) and ragged k: SYRK and SYR2K
+    through T2 at each, bit-exact (the geometry never changes an element's
+    k order)."""
+    for n, m in [(1537, 9), (1999, 17), (2047, 5), (2101, 16), (2304, 3), (2561, 11)]:
+        A, B, C = si.matrix(6, n, m), si.matrix(8, n, m), si.matrix(106, n, n)
+        Cd = dev(C)
+        catt.syrk(dev(A), Cd, 1.5, 1.2, t=catt.Throttle(variant="staged"))
+        assert bits_equal(host(Cd), oracle.syrk(A, C, 1.5, 1.2)), n
+        if n < 2200:
+            Cd = dev(C)
+            catt.syr2k(dev(A), dev(B), Cd, 1.5, 1.2, t=catt.Throttle(variant="staged"))
+            assert bits_equal(host(Cd), oracle.syr2k(A, B, C, 1.5, 1.2)), n
+
+
 @pytest.mark.parametrize("alpha,beta", [(1.0, 0.5), (1.5, 0.0), (-0.75, 1.0)])
 def test_syrk_syr2k_staged_alpha_beta_forms(alpha, beta):
     """T2 with alpha == 1 (one k-major copy serves both operands), beta == 0
