@@ -45,3 +45,38 @@ def test_reference_arm_line():
     assert d["impl"] == "reference" and d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["d2h_bytes_per_step"] == 0
     assert d["unit"] == "GB/s" and d["higher_is_better"] is True
+
+
+def _run_torchrun(args, nproc=2, timeout=900, extra_env=None):
+    env = dict(os.environ, PYTHONPATH=ROOT, **(extra_env or {}))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes", "1", "--nproc-per-node", str(nproc),
+           "--master-addr", "127.0.0.1", "--master-port", str(29600 + os.getpid() % 300),
+           os.path.join(ROOT, "bench.py"), "--gpus", str(nproc)] + args
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout, cwd=ROOT, env=env)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.strip().splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout          # rank 0 alone prints
+    return json.loads(lines[0])
+
+
+def test_reference_arm_under_torchrun_rank0_only():
+    """The driver launches --impl reference through torchrun for N > 1: rank 0
+    runs the oracle and prints the one line, the other ranks exit 0."""
+    d = _run_torchrun(["--impl", "reference", "--steps", "1", "--warmup", "3"])
+    assert d["impl"] == "reference" and d["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("variant", [None, "fused_peer"])
+def test_bench_two_ranks_share_one_gpu(variant):
+    """The N > 1 bench path end to end (row shards, the A^T all-reduce between
+    the ranks or inside the fused kernel, max-over-ranks timing, one line from
+    rank 0), with both ranks on cuda:0 over gloo (CATT_BENCH_SHARE_GPU, tests
+    only: NCCL refuses two ranks on one device). Not a bench number."""
+    args = ["--steps", "2", "--warmup", "3", "--no-study", "--no-l1", "--cpu-seconds", "0"]
+    if variant:
+        args += ["--variant", variant]
+    d = _run_torchrun(args, extra_env={"CATT_BENCH_SHARE_GPU": "1"})
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["gpu_launches"] > 0
+    assert d["config"]["parallelism"] == "row-shard x2" and d["config"]["rows_per_rank"] == 65536 // 2
+    assert isinstance(d["roofline"], dict) and d["roofline"]["achieved"] > 0
