@@ -15,6 +15,7 @@ import oracle
 import seeded_inputs as si
 from oracle import footprint as fp
 from oracle import lru
+from oracle import b200_rule
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 
@@ -457,6 +458,64 @@ def test_no_locality_no_throttle():
     hw = _hw_small([4, 4, 4, 4])
     res = fp.analyse(_row_loop(256, 4, 256, 1, vec=4), hw)
     assert res["flags"] == fp.FIT_NONE_NEEDED and res["active_warps"] == 8
+
+
+def test_locality_strict_at_one_line_model_level():
+    # Eq 6 / P:221 strictness at the decision level: a divergent row reference
+    # whose iteration stride is exactly one line (32 floats = 128 B) re-touches
+    # nothing, so the loop is never throttled; 31 floats re-touch the line and
+    # the same loop (footprint far above the L1D) is throttled
+    hw = fp.titan_v()
+    one_line = fp.analyse(_paper_loop([(40960, 32)], grid=640), hw)
+    assert not fp.has_locality(fp.Ref(c_gid=(40960, 0, 0), c_iter=(32,)), (40960,), 128)
+    assert one_line["flags"] == fp.FIT_NONE_NEEDED and one_line["active_warps"] == one_line["base_warps"]
+    below = fp.analyse(_paper_loop([(40960, 31)], grid=640), hw)
+    assert fp.has_locality(fp.Ref(c_gid=(40960, 0, 0), c_iter=(31,)), (40960,), 128)
+    assert below["active_warps"] < below["base_warps"]
+
+
+@pytest.mark.parametrize("e", [1, 2, 4, 8, 16])
+@pytest.mark.parametrize("c", [1, 2, 3, 5, 7])
+def test_req_warp_equals_brute_force_line_count(c, e):
+    # Eq 7 against brute force: the distinct 128-B lines that the 32
+    # lanes' addresses (lane * c * e bytes from a line-aligned base) fall in.
+    # 1-, 2- and 8-byte elements make 32*c*e/128 fractional, where Eq 7's
+    # ceiling matters (a floor would give 0 lines for c = 1, e = 2).
+    hw = fp.titan_v()
+    loop = _paper_loop([(c, 1)], grid=80)
+    loop.refs[0].elem_bytes = e
+    want = len({(lane * c * e) // 128 for lane in range(32)})
+    assert fp.req_warp_paper(loop.refs[0], loop, hw) == want
+
+
+def test_req_warp_printed_form_overcounts_a_partial_stride():
+    # Eq 7 as printed counts 32 whole strides: c = 33 one-byte elements span
+    # 31*33 + 1 = 1024 B (8 lines) but ceil(32*33/128) = 9 (R2 takes the printed
+    # form in paper mode; union mode enumerates the lanes' lines instead)
+    hw = fp.titan_v()
+    for c, e, printed, lines in ((33, 1, 9, 8), (33, 2, 17, 16)):
+        loop = _paper_loop([(c, 1)], grid=80)
+        loop.refs[0].elem_bytes = e
+        assert fp.req_warp_paper(loop.refs[0], loop, hw) == printed == math.ceil(32 * c * e / 128)
+        assert len({(lane * c * e) // 128 for lane in range(32)}) == lines
+
+
+@pytest.mark.parametrize("regs,want", [(32, 8), (40, 6), (64, 4), (128, 2), (255, 1)])
+def test_b200_register_limit_closed_form(regs, want):
+    # Eq 2 on B200 (DESIGN Eq 1-3 reading): 64 K registers per SM in 4
+    # sub-partitions of 16 K, allocated per warp in units of 256 registers.
+    # A 256-thread CTA (8 warps) with r registers per thread: a warp takes
+    # roundup(32 r, 256) registers, a sub-partition holds 16384 // that many
+    # warps, the SM 4x as many; T = those warps // 8 (other limits: 64 warps
+    # -> 8 CTAs, 32 CTA slots, 148 x 64 CTAs in the grid, no shared memory).
+    #   r = 32: 1024 -> 16 warps/SP -> 64 -> T 8;  r = 40: 1280 -> 12 -> 48 -> 6
+    #   r = 64: 2048 -> 8 -> 32 -> 4;  r = 128: 4096 -> 4 -> 16 -> 2
+    #   r = 255: 8160 -> 8192 -> 2 -> 8 -> 1
+    hw = b200_rule.b200_hw()
+    loop = fp.Loop(refs=[fp.Ref(c_gid=(1, 0, 0), c_iter=(1,))], trips=(4,), block=(256, 1, 1),
+                   grid=(148 * 64, 1, 1), regs=regs, mode=fp.MODE_UNION, force_carveout_kb=-1)
+    W, T, _, _ = fp.occupancy(loop, hw)
+    assert (W, T) == (8, want)
 
 
 def test_gemm_pins():
