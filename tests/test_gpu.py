@@ -421,6 +421,22 @@ def test_corr_2048_full_size():
 
 # ------------------------------------------------------------------ KMEANS
 @pytest.mark.parametrize("variant", ["literal", "regs", "staged", "coop"])
+def test_kmeans_distance_fused_per_feature(variant):
+    """R16 on the device: the crafted case of the oracle pin
+    tests/test_oracle.py::test_kmeans_distance_is_fused_per_feature (equal
+    exact distances, one rounding per feature makes centre 1 nearer; an
+    unfused order would tie and pick centre 0). Every point at the origin."""
+    a, b = np.float32(0.7971469759941101), np.float32(0.13876742124557495)
+    npts, nf = 64, 2
+    feat = np.zeros(nf * npts, np.float32)
+    cl = np.array([[a, b], [b, a]], np.float32)
+    memb_o, _ = oracle.kmeans_assign(feat, npts, npts, nf, cl)
+    assert np.all(memb_o == 1)
+    memb = catt.kmeans_assign(dev(feat), npts, npts, nf, dev(cl), t=catt.Throttle(variant=variant))
+    assert np.array_equal(host(memb), memb_o)
+
+
+@pytest.mark.parametrize("variant", ["literal", "regs", "staged", "coop"])
 @pytest.mark.parametrize("npts,nf,k,pad", [(1000, 34, 5, 4), (4099, 34, 5, 29), (257, 7, 3, 3), (300, 50, 12, 4),
                                            (70000, 34, 5, 4), (1, 3, 1, 3), (131, 34, 8, 1), (130, 9, 2, 2)])
 def test_kmeans_exact(variant, npts, nf, k, pad):

@@ -226,6 +226,29 @@ def test_kmeans_vs_bruteforce_argmin():
     assert np.array_equal(memb[:k], np.arange(k))         # each centre is its own point
 
 
+def test_kmeans_distance_is_fused_per_feature():
+    # R16: d = fmaf(diff, diff, d) per feature, f ascending (one rounding per
+    # feature). With the point at the origin and the centres (a, b) and (b, a)
+    # the exact distances are equal; one rounding per feature makes (b, a)
+    # strictly nearer for these a, b, while a mul-then-add order rounds both to
+    # the same value (a tie: centre 0). Expected value from exact rationals
+    # rounded once (oracle.kmeans.round_f32, pinned on its own).
+    from fractions import Fraction
+    from oracle.kmeans import round_f32
+    a, b = np.float32(0.7971469759941101), np.float32(0.13876742124557495)
+
+    def fused(c):
+        d = np.float32(0)
+        for ci in c:
+            df = np.float32(np.float32(0) - ci)
+            d = round_f32(Fraction(float(df)) ** 2 + Fraction(float(d)))
+        return d
+    assert fused([b, a]) < fused([a, b])
+    assert np.float32(a * a) + np.float32(b * b) == np.float32(b * b) + np.float32(a * a)   # unfused: a tie
+    memb, _ = oracle.kmeans_assign(np.zeros(2, np.float32), 1, 1, 2, np.array([[a, b], [b, a]], np.float32))
+    assert memb.tolist() == [1]
+
+
 def test_kmeans_ties_lowest_index():
     nf, k, npts = 4, 3, 8
     feat = np.zeros(nf * npts, np.float32)

@@ -67,6 +67,12 @@ MUTANTS = {
     "seq_fmaf_unfused": ("loops.c", "for (int64_t j = 0; j < n; ++j) acc = fmaf(A[i * n + j], x[j], acc);",
                          "for (int64_t j = 0; j < n; ++j) acc = acc + A[i * n + j] * x[j];", 1,
                          "ATAX row dot rounded twice per step (mul then add)"),
+    "kmeans_assign_unfused": ("loops.c", "\n        d = fmaf(diff, diff, d);", "\n        d = d + diff * diff;", 1,
+                              "KMEANS distance rounded twice per feature"),
+    "generator_constant": ("loops.c", "h *= 0x85EBCA6Bu;", "h *= 0x85EBCA6Du;", 1,
+                           "the counter-based generator's mixing constant mistyped"),
+    "generator_dyadic_grid": ("loops.c", "(float)(h & 15u) * (1.0f / 16.0f)", "(float)(h & 15u) * (1.0f / 8.0f)", 1,
+                              "dyadic inputs on the 1/8 grid (range up to 15/8)"),
     # ---- Eq 1-9 (oracle/footprint.py)
     "eq6_not_strict": ("footprint.py", "abs(ref.c_iter[k]) * ref.elem_bytes < line and trips[k] >= 2 for k",
                        "abs(ref.c_iter[k]) * ref.elem_bytes <= line and trips[k] >= 2 for k", 1,
@@ -79,17 +85,30 @@ MUTANTS = {
                           "", 1, "Eq 3 without the grid bound"),
     "eq4_largest_carveout": ("footprint.py", "idx = next(i for i, c in enumerate(carve) if c * 1024 >= need)",
                              "idx = len(carve) - 1", 1, "Eq 4 always takes the largest shared-memory option"),
+    "eq8_paper_drops_ctas": ("footprint.py", "return self.req * a * m", "return self.req * a", 1,
+                             "Eq 8 (paper mode) forgets the co-resident CTAs"),
     # ---- the LRU simulator (oracle/lru.py)
     "lru_evicts_mru": ("lru.py", "cache.popitem(last=False)", "cache.popitem(last=True)", 1,
                        "the simulator evicts the most recent line"),
     "lru_no_refresh_on_hit": ("lru.py", "                    cache.move_to_end(ln)\n", "", 1,
                               "a hit does not refresh its line (FIFO, not LRU)"),
+    "lru_row_trace_transposed": ("lru.py", "out.append((X, False, nb, tuple((_line(X, i * self.N + j), i) for i in rows)))",
+                                 "out.append((X, False, nb, tuple((_line(X, j * self.M + i), i) for i in rows)))", 1,
+                                 "the row loop's trace reads A column-major (coalesced)"),
     # ---- the B200 rule oracle (oracle/b200_rule.py)
     "rule_floor_4": ("b200_rule.py", "min_warps_sm=8,", "min_warps_sm=4,", 1, "R18 floor of 4 warps instead of 8"),
     "rule_fewest_warps_first": ("b200_rule.py", "a, m = max(fitting, key=lambda am: (am[0] * am[1], am[0]))",
                                 "a, m = min(fitting, key=lambda am: (am[0] * am[1], am[0]))", 1,
                                 "Eq 9 takes the most throttled fitting pair"),
     "rule_no_stream_floor": ("b200_rule.py", "floor = -(-floor // S)", "floor = floor", 1, "R29 not applied"),
+    "rule_retouch_2": ("b200_rule.py", "min_retouch=16,", "min_retouch=2,", 1, "R23 re-touch threshold 2 instead of 16"),
+    "rule_stream_pct_50": ("b200_rule.py", "max_stream_pct=25,", "max_stream_pct=50,", 1, "R24 stream share 50 % instead of 25 %"),
+    "rule_divergent_lines_2": ("b200_rule.py", "divergent_lines=8,", "divergent_lines=2,", 1,
+                               "R18 divergence at 2 lines per request instead of 8"),
+    "rule_shared_ignored": ("b200_rule.py", " and not (guards.get(\"private_streams\", 0) and inp.shared[i])", "", 1,
+                            "R32 not applied (CTA-shared loads counted as streams)"),
+    "exact_sum_drops_group": ("kmeans.py", "for ex in np.unique(e):", "for ex in np.unique(e)[1:]:", 1,
+                              "the exact sum drops the smallest-exponent values"),
     # ---- the exact k-means update (oracle/kmeans.py)
     "round_ties_away": ("kmeans.py", "if rem > Fraction(1, 2) or (rem == Fraction(1, 2) and n % 2 == 1):",
                         "if rem >= Fraction(1, 2):", 1, "round half away from zero instead of to even"),
