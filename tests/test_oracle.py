@@ -587,3 +587,19 @@ def test_corr_pins():
     # the fp64 mode is the textbook value
     sym64, _, _, _ = oracle.corr(data[:, :5], mode=oracle.SEQ_F64)
     assert np.max(np.abs(sym64 - np.corrcoef(data[:, :5].astype(np.float64).T))) < 1e-6
+
+
+def test_mutation_harness_still_applies():
+    # tools/oracle_mutants.py (DESIGN 3, "Do the pins have teeth?") types each
+    # mistake into a copy of oracle/ by text replacement: every mutant's text
+    # must still occur exactly once, or an oracle edit silently retired it
+    import importlib.util
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    spec = importlib.util.spec_from_file_location("oracle_mutants", os.path.join(root, "tools", "oracle_mutants.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    assert len(m.MUTANTS) >= 40
+    for name, (fn, old, new, count, what) in m.MUTANTS.items():
+        src = open(os.path.join(root, "oracle", fn)).read()
+        assert src.count(old) == 1, name
+        assert (old == new) == (name == "control_unchanged"), name
