@@ -149,6 +149,7 @@ class Workload:
     desc = ""
     variant = "coop"
     scaling = "weak"          # every rank's work is fixed as N grows (the JSON line's "scaling")
+    parallelism = "independent problem per rank"   # how N > 1 splits the work (config.parallelism)
 
     def __init__(self, catt, torch, rank, world, variant):
         self.catt, self.torch, self.rank, self.world = catt, torch, rank, world
@@ -184,6 +185,7 @@ class Workload:
 
 
 class BicgMvt(Workload):
+    parallelism = "row-shard"
     name = "bicg_mvt"
     variant = "fused"
     desc = "BICG and MVT 4096x4096 fp32 row-per-thread (memory-divergent) on 1 B200 (BASELINE configs[1])"
@@ -343,6 +345,7 @@ class Kmeans(Workload):
 
 
 class KmeansIter(Workload):
+    parallelism = "point-shard"
     name = "kmeans_iter"
     desc = ("KMEANS full iteration (assign + exact centroid update), 494020 points x 34 features, k=5, "
             "feature-major, points sharded per rank (SURVEY 8(f) f2)")
@@ -402,6 +405,7 @@ class KmeansIter(Workload):
 
 
 class Gesummv(Workload):
+    parallelism = "row-shard"
     name = "gesummv"
     desc = "GESUMMV 8192 fp32 (configs[3])"
 
@@ -587,6 +591,7 @@ class Gemm(Workload):
 
 
 class Atax(Workload):
+    parallelism = "row-shard"
     name = "atax"
     variant = "fused"
     desc = "ATAX 65536x16384 fp32 row-sharded with NCCL all-reduce of A^T partials (configs[4])"
@@ -1321,7 +1326,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": w.scaling,
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded counter hash, generated on device)",
             "config": {"workload": w.desc, "variant": w.variant, "l2": "flushed before every step (256 MiB write, then 256 MiB clean read)", "flush_order": args.flush_order,
-                       "rows_per_rank": getattr(w, "rows", None), "parallelism": f"row-shard x{world}"},
+                       "rows_per_rank": getattr(w, "rows", None), "parallelism": f"{w.parallelism} x{world}"},
             "loops": {lp.name: {"ms": round(loop_ms[i], 5),
                                 "gbs": round(lp.nbytes / (loop_ms[i] * 1e-3) / 1e9, 1),
                                 "plan": [dict(w.plans[k], loop=k) for k in lp.plans if k in w.plans] or None}

@@ -67,16 +67,23 @@ def test_reference_arm_under_torchrun_rank0_only():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("variant", [None, "fused_peer"])
-def test_bench_two_ranks_share_one_gpu(variant):
-    """The N > 1 bench path end to end (row shards, the A^T all-reduce between
-    the ranks or inside the fused kernel, max-over-ranks timing, one line from
-    rank 0), with both ranks on cuda:0 over gloo (CATT_BENCH_SHARE_GPU, tests
-    only: NCCL refuses two ranks on one device). Not a bench number."""
-    args = ["--steps", "2", "--warmup", "3", "--no-study", "--no-l1", "--cpu-seconds", "0"]
+@pytest.mark.parametrize("workload,variant,par", [("atax", None, "row-shard"), ("atax", "fused_peer", "row-shard"),
+                                                  ("bicg_mvt", None, "row-shard"),
+                                                  ("kmeans_iter", None, "point-shard"),
+                                                  ("syrk", None, "independent problem per rank")])
+def test_bench_two_ranks_share_one_gpu(workload, variant, par):
+    """The N > 1 bench path end to end (row shards with the A^T all-reduce
+    between the ranks or inside the fused kernel, k-means points with the
+    exact-sum all-reduce, independent replicas; max-over-ranks timing, one
+    line from rank 0), with both ranks on cuda:0 over gloo
+    (CATT_BENCH_SHARE_GPU, tests only: NCCL refuses two ranks on one device).
+    Not a bench number."""
+    args = ["--workload", workload, "--steps", "2", "--warmup", "3", "--no-study", "--no-l1", "--cpu-seconds", "0"]
     if variant:
         args += ["--variant", variant]
     d = _run_torchrun(args, extra_env={"CATT_BENCH_SHARE_GPU": "1"})
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["gpu_launches"] > 0
-    assert d["config"]["parallelism"] == "row-shard x2" and d["config"]["rows_per_rank"] == 65536 // 2
+    assert d["config"]["parallelism"] == f"{par} x2"
+    if workload == "atax":
+        assert d["config"]["rows_per_rank"] == 65536 // 2
     assert isinstance(d["roofline"], dict) and d["roofline"]["achieved"] > 0
