@@ -65,6 +65,10 @@ def test_trace_inputs_of_the_other_loops():
     # CORR: lanes at j2 = j1 + 1 + q read coalesced columns (j2 = 1..32 spans two lines)
     r = br.trace_inputs(lru.CorrKernel(96, 4, 32))
     assert r.lines["d_j1"] == 1 and r.lines["d_j2"] == 2 and r.reuse["d_j1"] and r.stored["sym_12"]
+    # R24 counts every store as stream bytes, the re-touched symmat[j1*m + j2]
+    # too: per (j1, j2), n = 4 rows of two 4-byte loads (both re-touched) and
+    # two 4-byte stores -> stream 8 of 40 bytes
+    assert r.reuse["sym_12"] and 5 * r.stream_bytes == r.total_bytes
 
 
 def test_divergence_predicate():

@@ -95,6 +95,15 @@ MUTANTS = {
     "lru_row_trace_transposed": ("lru.py", "out.append((X, False, nb, tuple((_line(X, i * self.N + j), i) for i in rows)))",
                                  "out.append((X, False, nb, tuple((_line(X, j * self.M + i), i) for i in rows)))", 1,
                                  "the row loop's trace reads A column-major (coalesced)"),
+    "lru_syrk_trace_aj_row": ("lru.py", 'out.append(("a_j", False, 4, tuple((_line("a", j * self.Mk + k), (i, j)) for i, j in th)))',
+                              'out.append(("a_j", False, 4, tuple((_line("a", i * self.Mk + k), (i, j)) for i, j in th)))', 1,
+                              "the SYRK trace reads row i for a_jk"),
+    "lru_kmeans_trace_point_major": ("lru.py", 'ev.append(tuple((_line("F", f * self.ld + p), p) for p in pts))',
+                                     'ev.append(tuple((_line("F", p * self.nf + f), p) for p in pts))', 1,
+                                     "the KMEANS trace reads features point-major"),
+    "lru_transpose_store_as_load": ("lru.py", 'out.append(("out", True, 4, tuple((_line("out", f * self.ld + p), p) for p in pts)))',
+                                    'out.append(("out", False, 4, tuple((_line("out", f * self.ld + p), p) for p in pts)))', 1,
+                                    "the KM transpose's store traced as a load"),
     # ---- the B200 rule oracle (oracle/b200_rule.py)
     "rule_floor_4": ("b200_rule.py", "min_warps_sm=8,", "min_warps_sm=4,", 1, "R18 floor of 4 warps instead of 8"),
     "rule_fewest_warps_first": ("b200_rule.py", "a, m = max(fitting, key=lambda am: (am[0] * am[1], am[0]))",
@@ -109,6 +118,11 @@ MUTANTS = {
                             "R32 not applied (CTA-shared loads counted as streams)"),
     "exact_sum_drops_group": ("kmeans.py", "for ex in np.unique(e):", "for ex in np.unique(e)[1:]:", 1,
                               "the exact sum drops the smallest-exponent values"),
+    "rule_stream_ignores_stores": ("b200_rule.py", "stream = sum(nbytes[i] for i in first if stored[i] or not reuse[i])",
+                                   "stream = sum(nbytes[i] for i in first if not reuse[i])", 1,
+                                   "R24's stream share leaves out the stores"),
+    "rule_retouch_min": ("b200_rule.py", "retouch[instr] = max(retouch[instr], c)", "retouch[instr] = min(retouch[instr] or c, c)", 1,
+                         "re-touches measured as the fewest, not the most, touches of a line"),
     # ---- the exact k-means update (oracle/kmeans.py)
     "round_ties_away": ("kmeans.py", "if rem > Fraction(1, 2) or (rem == Fraction(1, 2) and n % 2 == 1):",
                         "if rem >= Fraction(1, 2):", 1, "round half away from zero instead of to even"),
