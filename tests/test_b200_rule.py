@@ -170,14 +170,14 @@ def _golden():
     return json.load(open(GOLDEN))
 
 
-def test_library_rule_equals_trace_oracle_on_the_229_replayed_launches():
-    """Every launch of the stored sweeps (tools/rule_replay.py's 229: the round-1
+def test_library_rule_equals_trace_oracle_on_the_243_replayed_launches():
+    """Every launch of the stored sweeps (tools/rule_replay.py's 243: the round-1
     final pass, held-out sets 1-9, the SM partitions, round 2's held-out sets
-    10-13), at its full shape: the
+    10-14), at its full shape: the
     library's (W, T), L1D and pick equal those tools/gen_rule_golden.py derived
     from oracle/ alone (traces + LRU + Eq 1-4)."""
     g = _golden()
-    assert len(g["launches"]) == 229 and g["guards"] == br.B200_GUARDS
+    assert len(g["launches"]) == 243 and g["guards"] == br.B200_GUARDS
     b200 = catt.hw_b200()
     keys = ("min_warps_sm", "divergent_lines", "min_retouch", "max_stream_pct", "cta_fallback", "stream_floor",
             "private_streams")

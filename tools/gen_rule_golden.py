@@ -1,6 +1,6 @@
 """Write tests/golden/b200_rule_picks.json: the B200 rule's pick at every
-launch of the stored throttle sweeps (the 229 replayed launches of
-tools/rule_replay.py: round 1's 160 and round 2's held-out studies 10-13), derived ONLY from oracle/ (address traces of the loop
+launch of the stored throttle sweeps (the 243 replayed launches of
+tools/rule_replay.py: round 1's 160 and round 2's held-out studies 10-14), derived ONLY from oracle/ (address traces of the loop
 bodies, the LRU L1D simulator, oracle.footprint.occupancy for W and T).
 
 TEST INFRASTRUCTURE: calls nothing but oracle/ (no library, no device). The
@@ -61,7 +61,8 @@ FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["p
          "heldout11": ["profiles/r2/heldout11/heldout11_study.json"],
          "heldout12": ["profiles/r2/heldout12/heldout12_study.json"],
          # round 2, last session: a second out-of-sample check (no change under test)
-         "heldout13": ["profiles/r2/heldout13/heldout13_study.json"]}
+         "heldout13": ["profiles/r2/heldout13/heldout13_study.json"],
+         "heldout14": ["profiles/r2/heldout14/heldout14_study.json"]}
 SETS = list(FILES)
 
 

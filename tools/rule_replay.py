@@ -67,7 +67,8 @@ FILES = {"final": sorted(glob.glob("profiles/r1p/bench_*.json")), "heldout": ["p
          # round 2, closing: an out-of-sample check of the final rule (no change under test)
          "heldout12": ["profiles/r2/heldout12/heldout12_study.json"],
          # round 2, last session: a second out-of-sample check (no change under test)
-         "heldout13": ["profiles/r2/heldout13/heldout13_study.json"]}
+         "heldout13": ["profiles/r2/heldout13/heldout13_study.json"],
+         "heldout14": ["profiles/r2/heldout14/heldout14_study.json"]}
 ATAX = {"bench_atax.json": P(catt.K_ATAX_1, m=65536, n=16384), "bench_atax256.json": P(catt.K_ATAX_1, m=256, n=256)}
 
 
@@ -144,10 +145,10 @@ def replay(rule, sets, verbose):
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--rule", default="b200", choices=["b200", "r29", "r27", "r24", "r23", "r18", "paper"])
-    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "heldout11", "heldout12", "heldout13", "all"])
+    ap.add_argument("--set", default="all", choices=["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "heldout11", "heldout12", "heldout13", "heldout14", "all"])
     ap.add_argument("-v", action="store_true")
     a = ap.parse_args()
-    sets = ["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "heldout11", "heldout12", "heldout13"] if a.set == "all" else [a.set]
+    sets = ["final", "heldout", "heldout2", "heldout3", "heldout4", "heldout5", "heldout6", "heldout7", "heldout8", "heldout9", "partition", "heldout10", "heldout11", "heldout12", "heldout13", "heldout14"] if a.set == "all" else [a.set]
     res = replay(a.rule, sets, a.v)
     for s in sets:
         rs = [x for x in res if x[0] == s]
